@@ -1,0 +1,160 @@
+/*
+ * mv.h -- C ABI of the B200-native batched IVF k-NN hot path (Milvus, SIGMOD'21).
+ *
+ * Problem (§3.2.1): given a batch of m queries and n data vectors, find for
+ * each query its top-k most similar vectors; results are (int64 id, float distance) pairs
+ * (Eq. (1) sizes heap entries as sizeof(int64)+sizeof(float)).
+ * Indexes: IVF_FLAT and IVF_SQ8 (§2.2, 510-520 §3.1), metrics squared L2 and
+ * inner product (§2.1).  Query processing is the two-step IVF procedure of
+ * PAPER.md:523-532 (§3.1): find the nprobe closest buckets, then scan them.  k <= 16384
+ * (§3.3).  A bitmap of entity ids is checked whenever a vector is
+ * encountered, before the top-k (strategy B, §4.1).
+ *
+ * Conventions (all entry points):
+ *   - Every call returns mv_status (MV_OK = 0).  No exception or abort crosses the ABI.  On a
+ *     non-OK status, mv_last_error() returns a thread-local message.
+ *   - Pointers are device pointers on the index's device, OR host pointers: host buffers are
+ *     detected (cudaPointerGetAttributes), staged through device memory, and the call then
+ *     completes synchronously before returning.
+ *   - `stream` is a cudaStream_t (NULL = the legacy default stream).  With device pointers the
+ *     work is enqueued on `stream` and the call returns without synchronising (cudaMemcpyAsync
+ *     semantics): inputs must stay valid and outputs must not be read until the stream reaches
+ *     the work.  Exceptions that synchronise are documented per call.
+ *   - Argument errors return MV_EINVAL synchronously, before any work is enqueued.
+ *     Asynchronous CUDA faults surface as MV_ECUDA from a later call.
+ *   - The index owns all of its device storage; `add` copies.  Inputs and outputs are owned by
+ *     the caller; outputs are caller-allocated.
+ *   - State machine: create -> set_centroids -> (SQ8 only: train_sq8 | set_sq8) -> add* ->
+ *     search*.  Out-of-order calls return MV_ESTATE.  `add` and `search` on one index must not
+ *     overlap (the caller serialises); concurrent searches on different streams are allowed
+ *     (read-only index, per-call workspace).
+ */
+#ifndef MV_H
+#define MV_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#if defined(__GNUC__)
+#define MV_API __attribute__((visibility("default")))
+#else
+#define MV_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct mv_index mv_index; /* opaque; owned by the library */
+
+typedef enum {
+  MV_L2 = 0, /* squared Euclidean distance; smaller is better */
+  MV_IP = 1  /* inner product; larger is better */
+} mv_metric;
+
+typedef enum {
+  MV_IVF_FLAT = 0, /* fine quantizer keeps the fp32 vector */
+  MV_IVF_SQ8 = 1   /* fine quantizer keeps one byte per dimension */
+} mv_type;
+
+typedef enum {
+  MV_OK = 0,
+  MV_EINVAL = -1, /* bad argument (range, null pointer, reserved id -1 in add, ...) */
+  MV_ESTATE = -2, /* call out of order for the index state machine */
+  MV_ENOMEM = -3, /* device allocation failed */
+  MV_ECUDA = -4,  /* a CUDA runtime/driver error (possibly from earlier asynchronous work) */
+  MV_ENCCL = -5   /* reserved for collective failures reported by the sharding layer */
+} mv_status;
+
+/* Create an empty index on CUDA device `device`.
+ *   d      >= 1 (rows are stored zero-padded to a multiple of 32 elements, which changes neither
+ *             L2 nor IP); nlist >= 1 buckets (K-means buckets, K=16384 default).
+ * Synchronous.  *out receives the handle (destroy with mv_index_destroy). */
+MV_API mv_status mv_index_create(int32_t d, mv_metric metric, mv_type type, int32_t nlist, int32_t device,
+                          mv_index** out);
+
+/* Supply the coarse codebook C (§3.1): nlist x d fp32, row-major.  The
+ * north star consumes supplied centroids; training them (k-means) is outside the library.
+ * Synchronous (the centroid array is copied before return). */
+MV_API mv_status mv_index_set_centroids(mv_index* index, const float* centroids);
+
+/* SQ8 only.  Per-dimension range from a training sample (n x d fp32, n >= 1):
+ *   vmin_j = min_i x_ij, vdiff_j = max_i x_ij - vmin_j  (fp32).  (the exact
+ * formula is reading O3 of DESIGN.md §2.)  Synchronous. */
+MV_API mv_status mv_index_train_sq8(mv_index* index, const float* sample, int64_t n);
+
+/* SQ8 only.  Supply the quantizer parameters directly (d floats each, host or device).
+ * vdiff_j >= 0; vdiff_j == 0 encodes every value of dimension j as code 0.  Synchronous. */
+MV_API mv_status mv_index_set_sq8(mv_index* index, const float* vmin, const float* vdiff);
+
+/* Insert n vectors (n x d fp32, row-major) with caller ids (n int64, any values except the
+ * reserved -1; duplicates allowed).  Each vector goes to bucket I(v) = its closest centroid
+ * (L2: argmin ||v-c||^2, IP: argmax <v,c>; ties -> smaller bucket id);
+ * SQ8 codes are code = floor(255*clamp((x-vmin)/vdiff,0,1)) in fp32 with one rounding per
+ * operation (bit-exact with the oracle).  Storage is list-major, each list in insertion order.
+ * Synchronous (returns after the index is updated; re-allocates list storage). */
+MV_API mv_status mv_index_add(mv_index* index, const float* vectors, const int64_t* ids, int64_t n, void* stream);
+
+/* Batched k-NN search (§3.1, 537-546 §3.2.1).
+ *   queries   nq x d fp32 row-major; nq >= 0 (nq == 0 is a no-op)
+ *   k         1 <= k <= 16384
+ *   nprobe    >= 1; values > nlist are clamped to nlist
+ *   bitset    nullable; bit i = (bitset[i>>3] >> (i&7)) & 1, indexed by ID; 1 = EXCLUDED
+ *             (deleted / failing the attribute filter; reading of PAPER.md:916-922).  ids >= nbits
+ *             are never excluded.  Applied inside the scan, before selection.
+ *   distances nq x k fp32 (out), ids nq x k int64 (out), row-major, best-first: ascending L2 /
+ *             descending IP; exact ties ordered by smaller id, then storage position.  Slots
+ *             beyond the number of candidates hold id -1 and distance +inf (L2) / -inf (IP).
+ * Results are deterministic and independent of the rest of the batch.  Asynchronous on
+ * `stream` for device pointers, except when k > 1024 (one stream synchronisation sizes the
+ * candidate workspace). */
+MV_API mv_status mv_search(mv_index* index, const float* queries, int64_t nq, int32_t k, int32_t nprobe,
+                    const uint8_t* bitset, int64_t nbits, float* distances, int64_t* ids, void* stream);
+
+/* Step (1) only: the nprobe closest buckets per query, best-first by
+ * (centroid score, bucket id) -> probes nq x nprobe' int32 where nprobe' = min(nprobe, nlist).
+ * When nprobe >= nlist every bucket is probed and they are listed in id order.  Parity hook for
+ * the conditional-oracle protocol; same kernels as mv_search.  Asynchronous like mv_search. */
+MV_API mv_status mv_search_probes(mv_index* index, const float* queries, int64_t nq, int32_t nprobe, int32_t* probes,
+                           void* stream);
+
+/* Merge nsrc per-shard top-k results (segments, §3.3; heap merge,
+ * PAPER.md:590-596): dists nsrc x nq x k fp32, ids nsrc x nq x k int64, each row best-first
+ * with -1 padding -> out_d / out_i nq x k, ordered by (distance, id, source, position).  Device
+ * pointers (or host; staged).  Asynchronous on `stream` for device pointers. */
+MV_API mv_status mv_merge_topk(mv_metric metric, const float* dists, const int64_t* ids, int32_t nsrc, int64_t nq,
+                        int32_t k, float* out_d, int64_t* out_i, void* stream);
+
+/* Number of stored vectors. */
+MV_API int64_t mv_index_ntotal(const mv_index* index);
+
+/* Parity hook: copy the list-major storage description.  list_off: nlist+1 int64 (may be
+ * NULL); ids: ntotal int64 in storage order (may be NULL); codes: ntotal x d uint8 (SQ8 only,
+ * unpadded, may be NULL).  Host or device pointers.  Synchronous. */
+MV_API mv_status mv_index_storage(const mv_index* index, int64_t* list_off, int64_t* ids, uint8_t* codes);
+
+/* Parity hook: SQ8 parameters (d floats each). Synchronous. */
+MV_API mv_status mv_index_get_sq8(const mv_index* index, float* vmin, float* vdiff);
+
+/* Stage profiling (measurement, §8(d)).  When enabled, mv_search records CUDA events on its
+ * stream around each stage:  0 = query staging + coarse (a1-a3), 1 = bucketing (a4),
+ * 2 = grouped list scan with fused partial top-k (a5-a6), 3 = final select (a7).
+ * mv_profile_read synchronises on the recorded events and returns, per stage, the summed
+ * milliseconds since the last reset (ms[4]); *searches = profiled mv_search calls; *launches =
+ * kernels libmv launched in them.  `reset` != 0 clears the accumulators after reading. */
+MV_API mv_status mv_profile_enable(mv_index* index, int on);
+MV_API mv_status mv_profile_read(mv_index* index, double* ms, int64_t* searches, int64_t* launches, int reset);
+
+/* Release the index and all of its device storage (NULL is a no-op). */
+MV_API void mv_index_destroy(mv_index* index);
+
+/* Thread-local message for the last non-OK status on this thread ("" if none). */
+MV_API const char* mv_last_error(void);
+
+/* Library build string (compile target and version). */
+MV_API const char* mv_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* MV_H */

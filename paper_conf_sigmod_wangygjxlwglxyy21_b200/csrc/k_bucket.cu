@@ -1,0 +1,146 @@
+// k_bucket.cu -- §8 row a4: invert the (query, probed list) pairs into per-list query buckets
+// and work items.  The grouping is the B200 form of the paper's cache-aware idea: "reuse the
+// accessed data vectors as much as possible for multiple queries" (§3.2.1),
+// because in step 2 "different queries do not necessarily access the same buckets"
+// (§3.4).  A counting sort by list id: histogram, exclusive scan, scatter.
+// Also the per-pair candidate-region offsets for the scan's partial top-k output.
+#include "mv_internal.cuh"
+
+namespace mv {
+
+// Single-CTA exclusive scan (n up to a few million): out[0..n], out[n] = total.
+template <typename T>
+__global__ void __launch_bounds__(1024) k_scan_single(const T* __restrict__ in, int64_t n, T* __restrict__ out) {
+  __shared__ T part[1024];
+  const int tid = threadIdx.x;
+  const int64_t per = (n + 1023) / 1024;
+  const int64_t s = tid * per, e = min64(n, s + per);
+  T acc = 0;
+  for (int64_t i = s; i < e; ++i) acc += in[i];
+  part[tid] = acc;
+  __syncthreads();
+  for (int off = 1; off < 1024; off <<= 1) {  // Hillis-Steele inclusive scan of 1024 partials
+    T v = tid >= off ? part[tid - off] : (T)0;
+    __syncthreads();
+    part[tid] += v;
+    __syncthreads();
+  }
+  T run = tid ? part[tid - 1] : (T)0;
+  for (int64_t i = s; i < e; ++i) {
+    out[i] = run;
+    run += in[i];
+  }
+  if (tid == 1023) out[n] = part[1023];
+}
+
+cudaError_t launch_scan_i32(const int32_t* in, int n, int32_t* out, cudaStream_t st) {
+  k_scan_single<int32_t><<<1, 1024, 0, st>>>(in, n, out);
+  return cudaGetLastError();
+}
+cudaError_t launch_scan_i64(const int64_t* in, int64_t n, int64_t* out, cudaStream_t st) {
+  k_scan_single<int64_t><<<1, 1024, 0, st>>>(in, n, out);
+  return cudaGetLastError();
+}
+
+__global__ void k_bucket_fill(const int32_t* __restrict__ probes, int64_t npairs, const int32_t* __restrict__ boff,
+                              int32_t* bfill, int32_t* bq) {
+  for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < npairs; p += (int64_t)gridDim.x * blockDim.x) {
+    const int l = probes[p];
+    const int pos = boff[l] + atomicAdd(bfill + l, 1);
+    bq[pos] = (int32_t)p;
+  }
+}
+
+__global__ void k_work_count(const int32_t* __restrict__ lcount, int nlist, int qchunk, int32_t* wcount) {
+  const int l = blockIdx.x * blockDim.x + threadIdx.x;
+  if (l < nlist) wcount[l] = (lcount[l] + qchunk - 1) / qchunk;
+}
+
+__global__ void k_work_fill(const int32_t* __restrict__ wcount, const int32_t* __restrict__ woff,
+                            const int32_t* __restrict__ boff, int nlist, int qchunk, int2* witems) {
+  const int l = blockIdx.x * blockDim.x + threadIdx.x;
+  if (l >= nlist) return;
+  const int n = wcount[l], o = woff[l], b = boff[l];
+  for (int c = 0; c < n; ++c) witems[o + c] = make_int2(l, b + c * qchunk);
+}
+
+cudaError_t launch_bucket(const int32_t* probes, int64_t nq, int npb, int nlist, const int64_t* list_off, int k,
+                          int qchunk, const Bucketing& b, cudaStream_t st) {
+  (void)list_off; (void)k;
+  const int64_t npairs = nq * npb;
+  cudaMemsetAsync(b.lcount, 0, sizeof(int32_t) * nlist, st);
+  cudaMemsetAsync(b.bfill, 0, sizeof(int32_t) * nlist, st);
+  cudaMemsetAsync(b.counter, 0, sizeof(int32_t), st);
+  cudaError_t e = launch_count_lists(probes, npairs, b.lcount, st);
+  if (e != cudaSuccess) return e;
+  if ((e = launch_scan_i32(b.lcount, nlist, b.boff, st)) != cudaSuccess) return e;
+  const int grid = (int)min64(kNumSMs * 8, (npairs + 255) / 256);
+  if (npairs) k_bucket_fill<<<grid, 256, 0, st>>>(probes, npairs, b.boff, b.bfill, b.bq);
+  k_work_count<<<(nlist + 255) / 256, 256, 0, st>>>(b.lcount, nlist, qchunk, b.wcount);
+  if ((e = launch_scan_i32(b.wcount, nlist, b.woff, st)) != cudaSuccess) return e;
+  k_work_fill<<<(nlist + 255) / 256, 256, 0, st>>>(b.wcount, b.woff, b.boff, nlist, qchunk, b.witems);
+  return cudaGetLastError();
+}
+
+// Region capacity of pair (q, j): min(k, |list|) when the scan selects locally (k <= 1024),
+// else |list| (every candidate that survives the bitset is emitted).
+__device__ __forceinline__ int64_t pair_cap(int64_t len, int k) {
+  return k <= kLocalSelectMaxK ? min64(k, len) : len;
+}
+
+// one warp per query: qtot[q] = sum_j cap(q, j)
+__global__ void k_query_tot(const int32_t* __restrict__ probes, int64_t nq, int npb,
+                            const int64_t* __restrict__ list_off, int k, int64_t* qtot) {
+  const int lane = threadIdx.x & 31;
+  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t q = warp; q < nq; q += nwarps) {
+    int64_t acc = 0;
+    for (int j = lane; j < npb; j += 32) {
+      const int l = probes[q * npb + j];
+      acc += pair_cap(list_off[l + 1] - list_off[l], k);
+    }
+    for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(MV_FULL, acc, o);
+    if (lane == 0) qtot[q] = acc;
+  }
+}
+
+// one warp per query: poff[q*npb + j] = qbase[q] + sum_{j' < j} cap(q, j')
+__global__ void k_pair_off(const int32_t* __restrict__ probes, int64_t nq, int npb, const int64_t* __restrict__ list_off,
+                           int k, const int64_t* __restrict__ qbase, int64_t* poff) {
+  const int lane = threadIdx.x & 31;
+  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t q = warp; q < nq; q += nwarps) {
+    int64_t run = qbase[q];
+    for (int j0 = 0; j0 < npb; j0 += 32) {
+      const int j = j0 + lane;
+      int64_t c = 0;
+      if (j < npb) {
+        const int l = probes[q * npb + j];
+        c = pair_cap(list_off[l + 1] - list_off[l], k);
+      }
+      int64_t incl = c;
+      for (int o = 1; o < 32; o <<= 1) {
+        const int64_t v = __shfl_up_sync(MV_FULL, incl, o);
+        if (lane >= o) incl += v;
+      }
+      if (j < npb) poff[q * npb + j] = run + incl - c;
+      run += __shfl_sync(MV_FULL, incl, 31);
+    }
+  }
+}
+
+cudaError_t launch_pair_offsets(const int32_t* probes, int64_t nq, int npb, const int64_t* list_off, int k,
+                                const Bucketing& b, cudaStream_t st) {
+  if (nq == 0) return cudaSuccess;
+  const int grid = (int)min64(kNumSMs * 8, (nq * 32 + 255) / 256);
+  int64_t* qbase = b.qtot + (nq + 1);  // second half of the qtot allocation
+  k_query_tot<<<grid, 256, 0, st>>>(probes, nq, npb, list_off, k, b.qtot);
+  cudaError_t e = launch_scan_i64(b.qtot, nq, qbase, st);
+  if (e != cudaSuccess) return e;
+  k_pair_off<<<grid, 256, 0, st>>>(probes, nq, npb, list_off, k, qbase, b.poff);
+  return cudaGetLastError();
+}
+
+}  // namespace mv

@@ -1,0 +1,603 @@
+// mv_api.cu -- the C ABI of include/mv.h: index state, validation, host-pointer staging, and the
+// search pipeline a1 -> a2/a3 -> a4 -> a5/a6 -> a7 enqueued on the caller's stream.
+#include <cub/device/device_radix_sort.cuh>
+
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "mv_internal.cuh"
+
+using namespace mv;
+
+struct mv_index {
+  int d = 0, dpad = 0, metric = 0, type = 0, nlist = 0, device = 0;
+  bool has_centroids = false, has_sq8 = false;
+  float* cpad = nullptr;    // nlist x dpad
+  float* cnorm = nullptr;   // nlist
+  float* vmin = nullptr;    // dpad (zero padded)
+  float* vdiff = nullptr;   // dpad (zero padded)
+  float* sq8_t = nullptr;   // 256: (c + 0.5f) / 255.f
+  int64_t ntotal = 0;
+  int64_t* list_off = nullptr;  // nlist + 1 (device)
+  std::vector<int64_t> h_list_off;
+  int64_t maxlen = 0;
+  void* payload = nullptr;      // ntotal x dpad (fp32 or u8)
+  float* norms = nullptr;       // ntotal
+  int64_t* ids = nullptr;       // ntotal, storage order
+  uint32_t* rank = nullptr;     // ntotal: position of (id, row) in sorted order
+  int64_t* sorted_ids = nullptr;  // ntotal: ids in (id, row) order
+  // profiling
+  bool prof = false;
+  std::vector<cudaEvent_t> ev;   // 5 events per profiled search
+  int64_t prof_searches = 0, launches = 0;
+};
+
+// ------------------------------------------------------------------------------------------
+namespace {
+thread_local std::string g_err;
+
+mv_status fail(mv_status s, const char* fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof buf, fmt, ap);
+  va_end(ap);
+  g_err = buf;
+  return s;
+}
+
+#define CK(x)                                                                          \
+  do {                                                                                 \
+    cudaError_t _e = (x);                                                              \
+    if (_e != cudaSuccess) return fail(MV_ECUDA, "%s: %s", #x, cudaGetErrorString(_e)); \
+  } while (0)
+
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    cudaGetDevice(&prev);
+    if (prev != dev) cudaSetDevice(dev);
+  }
+  ~DeviceGuard() {
+    int cur = -1;
+    cudaGetDevice(&cur);
+    if (prev >= 0 && cur != prev) cudaSetDevice(prev);
+  }
+};
+
+bool is_host_ptr(const void* p) {
+  if (p == nullptr) return false;
+  cudaPointerAttributes at;
+  if (cudaPointerGetAttributes(&at, p) != cudaSuccess) {
+    cudaGetLastError();
+    return true;
+  }
+  return at.type == cudaMemoryTypeHost || at.type == cudaMemoryTypeUnregistered;
+}
+
+// Stream-ordered scratch allocations released at scope exit.
+struct Scratch {
+  cudaStream_t st;
+  std::vector<void*> ptrs;
+  explicit Scratch(cudaStream_t s) : st(s) {}
+  ~Scratch() {
+    for (void* p : ptrs) cudaFreeAsync(p, st);
+  }
+  template <typename T>
+  cudaError_t alloc(T** p, size_t n) {
+    *p = nullptr;
+    if (n == 0) n = 1;
+    cudaError_t e = cudaMallocAsync(reinterpret_cast<void**>(p), n * sizeof(T), st);
+    if (e == cudaSuccess) ptrs.push_back(*p);
+    return e;
+  }
+};
+
+// Device view of a caller buffer: device pointers pass through; host buffers are staged.
+template <typename T>
+cudaError_t stage_in(Scratch& s, const T* p, size_t n, const T** out, bool* staged) {
+  *staged = is_host_ptr(p);
+  if (!*staged) {
+    *out = p;
+    return cudaSuccess;
+  }
+  T* d = nullptr;
+  cudaError_t e = s.alloc(&d, n);
+  if (e != cudaSuccess) return e;
+  e = cudaMemcpyAsync(d, p, n * sizeof(T), cudaMemcpyHostToDevice, s.st);
+  *out = d;
+  return e;
+}
+
+void set_pool_threshold(int dev) {
+  static bool done[64] = {false};
+  if (dev < 0 || dev >= 64 || done[dev]) return;
+  cudaMemPool_t pool;
+  if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+    uint64_t thr = UINT64_MAX;
+    cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+  }
+  done[dev] = true;
+}
+
+void prof_mark(mv_index* ix, cudaStream_t st) {
+  if (!ix->prof) return;
+  cudaEvent_t e;
+  if (cudaEventCreate(&e) != cudaSuccess) return;
+  cudaEventRecord(e, st);
+  ix->ev.push_back(e);
+}
+
+void free_storage(mv_index* ix) {
+  cudaFree(ix->payload);
+  cudaFree(ix->norms);
+  cudaFree(ix->ids);
+  cudaFree(ix->rank);
+  cudaFree(ix->sorted_ids);
+  ix->payload = nullptr;
+  ix->norms = nullptr;
+  ix->ids = nullptr;
+  ix->rank = nullptr;
+  ix->sorted_ids = nullptr;
+}
+}  // namespace
+
+// ------------------------------------------------------------------------------------------
+extern "C" {
+
+const char* mv_last_error(void) { return g_err.c_str(); }
+
+const char* mv_version(void) { return "libmv 0.1 (sm_100a; IVF_FLAT/IVF_SQ8; L2/IP)"; }
+
+int64_t mv_index_ntotal(const mv_index* ix) { return ix ? ix->ntotal : 0; }
+
+mv_status mv_index_create(int32_t d, mv_metric metric, mv_type type, int32_t nlist, int32_t device, mv_index** out) {
+  if (!out) return fail(MV_EINVAL, "out is NULL");
+  *out = nullptr;
+  if (d < 1 || d > 4096) return fail(MV_EINVAL, "d must be in [1, 4096] (got %d)", d);
+  if (metric != MV_L2 && metric != MV_IP) return fail(MV_EINVAL, "unknown metric %d", (int)metric);
+  if (type != MV_IVF_FLAT && type != MV_IVF_SQ8) return fail(MV_EINVAL, "unknown index type %d", (int)type);
+  if (nlist < 1) return fail(MV_EINVAL, "nlist must be >= 1 (got %d)", nlist);
+  int ndev = 0;
+  CK(cudaGetDeviceCount(&ndev));
+  if (device < 0 || device >= ndev) return fail(MV_EINVAL, "device %d out of range (%d devices)", device, ndev);
+  DeviceGuard g(device);
+  set_pool_threshold(device);
+  mv_index* ix = new mv_index();
+  ix->d = d;
+  ix->dpad = (d + 31) / 32 * 32;
+  ix->metric = metric;
+  ix->type = type;
+  ix->nlist = nlist;
+  ix->device = device;
+  ix->h_list_off.assign(nlist + 1, 0);
+  cudaError_t e = cudaMalloc(&ix->list_off, sizeof(int64_t) * (nlist + 1));
+  if (e == cudaSuccess) e = cudaMemset(ix->list_off, 0, sizeof(int64_t) * (nlist + 1));
+  if (e == cudaSuccess) e = cudaMalloc(&ix->cpad, sizeof(float) * (size_t)nlist * ix->dpad);
+  if (e == cudaSuccess) e = cudaMalloc(&ix->cnorm, sizeof(float) * nlist);
+  if (e == cudaSuccess) e = cudaMalloc(&ix->vmin, sizeof(float) * ix->dpad);
+  if (e == cudaSuccess) e = cudaMalloc(&ix->vdiff, sizeof(float) * ix->dpad);
+  if (e == cudaSuccess) e = cudaMalloc(&ix->sq8_t, sizeof(float) * 256);
+  if (e == cudaSuccess) {
+    float t[256];
+    for (int c = 0; c < 256; ++c) t[c] = ((float)c + 0.5f) / 255.0f;  // oracle.sq8_decode's first two ops
+    e = cudaMemcpy(ix->sq8_t, t, sizeof t, cudaMemcpyHostToDevice);
+  }
+  if (e == cudaSuccess) e = cudaMemset(ix->vmin, 0, sizeof(float) * ix->dpad);
+  if (e == cudaSuccess) e = cudaMemset(ix->vdiff, 0, sizeof(float) * ix->dpad);
+  if (e != cudaSuccess) {
+    mv_index_destroy(ix);
+    return fail(e == cudaErrorMemoryAllocation ? MV_ENOMEM : MV_ECUDA, "create: %s", cudaGetErrorString(e));
+  }
+  *out = ix;
+  return MV_OK;
+}
+
+void mv_index_destroy(mv_index* ix) {
+  if (!ix) return;
+  DeviceGuard g(ix->device);
+  cudaDeviceSynchronize();
+  free_storage(ix);
+  for (cudaEvent_t e : ix->ev) cudaEventDestroy(e);
+  cudaFree(ix->list_off);
+  cudaFree(ix->cpad);
+  cudaFree(ix->cnorm);
+  cudaFree(ix->vmin);
+  cudaFree(ix->vdiff);
+  cudaFree(ix->sq8_t);
+  delete ix;
+}
+
+mv_status mv_index_set_centroids(mv_index* ix, const float* centroids) {
+  if (!ix || !centroids) return fail(MV_EINVAL, "null argument");
+  if (ix->ntotal > 0) return fail(MV_ESTATE, "centroids cannot change after vectors were added");
+  DeviceGuard g(ix->device);
+  cudaStream_t st = 0;
+  Scratch s(st);
+  bool staged;
+  const float* c;
+  CK(stage_in(s, centroids, (size_t)ix->nlist * ix->d, &c, &staged));
+  CK(launch_centroid_prep(c, ix->nlist, ix->d, ix->dpad, ix->cpad, ix->cnorm, st));
+  CK(cudaStreamSynchronize(st));
+  ix->has_centroids = true;
+  return MV_OK;
+}
+
+mv_status mv_index_train_sq8(mv_index* ix, const float* sample, int64_t n) {
+  if (!ix || !sample) return fail(MV_EINVAL, "null argument");
+  if (ix->type != MV_IVF_SQ8) return fail(MV_ESTATE, "train_sq8 on a non-SQ8 index");
+  if (n < 1) return fail(MV_EINVAL, "train_sq8 needs n >= 1");
+  if (ix->ntotal > 0) return fail(MV_ESTATE, "SQ8 parameters cannot change after vectors were added");
+  DeviceGuard g(ix->device);
+  cudaStream_t st = 0;
+  Scratch s(st);
+  bool staged;
+  const float* x;
+  CK(stage_in(s, sample, (size_t)n * ix->d, &x, &staged));
+  CK(launch_sq8_minmax(x, n, ix->d, ix->vmin, ix->vdiff, st));
+  CK(cudaStreamSynchronize(st));
+  ix->has_sq8 = true;
+  return MV_OK;
+}
+
+mv_status mv_index_set_sq8(mv_index* ix, const float* vmin, const float* vdiff) {
+  if (!ix || !vmin || !vdiff) return fail(MV_EINVAL, "null argument");
+  if (ix->type != MV_IVF_SQ8) return fail(MV_ESTATE, "set_sq8 on a non-SQ8 index");
+  if (ix->ntotal > 0) return fail(MV_ESTATE, "SQ8 parameters cannot change after vectors were added");
+  DeviceGuard g(ix->device);
+  std::vector<float> hv(ix->d), hd(ix->d);
+  CK(cudaMemcpy(hv.data(), vmin, sizeof(float) * ix->d, cudaMemcpyDefault));
+  CK(cudaMemcpy(hd.data(), vdiff, sizeof(float) * ix->d, cudaMemcpyDefault));
+  for (int j = 0; j < ix->d; ++j)
+    if (!(hd[j] >= 0.0f)) return fail(MV_EINVAL, "vdiff[%d] must be >= 0", j);
+  CK(cudaMemcpy(ix->vmin, hv.data(), sizeof(float) * ix->d, cudaMemcpyHostToDevice));
+  CK(cudaMemcpy(ix->vdiff, hd.data(), sizeof(float) * ix->d, cudaMemcpyHostToDevice));
+  ix->has_sq8 = true;
+  return MV_OK;
+}
+
+mv_status mv_index_get_sq8(const mv_index* ix, float* vmin, float* vdiff) {
+  if (!ix) return fail(MV_EINVAL, "null index");
+  if (ix->type != MV_IVF_SQ8 || !ix->has_sq8) return fail(MV_ESTATE, "no SQ8 parameters");
+  DeviceGuard g(ix->device);
+  if (vmin) CK(cudaMemcpy(vmin, ix->vmin, sizeof(float) * ix->d, cudaMemcpyDefault));
+  if (vdiff) CK(cudaMemcpy(vdiff, ix->vdiff, sizeof(float) * ix->d, cudaMemcpyDefault));
+  return MV_OK;
+}
+
+mv_status mv_index_add(mv_index* ix, const float* vectors, const int64_t* ids, int64_t n, void* stream) {
+  if (!ix) return fail(MV_EINVAL, "null index");
+  if (n < 0) return fail(MV_EINVAL, "n must be >= 0");
+  if (n == 0) return MV_OK;
+  if (!vectors || !ids) return fail(MV_EINVAL, "null vectors/ids");
+  if (!ix->has_centroids) return fail(MV_ESTATE, "add before set_centroids");
+  if (ix->type == MV_IVF_SQ8 && !ix->has_sq8) return fail(MV_ESTATE, "add on SQ8 index before train_sq8/set_sq8");
+  if (n > 0x7fffffffLL) return fail(MV_EINVAL, "one add call takes at most 2^31-1 vectors");
+  if (ix->ntotal + n > 0xffffffffLL) return fail(MV_EINVAL, "an index holds at most 2^32-1 vectors");
+  DeviceGuard g(ix->device);
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  Scratch s(st);
+  bool sv, si;
+  const float* x;
+  const int64_t* idv;
+  CK(stage_in(s, vectors, (size_t)n * ix->d, &x, &sv));
+  CK(stage_in(s, ids, (size_t)n, &idv, &si));
+  int* flag;
+  CK(s.alloc(&flag, 1));
+  CK(cudaMemsetAsync(flag, 0, sizeof(int), st));
+  CK(launch_check_ids(idv, n, flag, st));
+  int hflag = 0;
+  CK(cudaMemcpyAsync(&hflag, flag, sizeof(int), cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  if (hflag) return fail(MV_EINVAL, "id -1 is reserved (padding)");
+
+  const int nlist = ix->nlist, dpad = ix->dpad;
+  float *xpad, *xnorm;
+  int32_t *lists, *cnt, *addoff, *idx, *sidx, *slist;
+  int64_t *sizes, *new_off;
+  CK(s.alloc(&xpad, (size_t)n * dpad));
+  CK(s.alloc(&xnorm, (size_t)n));
+  CK(s.alloc(&lists, (size_t)n));
+  CK(s.alloc(&cnt, nlist));
+  CK(s.alloc(&addoff, nlist + 1));
+  CK(s.alloc(&idx, (size_t)n));
+  CK(s.alloc(&sidx, (size_t)n));
+  CK(s.alloc(&slist, (size_t)n));
+  CK(s.alloc(&sizes, nlist));
+  CK(s.alloc(&new_off, nlist + 1));
+  // a0: assignment I(v) = closest centroid (the coarse kernel with nprobe = 1)
+  CK(launch_query_prep(x, n, ix->d, dpad, xpad, xnorm, st));
+  CK(launch_coarse(xpad, n, dpad, ix->cpad, ix->cnorm, nlist, ix->metric, 1, lists, st));
+  CK(cudaMemsetAsync(cnt, 0, sizeof(int32_t) * nlist, st));
+  CK(launch_count_lists(lists, n, cnt, st));
+  CK(launch_scan_i32(cnt, nlist, addoff, st));
+  // stable order of the new rows by list (radix sort is stable; values = input order)
+  CK(launch_iota_i32(idx, n, st));
+  int endbit = 1;
+  while ((1 << endbit) < nlist && endbit < 31) ++endbit;
+  size_t tmp_bytes = 0;
+  CK(cub::DeviceRadixSort::SortPairs(nullptr, tmp_bytes, (const uint32_t*)lists, (uint32_t*)slist, idx, sidx, (int)n, 0,
+                                     endbit, st));
+  void* tmp;
+  CK(s.alloc(reinterpret_cast<uint8_t**>(&tmp), tmp_bytes));
+  CK(cub::DeviceRadixSort::SortPairs(tmp, tmp_bytes, (const uint32_t*)lists, (uint32_t*)slist, idx, sidx, (int)n, 0,
+                                     endbit, st));
+  CK(launch_new_sizes(cnt, nlist, ix->list_off, sizes, st));
+  CK(launch_scan_i64(sizes, nlist, new_off, st));
+
+  const int64_t ntot = ix->ntotal + n;
+  const size_t esize = ix->type == MV_IVF_FLAT ? 4 : 1;
+  void* payload = nullptr;
+  float* norms = nullptr;
+  int64_t *nids = nullptr, *sorted_ids = nullptr;
+  uint32_t* rank = nullptr;
+  cudaError_t e = cudaMalloc(&payload, (size_t)ntot * dpad * esize);
+  if (e == cudaSuccess) e = cudaMalloc(&norms, sizeof(float) * ntot);
+  if (e == cudaSuccess) e = cudaMalloc(&nids, sizeof(int64_t) * ntot);
+  if (e == cudaSuccess) e = cudaMalloc(&rank, sizeof(uint32_t) * ntot);
+  if (e == cudaSuccess) e = cudaMalloc(&sorted_ids, sizeof(int64_t) * ntot);
+  if (e != cudaSuccess) {
+    cudaFree(payload); cudaFree(norms); cudaFree(nids); cudaFree(rank); cudaFree(sorted_ids);
+    cudaGetLastError();
+    return fail(MV_ENOMEM, "add: cannot allocate storage for %lld vectors", (long long)ntot);
+  }
+  CK(launch_move_old(ix->type, dpad, nlist, ix->list_off, new_off, ix->payload, ix->norms, ix->ids, ix->ntotal, payload,
+                     norms, nids, st));
+  CK(launch_store_rows(ix->type, ix->metric, xpad, idv, sidx, slist, n, dpad, new_off, ix->list_off, addoff, payload,
+                       norms, nids, ix->vmin, ix->vdiff, ix->sq8_t, st));
+  // id ranks: stable radix sort of (id) over storage rows -> (id, row) order
+  uint64_t *keys, *skeys;
+  uint32_t *vals, *svals;
+  CK(s.alloc(&keys, (size_t)ntot));
+  CK(s.alloc(&skeys, (size_t)ntot));
+  CK(s.alloc(&vals, (size_t)ntot));
+  CK(s.alloc(&svals, (size_t)ntot));
+  CK(launch_id_keys(nids, ntot, keys, vals, st));
+  size_t tmp2 = 0;
+  CK(cub::DeviceRadixSort::SortPairs(nullptr, tmp2, keys, skeys, vals, svals, (int64_t)ntot, 0, 64, st));
+  void* t2;
+  CK(s.alloc(reinterpret_cast<uint8_t**>(&t2), tmp2));
+  CK(cub::DeviceRadixSort::SortPairs(t2, tmp2, keys, skeys, vals, svals, (int64_t)ntot, 0, 64, st));
+  CK(launch_rank_scatter(skeys, svals, ntot, rank, sorted_ids, st));
+  CK(cudaMemcpyAsync(ix->list_off, new_off, sizeof(int64_t) * (nlist + 1), cudaMemcpyDeviceToDevice, st));
+  CK(cudaMemcpyAsync(ix->h_list_off.data(), new_off, sizeof(int64_t) * (nlist + 1), cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  free_storage(ix);
+  ix->payload = payload;
+  ix->norms = norms;
+  ix->ids = nids;
+  ix->rank = rank;
+  ix->sorted_ids = sorted_ids;
+  ix->ntotal = ntot;
+  ix->maxlen = 0;
+  for (int l = 0; l < nlist; ++l) ix->maxlen = std::max(ix->maxlen, ix->h_list_off[l + 1] - ix->h_list_off[l]);
+  return MV_OK;
+}
+
+static mv_status validate_search(const mv_index* ix, const float* q, int64_t nq, int32_t k, int32_t nprobe,
+                                 const void* d, const void* i) {
+  if (!ix) return fail(MV_EINVAL, "null index");
+  if (nq < 0) return fail(MV_EINVAL, "nq must be >= 0");
+  if (k < 1 || k > kMaxK) return fail(MV_EINVAL, "k must be in [1, %d] (got %d)", kMaxK, k);
+  if (nprobe < 1) return fail(MV_EINVAL, "nprobe must be >= 1 (got %d)", nprobe);
+  const int npb = std::min(nprobe, ix->nlist);
+  if (npb < ix->nlist && npb > 1024) return fail(MV_EINVAL, "nprobe must be <= 1024 or >= nlist (got %d)", nprobe);
+  if (nq > 0 && (!q || !d || !i)) return fail(MV_EINVAL, "null queries/outputs");
+  if (!ix->has_centroids) return fail(MV_ESTATE, "search before set_centroids");
+  if (nq > 0x7fffffffLL / std::max(npb, 1)) return fail(MV_EINVAL, "nq * nprobe must be < 2^31");
+  return MV_OK;
+}
+
+mv_status mv_search_probes(mv_index* ix, const float* queries, int64_t nq, int32_t nprobe, int32_t* probes,
+                           void* stream) {
+  mv_status v = validate_search(ix, queries, nq, 1, nprobe, probes, probes);
+  if (v != MV_OK) return v;
+  if (nq == 0) return MV_OK;
+  DeviceGuard g(ix->device);
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  Scratch s(st);
+  const int npb = std::min(nprobe, ix->nlist);
+  bool sq, sp;
+  const float* q;
+  CK(stage_in(s, queries, (size_t)nq * ix->d, &q, &sq));
+  sp = is_host_ptr(probes);
+  int32_t* P = probes;
+  if (sp) CK(s.alloc(&P, (size_t)nq * npb));
+  float *qpad, *qnorm;
+  CK(s.alloc(&qpad, (size_t)nq * ix->dpad));
+  CK(s.alloc(&qnorm, (size_t)nq));
+  CK(launch_query_prep(q, nq, ix->d, ix->dpad, qpad, qnorm, st));
+  CK(launch_coarse(qpad, nq, ix->dpad, ix->cpad, ix->cnorm, ix->nlist, ix->metric, npb, P, st));
+  if (sp) {
+    CK(cudaMemcpyAsync(probes, P, sizeof(int32_t) * nq * npb, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+  }
+  return MV_OK;
+}
+
+mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, int32_t nprobe, const uint8_t* bitset,
+                    int64_t nbits, float* distances, int64_t* out_ids, void* stream) {
+  mv_status v = validate_search(ix, queries, nq, k, nprobe, distances, out_ids);
+  if (v != MV_OK) return v;
+  if (nbits < 0) return fail(MV_EINVAL, "nbits must be >= 0");
+  if (nq == 0) return MV_OK;
+  if (bitset == nullptr) nbits = 0;
+  DeviceGuard g(ix->device);
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  Scratch s(st);
+  const int nlist = ix->nlist, dpad = ix->dpad;
+  const int npb = std::min(nprobe, nlist);
+  bool sq, sb;
+  const float* q;
+  const uint8_t* bs = nullptr;
+  CK(stage_in(s, queries, (size_t)nq * ix->d, &q, &sq));
+  if (bitset && nbits > 0) CK(stage_in(s, bitset, (size_t)((nbits + 7) / 8), &bs, &sb));
+  const bool host_out = is_host_ptr(distances) || is_host_ptr(out_ids);
+  float* D = distances;
+  int64_t* I = out_ids;
+  if (host_out) {
+    CK(s.alloc(&D, (size_t)nq * k));
+    CK(s.alloc(&I, (size_t)nq * k));
+  }
+  if (ix->ntotal == 0) {
+    CK(launch_fill_pad((int64_t)nq * k, ix->metric, D, I, st));
+  } else {
+    // a1 + a2/a3
+    prof_mark(ix, st);
+    float *qpad, *qnorm;
+    int32_t* P;
+    CK(s.alloc(&qpad, (size_t)nq * dpad));
+    CK(s.alloc(&qnorm, (size_t)nq));
+    CK(s.alloc(&P, (size_t)nq * npb));
+    CK(launch_query_prep(q, nq, ix->d, dpad, qpad, qnorm, st));
+    CK(launch_coarse(qpad, nq, dpad, ix->cpad, ix->cnorm, nlist, ix->metric, npb, P, st));
+    prof_mark(ix, st);
+    // a4
+    const int qchunk = k <= kLocalSelectMaxK ? std::min(64, std::max(1, 65536 / (8 * k))) : 64;
+    const int64_t npairs = nq * npb;
+    Bucketing b;
+    CK(s.alloc(&b.lcount, nlist));
+    CK(s.alloc(&b.boff, nlist + 1));
+    CK(s.alloc(&b.bfill, nlist));
+    CK(s.alloc(&b.bq, (size_t)npairs));
+    CK(s.alloc(&b.wcount, nlist));
+    CK(s.alloc(&b.woff, nlist + 1));
+    CK(s.alloc(&b.witems, (size_t)(nlist + npairs / qchunk + 1)));
+    CK(s.alloc(&b.qtot, (size_t)(2 * (nq + 1))));
+    CK(s.alloc(&b.poff, (size_t)npairs));
+    CK(s.alloc(&b.pcnt, (size_t)npairs));
+    CK(s.alloc(&b.counter, 1));
+    CK(launch_bucket(P, nq, npb, nlist, ix->list_off, k, qchunk, b, st));
+    CK(launch_pair_offsets(P, nq, npb, ix->list_off, k, b, st));
+    prof_mark(ix, st);
+    int64_t cap;
+    if (k <= kLocalSelectMaxK) {
+      cap = nq * npb * min64(k, max64(ix->maxlen, 1));
+    } else {
+      CK(cudaMemcpyAsync(&cap, b.qtot + (nq + 1) + nq, sizeof(int64_t), cudaMemcpyDeviceToHost, st));
+      CK(cudaStreamSynchronize(st));
+    }
+    uint64_t* part;
+    cudaError_t ea = s.alloc(&part, (size_t)max64(cap, 1));
+    if (ea != cudaSuccess) {
+      cudaGetLastError();
+      return fail(MV_ENOMEM, "search: cannot allocate %lld candidate slots", (long long)cap);
+    }
+    // a5/a6
+    ScanArgs a;
+    a.type = ix->type; a.metric = ix->metric; a.d = ix->d; a.dpad = dpad; a.k = k; a.npb = npb;
+    a.qchunk = qchunk; a.nlist = nlist;
+    a.list_off = ix->list_off; a.payload = ix->payload; a.norms = ix->norms; a.ids = ix->ids; a.rank = ix->rank;
+    a.bitset = bs; a.nbits = bs ? nbits : 0;
+    a.qpad = qpad; a.qnorm = qnorm; a.vmin = ix->vmin; a.vdiff = ix->vdiff; a.sq8_t = ix->sq8_t;
+    a.bq = b.bq; a.boff = b.boff; a.witems = b.witems; a.nwitems = b.woff + nlist; a.counter = b.counter;
+    a.poff = b.poff; a.pcnt = b.pcnt; a.part = part;
+    CK(launch_scan(a, st));
+    prof_mark(ix, st);
+    // a7
+    CK(launch_final_select(b.poff, b.pcnt, part, nq, npb, k, ix->metric, ix->sorted_ids, D, I, st));
+    prof_mark(ix, st);
+    if (ix->prof) ix->prof_searches++;
+    ix->launches += 13;  // prep, coarse, 6 bucketing, 3 offsets, scan, select
+  }
+  if (host_out) {
+    CK(cudaMemcpyAsync(distances, D, sizeof(float) * nq * k, cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(out_ids, I, sizeof(int64_t) * nq * k, cudaMemcpyDeviceToHost, st));
+  }
+  if (host_out || sq) CK(cudaStreamSynchronize(st));
+  return MV_OK;
+}
+
+mv_status mv_merge_topk(mv_metric metric, const float* dists, const int64_t* ids, int32_t nsrc, int64_t nq, int32_t k,
+                        float* out_d, int64_t* out_i, void* stream) {
+  if (metric != MV_L2 && metric != MV_IP) return fail(MV_EINVAL, "unknown metric");
+  if (nsrc < 1 || k < 1 || k > kMaxK || nq < 0) return fail(MV_EINVAL, "bad nsrc/k/nq");
+  if (nq == 0) return MV_OK;
+  if (!dists || !ids || !out_d || !out_i) return fail(MV_EINVAL, "null argument");
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  Scratch s(st);
+  const size_t per = (size_t)nq * k;
+  bool sd, si;
+  const float* D;
+  const int64_t* I;
+  CK(stage_in(s, dists, per * nsrc, &D, &sd));
+  CK(stage_in(s, ids, per * nsrc, &I, &si));
+  const bool host_out = is_host_ptr(out_d) || is_host_ptr(out_i);
+  std::vector<const float*> cd;
+  std::vector<const int64_t*> ci;
+  for (int i = 0; i < nsrc; ++i) {
+    cd.push_back(D + per * i);
+    ci.push_back(I + per * i);
+  }
+  while (cd.size() > 1) {
+    std::vector<const float*> nd;
+    std::vector<const int64_t*> ni;
+    for (size_t i = 0; i + 1 < cd.size(); i += 2) {
+      float* od;
+      int64_t* oi;
+      CK(s.alloc(&od, per));
+      CK(s.alloc(&oi, per));
+      CK(launch_merge2(metric, cd[i], ci[i], cd[i + 1], ci[i + 1], nq, k, od, oi, st));
+      nd.push_back(od);
+      ni.push_back(oi);
+    }
+    if (cd.size() & 1) {
+      nd.push_back(cd.back());
+      ni.push_back(ci.back());
+    }
+    cd.swap(nd);
+    ci.swap(ni);
+  }
+  CK(cudaMemcpyAsync(out_d, cd[0], per * sizeof(float), cudaMemcpyDefault, st));
+  CK(cudaMemcpyAsync(out_i, ci[0], per * sizeof(int64_t), cudaMemcpyDefault, st));
+  if (host_out || sd || si) CK(cudaStreamSynchronize(st));
+  return MV_OK;
+}
+
+mv_status mv_profile_enable(mv_index* ix, int on) {
+  if (!ix) return fail(MV_EINVAL, "null index");
+  ix->prof = on != 0;
+  return MV_OK;
+}
+
+mv_status mv_profile_read(mv_index* ix, double* ms, int64_t* searches, int64_t* launches, int reset) {
+  if (!ix) return fail(MV_EINVAL, "null index");
+  DeviceGuard g(ix->device);
+  double acc[4] = {0, 0, 0, 0};
+  for (size_t i = 0; i + 5 <= ix->ev.size(); i += 5) {
+    CK(cudaEventSynchronize(ix->ev[i + 4]));
+    for (int s = 0; s < 4; ++s) {
+      float t = 0.f;
+      CK(cudaEventElapsedTime(&t, ix->ev[i + s], ix->ev[i + s + 1]));
+      acc[s] += t;
+    }
+  }
+  if (ms)
+    for (int s = 0; s < 4; ++s) ms[s] = acc[s];
+  if (searches) *searches = ix->prof_searches;
+  if (launches) *launches = ix->launches;
+  if (reset) {
+    for (cudaEvent_t e : ix->ev) cudaEventDestroy(e);
+    ix->ev.clear();
+    ix->prof_searches = 0;
+    ix->launches = 0;
+  }
+  return MV_OK;
+}
+
+mv_status mv_index_storage(const mv_index* ix, int64_t* list_off, int64_t* ids, uint8_t* codes) {
+  if (!ix) return fail(MV_EINVAL, "null index");
+  DeviceGuard g(ix->device);
+  if (list_off) CK(cudaMemcpy(list_off, ix->list_off, sizeof(int64_t) * (ix->nlist + 1), cudaMemcpyDefault));
+  if (ids && ix->ntotal) CK(cudaMemcpy(ids, ix->ids, sizeof(int64_t) * ix->ntotal, cudaMemcpyDefault));
+  if (codes && ix->ntotal) {
+    if (ix->type != MV_IVF_SQ8) return fail(MV_ESTATE, "codes requested from a non-SQ8 index");
+    CK(cudaMemcpy2D(codes, ix->d, ix->payload, ix->dpad, ix->d, ix->ntotal, cudaMemcpyDefault));
+  }
+  return MV_OK;
+}
+
+}  // extern "C"

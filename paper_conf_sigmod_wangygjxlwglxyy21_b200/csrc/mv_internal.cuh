@@ -1,0 +1,210 @@
+// mv_internal.cuh -- shared device helpers and host-side launcher declarations for libmv.
+// Nothing here is shared with oracle/ (tests/ compare the two).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+#include <string.h>
+#include <algorithm>
+
+#include "mv.h"
+
+#define MV_FULL 0xffffffffu
+#define MV_KEY_PAD 0xffffffffffffffffull
+
+namespace mv {
+
+constexpr int kMaxK = 16384;          // PAPER.md:801-802 (§3.3 fn. 5): k <= 16384
+constexpr int kLocalSelectMaxK = 1024;  // per-(query,list) selection in the scan for k <= 1024
+constexpr int kNumSMs = 148;
+
+__host__ __device__ __forceinline__ int64_t min64(int64_t a, int64_t b) { return a < b ? a : b; }
+__host__ __device__ __forceinline__ int64_t max64(int64_t a, int64_t b) { return a > b ? a : b; }
+
+// ------------------------------------------------------------------------------------------
+// Orderable keys.  A candidate is one u64: (distance key << 32) | id-rank.  The distance key
+// is the IEEE-754 order-preserving map of the "badness" (L2 distance, or -IP), so ascending
+// u64 order is the ABI's best-first order (distance, then id, then storage row) -- the id-rank
+// of a stored row is its position in the (id, row) sorted order (computed at add time).
+// ------------------------------------------------------------------------------------------
+__host__ __device__ __forceinline__ uint32_t f2key(float f) {
+#ifdef __CUDA_ARCH__
+  f = __fadd_rn(f, 0.0f);  // -0 -> +0: equal distances must give equal keys
+  uint32_t b = __float_as_uint(f);
+#else
+  f = f + 0.0f;
+  uint32_t b;
+  memcpy(&b, &f, 4);
+#endif
+  return (b & 0x80000000u) ? ~b : (b | 0x80000000u);
+}
+
+__host__ __device__ __forceinline__ float key2f(uint32_t k) {
+  uint32_t b = (k & 0x80000000u) ? (k ^ 0x80000000u) : ~k;
+#ifdef __CUDA_ARCH__
+  return __uint_as_float(b);
+#else
+  float f;
+  memcpy(&f, &b, 4);
+  return f;
+#endif
+}
+
+// badness key of a distance under the metric (L2: smaller better; IP: larger better)
+__device__ __forceinline__ uint32_t dist_key(float d, int metric) { return f2key(metric == MV_L2 ? d : -d); }
+__device__ __forceinline__ float key_dist(uint32_t k, int metric) {
+  float b = key2f(k);
+  return metric == MV_L2 ? b : -b;
+}
+
+__device__ __forceinline__ bool bit_excluded(const uint8_t* __restrict__ bitset, int64_t nbits, int64_t id) {
+  if (bitset == nullptr || id < 0 || id >= nbits) return false;
+  return (__ldg(bitset + (id >> 3)) >> (id & 7)) & 1;
+}
+
+// ------------------------------------------------------------------------------------------
+// Warp-cooperative insertion into a sorted (ascending) smem list of length L.  All 32 lanes
+// call it; lanes with `has` offer one candidate each.  Candidates not below the current last
+// element are dropped (the list keeps the L smallest keys seen; keys are unique).
+// ------------------------------------------------------------------------------------------
+__device__ __forceinline__ void warp_list_insert(uint64_t* list, int L, uint64_t cand, bool has) {
+  const int lane = threadIdx.x & 31;
+  uint32_t mask = __ballot_sync(MV_FULL, has && cand < list[L - 1]);
+  while (mask) {
+    const int src = __ffs(mask) - 1;
+    mask &= mask - 1;
+    const uint64_t c = __shfl_sync(MV_FULL, cand, src);
+    if (!(c < list[L - 1])) continue;  // uniform: every lane reads the same word
+    int pos = 0;
+    for (int base = 0; base < L; base += 32) {
+      const int i = base + lane;
+      pos += __popc(__ballot_sync(MV_FULL, i < L && list[i] < c));
+    }
+    for (int hi = L - 1; hi > pos; hi -= 32) {
+      const int i = hi - lane;
+      uint64_t v = 0;
+      const bool mv_ = i > pos;
+      if (mv_) v = list[i - 1];
+      __syncwarp();
+      if (mv_) list[i] = v;
+      __syncwarp();
+    }
+    if (lane == 0) list[pos] = c;
+    __syncwarp();
+  }
+}
+
+// Block-wide bitonic sort of n (power of two) u64 keys in shared memory, ascending.
+__device__ __forceinline__ void block_bitonic_sort(uint64_t* a, int n) {
+  for (int size = 2; size <= n; size <<= 1) {
+    for (int stride = size >> 1; stride > 0; stride >>= 1) {
+      __syncthreads();
+      for (int t = threadIdx.x; t < (n >> 1); t += blockDim.x) {
+        const int lo = 2 * t - (t & (stride - 1));
+        const int hi = lo + stride;
+        const bool up = ((lo & size) == 0);
+        const uint64_t x = a[lo], y = a[hi];
+        if ((x > y) == up) {
+          a[lo] = y;
+          a[hi] = x;
+        }
+      }
+    }
+  }
+  __syncthreads();
+}
+
+__host__ __device__ __forceinline__ int next_pow2(int x) {
+  int p = 1;
+  while (p < x) p <<= 1;
+  return p;
+}
+
+}  // namespace mv
+
+// ------------------------------------------------------------------------------------------
+// Host-side launchers (each .cu file owns its kernels).  All enqueue on `st` and return the
+// cudaError_t of the launch.
+// ------------------------------------------------------------------------------------------
+namespace mv {
+
+// k_add.cu
+cudaError_t launch_sq8_minmax(const float* x, int64_t n, int d, float* vmin, float* vdiff, cudaStream_t st);
+cudaError_t launch_prep_rows(const float* x, int64_t n, int d, int dpad, float* out, cudaStream_t st);
+cudaError_t launch_count_lists(const int32_t* lists, int64_t n, int32_t* counts, cudaStream_t st);
+cudaError_t launch_store_rows(int type, int metric, const float* xpad, const int64_t* ids, const int32_t* sorted_idx,
+                              const int32_t* sorted_list, int64_t n, int dpad, const int64_t* new_off,
+                              const int64_t* old_off, const int32_t* add_off, void* payload, float* norms,
+                              int64_t* out_ids, const float* vmin, const float* vdiff, const float* sq8_t,
+                              cudaStream_t st);
+cudaError_t launch_move_old(int type, int dpad, int nlist, const int64_t* old_off, const int64_t* new_off,
+                            const void* old_payload, const float* old_norms, const int64_t* old_ids,
+                            int64_t old_n, void* payload, float* norms, int64_t* ids, cudaStream_t st);
+cudaError_t launch_id_keys(const int64_t* ids, int64_t n, uint64_t* keys, uint32_t* vals, cudaStream_t st);
+cudaError_t launch_rank_scatter(const uint64_t* skeys, const uint32_t* svals, int64_t n, uint32_t* rank,
+                                int64_t* sorted_ids, cudaStream_t st);
+cudaError_t launch_check_ids(const int64_t* ids, int64_t n, int* flag, cudaStream_t st);
+cudaError_t launch_new_sizes(const int32_t* add, int nlist, const int64_t* old_off, int64_t* out, cudaStream_t st);
+cudaError_t launch_iota_i32(int32_t* out, int64_t n, cudaStream_t st);
+
+// k_coarse.cu
+cudaError_t launch_query_prep(const float* q, int64_t nq, int d, int dpad, float* qpad, float* qnorm, cudaStream_t st);
+cudaError_t launch_centroid_prep(const float* c, int nlist, int d, int dpad, float* cpad, float* cnorm, cudaStream_t st);
+cudaError_t launch_coarse(const float* qpad, int64_t nq, int dpad, const float* cpad, const float* cnorm, int nlist,
+                          int metric, int nprobe, int32_t* probes, cudaStream_t st);
+
+// k_bucket.cu
+struct Bucketing {
+  int32_t* lcount;   // nlist      pairs per list
+  int32_t* boff;     // nlist+1    exclusive scan of lcount
+  int32_t* bfill;    // nlist      scratch
+  int32_t* bq;       // nq*npb     pair ids grouped by list
+  int32_t* wcount;   // nlist      work items per list
+  int32_t* woff;     // nlist+1
+  int2* witems;      // <= nlist + nq*npb   (list, first bucket position)
+  int64_t* qtot;     // nq+1       per-query candidate capacity, then exclusive scan
+  int64_t* poff;     // nq*npb     region offset per pair
+  int32_t* pcnt;     // nq*npb     candidates written per pair
+  int32_t* counter;  // 1          persistent scan work counter
+};
+cudaError_t launch_bucket(const int32_t* probes, int64_t nq, int npb, int nlist, const int64_t* list_off, int k,
+                          int qchunk, const Bucketing& b, cudaStream_t st);
+cudaError_t launch_pair_offsets(const int32_t* probes, int64_t nq, int npb, const int64_t* list_off, int k,
+                                const Bucketing& b, cudaStream_t st);
+cudaError_t launch_scan_i32(const int32_t* in, int n, int32_t* out, cudaStream_t st);   // out[n+1]
+cudaError_t launch_scan_i64(const int64_t* in, int64_t n, int64_t* out, cudaStream_t st);  // out[n+1]
+
+// k_scan.cu
+struct ScanArgs {
+  int type, metric, d, dpad, k, npb, qchunk, nlist;
+  const int64_t* list_off;
+  const void* payload;
+  const float* norms;
+  const int64_t* ids;
+  const uint32_t* rank;
+  const uint8_t* bitset;
+  int64_t nbits;
+  const float* qpad;
+  const float* qnorm;
+  const float* vmin;
+  const float* vdiff;
+  const float* sq8_t;  // 256-entry decode table t_c = (c + 0.5f) / 255.f
+  const int32_t* bq;
+  const int32_t* boff;
+  const int2* witems;
+  const int32_t* nwitems;  // device: woff[nlist]
+  int32_t* counter;
+  const int64_t* poff;
+  int32_t* pcnt;
+  uint64_t* part;
+};
+cudaError_t launch_scan(const ScanArgs& a, cudaStream_t st);
+
+// k_select.cu
+cudaError_t launch_final_select(const int64_t* poff, const int32_t* pcnt, const uint64_t* part, int64_t nq, int npb,
+                                int k, int metric, const int64_t* sorted_ids, float* out_d, int64_t* out_i,
+                                cudaStream_t st);
+cudaError_t launch_fill_pad(int64_t n, int metric, float* d, int64_t* i, cudaStream_t st);
+cudaError_t launch_merge2(int metric, const float* ad, const int64_t* ai, const float* bd, const int64_t* bi,
+                          int64_t nq, int k, float* od, int64_t* oi, cudaStream_t st);
+
+}  // namespace mv

@@ -1,0 +1,262 @@
+"""GPU parity: the CUDA path (through the C ABI) against the oracle on the same seeded inputs.
+
+Sizes span several tiles and ragged tails while the oracle still finishes in seconds.  The
+protocol is the conditional oracle of DESIGN.md §6: assignment checked first (equal or tied),
+then the oracle re-runs the scan with the GPU's accepted assignment and probes, and ids must
+match except at ties.  Integer-valued (SIFT-shaped) data are exact in fp32 and are compared
+bit-for-bit.
+"""
+import numpy as np
+import pytest
+import torch
+
+import mvgen as G
+import oracle as O
+from mvgen.kmeans import kmeans
+
+from ._parity import candidate_map, check_assignment, check_probes, check_topk, oracle_from_gpu_storage
+
+pytestmark = pytest.mark.gpu
+
+
+def _mv():
+    from paper_conf_sigmod_wangygjxlwglxyy21_b200 import Index, merge_topk
+    return Index, merge_topk
+
+
+def _sift(n, nq, d=128, n_micro=4096):
+    spec = G.SiftSpec(d=d, n_micro=n_micro)
+    return G.sift_base(n, d=d, spec=spec), G.sift_queries(nq, d=d, spec=spec)
+
+
+def _deep(n, nq, d=96, n_micro=4096):
+    spec = G.DeepSpec(d=d, n_micro=n_micro)
+    return G.deep_base(n, d=d, spec=spec), G.deep_queries(nq, d=d, spec=spec)
+
+
+def _build(X, ids, C, metric, kind, sq8_sample=None):
+    Index, _ = _mv()
+    ix = Index(X.shape[1], metric, kind, C.shape[0])
+    ix.set_centroids(C.cuda())
+    if kind == "sq8":
+        ix.train_sq8((X if sq8_sample is None else sq8_sample).cuda())
+    ix.add(X.cuda(), ids.cuda())
+    return ix
+
+
+def _run_conditional(ix, X, ids, C, Q, k, nprobe, metric_o, kind_o, bitset=None, nbits=0, atol=0.0, exact=False,
+                     sample_assign=None):
+    Xn, Cn, Qn, idn = X.numpy(), C.numpy(), Q.numpy(), ids.numpy()
+    sq8 = ix.get_sq8() if kind_o == O.SQ8 else None
+    oi, gl = oracle_from_gpu_storage(ix, metric_o, kind_o, Cn, Xn, idn, sq8)
+    check_assignment(gl, Xn, Cn, metric_o, sample=sample_assign)
+    P = ix.search_probes(Q.cuda(), nprobe).cpu().numpy()
+    check_probes(P, Qn, Cn, nprobe, metric_o)
+    bs_t = None if bitset is None else bitset.cuda()
+    D, I = ix.search(Q.cuda(), k, nprobe, bitset=bs_t, nbits=nbits)
+    torch.cuda.synchronize()
+    Do, Io, _ = oi.search(Qn, k, nprobe, bitset=None if bitset is None else bitset.numpy(), nbits=nbits, probes=P)
+    cm = [candidate_map(oi, Qn[i], P[i], None if bitset is None else bitset.numpy(), nbits) for i in range(len(Qn))]
+    frac = check_topk(D.cpu().numpy(), I.cpu().numpy(), Do, Io, cm, atol=atol, exact=exact)
+    return frac, D, I
+
+
+# --------------------------------------------------------------------------------------------
+def test_c1_exact_equals_bruteforce():
+    """configs[0]: 10k x 128 SIFT-shaped, nlist = nprobe = 64, 100 queries, k = 10: IVF_FLAT with
+    nprobe = nlist IS exact k-NN; integer data make fp32 exact -> bit-for-bit equality."""
+    X, Q = _sift(10_000, 100)
+    ids = torch.arange(10_000, dtype=torch.int64)
+    C = kmeans(X, 64, iters=8)
+    ix = _build(X, ids, C, "l2", "flat")
+    D, I = ix.search(Q.cuda(), 10, 64)
+    De, Ie = O.exact_knn(X.numpy(), ids.numpy(), Q.numpy(), 10, O.L2)
+    check_topk(D.cpu().numpy(), I.cpu().numpy(), De, Ie, exact=True)
+
+
+@pytest.mark.parametrize("n,nlist,nprobe,nq,k", [(20_000, 256, 16, 200, 10), (7_777, 97, 5, 61, 37)])
+def test_flat_l2_sift_conditional(n, nlist, nprobe, nq, k):
+    X, Q = _sift(n, nq)
+    ids = G.permuted_ids(n, seed=3)
+    C = kmeans(X, nlist, iters=6)
+    ix = _build(X, ids, C, "l2", "flat")
+    frac, _, _ = _run_conditional(ix, X, ids, C, Q, k, nprobe, O.L2, O.FLAT, exact=False)
+    assert frac == 1.0  # integer data: no ties can be broken differently except exact ties by id
+
+
+def test_flat_ip_deep_conditional():
+    X, Q = _deep(20_000, 150)
+    ids = torch.arange(20_000, dtype=torch.int64) * 2 + 1
+    C = kmeans(X, 128, iters=6, spherical=True)
+    ix = _build(X, ids, C, "ip", "flat")
+    frac, _, _ = _run_conditional(ix, X, ids, C, Q, 20, 8, O.IP, O.FLAT, atol=1e-6)
+    assert frac > 0.999
+
+
+@pytest.mark.parametrize("metric", ["ip", "l2"])
+def test_sq8_deep_bitset_conditional(metric):
+    """configs[2] shape (downsized): Deep-shaped SQ8 with a 10% deletion bitset, k = 100 (lists
+    longer than k -> in-scan selection)."""
+    X, Q = _deep(30_000, 120)
+    ids = torch.arange(30_000, dtype=torch.int64)
+    C = kmeans(X, 48, iters=6, spherical=True)
+    ix = _build(X, ids, C, metric, "sq8")
+    mo = O.IP if metric == "ip" else O.L2
+    # SQ8 params and codes are bit-exact with the oracle's codec
+    vmin, vdiff = ix.get_sq8()
+    ovmin, ovdiff = O.sq8_train(X.numpy())
+    assert np.array_equal(vmin, ovmin) and np.array_equal(vdiff, ovdiff)
+    off, sids, codes = ix.storage(codes=True)
+    assert np.array_equal(codes, O.sq8_encode(X.numpy()[sids], ovmin, ovdiff))
+    nbits = 30_000
+    bs = G.mod_bitset(nbits, 10)
+    frac, D, I = _run_conditional(ix, X, ids, C, Q, 100, 6, mo, O.SQ8, bitset=bs, nbits=nbits, atol=2e-6)
+    assert frac > 0.999
+    excl = G.unpack_bits(bs, nbits).numpy().astype(bool)
+    got = I.cpu().numpy()
+    assert not excl[got[got >= 0]].any()
+
+
+@pytest.mark.parametrize("k", [2048, 16384])
+def test_large_k(k):
+    """k > 1024: single-pass radix select == plain top-k of the oracle."""
+    n = 20_000
+    X, Q = _sift(n, 12)
+    ids = G.permuted_ids(n, seed=5)
+    C = kmeans(X, 40, iters=5)
+    ix = _build(X, ids, C, "l2", "flat")
+    nprobe = 40 if k == 16384 else 12
+    frac, D, I = _run_conditional(ix, X, ids, C, Q, k, nprobe, O.L2, O.FLAT)
+    assert frac == 1.0
+
+
+def test_large_k_rounds_crosscheck():
+    """The paper's rounds-of-1024 procedure on the oracle candidates gives the GPU answer."""
+    n = 6000
+    X, Q = _sift(n, 4)
+    ids = torch.arange(n, dtype=torch.int64)
+    C = kmeans(X, 8, iters=4)
+    ix = _build(X, ids, C, "l2", "flat")
+    D, I = ix.search(Q.cuda(), 3000, 8)
+    for i in range(4):
+        Dall = O.distances(Q.numpy()[i], X.numpy(), O.L2)
+        Dr, Ir = O.topk_rounds(Dall, ids.numpy(), np.arange(n), 3000, O.L2, round_k=1024)
+        assert np.array_equal(I.cpu().numpy()[i], Ir)
+
+
+def test_edge_cases():
+    Index, _ = _mv()
+    d = 20  # not a multiple of 32: zero padding
+    X = G.gaussian(500, d, seed=1)
+    Q = G.gaussian(9, d, seed=2)
+    C = X[:7].clone()
+    # empty index -> all padding
+    ix = Index(d, "l2", "flat", 7)
+    ix.set_centroids(C.cuda())
+    D, I = ix.search(Q.cuda(), 5, 3)
+    assert (I == -1).all() and torch.isinf(D).all()
+    # nq = 0
+    D0, I0 = ix.search(Q[:0].cuda(), 5, 3)
+    assert D0.shape == (0, 5)
+    ids = torch.arange(500, dtype=torch.int64)
+    ix.add(X.cuda(), ids.cuda())
+    # k > candidates -> padding; nprobe > nlist clamps; all-ones bitset -> padding
+    D, I = ix.search(Q.cuda(), 600, 100)
+    De, Ie = O.exact_knn(X.numpy(), ids.numpy(), Q.numpy(), 600, O.L2)
+    check_topk(D.cpu().numpy(), I.cpu().numpy(), De, Ie, atol=1e-4,
+               cmaps=[{i: dd for i, dd in zip(range(500), O.distances(Q.numpy()[j], X.numpy(), O.L2))} for j in range(9)])
+    ones = torch.full((63,), 255, dtype=torch.uint8)
+    D, I = ix.search(Q.cuda(), 5, 7, bitset=ones.cuda(), nbits=500)
+    assert (I == -1).all()
+    # ids >= nbits are never excluded
+    D, I = ix.search(Q.cuda(), 5, 7, bitset=ones.cuda(), nbits=100)
+    assert (I >= 100).all()
+    # reserved id -1 rejected; k out of range rejected
+    from paper_conf_sigmod_wangygjxlwglxyy21_b200 import MvError
+    with pytest.raises(MvError):
+        ix.add(X[:2].cuda(), torch.tensor([3, -1]).cuda())
+    with pytest.raises(MvError):
+        ix.search(Q.cuda(), 16385, 3)
+    with pytest.raises(MvError):
+        ix.search(Q.cuda(), 0, 3)
+
+
+def test_duplicate_ids_and_incremental_add():
+    Index, _ = _mv()
+    X, Q = _sift(3000, 20, d=32, n_micro=64)
+    ids = torch.arange(3000, dtype=torch.int64) % 1000  # duplicates
+    C = kmeans(X, 16, iters=4)
+    ix = Index(32, "l2", "flat", 16)
+    ix.set_centroids(C.cuda())
+    ix.add(X[:1000].cuda(), ids[:1000].cuda())
+    ix.add(X[1000:].cuda(), ids[1000:].cuda())   # second add: lists keep insertion order
+    assert ix.ntotal == 3000
+    oi = O.IvfIndex(32, O.L2, O.FLAT, C.numpy())
+    oi.add(X.numpy(), ids.numpy())
+    off_o, order = oi.storage()
+    off_g, sids, _ = ix.storage()
+    assert np.array_equal(off_g, off_o) and np.array_equal(sids, ids.numpy()[order])
+    D, I = ix.search(Q.cuda(), 50, 4)
+    Do, Io, _ = oi.search(Q.numpy(), 50, 4)
+    check_topk(D.cpu().numpy(), I.cpu().numpy(), Do, Io, exact=True)
+
+
+def test_host_buffers_and_determinism():
+    X, Q = _sift(5000, 64, d=64, n_micro=256)
+    ids = torch.arange(5000, dtype=torch.int64)
+    C = kmeans(X, 32, iters=4)
+    ix = _build(X, ids, C, "l2", "flat")
+    Dd, Id = ix.search(Q.cuda(), 25, 5)
+    Dh = np.empty((64, 25), np.float32)
+    Ih = np.empty((64, 25), np.int64)
+    ix.search(Q.numpy(), 25, 5, out=(Dh, Ih))
+    assert np.array_equal(Dh, Dd.cpu().numpy()) and np.array_equal(Ih, Id.cpu().numpy())
+    D2, I2 = ix.search(Q.cuda(), 25, 5)
+    assert torch.equal(D2, Dd) and torch.equal(I2, Id)
+    # per-query results do not depend on the rest of the batch
+    D3, I3 = ix.search(Q[17:40].cuda(), 25, 5)
+    assert torch.equal(D3, Dd[17:40]) and torch.equal(I3, Id[17:40])
+
+
+@pytest.mark.parametrize("metric", ["l2", "ip"])
+@pytest.mark.parametrize("nsrc,k", [(2, 10), (3, 7), (8, 64), (4, 2048)])
+def test_merge_topk_vs_oracle(metric, nsrc, k):
+    _, merge_topk = _mv()
+    r = np.random.default_rng(nsrc * 100 + k)
+    mo = O.L2 if metric == "l2" else O.IP
+    nq = 33
+    X = r.integers(0, 5, (nsrc * 400, 3)).astype(np.float32)
+    ids = r.permutation(nsrc * 400).astype(np.int64)
+    Qn = r.integers(0, 5, (nq, 3)).astype(np.float32)
+    parts = [O.exact_knn(X[g::nsrc], ids[g::nsrc], Qn, k, mo) for g in range(nsrc)]
+    Ds = torch.tensor(np.stack([p[0] for p in parts]), dtype=torch.float32).cuda()
+    Is = torch.tensor(np.stack([p[1] for p in parts])).cuda()
+    D, I = merge_topk(Ds, Is, metric)
+    Do, Io = O.merge_topk(parts, k, mo)
+    check_topk(D.cpu().numpy(), I.cpu().numpy(), Do, Io, exact=True)
+
+
+@pytest.mark.slow
+def test_c2_full_size_sampled():
+    """configs[1] at full size (1M x 128, nlist 4096, nprobe 16, 10k queries, k 10) in the bench's
+    launch configuration; the oracle checks a seeded sample of assignments and queries."""
+    Index, _ = _mv()
+    n, nq = 1_000_000, 10_000
+    X = G.sift_base(n, device="cuda")
+    Q = G.sift_queries(nq, device="cuda")
+    ids = torch.arange(n, dtype=torch.int64, device="cuda")
+    C = kmeans(X, 4096, iters=10)
+    ix = Index(128, "l2", "flat", 4096)
+    ix.set_centroids(C)
+    ix.add(X, ids)
+    D, I = ix.search(Q, 10, 16)
+    torch.cuda.synchronize()
+    Xn, Cn = X.cpu().numpy(), C.cpu().numpy()
+    oi, gl = oracle_from_gpu_storage(ix, O.L2, O.FLAT, Cn, Xn, ids.cpu().numpy())
+    check_assignment(gl, Xn, Cn, O.L2, sample=2000)
+    sel = np.random.default_rng(7).choice(nq, 64, replace=False)
+    Qs = Q.cpu().numpy()[sel]
+    P = ix.search_probes(torch.tensor(Qs).cuda(), 16).cpu().numpy()
+    check_probes(P, Qs, Cn, 16, O.L2)
+    Do, Io, _ = oi.search(Qs, 10, 16, probes=P)
+    check_topk(D.cpu().numpy()[sel], I.cpu().numpy()[sel], Do, Io, exact=True)
