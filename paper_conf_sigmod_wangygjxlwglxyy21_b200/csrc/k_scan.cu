@@ -150,8 +150,9 @@ __global__ void __launch_bounds__(256) k_scan_simt(const ScanArgs a) {
       if (sel) {
         const uint64_t* L = lists + (int64_t)qi * k;
         int c = 0;
-        for (int j = lane; j < k; j += 32) {
-          const uint64_t v = L[j];
+        for (int j0 = 0; j0 < k; j0 += 32) {  // warp-uniform trip count: every lane reaches the ballot
+          const int j = j0 + lane;
+          const uint64_t v = j < k ? L[j] : MV_KEY_PAD;
           if (v != MV_KEY_PAD) a.part[a.poff[p] + j] = v;
           c += __popc(__ballot_sync(MV_FULL, v != MV_KEY_PAD));
         }
