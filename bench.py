@@ -391,6 +391,7 @@ def main():
                          "kernel": "k_scan (a5+a6)", "algorithmic_bytes_per_launch": scan_bytes,
                          "units_per_launch": units, "bytes_per_unit": bpv},
             "stage_ms": stage_ms,
+            "index": ix.describe(),
             "e2e": {"value": nq / (ms_e2e / 1e3), "unit": "queries/s", "h2d_bytes_per_step": nq * cfg["d"] * 4 +
                     ((nbits + 7) // 8 if bs is not None else 0), "d2h_bytes_per_step": nq * k * 12},
             "gpu_launches": launches,

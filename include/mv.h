@@ -145,6 +145,11 @@ MV_API mv_status mv_index_get_sq8(const mv_index* index, float* vmin, float* vdi
 MV_API mv_status mv_profile_enable(mv_index* index, int on);
 MV_API mv_status mv_profile_read(mv_index* index, double* ms, int64_t* searches, int64_t* launches, int reset);
 
+/* Human-readable index state (JSON object): d, nlist, ntotal, max list length, whether the
+ * tensor-core scan is available and which scan implementation the last search used.  Writes at
+ * most `len` bytes including the terminating NUL. */
+MV_API mv_status mv_index_describe(const mv_index* index, char* buf, size_t len);
+
 /* Release the index and all of its device storage (NULL is a no-op). */
 MV_API void mv_index_destroy(mv_index* index);
 

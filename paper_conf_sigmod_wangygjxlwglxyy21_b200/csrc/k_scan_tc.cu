@@ -1,0 +1,460 @@
+// k_scan_tc.cu -- §8 rows a5 + a6 on the 5th-generation tensor cores (sm_100a).
+//
+// PAPER.md:529-532 (§3.1) step (2): scan the nprobe probed buckets with the fine quantizer;
+// PAPER.md:916-922 (§4.1 B): the bitmap is checked for every encountered vector before the
+// top-k; PAPER.md:590-596 (§3.2.1): per-worker heaps merged at the end.  PAPER.md:569-575: the
+// loaded data vectors are reused for many queries -- here one 128-vector list tile in shared
+// memory meets every query of that list's bucket in one tensor-core contraction.
+//
+// Work item = (list l, <= qchunk queries probing l).  Persistent CTA per SM, warp-specialised:
+//   warp 0     TMA producer: list tiles (128 rows x one 128-B / 32-B swizzle atom per stage)
+//   warp 1     TMEM owner + single-thread tcgen05.mma issuer
+//              D[128 vectors x N] (+)= X_tile[128 x K] . Qplanes[N x K]^T, N = P x roundup16(nq)
+//   warps 2-3  query gatherer: the bucket's query planes -> swizzled K-major smem (double buffer)
+//   warps 4-7  epilogue: tcgen05.ld (row per thread) -> distance -> bitset -> transposed keys in
+//              smem -> one warp per query filters against its running k-th best (and the global
+//              per-query threshold tau) and inserts survivors (a6).
+// FLAT (kind::tf32): X = fp32 payload used as tf32 -- exact when the stored values are
+//   tf32-representable (integer SIFT data; the index checks this at add time); the query is
+//   split into hi + lo tf32 planes (P = 2), so the query side is exact to ~2^-22.
+// SQ8 (kind::i8): X = u8 codes straight from HBM; the query-side weights w_j = q_j * vdiff_j/255
+//   are expanded into P = 3 signed 8-bit digit planes with a per-query scale, so
+//   q.x_hat = q.a + s (D0 + D1/2^7 + D2/2^14) with int32-exact partials; no decode instructions.
+#include "mv_internal.cuh"
+#include "sm100.cuh"
+
+namespace mv {
+using namespace sm100;
+
+__device__ __forceinline__ void named_bar(int id, int n) { asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory"); }
+
+struct WorkInfo {
+  int l, bstart, nqc, len, ntiles;
+  int64_t lstart;
+};
+
+__device__ __forceinline__ WorkInfo work_info(const TcScanParams& p, int w) {
+  WorkInfo wi;
+  const int2 it = p.witems[w];
+  wi.l = it.x;
+  wi.bstart = it.y;
+  wi.nqc = min(p.qchunk, p.boff[wi.l + 1] - wi.bstart);
+  wi.lstart = p.list_off[wi.l];
+  wi.len = (int)(p.list_off[wi.l + 1] - wi.lstart);
+  wi.ntiles = (wi.len + 127) >> 7;
+  return wi;
+}
+
+template <int TYPE>
+__global__ void __launch_bounds__(256, 1) k_scan_tc(const __grid_constant__ CUtensorMap xmap, const TcScanParams p) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~(uintptr_t)1023);
+  constexpr int ESZ = TYPE == MV_IVF_FLAT ? 4 : 1;
+  constexpr int ATOM = TYPE == MV_IVF_FLAT ? 128 : 32;
+  constexpr int P = TYPE == MV_IVF_FLAT ? 2 : 3;
+  const int nstage = p.nstage, nchunks = p.nchunks, QC = p.qchunk, k = p.k;
+  const int rowbytes = p.dpad * ESZ;
+
+  uint8_t* Xs = sm + p.off_x;
+  uint8_t* Qs = sm + p.off_q;
+  uint32_t* Dt = reinterpret_cast<uint32_t*>(sm + p.off_dt);
+  uint64_t* lists = reinterpret_cast<uint64_t*>(sm + p.off_lists);
+  uint8_t* metab = sm + p.off_meta;
+  int32_t* ecnt = reinterpret_cast<int32_t*>(sm + p.off_misc);
+  uint32_t* rrank = reinterpret_cast<uint32_t*>(ecnt + 64);
+  uint64_t* bars = reinterpret_cast<uint64_t*>(sm + p.off_bar);
+  uint64_t* full_x = bars;
+  uint64_t* empty_x = bars + nstage;
+  uint64_t* full_q = empty_x + nstage;
+  uint64_t* empty_q = full_q + 2;
+  uint64_t* empty_m = empty_q + 2;
+  uint64_t* tfull = empty_m + 2;
+  uint64_t* tempty = tfull + 2;
+  uint32_t* tslot = reinterpret_cast<uint32_t*>(tempty + 2);
+
+  // metadata per Q buffer: pair[QC] i32 | qn[QC] f32 | qs[QC] f32 | qa[QC] f32 | lim[QC] u64
+  auto m_pair = [&](int b) { return reinterpret_cast<int32_t*>(metab + b * p.meta_bytes); };
+  auto m_qn = [&](int b) { return reinterpret_cast<float*>(metab + b * p.meta_bytes) + QC; };
+  auto m_qs = [&](int b) { return reinterpret_cast<float*>(metab + b * p.meta_bytes) + 2 * QC; };
+  auto m_qa = [&](int b) { return reinterpret_cast<float*>(metab + b * p.meta_bytes) + 3 * QC; };
+  auto m_lim = [&](int b) { return reinterpret_cast<uint64_t*>(metab + b * p.meta_bytes + p.meta_lim_off); };
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < nstage; ++s) {
+      mbar_init(&full_x[s], 1);
+      mbar_init(&empty_x[s], 1);
+    }
+    for (int b = 0; b < 2; ++b) {
+      mbar_init(&full_q[b], 64);
+      mbar_init(&empty_q[b], 1);
+      mbar_init(&empty_m[b], 4);
+      mbar_init(&tfull[b], 1);
+      mbar_init(&tempty[b], 4);
+    }
+    fence_mbar_init();
+  }
+  if (warp == 1) {
+    tmem_alloc(tslot, p.tmem_cols);
+    tmem_relinquish();
+  }
+  if (warp == 0 && lane == 0) tma_prefetch(&xmap);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tslot;
+  const int nwork = *p.nwitems;
+
+  if (warp == 0) {
+    // ------------------------------------------------------------------ TMA producer
+    if (lane == 0) {
+      uint32_t it = 0;
+      for (int w = blockIdx.x; w < nwork; w += gridDim.x) {
+        const WorkInfo wi = work_info(p, w);
+        for (int t = 0; t < wi.ntiles; ++t)
+          for (int c = 0; c < nchunks; ++c, ++it) {
+            const uint32_t s = it % nstage, r = it / nstage;
+            mbar_wait(&empty_x[s], (r & 1) ^ 1);
+            mbar_expect_tx(&full_x[s], 128 * ATOM);
+            tma_load_2d(Xs + s * 128 * ATOM, &xmap, &full_x[s], c * ATOM / ESZ, (int)(wi.lstart + t * 128));
+          }
+      }
+    }
+  } else if (warp == 1) {
+    // ------------------------------------------------------------------ MMA issuer
+    if (lane == 0) {
+      uint32_t it = 0, titer = 0, wcount = 0;
+      for (int w = blockIdx.x; w < nwork; w += gridDim.x, ++wcount) {
+        const WorkInfo wi = work_info(p, w);
+        const int NQ = (wi.nqc + 15) & ~15;
+        const int N = P * NQ;
+        const uint32_t idesc = TYPE == MV_IVF_FLAT ? idesc_tf32(N) : idesc_u8s8(N);
+        const uint32_t b = wcount & 1;
+        mbar_wait(&full_q[b], (wcount >> 1) & 1);
+        tc_fence_after();
+        const uint32_t qbase = smem_u32(Qs + b * p.q_bytes);
+        for (int t = 0; t < wi.ntiles; ++t, ++titer) {
+          const uint32_t a = titer & 1;
+          mbar_wait(&tempty[a], ((titer >> 1) & 1) ^ 1);
+          tc_fence_after();
+          const uint32_t dcol = tmem + a * p.ncol;
+          for (int c = 0; c < nchunks; ++c, ++it) {
+            const uint32_t s = it % nstage;
+            mbar_wait(&full_x[s], (it / nstage) & 1);
+            tc_fence_after();
+            const uint32_t xb = smem_u32(Xs + s * 128 * ATOM);
+            const uint32_t qb = qbase + c * N * ATOM;
+#pragma unroll
+            for (int ks = 0; ks < ATOM / 32; ++ks) {
+              const uint64_t ad = kmajor_desc(xb + ks * 32, ATOM);
+              const uint64_t bd = kmajor_desc(qb + ks * 32, ATOM);
+              if (TYPE == MV_IVF_FLAT) mma_tf32(dcol, ad, bd, idesc, (c | ks) != 0);
+              else mma_i8(dcol, ad, bd, idesc, (c | ks) != 0);
+            }
+            mma_commit(&empty_x[s]);
+          }
+          mma_commit(&tfull[a]);
+        }
+        mma_commit(&empty_q[b]);
+      }
+    }
+  } else if (warp < 4) {
+    // ------------------------------------------------------------------ query gatherer (64 thr)
+    const int tq = threadIdx.x - 64;
+    uint32_t wcount = 0;
+    for (int w = blockIdx.x; w < nwork; w += gridDim.x, ++wcount) {
+      const WorkInfo wi = work_info(p, w);
+      const int NQ = (wi.nqc + 15) & ~15;
+      const int N = P * NQ;
+      const uint32_t b = wcount & 1, r = wcount >> 1;
+      mbar_wait(&empty_q[b], (r & 1) ^ 1);
+      mbar_wait(&empty_m[b], (r & 1) ^ 1);
+      int32_t* mp = m_pair(b);
+      for (int i = tq; i < wi.nqc; i += 64) {
+        const int pr = p.bq[wi.bstart + i];
+        const int q = pr / p.npb;
+        mp[i] = pr;
+        m_qn(b)[i] = p.qnorm[q];
+        m_qs(b)[i] = TYPE == MV_IVF_SQ8 ? p.qscale[q] : 1.0f;
+        m_qa(b)[i] = TYPE == MV_IVF_SQ8 ? p.qa[q] : 0.0f;
+        m_lim(b)[i] = p.tau[q];
+      }
+      named_bar(2, 64);
+      uint8_t* Qb = Qs + b * p.q_bytes;
+      constexpr int PIECES = ATOM / 16;
+      const int total = wi.nqc * P * nchunks * PIECES;
+      for (int idx = tq; idx < total; idx += 64) {
+        const int pc = idx % PIECES;
+        int rest = idx / PIECES;
+        const int c = rest % nchunks;
+        rest /= nchunks;
+        const int pl = rest % P;
+        const int i = rest / P;
+        const int q = mp[i] / p.npb;
+        const uint4 v = __ldg(reinterpret_cast<const uint4*>(p.qplanes + ((int64_t)q * P + pl) * rowbytes + c * ATOM +
+                                                             pc * 16));
+        *reinterpret_cast<uint4*>(Qb + c * N * ATOM + swz_off(pl * NQ + i, pc, ATOM)) = v;
+      }
+      fence_proxy_async();
+      mbar_arrive(&full_q[b]);
+    }
+  } else {
+    // ------------------------------------------------------------------ epilogue (128 thr)
+    const int ew = warp - 4;
+    const int quarter = warp & 3;
+    const int row = quarter * 32 + lane;
+    const int et = threadIdx.x - 128;
+    uint32_t titer = 0, wcount = 0;
+    for (int w = blockIdx.x; w < nwork; w += gridDim.x, ++wcount) {
+      const WorkInfo wi = work_info(p, w);
+      const int NQ = (wi.nqc + 15) & ~15;
+      const uint32_t b = wcount & 1;
+      mbar_wait(&full_q[b], (wcount >> 1) & 1);
+      const int32_t* mp = m_pair(b);
+      const float* qn = m_qn(b);
+      const float* qs = m_qs(b);
+      const float* qa = m_qa(b);
+      const uint64_t* lim = m_lim(b);
+      const bool sel = (k <= kLocalSelectMaxK) && (wi.len > k);
+      if (sel)
+        for (int i = et; i < wi.nqc * k; i += 128) lists[i] = MV_KEY_PAD;
+      else
+        for (int i = et; i < wi.nqc; i += 128) ecnt[i] = 0;
+      named_bar(1, 128);
+      for (int t = 0; t < wi.ntiles; ++t, ++titer) {
+        const uint32_t a = titer & 1;
+        const int vrow = t * 128 + row;
+        const int64_t grow = wi.lstart + vrow;
+        bool valid = vrow < wi.len;
+        if (valid && p.bitset) valid = !bit_excluded(p.bitset, p.nbits, p.ids[grow]);
+        const float xn = (valid && p.metric == MV_L2) ? p.norms[grow] : 0.0f;
+        if (!sel) rrank[row] = valid ? p.rank[grow] : 0u;
+        mbar_wait(&tfull[a], (titer >> 1) & 1);
+        tc_fence_after();
+        const uint32_t tbase = tmem + a * p.ncol + ((uint32_t)(quarter * 32) << 16);
+        for (int qc = 0; qc < NQ; qc += 16) {
+          uint32_t r0[16], r1[16], r2[16];
+          tmem_ld16(tbase + qc, r0);
+          tmem_ld16(tbase + NQ + qc, r1);
+          if (P == 3) tmem_ld16(tbase + 2 * NQ + qc, r2);
+          tmem_wait_ld();
+#pragma unroll
+          for (int j = 0; j < 16; ++j) {
+            const int i = qc + j;
+            if (i < wi.nqc) {
+              float dot;
+              if (TYPE == MV_IVF_FLAT) {
+                dot = __uint_as_float(r0[j]) + __uint_as_float(r1[j]);
+              } else {
+                const float acc = (float)(int)r0[j] + (float)(int)r1[j] * (1.0f / 128.0f) +
+                                  (float)(int)r2[j] * (1.0f / 16384.0f);
+                dot = fmaf(qs[i], acc, qa[i]);
+              }
+              const float dist = p.metric == MV_L2 ? (qn[i] + xn) - 2.0f * dot : dot;
+              Dt[i * 128 + row] = valid ? dist_key(dist, p.metric) : 0xffffffffu;
+            }
+          }
+        }
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&tempty[a]);
+        named_bar(1, 128);
+        // ---- a6: per-query filtering + insertion (one warp per query slot)
+        for (int i = ew; i < wi.nqc; i += 4) {
+          const int pr = mp[i];
+          const uint64_t li = lim[i];
+#pragma unroll
+          for (int m = 0; m < 4; ++m) {
+            const int v = m * 32 + lane;
+            const uint32_t k32 = Dt[i * 128 + v];
+            if (sel) {
+              uint64_t* L = lists + (int64_t)i * k;
+              const uint64_t thr = L[k - 1] < li ? L[k - 1] : li;
+              bool pass = k32 != 0xffffffffu && k32 <= (uint32_t)(thr >> 32);
+              uint64_t key = MV_KEY_PAD;
+              if (pass) key = ((uint64_t)k32 << 32) | p.rank[wi.lstart + t * 128 + v];
+              pass = pass && key < li;
+              warp_list_insert(L, k, key, pass);
+            } else {
+              const uint64_t key = ((uint64_t)k32 << 32) | rrank[v];
+              const bool pass = k32 != 0xffffffffu && key < li;
+              const uint32_t msk = __ballot_sync(MV_FULL, pass);
+              const int base = ecnt[i];
+              if (pass) p.part[p.poff[pr] + base + __popc(msk & ((1u << lane) - 1))] = key;
+              __syncwarp();
+              if (lane == 0) ecnt[i] = base + __popc(msk);
+              __syncwarp();
+            }
+          }
+        }
+        named_bar(1, 128);
+      }
+      // ---- finalize this work item's (query, list) partial results
+      for (int i = ew; i < wi.nqc; i += 4) {
+        const int pr = mp[i];
+        if (sel) {
+          const uint64_t* L = lists + (int64_t)i * k;
+          int c = 0;
+          for (int j0 = 0; j0 < k; j0 += 32) {
+            const int j = j0 + lane;
+            const uint64_t v = j < k ? L[j] : MV_KEY_PAD;
+            if (v != MV_KEY_PAD) p.part[p.poff[pr] + j] = v;
+            c += __popc(__ballot_sync(MV_FULL, v != MV_KEY_PAD));
+          }
+          if (lane == 0) {
+            p.pcnt[pr] = c;
+            if (L[k - 1] != MV_KEY_PAD) atomicMin(reinterpret_cast<unsigned long long*>(p.tau + pr / p.npb),
+                                                  (unsigned long long)L[k - 1]);
+          }
+        } else if (lane == 0) {
+          p.pcnt[pr] = ecnt[i];
+        }
+      }
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&empty_m[b]);
+      named_bar(1, 128);
+    }
+  }
+  __syncthreads();
+  if (warp == 1) {
+    tc_fence_after();
+    tmem_dealloc(tmem, p.tmem_cols);
+  }
+}
+
+// ----------------------------------------------------------------------------------------------
+// a1 for the tensor-core path: query planes.
+//   FLAT: [hi, lo] tf32 planes (hi = q with the 13 low mantissa bits cleared, lo = q - hi)
+//   SQ8 : w_j = q_j * b_j, b_j = vdiff_j / 255, a_j = vmin_j + 0.5 b_j; qa = q.a;
+//         s = max|w| / 127; three int8 digits of w / s (base 2^7); qscale = s
+// ----------------------------------------------------------------------------------------------
+__global__ void k_qplanes(int type, const float* __restrict__ qpad, int64_t nq, int dpad, const float* __restrict__ vmin,
+                          const float* __restrict__ vdiff, uint8_t* __restrict__ out, float* __restrict__ qscale,
+                          float* __restrict__ qa) {
+  const int lane = threadIdx.x & 31;
+  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t q = warp; q < nq; q += nwarps) {
+    const float* x = qpad + q * dpad;
+    if (type == MV_IVF_FLAT) {
+      float* o = reinterpret_cast<float*>(out) + q * 2 * dpad;
+      for (int j = lane; j < dpad; j += 32) {
+        const float v = x[j];
+        const float hi = __uint_as_float(__float_as_uint(v) & 0xffffe000u);
+        o[j] = hi;
+        o[dpad + j] = v - hi;
+      }
+    } else {
+      float amax = 0.0f, dot = 0.0f;
+      for (int j = lane; j < dpad; j += 32) {
+        const float bj = vdiff[j] / 255.0f;
+        const float aj = fmaf(0.5f, bj, vmin[j]);
+        const float w = x[j] * bj;
+        dot = fmaf(x[j], aj, dot);
+        amax = fmaxf(amax, fabsf(w));
+      }
+      for (int o = 16; o > 0; o >>= 1) {
+        amax = fmaxf(amax, __shfl_xor_sync(MV_FULL, amax, o));
+        dot += __shfl_xor_sync(MV_FULL, dot, o);
+      }
+      const float s = amax > 0.0f ? amax / 127.0f : 1.0f;
+      int8_t* o = reinterpret_cast<int8_t*>(out) + q * 3 * dpad;
+      for (int j = lane; j < dpad; j += 32) {
+        const float bj = vdiff[j] / 255.0f;
+        const float u = (x[j] * bj) / s;
+        const float d0 = rintf(u);
+        const float r1 = (u - d0) * 128.0f;
+        const float d1 = rintf(r1);
+        const float r2 = (r1 - d1) * 128.0f;
+        const float d2 = fminf(fmaxf(rintf(r2), -127.0f), 127.0f);
+        o[j] = (int8_t)fminf(fmaxf(d0, -127.0f), 127.0f);
+        o[dpad + j] = (int8_t)fminf(fmaxf(d1, -127.0f), 127.0f);
+        o[2 * dpad + j] = (int8_t)d2;
+      }
+      if (lane == 0) {
+        qscale[q] = s;
+        qa[q] = dot;
+      }
+    }
+  }
+}
+
+cudaError_t launch_qplanes(int type, const float* qpad, int64_t nq, int dpad, const float* vmin, const float* vdiff,
+                           uint8_t* out, float* qscale, float* qa, cudaStream_t st) {
+  if (nq == 0) return cudaSuccess;
+  const int grid = (int)min64(kNumSMs * 16, (nq * 32 + 255) / 256);
+  k_qplanes<<<grid, 256, 0, st>>>(type, qpad, nq, dpad, vmin, vdiff, out, qscale, qa);
+  return cudaGetLastError();
+}
+
+// any stored fp32 value with low mantissa bits set (not exactly representable in tf32)?
+__global__ void k_tf32_check(const uint32_t* __restrict__ x, int64_t n, int* flag) {
+  bool bad = false;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    bad |= (x[i] & 0x1fffu) != 0;
+  if (__syncthreads_or(bad) && threadIdx.x == 0) atomicOr(flag, 1);
+}
+
+cudaError_t launch_tf32_check(const float* x, int64_t n, int* flag, cudaStream_t st) {
+  if (n == 0) return cudaSuccess;
+  const int grid = (int)min64(kNumSMs * 8, (n + 255) / 256);
+  k_tf32_check<<<grid, 256, 0, st>>>(reinterpret_cast<const uint32_t*>(x), n, flag);
+  return cudaGetLastError();
+}
+
+// ----------------------------------------------------------------------------------------------
+bool tc_scan_plan(int type, int dpad, int k, TcScanParams& p) {
+  const int esz = type == MV_IVF_FLAT ? 4 : 1;
+  const int atom = type == MV_IVF_FLAT ? 128 : 32;
+  const int P = type == MV_IVF_FLAT ? 2 : 3;
+  const int qcmax = type == MV_IVF_FLAT ? 48 : 64;
+  p.type = type;
+  p.dpad = dpad;
+  p.k = k;
+  p.nchunks = dpad * esz / atom;
+  int qc = qcmax;
+  if (k <= kLocalSelectMaxK) qc = std::max(1, std::min(qcmax, 53248 / (8 * k)));
+  p.qchunk = qc;
+  const int qcp = (qc + 15) & ~15;
+  p.ncol = P * qcp;
+  int cols = 32;
+  while (cols < 2 * p.ncol) cols <<= 1;
+  if (cols > 512) return false;
+  p.tmem_cols = cols;
+  auto up = [](int x, int a) { return (x + a - 1) / a * a; };
+  p.q_bytes = up(P * qcp * dpad * esz, 1024);
+  const int dt_bytes = qc * 128 * 4;
+  const int lists_bytes = k <= kLocalSelectMaxK ? qc * k * 8 : 0;
+  p.meta_lim_off = up(16 * qc, 8);
+  p.meta_bytes = up(p.meta_lim_off + 8 * qc, 16);
+  const int misc_bytes = 64 * 4 + 128 * 4;
+  const int stage = 128 * atom;
+  const int fixed = 2 * p.q_bytes + up(dt_bytes, 16) + up(lists_bytes, 16) + 2 * p.meta_bytes + misc_bytes;
+  const int budget = 227 * 1024 - 1024 - 512;  // alignment slack + barriers
+  int ns = (budget - fixed) / stage;
+  ns = std::min(ns, type == MV_IVF_FLAT ? 8 : 24);
+  if (ns < 2) return false;
+  p.nstage = ns;
+  p.off_x = 0;
+  p.off_q = ns * stage;
+  p.off_dt = p.off_q + 2 * p.q_bytes;
+  p.off_lists = p.off_dt + up(dt_bytes, 16);
+  p.off_meta = p.off_lists + up(lists_bytes, 16);
+  p.off_misc = p.off_meta + 2 * p.meta_bytes;
+  p.off_bar = up(p.off_misc + misc_bytes, 16);
+  p.smem_total = p.off_bar + (2 * ns + 10) * 8 + 16 + 1024;
+  return p.smem_total <= 227 * 1024;
+}
+
+cudaError_t launch_scan_tc(const CUtensorMap& xmap, const TcScanParams& p, cudaStream_t st) {
+  auto kern = p.type == MV_IVF_FLAT ? k_scan_tc<MV_IVF_FLAT> : k_scan_tc<MV_IVF_SQ8>;
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, p.smem_total);
+  if (e != cudaSuccess) return e;
+  int dev = 0, nsm = kNumSMs;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+  kern<<<nsm, 256, p.smem_total, st>>>(xmap, p);
+  return cudaGetLastError();
+}
+
+}  // namespace mv

@@ -3,12 +3,14 @@
 #include <cub/device/device_radix_sort.cuh>
 
 #include <cstdarg>
+#include <cstdlib>
 #include <cstdio>
 #include <cstring>
 #include <string>
 #include <vector>
 
 #include "mv_internal.cuh"
+#include "tmap.h"
 
 using namespace mv;
 
@@ -29,6 +31,11 @@ struct mv_index {
   int64_t* ids = nullptr;       // ntotal, storage order
   uint32_t* rank = nullptr;     // ntotal: position of (id, row) in sorted order
   int64_t* sorted_ids = nullptr;  // ntotal: ids in (id, row) order
+  // tensor-core scan state (rebuilt by every add)
+  CUtensorMap xmap;
+  bool xmap_ok = false;
+  bool tf32_exact = true;   // FLAT: every stored value exactly representable in tf32
+  const char* last_scan = "none";
   // profiling
   bool prof = false;
   std::vector<cudaEvent_t> ev;   // 5 events per profiled search
@@ -362,6 +369,11 @@ mv_status mv_index_add(mv_index* ix, const float* vectors, const int64_t* ids, i
   CK(s.alloc(reinterpret_cast<uint8_t**>(&t2), tmp2));
   CK(cub::DeviceRadixSort::SortPairs(t2, tmp2, keys, skeys, vals, svals, (int64_t)ntot, 0, 64, st));
   CK(launch_rank_scatter(skeys, svals, ntot, rank, sorted_ids, st));
+  if (ix->type == MV_IVF_FLAT) {
+    CK(cudaMemsetAsync(flag, 0, sizeof(int), st));
+    CK(launch_tf32_check(xpad, (int64_t)n * dpad, flag, st));
+    CK(cudaMemcpyAsync(&hflag, flag, sizeof(int), cudaMemcpyDeviceToHost, st));
+  }
   CK(cudaMemcpyAsync(ix->list_off, new_off, sizeof(int64_t) * (nlist + 1), cudaMemcpyDeviceToDevice, st));
   CK(cudaMemcpyAsync(ix->h_list_off.data(), new_off, sizeof(int64_t) * (nlist + 1), cudaMemcpyDeviceToHost, st));
   CK(cudaStreamSynchronize(st));
@@ -372,6 +384,12 @@ mv_status mv_index_add(mv_index* ix, const float* vectors, const int64_t* ids, i
   ix->rank = rank;
   ix->sorted_ids = sorted_ids;
   ix->ntotal = ntot;
+  if (ix->type == MV_IVF_FLAT && hflag) ix->tf32_exact = false;
+  ix->xmap_ok = ntot <= 0x7fffffffLL &&
+                make_tmap_2d(&ix->xmap, payload,
+                             ix->type == MV_IVF_FLAT ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_UINT8,
+                             (uint64_t)dpad, (uint64_t)ntot, (uint64_t)dpad * esize, 32, 128,
+                             ix->type == MV_IVF_FLAT ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_32B);
   ix->maxlen = 0;
   for (int l = 0; l < nlist; ++l) ix->maxlen = std::max(ix->maxlen, ix->h_list_off[l + 1] - ix->h_list_off[l]);
   return MV_OK;
@@ -455,8 +473,13 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
     CK(launch_query_prep(q, nq, ix->d, dpad, qpad, qnorm, st));
     CK(launch_coarse(qpad, nq, dpad, ix->cpad, ix->cnorm, nlist, ix->metric, npb, P, st));
     prof_mark(ix, st);
-    // a4
-    const int qchunk = k <= kLocalSelectMaxK ? std::min(64, std::max(1, 65536 / (8 * k))) : 64;
+    // a4 (work-item size depends on the scan implementation's shared-memory plan)
+    TcScanParams tp;
+    const char* force = getenv("MV_FORCE_SIMT");
+    const bool use_tc = ix->xmap_ok && !(force && force[0] == '1') &&
+                        (ix->type == MV_IVF_SQ8 || ix->tf32_exact) && tc_scan_plan(ix->type, dpad, k, tp);
+    const int qchunk = use_tc ? tp.qchunk
+                              : (k <= kLocalSelectMaxK ? std::min(64, std::max(1, 65536 / (8 * k))) : 64);
     const int64_t npairs = nq * npb;
     Bucketing b;
     CK(s.alloc(&b.lcount, nlist));
@@ -487,6 +510,28 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
       return fail(MV_ENOMEM, "search: cannot allocate %lld candidate slots", (long long)cap);
     }
     // a5/a6
+    if (use_tc) {
+      const int P = ix->type == MV_IVF_FLAT ? 2 : 3;
+      const size_t esz = ix->type == MV_IVF_FLAT ? 4 : 1;
+      uint8_t* qplanes;
+      float *qscale, *qa;
+      uint64_t* tau;
+      CK(s.alloc(&qplanes, (size_t)nq * P * dpad * esz));
+      CK(s.alloc(&qscale, (size_t)nq));
+      CK(s.alloc(&qa, (size_t)nq));
+      CK(s.alloc(&tau, (size_t)nq));
+      CK(cudaMemsetAsync(tau, 0xff, sizeof(uint64_t) * nq, st));
+      CK(launch_qplanes(ix->type, qpad, nq, dpad, ix->vmin, ix->vdiff, qplanes, qscale, qa, st));
+      tp.metric = ix->metric; tp.npb = npb;
+      tp.list_off = ix->list_off; tp.norms = ix->norms; tp.ids = ix->ids; tp.rank = ix->rank;
+      tp.bitset = bs; tp.nbits = bs ? nbits : 0;
+      tp.qplanes = qplanes; tp.qnorm = qnorm; tp.qscale = qscale; tp.qa = qa;
+      tp.bq = b.bq; tp.boff = b.boff; tp.witems = b.witems; tp.nwitems = b.woff + nlist;
+      tp.poff = b.poff; tp.pcnt = b.pcnt; tp.part = part; tp.tau = tau;
+      CK(launch_scan_tc(ix->xmap, tp, st));
+      ix->last_scan = ix->type == MV_IVF_FLAT ? "tcgen05.tf32" : "tcgen05.i8";
+      ix->launches += 1;
+    } else {
     ScanArgs a;
     a.type = ix->type; a.metric = ix->metric; a.d = ix->d; a.dpad = dpad; a.k = k; a.npb = npb;
     a.qchunk = qchunk; a.nlist = nlist;
@@ -496,6 +541,8 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
     a.bq = b.bq; a.boff = b.boff; a.witems = b.witems; a.nwitems = b.woff + nlist; a.counter = b.counter;
     a.poff = b.poff; a.pcnt = b.pcnt; a.part = part;
     CK(launch_scan(a, st));
+    ix->last_scan = "simt";
+    }
     prof_mark(ix, st);
     // a7
     CK(launch_final_select(b.poff, b.pcnt, part, nq, npb, k, ix->metric, ix->sorted_ids, D, I, st));
@@ -554,6 +601,17 @@ mv_status mv_merge_topk(mv_metric metric, const float* dists, const int64_t* ids
   CK(cudaMemcpyAsync(out_d, cd[0], per * sizeof(float), cudaMemcpyDefault, st));
   CK(cudaMemcpyAsync(out_i, ci[0], per * sizeof(int64_t), cudaMemcpyDefault, st));
   if (host_out || sd || si) CK(cudaStreamSynchronize(st));
+  return MV_OK;
+}
+
+mv_status mv_index_describe(const mv_index* ix, char* buf, size_t len) {
+  if (!ix || !buf || len == 0) return fail(MV_EINVAL, "null argument");
+  snprintf(buf, len,
+           "{\"d\": %d, \"dpad\": %d, \"nlist\": %d, \"ntotal\": %lld, \"maxlen\": %lld, \"type\": \"%s\", "
+           "\"metric\": \"%s\", \"tensor_map\": %s, \"tf32_exact\": %s, \"last_scan\": \"%s\"}",
+           ix->d, ix->dpad, ix->nlist, (long long)ix->ntotal, (long long)ix->maxlen,
+           ix->type == MV_IVF_FLAT ? "IVF_FLAT" : "IVF_SQ8", ix->metric == MV_L2 ? "L2" : "IP",
+           ix->xmap_ok ? "true" : "false", ix->tf32_exact ? "true" : "false", ix->last_scan);
   return MV_OK;
 }
 

@@ -1,6 +1,7 @@
 // mv_internal.cuh -- shared device helpers and host-side launcher declarations for libmv.
 // Nothing here is shared with oracle/ (tests/ compare the two).
 #pragma once
+#include <cuda.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
 #include <string.h>
@@ -198,6 +199,35 @@ struct ScanArgs {
   uint64_t* part;
 };
 cudaError_t launch_scan(const ScanArgs& a, cudaStream_t st);
+
+// k_scan_tc.cu (tcgen05 path)
+struct TcScanParams {
+  int type, metric, dpad, k, npb, qchunk, nchunks, nstage, ncol, tmem_cols;
+  int off_x, off_q, q_bytes, off_dt, off_lists, off_meta, meta_bytes, meta_lim_off, off_misc, off_bar, smem_total;
+  const int64_t* list_off;
+  const float* norms;
+  const int64_t* ids;
+  const uint32_t* rank;
+  const uint8_t* bitset;
+  int64_t nbits;
+  const uint8_t* qplanes;  // nq x P x dpad (fp32 hi/lo planes or int8 digit planes)
+  const float* qnorm;
+  const float* qscale;
+  const float* qa;
+  const int32_t* bq;
+  const int32_t* boff;
+  const int2* witems;
+  const int32_t* nwitems;
+  const int64_t* poff;
+  int32_t* pcnt;
+  uint64_t* part;
+  uint64_t* tau;           // nq: global per-query threshold (u64 key), atomicMin-updated
+};
+bool tc_scan_plan(int type, int dpad, int k, TcScanParams& p);
+cudaError_t launch_scan_tc(const CUtensorMap& xmap, const TcScanParams& p, cudaStream_t st);
+cudaError_t launch_qplanes(int type, const float* qpad, int64_t nq, int dpad, const float* vmin, const float* vdiff,
+                           uint8_t* out, float* qscale, float* qa, cudaStream_t st);
+cudaError_t launch_tf32_check(const float* x, int64_t n, int* flag, cudaStream_t st);
 
 // k_select.cu
 cudaError_t launch_final_select(const int64_t* poff, const int32_t* pcnt, const uint64_t* part, int64_t nq, int npb,

@@ -148,6 +148,12 @@ class Index:
         L.check(self._lib.mv_profile_read(self._h, ms, C.byref(ns), C.byref(nl), int(reset)))
         return dict(zip(self.STAGES, list(ms))), int(ns.value), int(nl.value)
 
+    def describe(self) -> dict:
+        import json
+        buf = C.create_string_buffer(1024)
+        L.check(self._lib.mv_index_describe(self._h, buf, 1024))
+        return json.loads(buf.value.decode())
+
     # -- parity hooks --------------------------------------------------------------------------
     def storage(self, codes: bool = False):
         off = np.empty(self.nlist + 1, np.int64)

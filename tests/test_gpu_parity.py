@@ -260,3 +260,27 @@ def test_c2_full_size_sampled():
     check_probes(P, Qs, Cn, 16, O.L2)
     Do, Io, _ = oi.search(Qs, 10, 16, probes=P)
     check_topk(D.cpu().numpy()[sel], I.cpu().numpy()[sel], Do, Io, exact=True)
+
+
+@pytest.mark.parametrize("kind,metric,k", [("flat", "l2", 10), ("flat", "l2", 300), ("flat", "ip", 10),
+                                           ("sq8", "l2", 10), ("sq8", "ip", 64)])
+def test_tensor_core_path_matches_simt_path(kind, metric, k, monkeypatch):
+    """The tcgen05 scan (default) and the SIMT bring-up scan (MV_FORCE_SIMT=1) agree: bit-for-bit
+    ids on integer data; SQ8 distances within the digit-plane tolerance."""
+    X, Q = _sift(12_000, 300, n_micro=512)
+    ids = G.permuted_ids(12_000, seed=11)
+    C = kmeans(X, 64, iters=4)
+    ix = _build(X, ids, C, metric, kind)
+    D1, I1 = ix.search(Q.cuda(), k, 6)
+    assert ix.describe()["last_scan"].startswith("tcgen05")
+    monkeypatch.setenv("MV_FORCE_SIMT", "1")
+    D2, I2 = ix.search(Q.cuda(), k, 6)
+    torch.cuda.synchronize()
+    if kind == "flat":
+        assert torch.equal(I1, I2) and torch.equal(D1, D2)
+    else:
+        # distances agree position by position; ids may differ only where distances tie
+        assert torch.allclose(D1, D2, rtol=1e-5, atol=1e-3)
+        diff = I1 != I2
+        assert torch.allclose(D1[diff], D2[diff], rtol=1e-5, atol=1e-3)
+        assert (~diff).float().mean().item() > 0.99
