@@ -79,7 +79,7 @@ cudaError_t launch_count_lists(const int32_t* lists, int64_t n, int32_t* counts,
 __global__ void k_store_rows(int type, int metric, const float* __restrict__ xpad, const int64_t* __restrict__ ids,
                              const int32_t* __restrict__ sorted_idx, const int32_t* __restrict__ sorted_list, int64_t n,
                              int dpad, const int64_t* __restrict__ new_off, const int64_t* __restrict__ old_off,
-                             const int32_t* __restrict__ add_off, void* payload, float* norms, int64_t* out_ids,
+                             const int32_t* __restrict__ add_off, void* payload, double* norms, int64_t* out_ids,
                              const float* __restrict__ vmin, const float* __restrict__ vdiff,
                              const float* __restrict__ sq8_t) {
   const int lane = threadIdx.x & 31;
@@ -90,13 +90,13 @@ __global__ void k_store_rows(int type, int metric, const float* __restrict__ xpa
     const int l = sorted_list[t];
     const int64_t pos = new_off[l] + (old_off[l + 1] - old_off[l]) + (t - add_off[l]);
     const float* src = xpad + (int64_t)i * dpad;
-    float acc = 0.0f;
+    double acc = 0.0;
     if (type == MV_IVF_FLAT) {
       float* dst = reinterpret_cast<float*>(payload) + pos * dpad;
       for (int j = lane; j < dpad; j += 32) {
         const float v = src[j];
         dst[j] = v;
-        acc = fmaf(v, v, acc);
+        acc = fma((double)v, (double)v, acc);
       }
     } else {
       uint8_t* dst = reinterpret_cast<uint8_t*>(payload) + pos * dpad;
@@ -108,7 +108,7 @@ __global__ void k_store_rows(int type, int metric, const float* __restrict__ xpa
         const int code = (int)floorf(__fmul_rn(255.0f, tt));
         dst[j] = (uint8_t)code;
         const float xh = __fadd_rn(__fmul_rn(sq8_t[code], vd), vm);  // decode, oracle op order
-        acc = fmaf(xh, xh, acc);
+        acc = fma((double)xh, (double)xh, acc);
       }
     }
     for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(MV_FULL, acc, o);
@@ -121,7 +121,7 @@ __global__ void k_store_rows(int type, int metric, const float* __restrict__ xpa
 
 cudaError_t launch_store_rows(int type, int metric, const float* xpad, const int64_t* ids, const int32_t* sorted_idx,
                               const int32_t* sorted_list, int64_t n, int dpad, const int64_t* new_off,
-                              const int64_t* old_off, const int32_t* add_off, void* payload, float* norms,
+                              const int64_t* old_off, const int32_t* add_off, void* payload, double* norms,
                               int64_t* out_ids, const float* vmin, const float* vdiff, const float* sq8_t,
                               cudaStream_t st) {
   if (n == 0) return cudaSuccess;
@@ -133,8 +133,8 @@ cudaError_t launch_store_rows(int type, int metric, const float* xpad, const int
 
 // One block per list: move the list's previous rows to their new offsets.
 __global__ void k_move_old(int esize, int dpad, const int64_t* __restrict__ old_off, const int64_t* __restrict__ new_off,
-                           const uint8_t* __restrict__ old_payload, const float* __restrict__ old_norms,
-                           const int64_t* __restrict__ old_ids, uint8_t* payload, float* norms, int64_t* ids) {
+                           const uint8_t* __restrict__ old_payload, const double* __restrict__ old_norms,
+                           const int64_t* __restrict__ old_ids, uint8_t* payload, double* norms, int64_t* ids) {
   const int l = blockIdx.x;
   const int64_t s = old_off[l], e = old_off[l + 1], ns = new_off[l];
   const int64_t row_bytes = (int64_t)esize * dpad;
@@ -149,8 +149,8 @@ __global__ void k_move_old(int esize, int dpad, const int64_t* __restrict__ old_
 }
 
 cudaError_t launch_move_old(int type, int dpad, int nlist, const int64_t* old_off, const int64_t* new_off,
-                            const void* old_payload, const float* old_norms, const int64_t* old_ids, int64_t old_n,
-                            void* payload, float* norms, int64_t* ids, cudaStream_t st) {
+                            const void* old_payload, const double* old_norms, const int64_t* old_ids, int64_t old_n,
+                            void* payload, double* norms, int64_t* ids, cudaStream_t st) {
   if (old_n == 0) return cudaSuccess;
   const int esize = type == MV_IVF_FLAT ? 4 : 1;
   k_move_old<<<nlist, 256, 0, st>>>(esize, dpad, old_off, new_off, (const uint8_t*)old_payload, old_norms, old_ids,

@@ -45,15 +45,41 @@ __device__ __forceinline__ WorkInfo work_info(const TcScanParams& p, int w) {
   return wi;
 }
 
+constexpr int kNTS = 4;          // per-tile side-data ring slots
+// side slot: norms f64 [1152 B] | rank u32 [640 B] | ids i64 [1152 B]; each copied as the 16-B aligned
+// superset of the tile's 128 rows (the arrays are padded at allocation so the copy stays in bounds)
+constexpr int kSideBytes = 3072;
+constexpr int kSideRank = 1152, kSideIds = 1792;
+constexpr int kEpiWarps = 8;      // two epilogue warps per TMEM lane quarter
+constexpr int kThreads = 128 + 32 * kEpiWarps;
+constexpr int kDLD = 129;         // padded transpose stride (conflict-free row and column access)
+
+// k-th smallest (1-indexed) of the 128 u32 values v[0..3] x 32 lanes: MSB-first bisection, one
+// ballot per value per bit, no divergence.
+__device__ __forceinline__ uint32_t warp_kth_u32(const uint32_t (&v)[4], int k) {
+  uint32_t ans = 0;
+#pragma unroll 1
+  for (int b = 31; b >= 0; --b) {
+    const uint32_t trial = ans | (1u << b);
+    int cnt = 0;
+#pragma unroll
+    for (int m = 0; m < 4; ++m) cnt += __popc(__ballot_sync(MV_FULL, v[m] < trial));
+    if (cnt < k) ans = trial;
+  }
+  return ans;
+}
+
 template <int TYPE>
-__global__ void __launch_bounds__(256, 1) k_scan_tc(const __grid_constant__ CUtensorMap xmap, const TcScanParams p) {
+__global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__ CUtensorMap xmap, const TcScanParams p) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~(uintptr_t)1023);
   constexpr int ESZ = TYPE == MV_IVF_FLAT ? 4 : 1;
   constexpr int ATOM = TYPE == MV_IVF_FLAT ? 128 : 32;
-  constexpr int P = TYPE == MV_IVF_FLAT ? 2 : 3;
+  constexpr int P = TYPE == MV_IVF_FLAT ? 2 : 4;
   const int nstage = p.nstage, nchunks = p.nchunks, QC = p.qchunk, k = p.k;
   const int rowbytes = p.dpad * ESZ;
+  const bool use_norms = p.metric == MV_L2;
+  const bool use_ids = p.bitset != nullptr;
 
   uint8_t* Xs = sm + p.off_x;
   uint8_t* Qs = sm + p.off_q;
@@ -61,7 +87,8 @@ __global__ void __launch_bounds__(256, 1) k_scan_tc(const __grid_constant__ CUte
   uint64_t* lists = reinterpret_cast<uint64_t*>(sm + p.off_lists);
   uint8_t* metab = sm + p.off_meta;
   int32_t* ecnt = reinterpret_cast<int32_t*>(sm + p.off_misc);
-  uint32_t* rrank = reinterpret_cast<uint32_t*>(ecnt + 64);
+  uint64_t* scratch = reinterpret_cast<uint64_t*>(sm + p.off_misc + 256);  // 32 per epilogue warp
+  uint8_t* side = sm + p.off_side;
   uint64_t* bars = reinterpret_cast<uint64_t*>(sm + p.off_bar);
   uint64_t* full_x = bars;
   uint64_t* empty_x = bars + nstage;
@@ -70,14 +97,16 @@ __global__ void __launch_bounds__(256, 1) k_scan_tc(const __grid_constant__ CUte
   uint64_t* empty_m = empty_q + 2;
   uint64_t* tfull = empty_m + 2;
   uint64_t* tempty = tfull + 2;
-  uint32_t* tslot = reinterpret_cast<uint32_t*>(tempty + 2);
+  uint64_t* full_t = tempty + 2;
+  uint64_t* empty_t = full_t + kNTS;
+  uint32_t* tslot = reinterpret_cast<uint32_t*>(empty_t + kNTS);
 
-  // metadata per Q buffer: pair[QC] i32 | qn[QC] f32 | qs[QC] f32 | qa[QC] f32 | lim[QC] u64
+  // metadata per Q buffer: pair[QC] i32 | qs[QC] f32 | (8-B aligned) lim[QC] u64 | qn[QC] f64 | qa[QC] f64
   auto m_pair = [&](int b) { return reinterpret_cast<int32_t*>(metab + b * p.meta_bytes); };
-  auto m_qn = [&](int b) { return reinterpret_cast<float*>(metab + b * p.meta_bytes) + QC; };
-  auto m_qs = [&](int b) { return reinterpret_cast<float*>(metab + b * p.meta_bytes) + 2 * QC; };
-  auto m_qa = [&](int b) { return reinterpret_cast<float*>(metab + b * p.meta_bytes) + 3 * QC; };
+  auto m_qs = [&](int b) { return reinterpret_cast<float*>(metab + b * p.meta_bytes) + QC; };
   auto m_lim = [&](int b) { return reinterpret_cast<uint64_t*>(metab + b * p.meta_bytes + p.meta_lim_off); };
+  auto m_qn = [&](int b) { return reinterpret_cast<double*>(metab + b * p.meta_bytes + p.meta_lim_off) + QC; };
+  auto m_qa = [&](int b) { return reinterpret_cast<double*>(metab + b * p.meta_bytes + p.meta_lim_off) + 2 * QC; };
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
@@ -88,9 +117,13 @@ __global__ void __launch_bounds__(256, 1) k_scan_tc(const __grid_constant__ CUte
     for (int b = 0; b < 2; ++b) {
       mbar_init(&full_q[b], 64);
       mbar_init(&empty_q[b], 1);
-      mbar_init(&empty_m[b], 4);
+      mbar_init(&empty_m[b], kEpiWarps);
       mbar_init(&tfull[b], 1);
-      mbar_init(&tempty[b], 4);
+      mbar_init(&tempty[b], kEpiWarps);
+    }
+    for (int s = 0; s < kNTS; ++s) {
+      mbar_init(&full_t[s], 1);
+      mbar_init(&empty_t[s], kEpiWarps);
     }
     fence_mbar_init();
   }
@@ -108,16 +141,26 @@ __global__ void __launch_bounds__(256, 1) k_scan_tc(const __grid_constant__ CUte
   if (warp == 0) {
     // ------------------------------------------------------------------ TMA producer
     if (lane == 0) {
-      uint32_t it = 0;
+      uint32_t it = 0, tcount = 0;
+      const uint32_t side_tx = 528 + (use_norms ? 1040 : 0) + (use_ids ? 1040 : 0);
       for (int w = blockIdx.x; w < nwork; w += gridDim.x) {
         const WorkInfo wi = work_info(p, w);
-        for (int t = 0; t < wi.ntiles; ++t)
+        for (int t = 0; t < wi.ntiles; ++t, ++tcount) {
+          const int row0 = (int)(wi.lstart + t * 128);
+          const uint32_t ts = tcount % kNTS, tr = tcount / kNTS;
+          mbar_wait(&empty_t[ts], (tr & 1) ^ 1);
+          mbar_expect_tx(&full_t[ts], side_tx);
+          uint8_t* sd = side + ts * kSideBytes;
+          bulk_g2s(sd + kSideRank, p.rank + (row0 & ~3), 528, &full_t[ts]);
+          if (use_norms) bulk_g2s(sd, p.norms + (row0 & ~1), 1040, &full_t[ts]);
+          if (use_ids) bulk_g2s(sd + kSideIds, p.ids + (row0 & ~1), 1040, &full_t[ts]);
           for (int c = 0; c < nchunks; ++c, ++it) {
             const uint32_t s = it % nstage, r = it / nstage;
             mbar_wait(&empty_x[s], (r & 1) ^ 1);
             mbar_expect_tx(&full_x[s], 128 * ATOM);
-            tma_load_2d(Xs + s * 128 * ATOM, &xmap, &full_x[s], c * ATOM / ESZ, (int)(wi.lstart + t * 128));
+            tma_load_2d(Xs + s * 128 * ATOM, &xmap, &full_x[s], c * ATOM / ESZ, row0);
           }
+        }
       }
     }
   } else if (warp == 1) {
@@ -176,13 +219,13 @@ __global__ void __launch_bounds__(256, 1) k_scan_tc(const __grid_constant__ CUte
         mp[i] = pr;
         m_qn(b)[i] = p.qnorm[q];
         m_qs(b)[i] = TYPE == MV_IVF_SQ8 ? p.qscale[q] : 1.0f;
-        m_qa(b)[i] = TYPE == MV_IVF_SQ8 ? p.qa[q] : 0.0f;
+        m_qa(b)[i] = TYPE == MV_IVF_SQ8 ? p.qa[q] : 0.0;
         m_lim(b)[i] = p.tau[q];
       }
       named_bar(2, 64);
       uint8_t* Qb = Qs + b * p.q_bytes;
       constexpr int PIECES = ATOM / 16;
-      const int total = wi.nqc * P * nchunks * PIECES;
+      const int total = (p.dbg & 4) ? 0 : wi.nqc * P * nchunks * PIECES;
       for (int idx = tq; idx < total; idx += 64) {
         const int pc = idx % PIECES;
         int rest = idx / PIECES;
@@ -191,19 +234,21 @@ __global__ void __launch_bounds__(256, 1) k_scan_tc(const __grid_constant__ CUte
         const int pl = rest % P;
         const int i = rest / P;
         const int q = mp[i] / p.npb;
-        const uint4 v = __ldg(reinterpret_cast<const uint4*>(p.qplanes + ((int64_t)q * P + pl) * rowbytes + c * ATOM +
-                                                             pc * 16));
-        *reinterpret_cast<uint4*>(Qb + c * N * ATOM + swz_off(pl * NQ + i, pc, ATOM)) = v;
+        cp_async16(Qb + c * N * ATOM + swz_off(pl * NQ + i, pc, ATOM),
+                   p.qplanes + ((int64_t)q * P + pl) * rowbytes + c * ATOM + pc * 16);
       }
+      cp_async_wait_all();
       fence_proxy_async();
       mbar_arrive(&full_q[b]);
     }
   } else {
-    // ------------------------------------------------------------------ epilogue (128 thr)
-    const int ew = warp - 4;
-    const int quarter = warp & 3;
+    // ------------------------------------------------------------------ epilogue (8 warps)
+    const int ew = warp - 4;            // 0..7
+    const int quarter = warp & 3;       // TMEM lane quarter this warp may access
+    const int half = ew >> 2;           // which 16-column chunks of the accumulator it reads
     const int row = quarter * 32 + lane;
-    const int et = threadIdx.x - 128;
+    const int et = threadIdx.x - 128;   // 0..255
+    uint64_t* wscr = scratch + ew * 32;
     uint32_t titer = 0, wcount = 0;
     for (int w = blockIdx.x; w < nwork; w += gridDim.x, ++wcount) {
       const WorkInfo wi = work_info(p, w);
@@ -211,73 +256,75 @@ __global__ void __launch_bounds__(256, 1) k_scan_tc(const __grid_constant__ CUte
       const uint32_t b = wcount & 1;
       mbar_wait(&full_q[b], (wcount >> 1) & 1);
       const int32_t* mp = m_pair(b);
-      const float* qn = m_qn(b);
+      const double* qn = m_qn(b);
       const float* qs = m_qs(b);
-      const float* qa = m_qa(b);
+      const double* qa = m_qa(b);
       const uint64_t* lim = m_lim(b);
       const bool sel = (k <= kLocalSelectMaxK) && (wi.len > k);
-      if (sel)
-        for (int i = et; i < wi.nqc * k; i += 128) lists[i] = MV_KEY_PAD;
-      else
-        for (int i = et; i < wi.nqc; i += 128) ecnt[i] = 0;
-      named_bar(1, 128);
+      if (sel) {
+        for (int i = et; i < wi.nqc * k; i += 32 * kEpiWarps) lists[i] = MV_KEY_PAD;
+      } else {
+        for (int i = et; i < wi.nqc; i += 32 * kEpiWarps) ecnt[i] = 0;
+      }
+      named_bar(1, 32 * kEpiWarps);
       for (int t = 0; t < wi.ntiles; ++t, ++titer) {
         const uint32_t a = titer & 1;
+        const uint32_t ts = titer % kNTS;
         const int vrow = t * 128 + row;
-        const int64_t grow = wi.lstart + vrow;
+        const int row0 = (int)(wi.lstart + t * 128);
+        mbar_wait(&full_t[ts], (titer / kNTS) & 1);
+        const uint8_t* sd = side + ts * kSideBytes;
+        const uint32_t* srank = reinterpret_cast<const uint32_t*>(sd + kSideRank) + (row0 & 3);
         bool valid = vrow < wi.len;
-        if (valid && p.bitset) valid = !bit_excluded(p.bitset, p.nbits, p.ids[grow]);
-        const float xn = (valid && p.metric == MV_L2) ? p.norms[grow] : 0.0f;
-        if (!sel) rrank[row] = valid ? p.rank[grow] : 0u;
+        if (valid && use_ids)
+          valid = !bit_excluded(p.bitset, p.nbits, reinterpret_cast<const int64_t*>(sd + kSideIds)[(row0 & 1) + row]);
+        const double xn = use_norms ? reinterpret_cast<const double*>(sd)[(row0 & 1) + row] : 0.0;
         mbar_wait(&tfull[a], (titer >> 1) & 1);
         tc_fence_after();
         const uint32_t tbase = tmem + a * p.ncol + ((uint32_t)(quarter * 32) << 16);
-        for (int qc = 0; qc < NQ; qc += 16) {
-          uint32_t r0[16], r1[16], r2[16];
-          tmem_ld16(tbase + qc, r0);
-          tmem_ld16(tbase + NQ + qc, r1);
-          if (P == 3) tmem_ld16(tbase + 2 * NQ + qc, r2);
+        for (int qc = half * 16; qc < ((p.dbg & 2) ? 0 : NQ); qc += 32) {
+          uint32_t r[P][16];
+#pragma unroll
+          for (int pl = 0; pl < P; ++pl) tmem_ld16(tbase + pl * NQ + qc, r[pl]);
           tmem_wait_ld();
 #pragma unroll
           for (int j = 0; j < 16; ++j) {
             const int i = qc + j;
             if (i < wi.nqc) {
-              float dot;
+              float dist;
               if (TYPE == MV_IVF_FLAT) {
-                dot = __uint_as_float(r0[j]) + __uint_as_float(r1[j]);
+                // exact for tf32-representable data (the only FLAT data this path accepts)
+                const float dot = __uint_as_float(r[0][j]) + __uint_as_float(r[1 % P][j]);
+                dist = use_norms ? ((float)qn[i] + (float)xn) - 2.0f * dot : dot;
               } else {
-                const float acc = (float)(int)r0[j] + (float)(int)r1[j] * (1.0f / 128.0f) +
-                                  (float)(int)r2[j] * (1.0f / 16384.0f);
-                dot = fmaf(qs[i], acc, qa[i]);
+                // int32-exact digit partials; the L2 expansion is combined in fp64 (the norms are
+                // ~400x the near-neighbour distances on SIFT-scale data)
+                const double acc = (double)(int)r[0][j] + (double)(int)r[1 % P][j] * (1.0 / 128.0) +
+                                   (double)(int)r[2 % P][j] * (1.0 / 16384.0) +
+                                   (double)(int)r[3 % P][j] * (1.0 / 2097152.0);
+                const double dot = fma((double)qs[i], acc, qa[i]);
+                dist = use_norms ? (float)((qn[i] + xn) - 2.0 * dot) : (float)dot;
               }
-              const float dist = p.metric == MV_L2 ? (qn[i] + xn) - 2.0f * dot : dot;
-              Dt[i * 128 + row] = valid ? dist_key(dist, p.metric) : 0xffffffffu;
+              Dt[i * kDLD + row] = valid ? dist_key(dist, p.metric) : 0xffffffffu;
             }
           }
         }
         tc_fence_before();
         __syncwarp();
         if (lane == 0) mbar_arrive(&tempty[a]);
-        named_bar(1, 128);
-        // ---- a6: per-query filtering + insertion (one warp per query slot)
-        for (int i = ew; i < wi.nqc; i += 4) {
+        named_bar(1, 32 * kEpiWarps);
+        // ---- a6: filter against min(list k-th, global tau) + select (one warp per query slot)
+        for (int i = ew; i < ((p.dbg & 1) ? 0 : wi.nqc); i += kEpiWarps) {
           const int pr = mp[i];
           const uint64_t li = lim[i];
+          uint32_t k32[4];
 #pragma unroll
-          for (int m = 0; m < 4; ++m) {
-            const int v = m * 32 + lane;
-            const uint32_t k32 = Dt[i * 128 + v];
-            if (sel) {
-              uint64_t* L = lists + (int64_t)i * k;
-              const uint64_t thr = L[k - 1] < li ? L[k - 1] : li;
-              bool pass = k32 != 0xffffffffu && k32 <= (uint32_t)(thr >> 32);
-              uint64_t key = MV_KEY_PAD;
-              if (pass) key = ((uint64_t)k32 << 32) | p.rank[wi.lstart + t * 128 + v];
-              pass = pass && key < li;
-              warp_list_insert(L, k, key, pass);
-            } else {
-              const uint64_t key = ((uint64_t)k32 << 32) | rrank[v];
-              const bool pass = k32 != 0xffffffffu && key < li;
+          for (int m = 0; m < 4; ++m) k32[m] = Dt[i * kDLD + m * 32 + lane];
+          if (!sel) {
+#pragma unroll
+            for (int m = 0; m < 4; ++m) {
+              const uint64_t key = ((uint64_t)k32[m] << 32) | srank[m * 32 + lane];
+              const bool pass = k32[m] != 0xffffffffu && key < li;
               const uint32_t msk = __ballot_sync(MV_FULL, pass);
               const int base = ecnt[i];
               if (pass) p.part[p.poff[pr] + base + __popc(msk & ((1u << lane) - 1))] = key;
@@ -285,12 +332,96 @@ __global__ void __launch_bounds__(256, 1) k_scan_tc(const __grid_constant__ CUte
               if (lane == 0) ecnt[i] = base + __popc(msk);
               __syncwarp();
             }
+            continue;
+          }
+          uint64_t* L = lists + (int64_t)i * k;
+          const uint64_t thr = L[k - 1] < li ? L[k - 1] : li;
+          const uint32_t thr32 = (uint32_t)(thr >> 32);
+          bool pass[4];
+          int npass = 0;
+#pragma unroll
+          for (int m = 0; m < 4; ++m) {
+            pass[m] = k32[m] != 0xffffffffu && k32[m] <= thr32;
+            npass += __popc(__ballot_sync(MV_FULL, pass[m]));
+          }
+          if (npass == 0) continue;
+          if (k <= 32 && npass > 32) {
+            // warm-up: narrow to the k smallest distance keys of this tile (plus exact ties)
+            uint32_t v[4];
+#pragma unroll
+            for (int m = 0; m < 4; ++m) v[m] = pass[m] ? k32[m] : 0xffffffffu;
+            const uint32_t t32 = warp_kth_u32(v, k);
+            npass = 0;
+#pragma unroll
+            for (int m = 0; m < 4; ++m) {
+              pass[m] = pass[m] && k32[m] <= t32;
+              npass += __popc(__ballot_sync(MV_FULL, pass[m]));
+            }
+          }
+          if (k <= 32 && npass <= 32 && npass > 2) {
+            // compact the survivors into one register per lane, sort, merge into the list
+            int off = 0;
+#pragma unroll
+            for (int m = 0; m < 4; ++m) {
+              const uint32_t bm = __ballot_sync(MV_FULL, pass[m]);
+              if (pass[m]) wscr[off + __popc(bm & ((1u << lane) - 1))] = ((uint64_t)k32[m] << 32) | srank[m * 32 + lane];
+              off += __popc(bm);
+            }
+            __syncwarp();
+            uint64_t c[1] = {lane < npass ? wscr[lane] : MV_KEY_PAD};
+            if (!(c[0] < thr)) c[0] = MV_KEY_PAD;
+            warp_bitonic_sort<1>(c);
+            uint64_t lv[1] = {lane < k ? L[lane] : MV_KEY_PAD};
+            warp_merge_smallest<1>(lv, c);
+            __syncwarp();
+            if (lane < k) L[lane] = lv[0];
+            __syncwarp();
+          } else if (npass <= 8 || k > 128) {
+#pragma unroll
+            for (int m = 0; m < 4; ++m) {
+              const uint64_t key = pass[m] ? (((uint64_t)k32[m] << 32) | srank[m * 32 + lane]) : MV_KEY_PAD;
+              warp_list_insert(L, k, key, pass[m] && key < thr);
+            }
+          } else {
+            uint64_t key[4];
+#pragma unroll
+            for (int m = 0; m < 4; ++m) {
+              key[m] = pass[m] ? (((uint64_t)k32[m] << 32) | srank[m * 32 + lane]) : MV_KEY_PAD;
+              if (!(key[m] < thr)) key[m] = MV_KEY_PAD;
+            }
+            warp_bitonic_sort<4>(key);
+            if (k <= 32) {
+              uint64_t lv[1] = {lane < k ? L[lane] : MV_KEY_PAD}, cv[1] = {key[0]};
+              warp_merge_smallest<1>(lv, cv);
+              __syncwarp();
+              if (lane < k) L[lane] = lv[0];
+            } else if (k <= 64) {
+              uint64_t lv[2], cv[2] = {key[0], key[1]};
+#pragma unroll
+              for (int r2 = 0; r2 < 2; ++r2) lv[r2] = r2 * 32 + lane < k ? L[r2 * 32 + lane] : MV_KEY_PAD;
+              warp_merge_smallest<2>(lv, cv);
+              __syncwarp();
+#pragma unroll
+              for (int r2 = 0; r2 < 2; ++r2)
+                if (r2 * 32 + lane < k) L[r2 * 32 + lane] = lv[r2];
+            } else {
+              uint64_t lv[4];
+#pragma unroll
+              for (int r2 = 0; r2 < 4; ++r2) lv[r2] = r2 * 32 + lane < k ? L[r2 * 32 + lane] : MV_KEY_PAD;
+              warp_merge_smallest<4>(lv, key);
+              __syncwarp();
+#pragma unroll
+              for (int r2 = 0; r2 < 4; ++r2)
+                if (r2 * 32 + lane < k) L[r2 * 32 + lane] = lv[r2];
+            }
+            __syncwarp();
           }
         }
-        named_bar(1, 128);
+        named_bar(1, 32 * kEpiWarps);
+        if (lane == 0) mbar_arrive(&empty_t[ts]);
       }
       // ---- finalize this work item's (query, list) partial results
-      for (int i = ew; i < wi.nqc; i += 4) {
+      for (int i = ew; i < wi.nqc; i += kEpiWarps) {
         const int pr = mp[i];
         if (sel) {
           const uint64_t* L = lists + (int64_t)i * k;
@@ -303,8 +434,8 @@ __global__ void __launch_bounds__(256, 1) k_scan_tc(const __grid_constant__ CUte
           }
           if (lane == 0) {
             p.pcnt[pr] = c;
-            if (L[k - 1] != MV_KEY_PAD) atomicMin(reinterpret_cast<unsigned long long*>(p.tau + pr / p.npb),
-                                                  (unsigned long long)L[k - 1]);
+            if (L[k - 1] != MV_KEY_PAD)
+              atomicMin(reinterpret_cast<unsigned long long*>(p.tau + pr / p.npb), (unsigned long long)L[k - 1]);
           }
         } else if (lane == 0) {
           p.pcnt[pr] = ecnt[i];
@@ -312,7 +443,7 @@ __global__ void __launch_bounds__(256, 1) k_scan_tc(const __grid_constant__ CUte
       }
       __syncwarp();
       if (lane == 0) mbar_arrive(&empty_m[b]);
-      named_bar(1, 128);
+      named_bar(1, 32 * kEpiWarps);
     }
   }
   __syncthreads();
@@ -326,16 +457,20 @@ __global__ void __launch_bounds__(256, 1) k_scan_tc(const __grid_constant__ CUte
 // a1 for the tensor-core path: query planes.
 //   FLAT: [hi, lo] tf32 planes (hi = q with the 13 low mantissa bits cleared, lo = q - hi)
 //   SQ8 : w_j = q_j * b_j, b_j = vdiff_j / 255, a_j = vmin_j + 0.5 b_j; qa = q.a;
-//         s = max|w| / 127; three int8 digits of w / s (base 2^7); qscale = s
+//         s = max|w| / 127; four int8 digits of w / s (base 2^7); qscale = s
 // ----------------------------------------------------------------------------------------------
 __global__ void k_qplanes(int type, const float* __restrict__ qpad, int64_t nq, int dpad, const float* __restrict__ vmin,
                           const float* __restrict__ vdiff, uint8_t* __restrict__ out, float* __restrict__ qscale,
-                          float* __restrict__ qa) {
+                          double* __restrict__ qa, double* __restrict__ qnorm) {
   const int lane = threadIdx.x & 31;
   const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
   for (int64_t q = warp; q < nq; q += nwarps) {
     const float* x = qpad + q * dpad;
+    double nn = 0.0;
+    for (int j = lane; j < dpad; j += 32) nn = fma((double)x[j], (double)x[j], nn);
+    for (int o = 16; o > 0; o >>= 1) nn += __shfl_xor_sync(MV_FULL, nn, o);
+    if (lane == 0) qnorm[q] = nn;
     if (type == MV_IVF_FLAT) {
       float* o = reinterpret_cast<float*>(out) + q * 2 * dpad;
       for (int j = lane; j < dpad; j += 32) {
@@ -345,34 +480,32 @@ __global__ void k_qplanes(int type, const float* __restrict__ qpad, int64_t nq, 
         o[dpad + j] = v - hi;
       }
     } else {
-      float amax = 0.0f, dot = 0.0f;
+      // fp64: w_j = q_j b_j, b_j = vdiff_j / 255, a_j = vmin_j + b_j / 2 (mid-bin decode)
+      double amax = 0.0, dot = 0.0;
       for (int j = lane; j < dpad; j += 32) {
-        const float bj = vdiff[j] / 255.0f;
-        const float aj = fmaf(0.5f, bj, vmin[j]);
-        const float w = x[j] * bj;
-        dot = fmaf(x[j], aj, dot);
-        amax = fmaxf(amax, fabsf(w));
+        const double bj = (double)vdiff[j] / 255.0;
+        const double aj = fma(0.5, bj, (double)vmin[j]);
+        dot = fma((double)x[j], aj, dot);
+        amax = fmax(amax, fabs((double)x[j] * bj));
       }
       for (int o = 16; o > 0; o >>= 1) {
-        amax = fmaxf(amax, __shfl_xor_sync(MV_FULL, amax, o));
+        amax = fmax(amax, __shfl_xor_sync(MV_FULL, amax, o));
         dot += __shfl_xor_sync(MV_FULL, dot, o);
       }
-      const float s = amax > 0.0f ? amax / 127.0f : 1.0f;
-      int8_t* o = reinterpret_cast<int8_t*>(out) + q * 3 * dpad;
+      // the scale is rounded up to fp32 first, so the digits and the epilogue use the same exact s
+      const double s = amax > 0.0 ? (double)__double2float_ru(amax / 127.0) : 1.0;
+      int8_t* o = reinterpret_cast<int8_t*>(out) + q * 4 * dpad;
       for (int j = lane; j < dpad; j += 32) {
-        const float bj = vdiff[j] / 255.0f;
-        const float u = (x[j] * bj) / s;
-        const float d0 = rintf(u);
-        const float r1 = (u - d0) * 128.0f;
-        const float d1 = rintf(r1);
-        const float r2 = (r1 - d1) * 128.0f;
-        const float d2 = fminf(fmaxf(rintf(r2), -127.0f), 127.0f);
-        o[j] = (int8_t)fminf(fmaxf(d0, -127.0f), 127.0f);
-        o[dpad + j] = (int8_t)fminf(fmaxf(d1, -127.0f), 127.0f);
-        o[2 * dpad + j] = (int8_t)d2;
+        double u = (double)x[j] * ((double)vdiff[j] / 255.0) / s;  // in [-127, 127]
+#pragma unroll
+        for (int dgt = 0; dgt < 4; ++dgt) {  // base-2^7 signed digits: u ~ d0 + d1/2^7 + d2/2^14 + d3/2^21
+          const double dd = fmin(fmax(rint(u), -127.0), 127.0);
+          o[dgt * dpad + j] = (int8_t)dd;
+          u = (u - dd) * 128.0;
+        }
       }
       if (lane == 0) {
-        qscale[q] = s;
+        qscale[q] = (float)s;
         qa[q] = dot;
       }
     }
@@ -380,10 +513,10 @@ __global__ void k_qplanes(int type, const float* __restrict__ qpad, int64_t nq, 
 }
 
 cudaError_t launch_qplanes(int type, const float* qpad, int64_t nq, int dpad, const float* vmin, const float* vdiff,
-                           uint8_t* out, float* qscale, float* qa, cudaStream_t st) {
+                           uint8_t* out, float* qscale, double* qa, double* qnorm, cudaStream_t st) {
   if (nq == 0) return cudaSuccess;
   const int grid = (int)min64(kNumSMs * 16, (nq * 32 + 255) / 256);
-  k_qplanes<<<grid, 256, 0, st>>>(type, qpad, nq, dpad, vmin, vdiff, out, qscale, qa);
+  k_qplanes<<<grid, 256, 0, st>>>(type, qpad, nq, dpad, vmin, vdiff, out, qscale, qa, qnorm);
   return cudaGetLastError();
 }
 
@@ -406,7 +539,7 @@ cudaError_t launch_tf32_check(const float* x, int64_t n, int* flag, cudaStream_t
 bool tc_scan_plan(int type, int dpad, int k, TcScanParams& p) {
   const int esz = type == MV_IVF_FLAT ? 4 : 1;
   const int atom = type == MV_IVF_FLAT ? 128 : 32;
-  const int P = type == MV_IVF_FLAT ? 2 : 3;
+  const int P = type == MV_IVF_FLAT ? 2 : 4;
   const int qcmax = type == MV_IVF_FLAT ? 48 : 64;
   p.type = type;
   p.dpad = dpad;
@@ -423,13 +556,14 @@ bool tc_scan_plan(int type, int dpad, int k, TcScanParams& p) {
   p.tmem_cols = cols;
   auto up = [](int x, int a) { return (x + a - 1) / a * a; };
   p.q_bytes = up(P * qcp * dpad * esz, 1024);
-  const int dt_bytes = qc * 128 * 4;
+  const int dt_bytes = qc * 129 * 4;
   const int lists_bytes = k <= kLocalSelectMaxK ? qc * k * 8 : 0;
-  p.meta_lim_off = up(16 * qc, 8);
-  p.meta_bytes = up(p.meta_lim_off + 8 * qc, 16);
-  const int misc_bytes = 64 * 4 + 128 * 4;
+  p.meta_lim_off = up(8 * qc, 8);
+  p.meta_bytes = up(p.meta_lim_off + 24 * qc, 16);
+  const int misc_bytes = 256 + 32 * 8 * kEpiWarps;
+  const int side_bytes = kNTS * kSideBytes;
   const int stage = 128 * atom;
-  const int fixed = 2 * p.q_bytes + up(dt_bytes, 16) + up(lists_bytes, 16) + 2 * p.meta_bytes + misc_bytes;
+  const int fixed = 2 * p.q_bytes + up(dt_bytes, 16) + up(lists_bytes, 16) + 2 * p.meta_bytes + misc_bytes + side_bytes;
   const int budget = 227 * 1024 - 1024 - 512;  // alignment slack + barriers
   int ns = (budget - fixed) / stage;
   ns = std::min(ns, type == MV_IVF_FLAT ? 8 : 24);
@@ -441,19 +575,20 @@ bool tc_scan_plan(int type, int dpad, int k, TcScanParams& p) {
   p.off_lists = p.off_dt + up(dt_bytes, 16);
   p.off_meta = p.off_lists + up(lists_bytes, 16);
   p.off_misc = p.off_meta + 2 * p.meta_bytes;
-  p.off_bar = up(p.off_misc + misc_bytes, 16);
-  p.smem_total = p.off_bar + (2 * ns + 10) * 8 + 16 + 1024;
+  p.off_side = up(p.off_misc + misc_bytes, 128);
+  p.off_bar = p.off_side + side_bytes;
+  p.smem_total = p.off_bar + (2 * ns + 10 + 2 * kNTS) * 8 + 16 + 1024;
   return p.smem_total <= 227 * 1024;
 }
 
-cudaError_t launch_scan_tc(const CUtensorMap& xmap, const TcScanParams& p, cudaStream_t st) {
+cudaError_t launch_scan_tc(const CUtensorMap* xmap, const TcScanParams& p, cudaStream_t st) {
   auto kern = p.type == MV_IVF_FLAT ? k_scan_tc<MV_IVF_FLAT> : k_scan_tc<MV_IVF_SQ8>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, p.smem_total);
   if (e != cudaSuccess) return e;
   int dev = 0, nsm = kNumSMs;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
-  kern<<<nsm, 256, p.smem_total, st>>>(xmap, p);
+  kern<<<nsm, kThreads, p.smem_total, st>>>(*xmap, p);
   return cudaGetLastError();
 }
 

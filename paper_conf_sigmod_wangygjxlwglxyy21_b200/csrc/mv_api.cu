@@ -27,7 +27,7 @@ struct mv_index {
   std::vector<int64_t> h_list_off;
   int64_t maxlen = 0;
   void* payload = nullptr;      // ntotal x dpad (fp32 or u8)
-  float* norms = nullptr;       // ntotal
+  double* norms = nullptr;      // ntotal (+pad): ||x||^2 / ||x_hat||^2 in fp64
   int64_t* ids = nullptr;       // ntotal, storage order
   uint32_t* rank = nullptr;     // ntotal: position of (id, row) in sorted order
   int64_t* sorted_ids = nullptr;  // ntotal: ids in (id, row) order
@@ -338,13 +338,19 @@ mv_status mv_index_add(mv_index* ix, const float* vectors, const int64_t* ids, i
   const int64_t ntot = ix->ntotal + n;
   const size_t esize = ix->type == MV_IVF_FLAT ? 4 : 1;
   void* payload = nullptr;
-  float* norms = nullptr;
+  double* norms = nullptr;
   int64_t *nids = nullptr, *sorted_ids = nullptr;
   uint32_t* rank = nullptr;
+  // per-row side arrays carry kSidePad zeroed tail elements: the scan bulk-copies 16-B aligned
+  // supersets of 128-row tiles
+  constexpr int64_t kSidePad = 256;
   cudaError_t e = cudaMalloc(&payload, (size_t)ntot * dpad * esize);
-  if (e == cudaSuccess) e = cudaMalloc(&norms, sizeof(float) * ntot);
-  if (e == cudaSuccess) e = cudaMalloc(&nids, sizeof(int64_t) * ntot);
-  if (e == cudaSuccess) e = cudaMalloc(&rank, sizeof(uint32_t) * ntot);
+  if (e == cudaSuccess) e = cudaMalloc(&norms, sizeof(double) * (ntot + kSidePad));
+  if (e == cudaSuccess) e = cudaMalloc(&nids, sizeof(int64_t) * (ntot + kSidePad));
+  if (e == cudaSuccess) e = cudaMalloc(&rank, sizeof(uint32_t) * (ntot + kSidePad));
+  if (e == cudaSuccess) e = cudaMemsetAsync(norms + ntot, 0, sizeof(double) * kSidePad, st);
+  if (e == cudaSuccess) e = cudaMemsetAsync(nids + ntot, 0, sizeof(int64_t) * kSidePad, st);
+  if (e == cudaSuccess) e = cudaMemsetAsync(rank + ntot, 0, sizeof(uint32_t) * kSidePad, st);
   if (e == cudaSuccess) e = cudaMalloc(&sorted_ids, sizeof(int64_t) * ntot);
   if (e != cudaSuccess) {
     cudaFree(payload); cudaFree(norms); cudaFree(nids); cudaFree(rank); cudaFree(sorted_ids);
@@ -511,24 +517,28 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
     }
     // a5/a6
     if (use_tc) {
-      const int P = ix->type == MV_IVF_FLAT ? 2 : 3;
+      const int P = ix->type == MV_IVF_FLAT ? 2 : 4;
       const size_t esz = ix->type == MV_IVF_FLAT ? 4 : 1;
       uint8_t* qplanes;
-      float *qscale, *qa;
+      float* qscale;
+      double *qa, *qn64;
       uint64_t* tau;
       CK(s.alloc(&qplanes, (size_t)nq * P * dpad * esz));
       CK(s.alloc(&qscale, (size_t)nq));
       CK(s.alloc(&qa, (size_t)nq));
+      CK(s.alloc(&qn64, (size_t)nq));
       CK(s.alloc(&tau, (size_t)nq));
       CK(cudaMemsetAsync(tau, 0xff, sizeof(uint64_t) * nq, st));
-      CK(launch_qplanes(ix->type, qpad, nq, dpad, ix->vmin, ix->vdiff, qplanes, qscale, qa, st));
+      CK(launch_qplanes(ix->type, qpad, nq, dpad, ix->vmin, ix->vdiff, qplanes, qscale, qa, qn64, st));
       tp.metric = ix->metric; tp.npb = npb;
       tp.list_off = ix->list_off; tp.norms = ix->norms; tp.ids = ix->ids; tp.rank = ix->rank;
       tp.bitset = bs; tp.nbits = bs ? nbits : 0;
-      tp.qplanes = qplanes; tp.qnorm = qnorm; tp.qscale = qscale; tp.qa = qa;
+      tp.qplanes = qplanes; tp.qnorm = qn64; tp.qscale = qscale; tp.qa = qa;
       tp.bq = b.bq; tp.boff = b.boff; tp.witems = b.witems; tp.nwitems = b.woff + nlist;
       tp.poff = b.poff; tp.pcnt = b.pcnt; tp.part = part; tp.tau = tau;
-      CK(launch_scan_tc(ix->xmap, tp, st));
+      const char* dbg = getenv("MV_SCAN_DEBUG");
+      tp.dbg = dbg ? atoi(dbg) : 0;
+      CK(launch_scan_tc(&ix->xmap, tp, st));
       ix->last_scan = ix->type == MV_IVF_FLAT ? "tcgen05.tf32" : "tcgen05.i8";
       ix->launches += 1;
     } else {

@@ -94,6 +94,78 @@ __device__ __forceinline__ void warp_list_insert(uint64_t* list, int L, uint64_t
   }
 }
 
+// ------------------------------------------------------------------------------------------
+// Warp-register bitonic networks over 32*R u64 keys; element e = r*32 + lane lives in v[r].
+// ------------------------------------------------------------------------------------------
+__device__ __forceinline__ uint64_t shfl_xor64(uint64_t v, int m) {
+  const uint32_t lo = __shfl_xor_sync(MV_FULL, (uint32_t)v, m);
+  const uint32_t hi = __shfl_xor_sync(MV_FULL, (uint32_t)(v >> 32), m);
+  return ((uint64_t)hi << 32) | lo;
+}
+__device__ __forceinline__ uint64_t shfl64(uint64_t v, int src) {
+  const uint32_t lo = __shfl_sync(MV_FULL, (uint32_t)v, src);
+  const uint32_t hi = __shfl_sync(MV_FULL, (uint32_t)(v >> 32), src);
+  return ((uint64_t)hi << 32) | lo;
+}
+__device__ __forceinline__ uint64_t umin64(uint64_t a, uint64_t b) { return a < b ? a : b; }
+__device__ __forceinline__ uint64_t umax64(uint64_t a, uint64_t b) { return a < b ? b : a; }
+
+// one compare-exchange step of a bitonic network: element pairs at distance `stride`, the
+// direction of block `size` ascending when (e & size) == 0 (size = 0 -> all ascending)
+template <int R>
+__device__ __forceinline__ void bitonic_step(uint64_t (&v)[R], int size, int stride) {
+  const int lane = threadIdx.x & 31;
+  if (stride >= 32) {
+    const int rs = stride >> 5;
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      if ((r & rs) == 0) {
+        const int e = r * 32 + lane;
+        const bool up = size == 0 || (e & size) == 0;
+        const uint64_t a = v[r], b = v[r | rs];
+        v[r] = up ? umin64(a, b) : umax64(a, b);
+        v[r | rs] = up ? umax64(a, b) : umin64(a, b);
+      }
+    }
+  } else {
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      const int e = r * 32 + lane;
+      const bool up = size == 0 || (e & size) == 0;
+      const bool lower = (lane & stride) == 0;
+      const uint64_t o = shfl_xor64(v[r], stride);
+      v[r] = (lower == up) ? umin64(v[r], o) : umax64(v[r], o);
+    }
+  }
+}
+
+template <int R>
+__device__ __forceinline__ void warp_bitonic_sort(uint64_t (&v)[R]) {
+#pragma unroll
+  for (int size = 2; size <= 32 * R; size <<= 1)
+#pragma unroll
+    for (int stride = size >> 1; stride > 0; stride >>= 1) bitonic_step<R>(v, size == 32 * R ? 0 : size, stride);
+}
+
+// bitonic sequence -> ascending
+template <int R>
+__device__ __forceinline__ void warp_bitonic_merge(uint64_t (&v)[R]) {
+#pragma unroll
+  for (int stride = 16 * R; stride > 0; stride >>= 1) bitonic_step<R>(v, 0, stride);
+}
+
+// list (sorted ascending, 32R entries) := smallest 32R of list U cand (cand sorted ascending)
+template <int R>
+__device__ __forceinline__ void warp_merge_smallest(uint64_t (&list)[R], const uint64_t (&cand)[R]) {
+  const int lane = threadIdx.x & 31;
+#pragma unroll
+  for (int r = 0; r < R; ++r) {
+    const uint64_t c = shfl64(cand[R - 1 - r], 31 - lane);  // reversed candidate element
+    list[r] = umin64(list[r], c);
+  }
+  warp_bitonic_merge<R>(list);
+}
+
 // Block-wide bitonic sort of n (power of two) u64 keys in shared memory, ascending.
 __device__ __forceinline__ void block_bitonic_sort(uint64_t* a, int n) {
   for (int size = 2; size <= n; size <<= 1) {
@@ -134,12 +206,12 @@ cudaError_t launch_prep_rows(const float* x, int64_t n, int d, int dpad, float* 
 cudaError_t launch_count_lists(const int32_t* lists, int64_t n, int32_t* counts, cudaStream_t st);
 cudaError_t launch_store_rows(int type, int metric, const float* xpad, const int64_t* ids, const int32_t* sorted_idx,
                               const int32_t* sorted_list, int64_t n, int dpad, const int64_t* new_off,
-                              const int64_t* old_off, const int32_t* add_off, void* payload, float* norms,
+                              const int64_t* old_off, const int32_t* add_off, void* payload, double* norms,
                               int64_t* out_ids, const float* vmin, const float* vdiff, const float* sq8_t,
                               cudaStream_t st);
 cudaError_t launch_move_old(int type, int dpad, int nlist, const int64_t* old_off, const int64_t* new_off,
-                            const void* old_payload, const float* old_norms, const int64_t* old_ids,
-                            int64_t old_n, void* payload, float* norms, int64_t* ids, cudaStream_t st);
+                            const void* old_payload, const double* old_norms, const int64_t* old_ids,
+                            int64_t old_n, void* payload, double* norms, int64_t* ids, cudaStream_t st);
 cudaError_t launch_id_keys(const int64_t* ids, int64_t n, uint64_t* keys, uint32_t* vals, cudaStream_t st);
 cudaError_t launch_rank_scatter(const uint64_t* skeys, const uint32_t* svals, int64_t n, uint32_t* rank,
                                 int64_t* sorted_ids, cudaStream_t st);
@@ -179,7 +251,7 @@ struct ScanArgs {
   int type, metric, d, dpad, k, npb, qchunk, nlist;
   const int64_t* list_off;
   const void* payload;
-  const float* norms;
+  const double* norms;
   const int64_t* ids;
   const uint32_t* rank;
   const uint8_t* bitset;
@@ -203,17 +275,18 @@ cudaError_t launch_scan(const ScanArgs& a, cudaStream_t st);
 // k_scan_tc.cu (tcgen05 path)
 struct TcScanParams {
   int type, metric, dpad, k, npb, qchunk, nchunks, nstage, ncol, tmem_cols;
-  int off_x, off_q, q_bytes, off_dt, off_lists, off_meta, meta_bytes, meta_lim_off, off_misc, off_bar, smem_total;
+  int off_x, off_q, q_bytes, off_dt, off_lists, off_meta, meta_bytes, meta_lim_off, off_misc, off_side, off_bar,
+      smem_total;
   const int64_t* list_off;
-  const float* norms;
+  const double* norms;     // ||x||^2 (FLAT) or ||x_hat||^2 (SQ8), fp64
   const int64_t* ids;
   const uint32_t* rank;
   const uint8_t* bitset;
   int64_t nbits;
   const uint8_t* qplanes;  // nq x P x dpad (fp32 hi/lo planes or int8 digit planes)
-  const float* qnorm;
+  const double* qnorm;     // ||q||^2 fp64
   const float* qscale;
-  const float* qa;
+  const double* qa;        // SQ8: q.a fp64
   const int32_t* bq;
   const int32_t* boff;
   const int2* witems;
@@ -222,11 +295,12 @@ struct TcScanParams {
   int32_t* pcnt;
   uint64_t* part;
   uint64_t* tau;           // nq: global per-query threshold (u64 key), atomicMin-updated
+  int dbg;                 // debug bitmask (MV_SCAN_DEBUG): 1 skip select, 2 skip epilogue math, 4 skip Q copy
 };
 bool tc_scan_plan(int type, int dpad, int k, TcScanParams& p);
-cudaError_t launch_scan_tc(const CUtensorMap& xmap, const TcScanParams& p, cudaStream_t st);
+cudaError_t launch_scan_tc(const CUtensorMap* xmap, const TcScanParams& p, cudaStream_t st);
 cudaError_t launch_qplanes(int type, const float* qpad, int64_t nq, int dpad, const float* vmin, const float* vdiff,
-                           uint8_t* out, float* qscale, float* qa, cudaStream_t st);
+                           uint8_t* out, float* qscale, double* qa, double* qnorm, cudaStream_t st);
 cudaError_t launch_tf32_check(const float* x, int64_t n, int* flag, cudaStream_t st);
 
 // k_select.cu

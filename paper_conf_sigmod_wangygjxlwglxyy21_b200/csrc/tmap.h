@@ -32,4 +32,17 @@ inline bool make_tmap_2d(CUtensorMap* m, const void* base, CUtensorMapDataType d
   return r == CUDA_SUCCESS;
 }
 
+// 1-D tensor [n] of `dt` elements, box of `box` elements (no swizzle).
+inline bool make_tmap_1d(CUtensorMap* m, const void* base, CUtensorMapDataType dt, uint64_t n, uint32_t box) {
+  auto enc = tmap_encoder();
+  if (!enc) return false;
+  cuuint64_t dims[1] = {n};
+  cuuint64_t strides[1] = {0};
+  cuuint32_t bx[1] = {box};
+  cuuint32_t es[1] = {1};
+  CUresult r = enc(m, dt, 1, const_cast<void*>(base), dims, strides, bx, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                   CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  return r == CUDA_SUCCESS;
+}
+
 }  // namespace mv
