@@ -54,21 +54,6 @@ constexpr int kEpiWarps = 8;      // two epilogue warps per TMEM lane quarter
 constexpr int kThreads = 128 + 32 * kEpiWarps;
 constexpr int kDLD = 129;         // padded transpose stride (conflict-free row and column access)
 
-// k-th smallest (1-indexed) of the 128 u32 values v[0..3] x 32 lanes: MSB-first bisection, one
-// ballot per value per bit, no divergence.
-__device__ __forceinline__ uint32_t warp_kth_u32(const uint32_t (&v)[4], int k) {
-  uint32_t ans = 0;
-#pragma unroll 1
-  for (int b = 31; b >= 0; --b) {
-    const uint32_t trial = ans | (1u << b);
-    int cnt = 0;
-#pragma unroll
-    for (int m = 0; m < 4; ++m) cnt += __popc(__ballot_sync(MV_FULL, v[m] < trial));
-    if (cnt < k) ans = trial;
-  }
-  return ans;
-}
-
 template <int TYPE>
 __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__ CUtensorMap xmap, const TcScanParams p) {
   extern __shared__ uint8_t smem_raw[];
@@ -234,8 +219,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
         const int pl = rest % P;
         const int i = rest / P;
         const int q = mp[i] / p.npb;
-        cp_async16(Qb + c * N * ATOM + swz_off(pl * NQ + i, pc, ATOM),
-                   p.qplanes + ((int64_t)q * P + pl) * rowbytes + c * ATOM + pc * 16);
+        const int64_t prow = TYPE == MV_IVF_FLAT ? (int64_t)pl * p.nq + q : (int64_t)q * P + pl;
+        cp_async16(Qb + c * N * ATOM + swz_off(pl * NQ + i, pc, ATOM), p.qplanes + prow * rowbytes + c * ATOM + pc * 16);
       }
       cp_async_wait_all();
       fence_proxy_async();
@@ -334,88 +319,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
             }
             continue;
           }
-          uint64_t* L = lists + (int64_t)i * k;
-          const uint64_t thr = L[k - 1] < li ? L[k - 1] : li;
-          const uint32_t thr32 = (uint32_t)(thr >> 32);
-          bool pass[4];
-          int npass = 0;
-#pragma unroll
-          for (int m = 0; m < 4; ++m) {
-            pass[m] = k32[m] != 0xffffffffu && k32[m] <= thr32;
-            npass += __popc(__ballot_sync(MV_FULL, pass[m]));
-          }
-          if (npass == 0) continue;
-          if (k <= 32 && npass > 32) {
-            // warm-up: narrow to the k smallest distance keys of this tile (plus exact ties)
-            uint32_t v[4];
-#pragma unroll
-            for (int m = 0; m < 4; ++m) v[m] = pass[m] ? k32[m] : 0xffffffffu;
-            const uint32_t t32 = warp_kth_u32(v, k);
-            npass = 0;
-#pragma unroll
-            for (int m = 0; m < 4; ++m) {
-              pass[m] = pass[m] && k32[m] <= t32;
-              npass += __popc(__ballot_sync(MV_FULL, pass[m]));
-            }
-          }
-          if (k <= 32 && npass <= 32 && npass > 2) {
-            // compact the survivors into one register per lane, sort, merge into the list
-            int off = 0;
-#pragma unroll
-            for (int m = 0; m < 4; ++m) {
-              const uint32_t bm = __ballot_sync(MV_FULL, pass[m]);
-              if (pass[m]) wscr[off + __popc(bm & ((1u << lane) - 1))] = ((uint64_t)k32[m] << 32) | srank[m * 32 + lane];
-              off += __popc(bm);
-            }
-            __syncwarp();
-            uint64_t c[1] = {lane < npass ? wscr[lane] : MV_KEY_PAD};
-            if (!(c[0] < thr)) c[0] = MV_KEY_PAD;
-            warp_bitonic_sort<1>(c);
-            uint64_t lv[1] = {lane < k ? L[lane] : MV_KEY_PAD};
-            warp_merge_smallest<1>(lv, c);
-            __syncwarp();
-            if (lane < k) L[lane] = lv[0];
-            __syncwarp();
-          } else if (npass <= 8 || k > 128) {
-#pragma unroll
-            for (int m = 0; m < 4; ++m) {
-              const uint64_t key = pass[m] ? (((uint64_t)k32[m] << 32) | srank[m * 32 + lane]) : MV_KEY_PAD;
-              warp_list_insert(L, k, key, pass[m] && key < thr);
-            }
-          } else {
-            uint64_t key[4];
-#pragma unroll
-            for (int m = 0; m < 4; ++m) {
-              key[m] = pass[m] ? (((uint64_t)k32[m] << 32) | srank[m * 32 + lane]) : MV_KEY_PAD;
-              if (!(key[m] < thr)) key[m] = MV_KEY_PAD;
-            }
-            warp_bitonic_sort<4>(key);
-            if (k <= 32) {
-              uint64_t lv[1] = {lane < k ? L[lane] : MV_KEY_PAD}, cv[1] = {key[0]};
-              warp_merge_smallest<1>(lv, cv);
-              __syncwarp();
-              if (lane < k) L[lane] = lv[0];
-            } else if (k <= 64) {
-              uint64_t lv[2], cv[2] = {key[0], key[1]};
-#pragma unroll
-              for (int r2 = 0; r2 < 2; ++r2) lv[r2] = r2 * 32 + lane < k ? L[r2 * 32 + lane] : MV_KEY_PAD;
-              warp_merge_smallest<2>(lv, cv);
-              __syncwarp();
-#pragma unroll
-              for (int r2 = 0; r2 < 2; ++r2)
-                if (r2 * 32 + lane < k) L[r2 * 32 + lane] = lv[r2];
-            } else {
-              uint64_t lv[4];
-#pragma unroll
-              for (int r2 = 0; r2 < 4; ++r2) lv[r2] = r2 * 32 + lane < k ? L[r2 * 32 + lane] : MV_KEY_PAD;
-              warp_merge_smallest<4>(lv, key);
-              __syncwarp();
-#pragma unroll
-              for (int r2 = 0; r2 < 4; ++r2)
-                if (r2 * 32 + lane < k) L[r2 * 32 + lane] = lv[r2];
-            }
-            __syncwarp();
-          }
+          warp_select_tile(lists + (int64_t)i * k, k, li, k32, [&](int v) { return srank[v]; }, wscr);
         }
         named_bar(1, 32 * kEpiWarps);
         if (lane == 0) mbar_arrive(&empty_t[ts]);
@@ -472,13 +376,7 @@ __global__ void k_qplanes(int type, const float* __restrict__ qpad, int64_t nq, 
     for (int o = 16; o > 0; o >>= 1) nn += __shfl_xor_sync(MV_FULL, nn, o);
     if (lane == 0) qnorm[q] = nn;
     if (type == MV_IVF_FLAT) {
-      float* o = reinterpret_cast<float*>(out) + q * 2 * dpad;
-      for (int j = lane; j < dpad; j += 32) {
-        const float v = x[j];
-        const float hi = __uint_as_float(__float_as_uint(v) & 0xffffe000u);
-        o[j] = hi;
-        o[dpad + j] = v - hi;
-      }
+      // FLAT planes are the plane-major hi/lo split made by launch_hilo (shared with the coarse step)
     } else {
       // fp64: w_j = q_j b_j, b_j = vdiff_j / 255, a_j = vmin_j + b_j / 2 (mid-bin decode)
       double amax = 0.0, dot = 0.0;

@@ -19,6 +19,9 @@ struct mv_index {
   bool has_centroids = false, has_sq8 = false;
   float* cpad = nullptr;    // nlist x dpad
   float* cnorm = nullptr;   // nlist
+  float* chl = nullptr;     // [2][nlist][dpad] tf32 hi / lo planes of the centroids (tcgen05 coarse)
+  CUtensorMap cmap;
+  bool cmap_ok = false;
   float* vmin = nullptr;    // dpad (zero padded)
   float* vdiff = nullptr;   // dpad (zero padded)
   float* sq8_t = nullptr;   // 256: (c + 0.5f) / 255.f
@@ -36,6 +39,7 @@ struct mv_index {
   bool xmap_ok = false;
   bool tf32_exact = true;   // FLAT: every stored value exactly representable in tf32
   const char* last_scan = "none";
+  const char* last_coarse = "none";
   // profiling
   bool prof = false;
   std::vector<cudaEvent_t> ev;   // 5 events per profiled search
@@ -152,6 +156,28 @@ void free_storage(mv_index* ix) {
 }
 }  // namespace
 
+// a2 + a3: tcgen05 coarse with fused top-nprobe when the shapes fit, else the SIMT kernel
+static cudaError_t run_coarse(mv_index* ix, const float* qpad, const float* qhl, int64_t nq, int npb, int32_t* P,
+                              cudaStream_t st) {
+  CoarseParams cp;
+  const char* force = getenv("MV_FORCE_SIMT");
+  if (npb < ix->nlist && ix->cmap_ok && !(force && force[0] == '1') && coarse_tc_plan(ix->dpad, npb, cp)) {
+    CUtensorMap qmap;
+    if (make_tmap_2d(&qmap, qhl, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, (uint64_t)ix->dpad, 2 * (uint64_t)nq,
+                     (uint64_t)ix->dpad * 4, 32, (uint32_t)cp.nqb, CU_TENSOR_MAP_SWIZZLE_128B)) {
+      cp.nq = nq;
+      cp.nlist = ix->nlist;
+      cp.metric = ix->metric;
+      cp.cnorm = ix->cnorm;
+      cp.probes = P;
+      ix->last_coarse = "tcgen05.tf32";
+      return launch_coarse_tc(&ix->cmap, &qmap, cp, nq, st);
+    }
+  }
+  ix->last_coarse = "simt";
+  return launch_coarse(qpad, nq, ix->dpad, ix->cpad, ix->cnorm, ix->nlist, ix->metric, npb, P, st);
+}
+
 // ------------------------------------------------------------------------------------------
 extern "C" {
 
@@ -212,6 +238,7 @@ void mv_index_destroy(mv_index* ix) {
   cudaFree(ix->list_off);
   cudaFree(ix->cpad);
   cudaFree(ix->cnorm);
+  cudaFree(ix->chl);
   cudaFree(ix->vmin);
   cudaFree(ix->vdiff);
   cudaFree(ix->sq8_t);
@@ -228,7 +255,11 @@ mv_status mv_index_set_centroids(mv_index* ix, const float* centroids) {
   const float* c;
   CK(stage_in(s, centroids, (size_t)ix->nlist * ix->d, &c, &staged));
   CK(launch_centroid_prep(c, ix->nlist, ix->d, ix->dpad, ix->cpad, ix->cnorm, st));
+  if (!ix->chl) CK(cudaMalloc(&ix->chl, sizeof(float) * 2 * (size_t)ix->nlist * ix->dpad));
+  CK(launch_hilo(c, ix->nlist, ix->d, ix->dpad, ix->chl, st));
   CK(cudaStreamSynchronize(st));
+  ix->cmap_ok = make_tmap_2d(&ix->cmap, ix->chl, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, (uint64_t)ix->dpad,
+                             2 * (uint64_t)ix->nlist, (uint64_t)ix->dpad * 4, 32, 128, CU_TENSOR_MAP_SWIZZLE_128B);
   ix->has_centroids = true;
   return MV_OK;
 }
@@ -434,7 +465,10 @@ mv_status mv_search_probes(mv_index* ix, const float* queries, int64_t nq, int32
   CK(s.alloc(&qpad, (size_t)nq * ix->dpad));
   CK(s.alloc(&qnorm, (size_t)nq));
   CK(launch_query_prep(q, nq, ix->d, ix->dpad, qpad, qnorm, st));
-  CK(launch_coarse(qpad, nq, ix->dpad, ix->cpad, ix->cnorm, ix->nlist, ix->metric, npb, P, st));
+  float* qhl;
+  CK(s.alloc(&qhl, (size_t)2 * nq * ix->dpad));
+  CK(launch_hilo(q, nq, ix->d, ix->dpad, qhl, st));
+  CK(run_coarse(ix, qpad, qhl, nq, npb, P, st));
   if (sp) {
     CK(cudaMemcpyAsync(probes, P, sizeof(int32_t) * nq * npb, cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
@@ -477,7 +511,10 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
     CK(s.alloc(&qnorm, (size_t)nq));
     CK(s.alloc(&P, (size_t)nq * npb));
     CK(launch_query_prep(q, nq, ix->d, dpad, qpad, qnorm, st));
-    CK(launch_coarse(qpad, nq, dpad, ix->cpad, ix->cnorm, nlist, ix->metric, npb, P, st));
+    float* qhl;  // plane-major tf32 hi/lo query planes: coarse B operand and the FLAT scan's query planes
+    CK(s.alloc(&qhl, (size_t)2 * nq * dpad));
+    CK(launch_hilo(q, nq, ix->d, dpad, qhl, st));
+    CK(run_coarse(ix, qpad, qhl, nq, npb, P, st));
     prof_mark(ix, st);
     // a4 (work-item size depends on the scan implementation's shared-memory plan)
     TcScanParams tp;
@@ -523,14 +560,16 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
       float* qscale;
       double *qa, *qn64;
       uint64_t* tau;
-      CK(s.alloc(&qplanes, (size_t)nq * P * dpad * esz));
+      if (ix->type == MV_IVF_SQ8) CK(s.alloc(&qplanes, (size_t)nq * P * dpad * esz));
+      else qplanes = reinterpret_cast<uint8_t*>(qhl);
       CK(s.alloc(&qscale, (size_t)nq));
       CK(s.alloc(&qa, (size_t)nq));
       CK(s.alloc(&qn64, (size_t)nq));
       CK(s.alloc(&tau, (size_t)nq));
       CK(cudaMemsetAsync(tau, 0xff, sizeof(uint64_t) * nq, st));
-      CK(launch_qplanes(ix->type, qpad, nq, dpad, ix->vmin, ix->vdiff, qplanes, qscale, qa, qn64, st));
-      tp.metric = ix->metric; tp.npb = npb;
+      CK(launch_qplanes(ix->type, qpad, nq, dpad, ix->vmin, ix->vdiff, ix->type == MV_IVF_SQ8 ? qplanes : nullptr,
+                        qscale, qa, qn64, st));
+      tp.metric = ix->metric; tp.npb = npb; tp.nq = nq;
       tp.list_off = ix->list_off; tp.norms = ix->norms; tp.ids = ix->ids; tp.rank = ix->rank;
       tp.bitset = bs; tp.nbits = bs ? nbits : 0;
       tp.qplanes = qplanes; tp.qnorm = qn64; tp.qscale = qscale; tp.qa = qa;
@@ -618,10 +657,10 @@ mv_status mv_index_describe(const mv_index* ix, char* buf, size_t len) {
   if (!ix || !buf || len == 0) return fail(MV_EINVAL, "null argument");
   snprintf(buf, len,
            "{\"d\": %d, \"dpad\": %d, \"nlist\": %d, \"ntotal\": %lld, \"maxlen\": %lld, \"type\": \"%s\", "
-           "\"metric\": \"%s\", \"tensor_map\": %s, \"tf32_exact\": %s, \"last_scan\": \"%s\"}",
+           "\"metric\": \"%s\", \"tensor_map\": %s, \"tf32_exact\": %s, \"last_scan\": \"%s\", \"last_coarse\": \"%s\"}",
            ix->d, ix->dpad, ix->nlist, (long long)ix->ntotal, (long long)ix->maxlen,
            ix->type == MV_IVF_FLAT ? "IVF_FLAT" : "IVF_SQ8", ix->metric == MV_L2 ? "L2" : "IP",
-           ix->xmap_ok ? "true" : "false", ix->tf32_exact ? "true" : "false", ix->last_scan);
+           ix->xmap_ok ? "true" : "false", ix->tf32_exact ? "true" : "false", ix->last_scan, ix->last_coarse);
   return MV_OK;
 }
 

@@ -166,6 +166,114 @@ __device__ __forceinline__ void warp_merge_smallest(uint64_t (&list)[R], const u
   warp_bitonic_merge<R>(list);
 }
 
+// k-th smallest (1-indexed) of the 128 u32 values v[0..3] x 32 lanes: MSB-first bisection, one
+// ballot per value per bit, no divergence.
+__device__ __forceinline__ uint32_t warp_kth_u32(const uint32_t (&v)[4], int k) {
+  uint32_t ans = 0;
+#pragma unroll 1
+  for (int b = 31; b >= 0; --b) {
+    const uint32_t trial = ans | (1u << b);
+    int cnt = 0;
+#pragma unroll
+    for (int m = 0; m < 4; ++m) cnt += __popc(__ballot_sync(MV_FULL, v[m] < trial));
+    if (cnt < k) ans = trial;
+  }
+  return ans;
+}
+
+// One warp folds a tile's 128 candidates -- distance keys k32[m] of element e = m*32 + lane
+// (0xffffffff = invalid), tie-break low word low(e) -- into the ascending list L[0..k) (u64 keys,
+// PAD-filled), keeping only keys below `li` (the global per-query threshold).  k <= 32: candidates
+// above min(L[k-1], li) are dropped with one compare; many survivors (warm-up) are first narrowed
+// to the k smallest by a warp radix select, then compacted, sorted and merged (bitonic); a few
+// survivors are inserted one by one.  k <= 128: sort-128 + merge; larger k: insertion.
+template <typename Low>
+__device__ __forceinline__ void warp_select_tile(uint64_t* L, int k, uint64_t li, const uint32_t (&k32)[4], Low low,
+                                                 uint64_t* wscr) {
+  const int lane = threadIdx.x & 31;
+  const uint64_t thr = L[k - 1] < li ? L[k - 1] : li;
+  const uint32_t thr32 = (uint32_t)(thr >> 32);
+  bool pass[4];
+  int npass = 0;
+#pragma unroll
+  for (int m = 0; m < 4; ++m) {
+    pass[m] = k32[m] != 0xffffffffu && k32[m] <= thr32;
+    npass += __popc(__ballot_sync(MV_FULL, pass[m]));
+  }
+  if (npass == 0) return;
+  if (k <= 32 && npass > 32) {
+    // warm-up: narrow to the k smallest distance keys of this tile (plus exact ties)
+    uint32_t v[4];
+#pragma unroll
+    for (int m = 0; m < 4; ++m) v[m] = pass[m] ? k32[m] : 0xffffffffu;
+    const uint32_t t32 = warp_kth_u32(v, k);
+    npass = 0;
+#pragma unroll
+    for (int m = 0; m < 4; ++m) {
+      pass[m] = pass[m] && k32[m] <= t32;
+      npass += __popc(__ballot_sync(MV_FULL, pass[m]));
+    }
+  }
+  if (k <= 32 && npass <= 32 && npass > 2) {
+    // compact the survivors into one register per lane, sort, merge into the list
+    int off = 0;
+#pragma unroll
+    for (int m = 0; m < 4; ++m) {
+      const uint32_t bm = __ballot_sync(MV_FULL, pass[m]);
+      if (pass[m]) wscr[off + __popc(bm & ((1u << lane) - 1))] = ((uint64_t)k32[m] << 32) | low(m * 32 + lane);
+      off += __popc(bm);
+    }
+    __syncwarp();
+    uint64_t c[1] = {lane < npass ? wscr[lane] : MV_KEY_PAD};
+    if (!(c[0] < thr)) c[0] = MV_KEY_PAD;
+    warp_bitonic_sort<1>(c);
+    uint64_t lv[1] = {lane < k ? L[lane] : MV_KEY_PAD};
+    warp_merge_smallest<1>(lv, c);
+    __syncwarp();
+    if (lane < k) L[lane] = lv[0];
+    __syncwarp();
+  } else if (npass <= 8 || k > 128) {
+#pragma unroll
+    for (int m = 0; m < 4; ++m) {
+      const uint64_t key = pass[m] ? (((uint64_t)k32[m] << 32) | low(m * 32 + lane)) : MV_KEY_PAD;
+      warp_list_insert(L, k, key, pass[m] && key < thr);
+    }
+  } else {
+    uint64_t key[4];
+#pragma unroll
+    for (int m = 0; m < 4; ++m) {
+      key[m] = pass[m] ? (((uint64_t)k32[m] << 32) | low(m * 32 + lane)) : MV_KEY_PAD;
+      if (!(key[m] < thr)) key[m] = MV_KEY_PAD;
+    }
+    warp_bitonic_sort<4>(key);
+    if (k <= 32) {
+      uint64_t lv[1] = {lane < k ? L[lane] : MV_KEY_PAD}, cv[1] = {key[0]};
+      warp_merge_smallest<1>(lv, cv);
+      __syncwarp();
+      if (lane < k) L[lane] = lv[0];
+    } else if (k <= 64) {
+      uint64_t lv[2], cv[2] = {key[0], key[1]};
+#pragma unroll
+      for (int r2 = 0; r2 < 2; ++r2) lv[r2] = r2 * 32 + lane < k ? L[r2 * 32 + lane] : MV_KEY_PAD;
+      warp_merge_smallest<2>(lv, cv);
+      __syncwarp();
+#pragma unroll
+      for (int r2 = 0; r2 < 2; ++r2)
+        if (r2 * 32 + lane < k) L[r2 * 32 + lane] = lv[r2];
+    } else {
+      uint64_t lv[4];
+#pragma unroll
+      for (int r2 = 0; r2 < 4; ++r2) lv[r2] = r2 * 32 + lane < k ? L[r2 * 32 + lane] : MV_KEY_PAD;
+      warp_merge_smallest<4>(lv, key);
+      __syncwarp();
+#pragma unroll
+      for (int r2 = 0; r2 < 4; ++r2)
+        if (r2 * 32 + lane < k) L[r2 * 32 + lane] = lv[r2];
+    }
+    __syncwarp();
+  }
+}
+
 // Block-wide bitonic sort of n (power of two) u64 keys in shared memory, ascending.
 __device__ __forceinline__ void block_bitonic_sort(uint64_t* a, int n) {
   for (int size = 2; size <= n; size <<= 1) {
@@ -275,6 +383,7 @@ cudaError_t launch_scan(const ScanArgs& a, cudaStream_t st);
 // k_scan_tc.cu (tcgen05 path)
 struct TcScanParams {
   int type, metric, dpad, k, npb, qchunk, nchunks, nstage, ncol, tmem_cols;
+  int64_t nq;              // FLAT query planes are plane-major [2][nq][dpad]
   int off_x, off_q, q_bytes, off_dt, off_lists, off_meta, meta_bytes, meta_lim_off, off_misc, off_side, off_bar,
       smem_total;
   const int64_t* list_off;
@@ -302,6 +411,18 @@ cudaError_t launch_scan_tc(const CUtensorMap* xmap, const TcScanParams& p, cudaS
 cudaError_t launch_qplanes(int type, const float* qpad, int64_t nq, int dpad, const float* vmin, const float* vdiff,
                            uint8_t* out, float* qscale, double* qa, double* qnorm, cudaStream_t st);
 cudaError_t launch_tf32_check(const float* x, int64_t n, int* flag, cudaStream_t st);
+
+// k_coarse_tc.cu (tcgen05 coarse + fused top-nprobe)
+struct CoarseParams {
+  int64_t nq;
+  int nlist, nchunks, nstage, nprobe, nqb, metric, smem_total;
+  const float* cnorm;
+  int32_t* probes;
+};
+bool coarse_tc_plan(int dpad, int nprobe, CoarseParams& p);
+cudaError_t launch_coarse_tc(const CUtensorMap* cmap, const CUtensorMap* qmap, const CoarseParams& p, int64_t nq,
+                             cudaStream_t st);
+cudaError_t launch_hilo(const float* x, int64_t n, int d, int dpad, float* out, cudaStream_t st);
 
 // k_select.cu
 cudaError_t launch_final_select(const int64_t* poff, const int32_t* pcnt, const uint64_t* part, int64_t nq, int npb,

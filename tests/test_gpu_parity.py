@@ -286,6 +286,7 @@ def test_tensor_core_path_matches_simt_path(kind, metric, k, monkeypatch):
     ix = _build(X, ids, C, metric, kind)
     D1, I1 = ix.search(Q.cuda(), k, 6)
     assert ix.describe()["last_scan"].startswith("tcgen05")
+    assert ix.describe()["last_coarse"].startswith("tcgen05")
     monkeypatch.setenv("MV_FORCE_SIMT", "1")
     D2, I2 = ix.search(Q.cuda(), k, 6)
     torch.cuda.synchronize()
