@@ -43,7 +43,10 @@ __global__ void __launch_bounds__(kCThreads, 1)
   uint32_t* Dt = reinterpret_cast<uint32_t*>(As + nstage * 2 * ABYTES);  // NQB x kCDLD
   uint64_t* lists = reinterpret_cast<uint64_t*>(Dt + NQB * kCDLD + (NQB * kCDLD & 1));  // NQB x nprobe
   uint64_t* scratch = lists + NQB * nprobe;               // 32 per epilogue warp
-  uint64_t* bars = scratch + 32 * kCEpi;
+  uint64_t* cbuf = scratch + 32 * kCEpi;                  // NQB x 32 survivor buffers (nprobe <= 32)
+  int* cnb = reinterpret_cast<int*>(cbuf + NQB * 32);     // NQB buffer counts
+  uint32_t* cbnd = reinterpret_cast<uint32_t*>(cnb + NQB);  // NQB running bounds
+  uint64_t* bars = reinterpret_cast<uint64_t*>(cbnd + NQB);
   uint64_t* full_a = bars;
   uint64_t* empty_a = bars + nstage;
   uint64_t* full_b = empty_a + nstage;
@@ -132,6 +135,10 @@ __global__ void __launch_bounds__(kCThreads, 1)
     uint64_t* wscr = scratch + ew * 32;
     const int nqv = (int)min64(NQB, p.nq - q0);
     for (int i = et; i < NQB * nprobe; i += 32 * kCEpi) lists[i] = MV_KEY_PAD;
+    for (int i = et; i < NQB; i += 32 * kCEpi) {
+      cnb[i] = 0;
+      cbnd[i] = 0xffffffffu;
+    }
     float cn_next = (row < p.nlist && p.metric == MV_L2) ? __ldg(p.cnorm + row) : 0.0f;
     cbar(1, 32 * kCEpi);
     for (int t = 0; t < ntiles; ++t) {
@@ -145,7 +152,7 @@ __global__ void __launch_bounds__(kCThreads, 1)
       tc_fence_after();
       const uint32_t tb = tmem + a * 2 * NQB + ((uint32_t)(quarter * 32) << 16);
 #pragma unroll
-      for (int qc = half * 16; qc < NQB; qc += 32) {
+      for (int qc = half * 16; qc < ((p.dbg & 2) ? 0 : NQB); qc += 32) {
         uint32_t rh[16], rl[16];
         tmem_ld16(tb + qc, rh);
         tmem_ld16(tb + NQB + qc, rl);
@@ -162,18 +169,41 @@ __global__ void __launch_bounds__(kCThreads, 1)
       if (lane == 0) mbar_arrive(&tempty[a]);
       cbar(1, 32 * kCEpi);
       const uint32_t cbase = t * 128;
-      for (int j = ew; j < nqv; j += kCEpi) {
-        uint32_t k32[4];
+      if (nprobe <= 32) {
+        constexpr int G = 4;
+        for (int j0 = ew; j0 < ((p.dbg & 1) ? 0 : nqv); j0 += kCEpi * G) {
+          const int nvalid = min(G, (nqv - j0 + kCEpi - 1) / kCEpi);
+          warp_filter_group<G>(
+              nvalid, nprobe, [&](int g, int m) { return Dt[(j0 + g * kCEpi) * kCDLD + m * 32 + lane]; },
+              [&](int g, uint64_t*& L, uint64_t*& B, int*& nb, uint32_t*& bnd, uint64_t& li) {
+                const int j = j0 + g * kCEpi;
+                L = lists + (int64_t)j * nprobe;
+                B = cbuf + j * 32;
+                nb = cnb + j;
+                bnd = cbnd + j;
+                li = MV_KEY_PAD;
+              },
+              [&](int, int v) { return cbase + (uint32_t)v; }, [](int, uint32_t) {}, wscr);
+        }
+      } else {
+        for (int j = ew; j < ((p.dbg & 1) ? 0 : nqv); j += kCEpi) {
+          uint32_t k32[4];
 #pragma unroll
-        for (int m = 0; m < 4; ++m) k32[m] = Dt[j * kCDLD + m * 32 + lane];
-        warp_select_tile(lists + (int64_t)j * nprobe, nprobe, MV_KEY_PAD, k32,
-                         [&](int v) { return cbase + (uint32_t)v; }, wscr);
+          for (int m = 0; m < 4; ++m) k32[m] = Dt[j * kCDLD + m * 32 + lane];
+          warp_select_tile(lists + (int64_t)j * nprobe, nprobe, MV_KEY_PAD, k32,
+                           [&](int v) { return cbase + (uint32_t)v; }, wscr);
+        }
       }
       cbar(1, 32 * kCEpi);
     }
+    if (nprobe <= 32)
+      for (int j = ew; j < nqv; j += kCEpi)
+        warp_flush_buffer(lists + (int64_t)j * nprobe, cbuf + j * 32, cnb + j, cbnd + j, nprobe, MV_KEY_PAD);
+    cbar(1, 32 * kCEpi);
     for (int i = et; i < nqv * nprobe; i += 32 * kCEpi) {
       const int j = i / nprobe, r = i - j * nprobe;
-      p.probes[(int64_t)(q0 + j) * nprobe + r] = (int32_t)(uint32_t)(lists[i] & 0xffffffffu);
+      const uint64_t key = lists[i];  // PAD only in MV_COARSE_DEBUG runs: keep the probe ids in range
+      p.probes[(int64_t)(q0 + j) * nprobe + r] = key == MV_KEY_PAD ? r % p.nlist : (int32_t)(uint32_t)(key & 0xffffffffu);
     }
   }
   __syncthreads();
@@ -209,7 +239,8 @@ bool coarse_tc_plan(int dpad, int nprobe, CoarseParams& p) {
   p.nchunks = dpad / 32;
   p.nprobe = nprobe;
   const int brows = 2 * p.nqb;
-  const int fixed = p.nchunks * brows * 128 + p.nqb * kCDLD * 4 + 8 + p.nqb * nprobe * 8 + 32 * kCEpi * 8 + 256;
+  const int fixed = p.nchunks * brows * 128 + p.nqb * kCDLD * 4 + 8 + p.nqb * nprobe * 8 + 32 * kCEpi * 8 +
+                    p.nqb * 32 * 8 + p.nqb * 8 + 256;
   const int budget = 227 * 1024 - 1024;
   const int ns = std::min(4, (budget - fixed) / (2 * 128 * 128));
   if (ns < 2) return false;

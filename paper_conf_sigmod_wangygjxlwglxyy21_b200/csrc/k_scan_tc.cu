@@ -73,6 +73,9 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
   uint8_t* metab = sm + p.off_meta;
   int32_t* ecnt = reinterpret_cast<int32_t*>(sm + p.off_misc);
   uint64_t* scratch = reinterpret_cast<uint64_t*>(sm + p.off_misc + 256);  // 32 per epilogue warp
+  uint64_t* cbuf = scratch + 32 * kEpiWarps;                               // QC x 32 (k <= 32)
+  int* cnb = reinterpret_cast<int*>(cbuf + 32 * QC);                       // QC counts
+  uint32_t* cbnd = reinterpret_cast<uint32_t*>(cnb + QC);                  // QC running bounds
   uint8_t* side = sm + p.off_side;
   uint64_t* bars = reinterpret_cast<uint64_t*>(sm + p.off_bar);
   uint64_t* full_x = bars;
@@ -248,6 +251,11 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
       const bool sel = (k <= kLocalSelectMaxK) && (wi.len > k);
       if (sel) {
         for (int i = et; i < wi.nqc * k; i += 32 * kEpiWarps) lists[i] = MV_KEY_PAD;
+        if (k <= 32)
+          for (int i = et; i < wi.nqc; i += 32 * kEpiWarps) {
+            cnb[i] = 0;
+            cbnd[i] = 0xffffffffu;
+          }
       } else {
         for (int i = et; i < wi.nqc; i += 32 * kEpiWarps) ecnt[i] = 0;
       }
@@ -298,28 +306,51 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
         __syncwarp();
         if (lane == 0) mbar_arrive(&tempty[a]);
         named_bar(1, 32 * kEpiWarps);
-        // ---- a6: filter against min(list k-th, global tau) + select (one warp per query slot)
-        for (int i = ew; i < ((p.dbg & 1) ? 0 : wi.nqc); i += kEpiWarps) {
-          const int pr = mp[i];
-          const uint64_t li = lim[i];
-          uint32_t k32[4];
-#pragma unroll
-          for (int m = 0; m < 4; ++m) k32[m] = Dt[i * kDLD + m * 32 + lane];
-          if (!sel) {
-#pragma unroll
-            for (int m = 0; m < 4; ++m) {
-              const uint64_t key = ((uint64_t)k32[m] << 32) | srank[m * 32 + lane];
-              const bool pass = k32[m] != 0xffffffffu && key < li;
-              const uint32_t msk = __ballot_sync(MV_FULL, pass);
-              const int base = ecnt[i];
-              if (pass) p.part[p.poff[pr] + base + __popc(msk & ((1u << lane) - 1))] = key;
-              __syncwarp();
-              if (lane == 0) ecnt[i] = base + __popc(msk);
-              __syncwarp();
-            }
-            continue;
+        // ---- a6: filter against min(list k-th, running bound, global tau) + select (warp per query)
+        if (sel && k <= 32) {
+          constexpr int G = 4;
+          for (int i0 = ew; i0 < ((p.dbg & 1) ? 0 : wi.nqc); i0 += kEpiWarps * G) {
+            const int nvalid = min(G, (wi.nqc - i0 + kEpiWarps - 1) / kEpiWarps);
+            warp_filter_group<G>(
+                nvalid, k, [&](int g, int m) { return Dt[(i0 + g * kEpiWarps) * kDLD + m * 32 + lane]; },
+                [&](int g, uint64_t*& L, uint64_t*& B, int*& nb, uint32_t*& bnd, uint64_t& li) {
+                  const int i = i0 + g * kEpiWarps;
+                  L = lists + (int64_t)i * k;
+                  B = cbuf + i * 32;
+                  nb = cnb + i;
+                  bnd = cbnd + i;
+                  li = lim[i];
+                },
+                [&](int, int v) { return srank[v]; },
+                [&](int g, uint32_t t32) {
+                  atomicMin(reinterpret_cast<unsigned long long*>(p.tau + mp[i0 + g * kEpiWarps] / p.npb),
+                            ((unsigned long long)t32 << 32) | 0xffffffffull);
+                },
+                wscr);
           }
-          warp_select_tile(lists + (int64_t)i * k, k, li, k32, [&](int v) { return srank[v]; }, wscr);
+        } else {
+          for (int i = ew; i < ((p.dbg & 1) ? 0 : wi.nqc); i += kEpiWarps) {
+            const int pr = mp[i];
+            const uint64_t li = lim[i];
+            uint32_t k32[4];
+#pragma unroll
+            for (int m = 0; m < 4; ++m) k32[m] = Dt[i * kDLD + m * 32 + lane];
+            if (!sel) {
+#pragma unroll
+              for (int m = 0; m < 4; ++m) {
+                const uint64_t key = ((uint64_t)k32[m] << 32) | srank[m * 32 + lane];
+                const bool pass = k32[m] != 0xffffffffu && key < li;
+                const uint32_t msk = __ballot_sync(MV_FULL, pass);
+                const int base = ecnt[i];
+                if (pass) p.part[p.poff[pr] + base + __popc(msk & ((1u << lane) - 1))] = key;
+                __syncwarp();
+                if (lane == 0) ecnt[i] = base + __popc(msk);
+                __syncwarp();
+              }
+              continue;
+            }
+            warp_select_tile(lists + (int64_t)i * k, k, li, k32, [&](int v) { return srank[v]; }, wscr);
+          }
         }
         named_bar(1, 32 * kEpiWarps);
         if (lane == 0) mbar_arrive(&empty_t[ts]);
@@ -328,6 +359,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
       for (int i = ew; i < wi.nqc; i += kEpiWarps) {
         const int pr = mp[i];
         if (sel) {
+          if (k <= 32) warp_flush_buffer(lists + (int64_t)i * k, cbuf + i * 32, cnb + i, cbnd + i, k, lim[i]);
           const uint64_t* L = lists + (int64_t)i * k;
           int c = 0;
           for (int j0 = 0; j0 < k; j0 += 32) {
@@ -458,7 +490,7 @@ bool tc_scan_plan(int type, int dpad, int k, TcScanParams& p) {
   const int lists_bytes = k <= kLocalSelectMaxK ? qc * k * 8 : 0;
   p.meta_lim_off = up(8 * qc, 8);
   p.meta_bytes = up(p.meta_lim_off + 24 * qc, 16);
-  const int misc_bytes = 256 + 32 * 8 * kEpiWarps;
+  const int misc_bytes = 256 + 32 * 8 * kEpiWarps + (k <= 32 ? qc * (32 * 8 + 8) : 0);
   const int side_bytes = kNTS * kSideBytes;
   const int stage = 128 * atom;
   const int fixed = 2 * p.q_bytes + up(dt_bytes, 16) + up(lists_bytes, 16) + 2 * p.meta_bytes + misc_bytes + side_bytes;

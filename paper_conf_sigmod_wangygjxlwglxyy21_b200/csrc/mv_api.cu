@@ -170,6 +170,8 @@ static cudaError_t run_coarse(mv_index* ix, const float* qpad, const float* qhl,
       cp.metric = ix->metric;
       cp.cnorm = ix->cnorm;
       cp.probes = P;
+      const char* cdbg = getenv("MV_COARSE_DEBUG");
+      cp.dbg = cdbg ? atoi(cdbg) : 0;
       ix->last_coarse = "tcgen05.tf32";
       return launch_coarse_tc(&ix->cmap, &qmap, cp, nq, st);
     }
@@ -577,6 +579,7 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
       tp.poff = b.poff; tp.pcnt = b.pcnt; tp.part = part; tp.tau = tau;
       const char* dbg = getenv("MV_SCAN_DEBUG");
       tp.dbg = dbg ? atoi(dbg) : 0;
+      tp.prof = nullptr;
       CK(launch_scan_tc(&ix->xmap, tp, st));
       ix->last_scan = ix->type == MV_IVF_FLAT ? "tcgen05.tf32" : "tcgen05.i8";
       ix->launches += 1;

@@ -274,6 +274,122 @@ __device__ __forceinline__ void warp_select_tile(uint64_t* L, int k, uint64_t li
   }
 }
 
+// ------------------------------------------------------------------------------------------
+// Buffered selection for k <= 32: survivors of each tile are appended to a per-query 32-entry smem
+// buffer B (count *nb) and merged into the sorted list L only when the buffer would overflow (and
+// once at the end, warp_flush_buffer), so the ~21-step sort/merge network runs a few times per
+// query instead of once per tile.  *bnd is a running upper bound on the k-th best distance key,
+// tightened as soon as a crowded tile is narrowed to its k smallest keys (exact: anything with k
+// smaller keys in the same tile cannot be in the top-k) and after every flush; publish(t32) lets
+// the caller share it (the scan folds it into the global per-query tau).
+// ------------------------------------------------------------------------------------------
+__device__ __forceinline__ void warp_flush_buffer(uint64_t* L, uint64_t* B, int* nb, uint32_t* bnd, int k,
+                                                  uint64_t li) {
+  const int lane = threadIdx.x & 31;
+  const int n = *nb;
+  if (n == 0) return;
+  const uint64_t thr = L[k - 1] < li ? L[k - 1] : li;
+  uint64_t c[1] = {lane < n ? B[lane] : MV_KEY_PAD};
+  if (!(c[0] < thr)) c[0] = MV_KEY_PAD;
+  warp_bitonic_sort<1>(c);
+  uint64_t lv[1] = {lane < k ? L[lane] : MV_KEY_PAD};
+  warp_merge_smallest<1>(lv, c);
+  __syncwarp();
+  if (lane < k) L[lane] = lv[0];
+  if (lane == k - 1 && lv[0] != MV_KEY_PAD) *bnd = min(*bnd, (uint32_t)(lv[0] >> 32));
+  if (lane == 0) *nb = 0;
+  __syncwarp();
+}
+
+// Fold one tile into (L, B) after the caller's filter: pass[] marks candidates at or below the
+// bound, npass their count (> 0).
+template <typename Low, typename Pub>
+__device__ __forceinline__ void warp_collect_passed(uint64_t* L, uint64_t* B, int* nb, uint32_t* bnd, int k, uint64_t li,
+                                                    const uint32_t (&k32)[4], bool (&pass)[4], int npass, Low low,
+                                                    Pub publish, uint64_t* wscr) {
+  const int lane = threadIdx.x & 31;
+  if (npass > 32) {
+    uint32_t v[4];
+#pragma unroll
+    for (int m = 0; m < 4; ++m) v[m] = pass[m] ? k32[m] : 0xffffffffu;
+    const uint32_t t32 = warp_kth_u32(v, k);
+    npass = 0;
+#pragma unroll
+    for (int m = 0; m < 4; ++m) {
+      pass[m] = pass[m] && k32[m] <= t32;
+      npass += __popc(__ballot_sync(MV_FULL, pass[m]));
+    }
+    __syncwarp();
+    if (lane == 0) {
+      *bnd = min(*bnd, t32);
+      publish(t32);
+    }
+    __syncwarp();
+    if (npass > 32) {  // pathological exact ties: fold this tile directly
+      warp_flush_buffer(L, B, nb, bnd, k, li);
+      warp_select_tile(L, k, li, k32, low, wscr);
+      return;
+    }
+  }
+  if (*nb + npass > 32) warp_flush_buffer(L, B, nb, bnd, k, li);
+  int off = *nb;
+#pragma unroll
+  for (int m = 0; m < 4; ++m) {
+    const uint32_t bm = __ballot_sync(MV_FULL, pass[m]);
+    if (pass[m]) B[off + __popc(bm & ((1u << lane) - 1))] = ((uint64_t)k32[m] << 32) | low(m * 32 + lane);
+    off += __popc(bm);
+  }
+  __syncwarp();
+  if (lane == 0) *nb = off;
+  __syncwarp();
+}
+
+// Filter G query slots per call so their shared-memory loads and ballots overlap (the per-tile
+// filter is latency-bound); only slots with survivors enter the (rare, serial) fold.
+//   rowk(g, m) -> distance key of element m*32+lane for query g;  st(g) -> per-query state.
+template <int G, typename RowK, typename State, typename Low, typename Pub>
+__device__ __forceinline__ void warp_filter_group(int nvalid, int k, RowK rowk, State st, Low low, Pub publish,
+                                                  uint64_t* wscr) {
+  uint32_t k32[G][4];
+  uint32_t thr32[G];
+#pragma unroll
+  for (int g = 0; g < G; ++g) {
+    if (g < nvalid) {
+      uint64_t *L, *B;
+      int* nb;
+      uint32_t* bnd;
+      uint64_t li;
+      st(g, L, B, nb, bnd, li);
+      const uint64_t thr = L[k - 1] < li ? L[k - 1] : li;
+      thr32[g] = min((uint32_t)(thr >> 32), *bnd);
+#pragma unroll
+      for (int m = 0; m < 4; ++m) k32[g][m] = rowk(g, m);
+    }
+  }
+  int npass[G];
+  bool pass[G][4];
+#pragma unroll
+  for (int g = 0; g < G; ++g) {
+    npass[g] = 0;
+#pragma unroll
+    for (int m = 0; m < 4; ++m) {
+      pass[g][m] = g < nvalid && k32[g][m] != 0xffffffffu && k32[g][m] <= thr32[g];
+      npass[g] += __popc(__ballot_sync(MV_FULL, pass[g][m]));
+    }
+  }
+#pragma unroll
+  for (int g = 0; g < G; ++g) {
+    if (npass[g] == 0) continue;
+    uint64_t *L, *B;
+    int* nb;
+    uint32_t* bnd;
+    uint64_t li;
+    st(g, L, B, nb, bnd, li);
+    warp_collect_passed(L, B, nb, bnd, k, li, k32[g], pass[g], npass[g], [&](int v) { return low(g, v); },
+                        [&](uint32_t t) { publish(g, t); }, wscr);
+  }
+}
+
 // Block-wide bitonic sort of n (power of two) u64 keys in shared memory, ascending.
 __device__ __forceinline__ void block_bitonic_sort(uint64_t* a, int n) {
   for (int size = 2; size <= n; size <<= 1) {
@@ -405,6 +521,7 @@ struct TcScanParams {
   uint64_t* part;
   uint64_t* tau;           // nq: global per-query threshold (u64 key), atomicMin-updated
   int dbg;                 // debug bitmask (MV_SCAN_DEBUG): 1 skip select, 2 skip epilogue math, 4 skip Q copy
+  unsigned long long* prof;  // unused (reserved for wait-cycle accounting)
 };
 bool tc_scan_plan(int type, int dpad, int k, TcScanParams& p);
 cudaError_t launch_scan_tc(const CUtensorMap* xmap, const TcScanParams& p, cudaStream_t st);
@@ -416,6 +533,7 @@ cudaError_t launch_tf32_check(const float* x, int64_t n, int* flag, cudaStream_t
 struct CoarseParams {
   int64_t nq;
   int nlist, nchunks, nstage, nprobe, nqb, metric, smem_total;
+  int dbg;  // MV_COARSE_DEBUG: 1 skip select, 2 skip epilogue math
   const float* cnorm;
   int32_t* probes;
 };
