@@ -64,9 +64,52 @@ __global__ void k_work_fill(const int32_t* __restrict__ wcount, const int32_t* _
   for (int c = 0; c < n; ++c) witems[o + c] = make_int2(l, b + c * qchunk);
 }
 
+// Longest-first order for the persistent scan's static round-robin: a single-CTA counting sort of
+// the work items by descending cost key = 64 * tiles + queries (tiles = ceil(|list| / 128)).
+__global__ void __launch_bounds__(1024) k_sort_work(const int2* __restrict__ in, const int32_t* __restrict__ nwork_p,
+                                                    const int32_t* __restrict__ boff, const int64_t* __restrict__ list_off,
+                                                    int qchunk, int2* __restrict__ out) {
+  constexpr int NB = 4096;
+  __shared__ int hist[NB];
+  __shared__ int part[1024];
+  const int nwork = *nwork_p, tid = threadIdx.x;
+  for (int i = tid; i < NB; i += 1024) hist[i] = 0;
+  __syncthreads();
+  auto key = [&](int w) {
+    const int2 it = in[w];
+    const int nq = min(qchunk, boff[it.x + 1] - it.y);
+    const int64_t len = list_off[it.x + 1] - list_off[it.x];
+    const int tiles = (int)min64((len + 127) / 128, 63);
+    return NB - 1 - min(NB - 1, tiles * 64 + min(nq, 63));  // descending cost -> ascending bin
+  };
+  for (int w = tid; w < nwork; w += 1024) atomicAdd(&hist[key(w)], 1);
+  __syncthreads();
+  // exclusive scan of 4096 bins: 4 per thread
+  int loc[4], acc = 0;
+#pragma unroll
+  for (int j = 0; j < 4; ++j) {
+    loc[j] = acc;
+    acc += hist[tid * 4 + j];
+  }
+  part[tid] = acc;
+  __syncthreads();
+  for (int off = 1; off < 1024; off <<= 1) {
+    const int v = tid >= off ? part[tid - off] : 0;
+    __syncthreads();
+    part[tid] += v;
+    __syncthreads();
+  }
+  const int base = tid ? part[tid - 1] : 0;
+  __syncthreads();
+#pragma unroll
+  for (int j = 0; j < 4; ++j) hist[tid * 4 + j] = base + loc[j];
+  __syncthreads();
+  for (int w = tid; w < nwork; w += 1024) out[atomicAdd(&hist[key(w)], 1)] = in[w];
+}
+
 cudaError_t launch_bucket(const int32_t* probes, int64_t nq, int npb, int nlist, const int64_t* list_off, int k,
                           int qchunk, const Bucketing& b, cudaStream_t st) {
-  (void)list_off; (void)k;
+  (void)k;
   const int64_t npairs = nq * npb;
   cudaMemsetAsync(b.lcount, 0, sizeof(int32_t) * nlist, st);
   cudaMemsetAsync(b.bfill, 0, sizeof(int32_t) * nlist, st);
@@ -78,19 +121,20 @@ cudaError_t launch_bucket(const int32_t* probes, int64_t nq, int npb, int nlist,
   if (npairs) k_bucket_fill<<<grid, 256, 0, st>>>(probes, npairs, b.boff, b.bfill, b.bq);
   k_work_count<<<(nlist + 255) / 256, 256, 0, st>>>(b.lcount, nlist, qchunk, b.wcount);
   if ((e = launch_scan_i32(b.wcount, nlist, b.woff, st)) != cudaSuccess) return e;
-  k_work_fill<<<(nlist + 255) / 256, 256, 0, st>>>(b.wcount, b.woff, b.boff, nlist, qchunk, b.witems);
+  k_work_fill<<<(nlist + 255) / 256, 256, 0, st>>>(b.wcount, b.woff, b.boff, nlist, qchunk, b.witems_unsorted);
+  k_sort_work<<<1, 1024, 0, st>>>(b.witems_unsorted, b.woff + nlist, b.boff, list_off, qchunk, b.witems);
   return cudaGetLastError();
 }
 
 // Region capacity of pair (q, j): min(k, |list|) when the scan selects locally (k <= 1024),
 // else |list| (every candidate that survives the bitset is emitted).
-__device__ __forceinline__ int64_t pair_cap(int64_t len, int k) {
-  return k <= kLocalSelectMaxK ? min64(k, len) : len;
+__device__ __forceinline__ int64_t pair_cap(int64_t len, int k, int capk) {
+  return k <= kLocalSelectMaxK ? min64(capk, len) : len;
 }
 
 // one warp per query: qtot[q] = sum_j cap(q, j)
 __global__ void k_query_tot(const int32_t* __restrict__ probes, int64_t nq, int npb,
-                            const int64_t* __restrict__ list_off, int k, int64_t* qtot) {
+                            const int64_t* __restrict__ list_off, int k, int capk, int64_t* qtot) {
   const int lane = threadIdx.x & 31;
   const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
@@ -98,7 +142,7 @@ __global__ void k_query_tot(const int32_t* __restrict__ probes, int64_t nq, int 
     int64_t acc = 0;
     for (int j = lane; j < npb; j += 32) {
       const int l = probes[q * npb + j];
-      acc += pair_cap(list_off[l + 1] - list_off[l], k);
+      acc += pair_cap(list_off[l + 1] - list_off[l], k, capk);
     }
     for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(MV_FULL, acc, o);
     if (lane == 0) qtot[q] = acc;
@@ -107,7 +151,7 @@ __global__ void k_query_tot(const int32_t* __restrict__ probes, int64_t nq, int 
 
 // one warp per query: poff[q*npb + j] = qbase[q] + sum_{j' < j} cap(q, j')
 __global__ void k_pair_off(const int32_t* __restrict__ probes, int64_t nq, int npb, const int64_t* __restrict__ list_off,
-                           int k, const int64_t* __restrict__ qbase, int64_t* poff) {
+                           int k, int capk, const int64_t* __restrict__ qbase, int64_t* poff) {
   const int lane = threadIdx.x & 31;
   const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
@@ -118,7 +162,7 @@ __global__ void k_pair_off(const int32_t* __restrict__ probes, int64_t nq, int n
       int64_t c = 0;
       if (j < npb) {
         const int l = probes[q * npb + j];
-        c = pair_cap(list_off[l + 1] - list_off[l], k);
+        c = pair_cap(list_off[l + 1] - list_off[l], k, capk);
       }
       int64_t incl = c;
       for (int o = 1; o < 32; o <<= 1) {
@@ -131,15 +175,15 @@ __global__ void k_pair_off(const int32_t* __restrict__ probes, int64_t nq, int n
   }
 }
 
-cudaError_t launch_pair_offsets(const int32_t* probes, int64_t nq, int npb, const int64_t* list_off, int k,
+cudaError_t launch_pair_offsets(const int32_t* probes, int64_t nq, int npb, const int64_t* list_off, int k, int capk,
                                 const Bucketing& b, cudaStream_t st) {
   if (nq == 0) return cudaSuccess;
   const int grid = (int)min64(kNumSMs * 8, (nq * 32 + 255) / 256);
   int64_t* qbase = b.qtot + (nq + 1);  // second half of the qtot allocation
-  k_query_tot<<<grid, 256, 0, st>>>(probes, nq, npb, list_off, k, b.qtot);
+  k_query_tot<<<grid, 256, 0, st>>>(probes, nq, npb, list_off, k, capk, b.qtot);
   cudaError_t e = launch_scan_i64(b.qtot, nq, qbase, st);
   if (e != cudaSuccess) return e;
-  k_pair_off<<<grid, 256, 0, st>>>(probes, nq, npb, list_off, k, qbase, b.poff);
+  k_pair_off<<<grid, 256, 0, st>>>(probes, nq, npb, list_off, k, capk, qbase, b.poff);
   return cudaGetLastError();
 }
 

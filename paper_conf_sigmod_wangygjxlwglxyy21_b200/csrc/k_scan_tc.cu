@@ -28,6 +28,12 @@ using namespace sm100;
 
 __device__ __forceinline__ void named_bar(int id, int n) { asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory"); }
 
+// CTA-0 event timeline for MV_SCAN_TRACE (row r holds up to 1024 clock64 stamps)
+#define MV_TRACE(row, idx)                                                                      \
+  do {                                                                                        \
+    if (p.prof && blockIdx.x == 0 && (idx) < 1024) p.prof[(row) * 1024 + (idx)] = clock64();  \
+  } while (0)
+
 struct WorkInfo {
   int l, bstart, nqc, len, ntiles;
   int64_t lstart;
@@ -125,6 +131,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
   tc_fence_after();
   const uint32_t tmem = *tslot;
   const int nwork = *p.nwitems;
+  unsigned long long gt0 = 0;
+  if (p.prof) asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(gt0));
 
   if (warp == 0) {
     // ------------------------------------------------------------------ TMA producer
@@ -145,6 +153,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
           for (int c = 0; c < nchunks; ++c, ++it) {
             const uint32_t s = it % nstage, r = it / nstage;
             mbar_wait(&empty_x[s], (r & 1) ^ 1);
+            MV_TRACE(0, it);
             mbar_expect_tx(&full_x[s], 128 * ATOM);
             tma_load_2d(Xs + s * 128 * ATOM, &xmap, &full_x[s], c * ATOM / ESZ, row0);
           }
@@ -162,11 +171,13 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
         const uint32_t idesc = TYPE == MV_IVF_FLAT ? idesc_tf32(N) : idesc_u8s8(N);
         const uint32_t b = wcount & 1;
         mbar_wait(&full_q[b], (wcount >> 1) & 1);
+        MV_TRACE(1, wcount);
         tc_fence_after();
         const uint32_t qbase = smem_u32(Qs + b * p.q_bytes);
         for (int t = 0; t < wi.ntiles; ++t, ++titer) {
           const uint32_t a = titer & 1;
           mbar_wait(&tempty[a], ((titer >> 1) & 1) ^ 1);
+          MV_TRACE(2, titer);
           tc_fence_after();
           const uint32_t dcol = tmem + a * p.ncol;
           for (int c = 0; c < nchunks; ++c, ++it) {
@@ -185,6 +196,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
             mma_commit(&empty_x[s]);
           }
           mma_commit(&tfull[a]);
+          MV_TRACE(3, titer);
         }
         mma_commit(&empty_q[b]);
       }
@@ -265,6 +277,10 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
         const uint32_t ts = titer % kNTS;
         const int vrow = t * 128 + row;
         const int row0 = (int)(wi.lstart + t * 128);
+        // refresh the global per-query threshold tau once per tile (other work items of the same
+        // query keep tightening it); the load latency overlaps the wait for the accumulator
+        uint64_t tau_now = MV_KEY_PAD;
+        if (et < wi.nqc) tau_now = *reinterpret_cast<volatile const uint64_t*>(p.tau + mp[et] / p.npb);
         mbar_wait(&full_t[ts], (titer / kNTS) & 1);
         const uint8_t* sd = side + ts * kSideBytes;
         const uint32_t* srank = reinterpret_cast<const uint32_t*>(sd + kSideRank) + (row0 & 3);
@@ -273,6 +289,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
           valid = !bit_excluded(p.bitset, p.nbits, reinterpret_cast<const int64_t*>(sd + kSideIds)[(row0 & 1) + row]);
         const double xn = use_norms ? reinterpret_cast<const double*>(sd)[(row0 & 1) + row] : 0.0;
         mbar_wait(&tfull[a], (titer >> 1) & 1);
+        if (et == 0) MV_TRACE(6, titer);
         tc_fence_after();
         const uint32_t tbase = tmem + a * p.ncol + ((uint32_t)(quarter * 32) << 16);
         for (int qc = half * 16; qc < ((p.dbg & 2) ? 0 : NQ); qc += 32) {
@@ -302,10 +319,13 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
             }
           }
         }
+        if (et < wi.nqc && tau_now < lim[et]) const_cast<uint64_t*>(lim)[et] = tau_now;
         tc_fence_before();
+        if (et == 0) MV_TRACE(4, titer);
         __syncwarp();
         if (lane == 0) mbar_arrive(&tempty[a]);
         named_bar(1, 32 * kEpiWarps);
+        if (et == 0) MV_TRACE(5, titer);
         // ---- a6: filter against min(list k-th, running bound, global tau) + select (warp per query)
         if (sel && k <= 32) {
           constexpr int G = 4;
@@ -326,7 +346,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
                   atomicMin(reinterpret_cast<unsigned long long*>(p.tau + mp[i0 + g * kEpiWarps] / p.npb),
                             ((unsigned long long)t32 << 32) | 0xffffffffull);
                 },
-                wscr);
+                wscr, (p.prof && (p.dbg & 64)) ? p.prof + 8 * 1024 + 1000 : nullptr, !(p.dbg & 32));
           }
         } else {
           for (int i = ew; i < ((p.dbg & 1) ? 0 : wi.nqc); i += kEpiWarps) {
@@ -353,13 +373,27 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
           }
         }
         named_bar(1, 32 * kEpiWarps);
+        if (et == 0) MV_TRACE(7, titer);
         if (lane == 0) mbar_arrive(&empty_t[ts]);
       }
       // ---- finalize this work item's (query, list) partial results
       for (int i = ew; i < wi.nqc; i += kEpiWarps) {
         const int pr = mp[i];
-        if (sel) {
-          if (k <= 32) warp_flush_buffer(lists + (int64_t)i * k, cbuf + i * 32, cnb + i, cbnd + i, k, lim[i]);
+        if (sel && k <= 32) {
+          // the sorted list (<= k) followed by the unsorted survivor buffer (<= 32): the final select
+          // merges them exactly, so no end-of-pair sort is needed
+          const uint64_t* L = lists + (int64_t)i * k;
+          const uint64_t v = lane < k ? L[lane] : MV_KEY_PAD;
+          const uint32_t lm = __ballot_sync(MV_FULL, v != MV_KEY_PAD);
+          const int nl = __popc(lm), n = cnb[i];
+          if (v != MV_KEY_PAD) p.part[p.poff[pr] + __popc(lm & ((1u << lane) - 1))] = v;
+          if (lane < n) p.part[p.poff[pr] + nl + lane] = cbuf[i * 32 + lane];
+          if (lane == 0) {
+            p.pcnt[pr] = nl + n;
+            if (L[k - 1] != MV_KEY_PAD)
+              atomicMin(reinterpret_cast<unsigned long long*>(p.tau + pr / p.npb), (unsigned long long)L[k - 1]);
+          }
+        } else if (sel) {
           const uint64_t* L = lists + (int64_t)i * k;
           int c = 0;
           for (int j0 = 0; j0 < k; j0 += 32) {
@@ -383,6 +417,15 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
     }
   }
   __syncthreads();
+  if (p.prof && threadIdx.x == 0) {  // per-CTA start / end (ns) in rows 8.. of the debug buffer
+    unsigned long long gt1;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(gt1));
+    int ntl = 0;
+    for (int w = blockIdx.x; w < nwork; w += gridDim.x) ntl += work_info(p, w).ntiles;
+    p.prof[8 * 1024 + blockIdx.x * 3 + 0] = gt0;
+    p.prof[8 * 1024 + blockIdx.x * 3 + 1] = gt1;
+    p.prof[8 * 1024 + blockIdx.x * 3 + 2] = ntl;
+  }
   if (warp == 1) {
     tc_fence_after();
     tmem_dealloc(tmem, p.tmem_cols);

@@ -534,16 +534,18 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
     CK(s.alloc(&b.wcount, nlist));
     CK(s.alloc(&b.woff, nlist + 1));
     CK(s.alloc(&b.witems, (size_t)(nlist + npairs / qchunk + 1)));
+    CK(s.alloc(&b.witems_unsorted, (size_t)(nlist + npairs / qchunk + 1)));
     CK(s.alloc(&b.qtot, (size_t)(2 * (nq + 1))));
     CK(s.alloc(&b.poff, (size_t)npairs));
     CK(s.alloc(&b.pcnt, (size_t)npairs));
     CK(s.alloc(&b.counter, 1));
     CK(launch_bucket(P, nq, npb, nlist, ix->list_off, k, qchunk, b, st));
-    CK(launch_pair_offsets(P, nq, npb, ix->list_off, k, b, st));
+    const int capk = (use_tc && k <= 32) ? k + 32 : k;  // tensor-core scan: sorted list + 32-entry buffer per pair
+    CK(launch_pair_offsets(P, nq, npb, ix->list_off, k, capk, b, st));
     prof_mark(ix, st);
     int64_t cap;
     if (k <= kLocalSelectMaxK) {
-      cap = nq * npb * min64(k, max64(ix->maxlen, 1));
+      cap = nq * npb * min64(capk, max64(ix->maxlen, 1));
     } else {
       CK(cudaMemcpyAsync(&cap, b.qtot + (nq + 1) + nq, sizeof(int64_t), cudaMemcpyDeviceToHost, st));
       CK(cudaStreamSynchronize(st));
@@ -580,7 +582,35 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
       const char* dbg = getenv("MV_SCAN_DEBUG");
       tp.dbg = dbg ? atoi(dbg) : 0;
       tp.prof = nullptr;
+      const char* trc = getenv("MV_SCAN_TRACE");
+      if (trc && trc[0] == '1') {
+        CK(s.alloc(&tp.prof, (size_t)9 * 1024));
+        CK(cudaMemsetAsync(tp.prof, 0, 9 * 1024 * 8, st));
+      }
       CK(launch_scan_tc(&ix->xmap, tp, st));
+      if (tp.prof) {  // debug timeline of CTA 0 (MV_SCAN_TRACE=1): rows = events, cycles since the first TMA issue
+        std::vector<unsigned long long> h(9 * 1024);
+        CK(cudaMemcpyAsync(h.data(), tp.prof, h.size() * 8, cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+        const char* nm[8] = {"tma_issue[chunk]", "mma_q_ready[wi]", "mma_tile_start[t]", "mma_tile_done[t]",
+                             "epi_math_done[t]", "epi_sel_start[t]", "epi_tfull[t]", "epi_tile_end[t]"};
+        const unsigned long long t0 = h[0];
+        for (int r = 0; r < 8; ++r) {
+          fprintf(stderr, "[trace] %-18s", nm[r]);
+          for (int i = 0; i < 48; ++i)
+            if (h[r * 1024 + i]) fprintf(stderr, " %lld", (long long)(h[r * 1024 + i] - t0));
+          fprintf(stderr, "\n");
+        }
+        unsigned long long gmin = ~0ull;
+        for (int b = 0; b < 148; ++b) gmin = std::min(gmin, h[8 * 1024 + b * 3]);
+        fprintf(stderr, "[events] tiles_with_survivors %llu warmups %llu flushes %llu fallbacks %llu survivors %llu\n",
+                h[8 * 1024 + 1000], h[8 * 1024 + 1001], h[8 * 1024 + 1002], h[8 * 1024 + 1003], h[8 * 1024 + 1004]);
+        fprintf(stderr, "[cta] start_us end_us tiles:");
+        for (int b = 0; b < 148; ++b)
+          fprintf(stderr, " %d:%.1f/%.1f/%llu", b, (h[8 * 1024 + b * 3] - gmin) / 1e3, (h[8 * 1024 + b * 3 + 1] - gmin) / 1e3,
+                  h[8 * 1024 + b * 3 + 2]);
+        fprintf(stderr, "\n");
+      }
       ix->last_scan = ix->type == MV_IVF_FLAT ? "tcgen05.tf32" : "tcgen05.i8";
       ix->launches += 1;
     } else {
@@ -600,7 +630,7 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
     CK(launch_final_select(b.poff, b.pcnt, part, nq, npb, k, ix->metric, ix->sorted_ids, D, I, st));
     prof_mark(ix, st);
     if (ix->prof) ix->prof_searches++;
-    ix->launches += 13;  // prep, coarse, 6 bucketing, 3 offsets, scan, select
+    ix->launches += 14;  // prep, coarse, 7 bucketing, 3 offsets, scan, select
   }
   if (host_out) {
     CK(cudaMemcpyAsync(distances, D, sizeof(float) * nq * k, cudaMemcpyDeviceToHost, st));

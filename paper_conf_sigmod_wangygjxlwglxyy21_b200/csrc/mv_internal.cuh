@@ -62,6 +62,12 @@ __device__ __forceinline__ bool bit_excluded(const uint8_t* __restrict__ bitset,
   return (__ldg(bitset + (id >> 3)) >> (id & 7)) & 1;
 }
 
+// debug event counters (set by the scan when MV_SCAN_TRACE=1): 0 tiles-with-survivors, 1 warm-ups,
+// 2 flushes, 3 bisection fallbacks, 4 survivors appended
+__device__ __forceinline__ void dbg_count(unsigned long long* c, int i, unsigned long long v) {
+  if (c && (threadIdx.x & 31) == 0) atomicAdd(c + i, v);
+}
+
 // ------------------------------------------------------------------------------------------
 // Warp-cooperative insertion into a sorted (ascending) smem list of length L.  All 32 lanes
 // call it; lanes with `has` offer one candidate each.  Candidates not below the current last
@@ -306,8 +312,10 @@ __device__ __forceinline__ void warp_flush_buffer(uint64_t* L, uint64_t* B, int*
 template <typename Low, typename Pub>
 __device__ __forceinline__ void warp_collect_passed(uint64_t* L, uint64_t* B, int* nb, uint32_t* bnd, int k, uint64_t li,
                                                     const uint32_t (&k32)[4], bool (&pass)[4], int npass, Low low,
-                                                    Pub publish, uint64_t* wscr) {
+                                                    Pub publish, uint64_t* wscr, unsigned long long* dc = nullptr) {
   const int lane = threadIdx.x & 31;
+  dbg_count(dc, 0, 1);
+  if (npass > 32) dbg_count(dc, 1, 1);
   if (npass > 32) {
     uint32_t v[4];
 #pragma unroll
@@ -331,7 +339,13 @@ __device__ __forceinline__ void warp_collect_passed(uint64_t* L, uint64_t* B, in
       return;
     }
   }
-  if (*nb + npass > 32) warp_flush_buffer(L, B, nb, bnd, k, li);
+  if (*nb + npass > 32) {
+    warp_flush_buffer(L, B, nb, bnd, k, li);
+    dbg_count(dc, 2, 1);
+    // the list's k-th key is an exact upper bound of the query's k-th best: share it
+    if (lane == 0 && L[k - 1] != MV_KEY_PAD) publish((uint32_t)(L[k - 1] >> 32));
+  }
+  dbg_count(dc, 4, npass);
   int off = *nb;
 #pragma unroll
   for (int m = 0; m < 4; ++m) {
@@ -349,7 +363,7 @@ __device__ __forceinline__ void warp_collect_passed(uint64_t* L, uint64_t* B, in
 //   rowk(g, m) -> distance key of element m*32+lane for query g;  st(g) -> per-query state.
 template <int G, typename RowK, typename State, typename Low, typename Pub>
 __device__ __forceinline__ void warp_filter_group(int nvalid, int k, RowK rowk, State st, Low low, Pub publish,
-                                                  uint64_t* wscr) {
+                                                  uint64_t* wscr, unsigned long long* dc = nullptr, bool fold = true) {
   uint32_t k32[G][4];
   uint32_t thr32[G];
 #pragma unroll
@@ -377,6 +391,7 @@ __device__ __forceinline__ void warp_filter_group(int nvalid, int k, RowK rowk, 
       npass[g] += __popc(__ballot_sync(MV_FULL, pass[g][m]));
     }
   }
+  if (!fold) return;
 #pragma unroll
   for (int g = 0; g < G; ++g) {
     if (npass[g] == 0) continue;
@@ -386,7 +401,7 @@ __device__ __forceinline__ void warp_filter_group(int nvalid, int k, RowK rowk, 
     uint64_t li;
     st(g, L, B, nb, bnd, li);
     warp_collect_passed(L, B, nb, bnd, k, li, k32[g], pass[g], npass[g], [&](int v) { return low(g, v); },
-                        [&](uint32_t t) { publish(g, t); }, wscr);
+                        [&](uint32_t t) { publish(g, t); }, wscr, dc);
   }
 }
 
@@ -457,7 +472,8 @@ struct Bucketing {
   int32_t* bq;       // nq*npb     pair ids grouped by list
   int32_t* wcount;   // nlist      work items per list
   int32_t* woff;     // nlist+1
-  int2* witems;      // <= nlist + nq*npb   (list, first bucket position)
+  int2* witems;      // <= nlist + nq*npb   (list, first bucket position), longest first
+  int2* witems_unsorted;
   int64_t* qtot;     // nq+1       per-query candidate capacity, then exclusive scan
   int64_t* poff;     // nq*npb     region offset per pair
   int32_t* pcnt;     // nq*npb     candidates written per pair
@@ -465,7 +481,7 @@ struct Bucketing {
 };
 cudaError_t launch_bucket(const int32_t* probes, int64_t nq, int npb, int nlist, const int64_t* list_off, int k,
                           int qchunk, const Bucketing& b, cudaStream_t st);
-cudaError_t launch_pair_offsets(const int32_t* probes, int64_t nq, int npb, const int64_t* list_off, int k,
+cudaError_t launch_pair_offsets(const int32_t* probes, int64_t nq, int npb, const int64_t* list_off, int k, int capk,
                                 const Bucketing& b, cudaStream_t st);
 cudaError_t launch_scan_i32(const int32_t* in, int n, int32_t* out, cudaStream_t st);   // out[n+1]
 cudaError_t launch_scan_i64(const int64_t* in, int64_t n, int64_t* out, cudaStream_t st);  // out[n+1]
