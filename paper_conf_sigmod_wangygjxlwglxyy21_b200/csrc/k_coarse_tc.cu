@@ -27,6 +27,11 @@ __device__ __forceinline__ void cbar(int id, int n) { asm volatile("bar.sync %0,
 }  // namespace
 
 template <int NQB>
+constexpr uint32_t coarse_tmem_cols() {
+  return 4 * NQB <= 128 ? 128 : (4 * NQB <= 256 ? 256 : 512);
+}
+
+template <int NQB>
 __global__ void __launch_bounds__(kCThreads, 1)
     k_coarse_tc(const __grid_constant__ CUtensorMap cmap, const __grid_constant__ CUtensorMap qmap, const CoarseParams p) {
   extern __shared__ uint8_t smem_raw[];
@@ -68,7 +73,7 @@ __global__ void __launch_bounds__(kCThreads, 1)
     fence_mbar_init();
   }
   if (warp == 1) {
-    tmem_alloc(tslot, 4 * NQB);
+    tmem_alloc(tslot, coarse_tmem_cols<NQB>());
     tmem_relinquish();
   }
   if (warp == 0 && lane == 0) {
@@ -209,7 +214,7 @@ __global__ void __launch_bounds__(kCThreads, 1)
   __syncthreads();
   if (warp == 1) {
     tc_fence_after();
-    tmem_dealloc(tmem, 4 * NQB);
+    tmem_dealloc(tmem, coarse_tmem_cols<NQB>());
   }
 }
 
@@ -233,36 +238,57 @@ cudaError_t launch_hilo(const float* x, int64_t n, int d, int dpad, float* out, 
   return cudaGetLastError();
 }
 
-bool coarse_tc_plan(int dpad, int nprobe, CoarseParams& p) {
+static int coarse_fixed_smem(int nqb, int nchunks, int nprobe) {
+  return nchunks * 2 * nqb * 128 + nqb * kCDLD * 4 + 8 + nqb * nprobe * 8 + 32 * kCEpi * 8 + nqb * 32 * 8 + nqb * 8 + 256;
+}
+
+// Query-block size: the one that minimises (waves x block size) -- a second, mostly empty wave
+// doubles the coarse time -- among the shapes whose shared memory fits with >= 2 centroid stages.
+bool coarse_tc_plan(int dpad, int nprobe, int64_t nq, int nsm, CoarseParams& p) {
   if (dpad % 32 != 0 || nprobe > 128) return false;
-  p.nqb = nprobe <= 32 ? 64 : 32;
   p.nchunks = dpad / 32;
   p.nprobe = nprobe;
-  const int brows = 2 * p.nqb;
-  const int fixed = p.nchunks * brows * 128 + p.nqb * kCDLD * 4 + 8 + p.nqb * nprobe * 8 + 32 * kCEpi * 8 +
-                    p.nqb * 32 * 8 + p.nqb * 8 + 256;
   const int budget = 227 * 1024 - 1024;
-  const int ns = std::min(4, (budget - fixed) / (2 * 128 * 128));
-  if (ns < 2) return false;
-  p.nstage = ns;
-  p.smem_total = fixed + ns * 2 * 128 * 128 + 1024;
+  const int stage = 2 * 128 * 128;
+  int best = -1;
+  int64_t best_cost = 0;
+  for (int nqb : {32, 48, 64, 80}) {
+    if (nprobe > 32 && nqb > 32) continue;
+    const int fixed = coarse_fixed_smem(nqb, p.nchunks, nprobe);
+    if ((budget - fixed) / stage < 2) continue;
+    const int64_t blocks = (nq + nqb - 1) / nqb;
+    const int64_t cost = ((blocks + nsm - 1) / nsm) * (int64_t)(nqb + 32);  // + fixed per-CTA streaming
+    if (best < 0 || cost < best_cost) {
+      best = nqb;
+      best_cost = cost;
+    }
+  }
+  if (best < 0) return false;
+  p.nqb = best;
+  const int fixed = coarse_fixed_smem(best, p.nchunks, nprobe);
+  p.nstage = std::min(4, (budget - fixed) / stage);
+  p.smem_total = fixed + p.nstage * stage + 1024;
   return p.smem_total <= 227 * 1024;
+}
+
+template <int NQB>
+static cudaError_t run_coarse_tc(const CUtensorMap* cmap, const CUtensorMap* qmap, const CoarseParams& p, unsigned grid,
+                                 cudaStream_t st) {
+  cudaError_t e = cudaFuncSetAttribute(k_coarse_tc<NQB>, cudaFuncAttributeMaxDynamicSharedMemorySize, p.smem_total);
+  if (e != cudaSuccess) return e;
+  k_coarse_tc<NQB><<<grid, kCThreads, p.smem_total, st>>>(*cmap, *qmap, p);
+  return cudaGetLastError();
 }
 
 cudaError_t launch_coarse_tc(const CUtensorMap* cmap, const CUtensorMap* qmap, const CoarseParams& p, int64_t nq,
                              cudaStream_t st) {
   const unsigned grid = (unsigned)((nq + p.nqb - 1) / p.nqb);
-  cudaError_t e;
-  if (p.nqb == 64) {
-    e = cudaFuncSetAttribute(k_coarse_tc<64>, cudaFuncAttributeMaxDynamicSharedMemorySize, p.smem_total);
-    if (e != cudaSuccess) return e;
-    k_coarse_tc<64><<<grid, kCThreads, p.smem_total, st>>>(*cmap, *qmap, p);
-  } else {
-    e = cudaFuncSetAttribute(k_coarse_tc<32>, cudaFuncAttributeMaxDynamicSharedMemorySize, p.smem_total);
-    if (e != cudaSuccess) return e;
-    k_coarse_tc<32><<<grid, kCThreads, p.smem_total, st>>>(*cmap, *qmap, p);
+  switch (p.nqb) {
+    case 32: return run_coarse_tc<32>(cmap, qmap, p, grid, st);
+    case 48: return run_coarse_tc<48>(cmap, qmap, p, grid, st);
+    case 64: return run_coarse_tc<64>(cmap, qmap, p, grid, st);
+    default: return run_coarse_tc<80>(cmap, qmap, p, grid, st);
   }
-  return cudaGetLastError();
 }
 
 }  // namespace mv

@@ -82,6 +82,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
   uint64_t* cbuf = scratch + 32 * kEpiWarps;                               // QC x 32 (k <= 32)
   int* cnb = reinterpret_cast<int*>(cbuf + 32 * QC);                       // QC counts
   uint32_t* cbnd = reinterpret_cast<uint32_t*>(cnb + QC);                  // QC running bounds
+  int* selctr = reinterpret_cast<int*>(sm + p.off_ctr);                    // per-tile slot dispenser
   uint8_t* side = sm + p.off_side;
   uint64_t* bars = reinterpret_cast<uint64_t*>(sm + p.off_bar);
   uint64_t* full_x = bars;
@@ -320,6 +321,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
           }
         }
         if (et < wi.nqc && tau_now < lim[et]) const_cast<uint64_t*>(lim)[et] = tau_now;
+        if (et == 0) *selctr = 0;
         tc_fence_before();
         if (et == 0) MV_TRACE(4, titer);
         __syncwarp();
@@ -329,12 +331,18 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
         // ---- a6: filter against min(list k-th, running bound, global tau) + select (warp per query)
         if (sel && k <= 32) {
           constexpr int G = 4;
-          for (int i0 = ew; i0 < ((p.dbg & 1) ? 0 : wi.nqc); i0 += kEpiWarps * G) {
-            const int nvalid = min(G, (wi.nqc - i0 + kEpiWarps - 1) / kEpiWarps);
+          // query slots are handed out G at a time through a shared counter, so a warp stuck in a
+          // warm-up or flush does not hold the others at the end-of-tile barrier
+          for (;;) {
+            int i0 = 0;
+            if (lane == 0) i0 = atomicAdd(selctr, G);
+            i0 = __shfl_sync(MV_FULL, i0, 0);
+            if (i0 >= ((p.dbg & 1) ? 0 : wi.nqc)) break;
+            const int nvalid = min(G, wi.nqc - i0);
             warp_filter_group<G>(
-                nvalid, k, [&](int g, int m) { return Dt[(i0 + g * kEpiWarps) * kDLD + m * 32 + lane]; },
+                nvalid, k, [&](int g, int m) { return Dt[(i0 + g) * kDLD + m * 32 + lane]; },
                 [&](int g, uint64_t*& L, uint64_t*& B, int*& nb, uint32_t*& bnd, uint64_t& li) {
-                  const int i = i0 + g * kEpiWarps;
+                  const int i = i0 + g;
                   L = lists + (int64_t)i * k;
                   B = cbuf + i * 32;
                   nb = cnb + i;
@@ -343,7 +351,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
                 },
                 [&](int, int v) { return srank[v]; },
                 [&](int g, uint32_t t32) {
-                  atomicMin(reinterpret_cast<unsigned long long*>(p.tau + mp[i0 + g * kEpiWarps] / p.npb),
+                  atomicMin(reinterpret_cast<unsigned long long*>(p.tau + mp[i0 + g] / p.npb),
                             ((unsigned long long)t32 << 32) | 0xffffffffull);
                 },
                 wscr, (p.prof && (p.dbg & 64)) ? p.prof + 8 * 1024 + 1000 : nullptr, !(p.dbg & 32));
@@ -548,7 +556,8 @@ bool tc_scan_plan(int type, int dpad, int k, TcScanParams& p) {
   p.off_lists = p.off_dt + up(dt_bytes, 16);
   p.off_meta = p.off_lists + up(lists_bytes, 16);
   p.off_misc = p.off_meta + 2 * p.meta_bytes;
-  p.off_side = up(p.off_misc + misc_bytes, 128);
+  p.off_ctr = p.off_misc + misc_bytes;
+  p.off_side = up(p.off_ctr + 16, 128);
   p.off_bar = p.off_side + side_bytes;
   p.smem_total = p.off_bar + (2 * ns + 10 + 2 * kNTS) * 8 + 16 + 1024;
   return p.smem_total <= 227 * 1024;

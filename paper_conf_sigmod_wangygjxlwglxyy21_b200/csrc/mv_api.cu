@@ -161,7 +161,10 @@ static cudaError_t run_coarse(mv_index* ix, const float* qpad, const float* qhl,
                               cudaStream_t st) {
   CoarseParams cp;
   const char* force = getenv("MV_FORCE_SIMT");
-  if (npb < ix->nlist && ix->cmap_ok && !(force && force[0] == '1') && coarse_tc_plan(ix->dpad, npb, cp)) {
+  int dev = 0, nsm = kNumSMs;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+  if (npb < ix->nlist && ix->cmap_ok && !(force && force[0] == '1') && coarse_tc_plan(ix->dpad, npb, nq, nsm, cp)) {
     CUtensorMap qmap;
     if (make_tmap_2d(&qmap, qhl, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, (uint64_t)ix->dpad, 2 * (uint64_t)nq,
                      (uint64_t)ix->dpad * 4, 32, (uint32_t)cp.nqb, CU_TENSOR_MAP_SWIZZLE_128B)) {

@@ -517,7 +517,7 @@ struct TcScanParams {
   int type, metric, dpad, k, npb, qchunk, nchunks, nstage, ncol, tmem_cols;
   int64_t nq;              // FLAT query planes are plane-major [2][nq][dpad]
   int off_x, off_q, q_bytes, off_dt, off_lists, off_meta, meta_bytes, meta_lim_off, off_misc, off_side, off_bar,
-      smem_total;
+      off_ctr, smem_total;
   const int64_t* list_off;
   const double* norms;     // ||x||^2 (FLAT) or ||x_hat||^2 (SQ8), fp64
   const int64_t* ids;
@@ -553,7 +553,7 @@ struct CoarseParams {
   const float* cnorm;
   int32_t* probes;
 };
-bool coarse_tc_plan(int dpad, int nprobe, CoarseParams& p);
+bool coarse_tc_plan(int dpad, int nprobe, int64_t nq, int nsm, CoarseParams& p);
 cudaError_t launch_coarse_tc(const CUtensorMap* cmap, const CUtensorMap* qmap, const CoarseParams& p, int64_t nq,
                              cudaStream_t st);
 cudaError_t launch_hilo(const float* x, int64_t n, int d, int dpad, float* out, cudaStream_t st);
