@@ -352,7 +352,7 @@ def main():
     bpv = (4 * dpad if cfg["kind"] == "flat" else dpad) + (8 if bs is not None else 0)
     units = int(lens[probed].sum())  # distinct probed vectors per launch (this GPU's shard)
     scan_bytes = units * bpv
-    scan_ms = stage_ms["scan"]
+    scan_ms = stage_ms["scan_a"] + stage_ms["scan"]  # both launches of the scan kernel (phases A and B)
     achieved = scan_bytes / (scan_ms / 1e3) / 1e9
     traffic = None
     tf = os.path.join(ROOT, "profiles", "scan_traffic.json")

@@ -138,9 +138,11 @@ MV_API mv_status mv_index_get_sq8(const mv_index* index, float* vmin, float* vdi
 
 /* Stage profiling (measurement, §8(d)).  When enabled, mv_search records CUDA events on its
  * stream around each stage:  0 = query staging + coarse (a1-a3), 1 = bucketing (a4),
- * 2 = grouped list scan with fused partial top-k (a5-a6), 3 = final select (a7).
+ * 2 = list scan phase A (a5-a6: the seeding lists, every candidate emitted; the whole scan when
+ * there is no seeding), 3 = seed select (tau_q = k-th best key of phase A), 4 = list scan phase B
+ * (a5-a6: candidates below tau_q), 5 = final select (a7).
  * mv_profile_read synchronises on the recorded events and returns, per stage, the summed
- * milliseconds since the last reset (ms[4]); *searches = profiled mv_search calls; *launches =
+ * milliseconds since the last reset (ms[6]); *searches = profiled mv_search calls; *launches =
  * kernels libmv launched in them.  `reset` != 0 clears the accumulators after reading. */
 MV_API mv_status mv_profile_enable(mv_index* index, int on);
 MV_API mv_status mv_profile_read(mv_index* index, double* ms, int64_t* searches, int64_t* launches, int reset);

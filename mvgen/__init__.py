@@ -149,9 +149,12 @@ def _gauss(seed: int, stream: int, ctr: torch.Tensor) -> torch.Tensor:
 
 
 class DeepSpec:
-    """mu_t ~ N(0,I) normalised; micro = normalise(mu_t + s1 g); x = normalise(micro + s2 g)."""
+    """mu_t ~ N(0,I) normalised; micro = normalise(mu_t + s1 g/sqrt(d)); x = normalise(micro + s2 g/sqrt(d)).
 
-    def __init__(self, d: int = 96, n_top: int = 256, n_micro: int = 262144, s1: float = 0.6, s2: float = 0.35,
+    s1 and s2 are relative noise norms (g/sqrt(d) has norm ~1), so the cluster structure does not
+    dissolve into isotropic noise as d grows."""
+
+    def __init__(self, d: int = 96, n_top: int = 256, n_micro: int = 262144, s1: float = 0.6, s2: float = 0.5,
                  seed: int = SEED_BASE):
         self.d, self.n_top, self.n_micro, self.s1, self.s2, self.seed = d, n_top, n_micro, s1, s2, seed
         g = _gauss(seed, 51, torch.arange(n_top * d, dtype=torch.int64)).reshape(n_top, d)
@@ -163,9 +166,9 @@ class DeepSpec:
         m = hash_u31(row_seed, 61, rows) % self.n_micro
         t = hash_u31(self.seed, 63, m) % self.n_top
         j = torch.arange(d, dtype=torch.int64, device=device)
-        mc = self.top.to(device)[t] + self.s1 * _gauss(self.seed, 71, m[:, None] * d + j[None, :])
+        mc = self.top.to(device)[t] + (self.s1 / d ** 0.5) * _gauss(self.seed, 71, m[:, None] * d + j[None, :])
         mc = mc / mc.norm(dim=1, keepdim=True)
-        x = mc + self.s2 * _gauss(row_seed, 81, rows[:, None] * d + j[None, :])
+        x = mc + (self.s2 / d ** 0.5) * _gauss(row_seed, 81, rows[:, None] * d + j[None, :])
         x = x / x.norm(dim=1, keepdim=True)
         return x.to(torch.float32)
 

@@ -10,6 +10,7 @@ import hashlib
 import os
 import subprocess
 import sys
+from concurrent.futures import ThreadPoolExecutor
 
 PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
@@ -38,14 +39,39 @@ def build(force: bool = False, verbose: bool = False) -> str:
     dg = _digest()
     if not force and os.path.exists(LIB) and os.path.exists(stamp) and open(stamp).read().strip() == dg:
         return LIB
-    cmd = [NVCC, *ARCH, *FLAGS, "-I", os.path.join(ROOT, "include"), "-I", CSRC, "-o", LIB, *sources()]
-    r = subprocess.run(cmd, capture_output=True, text=True)
+    # one nvcc per source in parallel (each .cu owns its kernels: no device linking), then link
+    objdir = os.path.join(PKG, "build")
+    os.makedirs(objdir, exist_ok=True)
+    inc = ["-I", os.path.join(ROOT, "include"), "-I", CSRC]
+    cflags = [f for f in FLAGS if f != "-shared"]
+
+    def compile_one(src):
+        obj = os.path.join(objdir, os.path.basename(src) + ".o")
+        cmd = [NVCC, *ARCH, *cflags, *inc, "-c", "-o", obj, src]
+        r = subprocess.run(cmd, capture_output=True, text=True)
+        return obj, cmd, r
+
+    with ThreadPoolExecutor(max_workers=min(16, os.cpu_count() or 4)) as ex:
+        results = list(ex.map(compile_one, sources()))
     log = os.path.join(PKG, "build.log")
+    text = ""
+    failed = None
+    for obj, cmd, r in results:
+        text += " ".join(cmd) + "\n" + r.stdout + r.stderr
+        if r.returncode != 0 and failed is None:
+            failed = r
+    if failed is None:
+        lcmd = [NVCC, *ARCH, "-shared", "-Xcompiler", "-fPIC", "-o", LIB, *[o for o, _, _ in results]]
+        failed_link = subprocess.run(lcmd, capture_output=True, text=True)
+        text += " ".join(lcmd) + "\n" + failed_link.stdout + failed_link.stderr
+        if failed_link.returncode != 0:
+            failed = failed_link
     with open(log, "w") as f:
-        f.write(" ".join(cmd) + "\n" + r.stdout + r.stderr)
-    if r.returncode != 0:
-        sys.stderr.write(r.stderr[-8000:])
-        raise RuntimeError(f"nvcc failed (exit {r.returncode}); see {log}")
+        f.write(text)
+    if failed is not None:
+        sys.stderr.write(failed.stderr[-8000:])
+        raise RuntimeError(f"nvcc failed (exit {failed.returncode}); see {log}")
+    r = subprocess.CompletedProcess([], 0, "", text)
     if verbose:
         sys.stderr.write(r.stderr)
     with open(stamp, "w") as f:

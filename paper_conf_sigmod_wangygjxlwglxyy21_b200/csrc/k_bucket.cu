@@ -42,13 +42,68 @@ cudaError_t launch_scan_i64(const int64_t* in, int64_t n, int64_t* out, cudaStre
   return cudaGetLastError();
 }
 
-__global__ void k_bucket_fill(const int32_t* __restrict__ probes, int64_t npairs, const int32_t* __restrict__ boff,
-                              int32_t* bfill, int32_t* bq) {
+// Virtual list of pair p = q*npb + r: its list l, or l + nlist for the pairs of the second phase
+// when the seeding phase is on (ra != nullptr): phase A = the ra[q] nearest lists of query q,
+// scanned first so that their k-th best bounds tau_q before the other lists are scanned.
+__device__ __forceinline__ int vlist_of(const int32_t* probes, int64_t p, int npb, int nlist, const int32_t* ra) {
+  const int l = probes[p];
+  return (ra && (int)(p % npb) >= ra[p / npb]) ? l + nlist : l;
+}
+
+__global__ void k_count_pairs(const int32_t* __restrict__ probes, int64_t npairs, int npb, int nlist,
+                              const int32_t* __restrict__ ra, int32_t* counts) {
+  for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < npairs; p += (int64_t)gridDim.x * blockDim.x)
+    atomicAdd(counts + vlist_of(probes, p, npb, nlist, ra), 1);
+}
+
+__global__ void k_bucket_fill(const int32_t* __restrict__ probes, int64_t npairs, int npb, int nlist,
+                              const int32_t* __restrict__ ra, const int32_t* __restrict__ boff, int32_t* bfill,
+                              int32_t* bq) {
   for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < npairs; p += (int64_t)gridDim.x * blockDim.x) {
-    const int l = probes[p];
+    const int l = vlist_of(probes, p, npb, nlist, ra);
     const int pos = boff[l] + atomicAdd(bfill + l, 1);
     bq[pos] = (int32_t)p;
   }
+}
+
+// one warp per query: ra[q] = the fewest nearest lists holding >= need candidates (at most npb)
+__global__ void k_seed_ranks(const int32_t* __restrict__ probes, int64_t nq, int npb,
+                             const int64_t* __restrict__ list_off, int64_t need, int32_t* ra) {
+  const int lane = threadIdx.x & 31;
+  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t q = warp; q < nq; q += nwarps) {
+    int64_t run = 0;
+    int r = npb;
+    for (int j0 = 0; j0 < npb; j0 += 32) {
+      const int j = j0 + lane;
+      int64_t c = 0;
+      if (j < npb) {
+        const int l = probes[q * npb + j];
+        c = list_off[l + 1] - list_off[l];
+      }
+      int64_t incl = c;
+      for (int o = 1; o < 32; o <<= 1) {
+        const int64_t v = __shfl_up_sync(MV_FULL, incl, o);
+        if (lane >= o) incl += v;
+      }
+      const uint32_t hit = __ballot_sync(MV_FULL, j < npb && run + incl >= need);
+      if (hit) {
+        r = j0 + __ffs(hit);  // ranks 0 .. first hit
+        break;
+      }
+      run += __shfl_sync(MV_FULL, incl, 31);
+    }
+    if (lane == 0) ra[q] = r;
+  }
+}
+
+cudaError_t launch_seed_ranks(const int32_t* probes, int64_t nq, int npb, const int64_t* list_off, int64_t need,
+                              int32_t* ra, cudaStream_t st) {
+  if (nq == 0) return cudaSuccess;
+  const int grid = (int)min64(kNumSMs * 8, (nq * 32 + 255) / 256);
+  k_seed_ranks<<<grid, 256, 0, st>>>(probes, nq, npb, list_off, need, ra);
+  return cudaGetLastError();
 }
 
 __global__ void k_work_count(const int32_t* __restrict__ lcount, int nlist, int qchunk, int32_t* wcount) {
@@ -65,11 +120,12 @@ __global__ void k_work_fill(const int32_t* __restrict__ wcount, const int32_t* _
 }
 
 // Longest-first order for the persistent scan's static round-robin: a single-CTA counting sort of
-// the work items by descending cost key = 64 * tiles + queries (tiles = ceil(|list| / 128)).
+// the work items by descending cost key = 64 * tiles + queries (tiles = ceil(|list| / 128)); with
+// the seeding split, every phase-A item (virtual list < nlist) precedes every phase-B item.
 __global__ void __launch_bounds__(1024) k_sort_work(const int2* __restrict__ in, const int32_t* __restrict__ nwork_p,
                                                     const int32_t* __restrict__ boff, const int64_t* __restrict__ list_off,
-                                                    int qchunk, int2* __restrict__ out) {
-  constexpr int NB = 4096;
+                                                    int nlist, int qchunk, int2* __restrict__ out) {
+  constexpr int NB = 8192, HB = 4096;
   __shared__ int hist[NB];
   __shared__ int part[1024];
   const int nwork = *nwork_p, tid = threadIdx.x;
@@ -77,19 +133,20 @@ __global__ void __launch_bounds__(1024) k_sort_work(const int2* __restrict__ in,
   __syncthreads();
   auto key = [&](int w) {
     const int2 it = in[w];
+    const int l = it.x >= nlist ? it.x - nlist : it.x;
     const int nq = min(qchunk, boff[it.x + 1] - it.y);
-    const int64_t len = list_off[it.x + 1] - list_off[it.x];
+    const int64_t len = list_off[l + 1] - list_off[l];
     const int tiles = (int)min64((len + 127) / 128, 63);
-    return NB - 1 - min(NB - 1, tiles * 64 + min(nq, 63));  // descending cost -> ascending bin
+    return (it.x >= nlist ? HB : 0) + HB - 1 - min(HB - 1, tiles * 64 + min(nq, 63));  // descending cost
   };
   for (int w = tid; w < nwork; w += 1024) atomicAdd(&hist[key(w)], 1);
   __syncthreads();
-  // exclusive scan of 4096 bins: 4 per thread
-  int loc[4], acc = 0;
+  // exclusive scan of 8192 bins: 8 per thread
+  int loc[8], acc = 0;
 #pragma unroll
-  for (int j = 0; j < 4; ++j) {
+  for (int j = 0; j < 8; ++j) {
     loc[j] = acc;
-    acc += hist[tid * 4 + j];
+    acc += hist[tid * 8 + j];
   }
   part[tid] = acc;
   __syncthreads();
@@ -102,34 +159,35 @@ __global__ void __launch_bounds__(1024) k_sort_work(const int2* __restrict__ in,
   const int base = tid ? part[tid - 1] : 0;
   __syncthreads();
 #pragma unroll
-  for (int j = 0; j < 4; ++j) hist[tid * 4 + j] = base + loc[j];
+  for (int j = 0; j < 8; ++j) hist[tid * 8 + j] = base + loc[j];
   __syncthreads();
   for (int w = tid; w < nwork; w += 1024) out[atomicAdd(&hist[key(w)], 1)] = in[w];
 }
 
 cudaError_t launch_bucket(const int32_t* probes, int64_t nq, int npb, int nlist, const int64_t* list_off, int k,
-                          int qchunk, const Bucketing& b, cudaStream_t st) {
+                          int qchunk, const int32_t* ra, const Bucketing& b, cudaStream_t st) {
   (void)k;
   const int64_t npairs = nq * npb;
-  cudaMemsetAsync(b.lcount, 0, sizeof(int32_t) * nlist, st);
-  cudaMemsetAsync(b.bfill, 0, sizeof(int32_t) * nlist, st);
+  const int nv = ra ? 2 * nlist : nlist;  // virtual lists
+  cudaMemsetAsync(b.lcount, 0, sizeof(int32_t) * nv, st);
+  cudaMemsetAsync(b.bfill, 0, sizeof(int32_t) * nv, st);
   cudaMemsetAsync(b.counter, 0, sizeof(int32_t), st);
-  cudaError_t e = launch_count_lists(probes, npairs, b.lcount, st);
-  if (e != cudaSuccess) return e;
-  if ((e = launch_scan_i32(b.lcount, nlist, b.boff, st)) != cudaSuccess) return e;
   const int grid = (int)min64(kNumSMs * 8, (npairs + 255) / 256);
-  if (npairs) k_bucket_fill<<<grid, 256, 0, st>>>(probes, npairs, b.boff, b.bfill, b.bq);
-  k_work_count<<<(nlist + 255) / 256, 256, 0, st>>>(b.lcount, nlist, qchunk, b.wcount);
-  if ((e = launch_scan_i32(b.wcount, nlist, b.woff, st)) != cudaSuccess) return e;
-  k_work_fill<<<(nlist + 255) / 256, 256, 0, st>>>(b.wcount, b.woff, b.boff, nlist, qchunk, b.witems_unsorted);
-  k_sort_work<<<1, 1024, 0, st>>>(b.witems_unsorted, b.woff + nlist, b.boff, list_off, qchunk, b.witems);
+  if (npairs) k_count_pairs<<<grid, 256, 0, st>>>(probes, npairs, npb, nlist, ra, b.lcount);
+  cudaError_t e;
+  if ((e = launch_scan_i32(b.lcount, nv, b.boff, st)) != cudaSuccess) return e;
+  if (npairs) k_bucket_fill<<<grid, 256, 0, st>>>(probes, npairs, npb, nlist, ra, b.boff, b.bfill, b.bq);
+  k_work_count<<<(nv + 255) / 256, 256, 0, st>>>(b.lcount, nv, qchunk, b.wcount);
+  if ((e = launch_scan_i32(b.wcount, nv, b.woff, st)) != cudaSuccess) return e;
+  k_work_fill<<<(nv + 255) / 256, 256, 0, st>>>(b.wcount, b.woff, b.boff, nv, qchunk, b.witems_unsorted);
+  k_sort_work<<<1, 1024, 0, st>>>(b.witems_unsorted, b.woff + nv, b.boff, list_off, nlist, qchunk, b.witems);
   return cudaGetLastError();
 }
 
-// Region capacity of pair (q, j): min(k, |list|) when the scan selects locally (k <= 1024),
-// else |list| (every candidate that survives the bitset is emitted).
+// Region capacity of pair (q, j): min(capk, |list|) when the SIMT scan selects locally (k <= 1024,
+// capk > 0), else |list| (every candidate that survives the bitset may be emitted).
 __device__ __forceinline__ int64_t pair_cap(int64_t len, int k, int capk) {
-  return k <= kLocalSelectMaxK ? min64(capk, len) : len;
+  return (capk > 0 && k <= kLocalSelectMaxK) ? min64(capk, len) : len;
 }
 
 // one warp per query: qtot[q] = sum_j cap(q, j)

@@ -2,24 +2,35 @@
 //
 // PAPER.md:529-532 (§3.1) step (2): scan the nprobe probed buckets with the fine quantizer;
 // PAPER.md:916-922 (§4.1 B): the bitmap is checked for every encountered vector before the
-// top-k; PAPER.md:590-596 (§3.2.1): per-worker heaps merged at the end.  PAPER.md:569-575: the
-// loaded data vectors are reused for many queries -- here one 128-vector list tile in shared
-// memory meets every query of that list's bucket in one tensor-core contraction.
+// top-k.  PAPER.md:569-575 (§3.2.1): the loaded data vectors are reused for many queries -- here
+// one 128-vector list tile in shared memory meets every query of that list's bucket in one
+// tensor-core contraction.  PAPER.md:590-596: per-worker partial results merged at the end.
 //
 // Work item = (list l, <= qchunk queries probing l).  Persistent CTA per SM, warp-specialised:
-//   warp 0     TMA producer: list tiles (128 rows x one 128-B / 32-B swizzle atom per stage)
+//   warp 0     TMA producer: list tiles (128 rows x one 128-B / 32-B swizzle atom per stage) and
+//              the tiles' side data (norms, id ranks, ids) by bulk copy
 //   warp 1     TMEM owner + single-thread tcgen05.mma issuer
 //              D[128 vectors x N] (+)= X_tile[128 x K] . Qplanes[N x K]^T, N = P x roundup16(nq)
-//   warps 2-3  query gatherer: the bucket's query planes -> swizzled K-major smem (double buffer)
-//   warps 4-7  epilogue: tcgen05.ld (row per thread) -> distance -> bitset -> transposed keys in
-//              smem -> one warp per query filters against its running k-th best (and the global
-//              per-query threshold tau) and inserts survivors (a6).
+//   warps 2-3  query gatherer: the bucket's query planes -> swizzled K-major smem, and the
+//              per-query metadata (threshold, output region) -- both double-buffered
+//   warps 4-11 epilogue, two warps per TMEM lane quarter: every thread owns one vector row and
+//              half of the query columns; tcgen05.ld -> distance -> bitset -> threshold test ->
+//              survivors are appended to the (query, list) pair's output region (a6).
+//
+// a6 is a filter, not a selection.  The search runs the scan twice:
+//   phase A (p.phase 0) scans each query's rA nearest lists and emits every candidate; a
+//     per-query select (k_select.cu) turns them into tau_q = the k-th best key so far -- an exact
+//     upper bound of the query's final k-th best;
+//   phase B (p.phase 1) scans the other pairs and emits only keys below tau_q.
+// The final select takes the exact top-k of everything emitted.  No per-pair selection state,
+// no epilogue-wide barrier per tile: the epilogue warps run independently.
+//
 // FLAT (kind::tf32): X = fp32 payload used as tf32 -- exact when the stored values are
 //   tf32-representable (integer SIFT data; the index checks this at add time); the query is
 //   split into hi + lo tf32 planes (P = 2), so the query side is exact to ~2^-22.
 // SQ8 (kind::i8): X = u8 codes straight from HBM; the query-side weights w_j = q_j * vdiff_j/255
-//   are expanded into P = 3 signed 8-bit digit planes with a per-query scale, so
-//   q.x_hat = q.a + s (D0 + D1/2^7 + D2/2^14) with int32-exact partials; no decode instructions.
+//   are expanded into P = 4 signed 8-bit digit planes with a per-query scale, so
+//   q.x_hat = q.a + s (D0 + D1/2^7 + D2/2^14 + D3/2^21) with int32-exact partials; no decode.
 #include "mv_internal.cuh"
 #include "sm100.cuh"
 
@@ -42,9 +53,9 @@ struct WorkInfo {
 __device__ __forceinline__ WorkInfo work_info(const TcScanParams& p, int w) {
   WorkInfo wi;
   const int2 it = p.witems[w];
-  wi.l = it.x;
+  wi.l = it.x >= p.nlist ? it.x - p.nlist : it.x;
   wi.bstart = it.y;
-  wi.nqc = min(p.qchunk, p.boff[wi.l + 1] - wi.bstart);
+  wi.nqc = min(p.qchunk, p.boff[it.x + 1] - wi.bstart);
   wi.lstart = p.list_off[wi.l];
   wi.len = (int)(p.list_off[wi.l + 1] - wi.lstart);
   wi.ntiles = (wi.len + 127) >> 7;
@@ -58,7 +69,33 @@ constexpr int kSideBytes = 3072;
 constexpr int kSideRank = 1152, kSideIds = 1792;
 constexpr int kEpiWarps = 8;      // two epilogue warps per TMEM lane quarter
 constexpr int kThreads = 128 + 32 * kEpiWarps;
-constexpr int kDLD = 129;         // padded transpose stride (conflict-free row and column access)
+
+// per-query metadata of one work item (QCP = roundup16(qchunk) entries per array)
+struct Meta {
+  int32_t* pair;   // (query, rank) pair id, q * npb + r
+  int32_t* cnt;    // candidates emitted so far (smem atomics)
+  float* thf;      // badness bound: a candidate can pass only if badness <= thf (NaN: padding column)
+  float* qnf;      // (float)||q||^2
+  float* qs;       // SQ8 digit scale
+  uint64_t* tau;   // exact bound: emit only keys < tau
+  int64_t* base;   // output region of the pair
+  double* qn;      // ||q||^2 (fp64)
+  double* qa;      // SQ8 q.a (fp64)
+};
+__device__ __forceinline__ Meta meta_at(uint8_t* m, int QCP) {
+  Meta r;
+  r.pair = reinterpret_cast<int32_t*>(m);
+  r.cnt = r.pair + QCP;
+  r.thf = reinterpret_cast<float*>(r.cnt + QCP);
+  r.qnf = r.thf + QCP;
+  r.qs = r.qnf + QCP;
+  r.tau = reinterpret_cast<uint64_t*>(m + 20 * QCP);
+  r.base = reinterpret_cast<int64_t*>(r.tau + QCP);
+  r.qn = reinterpret_cast<double*>(r.base + QCP);
+  r.qa = r.qn + QCP;
+  return r;
+}
+constexpr int kMetaPerQuery = 52;  // bytes
 
 template <int TYPE>
 __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__ CUtensorMap xmap, const TcScanParams p) {
@@ -67,22 +104,16 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
   constexpr int ESZ = TYPE == MV_IVF_FLAT ? 4 : 1;
   constexpr int ATOM = TYPE == MV_IVF_FLAT ? 128 : 32;
   constexpr int P = TYPE == MV_IVF_FLAT ? 2 : 4;
-  const int nstage = p.nstage, nchunks = p.nchunks, QC = p.qchunk, k = p.k;
+  const int nstage = p.nstage, nchunks = p.nchunks;
+  const int QCP = (p.qchunk + 15) & ~15;
   const int rowbytes = p.dpad * ESZ;
   const bool use_norms = p.metric == MV_L2;
   const bool use_ids = p.bitset != nullptr;
+  const bool phaseB = p.phase != 0;
 
   uint8_t* Xs = sm + p.off_x;
   uint8_t* Qs = sm + p.off_q;
-  uint32_t* Dt = reinterpret_cast<uint32_t*>(sm + p.off_dt);
-  uint64_t* lists = reinterpret_cast<uint64_t*>(sm + p.off_lists);
   uint8_t* metab = sm + p.off_meta;
-  int32_t* ecnt = reinterpret_cast<int32_t*>(sm + p.off_misc);
-  uint64_t* scratch = reinterpret_cast<uint64_t*>(sm + p.off_misc + 256);  // 32 per epilogue warp
-  uint64_t* cbuf = scratch + 32 * kEpiWarps;                               // QC x 32 (k <= 32)
-  int* cnb = reinterpret_cast<int*>(cbuf + 32 * QC);                       // QC counts
-  uint32_t* cbnd = reinterpret_cast<uint32_t*>(cnb + QC);                  // QC running bounds
-  int* selctr = reinterpret_cast<int*>(sm + p.off_ctr);                    // per-tile slot dispenser
   uint8_t* side = sm + p.off_side;
   uint64_t* bars = reinterpret_cast<uint64_t*>(sm + p.off_bar);
   uint64_t* full_x = bars;
@@ -95,13 +126,6 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
   uint64_t* full_t = tempty + 2;
   uint64_t* empty_t = full_t + kNTS;
   uint32_t* tslot = reinterpret_cast<uint32_t*>(empty_t + kNTS);
-
-  // metadata per Q buffer: pair[QC] i32 | qs[QC] f32 | (8-B aligned) lim[QC] u64 | qn[QC] f64 | qa[QC] f64
-  auto m_pair = [&](int b) { return reinterpret_cast<int32_t*>(metab + b * p.meta_bytes); };
-  auto m_qs = [&](int b) { return reinterpret_cast<float*>(metab + b * p.meta_bytes) + QC; };
-  auto m_lim = [&](int b) { return reinterpret_cast<uint64_t*>(metab + b * p.meta_bytes + p.meta_lim_off); };
-  auto m_qn = [&](int b) { return reinterpret_cast<double*>(metab + b * p.meta_bytes + p.meta_lim_off) + QC; };
-  auto m_qa = [&](int b) { return reinterpret_cast<double*>(metab + b * p.meta_bytes + p.meta_lim_off) + 2 * QC; };
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
@@ -132,15 +156,14 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
   tc_fence_after();
   const uint32_t tmem = *tslot;
   const int nwork = *p.nwitems;
-  unsigned long long gt0 = 0;
-  if (p.prof) asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(gt0));
+  const int w0 = (p.wbeg ? *p.wbeg : 0) + blockIdx.x;
 
   if (warp == 0) {
     // ------------------------------------------------------------------ TMA producer
     if (lane == 0) {
       uint32_t it = 0, tcount = 0;
       const uint32_t side_tx = 528 + (use_norms ? 1040 : 0) + (use_ids ? 1040 : 0);
-      for (int w = blockIdx.x; w < nwork; w += gridDim.x) {
+      for (int w = w0; w < nwork; w += gridDim.x) {
         const WorkInfo wi = work_info(p, w);
         for (int t = 0; t < wi.ntiles; ++t, ++tcount) {
           const int row0 = (int)(wi.lstart + t * 128);
@@ -165,7 +188,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
     // ------------------------------------------------------------------ MMA issuer
     if (lane == 0) {
       uint32_t it = 0, titer = 0, wcount = 0;
-      for (int w = blockIdx.x; w < nwork; w += gridDim.x, ++wcount) {
+      for (int w = w0; w < nwork; w += gridDim.x, ++wcount) {
         const WorkInfo wi = work_info(p, w);
         const int NQ = (wi.nqc + 15) & ~15;
         const int N = P * NQ;
@@ -206,22 +229,37 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
     // ------------------------------------------------------------------ query gatherer (64 thr)
     const int tq = threadIdx.x - 64;
     uint32_t wcount = 0;
-    for (int w = blockIdx.x; w < nwork; w += gridDim.x, ++wcount) {
+    for (int w = w0; w < nwork; w += gridDim.x, ++wcount) {
       const WorkInfo wi = work_info(p, w);
       const int NQ = (wi.nqc + 15) & ~15;
       const int N = P * NQ;
       const uint32_t b = wcount & 1, r = wcount >> 1;
       mbar_wait(&empty_q[b], (r & 1) ^ 1);
       mbar_wait(&empty_m[b], (r & 1) ^ 1);
-      int32_t* mp = m_pair(b);
-      for (int i = tq; i < wi.nqc; i += 64) {
-        const int pr = p.bq[wi.bstart + i];
-        const int q = pr / p.npb;
-        mp[i] = pr;
-        m_qn(b)[i] = p.qnorm[q];
-        m_qs(b)[i] = TYPE == MV_IVF_SQ8 ? p.qscale[q] : 1.0f;
-        m_qa(b)[i] = TYPE == MV_IVF_SQ8 ? p.qa[q] : 0.0;
-        m_lim(b)[i] = p.tau[q];
+      const Meta mt = meta_at(metab + b * p.meta_bytes, QCP);
+      for (int i = tq; i < NQ; i += 64) {
+        if (i < wi.nqc) {
+          const int pr = p.bq[wi.bstart + i];
+          const int q = pr / p.npb;
+          const double qn = p.qnorm[q];
+          const uint64_t t = phaseB ? p.tau[q] : MV_KEY_PAD;
+          const uint32_t t32 = (uint32_t)(t >> 32);
+          mt.pair[i] = pr;
+          mt.cnt[i] = 0;
+          mt.tau[i] = t;
+          mt.thf[i] = t32 >= 0xff800000u ? __int_as_float(0x7f800000) : key2f(t32);
+          mt.qnf[i] = (float)qn;
+          mt.qn[i] = qn;
+          mt.qs[i] = TYPE == MV_IVF_SQ8 ? p.qscale[q] : 1.0f;
+          mt.qa[i] = TYPE == MV_IVF_SQ8 ? p.qa[q] : 0.0;
+          mt.base[i] = p.poff[pr];
+        } else {  // padding column: no comparison passes
+          mt.thf[i] = __int_as_float(0x7fffffff);
+          mt.qnf[i] = 0.f;
+          mt.qn[i] = 0.0;
+          mt.qs[i] = 0.f;
+          mt.qa[i] = 0.0;
+        }
       }
       named_bar(2, 64);
       uint8_t* Qb = Qs + b * p.q_bytes;
@@ -234,7 +272,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
         rest /= nchunks;
         const int pl = rest % P;
         const int i = rest / P;
-        const int q = mp[i] / p.npb;
+        const int q = mt.pair[i] / p.npb;
         const int64_t prow = TYPE == MV_IVF_FLAT ? (int64_t)pl * p.nq + q : (int64_t)q * P + pl;
         cp_async16(Qb + c * N * ATOM + swz_off(pl * NQ + i, pc, ATOM), p.qplanes + prow * rowbytes + c * ATOM + pc * 16);
       }
@@ -249,46 +287,27 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
     const int half = ew >> 2;           // which 16-column chunks of the accumulator it reads
     const int row = quarter * 32 + lane;
     const int et = threadIdx.x - 128;   // 0..255
-    uint64_t* wscr = scratch + ew * 32;
+    const uint32_t ltmask = (1u << lane) - 1;
     uint32_t titer = 0, wcount = 0;
-    for (int w = blockIdx.x; w < nwork; w += gridDim.x, ++wcount) {
+    for (int w = w0; w < nwork; w += gridDim.x, ++wcount) {
       const WorkInfo wi = work_info(p, w);
       const int NQ = (wi.nqc + 15) & ~15;
       const uint32_t b = wcount & 1;
       mbar_wait(&full_q[b], (wcount >> 1) & 1);
-      const int32_t* mp = m_pair(b);
-      const double* qn = m_qn(b);
-      const float* qs = m_qs(b);
-      const double* qa = m_qa(b);
-      const uint64_t* lim = m_lim(b);
-      const bool sel = (k <= kLocalSelectMaxK) && (wi.len > k);
-      if (sel) {
-        for (int i = et; i < wi.nqc * k; i += 32 * kEpiWarps) lists[i] = MV_KEY_PAD;
-        if (k <= 32)
-          for (int i = et; i < wi.nqc; i += 32 * kEpiWarps) {
-            cnb[i] = 0;
-            cbnd[i] = 0xffffffffu;
-          }
-      } else {
-        for (int i = et; i < wi.nqc; i += 32 * kEpiWarps) ecnt[i] = 0;
-      }
-      named_bar(1, 32 * kEpiWarps);
+      const Meta mt = meta_at(metab + b * p.meta_bytes, QCP);
       for (int t = 0; t < wi.ntiles; ++t, ++titer) {
         const uint32_t a = titer & 1;
         const uint32_t ts = titer % kNTS;
         const int vrow = t * 128 + row;
         const int row0 = (int)(wi.lstart + t * 128);
-        // refresh the global per-query threshold tau once per tile (other work items of the same
-        // query keep tightening it); the load latency overlaps the wait for the accumulator
-        uint64_t tau_now = MV_KEY_PAD;
-        if (et < wi.nqc) tau_now = *reinterpret_cast<volatile const uint64_t*>(p.tau + mp[et] / p.npb);
         mbar_wait(&full_t[ts], (titer / kNTS) & 1);
         const uint8_t* sd = side + ts * kSideBytes;
-        const uint32_t* srank = reinterpret_cast<const uint32_t*>(sd + kSideRank) + (row0 & 3);
+        const uint32_t rk = reinterpret_cast<const uint32_t*>(sd + kSideRank)[(row0 & 3) + row];
         bool valid = vrow < wi.len;
         if (valid && use_ids)
           valid = !bit_excluded(p.bitset, p.nbits, reinterpret_cast<const int64_t*>(sd + kSideIds)[(row0 & 1) + row]);
         const double xn = use_norms ? reinterpret_cast<const double*>(sd)[(row0 & 1) + row] : 0.0;
+        const float xnf = (float)xn;
         mbar_wait(&tfull[a], (titer >> 1) & 1);
         if (et == 0) MV_TRACE(6, titer);
         tc_fence_after();
@@ -298,142 +317,69 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
 #pragma unroll
           for (int pl = 0; pl < P; ++pl) tmem_ld16(tbase + pl * NQ + qc, r[pl]);
           tmem_wait_ld();
+          float bad[16];
+          uint32_t pm = 0;
 #pragma unroll
           for (int j = 0; j < 16; ++j) {
             const int i = qc + j;
-            if (i < wi.nqc) {
-              float dist;
-              if (TYPE == MV_IVF_FLAT) {
-                // exact for tf32-representable data (the only FLAT data this path accepts)
-                const float dot = __uint_as_float(r[0][j]) + __uint_as_float(r[1 % P][j]);
-                dist = use_norms ? ((float)qn[i] + (float)xn) - 2.0f * dot : dot;
-              } else {
-                // int32-exact digit partials; the L2 expansion is combined in fp64 (the norms are
-                // ~400x the near-neighbour distances on SIFT-scale data)
-                const double acc = (double)(int)r[0][j] + (double)(int)r[1 % P][j] * (1.0 / 128.0) +
-                                   (double)(int)r[2 % P][j] * (1.0 / 16384.0) +
-                                   (double)(int)r[3 % P][j] * (1.0 / 2097152.0);
-                const double dot = fma((double)qs[i], acc, qa[i]);
-                dist = use_norms ? (float)((qn[i] + xn) - 2.0 * dot) : (float)dot;
+            // badness = L2 distance or -IP (smaller is better)
+            if (TYPE == MV_IVF_FLAT) {
+              // exact for tf32-representable data (the only FLAT data this path accepts)
+              const float dot = __uint_as_float(r[0][j]) + __uint_as_float(r[1 % P][j]);
+              bad[j] = use_norms ? (mt.qnf[i] + xnf) - 2.0f * dot : -dot;
+            } else {
+              // int32-exact digit partials; the L2 expansion is combined in fp64 (the norms are
+              // ~400x the near-neighbour distances on SIFT-scale data)
+              const double acc = (double)(int)r[0][j] + (double)(int)r[1 % P][j] * (1.0 / 128.0) +
+                                 (double)(int)r[2 % P][j] * (1.0 / 16384.0) +
+                                 (double)(int)r[3 % P][j] * (1.0 / 2097152.0);
+              const double dot = fma((double)mt.qs[i], acc, mt.qa[i]);
+              bad[j] = use_norms ? (float)((mt.qn[i] + xn) - 2.0 * dot) : (float)(-dot);
+            }
+            if (bad[j] <= mt.thf[i]) {
+              // exact test on the full key (distance key, id rank) < tau
+              const uint64_t key = ((uint64_t)f2key(bad[j]) << 32) | rk;
+              if (!phaseB || key < mt.tau[i]) pm |= 1u << j;
+            }
+          }
+          if (!valid) pm = 0;
+          if (__any_sync(MV_FULL, pm != 0) && !(p.dbg & 1)) {
+            // ballot per column; lane j reserves column j's slots with one shared atomic
+            uint32_t mj[16];
+            int mine = 0;
+#pragma unroll
+            for (int j = 0; j < 16; ++j) {
+              mj[j] = __ballot_sync(MV_FULL, (pm >> j) & 1);
+              if (lane == j) mine = __popc(mj[j]);
+            }
+            int pos = 0;
+            if (mine) pos = atomicAdd(mt.cnt + qc + lane, mine);
+#pragma unroll
+            for (int j = 0; j < 16; ++j) {
+              if (mj[j]) {
+                const int pj = __shfl_sync(MV_FULL, pos, j);
+                if ((pm >> j) & 1)
+                  p.part[mt.base[qc + j] + pj + __popc(mj[j] & ltmask)] = ((uint64_t)f2key(bad[j]) << 32) | rk;
               }
-              Dt[i * kDLD + row] = valid ? dist_key(dist, p.metric) : 0xffffffffu;
             }
           }
         }
-        if (et < wi.nqc && tau_now < lim[et]) const_cast<uint64_t*>(lim)[et] = tau_now;
-        if (et == 0) *selctr = 0;
         tc_fence_before();
         if (et == 0) MV_TRACE(4, titer);
         __syncwarp();
-        if (lane == 0) mbar_arrive(&tempty[a]);
-        named_bar(1, 32 * kEpiWarps);
-        if (et == 0) MV_TRACE(5, titer);
-        // ---- a6: filter against min(list k-th, running bound, global tau) + select (warp per query)
-        if (sel && k <= 32) {
-          constexpr int G = 4;
-          // query slots are handed out G at a time through a shared counter, so a warp stuck in a
-          // warm-up or flush does not hold the others at the end-of-tile barrier
-          for (;;) {
-            int i0 = 0;
-            if (lane == 0) i0 = atomicAdd(selctr, G);
-            i0 = __shfl_sync(MV_FULL, i0, 0);
-            if (i0 >= ((p.dbg & 1) ? 0 : wi.nqc)) break;
-            const int nvalid = min(G, wi.nqc - i0);
-            warp_filter_group<G>(
-                nvalid, k, [&](int g, int m) { return Dt[(i0 + g) * kDLD + m * 32 + lane]; },
-                [&](int g, uint64_t*& L, uint64_t*& B, int*& nb, uint32_t*& bnd, uint64_t& li) {
-                  const int i = i0 + g;
-                  L = lists + (int64_t)i * k;
-                  B = cbuf + i * 32;
-                  nb = cnb + i;
-                  bnd = cbnd + i;
-                  li = lim[i];
-                },
-                [&](int, int v) { return srank[v]; },
-                [&](int g, uint32_t t32) {
-                  atomicMin(reinterpret_cast<unsigned long long*>(p.tau + mp[i0 + g] / p.npb),
-                            ((unsigned long long)t32 << 32) | 0xffffffffull);
-                },
-                wscr, (p.prof && (p.dbg & 64)) ? p.prof + 8 * 1024 + 1000 : nullptr, !(p.dbg & 32));
-          }
-        } else {
-          for (int i = ew; i < ((p.dbg & 1) ? 0 : wi.nqc); i += kEpiWarps) {
-            const int pr = mp[i];
-            const uint64_t li = lim[i];
-            uint32_t k32[4];
-#pragma unroll
-            for (int m = 0; m < 4; ++m) k32[m] = Dt[i * kDLD + m * 32 + lane];
-            if (!sel) {
-#pragma unroll
-              for (int m = 0; m < 4; ++m) {
-                const uint64_t key = ((uint64_t)k32[m] << 32) | srank[m * 32 + lane];
-                const bool pass = k32[m] != 0xffffffffu && key < li;
-                const uint32_t msk = __ballot_sync(MV_FULL, pass);
-                const int base = ecnt[i];
-                if (pass) p.part[p.poff[pr] + base + __popc(msk & ((1u << lane) - 1))] = key;
-                __syncwarp();
-                if (lane == 0) ecnt[i] = base + __popc(msk);
-                __syncwarp();
-              }
-              continue;
-            }
-            warp_select_tile(lists + (int64_t)i * k, k, li, k32, [&](int v) { return srank[v]; }, wscr);
-          }
-        }
-        named_bar(1, 32 * kEpiWarps);
-        if (et == 0) MV_TRACE(7, titer);
-        if (lane == 0) mbar_arrive(&empty_t[ts]);
-      }
-      // ---- finalize this work item's (query, list) partial results
-      for (int i = ew; i < wi.nqc; i += kEpiWarps) {
-        const int pr = mp[i];
-        if (sel && k <= 32) {
-          // the sorted list (<= k) followed by the unsorted survivor buffer (<= 32): the final select
-          // merges them exactly, so no end-of-pair sort is needed
-          const uint64_t* L = lists + (int64_t)i * k;
-          const uint64_t v = lane < k ? L[lane] : MV_KEY_PAD;
-          const uint32_t lm = __ballot_sync(MV_FULL, v != MV_KEY_PAD);
-          const int nl = __popc(lm), n = cnb[i];
-          if (v != MV_KEY_PAD) p.part[p.poff[pr] + __popc(lm & ((1u << lane) - 1))] = v;
-          if (lane < n) p.part[p.poff[pr] + nl + lane] = cbuf[i * 32 + lane];
-          if (lane == 0) {
-            p.pcnt[pr] = nl + n;
-            if (L[k - 1] != MV_KEY_PAD)
-              atomicMin(reinterpret_cast<unsigned long long*>(p.tau + pr / p.npb), (unsigned long long)L[k - 1]);
-          }
-        } else if (sel) {
-          const uint64_t* L = lists + (int64_t)i * k;
-          int c = 0;
-          for (int j0 = 0; j0 < k; j0 += 32) {
-            const int j = j0 + lane;
-            const uint64_t v = j < k ? L[j] : MV_KEY_PAD;
-            if (v != MV_KEY_PAD) p.part[p.poff[pr] + j] = v;
-            c += __popc(__ballot_sync(MV_FULL, v != MV_KEY_PAD));
-          }
-          if (lane == 0) {
-            p.pcnt[pr] = c;
-            if (L[k - 1] != MV_KEY_PAD)
-              atomicMin(reinterpret_cast<unsigned long long*>(p.tau + pr / p.npb), (unsigned long long)L[k - 1]);
-          }
-        } else if (lane == 0) {
-          p.pcnt[pr] = ecnt[i];
+        if (lane == 0) {
+          mbar_arrive(&tempty[a]);
+          mbar_arrive(&empty_t[ts]);
         }
       }
+      // every epilogue warp is done with this work item: publish the pairs' counts, free the metadata
+      named_bar(1, 32 * kEpiWarps);
+      for (int i = et; i < wi.nqc; i += 32 * kEpiWarps) p.pcnt[mt.pair[i]] = mt.cnt[i];
       __syncwarp();
       if (lane == 0) mbar_arrive(&empty_m[b]);
-      named_bar(1, 32 * kEpiWarps);
     }
   }
   __syncthreads();
-  if (p.prof && threadIdx.x == 0) {  // per-CTA start / end (ns) in rows 8.. of the debug buffer
-    unsigned long long gt1;
-    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(gt1));
-    int ntl = 0;
-    for (int w = blockIdx.x; w < nwork; w += gridDim.x) ntl += work_info(p, w).ntiles;
-    p.prof[8 * 1024 + blockIdx.x * 3 + 0] = gt0;
-    p.prof[8 * 1024 + blockIdx.x * 3 + 1] = gt1;
-    p.prof[8 * 1024 + blockIdx.x * 3 + 2] = ntl;
-  }
   if (warp == 1) {
     tc_fence_after();
     tmem_dealloc(tmem, p.tmem_cols);
@@ -517,17 +463,16 @@ cudaError_t launch_tf32_check(const float* x, int64_t n, int* flag, cudaStream_t
 }
 
 // ----------------------------------------------------------------------------------------------
-bool tc_scan_plan(int type, int dpad, int k, TcScanParams& p) {
+// Shared-memory plan: X ring + double-buffered query planes + double-buffered per-query metadata
+// + the side-data ring; the deepest X ring (<= the type's cap) that fits in 227 KB.
+static bool tc_scan_layout(int type, int dpad, int qc, int ns, TcScanParams& p) {
   const int esz = type == MV_IVF_FLAT ? 4 : 1;
   const int atom = type == MV_IVF_FLAT ? 128 : 32;
   const int P = type == MV_IVF_FLAT ? 2 : 4;
-  const int qcmax = type == MV_IVF_FLAT ? 48 : 64;
+  auto up = [](int x, int a) { return (x + a - 1) / a * a; };
   p.type = type;
   p.dpad = dpad;
-  p.k = k;
   p.nchunks = dpad * esz / atom;
-  int qc = qcmax;
-  if (k <= kLocalSelectMaxK) qc = std::max(1, std::min(qcmax, 53248 / (8 * k)));
   p.qchunk = qc;
   const int qcp = (qc + 15) & ~15;
   p.ncol = P * qcp;
@@ -535,32 +480,28 @@ bool tc_scan_plan(int type, int dpad, int k, TcScanParams& p) {
   while (cols < 2 * p.ncol) cols <<= 1;
   if (cols > 512) return false;
   p.tmem_cols = cols;
-  auto up = [](int x, int a) { return (x + a - 1) / a * a; };
   p.q_bytes = up(P * qcp * dpad * esz, 1024);
-  const int dt_bytes = qc * 129 * 4;
-  const int lists_bytes = k <= kLocalSelectMaxK ? qc * k * 8 : 0;
-  p.meta_lim_off = up(8 * qc, 8);
-  p.meta_bytes = up(p.meta_lim_off + 24 * qc, 16);
-  const int misc_bytes = 256 + 32 * 8 * kEpiWarps + (k <= 32 ? qc * (32 * 8 + 8) : 0);
-  const int side_bytes = kNTS * kSideBytes;
+  p.meta_bytes = up(kMetaPerQuery * qcp, 16);
   const int stage = 128 * atom;
-  const int fixed = 2 * p.q_bytes + up(dt_bytes, 16) + up(lists_bytes, 16) + 2 * p.meta_bytes + misc_bytes + side_bytes;
-  const int budget = 227 * 1024 - 1024 - 512;  // alignment slack + barriers
-  int ns = (budget - fixed) / stage;
-  ns = std::min(ns, type == MV_IVF_FLAT ? 8 : 24);
-  if (ns < 2) return false;
   p.nstage = ns;
   p.off_x = 0;
   p.off_q = ns * stage;
-  p.off_dt = p.off_q + 2 * p.q_bytes;
-  p.off_lists = p.off_dt + up(dt_bytes, 16);
-  p.off_meta = p.off_lists + up(lists_bytes, 16);
-  p.off_misc = p.off_meta + 2 * p.meta_bytes;
-  p.off_ctr = p.off_misc + misc_bytes;
-  p.off_side = up(p.off_ctr + 16, 128);
-  p.off_bar = p.off_side + side_bytes;
-  p.smem_total = p.off_bar + (2 * ns + 10 + 2 * kNTS) * 8 + 16 + 1024;
+  p.off_meta = p.off_q + 2 * p.q_bytes;
+  p.off_side = up(p.off_meta + 2 * p.meta_bytes, 128);
+  p.off_bar = p.off_side + kNTS * kSideBytes;
+  p.smem_total = p.off_bar + (2 * ns + 10 + 2 * kNTS) * 8 + 16 + 1024;  // + 1 KB alignment slack
   return p.smem_total <= 227 * 1024;
+}
+
+bool tc_scan_plan(int type, int dpad, int k, TcScanParams& p) {
+  const int qcmax = type == MV_IVF_FLAT ? 48 : 64;
+  const int nscap = type == MV_IVF_FLAT ? 8 : 24;
+  const int nsmin = type == MV_IVF_FLAT ? 3 : 6;  // >= 48 KB (FLAT) / 24 KB (SQ8) of list tiles in flight
+  p.k = k;
+  for (int qc = qcmax; qc >= 16; qc -= 16)
+    for (int ns = nscap; ns >= nsmin; --ns)
+      if (tc_scan_layout(type, dpad, qc, ns, p)) return true;
+  return false;
 }
 
 cudaError_t launch_scan_tc(const CUtensorMap* xmap, const TcScanParams& p, cudaStream_t st) {

@@ -28,7 +28,8 @@ __device__ __forceinline__ bool seg_locate(const int32_t* s_pre, int npb, int id
 __global__ void __launch_bounds__(256) k_final_select(const int64_t* __restrict__ poff, const int32_t* __restrict__ pcnt,
                                                       const uint64_t* __restrict__ part, int64_t nq, int npb, int k,
                                                       int metric, const int64_t* __restrict__ sorted_ids, float* out_d,
-                                                      int64_t* out_i, int selcap) {
+                                                      int64_t* out_i, int selcap, const int32_t* __restrict__ nuse,
+                                                      uint64_t* tau_out) {
   extern __shared__ __align__(16) uint8_t smem[];
   uint64_t* sel = reinterpret_cast<uint64_t*>(smem);       // selcap
   uint64_t* bnd = sel + selcap;                             // kBoundCap
@@ -41,6 +42,7 @@ __global__ void __launch_bounds__(256) k_final_select(const int64_t* __restrict_
   const int tid = threadIdx.x;
   const int64_t* po = poff + q * npb;
   const int32_t* pc = pcnt + q * npb;
+  if (nuse) npb = nuse[q];  // the first nuse[q] pairs of the query (the seeding phase's), else all
   if (tid == 0) {
     int acc = 0;
     for (int j = 0; j < npb; ++j) {
@@ -128,6 +130,10 @@ __global__ void __launch_bounds__(256) k_final_select(const int64_t* __restrict_
     nout = k;
   }
   (void)s_u64;
+  if (tau_out) {  // seeding: the k-th best key of the first nuse pairs bounds the query's top-k
+    if (tid == 0 && nout == k) tau_out[q] = sel[k - 1];
+    return;
+  }
   for (int i = tid; i < k; i += 256) {
     float dv;
     int64_t iv;
@@ -144,16 +150,104 @@ __global__ void __launch_bounds__(256) k_final_select(const int64_t* __restrict_
   }
 }
 
+// k <= 32: one warp per query.  The pairs' regions are walked in 32-key chunks (a flattened index
+// over groups of 32 pairs, located by a shuffle binary search); a chunk is skipped unless some key
+// beats the running k-th best, else it is bitonic-sorted and merged into the sorted register list.
+__global__ void __launch_bounds__(256) k_final_small(const int64_t* __restrict__ poff, const int32_t* __restrict__ pcnt,
+                                                     const uint64_t* __restrict__ part, int64_t nq, int npb, int k,
+                                                     int metric, const int64_t* __restrict__ sorted_ids, float* out_d,
+                                                     int64_t* out_i, const int32_t* __restrict__ nuse,
+                                                     uint64_t* tau_out) {
+  const int lane = threadIdx.x & 31;
+  const int64_t q = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  if (q >= nq) return;
+  const int stride = npb;
+  if (nuse) npb = nuse[q];
+  uint64_t best[1] = {MV_KEY_PAD};  // ascending: lane i holds the i-th best so far
+  for (int g = 0; g < npb; g += 32) {
+    const int j = g + lane;
+    const int cnt = j < npb ? pcnt[q * stride + j] : 0;
+    const int64_t off = j < npb ? poff[q * stride + j] : 0;
+    int incl = cnt;
+    for (int o = 1; o < 32; o <<= 1) {
+      const int v = __shfl_up_sync(MV_FULL, incl, o);
+      if (lane >= o) incl += v;
+    }
+    const int excl = incl - cnt;
+    const int T = __shfl_sync(MV_FULL, incl, 31);
+    for (int e0 = 0; e0 < T; e0 += 32) {
+      const int e = e0 + lane;
+      // pair holding element e: the largest s with excl[s] <= e
+      int lo = 0;
+#pragma unroll
+      for (int step = 16; step > 0; step >>= 1) {
+        const int ex = __shfl_sync(MV_FULL, excl, lo + step);
+        if (lo + step < 32 && ex <= e) lo += step;
+      }
+      const int64_t o = __shfl_sync(MV_FULL, off, lo);
+      const int ex = __shfl_sync(MV_FULL, excl, lo);
+      uint64_t v[1] = {e < T ? part[o + (e - ex)] : MV_KEY_PAD};
+      const uint64_t kth = shfl64(best[0], k - 1);
+      if (!(v[0] < kth)) v[0] = MV_KEY_PAD;
+      if (__any_sync(MV_FULL, v[0] != MV_KEY_PAD)) {
+        warp_bitonic_sort<1>(v);
+        warp_merge_smallest<1>(best, v);
+      }
+    }
+  }
+  if (tau_out) {  // seeding: the k-th best key of the first nuse[q] pairs bounds the query's top-k
+    const uint64_t kth = shfl64(best[0], k - 1);
+    if (lane == 0 && kth != MV_KEY_PAD) tau_out[q] = kth;
+    return;
+  }
+  if (lane < k) {
+    const uint64_t key = best[0];
+    float dv;
+    int64_t iv;
+    if (key != MV_KEY_PAD) {
+      dv = key_dist((uint32_t)(key >> 32), metric);
+      iv = sorted_ids[(uint32_t)(key & 0xffffffffu)];
+    } else {
+      dv = metric == MV_L2 ? __int_as_float(0x7f800000) : __int_as_float(0xff800000);
+      iv = -1;
+    }
+    out_d[q * k + lane] = dv;
+    out_i[q * k + lane] = iv;
+  }
+}
+
 cudaError_t launch_final_select(const int64_t* poff, const int32_t* pcnt, const uint64_t* part, int64_t nq, int npb,
                                 int k, int metric, const int64_t* sorted_ids, float* out_d, int64_t* out_i,
                                 cudaStream_t st) {
   if (nq == 0) return cudaSuccess;
+  if (k <= 32) {
+    k_final_small<<<(unsigned)((nq * 32 + 255) / 256), 256, 0, st>>>(poff, pcnt, part, nq, npb, k, metric, sorted_ids,
+                                                                     out_d, out_i, nullptr, nullptr);
+    return cudaGetLastError();
+  }
   const int selcap = max(4096, next_pow2(k));
   size_t smem = (size_t)(selcap + kBoundCap) * 8 + (size_t)(npb + 1) * 4 + 256 * 4 + 8 * 4 + 64;
   cudaError_t e = cudaFuncSetAttribute(k_final_select, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   k_final_select<<<(unsigned)nq, 256, smem, st>>>(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d, out_i,
-                                                  selcap);
+                                                  selcap, nullptr, nullptr);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_tau_select(const int64_t* poff, const int32_t* pcnt, const uint64_t* part, int64_t nq, int npb,
+                              const int32_t* nuse, int k, uint64_t* tau, cudaStream_t st) {
+  if (nq == 0) return cudaSuccess;
+  if (k <= 32) {
+    k_final_small<<<(unsigned)((nq * 32 + 255) / 256), 256, 0, st>>>(poff, pcnt, part, nq, npb, k, MV_L2, nullptr,
+                                                                     nullptr, nullptr, nuse, tau);
+    return cudaGetLastError();
+  }
+  const int selcap = max(4096, next_pow2(k));
+  size_t smem = (size_t)(selcap + kBoundCap) * 8 + (size_t)(npb + 1) * 4 + 256 * 4 + 8 * 4 + 64;
+  cudaError_t e = cudaFuncSetAttribute(k_final_select, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  k_final_select<<<(unsigned)nq, 256, smem, st>>>(poff, pcnt, part, nq, npb, k, MV_L2, nullptr, nullptr, nullptr,
+                                                  selcap, nuse, tau);
   return cudaGetLastError();
 }
 

@@ -2,11 +2,13 @@
 // search pipeline a1 -> a2/a3 -> a4 -> a5/a6 -> a7 enqueued on the caller's stream.
 #include <cub/device/device_radix_sort.cuh>
 
+#include <cmath>
 #include <cstdarg>
 #include <cstdlib>
 #include <cstdio>
 #include <cstring>
 #include <string>
+#include <functional>
 #include <vector>
 
 #include "mv_internal.cuh"
@@ -28,6 +30,7 @@ struct mv_index {
   int64_t ntotal = 0;
   int64_t* list_off = nullptr;  // nlist + 1 (device)
   std::vector<int64_t> h_list_off;
+  std::vector<int64_t> top_len_prefix;  // [j] = total length of the j longest lists (j = 0..nlist)
   int64_t maxlen = 0;
   void* payload = nullptr;      // ntotal x dpad (fp32 or u8)
   double* norms = nullptr;      // ntotal (+pad): ||x||^2 / ||x_hat||^2 in fp64
@@ -42,7 +45,7 @@ struct mv_index {
   const char* last_coarse = "none";
   // profiling
   bool prof = false;
-  std::vector<cudaEvent_t> ev;   // 5 events per profiled search
+  std::vector<cudaEvent_t> ev;   // kProfStages + 1 events per profiled search
   int64_t prof_searches = 0, launches = 0;
 };
 
@@ -212,6 +215,7 @@ mv_status mv_index_create(int32_t d, mv_metric metric, mv_type type, int32_t nli
   ix->nlist = nlist;
   ix->device = device;
   ix->h_list_off.assign(nlist + 1, 0);
+  ix->top_len_prefix.assign(nlist + 1, 0);
   cudaError_t e = cudaMalloc(&ix->list_off, sizeof(int64_t) * (nlist + 1));
   if (e == cudaSuccess) e = cudaMemset(ix->list_off, 0, sizeof(int64_t) * (nlist + 1));
   if (e == cudaSuccess) e = cudaMalloc(&ix->cpad, sizeof(float) * (size_t)nlist * ix->dpad);
@@ -433,7 +437,14 @@ mv_status mv_index_add(mv_index* ix, const float* vectors, const int64_t* ids, i
                              (uint64_t)dpad, (uint64_t)ntot, (uint64_t)dpad * esize, 32, 128,
                              ix->type == MV_IVF_FLAT ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_32B);
   ix->maxlen = 0;
-  for (int l = 0; l < nlist; ++l) ix->maxlen = std::max(ix->maxlen, ix->h_list_off[l + 1] - ix->h_list_off[l]);
+  std::vector<int64_t> lens(nlist);
+  for (int l = 0; l < nlist; ++l) {
+    lens[l] = ix->h_list_off[l + 1] - ix->h_list_off[l];
+    ix->maxlen = std::max(ix->maxlen, lens[l]);
+  }
+  std::sort(lens.begin(), lens.end(), std::greater<int64_t>());
+  ix->top_len_prefix.assign(nlist + 1, 0);
+  for (int l = 0; l < nlist; ++l) ix->top_len_prefix[l + 1] = ix->top_len_prefix[l] + lens[l];
   return MV_OK;
 }
 
@@ -529,25 +540,40 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
     const int qchunk = use_tc ? tp.qchunk
                               : (k <= kLocalSelectMaxK ? std::min(64, std::max(1, 65536 / (8 * k))) : 64);
     const int64_t npairs = nq * npb;
+    // Seeding (tensor-core path, nprobe >= 2): phase A scans each query's ra[q] nearest lists --
+    // the fewest holding >= 2k candidates -- and emits all of them; their k-th best key tau_q is an
+    // exact upper bound of the query's final k-th best, so phase B emits only keys below it.
+    const char* seed_env = getenv("MV_SEED");
+    const bool split = use_tc && npb >= 2 && !(seed_env && seed_env[0] == '0');
+    int32_t* ra = nullptr;
+    if (split) {
+      CK(s.alloc(&ra, (size_t)nq));
+      CK(launch_seed_ranks(P, nq, npb, ix->list_off, std::max<int64_t>(2 * (int64_t)k, k + 32), ra, st));
+    }
+    const int nv = split ? 2 * nlist : nlist;
     Bucketing b;
-    CK(s.alloc(&b.lcount, nlist));
-    CK(s.alloc(&b.boff, nlist + 1));
-    CK(s.alloc(&b.bfill, nlist));
+    CK(s.alloc(&b.lcount, nv));
+    CK(s.alloc(&b.boff, nv + 1));
+    CK(s.alloc(&b.bfill, nv));
     CK(s.alloc(&b.bq, (size_t)npairs));
-    CK(s.alloc(&b.wcount, nlist));
-    CK(s.alloc(&b.woff, nlist + 1));
-    CK(s.alloc(&b.witems, (size_t)(nlist + npairs / qchunk + 1)));
-    CK(s.alloc(&b.witems_unsorted, (size_t)(nlist + npairs / qchunk + 1)));
+    CK(s.alloc(&b.wcount, nv));
+    CK(s.alloc(&b.woff, nv + 1));
+    CK(s.alloc(&b.witems, (size_t)(nv + npairs / qchunk + 1)));
+    CK(s.alloc(&b.witems_unsorted, (size_t)(nv + npairs / qchunk + 1)));
     CK(s.alloc(&b.qtot, (size_t)(2 * (nq + 1))));
     CK(s.alloc(&b.poff, (size_t)npairs));
     CK(s.alloc(&b.pcnt, (size_t)npairs));
     CK(s.alloc(&b.counter, 1));
-    CK(launch_bucket(P, nq, npb, nlist, ix->list_off, k, qchunk, b, st));
-    const int capk = (use_tc && k <= 32) ? k + 32 : k;  // tensor-core scan: sorted list + 32-entry buffer per pair
+    CK(launch_bucket(P, nq, npb, nlist, ix->list_off, k, qchunk, ra, b, st));
+    // pair regions: the whole list (tensor-core scan: emit-all bound), or min(k, |list|) (SIMT)
+    const int capk = use_tc ? 0 : k;
     CK(launch_pair_offsets(P, nq, npb, ix->list_off, k, capk, b, st));
     prof_mark(ix, st);
     int64_t cap;
-    if (k <= kLocalSelectMaxK) {
+    if (use_tc) {
+      // exact worst case without a device round trip: nq x (the npb longest lists)
+      cap = nq * ix->top_len_prefix[std::min<size_t>(npb, ix->top_len_prefix.size() - 1)];
+    } else if (k <= kLocalSelectMaxK) {
       cap = nq * npb * min64(capk, max64(ix->maxlen, 1));
     } else {
       CK(cudaMemcpyAsync(&cap, b.qtot + (nq + 1) + nq, sizeof(int64_t), cudaMemcpyDeviceToHost, st));
@@ -580,7 +606,7 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
       tp.list_off = ix->list_off; tp.norms = ix->norms; tp.ids = ix->ids; tp.rank = ix->rank;
       tp.bitset = bs; tp.nbits = bs ? nbits : 0;
       tp.qplanes = qplanes; tp.qnorm = qn64; tp.qscale = qscale; tp.qa = qa;
-      tp.bq = b.bq; tp.boff = b.boff; tp.witems = b.witems; tp.nwitems = b.woff + nlist;
+      tp.bq = b.bq; tp.boff = b.boff; tp.witems = b.witems; tp.nlist = nlist;
       tp.poff = b.poff; tp.pcnt = b.pcnt; tp.part = part; tp.tau = tau;
       const char* dbg = getenv("MV_SCAN_DEBUG");
       tp.dbg = dbg ? atoi(dbg) : 0;
@@ -590,7 +616,24 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
         CK(s.alloc(&tp.prof, (size_t)9 * 1024));
         CK(cudaMemsetAsync(tp.prof, 0, 9 * 1024 * 8, st));
       }
+      // phase A (or, without seeding, the whole scan emitting every candidate) ...
+      tp.phase = 0;
+      tp.wbeg = nullptr;
+      tp.nwitems = b.woff + nlist;
       CK(launch_scan_tc(&ix->xmap, tp, st));
+      prof_mark(ix, st);
+      if (split) {
+        // ... tau_q = k-th best key of phase A ...
+        CK(launch_tau_select(b.poff, b.pcnt, part, nq, npb, ra, k, tau, st));
+        prof_mark(ix, st);
+        // ... phase B over the remaining pairs, emitting keys < tau_q
+        tp.phase = 1;
+        tp.wbeg = b.woff + nlist;
+        tp.nwitems = b.woff + 2 * nlist;
+        CK(launch_scan_tc(&ix->xmap, tp, st));
+      } else {
+        prof_mark(ix, st);
+      }
       if (tp.prof) {  // debug timeline of CTA 0 (MV_SCAN_TRACE=1): rows = events, cycles since the first TMA issue
         std::vector<unsigned long long> h(9 * 1024);
         CK(cudaMemcpyAsync(h.data(), tp.prof, h.size() * 8, cudaMemcpyDeviceToHost, st));
@@ -606,8 +649,10 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
         }
         unsigned long long gmin = ~0ull;
         for (int b = 0; b < 148; ++b) gmin = std::min(gmin, h[8 * 1024 + b * 3]);
-        fprintf(stderr, "[events] tiles_with_survivors %llu warmups %llu flushes %llu fallbacks %llu survivors %llu\n",
-                h[8 * 1024 + 1000], h[8 * 1024 + 1001], h[8 * 1024 + 1002], h[8 * 1024 + 1003], h[8 * 1024 + 1004]);
+        fprintf(stderr, "[events] tiles_with_survivors %llu warmups %llu flushes %llu fallbacks %llu survivors %llu "
+                "folds %llu fold_survivors %llu\n",
+                h[8 * 1024 + 1000], h[8 * 1024 + 1001], h[8 * 1024 + 1002], h[8 * 1024 + 1003], h[8 * 1024 + 1004],
+                h[8 * 1024 + 1005], h[8 * 1024 + 1006]);
         fprintf(stderr, "[cta] start_us end_us tiles:");
         for (int b = 0; b < 148; ++b)
           fprintf(stderr, " %d:%.1f/%.1f/%llu", b, (h[8 * 1024 + b * 3] - gmin) / 1e3, (h[8 * 1024 + b * 3 + 1] - gmin) / 1e3,
@@ -615,7 +660,7 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
         fprintf(stderr, "\n");
       }
       ix->last_scan = ix->type == MV_IVF_FLAT ? "tcgen05.tf32" : "tcgen05.i8";
-      ix->launches += 1;
+      ix->launches += split ? 5 : 2;  // qplanes, scan A (+ seed ranks, tau select, scan B)
     } else {
     ScanArgs a;
     a.type = ix->type; a.metric = ix->metric; a.d = ix->d; a.dpad = dpad; a.k = k; a.npb = npb;
@@ -626,6 +671,8 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
     a.bq = b.bq; a.boff = b.boff; a.witems = b.witems; a.nwitems = b.woff + nlist; a.counter = b.counter;
     a.poff = b.poff; a.pcnt = b.pcnt; a.part = part;
     CK(launch_scan(a, st));
+    prof_mark(ix, st);
+    prof_mark(ix, st);
     ix->last_scan = "simt";
     }
     prof_mark(ix, st);
@@ -633,7 +680,8 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
     CK(launch_final_select(b.poff, b.pcnt, part, nq, npb, k, ix->metric, ix->sorted_ids, D, I, st));
     prof_mark(ix, st);
     if (ix->prof) ix->prof_searches++;
-    ix->launches += 14;  // prep, coarse, 7 bucketing, 3 offsets, scan, select
+    ix->launches += 14;  // prep, hilo, coarse, 7 bucketing, 3 offsets, final select (+ SIMT scan below)
+    if (!use_tc) ix->launches += 1;
   }
   if (host_out) {
     CK(cudaMemcpyAsync(distances, D, sizeof(float) * nq * k, cudaMemcpyDeviceToHost, st));
@@ -709,17 +757,18 @@ mv_status mv_profile_enable(mv_index* ix, int on) {
 mv_status mv_profile_read(mv_index* ix, double* ms, int64_t* searches, int64_t* launches, int reset) {
   if (!ix) return fail(MV_EINVAL, "null index");
   DeviceGuard g(ix->device);
-  double acc[4] = {0, 0, 0, 0};
-  for (size_t i = 0; i + 5 <= ix->ev.size(); i += 5) {
-    CK(cudaEventSynchronize(ix->ev[i + 4]));
-    for (int s = 0; s < 4; ++s) {
+  constexpr int NS = kProfStages;
+  double acc[NS] = {0};
+  for (size_t i = 0; i + NS + 1 <= ix->ev.size(); i += NS + 1) {
+    CK(cudaEventSynchronize(ix->ev[i + NS]));
+    for (int s = 0; s < NS; ++s) {
       float t = 0.f;
       CK(cudaEventElapsedTime(&t, ix->ev[i + s], ix->ev[i + s + 1]));
       acc[s] += t;
     }
   }
   if (ms)
-    for (int s = 0; s < 4; ++s) ms[s] = acc[s];
+    for (int s = 0; s < NS; ++s) ms[s] = acc[s];
   if (searches) *searches = ix->prof_searches;
   if (launches) *launches = ix->launches;
   if (reset) {

@@ -17,6 +17,7 @@ namespace mv {
 constexpr int kMaxK = 16384;          // PAPER.md:801-802 (§3.3 fn. 5): k <= 16384
 constexpr int kLocalSelectMaxK = 1024;  // per-(query,list) selection in the scan for k <= 1024
 constexpr int kNumSMs = 148;
+constexpr int kProfStages = 6;   // coarse, bucket, scan A, seed select, scan B, final select (mv.h)
 
 __host__ __device__ __forceinline__ int64_t min64(int64_t a, int64_t b) { return a < b ? a : b; }
 __host__ __device__ __forceinline__ int64_t max64(int64_t a, int64_t b) { return a > b ? a : b; }
@@ -479,8 +480,15 @@ struct Bucketing {
   int32_t* pcnt;     // nq*npb     candidates written per pair
   int32_t* counter;  // 1          persistent scan work counter
 };
+// ra != nullptr: the pairs of query q with probe rank < ra[q] form a first phase (virtual lists
+// 0..nlist-1, work items first) and the others a second (virtual lists nlist..2*nlist-1); arrays
+// are then sized for 2*nlist lists.
 cudaError_t launch_bucket(const int32_t* probes, int64_t nq, int npb, int nlist, const int64_t* list_off, int k,
-                          int qchunk, const Bucketing& b, cudaStream_t st);
+                          int qchunk, const int32_t* ra, const Bucketing& b, cudaStream_t st);
+// ra[q] = the fewest nearest lists of q holding >= need candidates (<= npb)
+cudaError_t launch_seed_ranks(const int32_t* probes, int64_t nq, int npb, const int64_t* list_off, int64_t need,
+                              int32_t* ra, cudaStream_t st);
+// capk > 0: region of a pair = min(capk, |list|) (SIMT local selection); capk = 0: |list|
 cudaError_t launch_pair_offsets(const int32_t* probes, int64_t nq, int npb, const int64_t* list_off, int k, int capk,
                                 const Bucketing& b, cudaStream_t st);
 cudaError_t launch_scan_i32(const int32_t* in, int n, int32_t* out, cudaStream_t st);   // out[n+1]
@@ -512,12 +520,13 @@ struct ScanArgs {
 };
 cudaError_t launch_scan(const ScanArgs& a, cudaStream_t st);
 
-// k_scan_tc.cu (tcgen05 path)
+// k_scan_tc.cu (tcgen05 path): a filter-and-emit scan run in two phases
 struct TcScanParams {
   int type, metric, dpad, k, npb, qchunk, nchunks, nstage, ncol, tmem_cols;
+  int nlist;               // virtual list v >= nlist is list v - nlist (phase-B pairs)
+  int phase;               // 0: seeding phase A (emit every candidate); 1: phase B (emit keys < tau_q)
   int64_t nq;              // FLAT query planes are plane-major [2][nq][dpad]
-  int off_x, off_q, q_bytes, off_dt, off_lists, off_meta, meta_bytes, meta_lim_off, off_misc, off_side, off_bar,
-      off_ctr, smem_total;
+  int off_x, off_q, q_bytes, off_meta, meta_bytes, off_side, off_bar, smem_total;
   const int64_t* list_off;
   const double* norms;     // ||x||^2 (FLAT) or ||x_hat||^2 (SQ8), fp64
   const int64_t* ids;
@@ -531,13 +540,14 @@ struct TcScanParams {
   const int32_t* bq;
   const int32_t* boff;
   const int2* witems;
-  const int32_t* nwitems;
-  const int64_t* poff;
-  int32_t* pcnt;
+  const int32_t* wbeg;     // device: first work item of this launch (nullable = 0)
+  const int32_t* nwitems;  // device: one past the last work item of this launch
+  const int64_t* poff;     // per pair: output region (capacity = the list length)
+  int32_t* pcnt;           // per pair: keys emitted
   uint64_t* part;
-  uint64_t* tau;           // nq: global per-query threshold (u64 key), atomicMin-updated
-  int dbg;                 // debug bitmask (MV_SCAN_DEBUG): 1 skip select, 2 skip epilogue math, 4 skip Q copy
-  unsigned long long* prof;  // unused (reserved for wait-cycle accounting)
+  const uint64_t* tau;     // nq: per-query bound for phase B (exact k-th key of phase A)
+  int dbg;                 // debug bitmask (MV_SCAN_DEBUG): 1 skip emission, 2 skip epilogue math, 4 skip Q copy
+  unsigned long long* prof;  // MV_SCAN_TRACE timeline (CTA 0)
 };
 bool tc_scan_plan(int type, int dpad, int k, TcScanParams& p);
 cudaError_t launch_scan_tc(const CUtensorMap* xmap, const TcScanParams& p, cudaStream_t st);
@@ -559,9 +569,13 @@ cudaError_t launch_coarse_tc(const CUtensorMap* cmap, const CUtensorMap* qmap, c
 cudaError_t launch_hilo(const float* x, int64_t n, int d, int dpad, float* out, cudaStream_t st);
 
 // k_select.cu
+// final select over the pairs of each query; with tau != nullptr instead: tau[q] = the k-th best
+// key over the first nuse[q] pairs of query q (left untouched when they hold fewer than k)
 cudaError_t launch_final_select(const int64_t* poff, const int32_t* pcnt, const uint64_t* part, int64_t nq, int npb,
                                 int k, int metric, const int64_t* sorted_ids, float* out_d, int64_t* out_i,
                                 cudaStream_t st);
+cudaError_t launch_tau_select(const int64_t* poff, const int32_t* pcnt, const uint64_t* part, int64_t nq, int npb,
+                              const int32_t* nuse, int k, uint64_t* tau, cudaStream_t st);
 cudaError_t launch_fill_pad(int64_t n, int metric, float* d, int64_t* i, cudaStream_t st);
 cudaError_t launch_merge2(int metric, const float* ad, const int64_t* ai, const float* bd, const int64_t* bi,
                           int64_t nq, int k, float* od, int64_t* oi, cudaStream_t st);

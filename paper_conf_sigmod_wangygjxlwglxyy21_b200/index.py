@@ -135,7 +135,7 @@ class Index:
         return P
 
     # -- measurement ---------------------------------------------------------------------------
-    STAGES = ("coarse", "bucket", "scan", "select")
+    STAGES = ("coarse", "bucket", "scan_a", "seed", "scan", "select")
 
     def profile(self, on: bool = True):
         L.check(self._lib.mv_profile_enable(self._h, int(bool(on))))
@@ -143,7 +143,7 @@ class Index:
     def profile_read(self, reset: bool = True):
         """Summed CUDA-event milliseconds per stage since the last reset, the number of profiled
         searches and the number of libmv kernel launches."""
-        ms = (C.c_double * 4)()
+        ms = (C.c_double * len(self.STAGES))()
         ns, nl = C.c_int64(), C.c_int64()
         L.check(self._lib.mv_profile_read(self._h, ms, C.byref(ns), C.byref(nl), int(reset)))
         return dict(zip(self.STAGES, list(ms))), int(ns.value), int(nl.value)
