@@ -98,6 +98,19 @@ __global__ void k_seed_ranks(const int32_t* __restrict__ probes, int64_t nq, int
   }
 }
 
+// qcfg = {query chunk, query planes}: the split (two-plane) shape when *qlo_any, else the exact one
+__global__ void k_scan_cfg(const int* qlo_any, int qc_exact, int p_exact, int qc_split, int p_split, int32_t* qcfg) {
+  const bool sp = qlo_any != nullptr && *qlo_any != 0;
+  qcfg[0] = sp ? qc_split : qc_exact;
+  qcfg[1] = sp ? p_split : p_exact;
+}
+
+cudaError_t launch_scan_cfg(const int* qlo_any, int qc_exact, int p_exact, int qc_split, int p_split, int32_t* qcfg,
+                            cudaStream_t st) {
+  k_scan_cfg<<<1, 1, 0, st>>>(qlo_any, qc_exact, p_exact, qc_split, p_split, qcfg);
+  return cudaGetLastError();
+}
+
 cudaError_t launch_seed_ranks(const int32_t* probes, int64_t nq, int npb, const int64_t* list_off, int64_t need,
                               int32_t* ra, cudaStream_t st) {
   if (nq == 0) return cudaSuccess;
@@ -106,14 +119,18 @@ cudaError_t launch_seed_ranks(const int32_t* probes, int64_t nq, int npb, const 
   return cudaGetLastError();
 }
 
-__global__ void k_work_count(const int32_t* __restrict__ lcount, int nlist, int qchunk, int32_t* wcount) {
+__global__ void k_work_count(const int32_t* __restrict__ lcount, int nlist, const int32_t* __restrict__ qcfg,
+                             int32_t* wcount) {
   const int l = blockIdx.x * blockDim.x + threadIdx.x;
+  const int qchunk = qcfg[0];
   if (l < nlist) wcount[l] = (lcount[l] + qchunk - 1) / qchunk;
 }
 
 __global__ void k_work_fill(const int32_t* __restrict__ wcount, const int32_t* __restrict__ woff,
-                            const int32_t* __restrict__ boff, int nlist, int qchunk, int2* witems) {
+                            const int32_t* __restrict__ boff, int nlist, const int32_t* __restrict__ qcfg,
+                            int2* witems) {
   const int l = blockIdx.x * blockDim.x + threadIdx.x;
+  const int qchunk = qcfg[0];
   if (l >= nlist) return;
   const int n = wcount[l], o = woff[l], b = boff[l];
   for (int c = 0; c < n; ++c) witems[o + c] = make_int2(l, b + c * qchunk);
@@ -124,8 +141,10 @@ __global__ void k_work_fill(const int32_t* __restrict__ wcount, const int32_t* _
 // the seeding split, every phase-A item (virtual list < nlist) precedes every phase-B item.
 __global__ void __launch_bounds__(1024) k_sort_work(const int2* __restrict__ in, const int32_t* __restrict__ nwork_p,
                                                     const int32_t* __restrict__ boff, const int64_t* __restrict__ list_off,
-                                                    int nlist, int qchunk, int2* __restrict__ out) {
+                                                    int nlist, const int32_t* __restrict__ qcfg,
+                                                    int2* __restrict__ out) {
   constexpr int NB = 8192, HB = 4096;
+  const int qchunk = qcfg[0];
   __shared__ int hist[NB];
   __shared__ int part[1024];
   const int nwork = *nwork_p, tid = threadIdx.x;
@@ -165,7 +184,7 @@ __global__ void __launch_bounds__(1024) k_sort_work(const int2* __restrict__ in,
 }
 
 cudaError_t launch_bucket(const int32_t* probes, int64_t nq, int npb, int nlist, const int64_t* list_off, int k,
-                          int qchunk, const int32_t* ra, const Bucketing& b, cudaStream_t st) {
+                          const int32_t* qcfg, const int32_t* ra, const Bucketing& b, cudaStream_t st) {
   (void)k;
   const int64_t npairs = nq * npb;
   const int nv = ra ? 2 * nlist : nlist;  // virtual lists
@@ -177,10 +196,10 @@ cudaError_t launch_bucket(const int32_t* probes, int64_t nq, int npb, int nlist,
   cudaError_t e;
   if ((e = launch_scan_i32(b.lcount, nv, b.boff, st)) != cudaSuccess) return e;
   if (npairs) k_bucket_fill<<<grid, 256, 0, st>>>(probes, npairs, npb, nlist, ra, b.boff, b.bfill, b.bq);
-  k_work_count<<<(nv + 255) / 256, 256, 0, st>>>(b.lcount, nv, qchunk, b.wcount);
+  k_work_count<<<(nv + 255) / 256, 256, 0, st>>>(b.lcount, nv, qcfg, b.wcount);
   if ((e = launch_scan_i32(b.wcount, nv, b.woff, st)) != cudaSuccess) return e;
-  k_work_fill<<<(nv + 255) / 256, 256, 0, st>>>(b.wcount, b.woff, b.boff, nv, qchunk, b.witems_unsorted);
-  k_sort_work<<<1, 1024, 0, st>>>(b.witems_unsorted, b.woff + nv, b.boff, list_off, nlist, qchunk, b.witems);
+  k_work_fill<<<(nv + 255) / 256, 256, 0, st>>>(b.wcount, b.woff, b.boff, nv, qcfg, b.witems_unsorted);
+  k_sort_work<<<1, 1024, 0, st>>>(b.witems_unsorted, b.woff + nv, b.boff, list_off, nlist, qcfg, b.witems);
   return cudaGetLastError();
 }
 

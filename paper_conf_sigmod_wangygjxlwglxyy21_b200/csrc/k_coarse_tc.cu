@@ -191,19 +191,33 @@ __global__ void __launch_bounds__(kCThreads, 1)
               [&](int, int v) { return cbase + (uint32_t)v; }, [](int, uint32_t) {}, wscr);
         }
       } else {
+        // 32 < nprobe <= 128: filter against the list's nprobe-th best, buffered merges
         for (int j = ew; j < ((p.dbg & 1) ? 0 : nqv); j += kCEpi) {
+          uint64_t* L = lists + (int64_t)j * nprobe;
+          const uint32_t thr32 = (uint32_t)(L[nprobe - 1] >> 32);
           uint32_t k32[4];
+          bool pass[4];
+          int npass = 0;
 #pragma unroll
-          for (int m = 0; m < 4; ++m) k32[m] = Dt[j * kCDLD + m * 32 + lane];
-          warp_select_tile(lists + (int64_t)j * nprobe, nprobe, MV_KEY_PAD, k32,
-                           [&](int v) { return cbase + (uint32_t)v; }, wscr);
+          for (int m = 0; m < 4; ++m) {
+            k32[m] = Dt[j * kCDLD + m * 32 + lane];
+            pass[m] = k32[m] != 0xffffffffu && k32[m] <= thr32;
+            npass += __popc(__ballot_sync(MV_FULL, pass[m]));
+          }
+          if (npass == 0) continue;
+          auto low = [&](int v) { return cbase + (uint32_t)v; };
+          if (nprobe <= 64) warp_collect_R<2>(L, cbuf + j * 32, cnb + j, nprobe, k32, pass, npass, low);
+          else warp_collect_R<4>(L, cbuf + j * 32, cnb + j, nprobe, k32, pass, npass, low);
         }
       }
       cbar(1, 32 * kCEpi);
     }
-    if (nprobe <= 32)
-      for (int j = ew; j < nqv; j += kCEpi)
-        warp_flush_buffer(lists + (int64_t)j * nprobe, cbuf + j * 32, cnb + j, cbnd + j, nprobe, MV_KEY_PAD);
+    for (int j = ew; j < nqv; j += kCEpi) {
+      uint64_t* L = lists + (int64_t)j * nprobe;
+      if (nprobe <= 32) warp_flush_buffer(L, cbuf + j * 32, cnb + j, cbnd + j, nprobe, MV_KEY_PAD);
+      else if (nprobe <= 64) warp_flush_buffer_R<2>(L, cbuf + j * 32, cnb + j, nprobe);
+      else warp_flush_buffer_R<4>(L, cbuf + j * 32, cnb + j, nprobe);
+    }
     cbar(1, 32 * kCEpi);
     for (int i = et; i < nqv * nprobe; i += 32 * kCEpi) {
       const int j = i / nprobe, r = i - j * nprobe;
@@ -219,22 +233,35 @@ __global__ void __launch_bounds__(kCThreads, 1)
 }
 
 // plane-major tf32 split: out[0][r][:] = hi(x_r), out[1][r][:] = x_r - hi(x_r)
-__global__ void k_hilo(const float* __restrict__ x, int64_t n, int d, int dpad, float* __restrict__ out) {
+// tf32 round-to-nearest (ties away): the value with the low 13 mantissa bits cleared nearest to v
+__device__ __forceinline__ float tf32_rn(float v) {
+  const uint32_t b = __float_as_uint(v);
+  if ((b & 0x7f800000u) == 0x7f800000u) return __uint_as_float(b & 0xffffe000u);  // inf / nan
+  return __uint_as_float((b + 0x1000u) & 0xffffe000u);
+}
+
+// Both planes are tf32-representable (the MMA's operand truncation is then exact): hi = rn(x) and
+// lo = rn(x - hi), |lo| <= 2^-11 |x|, so hi + lo = x to ~2^-22 relative with unbiased rounding.
+__global__ void k_hilo(const float* __restrict__ x, int64_t n, int d, int dpad, float* __restrict__ out, int* lo_any) {
   const int64_t total = n * dpad;
+  bool nz = false;
   for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < total; t += (int64_t)gridDim.x * blockDim.x) {
     const int64_t r = t / dpad;
     const int j = (int)(t - r * dpad);
     const float v = j < d ? x[r * d + j] : 0.0f;
-    const float hi = __uint_as_float(__float_as_uint(v) & 0xffffe000u);
+    const float hi = tf32_rn(v);
+    const float lo = tf32_rn(v - hi);
     out[t] = hi;
-    out[total + t] = v - hi;
+    out[total + t] = lo;
+    nz |= lo != 0.0f;
   }
+  if (lo_any && __syncthreads_or(nz) && threadIdx.x == 0) atomicOr(lo_any, 1);
 }
 
-cudaError_t launch_hilo(const float* x, int64_t n, int d, int dpad, float* out, cudaStream_t st) {
+cudaError_t launch_hilo(const float* x, int64_t n, int d, int dpad, float* out, int* lo_any, cudaStream_t st) {
   if (n == 0) return cudaSuccess;
   const int grid = (int)min64(kNumSMs * 16, (n * dpad + 255) / 256);
-  k_hilo<<<grid, 256, 0, st>>>(x, n, d, dpad, out);
+  k_hilo<<<grid, 256, 0, st>>>(x, n, d, dpad, out, lo_any);
   return cudaGetLastError();
 }
 

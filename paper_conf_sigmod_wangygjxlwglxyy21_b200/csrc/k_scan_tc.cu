@@ -50,12 +50,12 @@ struct WorkInfo {
   int64_t lstart;
 };
 
-__device__ __forceinline__ WorkInfo work_info(const TcScanParams& p, int w) {
+__device__ __forceinline__ WorkInfo work_info(const TcScanParams& p, int w, int qchunk) {
   WorkInfo wi;
   const int2 it = p.witems[w];
   wi.l = it.x >= p.nlist ? it.x - p.nlist : it.x;
   wi.bstart = it.y;
-  wi.nqc = min(p.qchunk, p.boff[it.x + 1] - wi.bstart);
+  wi.nqc = min(qchunk, p.boff[it.x + 1] - wi.bstart);
   wi.lstart = p.list_off[wi.l];
   wi.len = (int)(p.list_off[wi.l + 1] - wi.lstart);
   wi.ntiles = (wi.len + 127) >> 7;
@@ -103,9 +103,11 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
   uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~(uintptr_t)1023);
   constexpr int ESZ = TYPE == MV_IVF_FLAT ? 4 : 1;
   constexpr int ATOM = TYPE == MV_IVF_FLAT ? 128 : 32;
-  constexpr int P = TYPE == MV_IVF_FLAT ? 2 : 4;
+  constexpr int PMAX = TYPE == MV_IVF_FLAT ? 2 : 4;
   const int nstage = p.nstage, nchunks = p.nchunks;
-  const int QCP = (p.qchunk + 15) & ~15;
+  const int QCP = (p.qchunk + 15) & ~15;       // metadata capacity (the largest chunk)
+  const int QC = p.cfg[0];                      // queries per work item in this search
+  const int P = TYPE == MV_IVF_FLAT ? p.cfg[1] : 4;  // query planes: FLAT 1 (tf32-exact queries) or 2
   const int rowbytes = p.dpad * ESZ;
   const bool use_norms = p.metric == MV_L2;
   const bool use_ids = p.bitset != nullptr;
@@ -164,7 +166,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
       uint32_t it = 0, tcount = 0;
       const uint32_t side_tx = 528 + (use_norms ? 1040 : 0) + (use_ids ? 1040 : 0);
       for (int w = w0; w < nwork; w += gridDim.x) {
-        const WorkInfo wi = work_info(p, w);
+        const WorkInfo wi = work_info(p, w, QC);
         for (int t = 0; t < wi.ntiles; ++t, ++tcount) {
           const int row0 = (int)(wi.lstart + t * 128);
           const uint32_t ts = tcount % kNTS, tr = tcount / kNTS;
@@ -189,7 +191,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
     if (lane == 0) {
       uint32_t it = 0, titer = 0, wcount = 0;
       for (int w = w0; w < nwork; w += gridDim.x, ++wcount) {
-        const WorkInfo wi = work_info(p, w);
+        const WorkInfo wi = work_info(p, w, QC);
         const int NQ = (wi.nqc + 15) & ~15;
         const int N = P * NQ;
         const uint32_t idesc = TYPE == MV_IVF_FLAT ? idesc_tf32(N) : idesc_u8s8(N);
@@ -230,7 +232,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
     const int tq = threadIdx.x - 64;
     uint32_t wcount = 0;
     for (int w = w0; w < nwork; w += gridDim.x, ++wcount) {
-      const WorkInfo wi = work_info(p, w);
+      const WorkInfo wi = work_info(p, w, QC);
       const int NQ = (wi.nqc + 15) & ~15;
       const int N = P * NQ;
       const uint32_t b = wcount & 1, r = wcount >> 1;
@@ -290,7 +292,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
     const uint32_t ltmask = (1u << lane) - 1;
     uint32_t titer = 0, wcount = 0;
     for (int w = w0; w < nwork; w += gridDim.x, ++wcount) {
-      const WorkInfo wi = work_info(p, w);
+      const WorkInfo wi = work_info(p, w, QC);
       const int NQ = (wi.nqc + 15) & ~15;
       const uint32_t b = wcount & 1;
       mbar_wait(&full_q[b], (wcount >> 1) & 1);
@@ -313,9 +315,14 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
         tc_fence_after();
         const uint32_t tbase = tmem + a * p.ncol + ((uint32_t)(quarter * 32) << 16);
         for (int qc = half * 16; qc < ((p.dbg & 2) ? 0 : NQ); qc += 32) {
-          uint32_t r[P][16];
+          uint32_t r[PMAX][16];
 #pragma unroll
-          for (int pl = 0; pl < P; ++pl) tmem_ld16(tbase + pl * NQ + qc, r[pl]);
+          for (int pl = 0; pl < PMAX; ++pl) {
+            if (pl < P) tmem_ld16(tbase + pl * NQ + qc, r[pl]);
+            else
+#pragma unroll
+              for (int j = 0; j < 16; ++j) r[pl][j] = 0u;
+          }
           tmem_wait_ld();
           float bad[16];
           uint32_t pm = 0;
@@ -325,14 +332,14 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
             // badness = L2 distance or -IP (smaller is better)
             if (TYPE == MV_IVF_FLAT) {
               // exact for tf32-representable data (the only FLAT data this path accepts)
-              const float dot = __uint_as_float(r[0][j]) + __uint_as_float(r[1 % P][j]);
+              const float dot = __uint_as_float(r[0][j]) + __uint_as_float(r[1 % PMAX][j]);
               bad[j] = use_norms ? (mt.qnf[i] + xnf) - 2.0f * dot : -dot;
             } else {
               // int32-exact digit partials; the L2 expansion is combined in fp64 (the norms are
               // ~400x the near-neighbour distances on SIFT-scale data)
-              const double acc = (double)(int)r[0][j] + (double)(int)r[1 % P][j] * (1.0 / 128.0) +
-                                 (double)(int)r[2 % P][j] * (1.0 / 16384.0) +
-                                 (double)(int)r[3 % P][j] * (1.0 / 2097152.0);
+              const double acc = (double)(int)r[0][j] + (double)(int)r[1 % PMAX][j] * (1.0 / 128.0) +
+                                 (double)(int)r[2 % PMAX][j] * (1.0 / 16384.0) +
+                                 (double)(int)r[3 % PMAX][j] * (1.0 / 2097152.0);
               const double dot = fma((double)mt.qs[i], acc, mt.qa[i]);
               bad[j] = use_norms ? (float)((mt.qn[i] + xn) - 2.0 * dot) : (float)(-dot);
             }
@@ -468,19 +475,22 @@ cudaError_t launch_tf32_check(const float* x, int64_t n, int* flag, cudaStream_t
 static bool tc_scan_layout(int type, int dpad, int qc, int ns, TcScanParams& p) {
   const int esz = type == MV_IVF_FLAT ? 4 : 1;
   const int atom = type == MV_IVF_FLAT ? 128 : 32;
-  const int P = type == MV_IVF_FLAT ? 2 : 4;
+  // FLAT: qc queries of one plane (tf32-exact queries) or qc/2 queries of two (hi/lo) in the same
+  // operand rows; SQ8: four digit planes
+  const int rows_per_q = type == MV_IVF_FLAT ? 1 : 4;
   auto up = [](int x, int a) { return (x + a - 1) / a * a; };
   p.type = type;
   p.dpad = dpad;
   p.nchunks = dpad * esz / atom;
   p.qchunk = qc;
+  p.qchunk_split = type == MV_IVF_FLAT ? qc / 2 : qc;
   const int qcp = (qc + 15) & ~15;
-  p.ncol = P * qcp;
+  p.ncol = rows_per_q * qcp;
   int cols = 32;
   while (cols < 2 * p.ncol) cols <<= 1;
   if (cols > 512) return false;
   p.tmem_cols = cols;
-  p.q_bytes = up(P * qcp * dpad * esz, 1024);
+  p.q_bytes = up(rows_per_q * qcp * dpad * esz, 1024);
   p.meta_bytes = up(kMetaPerQuery * qcp, 16);
   const int stage = 128 * atom;
   p.nstage = ns;
@@ -494,11 +504,11 @@ static bool tc_scan_layout(int type, int dpad, int qc, int ns, TcScanParams& p) 
 }
 
 bool tc_scan_plan(int type, int dpad, int k, TcScanParams& p) {
-  const int qcmax = type == MV_IVF_FLAT ? 48 : 64;
+  const int qcmax = type == MV_IVF_FLAT ? 96 : 64;
   const int nscap = type == MV_IVF_FLAT ? 8 : 24;
-  const int nsmin = type == MV_IVF_FLAT ? 3 : 6;  // >= 48 KB (FLAT) / 24 KB (SQ8) of list tiles in flight
+  const int nsmin = type == MV_IVF_FLAT ? 4 : 6;  // >= 64 KB (FLAT) / 24 KB (SQ8) of list tiles in flight
   p.k = k;
-  for (int qc = qcmax; qc >= 16; qc -= 16)
+  for (int qc = qcmax; qc >= 32; qc -= 32)
     for (int ns = nscap; ns >= nsmin; --ns)
       if (tc_scan_layout(type, dpad, qc, ns, p)) return true;
   return false;

@@ -29,7 +29,8 @@ __global__ void __launch_bounds__(256) k_final_select(const int64_t* __restrict_
                                                       const uint64_t* __restrict__ part, int64_t nq, int npb, int k,
                                                       int metric, const int64_t* __restrict__ sorted_ids, float* out_d,
                                                       int64_t* out_i, int selcap, const int32_t* __restrict__ nuse,
-                                                      uint64_t* tau_out) {
+                                                      uint64_t* tau_out, const uint8_t* __restrict__ only) {
+  if (only && !only[blockIdx.x]) return;  // handled by k_final_big
   extern __shared__ __align__(16) uint8_t smem[];
   uint64_t* sel = reinterpret_cast<uint64_t*>(smem);       // selcap
   uint64_t* bnd = sel + selcap;                             // kBoundCap
@@ -150,20 +151,212 @@ __global__ void __launch_bounds__(256) k_final_select(const int64_t* __restrict_
   }
 }
 
-// k <= 32: one warp per query.  The pairs' regions are walked in 32-key chunks (a flattened index
-// over groups of 32 pairs, located by a shuffle binary search); a chunk is skipped unless some key
-// beats the running k-th best, else it is bitonic-sorted and merged into the sorted register list.
-__global__ void __launch_bounds__(256) k_final_small(const int64_t* __restrict__ poff, const int32_t* __restrict__ pcnt,
-                                                     const uint64_t* __restrict__ part, int64_t nq, int npb, int k,
-                                                     int metric, const int64_t* __restrict__ sorted_ids, float* out_d,
-                                                     int64_t* out_i, const int32_t* __restrict__ nuse,
-                                                     uint64_t* tau_out) {
+// 256 < k: one CTA (512 threads) per query stages the query's candidates in shared memory (when
+// they fit, else it flags the query for k_final_select's global-memory path), then an MSB radix
+// select over the u64 keys -- 8-bit digits, histogram per pass in shared memory, stopping as soon
+// as the keys at or below the current prefix are exactly k -- and a bitonic sort of the k winners.
+constexpr int kBigThreads = 512;
+
+__global__ void __launch_bounds__(kBigThreads) k_final_big(const int64_t* __restrict__ poff,
+                                                           const int32_t* __restrict__ pcnt,
+                                                           const uint64_t* __restrict__ part, int64_t nq, int npb, int k,
+                                                           int metric, const int64_t* __restrict__ sorted_ids,
+                                                           float* out_d, int64_t* out_i, int cap,
+                                                           const int32_t* __restrict__ nuse, uint64_t* tau_out,
+                                                           uint8_t* over) {
+  extern __shared__ __align__(16) uint8_t smem[];
+  const int NK = next_pow2(max(k, 2));
+  uint64_t* buf = reinterpret_cast<uint64_t*>(smem);   // cap
+  uint64_t* win = buf + cap;                           // NK
+  uint32_t* hist = reinterpret_cast<uint32_t*>(win + NK);  // 256
+  int32_t* s_pre = reinterpret_cast<int32_t*>(hist + 256);  // npb + 1
+  int32_t* s_int = s_pre + npb + 1;                    // misc
+  const int64_t q = blockIdx.x;
+  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  const int64_t* po = poff + q * npb;
+  const int32_t* pc = pcnt + q * npb;
+  const int nu = nuse ? nuse[q] : npb;
+  if (wid == 0) {  // prefix of the pair counts, 32 pairs at a time
+    int run = 0;
+    for (int j0 = 0; j0 < nu; j0 += 32) {
+      const int j = j0 + lane;
+      const int c = j < nu ? pc[j] : 0;
+      int incl = c;
+      for (int o = 1; o < 32; o <<= 1) {
+        const int v = __shfl_up_sync(MV_FULL, incl, o);
+        if (lane >= o) incl += v;
+      }
+      if (j < nu) s_pre[j] = run + incl - c;
+      run += __shfl_sync(MV_FULL, incl, 31);
+    }
+    if (lane == 0) s_pre[nu] = run;
+  }
+  __syncthreads();
+  const int T = s_pre[nu];
+  if (T > cap) {
+    if (tid == 0) over[q] = 1;
+    return;
+  }
+  if (tid == 0) over[q] = 0;
+  for (int j = wid; j < nu; j += kBigThreads / 32) {
+    const int c = s_pre[j + 1] - s_pre[j];
+    const uint64_t* src = part + po[j];
+    uint64_t* dst = buf + s_pre[j];
+    for (int i = lane; i < c; i += 32) dst[i] = src[i];
+  }
+  __syncthreads();
+  int nsel;  // winners to sort, in win[]
+  if (T <= k) {
+    for (int i = tid; i < NK; i += kBigThreads) win[i] = i < T ? buf[i] : MV_KEY_PAD;
+    nsel = T;
+  } else {
+    // radix select: find the largest prefix such that #keys with top <= prefix is exactly k
+    uint64_t pfx = 0;
+    int fixed = 0, below = 0;  // below = #keys whose top bits are < the current prefix
+    for (;;) {
+      for (int i = tid; i < 256; i += kBigThreads) hist[i] = 0;
+      __syncthreads();
+      const int sh = 56 - fixed;
+      for (int i = tid; i < T; i += kBigThreads) {
+        const uint64_t x = buf[i];
+        if (fixed == 0 || (x >> (64 - fixed)) == pfx) atomicAdd(hist + ((x >> sh) & 0xff), 1u);
+      }
+      __syncthreads();
+      if (tid == 0) {
+        int cum = below, d = 0;
+        for (; d < 256; ++d) {
+          if (cum + (int)hist[d] >= k) break;
+          cum += hist[d];
+        }
+        s_int[0] = d;
+        s_int[1] = cum;
+        s_int[2] = cum + (int)hist[d] == k;
+      }
+      __syncthreads();
+      pfx = (pfx << 8) | (uint64_t)s_int[0];
+      below = s_int[1];
+      fixed += 8;
+      const bool done = s_int[2] || fixed == 64;
+      __syncthreads();
+      if (done) break;
+    }
+    // winners: keys whose top `fixed` bits are <= pfx (exactly k: keys are unique)
+    if (tid == 0) s_int[3] = 0;
+    __syncthreads();
+    const int sh = 64 - fixed;
+    for (int i = tid; i < T; i += kBigThreads) {
+      const uint64_t x = buf[i];
+      const uint64_t top = sh >= 64 ? 0 : (x >> sh);
+      if (top <= pfx) win[atomicAdd(s_int + 3, 1)] = x;
+    }
+    __syncthreads();
+    nsel = k;
+    for (int i = k + tid; i < NK; i += kBigThreads) win[i] = MV_KEY_PAD;
+  }
+  __syncthreads();
+  if (tau_out) {  // seeding: only the k-th best key is needed (the largest winner)
+    if (nsel < k) return;
+    uint64_t m = 0;
+    for (int i = tid; i < k; i += kBigThreads) m = umax64(m, win[i]);
+    for (int o = 16; o > 0; o >>= 1) m = umax64(m, shfl_xor64(m, o));
+    if (lane == 0) buf[wid] = m;
+    __syncthreads();
+    if (tid == 0) {
+      uint64_t mm = 0;
+      for (int w = 0; w < kBigThreads / 32; ++w) mm = umax64(mm, buf[w]);
+      tau_out[q] = mm;
+    }
+    return;
+  }
+  // bitonic sort of the NK winners (block-wide, shared memory)
+  for (int size = 2; size <= NK; size <<= 1) {
+    for (int stride = size >> 1; stride > 0; stride >>= 1) {
+      __syncthreads();
+      for (int t = tid; t < (NK >> 1); t += kBigThreads) {
+        const int lo = 2 * t - (t & (stride - 1));
+        const int hi = lo + stride;
+        const bool up = ((lo & size) == 0);
+        const uint64_t x = win[lo], y = win[hi];
+        if ((x > y) == up) {
+          win[lo] = y;
+          win[hi] = x;
+        }
+      }
+    }
+  }
+  __syncthreads();
+  for (int i = tid; i < k; i += kBigThreads) {
+    float dv;
+    int64_t iv;
+    const uint64_t key = win[i];
+    if (i < nsel && key != MV_KEY_PAD) {
+      dv = key_dist((uint32_t)(key >> 32), metric);
+      iv = sorted_ids[(uint32_t)(key & 0xffffffffu)];
+    } else {
+      dv = metric == MV_L2 ? __int_as_float(0x7f800000) : __int_as_float(0xff800000);
+      iv = -1;
+    }
+    out_d[q * k + i] = dv;
+    out_i[q * k + i] = iv;
+  }
+}
+
+// k > 256: k_final_big for every query whose candidates fit its shared-memory stage (cap keys),
+// k_final_select (global-memory radix) for the others -- launched only when some query could
+// exceed cap (tmax = an upper bound of the candidates per query)
+static cudaError_t launch_big_select(const int64_t* poff, const int32_t* pcnt, const uint64_t* part, int64_t nq,
+                                     int npb, int k, int metric, const int64_t* sorted_ids, float* out_d,
+                                     int64_t* out_i, const int32_t* nuse, uint64_t* tau, int64_t tmax,
+                                     uint8_t* over, cudaStream_t st) {
+  const int NK = next_pow2(max(k, 2));
+  const int fixed = NK * 8 + 256 * 4 + (npb + 1) * 4 + 64 + 64;
+  const int cap = (227 * 1024 - fixed) / 8;
+  if (over && cap >= k) {
+    const size_t smem = (size_t)cap * 8 + fixed;
+    cudaError_t e = cudaFuncSetAttribute(k_final_big, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    k_final_big<<<(unsigned)nq, kBigThreads, smem, st>>>(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d,
+                                                         out_i, cap, nuse, tau, over);
+    if (tmax <= cap) return cudaGetLastError();
+  } else {
+    over = nullptr;
+  }
+  const int selcap = max(4096, next_pow2(k));
+  size_t smem = (size_t)(selcap + kBoundCap) * 8 + (size_t)(npb + 1) * 4 + 256 * 4 + 8 * 4 + 64;
+  cudaError_t e = cudaFuncSetAttribute(k_final_select, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  k_final_select<<<(unsigned)nq, 256, smem, st>>>(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d, out_i,
+                                                  selcap, nuse, tau, over);
+  return cudaGetLastError();
+}
+
+// k <= 32 R: one warp per query, its running best-32R list sorted across registers (element
+// r*32 + lane in best[r]).  The pairs' regions are walked in 32-key chunks (a flattened index over
+// groups of 32 pairs, located by a shuffle binary search; the next chunk's load is issued before
+// the current one is folded); a chunk is skipped unless some key beats the running k-th best, else
+// it is bitonic-sorted and merged into the list.
+template <int R>
+__global__ void __launch_bounds__(256) k_final_warp(const int64_t* __restrict__ poff, const int32_t* __restrict__ pcnt,
+                                                    const uint64_t* __restrict__ part, int64_t nq, int npb, int k,
+                                                    int metric, const int64_t* __restrict__ sorted_ids, float* out_d,
+                                                    int64_t* out_i, const int32_t* __restrict__ nuse,
+                                                    uint64_t* tau_out) {
   const int lane = threadIdx.x & 31;
   const int64_t q = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   if (q >= nq) return;
   const int stride = npb;
   if (nuse) npb = nuse[q];
-  uint64_t best[1] = {MV_KEY_PAD};  // ascending: lane i holds the i-th best so far
+  uint64_t best[R];
+#pragma unroll
+  for (int r = 0; r < R; ++r) best[r] = MV_KEY_PAD;
+  const int kr = (k - 1) >> 5, kl = (k - 1) & 31;
+  auto kth_of = [&]() {
+    uint64_t v = best[0];
+#pragma unroll
+    for (int r = 1; r < R; ++r)
+      if (r == kr) v = best[r];
+    return shfl64(v, kl);
+  };
   for (int g = 0; g < npb; g += 32) {
     const int j = g + lane;
     const int cnt = j < npb ? pcnt[q * stride + j] : 0;
@@ -175,80 +368,95 @@ __global__ void __launch_bounds__(256) k_final_small(const int64_t* __restrict__
     }
     const int excl = incl - cnt;
     const int T = __shfl_sync(MV_FULL, incl, 31);
-    for (int e0 = 0; e0 < T; e0 += 32) {
+    auto load = [&](int e0) {
       const int e = e0 + lane;
       // pair holding element e: the largest s with excl[s] <= e
       int lo = 0;
 #pragma unroll
       for (int step = 16; step > 0; step >>= 1) {
-        const int ex = __shfl_sync(MV_FULL, excl, lo + step);
+        const int ex = __shfl_sync(MV_FULL, excl, (lo + step) & 31);
         if (lo + step < 32 && ex <= e) lo += step;
       }
       const int64_t o = __shfl_sync(MV_FULL, off, lo);
       const int ex = __shfl_sync(MV_FULL, excl, lo);
-      uint64_t v[1] = {e < T ? part[o + (e - ex)] : MV_KEY_PAD};
-      const uint64_t kth = shfl64(best[0], k - 1);
-      if (!(v[0] < kth)) v[0] = MV_KEY_PAD;
-      if (__any_sync(MV_FULL, v[0] != MV_KEY_PAD)) {
-        warp_bitonic_sort<1>(v);
-        warp_merge_smallest<1>(best, v);
+      return e < T ? part[o + (e - ex)] : MV_KEY_PAD;
+    };
+    uint64_t nxt = T > 0 ? load(0) : MV_KEY_PAD;
+    for (int e0 = 0; e0 < T; e0 += 32) {
+      uint64_t c[R];
+      c[0] = nxt;
+#pragma unroll
+      for (int r = 1; r < R; ++r) c[r] = MV_KEY_PAD;
+      if (e0 + 32 < T) nxt = load(e0 + 32);
+      if (!(c[0] < kth_of())) c[0] = MV_KEY_PAD;
+      if (__any_sync(MV_FULL, c[0] != MV_KEY_PAD)) {
+        uint64_t c1[1] = {c[0]};
+        warp_bitonic_sort<1>(c1);
+        c[0] = c1[0];
+        warp_merge_smallest<R>(best, c);
       }
     }
   }
   if (tau_out) {  // seeding: the k-th best key of the first nuse[q] pairs bounds the query's top-k
-    const uint64_t kth = shfl64(best[0], k - 1);
+    const uint64_t kth = kth_of();
     if (lane == 0 && kth != MV_KEY_PAD) tau_out[q] = kth;
     return;
   }
-  if (lane < k) {
-    const uint64_t key = best[0];
-    float dv;
-    int64_t iv;
-    if (key != MV_KEY_PAD) {
-      dv = key_dist((uint32_t)(key >> 32), metric);
-      iv = sorted_ids[(uint32_t)(key & 0xffffffffu)];
-    } else {
-      dv = metric == MV_L2 ? __int_as_float(0x7f800000) : __int_as_float(0xff800000);
-      iv = -1;
+#pragma unroll
+  for (int r = 0; r < R; ++r) {
+    const int i = r * 32 + lane;
+    if (i < k) {
+      const uint64_t key = best[r];
+      float dv;
+      int64_t iv;
+      if (key != MV_KEY_PAD) {
+        dv = key_dist((uint32_t)(key >> 32), metric);
+        iv = sorted_ids[(uint32_t)(key & 0xffffffffu)];
+      } else {
+        dv = metric == MV_L2 ? __int_as_float(0x7f800000) : __int_as_float(0xff800000);
+        iv = -1;
+      }
+      out_d[q * k + i] = dv;
+      out_i[q * k + i] = iv;
     }
-    out_d[q * k + lane] = dv;
-    out_i[q * k + lane] = iv;
   }
+}
+
+// k <= 256: the warp kernel with a 32R-entry register list (R = 1, 2, 4, 8)
+static bool launch_warp_select(const int64_t* poff, const int32_t* pcnt, const uint64_t* part, int64_t nq, int npb,
+                               int k, int metric, const int64_t* sorted_ids, float* out_d, int64_t* out_i,
+                               const int32_t* nuse, uint64_t* tau, cudaStream_t st) {
+  const unsigned grid = (unsigned)((nq * 32 + 255) / 256);
+  if (k <= 32)
+    k_final_warp<1><<<grid, 256, 0, st>>>(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d, out_i, nuse, tau);
+  else if (k <= 64)
+    k_final_warp<2><<<grid, 256, 0, st>>>(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d, out_i, nuse, tau);
+  else if (k <= 128)
+    k_final_warp<4><<<grid, 256, 0, st>>>(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d, out_i, nuse, tau);
+  else if (k <= 256)
+    k_final_warp<8><<<grid, 256, 0, st>>>(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d, out_i, nuse, tau);
+  else
+    return false;
+  return true;
 }
 
 cudaError_t launch_final_select(const int64_t* poff, const int32_t* pcnt, const uint64_t* part, int64_t nq, int npb,
                                 int k, int metric, const int64_t* sorted_ids, float* out_d, int64_t* out_i,
-                                cudaStream_t st) {
+                                int64_t tmax, uint8_t* over, cudaStream_t st) {
   if (nq == 0) return cudaSuccess;
-  if (k <= 32) {
-    k_final_small<<<(unsigned)((nq * 32 + 255) / 256), 256, 0, st>>>(poff, pcnt, part, nq, npb, k, metric, sorted_ids,
-                                                                     out_d, out_i, nullptr, nullptr);
+  if (launch_warp_select(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d, out_i, nullptr, nullptr, st))
     return cudaGetLastError();
-  }
-  const int selcap = max(4096, next_pow2(k));
-  size_t smem = (size_t)(selcap + kBoundCap) * 8 + (size_t)(npb + 1) * 4 + 256 * 4 + 8 * 4 + 64;
-  cudaError_t e = cudaFuncSetAttribute(k_final_select, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  if (e != cudaSuccess) return e;
-  k_final_select<<<(unsigned)nq, 256, smem, st>>>(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d, out_i,
-                                                  selcap, nullptr, nullptr);
-  return cudaGetLastError();
+  return launch_big_select(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d, out_i, nullptr, nullptr, tmax,
+                           over, st);
 }
 
 cudaError_t launch_tau_select(const int64_t* poff, const int32_t* pcnt, const uint64_t* part, int64_t nq, int npb,
-                              const int32_t* nuse, int k, uint64_t* tau, cudaStream_t st) {
+                              const int32_t* nuse, int k, uint64_t* tau, int64_t tmax, uint8_t* over,
+                              cudaStream_t st) {
   if (nq == 0) return cudaSuccess;
-  if (k <= 32) {
-    k_final_small<<<(unsigned)((nq * 32 + 255) / 256), 256, 0, st>>>(poff, pcnt, part, nq, npb, k, MV_L2, nullptr,
-                                                                     nullptr, nullptr, nuse, tau);
+  if (launch_warp_select(poff, pcnt, part, nq, npb, k, MV_L2, nullptr, nullptr, nullptr, nuse, tau, st))
     return cudaGetLastError();
-  }
-  const int selcap = max(4096, next_pow2(k));
-  size_t smem = (size_t)(selcap + kBoundCap) * 8 + (size_t)(npb + 1) * 4 + 256 * 4 + 8 * 4 + 64;
-  cudaError_t e = cudaFuncSetAttribute(k_final_select, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  if (e != cudaSuccess) return e;
-  k_final_select<<<(unsigned)nq, 256, smem, st>>>(poff, pcnt, part, nq, npb, k, MV_L2, nullptr, nullptr, nullptr,
-                                                  selcap, nuse, tau);
-  return cudaGetLastError();
+  return launch_big_select(poff, pcnt, part, nq, npb, k, MV_L2, nullptr, nullptr, nullptr, nuse, tau, tmax, over, st);
 }
 
 // ------------------------------------------------------------------------------------------

@@ -265,7 +265,7 @@ mv_status mv_index_set_centroids(mv_index* ix, const float* centroids) {
   CK(stage_in(s, centroids, (size_t)ix->nlist * ix->d, &c, &staged));
   CK(launch_centroid_prep(c, ix->nlist, ix->d, ix->dpad, ix->cpad, ix->cnorm, st));
   if (!ix->chl) CK(cudaMalloc(&ix->chl, sizeof(float) * 2 * (size_t)ix->nlist * ix->dpad));
-  CK(launch_hilo(c, ix->nlist, ix->d, ix->dpad, ix->chl, st));
+  CK(launch_hilo(c, ix->nlist, ix->d, ix->dpad, ix->chl, nullptr, st));
   CK(cudaStreamSynchronize(st));
   ix->cmap_ok = make_tmap_2d(&ix->cmap, ix->chl, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, (uint64_t)ix->dpad,
                              2 * (uint64_t)ix->nlist, (uint64_t)ix->dpad * 4, 32, 128, CU_TENSOR_MAP_SWIZZLE_128B);
@@ -483,7 +483,7 @@ mv_status mv_search_probes(mv_index* ix, const float* queries, int64_t nq, int32
   CK(launch_query_prep(q, nq, ix->d, ix->dpad, qpad, qnorm, st));
   float* qhl;
   CK(s.alloc(&qhl, (size_t)2 * nq * ix->dpad));
-  CK(launch_hilo(q, nq, ix->d, ix->dpad, qhl, st));
+  CK(launch_hilo(q, nq, ix->d, ix->dpad, qhl, nullptr, st));
   CK(run_coarse(ix, qpad, qhl, nq, npb, P, st));
   if (sp) {
     CK(cudaMemcpyAsync(probes, P, sizeof(int32_t) * nq * npb, cudaMemcpyDeviceToHost, st));
@@ -529,7 +529,10 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
     CK(launch_query_prep(q, nq, ix->d, dpad, qpad, qnorm, st));
     float* qhl;  // plane-major tf32 hi/lo query planes: coarse B operand and the FLAT scan's query planes
     CK(s.alloc(&qhl, (size_t)2 * nq * dpad));
-    CK(launch_hilo(q, nq, ix->d, dpad, qhl, st));
+    int* qlo_any;  // does any query need its lo plane (not tf32-exact)?  Decides the FLAT scan shape
+    CK(s.alloc(&qlo_any, 1));
+    CK(cudaMemsetAsync(qlo_any, 0, sizeof(int), st));
+    CK(launch_hilo(q, nq, ix->d, dpad, qhl, qlo_any, st));
     CK(run_coarse(ix, qpad, qhl, nq, npb, P, st));
     prof_mark(ix, st);
     // a4 (work-item size depends on the scan implementation's shared-memory plan)
@@ -539,6 +542,12 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
                         (ix->type == MV_IVF_SQ8 || ix->tf32_exact) && tc_scan_plan(ix->type, dpad, k, tp);
     const int qchunk = use_tc ? tp.qchunk
                               : (k <= kLocalSelectMaxK ? std::min(64, std::max(1, 65536 / (8 * k))) : 64);
+    // device-side work-item shape: FLAT tf32-exact queries take one plane and twice the queries
+    const int qchunk_min = use_tc ? tp.qchunk_split : qchunk;
+    int32_t* qcfg;
+    CK(s.alloc(&qcfg, 2));
+    if (use_tc && ix->type == MV_IVF_FLAT) CK(launch_scan_cfg(qlo_any, tp.qchunk, 1, tp.qchunk_split, 2, qcfg, st));
+    else CK(launch_scan_cfg(nullptr, qchunk, use_tc ? 4 : 1, qchunk, 4, qcfg, st));
     const int64_t npairs = nq * npb;
     // Seeding (tensor-core path, nprobe >= 2): phase A scans each query's ra[q] nearest lists --
     // the fewest holding >= 2k candidates -- and emits all of them; their k-th best key tau_q is an
@@ -558,13 +567,13 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
     CK(s.alloc(&b.bq, (size_t)npairs));
     CK(s.alloc(&b.wcount, nv));
     CK(s.alloc(&b.woff, nv + 1));
-    CK(s.alloc(&b.witems, (size_t)(nv + npairs / qchunk + 1)));
-    CK(s.alloc(&b.witems_unsorted, (size_t)(nv + npairs / qchunk + 1)));
+    CK(s.alloc(&b.witems, (size_t)(nv + npairs / qchunk_min + 1)));
+    CK(s.alloc(&b.witems_unsorted, (size_t)(nv + npairs / qchunk_min + 1)));
     CK(s.alloc(&b.qtot, (size_t)(2 * (nq + 1))));
     CK(s.alloc(&b.poff, (size_t)npairs));
     CK(s.alloc(&b.pcnt, (size_t)npairs));
     CK(s.alloc(&b.counter, 1));
-    CK(launch_bucket(P, nq, npb, nlist, ix->list_off, k, qchunk, ra, b, st));
+    CK(launch_bucket(P, nq, npb, nlist, ix->list_off, k, qcfg, ra, b, st));
     // pair regions: the whole list (tensor-core scan: emit-all bound), or min(k, |list|) (SIMT)
     const int capk = use_tc ? 0 : k;
     CK(launch_pair_offsets(P, nq, npb, ix->list_off, k, capk, b, st));
@@ -579,6 +588,11 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
       CK(cudaMemcpyAsync(&cap, b.qtot + (nq + 1) + nq, sizeof(int64_t), cudaMemcpyDeviceToHost, st));
       CK(cudaStreamSynchronize(st));
     }
+    // per-query candidate bound (the final select's shared-memory staging decision) + its scratch
+    const int64_t tmax = use_tc ? ix->top_len_prefix[std::min<size_t>(npb, ix->top_len_prefix.size() - 1)]
+                                : (int64_t)npb * (k <= kLocalSelectMaxK ? k : max64(ix->maxlen, 1));
+    uint8_t* over = nullptr;
+    if (k > 256) CK(s.alloc(&over, (size_t)nq));
     uint64_t* part;
     cudaError_t ea = s.alloc(&part, (size_t)max64(cap, 1));
     if (ea != cudaSuccess) {
@@ -606,7 +620,7 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
       tp.list_off = ix->list_off; tp.norms = ix->norms; tp.ids = ix->ids; tp.rank = ix->rank;
       tp.bitset = bs; tp.nbits = bs ? nbits : 0;
       tp.qplanes = qplanes; tp.qnorm = qn64; tp.qscale = qscale; tp.qa = qa;
-      tp.bq = b.bq; tp.boff = b.boff; tp.witems = b.witems; tp.nlist = nlist;
+      tp.bq = b.bq; tp.boff = b.boff; tp.witems = b.witems; tp.nlist = nlist; tp.cfg = qcfg;
       tp.poff = b.poff; tp.pcnt = b.pcnt; tp.part = part; tp.tau = tau;
       const char* dbg = getenv("MV_SCAN_DEBUG");
       tp.dbg = dbg ? atoi(dbg) : 0;
@@ -624,7 +638,7 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
       prof_mark(ix, st);
       if (split) {
         // ... tau_q = k-th best key of phase A ...
-        CK(launch_tau_select(b.poff, b.pcnt, part, nq, npb, ra, k, tau, st));
+        CK(launch_tau_select(b.poff, b.pcnt, part, nq, npb, ra, k, tau, tmax, over, st));
         prof_mark(ix, st);
         // ... phase B over the remaining pairs, emitting keys < tau_q
         tp.phase = 1;
@@ -677,10 +691,10 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
     }
     prof_mark(ix, st);
     // a7
-    CK(launch_final_select(b.poff, b.pcnt, part, nq, npb, k, ix->metric, ix->sorted_ids, D, I, st));
+    CK(launch_final_select(b.poff, b.pcnt, part, nq, npb, k, ix->metric, ix->sorted_ids, D, I, tmax, over, st));
     prof_mark(ix, st);
     if (ix->prof) ix->prof_searches++;
-    ix->launches += 14;  // prep, hilo, coarse, 7 bucketing, 3 offsets, final select (+ SIMT scan below)
+    ix->launches += 15;  // prep, hilo, coarse, cfg, 7 bucketing, 3 offsets, final select (+ SIMT scan below)
     if (!use_tc) ix->launches += 1;
   }
   if (host_out) {

@@ -406,6 +406,74 @@ __device__ __forceinline__ void warp_filter_group(int nvalid, int k, RowK rowk, 
   }
 }
 
+// Buffered selection for 32 < k <= 32R (R = 2, 4): the sorted list L (k keys in smem) takes
+// survivors through a 32-entry buffer B (count *nb), merged by sort-32 + a register bitonic merge
+// when full (and by warp_flush_buffer_R at the end); a dense tile (> 32 survivors) is sorted as a
+// whole and merged directly.  L[k-1] is always an exact bound of the k-th best seen so far.
+template <int R>
+__device__ __forceinline__ void warp_merge_into_list(uint64_t* L, int k, const uint64_t (&cand)[R]) {
+  const int lane = threadIdx.x & 31;
+  uint64_t lv[R];
+#pragma unroll
+  for (int r = 0; r < R; ++r) lv[r] = r * 32 + lane < k ? L[r * 32 + lane] : MV_KEY_PAD;
+  warp_merge_smallest<R>(lv, cand);
+  __syncwarp();
+#pragma unroll
+  for (int r = 0; r < R; ++r)
+    if (r * 32 + lane < k) L[r * 32 + lane] = lv[r];
+  __syncwarp();
+}
+
+template <int R>
+__device__ __forceinline__ void warp_flush_buffer_R(uint64_t* L, uint64_t* B, int* nb, int k) {
+  const int lane = threadIdx.x & 31;
+  const int n = *nb;
+  if (n == 0) return;
+  uint64_t c[1] = {lane < n ? B[lane] : MV_KEY_PAD};
+  if (!(c[0] < L[k - 1])) c[0] = MV_KEY_PAD;
+  warp_bitonic_sort<1>(c);
+  uint64_t cand[R];
+  cand[0] = c[0];
+#pragma unroll
+  for (int r = 1; r < R; ++r) cand[r] = MV_KEY_PAD;
+  warp_merge_into_list<R>(L, k, cand);
+  if (lane == 0) *nb = 0;
+  __syncwarp();
+}
+
+template <int R, typename Low>
+__device__ __forceinline__ void warp_collect_R(uint64_t* L, uint64_t* B, int* nb, int k, const uint32_t (&k32)[4],
+                                               const bool (&pass)[4], int npass, Low low) {
+  const int lane = threadIdx.x & 31;
+  if (npass > 32) {
+    warp_flush_buffer_R<R>(L, B, nb, k);
+    const uint64_t lk = L[k - 1];
+    uint64_t key[4];
+#pragma unroll
+    for (int m = 0; m < 4; ++m) {
+      key[m] = pass[m] ? (((uint64_t)k32[m] << 32) | low(m * 32 + lane)) : MV_KEY_PAD;
+      if (!(key[m] < lk)) key[m] = MV_KEY_PAD;
+    }
+    warp_bitonic_sort<4>(key);
+    uint64_t cand[R];
+#pragma unroll
+    for (int r = 0; r < R; ++r) cand[r] = key[r];  // the smallest 32R of the sorted 128
+    warp_merge_into_list<R>(L, k, cand);
+    return;
+  }
+  if (*nb + npass > 32) warp_flush_buffer_R<R>(L, B, nb, k);
+  int off = *nb;
+#pragma unroll
+  for (int m = 0; m < 4; ++m) {
+    const uint32_t bm = __ballot_sync(MV_FULL, pass[m]);
+    if (pass[m]) B[off + __popc(bm & ((1u << lane) - 1))] = ((uint64_t)k32[m] << 32) | low(m * 32 + lane);
+    off += __popc(bm);
+  }
+  __syncwarp();
+  if (lane == 0) *nb = off;
+  __syncwarp();
+}
+
 // Block-wide bitonic sort of n (power of two) u64 keys in shared memory, ascending.
 __device__ __forceinline__ void block_bitonic_sort(uint64_t* a, int n) {
   for (int size = 2; size <= n; size <<= 1) {
@@ -483,8 +551,11 @@ struct Bucketing {
 // ra != nullptr: the pairs of query q with probe rank < ra[q] form a first phase (virtual lists
 // 0..nlist-1, work items first) and the others a second (virtual lists nlist..2*nlist-1); arrays
 // are then sized for 2*nlist lists.
+// qcfg (device) = {query chunk, query planes} (launch_scan_cfg)
 cudaError_t launch_bucket(const int32_t* probes, int64_t nq, int npb, int nlist, const int64_t* list_off, int k,
-                          int qchunk, const int32_t* ra, const Bucketing& b, cudaStream_t st);
+                          const int32_t* qcfg, const int32_t* ra, const Bucketing& b, cudaStream_t st);
+cudaError_t launch_scan_cfg(const int* qlo_any, int qc_exact, int p_exact, int qc_split, int p_split, int32_t* qcfg,
+                            cudaStream_t st);
 // ra[q] = the fewest nearest lists of q holding >= need candidates (<= npb)
 cudaError_t launch_seed_ranks(const int32_t* probes, int64_t nq, int npb, const int64_t* list_off, int64_t need,
                               int32_t* ra, cudaStream_t st);
@@ -523,6 +594,8 @@ cudaError_t launch_scan(const ScanArgs& a, cudaStream_t st);
 // k_scan_tc.cu (tcgen05 path): a filter-and-emit scan run in two phases
 struct TcScanParams {
   int type, metric, dpad, k, npb, qchunk, nchunks, nstage, ncol, tmem_cols;
+  int qchunk_split;        // FLAT: queries per work item when the queries need the lo plane (P = 2)
+  const int32_t* cfg;      // device {query chunk, planes} of this search (launch_scan_cfg)
   int nlist;               // virtual list v >= nlist is list v - nlist (phase-B pairs)
   int phase;               // 0: seeding phase A (emit every candidate); 1: phase B (emit keys < tau_q)
   int64_t nq;              // FLAT query planes are plane-major [2][nq][dpad]
@@ -566,16 +639,19 @@ struct CoarseParams {
 bool coarse_tc_plan(int dpad, int nprobe, int64_t nq, int nsm, CoarseParams& p);
 cudaError_t launch_coarse_tc(const CUtensorMap* cmap, const CUtensorMap* qmap, const CoarseParams& p, int64_t nq,
                              cudaStream_t st);
-cudaError_t launch_hilo(const float* x, int64_t n, int d, int dpad, float* out, cudaStream_t st);
+// plane-major tf32 split of n rows; *lo_any (nullable) |= 1 when some lo element is nonzero
+cudaError_t launch_hilo(const float* x, int64_t n, int d, int dpad, float* out, int* lo_any, cudaStream_t st);
 
 // k_select.cu
 // final select over the pairs of each query; with tau != nullptr instead: tau[q] = the k-th best
-// key over the first nuse[q] pairs of query q (left untouched when they hold fewer than k)
+// key over the first nuse[q] pairs of query q (left untouched when they hold fewer than k).
+// tmax bounds the candidates of one query; over (nq bytes, nullable) is scratch for k > 256.
 cudaError_t launch_final_select(const int64_t* poff, const int32_t* pcnt, const uint64_t* part, int64_t nq, int npb,
                                 int k, int metric, const int64_t* sorted_ids, float* out_d, int64_t* out_i,
-                                cudaStream_t st);
+                                int64_t tmax, uint8_t* over, cudaStream_t st);
 cudaError_t launch_tau_select(const int64_t* poff, const int32_t* pcnt, const uint64_t* part, int64_t nq, int npb,
-                              const int32_t* nuse, int k, uint64_t* tau, cudaStream_t st);
+                              const int32_t* nuse, int k, uint64_t* tau, int64_t tmax, uint8_t* over,
+                              cudaStream_t st);
 cudaError_t launch_fill_pad(int64_t n, int metric, float* d, int64_t* i, cudaStream_t st);
 cudaError_t launch_merge2(int metric, const float* ad, const int64_t* ai, const float* bd, const int64_t* bi,
                           int64_t nq, int k, float* od, int64_t* oi, cudaStream_t st);

@@ -84,6 +84,46 @@ def test_flat_l2_sift_conditional(n, nlist, nprobe, nq, k):
     assert frac == 1.0  # integer data: no ties can be broken differently except exact ties by id
 
 
+@pytest.mark.parametrize("metric", ["l2", "ip"])
+def test_flat_tc_fractional_queries(metric):
+    """Integer (tf32-exact) base data with fractional queries: the tensor-core scan must take the
+    two-plane (hi/lo) query split instead of the one-plane shape used for tf32-exact queries."""
+    X, Q = _sift(15_000, 130)
+    Q = Q * 0.7311 + 0.377  # not tf32-representable
+    ids = G.permuted_ids(15_000, seed=5)
+    C = kmeans(X, 128, iters=5)
+    ix = _build(X, ids, C, metric, "flat")
+    mo = O.L2 if metric == "l2" else O.IP
+    # the fp32 expansion ||q||^2 + ||x||^2 - 2 q.x (and the fp32 MMA accumulation of q.x) carries an
+    # absolute error proportional to the norms, not to the distance (DESIGN.md §6)
+    atol = 2e-6 * float((Q * Q).sum(1).max() + (X * X).sum(1).max())
+    frac, _, _ = _run_conditional(ix, X, ids, C, Q, 10, 9, mo, O.FLAT, atol=atol)
+    assert ix.describe()["last_scan"] == "tcgen05.tf32"
+    assert frac > 0.999
+
+
+@pytest.mark.parametrize("nprobe,metric", [(7, "l2"), (33, "l2"), (64, "ip"), (100, "l2"), (128, "ip")])
+def test_coarse_probe_sets(nprobe, metric):
+    """a2+a3 on the tensor cores: the probe sets (best-first order included) equal the oracle's
+    fp64 top-nprobe modulo scores tied within 1e-5, across the nprobe <= 32, <= 64 and <= 128
+    selection shapes, with fractional (two-plane) queries."""
+    X, Q = _sift(20_000, 150)
+    Q = Q * 0.93 + 0.21
+    C = kmeans(X, 1000, iters=3)
+    Index, _ = _mv()
+    ix = Index(128, metric, "flat", 1000)
+    ix.set_centroids(C.cuda())
+    P = ix.search_probes(Q.cuda(), nprobe).cpu().numpy()
+    assert ix.describe()["last_coarse"] == "tcgen05.tf32"
+    mo = O.L2 if metric == "l2" else O.IP
+    check_probes(P, Q.numpy(), C.numpy(), nprobe, mo)
+    # best-first: the GPU's own order is non-decreasing in the fp64 score
+    sc = np.stack([O.distances(Q.numpy()[i], C.numpy(), mo)[P[i]] for i in range(len(P))])
+    if mo == O.IP:
+        sc = -sc
+    assert (np.diff(sc, axis=1) >= -1e-5 * np.abs(sc[:, 1:])).all()
+
+
 def test_flat_ip_deep_conditional():
     X, Q = _deep(20_000, 150)
     ids = torch.arange(20_000, dtype=torch.int64) * 2 + 1
