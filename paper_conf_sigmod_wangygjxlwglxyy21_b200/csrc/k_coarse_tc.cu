@@ -1,17 +1,24 @@
-// k_coarse_tc.cu -- §8 rows a2 + a3 on the tensor cores: the queries x centroids contraction with
-// the per-query top-nprobe fused into its epilogue (the score matrix never reaches HBM).
+// k_coarse_tc.cu -- §8 rows a2 + a3: the queries x centroids contraction on the tensor cores and
+// the per-query top-nprobe.
 //
 // PAPER.md:523-529 (§3.1) step (1): "find the closest nprobe buckets based on the distance between
 // q and the centroid of each bucket"; PAPER.md:838-843 (§3.4): this step "has a much higher
 // computation-to-I/O ratio than step 2 ... all the queries compare against the same K centroids".
 //
-// CTA = one block of NQB queries (B operand: tf32 hi/lo planes, loaded once by TMA) streaming all
-// centroid tiles (A operand: 128 centroids, tf32 hi and lo planes, TMA ring).  Per K-step two MMAs:
-//   D[:, 0:2NQB] (=) C_hi . [Q_hi ; Q_lo]^T        D[:, 0:NQB] += C_lo . Q_hi^T
-// so dot = D[:, j] + D[:, NQB + j] = q.c up to the dropped lo x lo term (~2^-22 relative).
-// Score = ||c||^2 - 2 q.c (L2) or -q.c (IP), key = (score key << 32) | centroid id; the epilogue
-// (8 warps, two per TMEM lane quarter) transposes the tile through shared memory and folds it into
-// each query's running top-nprobe with warp_select_tile (shared with the list scan).
+// k_coarse_gemm: CTA = one block of NQB queries (B operand: tf32 hi/lo planes, loaded once by TMA)
+// x a range of centroid tiles (A operand: 128 centroids, tf32 hi and lo planes, TMA ring).  Per
+// K-step two MMAs:  D[:, 0:2NQB] (=) C_hi . [Q_hi ; Q_lo]^T   and   D[:, 0:NQB] += C_lo . Q_hi^T,
+// so q.c = D[:, j] + D[:, NQB + j] up to the dropped lo x lo term (~2^-22 relative).  The epilogue
+// (8 warps, two per TMEM lane quarter) writes the score s(q, c) = ||c||^2 - 2 q.c (L2) or -q.c
+// (IP) to S[q][c] (coalesced: a warp's lanes are 32 consecutive centroids).
+// k_probe_select: one warp per query over its row of S -- pass 1 keeps every lane's R smallest
+// keys (key = score key << 32 | centroid id, so ties go to the smaller id), whose nprobe-th
+// smallest bounds the answer; pass 2 streams the keys at or below the bound through a 32-entry
+// staging buffer into a sorted register list (sort-32 + bitonic merge).
+//
+// (Round 1 fused the selection into the GEMM epilogue; with 10 warps per SM that epilogue was
+// latency-bound on the per-tile folds.  Writing S costs 2 x nq x nlist x 4 B of HBM traffic --
+// 0.33 GB for configs[1] -- and buys a selection kernel at full occupancy.)
 #include "mv_internal.cuh"
 #include "sm100.cuh"
 
@@ -21,37 +28,25 @@ using namespace sm100;
 namespace {
 constexpr int kCEpi = 8;
 constexpr int kCThreads = 64 + 32 * kCEpi;  // warp 0 TMA, warp 1 MMA, warps 2..9 epilogue
-constexpr int kCDLD = 129;
-
-__device__ __forceinline__ void cbar(int id, int n) { asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory"); }
 }  // namespace
 
-template <int NQB>
-constexpr uint32_t coarse_tmem_cols() {
-  return 4 * NQB <= 128 ? 128 : (4 * NQB <= 256 ? 256 : 512);
-}
-
-template <int NQB>
 __global__ void __launch_bounds__(kCThreads, 1)
-    k_coarse_tc(const __grid_constant__ CUtensorMap cmap, const __grid_constant__ CUtensorMap qmap, const CoarseParams p) {
+    k_coarse_gemm(const __grid_constant__ CUtensorMap cmap, const __grid_constant__ CUtensorMap qmap,
+                  const CoarseParams p) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~(uintptr_t)1023);
   constexpr int ATOM = 128;            // tf32: 32 fp32 per 128-B swizzle atom row
   constexpr int ABYTES = 128 * ATOM;   // one 128-centroid chunk of one plane
-  constexpr int BROWS = 2 * NQB;       // hi rows then lo rows
-  const int nchunks = p.nchunks, nstage = p.nstage, nprobe = p.nprobe;
-  const int ntiles = (p.nlist + 127) >> 7;
-  const int q0 = blockIdx.x * NQB;
+  const int NQB = p.nqb, BROWS = 2 * NQB;  // hi rows then lo rows
+  const int nchunks = p.nchunks, nstage = p.nstage;
+  const int ntiles_all = (p.nlist + 127) >> 7;
+  const int qb = blockIdx.x / p.csplit, cs = blockIdx.x % p.csplit;
+  const int t0 = (int)((int64_t)ntiles_all * cs / p.csplit), t1 = (int)((int64_t)ntiles_all * (cs + 1) / p.csplit);
+  const int q0 = qb * NQB;
 
   uint8_t* Bs = sm;                                       // nchunks x BROWS x 128 B
   uint8_t* As = Bs + nchunks * BROWS * ATOM;              // nstage x (hi chunk, lo chunk)
-  uint32_t* Dt = reinterpret_cast<uint32_t*>(As + nstage * 2 * ABYTES);  // NQB x kCDLD
-  uint64_t* lists = reinterpret_cast<uint64_t*>(Dt + NQB * kCDLD + (NQB * kCDLD & 1));  // NQB x nprobe
-  uint64_t* scratch = lists + NQB * nprobe;               // 32 per epilogue warp
-  uint64_t* cbuf = scratch + 32 * kCEpi;                  // NQB x 32 survivor buffers (nprobe <= 32)
-  int* cnb = reinterpret_cast<int*>(cbuf + NQB * 32);     // NQB buffer counts
-  uint32_t* cbnd = reinterpret_cast<uint32_t*>(cnb + NQB);  // NQB running bounds
-  uint64_t* bars = reinterpret_cast<uint64_t*>(cbnd + NQB);
+  uint64_t* bars = reinterpret_cast<uint64_t*>(As + nstage * 2 * ABYTES);
   uint64_t* full_a = bars;
   uint64_t* empty_a = bars + nstage;
   uint64_t* full_b = empty_a + nstage;
@@ -73,7 +68,7 @@ __global__ void __launch_bounds__(kCThreads, 1)
     fence_mbar_init();
   }
   if (warp == 1) {
-    tmem_alloc(tslot, coarse_tmem_cols<NQB>());
+    tmem_alloc(tslot, p.tmem_cols);
     tmem_relinquish();
   }
   if (warp == 0 && lane == 0) {
@@ -91,10 +86,10 @@ __global__ void __launch_bounds__(kCThreads, 1)
       mbar_expect_tx(full_b, nchunks * BROWS * ATOM);
       for (int c = 0; c < nchunks; ++c) {
         tma_load_2d(Bs + c * BROWS * ATOM, &qmap, full_b, c * 32, q0);
-        tma_load_2d(Bs + c * BROWS * ATOM + NQB * ATOM, &qmap, full_b, c * 32, p.nq + q0);
+        tma_load_2d(Bs + c * BROWS * ATOM + NQB * ATOM, &qmap, full_b, c * 32, (int)p.nq + q0);
       }
       uint32_t it = 0;
-      for (int t = 0; t < ntiles; ++t)
+      for (int t = t0; t < t1; ++t)
         for (int c = 0; c < nchunks; ++c, ++it) {
           const uint32_t s = it % nstage, r = it / nstage;
           mbar_wait(&empty_a[s], (r & 1) ^ 1);
@@ -109,9 +104,9 @@ __global__ void __launch_bounds__(kCThreads, 1)
       tc_fence_after();
       const uint32_t id_full = idesc_tf32(BROWS), id_hi = idesc_tf32(NQB);
       uint32_t it = 0;
-      for (int t = 0; t < ntiles; ++t) {
-        const uint32_t a = t & 1;
-        mbar_wait(&tempty[a], ((t >> 1) & 1) ^ 1);
+      for (int t = t0, tl = 0; t < t1; ++t, ++tl) {
+        const uint32_t a = tl & 1;
+        mbar_wait(&tempty[a], ((tl >> 1) & 1) ^ 1);
         tc_fence_after();
         const uint32_t d = tmem + a * 2 * NQB;
         for (int c = 0; c < nchunks; ++c, ++it) {
@@ -131,108 +126,139 @@ __global__ void __launch_bounds__(kCThreads, 1)
       }
     }
   } else {
-    // ------------------------------------------------------------------ epilogue
+    // ------------------------------------------------------------------ epilogue: scores -> S
     const int ew = warp - 2;             // 0..7
     const int quarter = warp & 3;
     const int half = ew >> 2;
     const int row = quarter * 32 + lane;  // centroid within the tile
-    const int et = threadIdx.x - 64;
-    uint64_t* wscr = scratch + ew * 32;
     const int nqv = (int)min64(NQB, p.nq - q0);
-    for (int i = et; i < NQB * nprobe; i += 32 * kCEpi) lists[i] = MV_KEY_PAD;
-    for (int i = et; i < NQB; i += 32 * kCEpi) {
-      cnb[i] = 0;
-      cbnd[i] = 0xffffffffu;
-    }
-    float cn_next = (row < p.nlist && p.metric == MV_L2) ? __ldg(p.cnorm + row) : 0.0f;
-    cbar(1, 32 * kCEpi);
-    for (int t = 0; t < ntiles; ++t) {
-      const uint32_t a = t & 1;
+    float* S = p.S + (int64_t)q0 * p.lds;
+    for (int t = t0, tl = 0; t < t1; ++t, ++tl) {
+      const uint32_t a = tl & 1;
       const int cid = t * 128 + row;
       const bool valid = cid < p.nlist;
-      const float cn = cn_next;
-      const int nid = cid + 128;
-      cn_next = (nid < p.nlist && p.metric == MV_L2) ? __ldg(p.cnorm + nid) : 0.0f;  // prefetch next tile
-      mbar_wait(&tfull[a], (t >> 1) & 1);
+      const float cn = (valid && p.metric == MV_L2) ? __ldg(p.cnorm + cid) : 0.0f;
+      mbar_wait(&tfull[a], (tl >> 1) & 1);
       tc_fence_after();
       const uint32_t tb = tmem + a * 2 * NQB + ((uint32_t)(quarter * 32) << 16);
-#pragma unroll
       for (int qc = half * 16; qc < ((p.dbg & 2) ? 0 : NQB); qc += 32) {
         uint32_t rh[16], rl[16];
         tmem_ld16(tb + qc, rh);
         tmem_ld16(tb + NQB + qc, rl);
         tmem_wait_ld();
+        if (valid) {
 #pragma unroll
-        for (int j = 0; j < 16; ++j) {
-          const float dot = __uint_as_float(rh[j]) + __uint_as_float(rl[j]);
-          const float sc = p.metric == MV_L2 ? cn - 2.0f * dot : -dot;
-          Dt[(qc + j) * kCDLD + row] = valid ? f2key(sc) : 0xffffffffu;
+          for (int j = 0; j < 16; ++j) {
+            const float dot = __uint_as_float(rh[j]) + __uint_as_float(rl[j]);
+            const float sc = p.metric == MV_L2 ? cn - 2.0f * dot : -dot;
+            if (qc + j < nqv) S[(int64_t)(qc + j) * p.lds + cid] = sc;
+          }
         }
       }
       tc_fence_before();
       __syncwarp();
       if (lane == 0) mbar_arrive(&tempty[a]);
-      cbar(1, 32 * kCEpi);
-      const uint32_t cbase = t * 128;
-      if (nprobe <= 32) {
-        constexpr int G = 4;
-        for (int j0 = ew; j0 < ((p.dbg & 1) ? 0 : nqv); j0 += kCEpi * G) {
-          const int nvalid = min(G, (nqv - j0 + kCEpi - 1) / kCEpi);
-          warp_filter_group<G>(
-              nvalid, nprobe, [&](int g, int m) { return Dt[(j0 + g * kCEpi) * kCDLD + m * 32 + lane]; },
-              [&](int g, uint64_t*& L, uint64_t*& B, int*& nb, uint32_t*& bnd, uint64_t& li) {
-                const int j = j0 + g * kCEpi;
-                L = lists + (int64_t)j * nprobe;
-                B = cbuf + j * 32;
-                nb = cnb + j;
-                bnd = cbnd + j;
-                li = MV_KEY_PAD;
-              },
-              [&](int, int v) { return cbase + (uint32_t)v; }, [](int, uint32_t) {}, wscr);
-        }
-      } else {
-        // 32 < nprobe <= 128: filter against the list's nprobe-th best, buffered merges
-        for (int j = ew; j < ((p.dbg & 1) ? 0 : nqv); j += kCEpi) {
-          uint64_t* L = lists + (int64_t)j * nprobe;
-          const uint32_t thr32 = (uint32_t)(L[nprobe - 1] >> 32);
-          uint32_t k32[4];
-          bool pass[4];
-          int npass = 0;
-#pragma unroll
-          for (int m = 0; m < 4; ++m) {
-            k32[m] = Dt[j * kCDLD + m * 32 + lane];
-            pass[m] = k32[m] != 0xffffffffu && k32[m] <= thr32;
-            npass += __popc(__ballot_sync(MV_FULL, pass[m]));
-          }
-          if (npass == 0) continue;
-          auto low = [&](int v) { return cbase + (uint32_t)v; };
-          if (nprobe <= 64) warp_collect_R<2>(L, cbuf + j * 32, cnb + j, nprobe, k32, pass, npass, low);
-          else warp_collect_R<4>(L, cbuf + j * 32, cnb + j, nprobe, k32, pass, npass, low);
-        }
-      }
-      cbar(1, 32 * kCEpi);
-    }
-    for (int j = ew; j < nqv; j += kCEpi) {
-      uint64_t* L = lists + (int64_t)j * nprobe;
-      if (nprobe <= 32) warp_flush_buffer(L, cbuf + j * 32, cnb + j, cbnd + j, nprobe, MV_KEY_PAD);
-      else if (nprobe <= 64) warp_flush_buffer_R<2>(L, cbuf + j * 32, cnb + j, nprobe);
-      else warp_flush_buffer_R<4>(L, cbuf + j * 32, cnb + j, nprobe);
-    }
-    cbar(1, 32 * kCEpi);
-    for (int i = et; i < nqv * nprobe; i += 32 * kCEpi) {
-      const int j = i / nprobe, r = i - j * nprobe;
-      const uint64_t key = lists[i];  // PAD only in MV_COARSE_DEBUG runs: keep the probe ids in range
-      p.probes[(int64_t)(q0 + j) * nprobe + r] = key == MV_KEY_PAD ? r % p.nlist : (int32_t)(uint32_t)(key & 0xffffffffu);
     }
   }
   __syncthreads();
   if (warp == 1) {
     tc_fence_after();
-    tmem_dealloc(tmem, coarse_tmem_cols<NQB>());
+    tmem_dealloc(tmem, p.tmem_cols);
   }
 }
 
-// plane-major tf32 split: out[0][r][:] = hi(x_r), out[1][r][:] = x_r - hi(x_r)
+// per-query top-nprobe of a score row (R = ceil(nprobe / 32) <= 4); see the file comment
+template <int R>
+__global__ void __launch_bounds__(256) k_probe_select(const float* __restrict__ S, int64_t lds, int64_t nq, int nlist,
+                                                      int nprobe, int32_t* __restrict__ probes) {
+  __shared__ uint64_t stage_all[8][64];
+  const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+  const int64_t q = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  if (q >= nq) return;
+  uint64_t* stage = stage_all[wib];
+  const float* s = S + q * lds;
+  auto keyof = [&](float v, int c) { return ((uint64_t)f2key(v) << 32) | (uint32_t)c; };
+  // pass 1: each lane's R smallest keys (sorted, t[0] smallest)
+  uint64_t t[R];
+#pragma unroll
+  for (int r = 0; r < R; ++r) t[r] = MV_KEY_PAD;
+  auto offer = [&](uint64_t key) {
+    if (key < t[R - 1]) {
+      t[R - 1] = key;
+#pragma unroll
+      for (int r = R - 1; r > 0; --r)
+        if (t[r] < t[r - 1]) {
+          const uint64_t x = t[r];
+          t[r] = t[r - 1];
+          t[r - 1] = x;
+        }
+    }
+  };
+  const int n4 = nlist & ~3;
+  for (int c = 4 * lane; c < n4; c += 128) {
+    const float4 v = *reinterpret_cast<const float4*>(s + c);
+    offer(keyof(v.x, c));
+    offer(keyof(v.y, c + 1));
+    offer(keyof(v.z, c + 2));
+    offer(keyof(v.w, c + 3));
+  }
+  for (int c = n4 + lane; c < nlist; c += 32) offer(keyof(s[c], c));
+  // bound: the nprobe-th smallest of the 32R lane keys (nprobe distinct keys are <= it)
+  warp_bitonic_sort<R>(t);
+  uint64_t bsel = t[0];
+#pragma unroll
+  for (int r = 1; r < R; ++r)
+    if (r == ((nprobe - 1) >> 5)) bsel = t[r];
+  const uint64_t bound = shfl64(bsel, (nprobe - 1) & 31);
+  // pass 2: keys <= bound -> staging -> sorted list L (32R, L[r] holds element r*32 + lane)
+  uint64_t L[R];
+#pragma unroll
+  for (int r = 0; r < R; ++r) L[r] = MV_KEY_PAD;
+  int ns = 0;
+  auto flush32 = [&]() {
+    uint64_t c[R];
+    uint64_t c1[1] = {lane < ns ? stage[lane] : MV_KEY_PAD};
+    warp_bitonic_sort<1>(c1);
+    c[0] = c1[0];
+#pragma unroll
+    for (int r = 1; r < R; ++r) c[r] = MV_KEY_PAD;
+    warp_merge_smallest<R>(L, c);
+    const int rest = ns > 32 ? ns - 32 : 0;
+    const uint64_t mv = lane < rest ? stage[32 + lane] : 0;
+    __syncwarp();
+    if (lane < rest) stage[lane] = mv;
+    __syncwarp();
+    ns = rest;
+  };
+  auto take = [&](uint64_t key) {
+    const bool ps = key <= bound;
+    const uint32_t m = __ballot_sync(MV_FULL, ps);
+    if (ps) stage[ns + __popc(m & ((1u << lane) - 1))] = key;
+    ns += __popc(m);
+    __syncwarp();
+    if (ns >= 32) flush32();
+  };
+  for (int c0 = 0; c0 < n4; c0 += 128) {
+    const int c = c0 + 4 * lane;
+    float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
+    if (c < n4) v = *reinterpret_cast<const float4*>(s + c);
+    take(c < n4 ? keyof(v.x, c) : MV_KEY_PAD);
+    take(c < n4 ? keyof(v.y, c + 1) : MV_KEY_PAD);
+    take(c < n4 ? keyof(v.z, c + 2) : MV_KEY_PAD);
+    take(c < n4 ? keyof(v.w, c + 3) : MV_KEY_PAD);
+  }
+  for (int c0 = n4; c0 < nlist; c0 += 32) {
+    const int c = c0 + lane;
+    take(c < nlist ? keyof(s[c], c) : MV_KEY_PAD);
+  }
+  if (ns > 0) flush32();
+#pragma unroll
+  for (int r = 0; r < R; ++r) {
+    const int i = r * 32 + lane;
+    if (i < nprobe) probes[q * nprobe + i] = (int32_t)(uint32_t)(L[r] & 0xffffffffu);
+  }
+}
+
 // tf32 round-to-nearest (ties away): the value with the low 13 mantissa bits cleared nearest to v
 __device__ __forceinline__ float tf32_rn(float v) {
   const uint32_t b = __float_as_uint(v);
@@ -265,57 +291,55 @@ cudaError_t launch_hilo(const float* x, int64_t n, int d, int dpad, float* out, 
   return cudaGetLastError();
 }
 
-static int coarse_fixed_smem(int nqb, int nchunks, int nprobe) {
-  return nchunks * 2 * nqb * 128 + nqb * kCDLD * 4 + 8 + nqb * nprobe * 8 + 32 * kCEpi * 8 + nqb * 32 * 8 + nqb * 8 + 256;
-}
-
-// Query-block size: the one that minimises (waves x block size) -- a second, mostly empty wave
-// doubles the coarse time -- among the shapes whose shared memory fits with >= 2 centroid stages.
-bool coarse_tc_plan(int dpad, int nprobe, int64_t nq, int nsm, CoarseParams& p) {
+// Plan: the query-block size NQB (multiple of 16, <= 128) and centroid split that minimise
+// (waves x per-CTA work) on nsm SMs, with >= 2 centroid stages in shared memory.
+bool coarse_tc_plan(int dpad, int nprobe, int64_t nq, int nlist, int nsm, CoarseParams& p) {
   if (dpad % 32 != 0 || nprobe > 128) return false;
   p.nchunks = dpad / 32;
   p.nprobe = nprobe;
-  const int budget = 227 * 1024 - 1024;
+  const int budget = 227 * 1024 - 1024 - 256;
   const int stage = 2 * 128 * 128;
-  int best = -1;
-  int64_t best_cost = 0;
-  for (int nqb : {32, 48, 64, 80}) {
-    if (nprobe > 32 && nqb > 32) continue;
-    const int fixed = coarse_fixed_smem(nqb, p.nchunks, nprobe);
+  const int ntiles = (nlist + 127) / 128;
+  int64_t best_cost = -1;
+  for (int nqb = 32; nqb <= 128; nqb += 16) {
+    const int fixed = p.nchunks * 2 * nqb * 128;
     if ((budget - fixed) / stage < 2) continue;
     const int64_t blocks = (nq + nqb - 1) / nqb;
-    const int64_t cost = ((blocks + nsm - 1) / nsm) * (int64_t)(nqb + 32);  // + fixed per-CTA streaming
-    if (best < 0 || cost < best_cost) {
-      best = nqb;
-      best_cost = cost;
+    for (int cs = 1; cs <= std::min(8, ntiles); ++cs) {
+      const int64_t units = blocks * cs;
+      const int64_t waves = (units + nsm - 1) / nsm;
+      // per-CTA: the query block load + its share of centroid tiles x (MMA/epilogue ~ nqb + stream)
+      const int64_t cost = waves * (4 * p.nchunks + (int64_t)((ntiles + cs - 1) / cs) * (nqb + 48));
+      if (best_cost < 0 || cost < best_cost) {
+        best_cost = cost;
+        p.nqb = nqb;
+        p.csplit = cs;
+      }
     }
   }
-  if (best < 0) return false;
-  p.nqb = best;
-  const int fixed = coarse_fixed_smem(best, p.nchunks, nprobe);
-  p.nstage = std::min(4, (budget - fixed) / stage);
-  p.smem_total = fixed + p.nstage * stage + 1024;
+  if (best_cost < 0) return false;
+  const int fixed = p.nchunks * 2 * p.nqb * 128;
+  p.nstage = std::min(6, (budget - fixed) / stage);
+  p.smem_total = fixed + p.nstage * stage + 256 + 1024;
+  int cols = 32;
+  while (cols < 4 * p.nqb) cols <<= 1;
+  p.tmem_cols = cols;
   return p.smem_total <= 227 * 1024;
-}
-
-template <int NQB>
-static cudaError_t run_coarse_tc(const CUtensorMap* cmap, const CUtensorMap* qmap, const CoarseParams& p, unsigned grid,
-                                 cudaStream_t st) {
-  cudaError_t e = cudaFuncSetAttribute(k_coarse_tc<NQB>, cudaFuncAttributeMaxDynamicSharedMemorySize, p.smem_total);
-  if (e != cudaSuccess) return e;
-  k_coarse_tc<NQB><<<grid, kCThreads, p.smem_total, st>>>(*cmap, *qmap, p);
-  return cudaGetLastError();
 }
 
 cudaError_t launch_coarse_tc(const CUtensorMap* cmap, const CUtensorMap* qmap, const CoarseParams& p, int64_t nq,
                              cudaStream_t st) {
-  const unsigned grid = (unsigned)((nq + p.nqb - 1) / p.nqb);
-  switch (p.nqb) {
-    case 32: return run_coarse_tc<32>(cmap, qmap, p, grid, st);
-    case 48: return run_coarse_tc<48>(cmap, qmap, p, grid, st);
-    case 64: return run_coarse_tc<64>(cmap, qmap, p, grid, st);
-    default: return run_coarse_tc<80>(cmap, qmap, p, grid, st);
-  }
+  const unsigned grid = (unsigned)(((nq + p.nqb - 1) / p.nqb) * p.csplit);
+  cudaError_t e = cudaFuncSetAttribute(k_coarse_gemm, cudaFuncAttributeMaxDynamicSharedMemorySize, p.smem_total);
+  if (e != cudaSuccess) return e;
+  k_coarse_gemm<<<grid, kCThreads, p.smem_total, st>>>(*cmap, *qmap, p);
+  if ((e = cudaGetLastError()) != cudaSuccess) return e;
+  const unsigned g2 = (unsigned)((nq * 32 + 255) / 256);
+  const int R = (p.nprobe + 31) / 32;
+  if (R <= 1) k_probe_select<1><<<g2, 256, 0, st>>>(p.S, p.lds, nq, p.nlist, p.nprobe, p.probes);
+  else if (R == 2) k_probe_select<2><<<g2, 256, 0, st>>>(p.S, p.lds, nq, p.nlist, p.nprobe, p.probes);
+  else k_probe_select<4><<<g2, 256, 0, st>>>(p.S, p.lds, nq, p.nlist, p.nprobe, p.probes);
+  return cudaGetLastError();
 }
 
 }  // namespace mv

@@ -161,13 +161,14 @@ void free_storage(mv_index* ix) {
 
 // a2 + a3: tcgen05 coarse with fused top-nprobe when the shapes fit, else the SIMT kernel
 static cudaError_t run_coarse(mv_index* ix, const float* qpad, const float* qhl, int64_t nq, int npb, int32_t* P,
-                              cudaStream_t st) {
+                              Scratch& s, cudaStream_t st) {
   CoarseParams cp;
   const char* force = getenv("MV_FORCE_SIMT");
   int dev = 0, nsm = kNumSMs;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
-  if (npb < ix->nlist && ix->cmap_ok && !(force && force[0] == '1') && coarse_tc_plan(ix->dpad, npb, nq, nsm, cp)) {
+  if (npb < ix->nlist && ix->cmap_ok && !(force && force[0] == '1') &&
+      coarse_tc_plan(ix->dpad, npb, nq, ix->nlist, nsm, cp) && nq <= 0x7fffffffLL - cp.nqb) {
     CUtensorMap qmap;
     if (make_tmap_2d(&qmap, qhl, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, (uint64_t)ix->dpad, 2 * (uint64_t)nq,
                      (uint64_t)ix->dpad * 4, 32, (uint32_t)cp.nqb, CU_TENSOR_MAP_SWIZZLE_128B)) {
@@ -176,6 +177,9 @@ static cudaError_t run_coarse(mv_index* ix, const float* qpad, const float* qhl,
       cp.metric = ix->metric;
       cp.cnorm = ix->cnorm;
       cp.probes = P;
+      cp.lds = (ix->nlist + 3) & ~3;
+      cudaError_t e = s.alloc(&cp.S, (size_t)nq * cp.lds);
+      if (e != cudaSuccess) return e;
       const char* cdbg = getenv("MV_COARSE_DEBUG");
       cp.dbg = cdbg ? atoi(cdbg) : 0;
       ix->last_coarse = "tcgen05.tf32";
@@ -484,7 +488,7 @@ mv_status mv_search_probes(mv_index* ix, const float* queries, int64_t nq, int32
   float* qhl;
   CK(s.alloc(&qhl, (size_t)2 * nq * ix->dpad));
   CK(launch_hilo(q, nq, ix->d, ix->dpad, qhl, nullptr, st));
-  CK(run_coarse(ix, qpad, qhl, nq, npb, P, st));
+  CK(run_coarse(ix, qpad, qhl, nq, npb, P, s, st));
   if (sp) {
     CK(cudaMemcpyAsync(probes, P, sizeof(int32_t) * nq * npb, cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
@@ -533,7 +537,7 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
     CK(s.alloc(&qlo_any, 1));
     CK(cudaMemsetAsync(qlo_any, 0, sizeof(int), st));
     CK(launch_hilo(q, nq, ix->d, dpad, qhl, qlo_any, st));
-    CK(run_coarse(ix, qpad, qhl, nq, npb, P, st));
+    CK(run_coarse(ix, qpad, qhl, nq, npb, P, s, st));
     prof_mark(ix, st);
     // a4 (work-item size depends on the scan implementation's shared-memory plan)
     TcScanParams tp;

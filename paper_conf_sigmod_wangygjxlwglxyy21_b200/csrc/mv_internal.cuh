@@ -628,15 +628,17 @@ cudaError_t launch_qplanes(int type, const float* qpad, int64_t nq, int dpad, co
                            uint8_t* out, float* qscale, double* qa, double* qnorm, cudaStream_t st);
 cudaError_t launch_tf32_check(const float* x, int64_t n, int* flag, cudaStream_t st);
 
-// k_coarse_tc.cu (tcgen05 coarse + fused top-nprobe)
+// k_coarse_tc.cu (tcgen05 coarse GEMM -> score matrix S, then a warp-per-query top-nprobe)
 struct CoarseParams {
   int64_t nq;
-  int nlist, nchunks, nstage, nprobe, nqb, metric, smem_total;
-  int dbg;  // MV_COARSE_DEBUG: 1 skip select, 2 skip epilogue math
+  int nlist, nchunks, nstage, nprobe, nqb, csplit, tmem_cols, metric, smem_total;
+  int dbg;                 // MV_COARSE_DEBUG: 2 skip the score stores
   const float* cnorm;
+  float* S;                // nq x lds scores (lds = roundup(nlist, 4))
+  int64_t lds;
   int32_t* probes;
 };
-bool coarse_tc_plan(int dpad, int nprobe, int64_t nq, int nsm, CoarseParams& p);
+bool coarse_tc_plan(int dpad, int nprobe, int64_t nq, int nlist, int nsm, CoarseParams& p);
 cudaError_t launch_coarse_tc(const CUtensorMap* cmap, const CUtensorMap* qmap, const CoarseParams& p, int64_t nq,
                              cudaStream_t st);
 // plane-major tf32 split of n rows; *lo_any (nullable) |= 1 when some lo element is nonzero
