@@ -3,24 +3,52 @@
 // accessed data vectors as much as possible for multiple queries" (§3.2.1),
 // because in step 2 "different queries do not necessarily access the same buckets"
 // (§3.4).  A counting sort by list id: histogram, exclusive scan, scatter.
-// Also the per-pair candidate-region offsets for the scan's partial top-k output.
+// Also the per-pair candidate-region offsets, the seeding split and the work-item order.
+//
+// One cooperative launch (grid-wide barriers between the steps) replaces a dozen small kernels:
+//   0  zero the counters; the work-item shape {query chunk, planes} (qlo_any decides FLAT's)
+//   1  per query (warp): ra[q] = the fewest nearest lists holding >= need candidates (seeding),
+//      the query's region capacity, and the pair counts per virtual list
+//   2  exclusive scans: pair counts -> bucket offsets (block 0), capacities -> query bases (1)
+//   3  per query: pair region offsets + bucket fill; per virtual list: work-item counts
+//   4  exclusive scan of the work-item counts (block 0)
+//   5  work items (virtual list, first bucket position)
+//   6  longest-first order (block 0, counting sort by cost; seeding phase first)
+#include <cooperative_groups.h>
+
 #include "mv_internal.cuh"
+
+namespace cg = cooperative_groups;
 
 namespace mv {
 
-// Single-CTA exclusive scan (n up to a few million): out[0..n], out[n] = total.
+constexpr int kPlanThreads = 1024;
+
+// Virtual list of pair p = q*npb + r: its list l, or l + nlist for the pairs of the second phase
+// when the seeding phase is on (ra != nullptr): phase A = the ra[q] nearest lists of query q.
+__device__ __forceinline__ int vlist_of(const int32_t* probes, int64_t p, int npb, int nlist, const int32_t* ra) {
+  const int l = probes[p];
+  return (ra && (int)(p % npb) >= ra[p / npb]) ? l + nlist : l;
+}
+
+// Region capacity of a pair: min(capk, |list|) when the SIMT scan selects locally (capk > 0,
+// k <= 1024), else |list| (every candidate that survives the bitset may be emitted).
+__device__ __forceinline__ int64_t pair_cap(int64_t len, int k, int capk) {
+  return (capk > 0 && k <= kLocalSelectMaxK) ? min64(capk, len) : len;
+}
+
+// single-block exclusive scan out[0..n] (out[n] = total) with all kPlanThreads threads
 template <typename T>
-__global__ void __launch_bounds__(1024) k_scan_single(const T* __restrict__ in, int64_t n, T* __restrict__ out) {
-  __shared__ T part[1024];
+__device__ void block_exclusive_scan(const T* __restrict__ in, int64_t n, T* __restrict__ out, T* part) {
   const int tid = threadIdx.x;
-  const int64_t per = (n + 1023) / 1024;
+  const int64_t per = (n + kPlanThreads - 1) / kPlanThreads;
   const int64_t s = tid * per, e = min64(n, s + per);
   T acc = 0;
   for (int64_t i = s; i < e; ++i) acc += in[i];
   part[tid] = acc;
   __syncthreads();
-  for (int off = 1; off < 1024; off <<= 1) {  // Hillis-Steele inclusive scan of 1024 partials
-    T v = tid >= off ? part[tid - off] : (T)0;
+  for (int off = 1; off < kPlanThreads; off <<= 1) {
+    const T v = tid >= off ? part[tid - off] : (T)0;
     __syncthreads();
     part[tid] += v;
     __syncthreads();
@@ -30,238 +58,183 @@ __global__ void __launch_bounds__(1024) k_scan_single(const T* __restrict__ in, 
     out[i] = run;
     run += in[i];
   }
-  if (tid == 1023) out[n] = part[1023];
+  if (tid == kPlanThreads - 1) out[n] = part[kPlanThreads - 1];
+  __syncthreads();
 }
 
-cudaError_t launch_scan_i32(const int32_t* in, int n, int32_t* out, cudaStream_t st) {
-  k_scan_single<int32_t><<<1, 1024, 0, st>>>(in, n, out);
-  return cudaGetLastError();
-}
-cudaError_t launch_scan_i64(const int64_t* in, int64_t n, int64_t* out, cudaStream_t st) {
-  k_scan_single<int64_t><<<1, 1024, 0, st>>>(in, n, out);
-  return cudaGetLastError();
-}
+__global__ void __launch_bounds__(kPlanThreads) k_plan(const PlanArgs a) {
+  cg::grid_group grid = cg::this_grid();
+  __shared__ int64_t part64[kPlanThreads];
+  __shared__ int hist[8192];
+  const int tid = threadIdx.x, lane = tid & 31;
+  const int64_t gtid = blockIdx.x * (int64_t)blockDim.x + tid;
+  const int64_t gthreads = (int64_t)gridDim.x * blockDim.x;
+  const int64_t gwarp = gtid >> 5, gwarps = gthreads >> 5;
+  const int nq_i = (int)a.nq, npb = a.npb, nlist = a.nlist;
+  const int nv = a.split ? 2 * nlist : nlist;
+  const Bucketing& b = a.b;
 
-// Virtual list of pair p = q*npb + r: its list l, or l + nlist for the pairs of the second phase
-// when the seeding phase is on (ra != nullptr): phase A = the ra[q] nearest lists of query q,
-// scanned first so that their k-th best bounds tau_q before the other lists are scanned.
-__device__ __forceinline__ int vlist_of(const int32_t* probes, int64_t p, int npb, int nlist, const int32_t* ra) {
-  const int l = probes[p];
-  return (ra && (int)(p % npb) >= ra[p / npb]) ? l + nlist : l;
-}
-
-__global__ void k_count_pairs(const int32_t* __restrict__ probes, int64_t npairs, int npb, int nlist,
-                              const int32_t* __restrict__ ra, int32_t* counts) {
-  for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < npairs; p += (int64_t)gridDim.x * blockDim.x)
-    atomicAdd(counts + vlist_of(probes, p, npb, nlist, ra), 1);
-}
-
-__global__ void k_bucket_fill(const int32_t* __restrict__ probes, int64_t npairs, int npb, int nlist,
-                              const int32_t* __restrict__ ra, const int32_t* __restrict__ boff, int32_t* bfill,
-                              int32_t* bq) {
-  for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < npairs; p += (int64_t)gridDim.x * blockDim.x) {
-    const int l = vlist_of(probes, p, npb, nlist, ra);
-    const int pos = boff[l] + atomicAdd(bfill + l, 1);
-    bq[pos] = (int32_t)p;
+  // 0 ---------------------------------------------------------------------------------------
+  for (int64_t i = gtid; i < nv; i += gthreads) {
+    b.lcount[i] = 0;
+    b.bfill[i] = 0;
   }
-}
+  if (gtid == 0) {
+    const bool sp = a.qlo_any != nullptr && *a.qlo_any != 0;
+    a.qcfg[0] = sp ? a.qc_split : a.qc_exact;
+    a.qcfg[1] = sp ? a.p_split : a.p_exact;
+    *b.counter = 0;
+  }
+  grid.sync();
+  const int qchunk = a.qcfg[0];
+  int32_t* ra = a.split ? a.ra : nullptr;
 
-// one warp per query: ra[q] = the fewest nearest lists holding >= need candidates (at most npb)
-__global__ void k_seed_ranks(const int32_t* __restrict__ probes, int64_t nq, int npb,
-                             const int64_t* __restrict__ list_off, int64_t need, int32_t* ra) {
-  const int lane = threadIdx.x & 31;
-  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
-  for (int64_t q = warp; q < nq; q += nwarps) {
-    int64_t run = 0;
+  // 1 ---------------------------------------------------------------------------------------
+  for (int64_t q = gwarp; q < nq_i; q += gwarps) {
+    const int32_t* pq = a.probes + q * npb;
+    int64_t run = 0, capsum = 0;
     int r = npb;
+    for (int j0 = 0; j0 < npb; j0 += 32) {
+      const int j = j0 + lane;
+      int64_t len = 0;
+      if (j < npb) {
+        const int l = pq[j];
+        len = a.list_off[l + 1] - a.list_off[l];
+        capsum += pair_cap(len, a.k, a.capk);
+      }
+      int64_t incl = len;
+      for (int o = 1; o < 32; o <<= 1) {
+        const int64_t v = __shfl_up_sync(MV_FULL, incl, o);
+        if (lane >= o) incl += v;
+      }
+      const uint32_t hit = __ballot_sync(MV_FULL, j < npb && run + incl >= a.need);
+      if (hit && r == npb) r = j0 + __ffs(hit);  // ranks 0 .. first hit
+      run += __shfl_sync(MV_FULL, incl, 31);
+    }
+    for (int o = 16; o > 0; o >>= 1) capsum += __shfl_xor_sync(MV_FULL, capsum, o);
+    if (lane == 0) {
+      if (ra) ra[q] = r;
+      b.qtot[q] = capsum;
+    }
+    for (int j = lane; j < npb; j += 32) {
+      const int l = pq[j];
+      atomicAdd(b.lcount + ((ra && j >= r) ? l + nlist : l), 1);
+    }
+  }
+  grid.sync();
+
+  // 2 ---------------------------------------------------------------------------------------
+  if (blockIdx.x == 0) block_exclusive_scan<int32_t>(b.lcount, nv, b.boff, reinterpret_cast<int32_t*>(part64));
+  if (blockIdx.x == gridDim.x - 1) block_exclusive_scan<int64_t>(b.qtot, a.nq, b.qtot + (a.nq + 1), part64);
+  grid.sync();
+
+  // 3 ---------------------------------------------------------------------------------------
+  const int64_t* qbase = b.qtot + (a.nq + 1);
+  for (int64_t q = gwarp; q < nq_i; q += gwarps) {
+    const int32_t* pq = a.probes + q * npb;
+    const int r = ra ? ra[q] : npb;
+    int64_t run = qbase[q];
     for (int j0 = 0; j0 < npb; j0 += 32) {
       const int j = j0 + lane;
       int64_t c = 0;
       if (j < npb) {
-        const int l = probes[q * npb + j];
-        c = list_off[l + 1] - list_off[l];
+        const int l = pq[j];
+        c = pair_cap(a.list_off[l + 1] - a.list_off[l], a.k, a.capk);
+        const int v = (ra && j >= r) ? l + nlist : l;
+        b.bq[b.boff[v] + atomicAdd(b.bfill + v, 1)] = (int32_t)(q * npb + j);
       }
       int64_t incl = c;
       for (int o = 1; o < 32; o <<= 1) {
         const int64_t v = __shfl_up_sync(MV_FULL, incl, o);
         if (lane >= o) incl += v;
       }
-      const uint32_t hit = __ballot_sync(MV_FULL, j < npb && run + incl >= need);
-      if (hit) {
-        r = j0 + __ffs(hit);  // ranks 0 .. first hit
-        break;
-      }
+      if (j < npb) b.poff[q * npb + j] = run + incl - c;
       run += __shfl_sync(MV_FULL, incl, 31);
     }
-    if (lane == 0) ra[q] = r;
   }
-}
+  for (int64_t v = gtid; v < nv; v += gthreads) b.wcount[v] = (b.lcount[v] + qchunk - 1) / qchunk;
+  grid.sync();
 
-// qcfg = {query chunk, query planes}: the split (two-plane) shape when *qlo_any, else the exact one
-__global__ void k_scan_cfg(const int* qlo_any, int qc_exact, int p_exact, int qc_split, int p_split, int32_t* qcfg) {
-  const bool sp = qlo_any != nullptr && *qlo_any != 0;
-  qcfg[0] = sp ? qc_split : qc_exact;
-  qcfg[1] = sp ? p_split : p_exact;
-}
+  // 4 ---------------------------------------------------------------------------------------
+  if (blockIdx.x == 0) block_exclusive_scan<int32_t>(b.wcount, nv, b.woff, reinterpret_cast<int32_t*>(part64));
+  grid.sync();
 
-cudaError_t launch_scan_cfg(const int* qlo_any, int qc_exact, int p_exact, int qc_split, int p_split, int32_t* qcfg,
-                            cudaStream_t st) {
-  k_scan_cfg<<<1, 1, 0, st>>>(qlo_any, qc_exact, p_exact, qc_split, p_split, qcfg);
-  return cudaGetLastError();
-}
+  // 5 ---------------------------------------------------------------------------------------
+  for (int64_t v = gtid; v < nv; v += gthreads) {
+    const int n = b.wcount[v], o = b.woff[v], bb = b.boff[v];
+    for (int c = 0; c < n; ++c) b.witems_unsorted[o + c] = make_int2((int)v, bb + c * qchunk);
+  }
+  grid.sync();
 
-cudaError_t launch_seed_ranks(const int32_t* probes, int64_t nq, int npb, const int64_t* list_off, int64_t need,
-                              int32_t* ra, cudaStream_t st) {
-  if (nq == 0) return cudaSuccess;
-  const int grid = (int)min64(kNumSMs * 8, (nq * 32 + 255) / 256);
-  k_seed_ranks<<<grid, 256, 0, st>>>(probes, nq, npb, list_off, need, ra);
-  return cudaGetLastError();
-}
-
-__global__ void k_work_count(const int32_t* __restrict__ lcount, int nlist, const int32_t* __restrict__ qcfg,
-                             int32_t* wcount) {
-  const int l = blockIdx.x * blockDim.x + threadIdx.x;
-  const int qchunk = qcfg[0];
-  if (l < nlist) wcount[l] = (lcount[l] + qchunk - 1) / qchunk;
-}
-
-__global__ void k_work_fill(const int32_t* __restrict__ wcount, const int32_t* __restrict__ woff,
-                            const int32_t* __restrict__ boff, int nlist, const int32_t* __restrict__ qcfg,
-                            int2* witems) {
-  const int l = blockIdx.x * blockDim.x + threadIdx.x;
-  const int qchunk = qcfg[0];
-  if (l >= nlist) return;
-  const int n = wcount[l], o = woff[l], b = boff[l];
-  for (int c = 0; c < n; ++c) witems[o + c] = make_int2(l, b + c * qchunk);
-}
-
-// Longest-first order for the persistent scan's static round-robin: a single-CTA counting sort of
-// the work items by descending cost key = 64 * tiles + queries (tiles = ceil(|list| / 128)); with
-// the seeding split, every phase-A item (virtual list < nlist) precedes every phase-B item.
-__global__ void __launch_bounds__(1024) k_sort_work(const int2* __restrict__ in, const int32_t* __restrict__ nwork_p,
-                                                    const int32_t* __restrict__ boff, const int64_t* __restrict__ list_off,
-                                                    int nlist, const int32_t* __restrict__ qcfg,
-                                                    int2* __restrict__ out) {
+  // 6 --------------------------------------------------------------------------------------- 
+  // counting sort by descending cost key = 64 * tiles + queries (tiles = ceil(|list| / 128));
+  // every phase-A item (virtual list < nlist) precedes every phase-B item
+  if (blockIdx.x != 0) return;
   constexpr int NB = 8192, HB = 4096;
-  const int qchunk = qcfg[0];
-  __shared__ int hist[NB];
-  __shared__ int part[1024];
-  const int nwork = *nwork_p, tid = threadIdx.x;
-  for (int i = tid; i < NB; i += 1024) hist[i] = 0;
+  const int nwork = b.woff[nv];
+  for (int i = tid; i < NB; i += kPlanThreads) hist[i] = 0;
   __syncthreads();
   auto key = [&](int w) {
-    const int2 it = in[w];
+    const int2 it = b.witems_unsorted[w];
     const int l = it.x >= nlist ? it.x - nlist : it.x;
-    const int nq = min(qchunk, boff[it.x + 1] - it.y);
-    const int64_t len = list_off[l + 1] - list_off[l];
+    const int nqw = min(qchunk, b.boff[it.x + 1] - it.y);
+    const int64_t len = a.list_off[l + 1] - a.list_off[l];
     const int tiles = (int)min64((len + 127) / 128, 63);
-    return (it.x >= nlist ? HB : 0) + HB - 1 - min(HB - 1, tiles * 64 + min(nq, 63));  // descending cost
+    return (it.x >= nlist ? HB : 0) + HB - 1 - min(HB - 1, tiles * 64 + min(nqw, 63));
   };
-  for (int w = tid; w < nwork; w += 1024) atomicAdd(&hist[key(w)], 1);
+  for (int w = tid; w < nwork; w += kPlanThreads) atomicAdd(&hist[key(w)], 1);
   __syncthreads();
-  // exclusive scan of 8192 bins: 8 per thread
   int loc[8], acc = 0;
 #pragma unroll
   for (int j = 0; j < 8; ++j) {
     loc[j] = acc;
     acc += hist[tid * 8 + j];
   }
-  part[tid] = acc;
+  int32_t* p32 = reinterpret_cast<int32_t*>(part64);
+  p32[tid] = acc;
   __syncthreads();
-  for (int off = 1; off < 1024; off <<= 1) {
-    const int v = tid >= off ? part[tid - off] : 0;
+  for (int off = 1; off < kPlanThreads; off <<= 1) {
+    const int v = tid >= off ? p32[tid - off] : 0;
     __syncthreads();
-    part[tid] += v;
+    p32[tid] += v;
     __syncthreads();
   }
-  const int base = tid ? part[tid - 1] : 0;
+  const int base = tid ? p32[tid - 1] : 0;
   __syncthreads();
 #pragma unroll
   for (int j = 0; j < 8; ++j) hist[tid * 8 + j] = base + loc[j];
   __syncthreads();
-  for (int w = tid; w < nwork; w += 1024) out[atomicAdd(&hist[key(w)], 1)] = in[w];
+  for (int w = tid; w < nwork; w += kPlanThreads) b.witems[atomicAdd(&hist[key(w)], 1)] = b.witems_unsorted[w];
 }
 
-cudaError_t launch_bucket(const int32_t* probes, int64_t nq, int npb, int nlist, const int64_t* list_off, int k,
-                          const int32_t* qcfg, const int32_t* ra, const Bucketing& b, cudaStream_t st) {
-  (void)k;
-  const int64_t npairs = nq * npb;
-  const int nv = ra ? 2 * nlist : nlist;  // virtual lists
-  cudaMemsetAsync(b.lcount, 0, sizeof(int32_t) * nv, st);
-  cudaMemsetAsync(b.bfill, 0, sizeof(int32_t) * nv, st);
-  cudaMemsetAsync(b.counter, 0, sizeof(int32_t), st);
-  const int grid = (int)min64(kNumSMs * 8, (npairs + 255) / 256);
-  if (npairs) k_count_pairs<<<grid, 256, 0, st>>>(probes, npairs, npb, nlist, ra, b.lcount);
-  cudaError_t e;
-  if ((e = launch_scan_i32(b.lcount, nv, b.boff, st)) != cudaSuccess) return e;
-  if (npairs) k_bucket_fill<<<grid, 256, 0, st>>>(probes, npairs, npb, nlist, ra, b.boff, b.bfill, b.bq);
-  k_work_count<<<(nv + 255) / 256, 256, 0, st>>>(b.lcount, nv, qcfg, b.wcount);
-  if ((e = launch_scan_i32(b.wcount, nv, b.woff, st)) != cudaSuccess) return e;
-  k_work_fill<<<(nv + 255) / 256, 256, 0, st>>>(b.wcount, b.woff, b.boff, nv, qcfg, b.witems_unsorted);
-  k_sort_work<<<1, 1024, 0, st>>>(b.witems_unsorted, b.woff + nv, b.boff, list_off, nlist, qcfg, b.witems);
+// single-CTA exclusive scan for the add path (n up to a few million)
+template <typename T>
+__global__ void __launch_bounds__(kPlanThreads) k_scan_single(const T* __restrict__ in, int64_t n, T* __restrict__ out) {
+  __shared__ T part[kPlanThreads];
+  block_exclusive_scan<T>(in, n, out, part);
+}
+
+cudaError_t launch_scan_i32(const int32_t* in, int n, int32_t* out, cudaStream_t st) {
+  k_scan_single<int32_t><<<1, kPlanThreads, 0, st>>>(in, n, out);
+  return cudaGetLastError();
+}
+cudaError_t launch_scan_i64(const int64_t* in, int64_t n, int64_t* out, cudaStream_t st) {
+  k_scan_single<int64_t><<<1, kPlanThreads, 0, st>>>(in, n, out);
   return cudaGetLastError();
 }
 
-// Region capacity of pair (q, j): min(capk, |list|) when the SIMT scan selects locally (k <= 1024,
-// capk > 0), else |list| (every candidate that survives the bitset may be emitted).
-__device__ __forceinline__ int64_t pair_cap(int64_t len, int k, int capk) {
-  return (capk > 0 && k <= kLocalSelectMaxK) ? min64(capk, len) : len;
-}
-
-// one warp per query: qtot[q] = sum_j cap(q, j)
-__global__ void k_query_tot(const int32_t* __restrict__ probes, int64_t nq, int npb,
-                            const int64_t* __restrict__ list_off, int k, int capk, int64_t* qtot) {
-  const int lane = threadIdx.x & 31;
-  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
-  for (int64_t q = warp; q < nq; q += nwarps) {
-    int64_t acc = 0;
-    for (int j = lane; j < npb; j += 32) {
-      const int l = probes[q * npb + j];
-      acc += pair_cap(list_off[l + 1] - list_off[l], k, capk);
-    }
-    for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(MV_FULL, acc, o);
-    if (lane == 0) qtot[q] = acc;
+cudaError_t launch_plan(const PlanArgs& a, cudaStream_t st) {
+  static int grid = 0;
+  if (grid == 0) {
+    int dev = 0, nsm = kNumSMs, per = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_plan, kPlanThreads, 0);
+    grid = nsm * std::max(1, std::min(per, 2));
   }
-}
-
-// one warp per query: poff[q*npb + j] = qbase[q] + sum_{j' < j} cap(q, j')
-__global__ void k_pair_off(const int32_t* __restrict__ probes, int64_t nq, int npb, const int64_t* __restrict__ list_off,
-                           int k, int capk, const int64_t* __restrict__ qbase, int64_t* poff) {
-  const int lane = threadIdx.x & 31;
-  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
-  for (int64_t q = warp; q < nq; q += nwarps) {
-    int64_t run = qbase[q];
-    for (int j0 = 0; j0 < npb; j0 += 32) {
-      const int j = j0 + lane;
-      int64_t c = 0;
-      if (j < npb) {
-        const int l = probes[q * npb + j];
-        c = pair_cap(list_off[l + 1] - list_off[l], k, capk);
-      }
-      int64_t incl = c;
-      for (int o = 1; o < 32; o <<= 1) {
-        const int64_t v = __shfl_up_sync(MV_FULL, incl, o);
-        if (lane >= o) incl += v;
-      }
-      if (j < npb) poff[q * npb + j] = run + incl - c;
-      run += __shfl_sync(MV_FULL, incl, 31);
-    }
-  }
-}
-
-cudaError_t launch_pair_offsets(const int32_t* probes, int64_t nq, int npb, const int64_t* list_off, int k, int capk,
-                                const Bucketing& b, cudaStream_t st) {
-  if (nq == 0) return cudaSuccess;
-  const int grid = (int)min64(kNumSMs * 8, (nq * 32 + 255) / 256);
-  int64_t* qbase = b.qtot + (nq + 1);  // second half of the qtot allocation
-  k_query_tot<<<grid, 256, 0, st>>>(probes, nq, npb, list_off, k, capk, b.qtot);
-  cudaError_t e = launch_scan_i64(b.qtot, nq, qbase, st);
-  if (e != cudaSuccess) return e;
-  k_pair_off<<<grid, 256, 0, st>>>(probes, nq, npb, list_off, k, capk, qbase, b.poff);
-  return cudaGetLastError();
+  PlanArgs args = a;
+  void* kargs[] = {&args};
+  return cudaLaunchCooperativeKernel((const void*)k_plan, dim3(grid), dim3(kPlanThreads), kargs, 0, st);
 }
 
 }  // namespace mv

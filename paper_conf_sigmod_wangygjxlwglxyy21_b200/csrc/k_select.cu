@@ -330,73 +330,109 @@ static cudaError_t launch_big_select(const int64_t* poff, const int32_t* pcnt, c
   return cudaGetLastError();
 }
 
-// k <= 32 R: one warp per query, its running best-32R list sorted across registers (element
-// r*32 + lane in best[r]).  The pairs' regions are walked in 32-key chunks (a flattened index over
-// groups of 32 pairs, located by a shuffle binary search; the next chunk's load is issued before
-// the current one is folded); a chunk is skipped unless some key beats the running k-th best, else
-// it is bitonic-sorted and merged into the list.
+// k <= 32 R: one warp per query, two passes over the query's candidates (its pairs' regions,
+// walked in 32-key chunks through a flattened index over groups of 32 pairs located by a shuffle
+// binary search).  Pass 1 keeps every lane's R smallest keys; the k-th smallest of those 32R keys
+// bounds the answer (k distinct keys are at or below it).  Pass 2 streams the keys at or below the
+// bound through a 32-entry staging buffer into a sorted register list (sort-32 + bitonic merge).
 template <int R>
 __global__ void __launch_bounds__(256) k_final_warp(const int64_t* __restrict__ poff, const int32_t* __restrict__ pcnt,
                                                     const uint64_t* __restrict__ part, int64_t nq, int npb, int k,
                                                     int metric, const int64_t* __restrict__ sorted_ids, float* out_d,
                                                     int64_t* out_i, const int32_t* __restrict__ nuse,
                                                     uint64_t* tau_out) {
+  __shared__ uint64_t stage_all[8][64];
   const int lane = threadIdx.x & 31;
   const int64_t q = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   if (q >= nq) return;
+  uint64_t* stage = stage_all[threadIdx.x >> 5];
   const int stride = npb;
   if (nuse) npb = nuse[q];
+  // visit every candidate key of the query, 32 at a time: f(key) with key = PAD past the end
+  auto for_each_chunk = [&](auto&& f) {
+    for (int g = 0; g < npb; g += 32) {
+      const int j = g + lane;
+      const int cnt = j < npb ? pcnt[q * stride + j] : 0;
+      const int64_t off = j < npb ? poff[q * stride + j] : 0;
+      int incl = cnt;
+      for (int o = 1; o < 32; o <<= 1) {
+        const int v = __shfl_up_sync(MV_FULL, incl, o);
+        if (lane >= o) incl += v;
+      }
+      const int excl = incl - cnt;
+      const int T = __shfl_sync(MV_FULL, incl, 31);
+      for (int e0 = 0; e0 < T; e0 += 32) {
+        const int e = e0 + lane;
+        int lo = 0;  // pair holding element e: the largest s with excl[s] <= e
+#pragma unroll
+        for (int step = 16; step > 0; step >>= 1) {
+          const int ex = __shfl_sync(MV_FULL, excl, (lo + step) & 31);
+          if (lo + step < 32 && ex <= e) lo += step;
+        }
+        const int64_t o = __shfl_sync(MV_FULL, off, lo);
+        const int ex = __shfl_sync(MV_FULL, excl, lo);
+        f(e < T ? part[o + (e - ex)] : MV_KEY_PAD);
+      }
+    }
+  };
+  // pass 1: each lane's R smallest keys
+  uint64_t t[R];
+#pragma unroll
+  for (int r = 0; r < R; ++r) t[r] = MV_KEY_PAD;
+  for_each_chunk([&](uint64_t key) {
+    if (key < t[R - 1]) {
+      t[R - 1] = key;
+#pragma unroll
+      for (int r = R - 1; r > 0; --r)
+        if (t[r] < t[r - 1]) {
+          const uint64_t x = t[r];
+          t[r] = t[r - 1];
+          t[r - 1] = x;
+        }
+    }
+  });
+  warp_bitonic_sort<R>(t);
+  uint64_t bsel = t[0];
+#pragma unroll
+  for (int r = 1; r < R; ++r)
+    if (r == ((k - 1) >> 5)) bsel = t[r];
+  const uint64_t bound = shfl64(bsel, (k - 1) & 31);  // PAD when fewer than k candidates
+  // pass 2: keys <= bound -> staging -> sorted list (best[r] holds element r*32 + lane)
   uint64_t best[R];
 #pragma unroll
   for (int r = 0; r < R; ++r) best[r] = MV_KEY_PAD;
-  const int kr = (k - 1) >> 5, kl = (k - 1) & 31;
+  int ns = 0;
+  auto flush32 = [&]() {
+    uint64_t c[R];
+    uint64_t c1[1] = {lane < ns ? stage[lane] : MV_KEY_PAD};
+    warp_bitonic_sort<1>(c1);
+    c[0] = c1[0];
+#pragma unroll
+    for (int r = 1; r < R; ++r) c[r] = MV_KEY_PAD;
+    warp_merge_smallest<R>(best, c);
+    const int rest = ns > 32 ? ns - 32 : 0;
+    const uint64_t mv = lane < rest ? stage[32 + lane] : 0;
+    __syncwarp();
+    if (lane < rest) stage[lane] = mv;
+    __syncwarp();
+    ns = rest;
+  };
+  for_each_chunk([&](uint64_t key) {
+    const bool ps = key != MV_KEY_PAD && key <= bound;
+    const uint32_t m = __ballot_sync(MV_FULL, ps);
+    if (ps) stage[ns + __popc(m & ((1u << lane) - 1))] = key;
+    ns += __popc(m);
+    __syncwarp();
+    if (ns >= 32) flush32();
+  });
+  if (ns > 0) flush32();
   auto kth_of = [&]() {
     uint64_t v = best[0];
 #pragma unroll
     for (int r = 1; r < R; ++r)
-      if (r == kr) v = best[r];
-    return shfl64(v, kl);
+      if (r == ((k - 1) >> 5)) v = best[r];
+    return shfl64(v, (k - 1) & 31);
   };
-  for (int g = 0; g < npb; g += 32) {
-    const int j = g + lane;
-    const int cnt = j < npb ? pcnt[q * stride + j] : 0;
-    const int64_t off = j < npb ? poff[q * stride + j] : 0;
-    int incl = cnt;
-    for (int o = 1; o < 32; o <<= 1) {
-      const int v = __shfl_up_sync(MV_FULL, incl, o);
-      if (lane >= o) incl += v;
-    }
-    const int excl = incl - cnt;
-    const int T = __shfl_sync(MV_FULL, incl, 31);
-    auto load = [&](int e0) {
-      const int e = e0 + lane;
-      // pair holding element e: the largest s with excl[s] <= e
-      int lo = 0;
-#pragma unroll
-      for (int step = 16; step > 0; step >>= 1) {
-        const int ex = __shfl_sync(MV_FULL, excl, (lo + step) & 31);
-        if (lo + step < 32 && ex <= e) lo += step;
-      }
-      const int64_t o = __shfl_sync(MV_FULL, off, lo);
-      const int ex = __shfl_sync(MV_FULL, excl, lo);
-      return e < T ? part[o + (e - ex)] : MV_KEY_PAD;
-    };
-    uint64_t nxt = T > 0 ? load(0) : MV_KEY_PAD;
-    for (int e0 = 0; e0 < T; e0 += 32) {
-      uint64_t c[R];
-      c[0] = nxt;
-#pragma unroll
-      for (int r = 1; r < R; ++r) c[r] = MV_KEY_PAD;
-      if (e0 + 32 < T) nxt = load(e0 + 32);
-      if (!(c[0] < kth_of())) c[0] = MV_KEY_PAD;
-      if (__any_sync(MV_FULL, c[0] != MV_KEY_PAD)) {
-        uint64_t c1[1] = {c[0]};
-        warp_bitonic_sort<1>(c1);
-        c[0] = c1[0];
-        warp_merge_smallest<R>(best, c);
-      }
-    }
-  }
   if (tau_out) {  // seeding: the k-th best key of the first nuse[q] pairs bounds the query's top-k
     const uint64_t kth = kth_of();
     if (lane == 0 && kth != MV_KEY_PAD) tau_out[q] = kth;

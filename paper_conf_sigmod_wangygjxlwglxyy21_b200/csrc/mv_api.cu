@@ -550,8 +550,6 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
     const int qchunk_min = use_tc ? tp.qchunk_split : qchunk;
     int32_t* qcfg;
     CK(s.alloc(&qcfg, 2));
-    if (use_tc && ix->type == MV_IVF_FLAT) CK(launch_scan_cfg(qlo_any, tp.qchunk, 1, tp.qchunk_split, 2, qcfg, st));
-    else CK(launch_scan_cfg(nullptr, qchunk, use_tc ? 4 : 1, qchunk, 4, qcfg, st));
     const int64_t npairs = nq * npb;
     // Seeding (tensor-core path, nprobe >= 2): phase A scans each query's ra[q] nearest lists --
     // the fewest holding >= 2k candidates -- and emits all of them; their k-th best key tau_q is an
@@ -559,10 +557,7 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
     const char* seed_env = getenv("MV_SEED");
     const bool split = use_tc && npb >= 2 && !(seed_env && seed_env[0] == '0');
     int32_t* ra = nullptr;
-    if (split) {
-      CK(s.alloc(&ra, (size_t)nq));
-      CK(launch_seed_ranks(P, nq, npb, ix->list_off, std::max<int64_t>(2 * (int64_t)k, k + 32), ra, st));
-    }
+    if (split) CK(s.alloc(&ra, (size_t)nq));
     const int nv = split ? 2 * nlist : nlist;
     Bucketing b;
     CK(s.alloc(&b.lcount, nv));
@@ -577,10 +572,17 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
     CK(s.alloc(&b.poff, (size_t)npairs));
     CK(s.alloc(&b.pcnt, (size_t)npairs));
     CK(s.alloc(&b.counter, 1));
-    CK(launch_bucket(P, nq, npb, nlist, ix->list_off, k, qcfg, ra, b, st));
     // pair regions: the whole list (tensor-core scan: emit-all bound), or min(k, |list|) (SIMT)
     const int capk = use_tc ? 0 : k;
-    CK(launch_pair_offsets(P, nq, npb, ix->list_off, k, capk, b, st));
+    PlanArgs pa;
+    pa.probes = P; pa.nq = nq; pa.npb = npb; pa.nlist = nlist; pa.k = k; pa.capk = capk;
+    pa.split = split ? 1 : 0; pa.need = std::max<int64_t>(2 * (int64_t)k, k + 32);
+    pa.list_off = ix->list_off;
+    pa.qlo_any = (use_tc && ix->type == MV_IVF_FLAT) ? qlo_any : nullptr;
+    pa.qc_exact = qchunk; pa.p_exact = use_tc ? (ix->type == MV_IVF_FLAT ? 1 : 4) : 1;
+    pa.qc_split = qchunk_min; pa.p_split = use_tc ? (ix->type == MV_IVF_FLAT ? 2 : 4) : 1;
+    pa.qcfg = qcfg; pa.ra = ra; pa.b = b;
+    CK(launch_plan(pa, st));
     prof_mark(ix, st);
     int64_t cap;
     if (use_tc) {
@@ -678,7 +680,7 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
         fprintf(stderr, "\n");
       }
       ix->last_scan = ix->type == MV_IVF_FLAT ? "tcgen05.tf32" : "tcgen05.i8";
-      ix->launches += split ? 5 : 2;  // qplanes, scan A (+ seed ranks, tau select, scan B)
+      ix->launches += split ? 4 : 2;  // qplanes, scan A (+ tau select, scan B)
     } else {
     ScanArgs a;
     a.type = ix->type; a.metric = ix->metric; a.d = ix->d; a.dpad = dpad; a.k = k; a.npb = npb;
@@ -698,7 +700,7 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
     CK(launch_final_select(b.poff, b.pcnt, part, nq, npb, k, ix->metric, ix->sorted_ids, D, I, tmax, over, st));
     prof_mark(ix, st);
     if (ix->prof) ix->prof_searches++;
-    ix->launches += 15;  // prep, hilo, coarse, cfg, 7 bucketing, 3 offsets, final select (+ SIMT scan below)
+    ix->launches += 6;  // prep, hilo, coarse GEMM + probe select (or SIMT coarse), plan, final select
     if (!use_tc) ix->launches += 1;
   }
   if (host_out) {

@@ -548,20 +548,24 @@ struct Bucketing {
   int32_t* pcnt;     // nq*npb     candidates written per pair
   int32_t* counter;  // 1          persistent scan work counter
 };
-// ra != nullptr: the pairs of query q with probe rank < ra[q] form a first phase (virtual lists
-// 0..nlist-1, work items first) and the others a second (virtual lists nlist..2*nlist-1); arrays
-// are then sized for 2*nlist lists.
-// qcfg (device) = {query chunk, query planes} (launch_scan_cfg)
-cudaError_t launch_bucket(const int32_t* probes, int64_t nq, int npb, int nlist, const int64_t* list_off, int k,
-                          const int32_t* qcfg, const int32_t* ra, const Bucketing& b, cudaStream_t st);
-cudaError_t launch_scan_cfg(const int* qlo_any, int qc_exact, int p_exact, int qc_split, int p_split, int32_t* qcfg,
-                            cudaStream_t st);
-// ra[q] = the fewest nearest lists of q holding >= need candidates (<= npb)
-cudaError_t launch_seed_ranks(const int32_t* probes, int64_t nq, int npb, const int64_t* list_off, int64_t need,
-                              int32_t* ra, cudaStream_t st);
-// capk > 0: region of a pair = min(capk, |list|) (SIMT local selection); capk = 0: |list|
-cudaError_t launch_pair_offsets(const int32_t* probes, int64_t nq, int npb, const int64_t* list_off, int k, int capk,
-                                const Bucketing& b, cudaStream_t st);
+// a4 in one cooperative launch (k_bucket.cu).  With the seeding split the pairs of query q with
+// probe rank < ra[q] form a first phase (virtual lists 0..nlist-1, work items first) and the
+// others a second (virtual lists nlist..2*nlist-1); arrays are then sized for 2*nlist lists.
+struct PlanArgs {
+  const int32_t* probes;   // nq x npb, best-first
+  int64_t nq;
+  int npb, nlist, k, capk;  // capk > 0: SIMT local-selection regions min(capk, |list|); 0: |list|
+  int split;               // 1: seeding phase (ra[q] nearest lists) + phase B
+  int64_t need;            // seeding: candidates the phase-A lists must hold
+  const int64_t* list_off;
+  const int* qlo_any;      // FLAT: some query needs its lo plane (nullable)
+  int qc_exact, p_exact, qc_split, p_split;
+  int32_t* qcfg;           // out: {query chunk, planes}
+  int32_t* ra;             // out (split): nq
+  Bucketing b;             // out
+};
+cudaError_t launch_plan(const PlanArgs& a, cudaStream_t st);
+// single-CTA exclusive scans (the add path): out[0..n], out[n] = total
 cudaError_t launch_scan_i32(const int32_t* in, int n, int32_t* out, cudaStream_t st);   // out[n+1]
 cudaError_t launch_scan_i64(const int64_t* in, int64_t n, int64_t* out, cudaStream_t st);  // out[n+1]
 
