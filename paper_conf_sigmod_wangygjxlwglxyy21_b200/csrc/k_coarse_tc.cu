@@ -102,23 +102,26 @@ __global__ void __launch_bounds__(kCThreads, 1)
     if (lane == 0) {
       mbar_wait(full_b, 0);
       tc_fence_after();
-      const uint32_t id_full = idesc_tf32(BROWS), id_hi = idesc_tf32(NQB);
+      const uint32_t id_q = idesc_tf32(NQB);
+      const bool qlo = p.qlo_any == nullptr || *p.qlo_any != 0;  // C_hi . Q_lo vanishes for tf32-exact queries
       uint32_t it = 0;
       for (int t = t0, tl = 0; t < t1; ++t, ++tl) {
         const uint32_t a = tl & 1;
         mbar_wait(&tempty[a], ((tl >> 1) & 1) ^ 1);
         tc_fence_after();
-        const uint32_t d = tmem + a * 2 * NQB;
+        const uint32_t d = tmem + a * NQB;
         for (int c = 0; c < nchunks; ++c, ++it) {
           const uint32_t s = it % nstage;
           mbar_wait(&full_a[s], (it / nstage) & 1);
           tc_fence_after();
           const uint32_t ah = smem_u32(As + s * 2 * ABYTES), al = ah + ABYTES;
-          const uint32_t bb = smem_u32(Bs + c * BROWS * ATOM);
+          const uint32_t bh = smem_u32(Bs + c * BROWS * ATOM), bl = bh + NQB * ATOM;
 #pragma unroll
           for (int ks = 0; ks < 4; ++ks) {
-            mma_tf32(d, kmajor_desc(ah + ks * 32, ATOM), kmajor_desc(bb + ks * 32, ATOM), id_full, (c | ks) != 0);
-            mma_tf32(d, kmajor_desc(al + ks * 32, ATOM), kmajor_desc(bb + ks * 32, ATOM), id_hi, 1);
+            // D += C_hi . Q_hi^T + C_lo . Q_hi^T (+ C_hi . Q_lo^T): q.c to ~2^-22, one accumulator
+            mma_tf32(d, kmajor_desc(ah + ks * 32, ATOM), kmajor_desc(bh + ks * 32, ATOM), id_q, (c | ks) != 0);
+            mma_tf32(d, kmajor_desc(al + ks * 32, ATOM), kmajor_desc(bh + ks * 32, ATOM), id_q, 1);
+            if (qlo) mma_tf32(d, kmajor_desc(ah + ks * 32, ATOM), kmajor_desc(bl + ks * 32, ATOM), id_q, 1);
           }
           mma_commit(&empty_a[s]);
         }
@@ -133,6 +136,7 @@ __global__ void __launch_bounds__(kCThreads, 1)
     const int row = quarter * 32 + lane;  // centroid within the tile
     const int nqv = (int)min64(NQB, p.nq - q0);
     float* S = p.S + (int64_t)q0 * p.lds;
+    uint32_t* G = p.G + (int64_t)q0 * p.ldg;
     for (int t = t0, tl = 0; t < t1; ++t, ++tl) {
       const uint32_t a = tl & 1;
       const int cid = t * 128 + row;
@@ -140,19 +144,26 @@ __global__ void __launch_bounds__(kCThreads, 1)
       const float cn = (valid && p.metric == MV_L2) ? __ldg(p.cnorm + cid) : 0.0f;
       mbar_wait(&tfull[a], (tl >> 1) & 1);
       tc_fence_after();
-      const uint32_t tb = tmem + a * 2 * NQB + ((uint32_t)(quarter * 32) << 16);
+      const uint32_t tb = tmem + a * NQB + ((uint32_t)(quarter * 32) << 16);
       for (int qc = half * 16; qc < ((p.dbg & 2) ? 0 : NQB); qc += 32) {
-        uint32_t rh[16], rl[16];
-        tmem_ld16(tb + qc, rh);
-        tmem_ld16(tb + NQB + qc, rl);
+        uint32_t rd[16];
+        tmem_ld16(tb + qc, rd);
         tmem_wait_ld();
-        if (valid) {
+        float* sp = S + (int64_t)qc * p.lds + cid;
+        uint32_t* gp = G + (int64_t)qc * p.ldg + t * 4 + quarter;
+        const int jn = min(16, nqv - qc);
 #pragma unroll
-          for (int j = 0; j < 16; ++j) {
-            const float dot = __uint_as_float(rh[j]) + __uint_as_float(rl[j]);
-            const float sc = p.metric == MV_L2 ? cn - 2.0f * dot : -dot;
-            if (qc + j < nqv) S[(int64_t)(qc + j) * p.lds + cid] = sc;
+        for (int j = 0; j < 16; ++j) {
+          const float dot = __uint_as_float(rd[j]);
+          const float sc = p.metric == MV_L2 ? cn - 2.0f * dot : -dot;
+          // the minimum score key of the warp's 32 centroids: lets the select skip whole groups
+          const uint32_t gm = __reduce_min_sync(MV_FULL, valid ? f2key(sc) : 0xffffffffu);
+          if (j < jn) {
+            if (valid) *sp = sc;
+            if (lane == 0) *gp = gm;
           }
+          sp += p.lds;
+          gp += p.ldg;
         }
       }
       tc_fence_before();
@@ -169,20 +180,24 @@ __global__ void __launch_bounds__(kCThreads, 1)
 
 // per-query top-nprobe of a score row (R = ceil(nprobe / 32) <= 4); see the file comment
 template <int R>
-__global__ void __launch_bounds__(256) k_probe_select(const float* __restrict__ S, int64_t lds, int64_t nq, int nlist,
-                                                      int nprobe, int32_t* __restrict__ probes) {
+__global__ void __launch_bounds__(256) k_probe_select(const float* __restrict__ S, int64_t lds,
+                                                      const uint32_t* __restrict__ G, int64_t ldg, int64_t nq,
+                                                      int nlist, int nprobe, int32_t* __restrict__ probes) {
   __shared__ uint64_t stage_all[8][64];
   const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
   const int64_t q = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   if (q >= nq) return;
   uint64_t* stage = stage_all[wib];
   const float* s = S + q * lds;
-  auto keyof = [&](float v, int c) { return ((uint64_t)f2key(v) << 32) | (uint32_t)c; };
-  // pass 1: each lane's R smallest keys (sorted, t[0] smallest)
+  const uint32_t* g = G + q * ldg;
+  const int ng = (int)ldg;
+  // pass 1: each lane's R smallest group minima; the nprobe-th smallest of those 32R bounds the
+  // answer (nprobe distinct centroids have score keys at or below it)
   uint64_t t[R];
 #pragma unroll
   for (int r = 0; r < R; ++r) t[r] = MV_KEY_PAD;
-  auto offer = [&](uint64_t key) {
+  for (int i = lane; i < ng; i += 32) {
+    const uint64_t key = ((uint64_t)g[i] << 32) | (uint32_t)i;
     if (key < t[R - 1]) {
       t[R - 1] = key;
 #pragma unroll
@@ -193,24 +208,15 @@ __global__ void __launch_bounds__(256) k_probe_select(const float* __restrict__ 
           t[r - 1] = x;
         }
     }
-  };
-  const int n4 = nlist & ~3;
-  for (int c = 4 * lane; c < n4; c += 128) {
-    const float4 v = *reinterpret_cast<const float4*>(s + c);
-    offer(keyof(v.x, c));
-    offer(keyof(v.y, c + 1));
-    offer(keyof(v.z, c + 2));
-    offer(keyof(v.w, c + 3));
   }
-  for (int c = n4 + lane; c < nlist; c += 32) offer(keyof(s[c], c));
-  // bound: the nprobe-th smallest of the 32R lane keys (nprobe distinct keys are <= it)
   warp_bitonic_sort<R>(t);
   uint64_t bsel = t[0];
 #pragma unroll
   for (int r = 1; r < R; ++r)
     if (r == ((nprobe - 1) >> 5)) bsel = t[r];
-  const uint64_t bound = shfl64(bsel, (nprobe - 1) & 31);
-  // pass 2: keys <= bound -> staging -> sorted list L (32R, L[r] holds element r*32 + lane)
+  const uint32_t bound = (uint32_t)(shfl64(bsel, (nprobe - 1) & 31) >> 32);
+  // pass 2: the groups whose minimum is within the bound; their keys at or below it -> staging ->
+  // sorted list L (32R, L[r] holds element r*32 + lane)
   uint64_t L[R];
 #pragma unroll
   for (int r = 0; r < R; ++r) L[r] = MV_KEY_PAD;
@@ -230,26 +236,25 @@ __global__ void __launch_bounds__(256) k_probe_select(const float* __restrict__ 
     __syncwarp();
     ns = rest;
   };
-  auto take = [&](uint64_t key) {
-    const bool ps = key <= bound;
-    const uint32_t m = __ballot_sync(MV_FULL, ps);
-    if (ps) stage[ns + __popc(m & ((1u << lane) - 1))] = key;
-    ns += __popc(m);
-    __syncwarp();
-    if (ns >= 32) flush32();
-  };
-  for (int c0 = 0; c0 < n4; c0 += 128) {
-    const int c = c0 + 4 * lane;
-    float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
-    if (c < n4) v = *reinterpret_cast<const float4*>(s + c);
-    take(c < n4 ? keyof(v.x, c) : MV_KEY_PAD);
-    take(c < n4 ? keyof(v.y, c + 1) : MV_KEY_PAD);
-    take(c < n4 ? keyof(v.z, c + 2) : MV_KEY_PAD);
-    take(c < n4 ? keyof(v.w, c + 3) : MV_KEY_PAD);
-  }
-  for (int c0 = n4; c0 < nlist; c0 += 32) {
-    const int c = c0 + lane;
-    take(c < nlist ? keyof(s[c], c) : MV_KEY_PAD);
+  for (int i0 = 0; i0 < ng; i0 += 32) {
+    const int gi = i0 + lane;
+    uint32_t m = __ballot_sync(MV_FULL, gi < ng && g[gi] <= bound);
+    while (m) {
+      const int grp = i0 + __ffs(m) - 1;
+      m &= m - 1;
+      const int c = grp * 32 + lane;
+      uint64_t key = MV_KEY_PAD;
+      if (c < nlist) {
+        const uint32_t k32 = f2key(s[c]);
+        if (k32 <= bound) key = ((uint64_t)k32 << 32) | (uint32_t)c;
+      }
+      const bool ps = key != MV_KEY_PAD;
+      const uint32_t bm = __ballot_sync(MV_FULL, ps);
+      if (ps) stage[ns + __popc(bm & ((1u << lane) - 1))] = key;
+      ns += __popc(bm);
+      __syncwarp();
+      if (ns >= 32) flush32();
+    }
   }
   if (ns > 0) flush32();
 #pragma unroll
@@ -322,7 +327,7 @@ bool coarse_tc_plan(int dpad, int nprobe, int64_t nq, int nlist, int nsm, Coarse
   p.nstage = std::min(6, (budget - fixed) / stage);
   p.smem_total = fixed + p.nstage * stage + 256 + 1024;
   int cols = 32;
-  while (cols < 4 * p.nqb) cols <<= 1;
+  while (cols < 2 * p.nqb) cols <<= 1;
   p.tmem_cols = cols;
   return p.smem_total <= 227 * 1024;
 }
@@ -336,9 +341,9 @@ cudaError_t launch_coarse_tc(const CUtensorMap* cmap, const CUtensorMap* qmap, c
   if ((e = cudaGetLastError()) != cudaSuccess) return e;
   const unsigned g2 = (unsigned)((nq * 32 + 255) / 256);
   const int R = (p.nprobe + 31) / 32;
-  if (R <= 1) k_probe_select<1><<<g2, 256, 0, st>>>(p.S, p.lds, nq, p.nlist, p.nprobe, p.probes);
-  else if (R == 2) k_probe_select<2><<<g2, 256, 0, st>>>(p.S, p.lds, nq, p.nlist, p.nprobe, p.probes);
-  else k_probe_select<4><<<g2, 256, 0, st>>>(p.S, p.lds, nq, p.nlist, p.nprobe, p.probes);
+  if (R <= 1) k_probe_select<1><<<g2, 256, 0, st>>>(p.S, p.lds, p.G, p.ldg, nq, p.nlist, p.nprobe, p.probes);
+  else if (R == 2) k_probe_select<2><<<g2, 256, 0, st>>>(p.S, p.lds, p.G, p.ldg, nq, p.nlist, p.nprobe, p.probes);
+  else k_probe_select<4><<<g2, 256, 0, st>>>(p.S, p.lds, p.G, p.ldg, nq, p.nlist, p.nprobe, p.probes);
   return cudaGetLastError();
 }
 

@@ -323,6 +323,15 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
 #pragma unroll
               for (int j = 0; j < 16; ++j) r[pl][j] = 0u;
           }
+          // the chunk's per-query constants, vector loads overlapping the TMEM load latency
+          float qn16[16], th16[16];
+#pragma unroll
+          for (int v = 0; v < 4; ++v) {
+            const float4 a4 = reinterpret_cast<const float4*>(mt.qnf + qc)[v];
+            const float4 t4 = reinterpret_cast<const float4*>(mt.thf + qc)[v];
+            qn16[4 * v] = a4.x; qn16[4 * v + 1] = a4.y; qn16[4 * v + 2] = a4.z; qn16[4 * v + 3] = a4.w;
+            th16[4 * v] = t4.x; th16[4 * v + 1] = t4.y; th16[4 * v + 2] = t4.z; th16[4 * v + 3] = t4.w;
+          }
           tmem_wait_ld();
           float bad[16];
           uint32_t pm = 0;
@@ -333,7 +342,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
             if (TYPE == MV_IVF_FLAT) {
               // exact for tf32-representable data (the only FLAT data this path accepts)
               const float dot = __uint_as_float(r[0][j]) + __uint_as_float(r[1 % PMAX][j]);
-              bad[j] = use_norms ? (mt.qnf[i] + xnf) - 2.0f * dot : -dot;
+              bad[j] = use_norms ? (qn16[j] + xnf) - 2.0f * dot : -dot;
             } else {
               // int32-exact digit partials; the L2 expansion is combined in fp64 (the norms are
               // ~400x the near-neighbour distances on SIFT-scale data)
@@ -343,7 +352,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
               const double dot = fma((double)mt.qs[i], acc, mt.qa[i]);
               bad[j] = use_norms ? (float)((mt.qn[i] + xn) - 2.0 * dot) : (float)(-dot);
             }
-            if (bad[j] <= mt.thf[i]) {
+            if (bad[j] <= th16[j]) {
               // exact test on the full key (distance key, id rank) < tau
               const uint64_t key = ((uint64_t)f2key(bad[j]) << 32) | rk;
               if (!phaseB || key < mt.tau[i]) pm |= 1u << j;

@@ -160,8 +160,8 @@ void free_storage(mv_index* ix) {
 }  // namespace
 
 // a2 + a3: tcgen05 coarse with fused top-nprobe when the shapes fit, else the SIMT kernel
-static cudaError_t run_coarse(mv_index* ix, const float* qpad, const float* qhl, int64_t nq, int npb, int32_t* P,
-                              Scratch& s, cudaStream_t st) {
+static cudaError_t run_coarse(mv_index* ix, const float* qpad, const float* qhl, const int* qlo_any, int64_t nq,
+                              int npb, int32_t* P, Scratch& s, cudaStream_t st) {
   CoarseParams cp;
   const char* force = getenv("MV_FORCE_SIMT");
   int dev = 0, nsm = kNumSMs;
@@ -178,7 +178,10 @@ static cudaError_t run_coarse(mv_index* ix, const float* qpad, const float* qhl,
       cp.cnorm = ix->cnorm;
       cp.probes = P;
       cp.lds = (ix->nlist + 3) & ~3;
+      cp.ldg = ((ix->nlist + 127) / 128) * 4;
+      cp.qlo_any = qlo_any;
       cudaError_t e = s.alloc(&cp.S, (size_t)nq * cp.lds);
+      if (e == cudaSuccess) e = s.alloc(&cp.G, (size_t)nq * cp.ldg);
       if (e != cudaSuccess) return e;
       const char* cdbg = getenv("MV_COARSE_DEBUG");
       cp.dbg = cdbg ? atoi(cdbg) : 0;
@@ -488,7 +491,7 @@ mv_status mv_search_probes(mv_index* ix, const float* queries, int64_t nq, int32
   float* qhl;
   CK(s.alloc(&qhl, (size_t)2 * nq * ix->dpad));
   CK(launch_hilo(q, nq, ix->d, ix->dpad, qhl, nullptr, st));
-  CK(run_coarse(ix, qpad, qhl, nq, npb, P, s, st));
+  CK(run_coarse(ix, qpad, qhl, nullptr, nq, npb, P, s, st));
   if (sp) {
     CK(cudaMemcpyAsync(probes, P, sizeof(int32_t) * nq * npb, cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
@@ -537,7 +540,7 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
     CK(s.alloc(&qlo_any, 1));
     CK(cudaMemsetAsync(qlo_any, 0, sizeof(int), st));
     CK(launch_hilo(q, nq, ix->d, dpad, qhl, qlo_any, st));
-    CK(run_coarse(ix, qpad, qhl, nq, npb, P, s, st));
+    CK(run_coarse(ix, qpad, qhl, qlo_any, nq, npb, P, s, st));
     prof_mark(ix, st);
     // a4 (work-item size depends on the scan implementation's shared-memory plan)
     TcScanParams tp;

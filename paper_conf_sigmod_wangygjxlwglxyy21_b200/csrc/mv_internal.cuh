@@ -640,6 +640,9 @@ struct CoarseParams {
   const float* cnorm;
   float* S;                // nq x lds scores (lds = roundup(nlist, 4))
   int64_t lds;
+  uint32_t* G;             // nq x ldg: minimum score key of each 32-centroid group (ldg = ceil(nlist/32))
+  int64_t ldg;
+  const int* qlo_any;      // device: some query needs its lo plane (nullable = yes)
   int32_t* probes;
 };
 bool coarse_tc_plan(int dpad, int nprobe, int64_t nq, int nlist, int nsm, CoarseParams& p);

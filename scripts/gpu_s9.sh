@@ -1,0 +1,9 @@
+python -c "import __graft_entry__ as g; g.build()" || exit 1
+timeout 900 python -m pytest tests -m "gpu and not slow" -x -q --timeout 300 2>&1 | tail -2
+for c in c2 c3; do
+  timeout 600 python bench.py --config $c --steps 20 --warmup 3 --no-cpu-baseline > gpurun_out/bench_$c.json 2> gpurun_out/bench_$c.err
+  python -c "import json; d=json.load(open('gpurun_out/bench_$c.json')); print('$c', round(d['value']), 'qps', d['config'].get('recall@10'), {a: round(b,3) for a,b in d['stage_ms'].items()}, 'frac', round(d['roofline']['frac'],3), d['index']['last_scan'])" || tail -5 gpurun_out/bench_$c.err
+done
+export PATH=/usr/local/cuda/bin:$PATH
+timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches_c2.csv python bench.py --steps 3 --warmup 3 --no-cpu-baseline > /dev/null 2>&1; echo launches rc=$?
+python scripts/launch_summary.py gpurun_out/launches_c2.csv

@@ -1,0 +1,32 @@
+"""Per-search kernel time shares from an `ncu --metrics gpu__time_duration.sum --csv` launch list.
+Counts the libmv kernels (mv:: namespace) launched per search (= per k_plan launch) and their mean
+cold-cache, serialised durations.  Usage: launch_summary.py launches.csv"""
+import csv
+import sys
+from collections import defaultdict
+
+rows = [r for r in csv.reader(open(sys.argv[1])) if len(r) > 14 and r[12] == "gpu__time_duration.sum"]
+tot = defaultdict(float)
+cnt = defaultdict(int)
+nplan = 0
+for r in rows:
+    name = r[4]
+    short = name.split("(")[0].replace("void ", "").replace("mv::", "")
+    if "k_plan" in short:
+        nplan += 1
+    if nplan == 0 and "k_coarse_gemm" not in short and "k_probe_select" not in short and "k_hilo" not in short \
+            and "k_row_prep" not in short:
+        continue  # data preparation and the add path precede the first search
+    if not any(t in name for t in ("mv::", "k_scan", "k_final", "k_coarse", "k_probe", "k_plan", "k_hilo",
+                                    "k_query_prep", "k_qplanes", "k_final_big", "k_merge")):
+        continue
+    v = float(r[14].replace(",", ""))
+    unit = r[13]
+    us = {"nsecond": v / 1000.0, "ns": v / 1000.0, "usecond": v, "us": v, "msecond": v * 1000.0, "ms": v * 1000.0}.get(unit, v)
+    tot[short] += us
+    cnt[short] += 1
+n = max(nplan, 1)
+total = sum(tot.values()) / n
+print(f"searches (k_plan launches): {nplan}; libmv device time per search {total:.1f} us")
+for k, v in sorted(tot.items(), key=lambda kv: -kv[1]):
+    print(f"  {k:<40} {v / n:9.1f} us  {100 * v / n / total:5.1f}%  launches/search {cnt[k] / n:.2f}")
