@@ -385,7 +385,7 @@ def main():
                        "recall@10": rec},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm_peak, "unit": "GB/s",
                          "frac": achieved / hbm_peak, "traffic": traffic, "peak_source": peak_src,
-                         "kernel": "k_scan (a5+a6)", "algorithmic_bytes_per_launch": scan_bytes,
+                         "kernel": "k_scan_tc (a5+a6), phases A+B", "algorithmic_bytes_per_launch": scan_bytes,
                          "units_per_launch": units, "bytes_per_unit": bpv},
             "stage_ms": stage_ms,
             "index": ix.describe(),
