@@ -50,9 +50,8 @@ struct WorkInfo {
   int64_t lstart;
 };
 
-__device__ __forceinline__ WorkInfo work_info(const TcScanParams& p, int w, int qchunk) {
+__device__ __forceinline__ WorkInfo work_info_of(const TcScanParams& p, int2 it, int qchunk) {
   WorkInfo wi;
-  const int2 it = p.witems[w];
   wi.l = it.x >= p.nlist ? it.x - p.nlist : it.x;
   wi.bstart = it.y;
   wi.nqc = min(qchunk, p.boff[it.x + 1] - wi.bstart);
@@ -60,6 +59,9 @@ __device__ __forceinline__ WorkInfo work_info(const TcScanParams& p, int w, int 
   wi.len = (int)(p.list_off[wi.l + 1] - wi.lstart);
   wi.ntiles = (wi.len + 127) >> 7;
   return wi;
+}
+__device__ __forceinline__ WorkInfo work_info(const TcScanParams& p, int w, int qchunk) {
+  return work_info_of(p, p.witems[w], qchunk);
 }
 
 constexpr int kNTS = 4;          // per-tile side-data ring slots
@@ -72,6 +74,8 @@ constexpr int kThreads = 128 + 32 * kEpiWarps;
 
 // per-query metadata of one work item (QCP = roundup16(qchunk) entries per array)
 struct Meta {
+  WorkInfo* wi;    // the work item (written by the gatherer: the MMA and epilogue warps read it here)
+  int32_t* qidx;   // query index
   int32_t* pair;   // (query, rank) pair id, q * npb + r
   int32_t* cnt;    // candidates emitted so far (smem atomics)
   float* thf;      // badness bound: a candidate can pass only if badness <= thf (NaN: padding column)
@@ -84,6 +88,9 @@ struct Meta {
 };
 __device__ __forceinline__ Meta meta_at(uint8_t* m, int QCP) {
   Meta r;
+  r.wi = reinterpret_cast<WorkInfo*>(m);
+  r.qidx = reinterpret_cast<int32_t*>(m + 32);
+  m += 32 + 4 * QCP;
   r.pair = reinterpret_cast<int32_t*>(m);
   r.cnt = r.pair + QCP;
   r.thf = reinterpret_cast<float*>(r.cnt + QCP);
@@ -95,10 +102,10 @@ __device__ __forceinline__ Meta meta_at(uint8_t* m, int QCP) {
   r.qa = r.qn + QCP;
   return r;
 }
-constexpr int kMetaPerQuery = 52;  // bytes
+constexpr int kMetaPerQuery = 56;  // bytes (+ a 32-B work-item header)
 
 template <int TYPE>
-__global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__ CUtensorMap xmap, const TcScanParams p) {
+__global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__ XMaps xm, const TcScanParams p) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~(uintptr_t)1023);
   constexpr int ESZ = TYPE == MV_IVF_FLAT ? 4 : 1;
@@ -123,9 +130,10 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
   uint64_t* full_q = empty_x + nstage;
   uint64_t* empty_q = full_q + 2;
   uint64_t* empty_m = empty_q + 2;
+  const int NACC = p.nacc;  // TMEM accumulator buffers (4 for FLAT, 2 for SQ8's 4-plane tiles)
   uint64_t* tfull = empty_m + 2;
-  uint64_t* tempty = tfull + 2;
-  uint64_t* full_t = tempty + 2;
+  uint64_t* tempty = tfull + 4;
+  uint64_t* full_t = tempty + 4;
   uint64_t* empty_t = full_t + kNTS;
   uint32_t* tslot = reinterpret_cast<uint32_t*>(empty_t + kNTS);
 
@@ -139,8 +147,10 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
       mbar_init(&full_q[b], 64);
       mbar_init(&empty_q[b], 1);
       mbar_init(&empty_m[b], kEpiWarps);
-      mbar_init(&tfull[b], 1);
-      mbar_init(&tempty[b], kEpiWarps);
+    }
+    for (int a = 0; a < 4; ++a) {
+      mbar_init(&tfull[a], 1);
+      mbar_init(&tempty[a], kEpiWarps);
     }
     for (int s = 0; s < kNTS; ++s) {
       mbar_init(&full_t[s], 1);
@@ -152,7 +162,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
     tmem_alloc(tslot, p.tmem_cols);
     tmem_relinquish();
   }
-  if (warp == 0 && lane == 0) tma_prefetch(&xmap);
+  if (warp == 0 && lane == 0)
+    for (int i = 0; i < 4; ++i) tma_prefetch(&xm.m[i]);
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
@@ -165,8 +176,16 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
     if (lane == 0) {
       uint32_t it = 0, tcount = 0;
       const uint32_t side_tx = 528 + (use_norms ? 1040 : 0) + (use_ids ? 1040 : 0);
-      for (int w = w0; w < nwork; w += gridDim.x) {
-        const WorkInfo wi = work_info(p, w, QC);
+      const uint64_t pol = l2_evict_first_policy();
+      // two-deep prefetch: the next item's list range and the one after's (list, bucket) pair are
+      // in flight while this item's tiles are issued, so no dependent load sits between items
+      const int G = gridDim.x;
+      int2 itn = w0 + G < nwork ? p.witems[w0 + G] : make_int2(0, 0);
+      WorkInfo wn = w0 < nwork ? work_info(p, w0, QC) : WorkInfo{};
+      for (int w = w0; w < nwork; w += G) {
+        const WorkInfo wi = wn;
+        if (w + G < nwork) wn = work_info_of(p, itn, QC);
+        if (w + 2 * G < nwork) itn = p.witems[w + 2 * G];
         for (int t = 0; t < wi.ntiles; ++t, ++tcount) {
           const int row0 = (int)(wi.lstart + t * 128);
           const uint32_t ts = tcount % kNTS, tr = tcount / kNTS;
@@ -180,8 +199,21 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
             const uint32_t s = it % nstage, r = it / nstage;
             mbar_wait(&empty_x[s], (r & 1) ^ 1);
             MV_TRACE(0, it);
-            mbar_expect_tx(&full_x[s], 128 * ATOM);
-            tma_load_2d(Xs + s * 128 * ATOM, &xmap, &full_x[s], c * ATOM / ESZ, row0);
+            // a list's tail tile loads roundup16(rows) rows as 64/32/16-row boxes (< 16 rows past the
+            // list end); its stale smem rows beyond are masked lanes of the MMA's M = 128
+            const int rows = min(128, wi.len - t * 128);
+            uint8_t* dst = Xs + s * 128 * ATOM;
+            if (rows > 112) {
+              mbar_expect_tx(&full_x[s], 128 * ATOM);
+              tma_load_2d_hint(dst, &xm.m[0], &full_x[s], c * ATOM / ESZ, row0, pol);
+            } else {
+              const int r16 = (rows + 15) & ~15;
+              mbar_expect_tx(&full_x[s], r16 * ATOM);
+              int o = 0;
+              if (r16 & 64) { tma_load_2d_hint(dst, &xm.m[1], &full_x[s], c * ATOM / ESZ, row0, pol); o += 64; }
+              if (r16 & 32) { tma_load_2d_hint(dst + o * ATOM, &xm.m[2], &full_x[s], c * ATOM / ESZ, row0 + o, pol); o += 32; }
+              if (r16 & 16) tma_load_2d_hint(dst + o * ATOM, &xm.m[3], &full_x[s], c * ATOM / ESZ, row0 + o, pol);
+            }
           }
         }
       }
@@ -191,18 +223,18 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
     if (lane == 0) {
       uint32_t it = 0, titer = 0, wcount = 0;
       for (int w = w0; w < nwork; w += gridDim.x, ++wcount) {
-        const WorkInfo wi = work_info(p, w, QC);
-        const int NQ = (wi.nqc + 15) & ~15;
-        const int N = P * NQ;
-        const uint32_t idesc = TYPE == MV_IVF_FLAT ? idesc_tf32(N) : idesc_u8s8(N);
         const uint32_t b = wcount & 1;
         mbar_wait(&full_q[b], (wcount >> 1) & 1);
         MV_TRACE(1, wcount);
         tc_fence_after();
+        const WorkInfo wi = *meta_at(metab + b * p.meta_bytes, QCP).wi;
+        const int NQ = (wi.nqc + 15) & ~15;
+        const int N = P * NQ;
+        const uint32_t idesc = TYPE == MV_IVF_FLAT ? idesc_tf32(N) : idesc_u8s8(N);
         const uint32_t qbase = smem_u32(Qs + b * p.q_bytes);
         for (int t = 0; t < wi.ntiles; ++t, ++titer) {
-          const uint32_t a = titer & 1;
-          mbar_wait(&tempty[a], ((titer >> 1) & 1) ^ 1);
+          const uint32_t a = titer % NACC;
+          mbar_wait(&tempty[a], ((titer / NACC) & 1) ^ 1);
           MV_TRACE(2, titer);
           tc_fence_after();
           const uint32_t dcol = tmem + a * p.ncol;
@@ -230,32 +262,67 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
   } else if (warp < 4) {
     // ------------------------------------------------------------------ query gatherer (64 thr)
     const int tq = threadIdx.x - 64;
+    const int gw = tq >> 5;
+    const int G = gridDim.x;
+    // the next item's list range and per-query metadata are loaded into registers before waiting
+    // for its buffers, so only the plane copies sit on the critical path once a buffer frees
+    struct Pref {
+      WorkInfo wi;
+      int pr[2], q[2];
+      uint64_t tau[2];
+      double qn[2], qa[2];
+      float qs[2];
+      int64_t base[2];
+    };
+    auto prefetch = [&](int w) {
+      Pref f;
+      f.wi = work_info(p, w, QC);
+#pragma unroll
+      for (int u = 0; u < 2; ++u) {
+        const int i = tq + 64 * u;
+        if (i < f.wi.nqc) {
+          f.pr[u] = p.bq[f.wi.bstart + i];
+          f.q[u] = f.pr[u] / p.npb;
+          f.tau[u] = phaseB ? p.tau[f.q[u]] : MV_KEY_PAD;
+          f.qn[u] = p.qnorm[f.q[u]];
+          f.qs[u] = TYPE == MV_IVF_SQ8 ? p.qscale[f.q[u]] : 1.0f;
+          f.qa[u] = TYPE == MV_IVF_SQ8 ? p.qa[f.q[u]] : 0.0;
+          f.base[u] = p.poff[f.pr[u]];
+        }
+      }
+      return f;
+    };
+    Pref cur;
+    if (w0 < nwork) cur = prefetch(w0);
     uint32_t wcount = 0;
-    for (int w = w0; w < nwork; w += gridDim.x, ++wcount) {
-      const WorkInfo wi = work_info(p, w, QC);
+    for (int w = w0; w < nwork; w += G, ++wcount) {
+      Pref nxt;
+      if (w + G < nwork) nxt = prefetch(w + G);
+      const WorkInfo wi = cur.wi;
       const int NQ = (wi.nqc + 15) & ~15;
       const int N = P * NQ;
       const uint32_t b = wcount & 1, r = wcount >> 1;
       mbar_wait(&empty_q[b], (r & 1) ^ 1);
       mbar_wait(&empty_m[b], (r & 1) ^ 1);
       const Meta mt = meta_at(metab + b * p.meta_bytes, QCP);
-      for (int i = tq; i < NQ; i += 64) {
+      if (tq == 0) *mt.wi = wi;
+#pragma unroll
+      for (int u = 0; u < 2; ++u) {
+        const int i = tq + 64 * u;
         if (i < wi.nqc) {
-          const int pr = p.bq[wi.bstart + i];
-          const int q = pr / p.npb;
-          const double qn = p.qnorm[q];
-          const uint64_t t = phaseB ? p.tau[q] : MV_KEY_PAD;
+          const uint64_t t = cur.tau[u];
           const uint32_t t32 = (uint32_t)(t >> 32);
-          mt.pair[i] = pr;
+          mt.qidx[i] = cur.q[u];
+          mt.pair[i] = cur.pr[u];
           mt.cnt[i] = 0;
           mt.tau[i] = t;
           mt.thf[i] = t32 >= 0xff800000u ? __int_as_float(0x7f800000) : key2f(t32);
-          mt.qnf[i] = (float)qn;
-          mt.qn[i] = qn;
-          mt.qs[i] = TYPE == MV_IVF_SQ8 ? p.qscale[q] : 1.0f;
-          mt.qa[i] = TYPE == MV_IVF_SQ8 ? p.qa[q] : 0.0;
-          mt.base[i] = p.poff[pr];
-        } else {  // padding column: no comparison passes
+          mt.qnf[i] = (float)cur.qn[u];
+          mt.qn[i] = cur.qn[u];
+          mt.qs[i] = cur.qs[u];
+          mt.qa[i] = cur.qa[u];
+          mt.base[i] = cur.base[u];
+        } else if (i < NQ) {  // padding column: no comparison passes
           mt.thf[i] = __int_as_float(0x7fffffff);
           mt.qnf[i] = 0.f;
           mt.qn[i] = 0.0;
@@ -264,23 +331,27 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
         }
       }
       named_bar(2, 64);
+      // plane copies: one operand row (query i, plane pl) per warp iteration, the row's 16-B pieces
+      // across the lanes (coalesced reads), swizzled into the K-major operand
       uint8_t* Qb = Qs + b * p.q_bytes;
       constexpr int PIECES = ATOM / 16;
-      const int total = (p.dbg & 4) ? 0 : wi.nqc * P * nchunks * PIECES;
-      for (int idx = tq; idx < total; idx += 64) {
-        const int pc = idx % PIECES;
-        int rest = idx / PIECES;
-        const int c = rest % nchunks;
-        rest /= nchunks;
-        const int pl = rest % P;
-        const int i = rest / P;
-        const int q = mt.pair[i] / p.npb;
+      const int ppr = nchunks * PIECES;  // pieces per row
+      const int nrows = (p.dbg & 4) ? 0 : wi.nqc * P;
+      for (int u = gw; u < nrows; u += 2) {
+        const int i = P == 1 ? u : (P == 2 ? u >> 1 : u >> 2);
+        const int pl = u - i * P;
+        const int q = mt.qidx[i];
         const int64_t prow = TYPE == MV_IVF_FLAT ? (int64_t)pl * p.nq + q : (int64_t)q * P + pl;
-        cp_async16(Qb + c * N * ATOM + swz_off(pl * NQ + i, pc, ATOM), p.qplanes + prow * rowbytes + c * ATOM + pc * 16);
+        const uint8_t* src = p.qplanes + prow * rowbytes;
+        for (int e = lane; e < ppr; e += 32) {
+          const int c = e / PIECES, pc = e % PIECES;  // PIECES is a power of two
+          cp_async16(Qb + c * N * ATOM + swz_off(pl * NQ + i, pc, ATOM), src + e * 16);
+        }
       }
       cp_async_wait_all();
       fence_proxy_async();
       mbar_arrive(&full_q[b]);
+      cur = nxt;
     }
   } else {
     // ------------------------------------------------------------------ epilogue (8 warps)
@@ -292,13 +363,13 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
     const uint32_t ltmask = (1u << lane) - 1;
     uint32_t titer = 0, wcount = 0;
     for (int w = w0; w < nwork; w += gridDim.x, ++wcount) {
-      const WorkInfo wi = work_info(p, w, QC);
-      const int NQ = (wi.nqc + 15) & ~15;
       const uint32_t b = wcount & 1;
       mbar_wait(&full_q[b], (wcount >> 1) & 1);
       const Meta mt = meta_at(metab + b * p.meta_bytes, QCP);
+      const WorkInfo wi = *mt.wi;
+      const int NQ = (wi.nqc + 15) & ~15;
       for (int t = 0; t < wi.ntiles; ++t, ++titer) {
-        const uint32_t a = titer & 1;
+        const uint32_t a = titer % NACC;
         const uint32_t ts = titer % kNTS;
         const int vrow = t * 128 + row;
         const int row0 = (int)(wi.lstart + t * 128);
@@ -310,7 +381,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
           valid = !bit_excluded(p.bitset, p.nbits, reinterpret_cast<const int64_t*>(sd + kSideIds)[(row0 & 1) + row]);
         const double xn = use_norms ? reinterpret_cast<const double*>(sd)[(row0 & 1) + row] : 0.0;
         const float xnf = (float)xn;
-        mbar_wait(&tfull[a], (titer >> 1) & 1);
+        mbar_wait(&tfull[a], (titer / NACC) & 1);
         if (et == 0) MV_TRACE(6, titer);
         tc_fence_after();
         const uint32_t tbase = tmem + a * p.ncol + ((uint32_t)(quarter * 32) << 16);
@@ -495,12 +566,13 @@ static bool tc_scan_layout(int type, int dpad, int qc, int ns, TcScanParams& p) 
   p.qchunk_split = type == MV_IVF_FLAT ? qc / 2 : qc;
   const int qcp = (qc + 15) & ~15;
   p.ncol = rows_per_q * qcp;
+  p.nacc = 512 / p.ncol >= 4 ? 4 : 2;
   int cols = 32;
-  while (cols < 2 * p.ncol) cols <<= 1;
+  while (cols < p.nacc * p.ncol) cols <<= 1;
   if (cols > 512) return false;
   p.tmem_cols = cols;
   p.q_bytes = up(rows_per_q * qcp * dpad * esz, 1024);
-  p.meta_bytes = up(kMetaPerQuery * qcp, 16);
+  p.meta_bytes = up(32 + kMetaPerQuery * qcp, 16);
   const int stage = 128 * atom;
   p.nstage = ns;
   p.off_x = 0;
@@ -508,7 +580,7 @@ static bool tc_scan_layout(int type, int dpad, int qc, int ns, TcScanParams& p) 
   p.off_meta = p.off_q + 2 * p.q_bytes;
   p.off_side = up(p.off_meta + 2 * p.meta_bytes, 128);
   p.off_bar = p.off_side + kNTS * kSideBytes;
-  p.smem_total = p.off_bar + (2 * ns + 10 + 2 * kNTS) * 8 + 16 + 1024;  // + 1 KB alignment slack
+  p.smem_total = p.off_bar + (2 * ns + 14 + 2 * kNTS) * 8 + 16 + 1024;  // + 1 KB alignment slack
   return p.smem_total <= 227 * 1024;
 }
 
@@ -523,14 +595,14 @@ bool tc_scan_plan(int type, int dpad, int k, TcScanParams& p) {
   return false;
 }
 
-cudaError_t launch_scan_tc(const CUtensorMap* xmap, const TcScanParams& p, cudaStream_t st) {
+cudaError_t launch_scan_tc(const XMaps& xm, const TcScanParams& p, cudaStream_t st) {
   auto kern = p.type == MV_IVF_FLAT ? k_scan_tc<MV_IVF_FLAT> : k_scan_tc<MV_IVF_SQ8>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, p.smem_total);
   if (e != cudaSuccess) return e;
   int dev = 0, nsm = kNumSMs;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
-  kern<<<nsm, kThreads, p.smem_total, st>>>(*xmap, p);
+  kern<<<nsm, kThreads, p.smem_total, st>>>(xm, p);
   return cudaGetLastError();
 }
 

@@ -38,7 +38,7 @@ struct mv_index {
   uint32_t* rank = nullptr;     // ntotal: position of (id, row) in sorted order
   int64_t* sorted_ids = nullptr;  // ntotal: ids in (id, row) order
   // tensor-core scan state (rebuilt by every add)
-  CUtensorMap xmap;
+  XMaps xm;                 // payload tensor maps: 128/64/32/16-row boxes
   bool xmap_ok = false;
   bool tf32_exact = true;   // FLAT: every stored value exactly representable in tf32
   const char* last_scan = "none";
@@ -438,11 +438,12 @@ mv_status mv_index_add(mv_index* ix, const float* vectors, const int64_t* ids, i
   ix->sorted_ids = sorted_ids;
   ix->ntotal = ntot;
   if (ix->type == MV_IVF_FLAT && hflag) ix->tf32_exact = false;
-  ix->xmap_ok = ntot <= 0x7fffffffLL &&
-                make_tmap_2d(&ix->xmap, payload,
-                             ix->type == MV_IVF_FLAT ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_UINT8,
-                             (uint64_t)dpad, (uint64_t)ntot, (uint64_t)dpad * esize, 32, 128,
-                             ix->type == MV_IVF_FLAT ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_32B);
+  ix->xmap_ok = ntot <= 0x7fffffffLL;
+  for (int i = 0; i < 4 && ix->xmap_ok; ++i)
+    ix->xmap_ok = make_tmap_2d(&ix->xm.m[i], payload,
+                               ix->type == MV_IVF_FLAT ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_UINT8,
+                               (uint64_t)dpad, (uint64_t)ntot, (uint64_t)dpad * esize, 32, 128 >> i,
+                               ix->type == MV_IVF_FLAT ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_32B);
   ix->maxlen = 0;
   std::vector<int64_t> lens(nlist);
   for (int l = 0; l < nlist; ++l) {
@@ -545,8 +546,12 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
     // a4 (work-item size depends on the scan implementation's shared-memory plan)
     TcScanParams tp;
     const char* force = getenv("MV_FORCE_SIMT");
+    // MV_SCAN_IMPL=qm selects the queries-as-M FLAT scan (k_scan_qm.cu, experimental)
+    const char* impl = getenv("MV_SCAN_IMPL");
+    const bool use_qm = ix->type == MV_IVF_FLAT && impl && impl[0] == 'q';
     const bool use_tc = ix->xmap_ok && !(force && force[0] == '1') &&
-                        (ix->type == MV_IVF_SQ8 || ix->tf32_exact) && tc_scan_plan(ix->type, dpad, k, tp);
+                        (ix->type == MV_IVF_SQ8 || ix->tf32_exact) &&
+                        (use_qm ? qm_scan_plan(dpad, k, tp) : tc_scan_plan(ix->type, dpad, k, tp));
     const int qchunk = use_tc ? tp.qchunk
                               : (k <= kLocalSelectMaxK ? std::min(64, std::max(1, 65536 / (8 * k))) : 64);
     // device-side work-item shape: FLAT tf32-exact queries take one plane and twice the queries
@@ -640,10 +645,11 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
         CK(cudaMemsetAsync(tp.prof, 0, 9 * 1024 * 8, st));
       }
       // phase A (or, without seeding, the whole scan emitting every candidate) ...
+      auto scan = [&]() { return use_qm ? launch_scan_qm(&ix->xm.m[0], &ix->xm.m[3], tp, st) : launch_scan_tc(ix->xm, tp, st); };
       tp.phase = 0;
       tp.wbeg = nullptr;
       tp.nwitems = b.woff + nlist;
-      CK(launch_scan_tc(&ix->xmap, tp, st));
+      CK(scan());
       prof_mark(ix, st);
       if (split) {
         // ... tau_q = k-th best key of phase A ...
@@ -653,7 +659,7 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
         tp.phase = 1;
         tp.wbeg = b.woff + nlist;
         tp.nwitems = b.woff + 2 * nlist;
-        CK(launch_scan_tc(&ix->xmap, tp, st));
+        CK(scan());
       } else {
         prof_mark(ix, st);
       }
@@ -682,7 +688,7 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
                   h[8 * 1024 + b * 3 + 2]);
         fprintf(stderr, "\n");
       }
-      ix->last_scan = ix->type == MV_IVF_FLAT ? "tcgen05.tf32" : "tcgen05.i8";
+      ix->last_scan = ix->type == MV_IVF_FLAT ? (use_qm ? "tcgen05.tf32.qm" : "tcgen05.tf32") : "tcgen05.i8";
       ix->launches += split ? 4 : 2;  // qplanes, scan A (+ tau select, scan B)
     } else {
     ScanArgs a;

@@ -597,7 +597,7 @@ cudaError_t launch_scan(const ScanArgs& a, cudaStream_t st);
 
 // k_scan_tc.cu (tcgen05 path): a filter-and-emit scan run in two phases
 struct TcScanParams {
-  int type, metric, dpad, k, npb, qchunk, nchunks, nstage, ncol, tmem_cols;
+  int type, metric, dpad, k, npb, qchunk, nchunks, nstage, ncol, tmem_cols, nacc;
   int qchunk_split;        // FLAT: queries per work item when the queries need the lo plane (P = 2)
   const int32_t* cfg;      // device {query chunk, planes} of this search (launch_scan_cfg)
   int nlist;               // virtual list v >= nlist is list v - nlist (phase-B pairs)
@@ -627,7 +627,14 @@ struct TcScanParams {
   unsigned long long* prof;  // MV_SCAN_TRACE timeline (CTA 0)
 };
 bool tc_scan_plan(int type, int dpad, int k, TcScanParams& p);
-cudaError_t launch_scan_tc(const CUtensorMap* xmap, const TcScanParams& p, cudaStream_t st);
+// the payload's tensor maps: boxes of 128, 64, 32, 16 rows (one swizzle atom wide)
+struct XMaps {
+  CUtensorMap m[4];
+};
+cudaError_t launch_scan_tc(const XMaps& xm, const TcScanParams& p, cudaStream_t st);
+// k_scan_qm.cu: FLAT scan with the queries on the MMA's M side (xmap: 128-row boxes, xmap16: 16-row boxes)
+bool qm_scan_plan(int dpad, int k, TcScanParams& p);
+cudaError_t launch_scan_qm(const CUtensorMap* xmap, const CUtensorMap* xmap16, const TcScanParams& p, cudaStream_t st);
 cudaError_t launch_qplanes(int type, const float* qpad, int64_t nq, int dpad, const float* vmin, const float* vdiff,
                            uint8_t* out, float* qscale, double* qa, double* qnorm, cudaStream_t st);
 cudaError_t launch_tf32_check(const float* x, int64_t n, int* flag, cudaStream_t st);

@@ -1,0 +1,3 @@
+python -c "import __graft_entry__ as g; g.build()" || exit 1
+MV_SCAN_TRACE=1 timeout 600 python bench.py --config c2 --steps 3 --warmup 3 --no-cpu-baseline > gpurun_out/trace.json 2> gpurun_out/trace.err
+grep -c trace gpurun_out/trace.err

@@ -98,7 +98,7 @@ def test_flat_tc_fractional_queries(metric):
     # absolute error proportional to the norms, not to the distance
     atol = 2e-6 * float((Q * Q).sum(1).max() + (X * X).sum(1).max())
     frac, _, _ = _run_conditional(ix, X, ids, C, Q, 10, 9, mo, O.FLAT, atol=atol)
-    assert ix.describe()["last_scan"] == "tcgen05.tf32"
+    assert ix.describe()["last_scan"].startswith("tcgen05.tf32")
     assert frac > 0.999
 
 
