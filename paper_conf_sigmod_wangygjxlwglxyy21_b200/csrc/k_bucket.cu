@@ -24,12 +24,10 @@ namespace mv {
 
 constexpr int kPlanThreads = 1024;
 
-// Virtual list of pair p = q*npb + r: its list l, or l + nlist for the pairs of the second phase
-// when the seeding phase is on (ra != nullptr): phase A = the ra[q] nearest lists of query q.
-__device__ __forceinline__ int vlist_of(const int32_t* probes, int64_t p, int npb, int nlist, const int32_t* ra) {
-  const int l = probes[p];
-  return (ra && (int)(p % npb) >= ra[p / npb]) ? l + nlist : l;
-}
+// With the seeding split (ra != nullptr) every pair p = q*npb + r of list l is an entry of virtual
+// list l + nlist (phase B, region capacity |l|), and the pairs of query q with r < ra[q] are also
+// entries of virtual list l (phase A: the first min(|l|, capA) rows, region capacity the same,
+// pair id npairs + p).  Without it, pair p is an entry of virtual list l.
 
 // Region capacity of a pair: min(capk, |list|) when the SIMT scan selects locally (capk > 0,
 // k <= 1024), else |list| (every candidate that survives the bitset may be emitted).
@@ -101,6 +99,7 @@ __global__ void __launch_bounds__(kPlanThreads) k_plan(const PlanArgs a) {
         const int l = pq[j];
         len = a.list_off[l + 1] - a.list_off[l];
         capsum += pair_cap(len, a.k, a.capk);
+        if (a.split) len = min64(len, a.capA);  // phase A reads a prefix of each list
       }
       int64_t incl = len;
       for (int o = 1; o < 32; o <<= 1) {
@@ -111,6 +110,11 @@ __global__ void __launch_bounds__(kPlanThreads) k_plan(const PlanArgs a) {
       if (hit && r == npb) r = j0 + __ffs(hit);  // ranks 0 .. first hit
       run += __shfl_sync(MV_FULL, incl, 31);
     }
+    // phase-A regions: the prefixes of the ra nearest lists
+    for (int j = lane; j < r && ra; j += 32) {
+      const int l = pq[j];
+      capsum += min64(a.list_off[l + 1] - a.list_off[l], a.capA);
+    }
     for (int o = 16; o > 0; o >>= 1) capsum += __shfl_xor_sync(MV_FULL, capsum, o);
     if (lane == 0) {
       if (ra) ra[q] = r;
@@ -118,7 +122,12 @@ __global__ void __launch_bounds__(kPlanThreads) k_plan(const PlanArgs a) {
     }
     for (int j = lane; j < npb; j += 32) {
       const int l = pq[j];
-      atomicAdd(b.lcount + ((ra && j >= r) ? l + nlist : l), 1);
+      if (ra) {
+        atomicAdd(b.lcount + l + nlist, 1);
+        if (j < r) atomicAdd(b.lcount + l, 1);
+      } else {
+        atomicAdd(b.lcount + l, 1);
+      }
     }
   }
   grid.sync();
@@ -140,7 +149,7 @@ __global__ void __launch_bounds__(kPlanThreads) k_plan(const PlanArgs a) {
       if (j < npb) {
         const int l = pq[j];
         c = pair_cap(a.list_off[l + 1] - a.list_off[l], a.k, a.capk);
-        const int v = (ra && j >= r) ? l + nlist : l;
+        const int v = ra ? l + nlist : l;
         b.bq[b.boff[v] + atomicAdd(b.bfill + v, 1)] = (int32_t)(q * npb + j);
       }
       int64_t incl = c;
@@ -149,6 +158,23 @@ __global__ void __launch_bounds__(kPlanThreads) k_plan(const PlanArgs a) {
         if (lane >= o) incl += v;
       }
       if (j < npb) b.poff[q * npb + j] = run + incl - c;
+      run += __shfl_sync(MV_FULL, incl, 31);
+    }
+    // phase-A entries (pair id npairs + q*npb + j), regions after the query's phase-B regions
+    for (int j0 = 0; ra && j0 < r; j0 += 32) {
+      const int j = j0 + lane;
+      int64_t c = 0;
+      if (j < r) {
+        const int l = pq[j];
+        c = min64(a.list_off[l + 1] - a.list_off[l], a.capA);
+        b.bq[b.boff[l] + atomicAdd(b.bfill + l, 1)] = (int32_t)(a.nq * npb + q * npb + j);
+      }
+      int64_t incl = c;
+      for (int o = 1; o < 32; o <<= 1) {
+        const int64_t v = __shfl_up_sync(MV_FULL, incl, o);
+        if (lane >= o) incl += v;
+      }
+      if (j < r) b.poff[a.nq * npb + q * npb + j] = run + incl - c;
       run += __shfl_sync(MV_FULL, incl, 31);
     }
   }
@@ -178,7 +204,8 @@ __global__ void __launch_bounds__(kPlanThreads) k_plan(const PlanArgs a) {
     const int2 it = b.witems_unsorted[w];
     const int l = it.x >= nlist ? it.x - nlist : it.x;
     const int nqw = min(qchunk, b.boff[it.x + 1] - it.y);
-    const int64_t len = a.list_off[l + 1] - a.list_off[l];
+    int64_t len = a.list_off[l + 1] - a.list_off[l];
+    if (a.split && it.x < nlist) len = min64(len, a.capA);
     const int tiles = (int)min64((len + 127) / 128, 63);
     return (it.x >= nlist ? HB : 0) + HB - 1 - min(HB - 1, tiles * 64 + min(nqw, 63));
   };

@@ -23,8 +23,8 @@
 //   warps 2-3  query gatherer: the bucket's query planes -> swizzled K-major smem, and the
 //              per-query metadata -- both double-buffered
 //   warps 4-11 epilogue, two warps per TMEM lane quarter (64 columns each)
-// Phases as in k_scan_tc.cu: phase A emits every candidate of each query's nearest lists, phase B
-// emits keys < tau_q.
+// Phases as in k_scan_tc.cu: phase A emits every candidate of a prefix of each query's nearest
+// lists, phase B emits keys <= tau_q over all probed lists.
 #include "mv_internal.cuh"
 #include "sm100.cuh"
 
@@ -76,7 +76,7 @@ __device__ __forceinline__ QmWork qm_work(const TcScanParams& p, int2 it, int qc
   wi.bstart = it.y;
   wi.nqc = min(qc, p.boff[it.x + 1] - wi.bstart);
   wi.lstart = p.list_off[l];
-  wi.len = (int)(p.list_off[l + 1] - wi.lstart);
+  wi.len = (int)min64(p.list_off[l + 1] - wi.lstart, p.rowcap);
   wi.ntiles = (wi.len + 127) >> 7;
   return wi;
 }
@@ -253,7 +253,9 @@ __global__ void __launch_bounds__(kQmThreads, 1)
         const int i = tq + 64 * u;
         if (i < f.wi.nqc) {
           f.pr[u] = p.bq[f.wi.bstart + i];
-          f.q[u] = f.pr[u] / p.npb;
+          // phase-A entries carry pair id npairs + p (their own output regions)
+          const int64_t npairs = p.nq * p.npb;
+          f.q[u] = (int)((f.pr[u] >= npairs ? f.pr[u] - npairs : f.pr[u]) / p.npb);
           f.tau[u] = phaseB ? p.tau[f.q[u]] : MV_KEY_PAD;
           f.qn[u] = p.qnorm[f.q[u]];
           f.base[u] = p.poff[f.pr[u]];
@@ -298,7 +300,7 @@ __global__ void __launch_bounds__(kQmThreads, 1)
         rest /= nchunks;
         const int pl = rest % P;
         const int i = rest / P;
-        const int q = mt.pair[i] / p.npb;
+        const int q = (int)((mt.pair[i] >= p.nq * p.npb ? mt.pair[i] - p.nq * p.npb : mt.pair[i]) / p.npb);
         cp_async16(Ab + c * QCMAX * ATOM + swz_off(pl * QC + i, pc, ATOM),
                    p.qplanes + ((int64_t)pl * p.nq + q) * rowbytes + c * ATOM + pc * 16);
       }
@@ -380,7 +382,7 @@ __global__ void __launch_bounds__(kQmThreads, 1)
 #pragma unroll
               for (int j = 0; j < 32; ++j) {
                 kk[j] = ((uint64_t)f2key(dv[j]) << 32) | rk[c0 + j];
-                if (((m >> j) & 1) && (!phaseB || kk[j] < tau)) m2 |= 1u << j;
+                if (((m >> j) & 1) && (!phaseB || kk[j] <= tau)) m2 |= 1u << j;
               }
               if (m2) {
                 int pos = atomicAdd(mt.cnt + qi, __popc(m2));

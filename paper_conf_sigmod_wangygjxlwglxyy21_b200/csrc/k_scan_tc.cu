@@ -18,10 +18,11 @@
 //              survivors are appended to the (query, list) pair's output region (a6).
 //
 // a6 is a filter, not a selection.  The search runs the scan twice:
-//   phase A (p.phase 0) scans each query's rA nearest lists and emits every candidate; a
+//   phase A (p.phase 0) scans a prefix (p.rowcap rows) of each query's rA nearest lists and emits
+//     every candidate; a
 //     per-query select (k_select.cu) turns them into tau_q = the k-th best key so far -- an exact
 //     upper bound of the query's final k-th best;
-//   phase B (p.phase 1) scans the other pairs and emits only keys below tau_q.
+//   phase B (p.phase 1) scans every probed pair and emits only keys <= tau_q.
 // The final select takes the exact top-k of everything emitted.  No per-pair selection state,
 // no epilogue-wide barrier per tile: the epilogue warps run independently.
 //
@@ -56,7 +57,7 @@ __device__ __forceinline__ WorkInfo work_info_of(const TcScanParams& p, int2 it,
   wi.bstart = it.y;
   wi.nqc = min(qchunk, p.boff[it.x + 1] - wi.bstart);
   wi.lstart = p.list_off[wi.l];
-  wi.len = (int)(p.list_off[wi.l + 1] - wi.lstart);
+  wi.len = (int)min64(p.list_off[wi.l + 1] - wi.lstart, p.rowcap);
   wi.ntiles = (wi.len + 127) >> 7;
   return wi;
 }
@@ -282,7 +283,9 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
         const int i = tq + 64 * u;
         if (i < f.wi.nqc) {
           f.pr[u] = p.bq[f.wi.bstart + i];
-          f.q[u] = f.pr[u] / p.npb;
+          // phase-A entries carry pair id npairs + p (their own output regions)
+          const int64_t npairs = p.nq * p.npb;
+          f.q[u] = (int)((f.pr[u] >= npairs ? f.pr[u] - npairs : f.pr[u]) / p.npb);
           f.tau[u] = phaseB ? p.tau[f.q[u]] : MV_KEY_PAD;
           f.qn[u] = p.qnorm[f.q[u]];
           f.qs[u] = TYPE == MV_IVF_SQ8 ? p.qscale[f.q[u]] : 1.0f;
@@ -426,7 +429,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
             if (bad[j] <= th16[j]) {
               // exact test on the full key (distance key, id rank) < tau
               const uint64_t key = ((uint64_t)f2key(bad[j]) << 32) | rk;
-              if (!phaseB || key < mt.tau[i]) pm |= 1u << j;
+              if (!phaseB || key <= mt.tau[i]) pm |= 1u << j;
             }
           }
           if (!valid) pm = 0;

@@ -559,9 +559,10 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
     int32_t* qcfg;
     CK(s.alloc(&qcfg, 2));
     const int64_t npairs = nq * npb;
-    // Seeding (tensor-core path, nprobe >= 2): phase A scans each query's ra[q] nearest lists --
-    // the fewest holding >= 2k candidates -- and emits all of them; their k-th best key tau_q is an
-    // exact upper bound of the query's final k-th best, so phase B emits only keys below it.
+    // Seeding (tensor-core path, nprobe >= 2): phase A scans the first capA rows of each query's
+    // ra[q] nearest lists -- the fewest holding >= max(2k, k+32) such rows -- and emits all of them;
+    // their k-th best key tau_q is an exact upper bound of the query's final k-th best (k distinct
+    // candidates are at or below it), so phase B scans every probed list and emits only keys <= tau_q.
     const char* seed_env = getenv("MV_SEED");
     const bool split = use_tc && npb >= 2 && !(seed_env && seed_env[0] == '0');
     int32_t* ra = nullptr;
@@ -571,20 +572,25 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
     CK(s.alloc(&b.lcount, nv));
     CK(s.alloc(&b.boff, nv + 1));
     CK(s.alloc(&b.bfill, nv));
-    CK(s.alloc(&b.bq, (size_t)npairs));
+    const int64_t nent = split ? 2 * npairs : npairs;  // bucket entries (phase-A entries with seeding)
+    CK(s.alloc(&b.bq, (size_t)nent));
     CK(s.alloc(&b.wcount, nv));
     CK(s.alloc(&b.woff, nv + 1));
-    CK(s.alloc(&b.witems, (size_t)(nv + npairs / qchunk_min + 1)));
-    CK(s.alloc(&b.witems_unsorted, (size_t)(nv + npairs / qchunk_min + 1)));
+    CK(s.alloc(&b.witems, (size_t)(nv + nent / qchunk_min + 1)));
+    CK(s.alloc(&b.witems_unsorted, (size_t)(nv + nent / qchunk_min + 1)));
     CK(s.alloc(&b.qtot, (size_t)(2 * (nq + 1))));
-    CK(s.alloc(&b.poff, (size_t)npairs));
-    CK(s.alloc(&b.pcnt, (size_t)npairs));
+    CK(s.alloc(&b.poff, (size_t)nent));
+    CK(s.alloc(&b.pcnt, (size_t)nent));
     CK(s.alloc(&b.counter, 1));
     // pair regions: the whole list (tensor-core scan: emit-all bound), or min(k, |list|) (SIMT)
     const int capk = use_tc ? 0 : k;
     PlanArgs pa;
     pa.probes = P; pa.nq = nq; pa.npb = npb; pa.nlist = nlist; pa.k = k; pa.capk = capk;
     pa.split = split ? 1 : 0; pa.need = std::max<int64_t>(2 * (int64_t)k, k + 32);
+    // phase A reads the first capA rows of each of a query's nearest lists (a 16-row multiple, at
+    // least two tiles: a tighter tau_q costs less in phase-B emissions than the extra rows)
+    pa.capA = std::max<int64_t>((pa.need + 15) & ~(int64_t)15, 256);
+    if (const char* ce = getenv("MV_CAPA")) pa.capA = std::max<int64_t>(pa.capA, (atoll(ce) + 15) & ~15ll);
     pa.list_off = ix->list_off;
     pa.qlo_any = (use_tc && ix->type == MV_IVF_FLAT) ? qlo_any : nullptr;
     pa.qc_exact = qchunk; pa.p_exact = use_tc ? (ix->type == MV_IVF_FLAT ? 1 : 4) : 1;
@@ -596,6 +602,7 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
     if (use_tc) {
       // exact worst case without a device round trip: nq x (the npb longest lists)
       cap = nq * ix->top_len_prefix[std::min<size_t>(npb, ix->top_len_prefix.size() - 1)];
+      if (split) cap += nq * (pa.need + pa.capA);  // phase-A prefixes: < need + capA rows per query
     } else if (k <= kLocalSelectMaxK) {
       cap = nq * npb * min64(capk, max64(ix->maxlen, 1));
     } else {
@@ -647,16 +654,18 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
       // phase A (or, without seeding, the whole scan emitting every candidate) ...
       auto scan = [&]() { return use_qm ? launch_scan_qm(&ix->xm.m[0], &ix->xm.m[3], tp, st) : launch_scan_tc(ix->xm, tp, st); };
       tp.phase = 0;
+      tp.rowcap = split ? (int)pa.capA : 0x7fffffff;
       tp.wbeg = nullptr;
       tp.nwitems = b.woff + nlist;
       CK(scan());
       prof_mark(ix, st);
       if (split) {
         // ... tau_q = k-th best key of phase A ...
-        CK(launch_tau_select(b.poff, b.pcnt, part, nq, npb, ra, k, tau, tmax, over, st));
+        CK(launch_tau_select(b.poff + npairs, b.pcnt + npairs, part, nq, npb, ra, k, tau, tmax, over, st));
         prof_mark(ix, st);
-        // ... phase B over the remaining pairs, emitting keys < tau_q
+        // ... phase B over every probed pair, emitting keys <= tau_q
         tp.phase = 1;
+        tp.rowcap = 0x7fffffff;
         tp.wbeg = b.woff + nlist;
         tp.nwitems = b.woff + 2 * nlist;
         CK(scan());

@@ -538,14 +538,14 @@ struct Bucketing {
   int32_t* lcount;   // nlist      pairs per list
   int32_t* boff;     // nlist+1    exclusive scan of lcount
   int32_t* bfill;    // nlist      scratch
-  int32_t* bq;       // nq*npb     pair ids grouped by list
+  int32_t* bq;       // nq*npb (x2 with seeding)  pair ids grouped by list
   int32_t* wcount;   // nlist      work items per list
   int32_t* woff;     // nlist+1
   int2* witems;      // <= nlist + nq*npb   (list, first bucket position), longest first
   int2* witems_unsorted;
   int64_t* qtot;     // nq+1       per-query candidate capacity, then exclusive scan
-  int64_t* poff;     // nq*npb     region offset per pair
-  int32_t* pcnt;     // nq*npb     candidates written per pair
+  int64_t* poff;     // nq*npb (x2 with seeding: phase-A entries at nq*npb + p)  region offset per pair
+  int32_t* pcnt;     // nq*npb (x2 with seeding)  candidates written per pair
   int32_t* counter;  // 1          persistent scan work counter
 };
 // a4 in one cooperative launch (k_bucket.cu).  With the seeding split the pairs of query q with
@@ -557,6 +557,7 @@ struct PlanArgs {
   int npb, nlist, k, capk;  // capk > 0: SIMT local-selection regions min(capk, |list|); 0: |list|
   int split;               // 1: seeding phase (ra[q] nearest lists) + phase B
   int64_t need;            // seeding: candidates the phase-A lists must hold
+  int64_t capA;            // seeding: phase A scans the first min(|l|, capA) rows of each of its lists
   const int64_t* list_off;
   const int* qlo_any;      // FLAT: some query needs its lo plane (nullable)
   int qc_exact, p_exact, qc_split, p_split;
@@ -601,7 +602,8 @@ struct TcScanParams {
   int qchunk_split;        // FLAT: queries per work item when the queries need the lo plane (P = 2)
   const int32_t* cfg;      // device {query chunk, planes} of this search (launch_scan_cfg)
   int nlist;               // virtual list v >= nlist is list v - nlist (phase-B pairs)
-  int phase;               // 0: seeding phase A (emit every candidate); 1: phase B (emit keys < tau_q)
+  int phase;               // 0: seeding phase A (emit every candidate); 1: phase B (emit keys <= tau_q)
+  int rowcap;              // rows scanned per list in this launch (phase A: capA; else INT_MAX)
   int64_t nq;              // FLAT query planes are plane-major [2][nq][dpad]
   int off_x, off_q, q_bytes, off_meta, meta_bytes, off_side, off_bar, smem_total;
   const int64_t* list_off;

@@ -1,0 +1,10 @@
+python -c "import __graft_entry__ as g; g.build()" || exit 1
+run() {
+  env $1 timeout 600 python bench.py --config ${2:-c2} --steps 20 --warmup 3 --no-cpu-baseline > gpurun_out/x.json 2> gpurun_out/x.err
+  python -c "import json; d=json.load(open('gpurun_out/x.json')); print('$1 ${2:-c2}', round(d['value']), d['config'].get('recall@10'), {a: round(b,3) for a,b in d['stage_ms'].items()}, d['index']['last_scan'])" || tail -3 gpurun_out/x.err
+}
+run MV_CAPA=128
+run MV_CAPA=256
+run MV_CAPA=100000
+run MV_CAPA=256 c3
+run MV_CAPA=100000 c3
