@@ -40,6 +40,10 @@ CONFIGS = {
                nlist=16384, nprobe=32, nq=10_000, k=100, kind="sq8", metric="ip", bitset=10),
     "c4": dict(workload="sift10m_ivfflat_l2_nlist16384_nprobe128_k2048", data="sift", n=10_000_000, d=128,
                nlist=16384, nprobe=128, nq=10_000, k=2048, kind="flat", metric="l2", bitset=0),
+    # 1B rows, vector-sharded (row r -> shard r mod S): each GPU holds one shard of 1B / S rows.
+    # At N=1 the GPU holds shard 0 of --c5-shards (default 8): the per-GPU workload of the 8-GPU job.
+    "c5": dict(workload="sift1b_ivfsq8_l2_nlist65536_nprobe64_k10", data="sift", n=1_000_000_000, d=128,
+               nlist=65536, nprobe=64, nq=10_000, k=10, kind="sq8", metric="l2", bitset=0, sharded_build=True),
 }
 METRIC = "queries/s at recall@10>=0.95 and % HBM/tensor roofline, 1/2/4/8 B200"
 L2_BYTES = 126 * 2**20
@@ -61,6 +65,54 @@ def peaks():
 # ------------------------------------------------------------------------------------------
 # data (seeded, synthetic; mvgen holds none of the method's arithmetic)
 # ------------------------------------------------------------------------------------------
+def build_sharded(cfg, device, shard, nshard, Index, chunk=1 << 24, ngt=1000):
+    """c5: 1B-row SIFT-shaped IVF_SQ8 index, this GPU's shard (rows r with r % nshard == shard),
+    generated on the device chunk by chunk (mvgen's counter hash regenerates any row anywhere) and
+    added through mv_index_add.  Centroids: seeded k-means on the first 64*nlist rows; SQ8 params:
+    per-dimension min/max of the same rows (replicated on every shard).  Ground truth for recall:
+    exact top-10 over this shard's raw rows for the first `ngt` queries (integer data: exact in fp32)."""
+    import mvgen as G
+    from mvgen.kmeans import kmeans
+    spec = G.SiftSpec(d=cfg["d"])
+    ntr = min(cfg["n"], 64 * cfg["nlist"])
+    Xtr = G.sift_base(ntr, d=cfg["d"], device=device, spec=spec)
+    C = kmeans(Xtr, cfg["nlist"], iters=10)
+    vmin = Xtr.min(0).values.contiguous()
+    vdiff = (Xtr.max(0).values - vmin).contiguous()
+    del Xtr
+    torch.cuda.empty_cache()
+    Q = G.sift_queries(cfg["nq"], d=cfg["d"], device=device, spec=spec)
+    ix = Index(cfg["d"], cfg["metric"], cfg["kind"], cfg["nlist"], device=device.index)
+    ix.set_centroids(C)
+    ix.set_sq8(vmin, vdiff)
+    nloc = (cfg["n"] - shard + nshard - 1) // nshard
+    Qg = Q[:ngt]
+    qn = (Qg * Qg).sum(1)
+    gd = torch.full((ngt, 10), float("inf"), device=device)
+    gi = torch.full((ngt, 10), -1, dtype=torch.int64, device=device)
+    Xc = torch.empty((min(chunk, nloc), cfg["d"]), dtype=torch.float32, device=device)
+    for s0 in range(0, nloc, chunk):
+        m = min(chunk, nloc - s0)
+        rows = torch.arange(s0, s0 + m, dtype=torch.int64, device=device) * nshard + shard
+        for a in range(0, m, 1 << 18):
+            b = min(m, a + (1 << 18))
+            Xc[a:b] = spec.rows_at(rows[a:b], G.SEED_BASE)
+        ix.add(Xc[:m], rows)
+        for a in range(0, m, 1 << 20):
+            b = min(m, a + (1 << 20))
+            xb = Xc[a:b]
+            d = qn[:, None] + (xb * xb).sum(1)[None, :] - 2.0 * (Qg @ xb.T)
+            td, ti = torch.topk(d, 10, dim=1, largest=False)
+            cd = torch.cat([gd, td], 1)
+            ci = torch.cat([gi, rows[a:b][ti]], 1)
+            o = torch.argsort(cd, dim=1)[:, :10]
+            gd, gi = torch.gather(cd, 1, o), torch.gather(ci, 1, o)
+        log(f"[bench] c5 shard {shard}/{nshard}: {s0 + m}/{nloc} rows added")
+    del Xc
+    torch.cuda.empty_cache()
+    return ix, Q, C, gi, nloc
+
+
 def make_data(cfg, device):
     import mvgen as G
     from mvgen.kmeans import kmeans
@@ -213,6 +265,7 @@ def main():
     ap.add_argument("--oracle-sample", type=int, default=0, help="queries for the CPU oracle (0 = auto)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--nprobe", type=int, default=0)
+    ap.add_argument("--c5-shards", type=int, default=8, help="c5: shards of the 1B index (>= the GPU count)")
     args = ap.parse_args()
     cfg = dict(CONFIGS[args.config])
     if args.nprobe:
@@ -236,30 +289,43 @@ def main():
     from paper_conf_sigmod_wangygjxlwglxyy21_b200 import Index, merge_topk
 
     t0 = time.perf_counter()
-    X, Q, C, bs = make_data(cfg, dev)
-    if dist:
-        tdist.broadcast(C, 0)
-    n = cfg["n"]
-    ids = torch.arange(n, dtype=torch.int64, device=dev)
     from paper_conf_sigmod_wangygjxlwglxyy21_b200.sharded import ShardedIndex
-    ix = Index(cfg["d"], cfg["metric"], cfg["kind"], cfg["nlist"], device=local)
-    sh = ShardedIndex(ix) if dist else None
-    if dist:
-        sh.set_centroids(C)
+    sharded_build = cfg.get("sharded_build", False)
+    gt_c5 = None
+    if sharded_build:
+        if args.impl == "reference":
+            print(json.dumps({"impl": "reference", "unavailable": "c5 (1B rows): the CPU oracle cannot hold a "
+                              "125M-row shard; the reference arm covers c1-c4"}), flush=True)
+            return 0
+        nshard = max(args.c5_shards, world)
+        ix, Q, C, gt_c5, n = build_sharded(cfg, dev, rank, nshard, Index)
+        X, bs, ids = None, None, None
+        sh = ShardedIndex(ix) if dist else None
+        cfg["workload"] += f"_shard{'0' if world == 1 else 'r'}of{nshard}"
     else:
-        ix.set_centroids(C)
-    if cfg["kind"] == "sq8":
-        import mvgen as G
-        g = torch.Generator(device="cpu").manual_seed(G.SEED_SQ8)
-        samp = torch.randperm(n, generator=g)[: min(n, 64 * cfg["nlist"])].to(dev)
-        xs = X[samp]
-        vmin = xs.min(0).values.contiguous()
-        vdiff = (xs.max(0).values - vmin).contiguous()
-        (sh.set_sq8 if dist else ix.set_sq8)(vmin, vdiff)
-    if dist:
-        sh.add(X, ids)   # every rank keeps the rows it owns (id % world == rank)
-    else:
-        ix.add(X, ids)
+        X, Q, C, bs = make_data(cfg, dev)
+        if dist:
+            tdist.broadcast(C, 0)
+        n = cfg["n"]
+        ids = torch.arange(n, dtype=torch.int64, device=dev)
+        ix = Index(cfg["d"], cfg["metric"], cfg["kind"], cfg["nlist"], device=local)
+        sh = ShardedIndex(ix) if dist else None
+        if dist:
+            sh.set_centroids(C)
+        else:
+            ix.set_centroids(C)
+        if cfg["kind"] == "sq8":
+            import mvgen as G
+            g = torch.Generator(device="cpu").manual_seed(G.SEED_SQ8)
+            samp = torch.randperm(n, generator=g)[: min(n, 64 * cfg["nlist"])].to(dev)
+            xs = X[samp]
+            vmin = xs.min(0).values.contiguous()
+            vdiff = (xs.max(0).values - vmin).contiguous()
+            (sh.set_sq8 if dist else ix.set_sq8)(vmin, vdiff)
+        if dist:
+            sh.add(X, ids)   # every rank keeps the rows it owns (id % world == rank)
+        else:
+            ix.add(X, ids)
     torch.cuda.synchronize()
     log(f"[bench] rank {rank}: data + index build {time.perf_counter() - t0:.1f}s (ntotal {ix.ntotal})")
     k, nprobe, nq = cfg["k"], cfg["nprobe"], cfg["nq"]
@@ -339,7 +405,12 @@ def main():
 
     # ---- recall@10 vs exact ground truth (rank 0 holds the full data) ----
     rec = None
-    if rank == 0:
+    if rank == 0 and gt_c5 is not None:
+        if dist:  # the merged result against the union of the shards' exact top-10 is not held here
+            rec = None
+        else:     # this shard's search against this shard's exact top-10 (first 1000 queries)
+            rec = recall_at(gt_c5, I[: gt_c5.shape[0]], 10)
+    elif rank == 0:
         gt = ground_truth(X, Q, 10, cfg["metric"], bs, nbits)
         rec = recall_at(gt, I, 10)
 
@@ -365,7 +436,9 @@ def main():
             pass
 
     cpu = None
-    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+    if rank == 0 and world == 1 and not args.no_cpu_baseline and sharded_build:
+        cpu = {"skipped": "c5: the numpy oracle cannot hold a 125M-row shard; see c1-c4"}
+    elif rank == 0 and world == 1 and not args.no_cpu_baseline:
         try:
             cpu = cpu_baseline(cfg, ix, X, ids, Q, C, bs, args.oracle_sample)
         except Exception as ex:  # reported, never fatal for the GPU number
@@ -382,7 +455,10 @@ def main():
                        "bitset": f"{cfg['bitset']}% excluded" if bs is not None else None,
                        "parallelism": f"vector-shard x{world}" if world > 1 else "single GPU",
                        "l2_flush": f"not needed: index payload {scan_bytes * world / 1e9:.2f} GB > 126 MB L2",
-                       "recall@10": rec},
+                       "recall@10": rec,
+                       **({"n_total": cfg["n"], "n_local": n, "shards": max(args.c5_shards, world),
+                           "recall_note": "recall@10 of this shard's result vs this shard's exact top-10, "
+                                          "first 1000 queries"} if sharded_build else {})},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm_peak, "unit": "GB/s",
                          "frac": achieved / hbm_peak, "traffic": traffic, "peak_source": peak_src,
                          "kernel": "k_scan_tc (a5+a6), phases A+B", "algorithmic_bytes_per_launch": scan_bytes,

@@ -109,8 +109,12 @@ class SiftSpec:
         return hash_u31(row_seed, 21, rows) % self.n_micro
 
     def rows(self, row0: int, n: int, row_seed: int, device="cpu") -> torch.Tensor:
-        d = self.d
-        rows = torch.arange(row0, row0 + n, dtype=torch.int64, device=device)
+        return self.rows_at(torch.arange(row0, row0 + n, dtype=torch.int64, device=device), row_seed)
+
+    def rows_at(self, rows: torch.Tensor, row_seed: int) -> torch.Tensor:
+        """Rows with the given global indices (int64 tensor): any subset of the base set, e.g. the
+        rows one shard of a vector-sharded index owns, regenerated bit-identically anywhere."""
+        d, device = self.d, rows.device
         m = self.micro_of(rows, row_seed)                       # micro centre per row
         t = hash_u31(self.seed, 13, m) % self.n_top             # its top centre
         j = torch.arange(d, dtype=torch.int64, device=device)

@@ -7,7 +7,8 @@
 // tensor-core contraction.  PAPER.md:590-596: per-worker partial results merged at the end.
 //
 // Work item = (list l, <= qchunk queries probing l).  Persistent CTA per SM, warp-specialised:
-//   warp 0     TMA producer: list tiles (128 rows x one 128-B / 32-B swizzle atom per stage) and
+//   warp 0     TMA producer: list tiles (128 rows x one 128-B (FLAT; SQ8 with 128-multiple rows) or
+//              32-B (other SQ8) swizzle atom per stage) and
 //              the tiles' side data (norms, id ranks, ids) by bulk copy
 //   warp 1     TMEM owner + single-thread tcgen05.mma issuer
 //              D[128 vectors x N] (+)= X_tile[128 x K] . Qplanes[N x K]^T, N = P x roundup16(nq)
@@ -39,6 +40,14 @@ namespace mv {
 using namespace sm100;
 
 __device__ __forceinline__ void named_bar(int id, int n) { asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory"); }
+// 16-B shared-memory load through an explicit shared address (the metadata pointers are generic)
+__device__ __forceinline__ float4 lds_f4(const float* p) {
+  float4 v;
+  asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];"
+               : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w)
+               : "r"(sm100::smem_u32(p)));
+  return v;
+}
 
 // CTA-0 event timeline for MV_SCAN_TRACE (row r holds up to 1024 clock64 stamps)
 #define MV_TRACE(row, idx)                                                                      \
@@ -82,6 +91,8 @@ struct Meta {
   float* thf;      // badness bound: a candidate can pass only if badness <= thf (NaN: padding column)
   float* qnf;      // (float)||q||^2
   float* qs;       // SQ8 digit scale
+  float* qaf;      // SQ8 (float) q.a
+  float* thc;      // SQ8 fp32-filter bound: thf + the column's share of the filter error bound
   uint64_t* tau;   // exact bound: emit only keys < tau
   int64_t* base;   // output region of the pair
   double* qn;      // ||q||^2 (fp64)
@@ -97,20 +108,21 @@ __device__ __forceinline__ Meta meta_at(uint8_t* m, int QCP) {
   r.thf = reinterpret_cast<float*>(r.cnt + QCP);
   r.qnf = r.thf + QCP;
   r.qs = r.qnf + QCP;
-  r.tau = reinterpret_cast<uint64_t*>(m + 20 * QCP);
+  r.qaf = r.qs + QCP;
+  r.thc = r.qaf + QCP;
+  r.tau = reinterpret_cast<uint64_t*>(m + 28 * QCP);
   r.base = reinterpret_cast<int64_t*>(r.tau + QCP);
   r.qn = reinterpret_cast<double*>(r.base + QCP);
   r.qa = r.qn + QCP;
   return r;
 }
-constexpr int kMetaPerQuery = 56;  // bytes (+ a 32-B work-item header)
+constexpr int kMetaPerQuery = 64;  // bytes (+ a 32-B work-item header)
 
-template <int TYPE>
+template <int TYPE, int ATOM, bool SMALLD>
 __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__ XMaps xm, const TcScanParams p) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~(uintptr_t)1023);
   constexpr int ESZ = TYPE == MV_IVF_FLAT ? 4 : 1;
-  constexpr int ATOM = TYPE == MV_IVF_FLAT ? 128 : 32;
   constexpr int PMAX = TYPE == MV_IVF_FLAT ? 2 : 4;
   const int nstage = p.nstage, nchunks = p.nchunks;
   const int QCP = (p.qchunk + 15) & ~15;       // metadata capacity (the largest chunk)
@@ -324,6 +336,18 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
           mt.qn[i] = cur.qn[u];
           mt.qs[i] = cur.qs[u];
           mt.qa[i] = cur.qa[u];
+          mt.qaf[i] = (float)cur.qa[u];
+          if (TYPE == MV_IVF_SQ8) {
+            // |fp32 filter - exact| <= 2^-21 (||q||^2 + ||x||^2 + 2 (s Amax + |q.a|)) with Amax the
+            // largest |digit-weighted partial| (127 * 255 * dpad * (1 + 2^-7 + ...)); + 2^-23 |thf|
+            // for the final rounding to fp32.  ||x||^2's share is taken per row (xnlo).
+            const float thf = mt.thf[i];
+            const double amax = 127.0 * 255.0 * p.dpad * 1.0079;
+            const double mcol = 4.76837158203125e-7 * (cur.qn[u] + 2.0 * ((double)cur.qs[u] * amax + fabs(cur.qa[u])));
+            mt.thc[i] = (float)((double)thf + mcol + fabs((double)thf) * 1.1920928955078125e-7);
+          } else {
+            mt.thc[i] = mt.thf[i];
+          }
           mt.base[i] = cur.base[u];
         } else if (i < NQ) {  // padding column: no comparison passes
           mt.thf[i] = __int_as_float(0x7fffffff);
@@ -331,6 +355,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
           mt.qn[i] = 0.0;
           mt.qs[i] = 0.f;
           mt.qa[i] = 0.0;
+          mt.qaf[i] = 0.f;
+          mt.thc[i] = __int_as_float(0x7fffffff);
         }
       }
       named_bar(2, 64);
@@ -384,6 +410,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
           valid = !bit_excluded(p.bitset, p.nbits, reinterpret_cast<const int64_t*>(sd + kSideIds)[(row0 & 1) + row]);
         const double xn = use_norms ? reinterpret_cast<const double*>(sd)[(row0 & 1) + row] : 0.0;
         const float xnf = (float)xn;
+        const float xnlo = xnf - xnf * 4.76837158203125e-7f;  // SQ8 filter: the row's share of the margin
         mbar_wait(&tfull[a], (titer / NACC) & 1);
         if (et == 0) MV_TRACE(6, titer);
         tc_fence_after();
@@ -397,42 +424,70 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
 #pragma unroll
               for (int j = 0; j < 16; ++j) r[pl][j] = 0u;
           }
-          // the chunk's per-query constants, vector loads overlapping the TMEM load latency
-          float qn16[16], th16[16];
+          tmem_wait_ld();
+          // pass 1 (every row x column): the threshold filter, branch-free.  FLAT computes the exact
+          // fp32 distance; SQ8 an fp32 bound-checked approximation (the exact fp64 value in pass 2)
+          float bad[16];
+          uint32_t pm = 0, pe = 0;  // pe (FLAT): entries exactly at the bound, which need the key test
 #pragma unroll
           for (int v = 0; v < 4; ++v) {
-            const float4 a4 = reinterpret_cast<const float4*>(mt.qnf + qc)[v];
-            const float4 t4 = reinterpret_cast<const float4*>(mt.thf + qc)[v];
-            qn16[4 * v] = a4.x; qn16[4 * v + 1] = a4.y; qn16[4 * v + 2] = a4.z; qn16[4 * v + 3] = a4.w;
-            th16[4 * v] = t4.x; th16[4 * v + 1] = t4.y; th16[4 * v + 2] = t4.z; th16[4 * v + 3] = t4.w;
-          }
-          tmem_wait_ld();
-          float bad[16];
-          uint32_t pm = 0;
-#pragma unroll
-          for (int j = 0; j < 16; ++j) {
-            const int i = qc + j;
-            // badness = L2 distance or -IP (smaller is better)
-            if (TYPE == MV_IVF_FLAT) {
-              // exact for tf32-representable data (the only FLAT data this path accepts)
-              const float dot = __uint_as_float(r[0][j]) + __uint_as_float(r[1 % PMAX][j]);
-              bad[j] = use_norms ? (qn16[j] + xnf) - 2.0f * dot : -dot;
-            } else {
-              // int32-exact digit partials; the L2 expansion is combined in fp64 (the norms are
-              // ~400x the near-neighbour distances on SIFT-scale data)
-              const double acc = (double)(int)r[0][j] + (double)(int)r[1 % PMAX][j] * (1.0 / 128.0) +
-                                 (double)(int)r[2 % PMAX][j] * (1.0 / 16384.0) +
-                                 (double)(int)r[3 % PMAX][j] * (1.0 / 2097152.0);
-              const double dot = fma((double)mt.qs[i], acc, mt.qa[i]);
-              bad[j] = use_norms ? (float)((mt.qn[i] + xn) - 2.0 * dot) : (float)(-dot);
+            const float4 qn4 = lds_f4(mt.qnf + qc + 4 * v);
+            const float4 th4 = lds_f4((TYPE == MV_IVF_SQ8 ? mt.thc : mt.thf) + qc + 4 * v);
+            float4 qs4 = qn4, qa4 = qn4;
+            if (TYPE == MV_IVF_SQ8) {
+              qs4 = lds_f4(mt.qs + qc + 4 * v);
+              qa4 = lds_f4(mt.qaf + qc + 4 * v);
             }
-            if (bad[j] <= th16[j]) {
-              // exact test on the full key (distance key, id rank) < tau
-              const uint64_t key = ((uint64_t)f2key(bad[j]) << 32) | rk;
-              if (!phaseB || key <= mt.tau[i]) pm |= 1u << j;
+            const float qnv[4] = {qn4.x, qn4.y, qn4.z, qn4.w}, thv[4] = {th4.x, th4.y, th4.z, th4.w};
+            const float qsv[4] = {qs4.x, qs4.y, qs4.z, qs4.w}, qav[4] = {qa4.x, qa4.y, qa4.z, qa4.w};
+#pragma unroll
+            for (int u = 0; u < 4; ++u) {
+              const int j = 4 * v + u;
+              if (TYPE == MV_IVF_FLAT) {
+                // badness = L2 distance or -IP; exact for tf32-representable data
+                const float dot = __uint_as_float(r[0][j]) + __uint_as_float(r[1 % PMAX][j]);
+                bad[j] = use_norms ? (qnv[u] + xnf) - 2.0f * dot : -dot;
+              } else {
+                // digit partials converted exactly (magic number: |D| < 2^22 for rows of <= 128
+                // codes), combined in fp32; the error bound is folded into thc (per column) and xnlo
+                float fd[4];
+#pragma unroll
+                for (int pl = 0; pl < 4; ++pl)
+                  fd[pl] = SMALLD ? __int_as_float(0x4B400000 + (int)r[pl % PMAX][j]) - 12582912.0f
+                                  : __int2float_rn((int)r[pl % PMAX][j]);
+                const float accf =
+                    fmaf(fd[3], 4.76837158203125e-7f, fmaf(fd[2], 6.103515625e-5f, fmaf(fd[1], 0.0078125f, fd[0])));
+                const float dotf = fmaf(qsv[u], accf, qav[u]);
+                bad[j] = use_norms ? (qnv[u] + xnlo) - 2.0f * dotf : -dotf;
+              }
+              pm |= (bad[j] <= thv[u] ? 1u : 0u) << j;
+              if (TYPE == MV_IVF_FLAT) pe |= (bad[j] == thv[u] ? 1u : 0u) << j;
             }
           }
           if (!valid) pm = 0;
+          if (TYPE == MV_IVF_FLAT) pe &= phaseB ? pm : 0u;
+          // pass 2 (flagged entries only): SQ8's exact fp64 badness; the exact key test at the bound
+          if (__any_sync(MV_FULL, (TYPE == MV_IVF_SQ8 ? pm : pe) != 0)) {
+#pragma unroll
+            for (int j = 0; j < 16; ++j) {
+              if (((TYPE == MV_IVF_SQ8 ? pm : pe) >> j) & 1) {
+                const int i = qc + j;
+                const float thj = mt.thf[i];
+                if (TYPE == MV_IVF_SQ8) {
+                  // int32-exact digit partials; the L2 expansion is combined in fp64 (the norms are
+                  // ~400x the near-neighbour distances on SIFT-scale data)
+                  const double acc = (double)(int)r[0][j] + (double)(int)r[1 % PMAX][j] * (1.0 / 128.0) +
+                                     (double)(int)r[2 % PMAX][j] * (1.0 / 16384.0) +
+                                     (double)(int)r[3 % PMAX][j] * (1.0 / 2097152.0);
+                  const double dot = fma((double)mt.qs[i], acc, mt.qa[i]);
+                  bad[j] = use_norms ? (float)((mt.qn[i] + xn) - 2.0 * dot) : (float)(-dot);
+                }
+                bool ok = bad[j] <= thj;
+                if (ok && phaseB && bad[j] == thj) ok = (((uint64_t)f2key(bad[j]) << 32) | rk) <= mt.tau[i];
+                if (!ok) pm &= ~(1u << j);
+              }
+            }
+          }
           if (__any_sync(MV_FULL, pm != 0) && !(p.dbg & 1)) {
             // ballot per column; lane j reserves column j's slots with one shared atomic
             uint32_t mj[16];
@@ -557,7 +612,9 @@ cudaError_t launch_tf32_check(const float* x, int64_t n, int* flag, cudaStream_t
 // + the side-data ring; the deepest X ring (<= the type's cap) that fits in 227 KB.
 static bool tc_scan_layout(int type, int dpad, int qc, int ns, TcScanParams& p) {
   const int esz = type == MV_IVF_FLAT ? 4 : 1;
-  const int atom = type == MV_IVF_FLAT ? 128 : 32;
+  // swizzle-atom row: 128 B (FLAT: 32 fp32; SQ8 rows of a multiple of 128 codes), else 32 B (SQ8)
+  const int atom = (type == MV_IVF_FLAT || dpad % 128 == 0) ? 128 : 32;
+  p.atom = atom;
   // FLAT: qc queries of one plane (tf32-exact queries) or qc/2 queries of two (hi/lo) in the same
   // operand rows; SQ8: four digit planes
   const int rows_per_q = type == MV_IVF_FLAT ? 1 : 4;
@@ -588,9 +645,10 @@ static bool tc_scan_layout(int type, int dpad, int qc, int ns, TcScanParams& p) 
 }
 
 bool tc_scan_plan(int type, int dpad, int k, TcScanParams& p) {
+  const bool wide = type == MV_IVF_FLAT || dpad % 128 == 0;  // 16-KB stages
   const int qcmax = type == MV_IVF_FLAT ? 96 : 64;
-  const int nscap = type == MV_IVF_FLAT ? 8 : 24;
-  const int nsmin = type == MV_IVF_FLAT ? 4 : 6;  // >= 64 KB (FLAT) / 24 KB (SQ8) of list tiles in flight
+  const int nscap = wide ? 8 : 24;
+  const int nsmin = wide ? 4 : 6;  // >= 64 KB (16-KB stages) / 24 KB (4-KB stages) of list tiles in flight
   p.k = k;
   for (int qc = qcmax; qc >= 32; qc -= 32)
     for (int ns = nscap; ns >= nsmin; --ns)
@@ -599,7 +657,11 @@ bool tc_scan_plan(int type, int dpad, int k, TcScanParams& p) {
 }
 
 cudaError_t launch_scan_tc(const XMaps& xm, const TcScanParams& p, cudaStream_t st) {
-  auto kern = p.type == MV_IVF_FLAT ? k_scan_tc<MV_IVF_FLAT> : k_scan_tc<MV_IVF_SQ8>;
+  // SMALLD: SQ8 rows of <= 128 codes, whose digit partials stay below 2^22 in magnitude
+  const bool sd = p.dpad <= 128;
+  auto kern = p.type == MV_IVF_FLAT ? k_scan_tc<MV_IVF_FLAT, 128, true>
+              : p.atom == 128       ? (sd ? k_scan_tc<MV_IVF_SQ8, 128, true> : k_scan_tc<MV_IVF_SQ8, 128, false>)
+                                    : (sd ? k_scan_tc<MV_IVF_SQ8, 32, true> : k_scan_tc<MV_IVF_SQ8, 32, false>);
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, p.smem_total);
   if (e != cudaSuccess) return e;
   int dev = 0, nsm = kNumSMs;

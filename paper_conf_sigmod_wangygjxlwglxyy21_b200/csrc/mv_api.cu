@@ -364,7 +364,24 @@ mv_status mv_index_add(mv_index* ix, const float* vectors, const int64_t* ids, i
   CK(s.alloc(&new_off, nlist + 1));
   // a0: assignment I(v) = closest centroid (the coarse kernel with nprobe = 1)
   CK(launch_query_prep(x, n, ix->d, dpad, xpad, xnorm, st));
-  CK(launch_coarse(xpad, n, dpad, ix->cpad, ix->cnorm, nlist, ix->metric, 1, lists, st));
+  // on the tensor cores in row blocks (each block's score matrix <= 1 GB), else SIMT
+  {
+    const int64_t lds = (nlist + 3) & ~3;
+    const int64_t sub = std::min<int64_t>(n, std::max<int64_t>(4096, (int64_t(1) << 28) / lds));
+    bool done = false;
+    if (nlist > 1 && ix->cmap_ok) {
+      float* qhl;
+      CK(s.alloc(&qhl, (size_t)2 * sub * dpad));
+      for (int64_t r0 = 0; r0 < n; r0 += sub) {
+        const int64_t m = std::min(sub, n - r0);
+        Scratch sb(st);  // the block's score matrix, freed (stream-ordered) before the next block
+        CK(launch_hilo(x + r0 * ix->d, m, ix->d, dpad, qhl, nullptr, st));
+        CK(run_coarse(ix, xpad + r0 * dpad, qhl, nullptr, m, 1, lists + r0, sb, st));
+      }
+      done = true;
+    }
+    if (!done) CK(launch_coarse(xpad, n, dpad, ix->cpad, ix->cnorm, nlist, ix->metric, 1, lists, st));
+  }
   CK(cudaMemsetAsync(cnt, 0, sizeof(int32_t) * nlist, st));
   CK(launch_count_lists(lists, n, cnt, st));
   CK(launch_scan_i32(cnt, nlist, addoff, st));
@@ -439,11 +456,14 @@ mv_status mv_index_add(mv_index* ix, const float* vectors, const int64_t* ids, i
   ix->ntotal = ntot;
   if (ix->type == MV_IVF_FLAT && hflag) ix->tf32_exact = false;
   ix->xmap_ok = ntot <= 0x7fffffffLL;
+  // one swizzle atom per box row: 128 B (FLAT: 32 fp32; SQ8 when dpad is a multiple of 128), else 32 B
+  const bool wide = ix->type == MV_IVF_FLAT || dpad % 128 == 0;
   for (int i = 0; i < 4 && ix->xmap_ok; ++i)
     ix->xmap_ok = make_tmap_2d(&ix->xm.m[i], payload,
                                ix->type == MV_IVF_FLAT ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_UINT8,
-                               (uint64_t)dpad, (uint64_t)ntot, (uint64_t)dpad * esize, 32, 128 >> i,
-                               ix->type == MV_IVF_FLAT ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_32B);
+                               (uint64_t)dpad, (uint64_t)ntot, (uint64_t)dpad * esize,
+                               ix->type == MV_IVF_FLAT ? 32 : (wide ? 128 : 32), 128 >> i,
+                               wide ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_32B);
   ix->maxlen = 0;
   std::vector<int64_t> lens(nlist);
   for (int l = 0; l < nlist; ++l) {

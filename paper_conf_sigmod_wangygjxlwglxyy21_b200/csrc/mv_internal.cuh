@@ -598,7 +598,7 @@ cudaError_t launch_scan(const ScanArgs& a, cudaStream_t st);
 
 // k_scan_tc.cu (tcgen05 path): a filter-and-emit scan run in two phases
 struct TcScanParams {
-  int type, metric, dpad, k, npb, qchunk, nchunks, nstage, ncol, tmem_cols, nacc;
+  int type, metric, dpad, k, npb, qchunk, nchunks, nstage, ncol, tmem_cols, nacc, atom;
   int qchunk_split;        // FLAT: queries per work item when the queries need the lo plane (P = 2)
   const int32_t* cfg;      // device {query chunk, planes} of this search (launch_scan_cfg)
   int nlist;               // virtual list v >= nlist is list v - nlist (phase-B pairs)
