@@ -40,6 +40,11 @@ namespace mv {
 using namespace sm100;
 
 __device__ __forceinline__ void named_bar(int id, int n) { asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory"); }
+template <int W>
+__device__ __forceinline__ void tmem_ld_w(uint32_t taddr, uint32_t (&r)[W]) {
+  if constexpr (W == 16) sm100::tmem_ld16(taddr, r);
+  else sm100::tmem_ld8(taddr, r);
+}
 // 16-B shared-memory load through an explicit shared address (the metadata pointers are generic)
 __device__ __forceinline__ float4 lds_f4(const float* p) {
   float4 v;
@@ -132,6 +137,9 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
   const bool use_norms = p.metric == MV_L2;
   const bool use_ids = p.bitset != nullptr;
   const bool phaseB = p.phase != 0;
+  // epilogue column chunk: 16 (FLAT), 8 (SQ8: few queries per list, so both warps of a lane quarter
+  // get columns)
+  constexpr int W = TYPE == MV_IVF_FLAT ? 16 : 8;
 
   uint8_t* Xs = sm + p.off_x;
   uint8_t* Qs = sm + p.off_q;
@@ -415,22 +423,22 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
         if (et == 0) MV_TRACE(6, titer);
         tc_fence_after();
         const uint32_t tbase = tmem + a * p.ncol + ((uint32_t)(quarter * 32) << 16);
-        for (int qc = half * 16; qc < ((p.dbg & 2) ? 0 : NQ); qc += 32) {
-          uint32_t r[PMAX][16];
+        for (int qc = half * W; qc < ((p.dbg & 2) ? 0 : NQ); qc += 2 * W) {
+          uint32_t r[PMAX][W];
 #pragma unroll
           for (int pl = 0; pl < PMAX; ++pl) {
-            if (pl < P) tmem_ld16(tbase + pl * NQ + qc, r[pl]);
+            if (pl < P) tmem_ld_w<W>(tbase + pl * NQ + qc, r[pl]);
             else
 #pragma unroll
-              for (int j = 0; j < 16; ++j) r[pl][j] = 0u;
+              for (int j = 0; j < W; ++j) r[pl][j] = 0u;
           }
           tmem_wait_ld();
           // pass 1 (every row x column): the threshold filter, branch-free.  FLAT computes the exact
           // fp32 distance; SQ8 an fp32 bound-checked approximation (the exact fp64 value in pass 2)
-          float bad[16];
+          float bad[W];
           uint32_t pm = 0, pe = 0;  // pe (FLAT): entries exactly at the bound, which need the key test
 #pragma unroll
-          for (int v = 0; v < 4; ++v) {
+          for (int v = 0; v < W / 4; ++v) {
             const float4 qn4 = lds_f4(mt.qnf + qc + 4 * v);
             const float4 th4 = lds_f4((TYPE == MV_IVF_SQ8 ? mt.thc : mt.thf) + qc + 4 * v);
             float4 qs4 = qn4, qa4 = qn4;
@@ -469,7 +477,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
           // pass 2 (flagged entries only): SQ8's exact fp64 badness; the exact key test at the bound
           if (__any_sync(MV_FULL, (TYPE == MV_IVF_SQ8 ? pm : pe) != 0)) {
 #pragma unroll
-            for (int j = 0; j < 16; ++j) {
+            for (int j = 0; j < W; ++j) {
               if (((TYPE == MV_IVF_SQ8 ? pm : pe) >> j) & 1) {
                 const int i = qc + j;
                 const float thj = mt.thf[i];
@@ -490,17 +498,17 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
           }
           if (__any_sync(MV_FULL, pm != 0) && !(p.dbg & 1)) {
             // ballot per column; lane j reserves column j's slots with one shared atomic
-            uint32_t mj[16];
+            uint32_t mj[W];
             int mine = 0;
 #pragma unroll
-            for (int j = 0; j < 16; ++j) {
+            for (int j = 0; j < W; ++j) {
               mj[j] = __ballot_sync(MV_FULL, (pm >> j) & 1);
               if (lane == j) mine = __popc(mj[j]);
             }
             int pos = 0;
             if (mine) pos = atomicAdd(mt.cnt + qc + lane, mine);
 #pragma unroll
-            for (int j = 0; j < 16; ++j) {
+            for (int j = 0; j < W; ++j) {
               if (mj[j]) {
                 const int pj = __shfl_sync(MV_FULL, pos, j);
                 if ((pm >> j) & 1)
@@ -646,11 +654,12 @@ static bool tc_scan_layout(int type, int dpad, int qc, int ns, TcScanParams& p) 
 
 bool tc_scan_plan(int type, int dpad, int k, TcScanParams& p) {
   const bool wide = type == MV_IVF_FLAT || dpad % 128 == 0;  // 16-KB stages
-  const int qcmax = type == MV_IVF_FLAT ? 96 : 64;
+  int qcmax = type == MV_IVF_FLAT ? 96 : 64;
+  if (const char* e = getenv("MV_SQ8_QC"); e && type == MV_IVF_SQ8) qcmax = std::max(16, std::min(64, atoi(e)));
   const int nscap = wide ? 8 : 24;
   const int nsmin = wide ? 4 : 6;  // >= 64 KB (16-KB stages) / 24 KB (4-KB stages) of list tiles in flight
   p.k = k;
-  for (int qc = qcmax; qc >= 32; qc -= 32)
+  for (int qc = qcmax; qc >= 16; qc -= 16)
     for (int ns = nscap; ns >= nsmin; --ns)
       if (tc_scan_layout(type, dpad, qc, ns, p)) return true;
   return false;

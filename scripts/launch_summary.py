@@ -1,5 +1,5 @@
 """Per-search kernel time shares from an `ncu --metrics gpu__time_duration.sum --csv` launch list.
-Counts the libmv kernels (mv:: namespace) launched per search (= per k_plan launch) and their mean
+Counts the libmv kernels (mv:: namespace) launched per search (k_plan to k_plan) and their mean
 cold-cache, serialised durations.  Usage: launch_summary.py launches.csv"""
 import csv
 import sys
@@ -8,15 +8,14 @@ from collections import defaultdict
 rows = [r for r in csv.reader(open(sys.argv[1])) if len(r) > 14 and r[12] == "gpu__time_duration.sum"]
 tot = defaultdict(float)
 cnt = defaultdict(int)
-nplan = 0
-for r in rows:
+# one search = the launches from one k_plan to the next (its scan and selects, then the next
+# search's query staging and coarse step); the add path and data preparation precede the first
+# k_plan, the tail after the last one is dropped
+plans = [i for i, r in enumerate(rows) if "k_plan" in r[4]]
+nplan = max(len(plans) - 1, 0)
+for r in rows[plans[0]:plans[-1]] if nplan else []:
     name = r[4]
     short = name.split("(")[0].replace("void ", "").replace("mv::", "")
-    if "k_plan" in short:
-        nplan += 1
-    if nplan == 0 and "k_coarse_gemm" not in short and "k_probe_select" not in short and "k_hilo" not in short \
-            and "k_row_prep" not in short:
-        continue  # data preparation and the add path precede the first search
     if not any(t in name for t in ("mv::", "k_scan", "k_final", "k_coarse", "k_probe", "k_plan", "k_hilo",
                                     "k_query_prep", "k_qplanes", "k_final_big", "k_merge")):
         continue
@@ -27,6 +26,6 @@ for r in rows:
     cnt[short] += 1
 n = max(nplan, 1)
 total = sum(tot.values()) / n
-print(f"searches (k_plan launches): {nplan}; libmv device time per search {total:.1f} us")
+print(f"searches (k_plan to k_plan): {nplan}; libmv device time per search {total:.1f} us")
 for k, v in sorted(tot.items(), key=lambda kv: -kv[1]):
     print(f"  {k:<40} {v / n:9.1f} us  {100 * v / n / total:5.1f}%  launches/search {cnt[k] / n:.2f}")

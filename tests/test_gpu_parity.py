@@ -84,6 +84,23 @@ def test_flat_l2_sift_conditional(n, nlist, nprobe, nq, k):
     assert frac == 1.0  # integer data: no ties can be broken differently except exact ties by id
 
 
+@pytest.mark.parametrize("frac_q", [False, True])
+def test_flat_qm_scan_conditional(frac_q, monkeypatch):
+    """The experimental queries-as-M FLAT scan (MV_SCAN_IMPL=qm) meets the same parity
+    bar: one-plane (tf32-exact) and two-plane (fractional) queries, lists longer than one tile."""
+    monkeypatch.setenv("MV_SCAN_IMPL", "qm")
+    X, Q = _sift(20_000, 150)
+    if frac_q:
+        Q = Q * 0.7311 + 0.377
+    ids = G.permuted_ids(20_000, seed=9)
+    C = kmeans(X, 64, iters=5)
+    ix = _build(X, ids, C, "l2", "flat")
+    atol = 2e-6 * float((Q * Q).sum(1).max() + (X * X).sum(1).max()) if frac_q else 0.0
+    frac, _, _ = _run_conditional(ix, X, ids, C, Q, 10, 7, O.L2, O.FLAT, atol=atol)
+    assert ix.describe()["last_scan"] == "tcgen05.tf32.qm"
+    assert frac > 0.999
+
+
 @pytest.mark.parametrize("metric", ["l2", "ip"])
 def test_flat_tc_fractional_queries(metric):
     """Integer (tf32-exact) base data with fractional queries: the tensor-core scan must take the
