@@ -19,6 +19,8 @@
 // (Round 1 fused the selection into the GEMM epilogue; with 10 warps per SM that epilogue was
 // latency-bound on the per-tile folds.  Writing S costs 2 x nq x nlist x 4 B of HBM traffic --
 // 0.33 GB for configs[1] -- and buys a selection kernel at full occupancy.)
+#include <cstdlib>
+
 #include "mv_internal.cuh"
 #include "sm100.cuh"
 
@@ -323,6 +325,8 @@ bool coarse_tc_plan(int dpad, int nprobe, int64_t nq, int nlist, int nsm, Coarse
     }
   }
   if (best_cost < 0) return false;
+  if (const char* e = getenv("MV_COARSE_NQB")) p.nqb = std::max(16, std::min(128, atoi(e) / 16 * 16));
+  if (const char* e = getenv("MV_COARSE_CS")) p.csplit = std::max(1, std::min(ntiles, atoi(e)));
   const int fixed = p.nchunks * 2 * p.nqb * 128;
   p.nstage = std::min(6, (budget - fixed) / stage);
   p.smem_total = fixed + p.nstage * stage + 256 + 1024;

@@ -656,6 +656,7 @@ bool tc_scan_plan(int type, int dpad, int k, TcScanParams& p) {
   const bool wide = type == MV_IVF_FLAT || dpad % 128 == 0;  // 16-KB stages
   int qcmax = type == MV_IVF_FLAT ? 96 : 64;
   if (const char* e = getenv("MV_SQ8_QC"); e && type == MV_IVF_SQ8) qcmax = std::max(16, std::min(64, atoi(e)));
+  if (const char* e = getenv("MV_FLAT_QC"); e && type == MV_IVF_FLAT) qcmax = std::max(32, std::min(96, atoi(e)));
   const int nscap = wide ? 8 : 24;
   const int nsmin = wide ? 4 : 6;  // >= 64 KB (16-KB stages) / 24 KB (4-KB stages) of list tiles in flight
   p.k = k;
