@@ -7,9 +7,19 @@ per-list load stays balanced); centroids and SQ8 parameters are replicated.  A s
 hot path on every rank (mv_search), exchanges the per-shard top-k with ONE all-gather over NCCL
 (NVLink/NVSwitch), and merges on device with mv_merge_topk -- every rank ends with the same result.
 
-The exchange is the only collective; there is no per-step synchronisation besides it.  Merge order is
-(distance, id, shard, position) -- identical to the single-index order whenever ids are unique, so
-results are G-invariant (tested).
+The exchange is the only collective step; there is no per-step synchronisation besides it.  Merge
+order is (distance, id, shard, position) -- identical to the single-index order whenever ids are
+unique, so results are G-invariant (tested).
+
+Two exchanges:
+  * "allgather" (small k): every rank receives all G local top-k lists, (G-1) x nq x k x 12 B, and
+    merges all nq queries;
+  * "alltoall" (large k, e.g. k = 2048, where the all-gather would move (G-1) x 246 MB per rank at
+    nq = 10k): rank r owns the query slice [r*m, (r+1)*m), m = ceil(nq / G); one all_to_all sends
+    every slice to its owner ((G-1)/G of the local result), the owner merges its m queries from G
+    sources, and one all-gather of the merged slices gives every rank the full result -- 2 (G-1)/G
+    x nq x k x 12 B per rank instead of (G-1) x nq x k x 12 B, and 1/G of the merge work.
+  The default picks "alltoall" when k >= 256.
 
 The local index and the merge are injectable so that the distributed logic can be tested with the
 gloo backend on CPU (tests/test_sharded_gloo.py); the product path uses the CUDA library.
@@ -28,10 +38,14 @@ def shard_of(ids: torch.Tensor, world: int) -> torch.Tensor:
 
 
 class ShardedIndex:
-    def __init__(self, local, group=None, merge: Callable | None = None):
+    def __init__(self, local, group=None, merge: Callable | None = None, exchange: str = "auto"):
         """local: an object with .search(q, k, nprobe, bitset=None, nbits=None) -> (D[nq,k], I[nq,k])
         and .add(x, ids); group: a torch.distributed process group (None = default);
-        merge(D[G,nq,k], I[G,nq,k], metric) -> (D, I) (default: mv_merge_topk on device)."""
+        merge(D[G,nq,k], I[G,nq,k], metric) -> (D, I) (default: mv_merge_topk on device);
+        exchange: "allgather", "alltoall" or "auto" (alltoall for k >= 256)."""
+        if exchange not in ("auto", "allgather", "alltoall"):
+            raise ValueError(f"unknown exchange {exchange!r}")
+        self.exchange = exchange
         self.local = local
         self.group = group
         self.world = dist.get_world_size(group) if dist.is_initialized() else 1
@@ -75,8 +89,31 @@ class ShardedIndex:
         D, I = self.local.search(q, k, nprobe, bitset=bitset, nbits=nbits)
         if self.world == 1:
             return D, I
+        mode = self.exchange if self.exchange != "auto" else ("alltoall" if k >= 256 else "allgather")
+        if mode == "alltoall":
+            return self._exchange_alltoall(D, I)
         gd, gi = self._all_gather(D), self._all_gather(I)
         return self.merge(gd, gi, self.metric)
+
+    def _pad_value(self):
+        # the padding convention of the library (R3): id -1, +inf (L2) / -inf (IP)
+        return float("-inf") if self.metric in (1, "ip") else float("inf")
+
+    def _exchange_alltoall(self, D: torch.Tensor, I: torch.Tensor):
+        """Query-slice exchange: all_to_all of the local top-k by owner slice, merge of the own
+        slice's G lists, all-gather of the merged slices.  Rows past nq are padding."""
+        G, nq, k = self.world, D.shape[0], D.shape[1]
+        m = (nq + G - 1) // G
+        if m * G != nq:
+            D = torch.cat([D, torch.full((m * G - nq, k), self._pad_value(), dtype=D.dtype, device=D.device)])
+            I = torch.cat([I, torch.full((m * G - nq, k), -1, dtype=I.dtype, device=I.device)])
+        # send block g = rows [g*m, (g+1)*m) to rank g; receive block s = rank s's rows of my slice
+        rd, ri = torch.empty_like(D), torch.empty_like(I)
+        dist.all_to_all_single(rd, D.contiguous(), group=self.group)
+        dist.all_to_all_single(ri, I.contiguous(), group=self.group)
+        md, mi = self.merge(rd.view(G, m, k), ri.view(G, m, k), self.metric)   # my m queries
+        gd, gi = self._all_gather(md.contiguous()), self._all_gather(mi.contiguous())
+        return gd.reshape(G * m, k)[:nq], gi.reshape(G * m, k)[:nq]
 
     def _all_gather(self, t: torch.Tensor) -> torch.Tensor:
         out = torch.empty((self.world, *t.shape), dtype=t.dtype, device=t.device)

@@ -50,19 +50,19 @@ def _free_port():
     return p
 
 
-def _worker(rank, world, port, metric, out):
+def _worker(rank, world, port, metric, out, exchange="auto", nq=25, k=37):
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     dist.init_process_group("gloo", rank=rank, world_size=world)
     try:
         r = np.random.default_rng(7)
         X = r.integers(0, 6, (900, 4)).astype(np.float32)   # small integers: many exact ties
         ids = r.permutation(5000)[:900].astype(np.int64)
-        Q = r.integers(0, 6, (25, 4)).astype(np.float32)
-        sh = ShardedIndex(OracleShard(metric), merge=oracle_merge)
+        Q = r.integers(0, 6, (nq, 4)).astype(np.float32)
+        sh = ShardedIndex(OracleShard(metric), merge=oracle_merge, exchange=exchange)
         sh.set_centroids(torch.zeros(1, 4))
         sh.add(torch.tensor(X), torch.tensor(ids))           # each rank keeps only its own rows
         assert (shard_of(torch.tensor(sh.local.ids), world) == rank).all()
-        D, I = sh.search(torch.tensor(Q), 37, 1)
+        D, I = sh.search(torch.tensor(Q), k, 1)
         if rank == 0:
             out.put((D.numpy(), I.numpy(), X, ids, Q))
     finally:
@@ -82,6 +82,26 @@ def test_two_rank_gloo_sharded_equals_single_index(metric):
         p.join(timeout=60)
         assert p.exitcode == 0
     De, Ie = O.exact_knn(X, ids, Q, 37, metric)
+    assert np.array_equal(I, Ie)
+    assert np.array_equal(D, De.astype(np.float32))
+
+
+@pytest.mark.parametrize("world,nq,k,metric", [(2, 25, 37, O.L2), (3, 25, 300, O.L2), (2, 7, 300, O.IP)])
+def test_gloo_alltoall_exchange_equals_single_index(world, nq, k, metric):
+    """The large-k exchange (query-slice all_to_all, merge of the own slice, all-gather of the merged
+    slices) equals one index, with nq not a multiple of the world size and k beyond
+    the candidates of some shards (padding entries)."""
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, world, port, metric, q, "alltoall", nq, k)) for r in range(world)]
+    for p in procs:
+        p.start()
+    D, I, X, ids, Q = q.get(timeout=240)
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    De, Ie = O.exact_knn(X, ids, Q, k, metric)
     assert np.array_equal(I, Ie)
     assert np.array_equal(D, De.astype(np.float32))
 
