@@ -118,6 +118,16 @@ MV_API mv_status mv_search(mv_index* index, const float* queries, int64_t nq, in
 MV_API mv_status mv_search_probes(mv_index* index, const float* queries, int64_t nq, int32_t nprobe, int32_t* probes,
                            void* stream);
 
+/* Steps (2)-(3) with caller-supplied probes (§3.1): probes nq x nprobe' int32
+ * (nprobe' = min(nprobe, nlist)), each row the query's buckets best-first (as mv_search_probes
+ * returns them; ids in [0, nlist), no duplicates -- not checked on the device).  Used by the
+ * multi-GPU query-split coarse step: each rank computes the probes of a slice of the batch and
+ * the slices are all-gathered.  Results equal mv_search's when the probes equal
+ * mv_search_probes'.  Other arguments, errors and asynchrony as mv_search; host probes are staged. */
+MV_API mv_status mv_search_with_probes(mv_index* index, const float* queries, int64_t nq, int32_t k, int32_t nprobe,
+                                       const int32_t* probes, const uint8_t* bitset, int64_t nbits, float* distances,
+                                       int64_t* ids, void* stream);
+
 /* Merge nsrc per-shard top-k results (segments, §3.3; heap merge,
  * PAPER.md:590-596): dists nsrc x nq x k fp32, ids nsrc x nq x k int64, each row best-first
  * with -1 padding -> out_d / out_i nq x k, ordered by (distance, id, source, position).  Device

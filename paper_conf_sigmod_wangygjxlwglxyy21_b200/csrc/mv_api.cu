@@ -520,8 +520,25 @@ mv_status mv_search_probes(mv_index* ix, const float* queries, int64_t nq, int32
   return MV_OK;
 }
 
+static mv_status search_impl(mv_index* ix, const float* queries, int64_t nq, int32_t k, int32_t nprobe,
+                             const int32_t* probes_in, const uint8_t* bitset, int64_t nbits, float* distances,
+                             int64_t* out_ids, void* stream);
+
 mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, int32_t nprobe, const uint8_t* bitset,
                     int64_t nbits, float* distances, int64_t* out_ids, void* stream) {
+  return search_impl(ix, queries, nq, k, nprobe, nullptr, bitset, nbits, distances, out_ids, stream);
+}
+
+mv_status mv_search_with_probes(mv_index* ix, const float* queries, int64_t nq, int32_t k, int32_t nprobe,
+                                const int32_t* probes, const uint8_t* bitset, int64_t nbits, float* distances,
+                                int64_t* out_ids, void* stream) {
+  if (probes == nullptr && nq > 0) return fail(MV_EINVAL, "probes is NULL");
+  return search_impl(ix, queries, nq, k, nprobe, probes, bitset, nbits, distances, out_ids, stream);
+}
+
+static mv_status search_impl(mv_index* ix, const float* queries, int64_t nq, int32_t k, int32_t nprobe,
+                             const int32_t* probes_in, const uint8_t* bitset, int64_t nbits, float* distances,
+                             int64_t* out_ids, void* stream) {
   mv_status v = validate_search(ix, queries, nq, k, nprobe, distances, out_ids);
   if (v != MV_OK) return v;
   if (nbits < 0) return fail(MV_EINVAL, "nbits must be >= 0");
@@ -553,7 +570,14 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
     int32_t* P;
     CK(s.alloc(&qpad, (size_t)nq * dpad));
     CK(s.alloc(&qnorm, (size_t)nq));
-    CK(s.alloc(&P, (size_t)nq * npb));
+    if (probes_in) {  // caller-supplied probes (staged when on the host): a2/a3 are skipped
+      bool sp;
+      const int32_t* pp;
+      CK(stage_in(s, probes_in, (size_t)nq * npb, &pp, &sp));
+      P = const_cast<int32_t*>(pp);
+    } else {
+      CK(s.alloc(&P, (size_t)nq * npb));
+    }
     CK(launch_query_prep(q, nq, ix->d, dpad, qpad, qnorm, st));
     float* qhl;  // plane-major tf32 hi/lo query planes: coarse B operand and the FLAT scan's query planes
     CK(s.alloc(&qhl, (size_t)2 * nq * dpad));
@@ -561,7 +585,7 @@ mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, i
     CK(s.alloc(&qlo_any, 1));
     CK(cudaMemsetAsync(qlo_any, 0, sizeof(int), st));
     CK(launch_hilo(q, nq, ix->d, dpad, qhl, qlo_any, st));
-    CK(run_coarse(ix, qpad, qhl, qlo_any, nq, npb, P, s, st));
+    if (!probes_in) CK(run_coarse(ix, qpad, qhl, qlo_any, nq, npb, P, s, st));
     prof_mark(ix, st);
     // a4 (work-item size depends on the scan implementation's shared-memory plan)
     TcScanParams tp;

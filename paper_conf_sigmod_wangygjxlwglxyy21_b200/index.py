@@ -109,8 +109,11 @@ class Index:
         L.check(self._lib.mv_index_add(self._h, _ptr(x), _ptr(ids), n, _stream(self.device, stream)))
 
     # -- search ------------------------------------------------------------------------------
-    def search(self, q, k: int, nprobe: int, bitset=None, nbits: int | None = None, out=None, stream=None):
-        """Returns (D[nq,k] float32, I[nq,k] int64) on the index device (or into `out`)."""
+    def search(self, q, k: int, nprobe: int, bitset=None, nbits: int | None = None, out=None, stream=None,
+               probes=None):
+        """Returns (D[nq,k] float32, I[nq,k] int64) on the index device (or into `out`).
+        probes: optional int32 [nq, min(nprobe, nlist)] best-first buckets per query (as
+        search_probes returns them); the coarse step is then skipped (mv_search_with_probes)."""
         q = _as_f32(q)
         nq = int(q.shape[0])
         if out is None:
@@ -122,6 +125,13 @@ class Index:
         nb = 0
         if bitset is not None:
             nb = int(nbits) if nbits is not None else int(bitset.shape[0]) * 8
+        if probes is not None:
+            npb = min(int(nprobe), self.nlist)
+            if probes.dtype != torch.int32 or tuple(probes.shape) != (nq, npb) or not probes.is_contiguous():
+                raise ValueError(f"probes must be a contiguous int32 tensor of shape ({nq}, {npb})")
+            L.check(self._lib.mv_search_with_probes(self._h, _ptr(q), nq, int(k), int(nprobe), _ptr(probes),
+                                                    _ptr(bitset), nb, _ptr(D), _ptr(I), _stream(self.device, stream)))
+            return D, I
         L.check(self._lib.mv_search(self._h, _ptr(q), nq, int(k), int(nprobe), _ptr(bitset), nb, _ptr(D), _ptr(I),
                                     _stream(self.device, stream)))
         return D, I

@@ -21,6 +21,12 @@ Two exchanges:
     x nq x k x 12 B per rank instead of (G-1) x nq x k x 12 B, and 1/G of the merge work.
   The default picks "alltoall" when k >= 256.
 
+Coarse step (a2/a3): "replicated" (every rank computes all nq probe lists; cheap for small nlist)
+or "split" (rank r computes the probes of its query slice and one all-gather of the int32
+[nq, nprobe] probe matrix gives every rank all of them -- 2.56 MB at nq = 10k, nprobe = 64 --
+then the local scan takes them through mv_search_with_probes).  The default splits when
+nq * nlist >= 2^28 (configs[4]: 10k x 65,536, a 2.6 GB score matrix per rank if replicated).
+
 The local index and the merge are injectable so that the distributed logic can be tested with the
 gloo backend on CPU (tests/test_sharded_gloo.py); the product path uses the CUDA library.
 """
@@ -38,14 +44,19 @@ def shard_of(ids: torch.Tensor, world: int) -> torch.Tensor:
 
 
 class ShardedIndex:
-    def __init__(self, local, group=None, merge: Callable | None = None, exchange: str = "auto"):
+    def __init__(self, local, group=None, merge: Callable | None = None, exchange: str = "auto",
+                 coarse: str = "auto"):
         """local: an object with .search(q, k, nprobe, bitset=None, nbits=None) -> (D[nq,k], I[nq,k])
         and .add(x, ids); group: a torch.distributed process group (None = default);
         merge(D[G,nq,k], I[G,nq,k], metric) -> (D, I) (default: mv_merge_topk on device);
-        exchange: "allgather", "alltoall" or "auto" (alltoall for k >= 256)."""
+        exchange: "allgather", "alltoall" or "auto" (alltoall for k >= 256);
+        coarse: "replicated", "split" or "auto" (split when nq * nlist >= 2^28)."""
         if exchange not in ("auto", "allgather", "alltoall"):
             raise ValueError(f"unknown exchange {exchange!r}")
+        if coarse not in ("auto", "replicated", "split"):
+            raise ValueError(f"unknown coarse mode {coarse!r}")
         self.exchange = exchange
+        self.coarse = coarse
         self.local = local
         self.group = group
         self.world = dist.get_world_size(group) if dist.is_initialized() else 1
@@ -86,7 +97,14 @@ class ShardedIndex:
 
     # -- search: local top-k, one all-gather, on-device merge -----------------------------------
     def search(self, q: torch.Tensor, k: int, nprobe: int, bitset=None, nbits: int | None = None):
-        D, I = self.local.search(q, k, nprobe, bitset=bitset, nbits=nbits)
+        nlist = int(getattr(self.local, "nlist", 1))
+        split = self.world > 1 and (self.coarse == "split" or
+                                    (self.coarse == "auto" and q.shape[0] * nlist >= (1 << 28)))
+        if split:
+            P = self._split_probes(q, nprobe, nlist)
+            D, I = self.local.search(q, k, nprobe, bitset=bitset, nbits=nbits, probes=P)
+        else:
+            D, I = self.local.search(q, k, nprobe, bitset=bitset, nbits=nbits)
         if self.world == 1:
             return D, I
         mode = self.exchange if self.exchange != "auto" else ("alltoall" if k >= 256 else "allgather")
@@ -94,6 +112,17 @@ class ShardedIndex:
             return self._exchange_alltoall(D, I)
         gd, gi = self._all_gather(D), self._all_gather(I)
         return self.merge(gd, gi, self.metric)
+
+    def _split_probes(self, q: torch.Tensor, nprobe: int, nlist: int) -> torch.Tensor:
+        """Query-split coarse step: probes of the rank's slice [r*m, (r+1)*m), one all-gather."""
+        G, nq = self.world, int(q.shape[0])
+        m = (nq + G - 1) // G
+        lo, hi = min(nq, self.rank * m), min(nq, (self.rank + 1) * m)
+        npb = min(int(nprobe), nlist)
+        mine = torch.zeros((m, npb), dtype=torch.int32, device=q.device)  # padding rows: bucket 0
+        if hi > lo:
+            mine[: hi - lo] = self.local.search_probes(q[lo:hi].contiguous(), nprobe)
+        return self._all_gather(mine).reshape(G * m, npb)[:nq].contiguous()
 
     def _pad_value(self):
         # the padding convention of the library (DESIGN.md R3): id -1, +inf (L2) / -inf (IP)

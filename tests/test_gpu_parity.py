@@ -356,3 +356,21 @@ def test_tensor_core_path_matches_simt_path(kind, metric, k, monkeypatch):
         diff = I1 != I2
         assert torch.allclose(D1[diff], D2[diff], rtol=2e-5, atol=1e-3)
         assert (~diff).float().mean().item() > 0.99
+
+
+@pytest.mark.parametrize("kind,metric", [("flat", "l2"), ("sq8", "ip")])
+def test_search_with_probes_equals_search(kind, metric):
+    """mv_search_with_probes (the multi-GPU query-split coarse step's entry point) with the probes
+    mv_search_probes returns gives bit-identical results to mv_search; host probes are staged."""
+    X, Q = _sift(12_000, 90)
+    ids = G.permuted_ids(12_000, seed=4)
+    C = kmeans(X, 96, iters=4)
+    ix = _build(X, ids, C, metric, kind)
+    Qd = Q.cuda()
+    D0, I0 = ix.search(Qd, 20, 9)
+    P = ix.search_probes(Qd, 9)
+    D1, I1 = ix.search(Qd, 20, 9, probes=P)
+    D2, I2 = ix.search(Qd, 20, 9, probes=P.cpu())
+    torch.cuda.synchronize()
+    assert torch.equal(I0, I1) and torch.equal(D0, D1)
+    assert torch.equal(I0, I2) and torch.equal(D0, D2)

@@ -36,6 +36,76 @@ class OracleShard:
         return torch.tensor(D, dtype=torch.float32), torch.tensor(I)
 
 
+class OracleIvfShard:
+    """Test double for an IVF shard: the oracle's two-step IVF search over this rank's rows, with
+    probes computed here (search_probes) or supplied (the query-split coarse step)."""
+
+    def __init__(self, metric, C):
+        self.metric = metric
+        self.ix = O.IvfIndex(C.shape[1], metric, O.FLAT, C)
+        self.nlist = C.shape[0]
+        self.calls = []
+
+    def set_centroids(self, c):
+        pass
+
+    def add(self, x, ids):
+        self.ix.add(x.numpy(), ids.numpy())
+
+    def search_probes(self, q, nprobe):
+        self.calls.append(("probes", int(q.shape[0])))
+        return torch.tensor(O.probe(q.numpy(), self.ix.C, nprobe, self.metric).astype(np.int32))
+
+    def search(self, q, k, nprobe, bitset=None, nbits=None, probes=None):
+        self.calls.append(("search", probes is not None))
+        D, I, _ = self.ix.search(q.numpy(), k, nprobe, probes=None if probes is None else probes.numpy())
+        return torch.tensor(D, dtype=torch.float32), torch.tensor(I)
+
+
+def _ivf_worker(rank, world, port, out, nq):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        r = np.random.default_rng(11)
+        X = r.integers(0, 40, (1200, 6)).astype(np.float32)
+        ids = r.permutation(9000)[:1200].astype(np.int64)
+        Q = r.integers(0, 40, (nq, 6)).astype(np.float32)
+        C = X[r.permutation(1200)[:24]] + 0.5
+        sh = ShardedIndex(OracleIvfShard(O.L2, C), merge=oracle_merge, coarse="split")
+        sh.add(torch.tensor(X), torch.tensor(ids))
+        D, I = sh.search(torch.tensor(Q), 9, 5)
+        m = (nq + world - 1) // world
+        assert ("probes", max(0, min(nq, (rank + 1) * m) - min(nq, rank * m))) in sh.local.calls or \
+            min(nq, (rank + 1) * m) <= min(nq, rank * m)
+        assert ("search", True) in sh.local.calls
+        if rank == 0:
+            out.put((D.numpy(), I.numpy(), X, ids, Q, C))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world,nq", [(2, 31), (3, 20)])
+def test_gloo_split_coarse_equals_single_ivf(world, nq):
+    """Query-split coarse step: each rank computes the probes of its query slice, one
+    all-gather of the probe matrix, local scans with the supplied probes, exchange and merge --
+    equal to one IVF index over all rows with the same centroids (oracle, nprobe 5 of 24)."""
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_ivf_worker, args=(r, world, port, q, nq)) for r in range(world)]
+    for p in procs:
+        p.start()
+    D, I, X, ids, Q, C = q.get(timeout=240)
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    ref = O.IvfIndex(6, O.L2, O.FLAT, C)
+    ref.add(X, ids)
+    De, Ie, _ = ref.search(Q, 9, 5)
+    assert np.array_equal(I, Ie)
+    assert np.array_equal(D, De.astype(np.float32))
+
+
 def oracle_merge(gd, gi, metric):
     parts = [(gd[s].double().numpy(), gi[s].numpy()) for s in range(gd.shape[0])]
     D, I = O.merge_topk(parts, gd.shape[2], metric)
