@@ -14,8 +14,8 @@
 //              D[128 vectors x N] (+)= X_tile[128 x K] . Qplanes[N x K]^T, N = P x roundup16(nq)
 //   warps 2-3  query gatherer: the bucket's query planes -> swizzled K-major smem, and the
 //              per-query metadata (threshold, output region) -- both double-buffered
-//   warps 4-11 epilogue, two warps per TMEM lane quarter: every thread owns one vector row and
-//              half of the query columns; tcgen05.ld -> distance -> bitset -> threshold test ->
+//   warps 4-15 (FLAT) / 4-11 (SQ8) epilogue, three / two warps per TMEM lane quarter: every thread owns one vector row and
+//              a share of the query columns; tcgen05.ld -> distance -> bitset -> threshold test ->
 //              survivors are appended to the (query, list) pair's output region (a6).
 //
 // a6 is a filter, not a selection.  The search runs the scan twice:
@@ -84,8 +84,10 @@ constexpr int kNTS = 4;          // per-tile side-data ring slots
 // superset of the tile's 128 rows (the arrays are padded at allocation so the copy stays in bounds)
 constexpr int kSideBytes = 3072;
 constexpr int kSideRank = 1152, kSideIds = 1792;
-constexpr int kEpiWarps = 8;      // two epilogue warps per TMEM lane quarter
-constexpr int kThreads = 128 + 32 * kEpiWarps;
+// epilogue warps: three per TMEM lane quarter for FLAT (112 registers: 512 threads fit the register
+// file), two for SQ8 (the 4-plane accumulators need ~150 registers)
+template <int TYPE>
+constexpr int epi_warps() { return TYPE == MV_IVF_FLAT ? 12 : 8; }
 
 // per-query metadata of one work item (QCP = roundup16(qchunk) entries per array)
 struct Meta {
@@ -124,7 +126,9 @@ __device__ __forceinline__ Meta meta_at(uint8_t* m, int QCP) {
 constexpr int kMetaPerQuery = 64;  // bytes (+ a 32-B work-item header)
 
 template <int TYPE, int ATOM, bool SMALLD>
-__global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__ XMaps xm, const TcScanParams p) {
+__global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
+    k_scan_tc(const __grid_constant__ XMaps xm, const TcScanParams p) {
+  constexpr int kEpiWarps = epi_warps<TYPE>();
   extern __shared__ uint8_t smem_raw[];
   uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~(uintptr_t)1023);
   constexpr int ESZ = TYPE == MV_IVF_FLAT ? 4 : 1;
@@ -190,6 +194,12 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
   tc_fence_after();
   const uint32_t tmem = *tslot;
   const int nwork = *p.nwitems;
+  auto gtimer = []() {
+    uint64_t t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    return t;
+  };
+  if (p.prof && threadIdx.x == 0 && blockIdx.x < 148) p.prof[8 * 1024 + blockIdx.x * 3] = gtimer();
   const int w0 = (p.wbeg ? *p.wbeg : 0) + blockIdx.x;
 
   if (warp == 0) {
@@ -278,6 +288,10 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
           MV_TRACE(3, titer);
         }
         mma_commit(&empty_q[b]);
+      }
+      if (p.prof && blockIdx.x < 148) {
+        p.prof[8 * 1024 + blockIdx.x * 3 + 1] = gtimer();
+        p.prof[8 * 1024 + blockIdx.x * 3 + 2] = titer;
       }
     }
   } else if (warp < 4) {
@@ -394,7 +408,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
     // ------------------------------------------------------------------ epilogue (8 warps)
     const int ew = warp - 4;            // 0..7
     const int quarter = warp & 3;       // TMEM lane quarter this warp may access
-    const int half = ew >> 2;           // which 16-column chunks of the accumulator it reads
+    const int half = ew >> 2;           // which column chunks of the accumulator it reads
+    constexpr int NPART = kEpiWarps / 4;  // epilogue warps per lane quarter
     const int row = quarter * 32 + lane;
     const int et = threadIdx.x - 128;   // 0..255
     const uint32_t ltmask = (1u << lane) - 1;
@@ -423,7 +438,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_scan_tc(const __grid_constant__
         if (et == 0) MV_TRACE(6, titer);
         tc_fence_after();
         const uint32_t tbase = tmem + a * p.ncol + ((uint32_t)(quarter * 32) << 16);
-        for (int qc = half * W; qc < ((p.dbg & 2) ? 0 : NQ); qc += 2 * W) {
+        for (int qc = half * W; qc < ((p.dbg & 2) ? 0 : NQ); qc += NPART * W) {
           uint32_t r[PMAX][W];
 #pragma unroll
           for (int pl = 0; pl < PMAX; ++pl) {
@@ -677,7 +692,8 @@ cudaError_t launch_scan_tc(const XMaps& xm, const TcScanParams& p, cudaStream_t 
   int dev = 0, nsm = kNumSMs;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
-  kern<<<nsm, kThreads, p.smem_total, st>>>(xm, p);
+  kern<<<nsm, 128 + 32 * (p.type == MV_IVF_FLAT ? epi_warps<MV_IVF_FLAT>() : epi_warps<MV_IVF_SQ8>()), p.smem_total,
+         st>>>(xm, p);
   return cudaGetLastError();
 }
 
