@@ -14,7 +14,7 @@
 //              D[128 vectors x N] (+)= X_tile[128 x K] . Qplanes[N x K]^T, N = P x roundup16(nq)
 //   warps 2-3  query gatherer: the bucket's query planes -> swizzled K-major smem, and the
 //              per-query metadata (threshold, output region) -- both double-buffered
-//   warps 4-15 (FLAT) / 4-11 (SQ8) epilogue, three / two warps per TMEM lane quarter: every thread owns one vector row and
+//   warps 4-15 epilogue, three warps per TMEM lane quarter: every thread owns one vector row and
 //              a share of the query columns; tcgen05.ld -> distance -> bitset -> threshold test ->
 //              survivors are appended to the (query, list) pair's output region (a6).
 //
@@ -84,10 +84,11 @@ constexpr int kNTS = 4;          // per-tile side-data ring slots
 // superset of the tile's 128 rows (the arrays are padded at allocation so the copy stays in bounds)
 constexpr int kSideBytes = 3072;
 constexpr int kSideRank = 1152, kSideIds = 1792;
-// epilogue warps: three per TMEM lane quarter for FLAT (112 registers: 512 threads fit the register
-// file), two for SQ8 (the 4-plane accumulators need ~150 registers)
+// epilogue warps: three per TMEM lane quarter (<= 128 registers per thread: 512 threads fit the
+// register file).  Measured: 8 -> 12 took configs[1]'s phase B from 289 to 256 us and configs[4]'s
+// per-GPU scan from 9.4 to 8.9 ms; 16 was slower for FLAT (6 chunks of 16 columns over 4 warps)
 template <int TYPE>
-constexpr int epi_warps() { return TYPE == MV_IVF_FLAT ? 12 : 8; }
+constexpr int epi_warps() { return 12; }
 
 // per-query metadata of one work item (QCP = roundup16(qchunk) entries per array)
 struct Meta {
