@@ -201,7 +201,11 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
     return t;
   };
   if (p.prof && threadIdx.x == 0 && blockIdx.x < 148) p.prof[8 * 1024 + blockIdx.x * 3] = gtimer();
-  const int w0 = (p.wbeg ? *p.wbeg : 0) + blockIdx.x;
+  // static schedule over the longest-first item order, snake-wise: round i gives CTA b the item
+  // i*G + b (even rounds) or i*G + G-1-b (odd rounds), which balances sorted costs far better than
+  // plain round-robin (every role walks the same sequence)
+  const int wb = p.wbeg ? *p.wbeg : 0, G = gridDim.x, bx = blockIdx.x;
+  auto item = [&](int i) { return wb + i * G + ((i & 1) ? G - 1 - bx : bx); };
 
   if (warp == 0) {
     // ------------------------------------------------------------------ TMA producer
@@ -211,13 +215,12 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
       const uint64_t pol = l2_evict_first_policy();
       // two-deep prefetch: the next item's list range and the one after's (list, bucket) pair are
       // in flight while this item's tiles are issued, so no dependent load sits between items
-      const int G = gridDim.x;
-      int2 itn = w0 + G < nwork ? p.witems[w0 + G] : make_int2(0, 0);
-      WorkInfo wn = w0 < nwork ? work_info(p, w0, QC) : WorkInfo{};
-      for (int w = w0; w < nwork; w += G) {
+      int2 itn = item(1) < nwork ? p.witems[item(1)] : make_int2(0, 0);
+      WorkInfo wn = item(0) < nwork ? work_info(p, item(0), QC) : WorkInfo{};
+      for (int i = 0; item(i) < nwork; ++i) {
         const WorkInfo wi = wn;
-        if (w + G < nwork) wn = work_info_of(p, itn, QC);
-        if (w + 2 * G < nwork) itn = p.witems[w + 2 * G];
+        if (item(i + 1) < nwork) wn = work_info_of(p, itn, QC);
+        if (item(i + 2) < nwork) itn = p.witems[item(i + 2)];
         for (int t = 0; t < wi.ntiles; ++t, ++tcount) {
           const int row0 = (int)(wi.lstart + t * 128);
           const uint32_t ts = tcount % kNTS, tr = tcount / kNTS;
@@ -254,7 +257,7 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
     // ------------------------------------------------------------------ MMA issuer
     if (lane == 0) {
       uint32_t it = 0, titer = 0, wcount = 0;
-      for (int w = w0; w < nwork; w += gridDim.x, ++wcount) {
+      for (int i = 0; item(i) < nwork; ++i, ++wcount) {
         const uint32_t b = wcount & 1;
         mbar_wait(&full_q[b], (wcount >> 1) & 1);
         MV_TRACE(1, wcount);
@@ -299,7 +302,6 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
     // ------------------------------------------------------------------ query gatherer (64 thr)
     const int tq = threadIdx.x - 64;
     const int gw = tq >> 5;
-    const int G = gridDim.x;
     // the next item's list range and per-query metadata are loaded into registers before waiting
     // for its buffers, so only the plane copies sit on the critical path once a buffer frees
     struct Pref {
@@ -331,11 +333,11 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
       return f;
     };
     Pref cur;
-    if (w0 < nwork) cur = prefetch(w0);
+    if (item(0) < nwork) cur = prefetch(item(0));
     uint32_t wcount = 0;
-    for (int w = w0; w < nwork; w += G, ++wcount) {
+    for (int i = 0; item(i) < nwork; ++i, ++wcount) {
       Pref nxt;
-      if (w + G < nwork) nxt = prefetch(w + G);
+      if (item(i + 1) < nwork) nxt = prefetch(item(i + 1));
       const WorkInfo wi = cur.wi;
       const int NQ = (wi.nqc + 15) & ~15;
       const int N = P * NQ;
@@ -415,7 +417,7 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
     const int et = threadIdx.x - 128;   // 0..255
     const uint32_t ltmask = (1u << lane) - 1;
     uint32_t titer = 0, wcount = 0;
-    for (int w = w0; w < nwork; w += gridDim.x, ++wcount) {
+    for (int i = 0; item(i) < nwork; ++i, ++wcount) {
       const uint32_t b = wcount & 1;
       mbar_wait(&full_q[b], (wcount >> 1) & 1);
       const Meta mt = meta_at(metab + b * p.meta_bytes, QCP);
