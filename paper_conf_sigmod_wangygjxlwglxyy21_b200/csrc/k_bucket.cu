@@ -15,6 +15,7 @@
 //   5  work items (virtual list, first bucket position)
 //   6  longest-first order (block 0, counting sort by cost; seeding phase first)
 #include <cooperative_groups.h>
+#include <cstdlib>
 
 #include "mv_internal.cuh"
 
@@ -257,7 +258,8 @@ cudaError_t launch_plan(const PlanArgs& a, cudaStream_t st) {
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_plan, kPlanThreads, 0);
-    grid = nsm * std::max(1, std::min(per, 2));
+    const char* pb = getenv("MV_PLAN_BPS");  // blocks per SM (grid-wide barriers cost more with more blocks)
+    grid = nsm * std::max(1, std::min(per, pb ? atoi(pb) : 2));
   }
   PlanArgs args = a;
   void* kargs[] = {&args};

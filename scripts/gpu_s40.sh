@@ -1,0 +1,8 @@
+python -c "import __graft_entry__ as g; g.build()" || exit 1
+timeout 900 python -m pytest tests -m "gpu and not slow" -x -q --timeout 300 2>&1 | tail -2
+run() {
+  env $1 timeout 1500 python bench.py --config ${2:-c2} --steps 10 --warmup 3 --no-cpu-baseline > gpurun_out/bench_$2.json 2> gpurun_out/bench_$2.err
+  python -c "import json; d=json.load(open('gpurun_out/bench_$2.json')); print('$1 ${2:-c2}', round(d['value']), d['config'].get('recall@10'), {a: round(b,3) for a,b in d['stage_ms'].items()}, 'frac', round(d['roofline']['frac'],3), d['index']['last_scan'])" || tail -3 gpurun_out/bench_$2.err
+}
+run MV_X=0 c4
+run MV_X=0 c3
