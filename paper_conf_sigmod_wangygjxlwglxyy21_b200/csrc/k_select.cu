@@ -156,6 +156,7 @@ __global__ void __launch_bounds__(256) k_final_select(const int64_t* __restrict_
 // select over the u64 keys -- 8-bit digits, histogram per pass in shared memory, stopping as soon
 // as the keys at or below the current prefix are exactly k -- and a bitonic sort of the k winners.
 constexpr int kBigThreads = 512;
+constexpr int kHistWarps = 8;  // private radix histograms (warps w and w + 8 share one)
 
 __global__ void __launch_bounds__(kBigThreads) k_final_big(const int64_t* __restrict__ poff,
                                                            const int32_t* __restrict__ pcnt,
@@ -168,8 +169,8 @@ __global__ void __launch_bounds__(kBigThreads) k_final_big(const int64_t* __rest
   const int NK = next_pow2(max(k, 2));
   uint64_t* buf = reinterpret_cast<uint64_t*>(smem);   // cap
   uint64_t* win = buf + cap;                           // NK
-  uint32_t* hist = reinterpret_cast<uint32_t*>(win + NK);  // 256
-  int32_t* s_pre = reinterpret_cast<int32_t*>(hist + 256);  // npb + 1
+  uint32_t* whist = reinterpret_cast<uint32_t*>(win + NK);  // kHistWarps x 256 (>= 66 u64 for the min/max)
+  int32_t* s_pre = reinterpret_cast<int32_t*>(whist + kHistWarps * 256);  // npb + 1
   int32_t* s_int = s_pre + npb + 1;                    // misc
   const int64_t q = blockIdx.x;
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
@@ -210,43 +211,92 @@ __global__ void __launch_bounds__(kBigThreads) k_final_big(const int64_t* __rest
     for (int i = tid; i < NK; i += kBigThreads) win[i] = i < T ? buf[i] : MV_KEY_PAD;
     nsel = T;
   } else {
-    // radix select: find the largest prefix such that #keys with top <= prefix is exactly k
-    uint64_t pfx = 0;
-    int fixed = 0, below = 0;  // below = #keys whose top bits are < the current prefix
+    // radix select over the bits below the keys' common prefix: the first digit starts at the
+    // highest bit where the smallest and largest key differ (near-neighbour distance keys share
+    // their top ~10 bits, which a fixed MSB digit would pile into one contended bin).  8-bit
+    // digits, per-warp private histograms, a warp prefix scan for the digit; it stops as soon as
+    // the keys at or below the current prefix are exactly k (keys are unique).
+    uint64_t mn = MV_KEY_PAD, mx = 0;
+    for (int i = tid; i < T; i += kBigThreads) {
+      const uint64_t x = buf[i];
+      mn = umin64(mn, x);
+      mx = umax64(mx, x);
+    }
+    for (int o = 16; o > 0; o >>= 1) {
+      mn = umin64(mn, shfl_xor64(mn, o));
+      mx = umax64(mx, shfl_xor64(mx, o));
+    }
+    uint64_t* red = reinterpret_cast<uint64_t*>(whist);
+    if (lane == 0) {
+      red[wid] = mn;
+      red[32 + wid] = mx;
+    }
+    __syncthreads();
+    if (tid == 0) {
+      for (int w = 1; w < kBigThreads / 32; ++w) {
+        mn = umin64(mn, red[w]);
+        mx = umax64(mx, red[32 + w]);
+      }
+      red[64] = mn;
+      red[65] = mx;
+    }
+    __syncthreads();
+    mn = red[64];
+    mx = red[65];
+    __syncthreads();
+    int lo = 64 - __clzll((long long)(mn ^ mx));  // bits [lo, 64) are common to every key
+    uint64_t pfx = lo >= 64 ? 0 : (mn >> lo);
+    int below = 0;  // keys whose bits above lo are < pfx
     for (;;) {
-      for (int i = tid; i < 256; i += kBigThreads) hist[i] = 0;
+      const int w = min(8, lo), sh = lo - w;
+      const uint32_t dmask = (1u << w) - 1;
+      for (int i = tid; i < kHistWarps * 256; i += kBigThreads) whist[i] = 0;
       __syncthreads();
-      const int sh = 56 - fixed;
+      uint32_t* hw = whist + (wid % kHistWarps) * 256;
       for (int i = tid; i < T; i += kBigThreads) {
         const uint64_t x = buf[i];
-        if (fixed == 0 || (x >> (64 - fixed)) == pfx) atomicAdd(hist + ((x >> sh) & 0xff), 1u);
+        if (lo >= 64 || (x >> lo) == pfx) atomicAdd(hw + ((uint32_t)(x >> sh) & dmask), 1u);
       }
       __syncthreads();
-      if (tid == 0) {
-        int cum = below, d = 0;
-        for (; d < 256; ++d) {
-          if (cum + (int)hist[d] >= k) break;
-          cum += hist[d];
+      if (wid == 0) {  // bins 8 * lane .. 8 * lane + 7, summed over the private histograms
+        uint32_t c[8];
+        uint32_t tot = 0;
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+          uint32_t v = 0;
+          for (int h = 0; h < kHistWarps; ++h) v += whist[h * 256 + 8 * lane + j];
+          c[j] = v;
+          tot += v;
         }
-        s_int[0] = d;
-        s_int[1] = cum;
-        s_int[2] = cum + (int)hist[d] == k;
+        uint32_t incl = tot;
+        for (int o = 1; o < 32; o <<= 1) {
+          const uint32_t v = __shfl_up_sync(MV_FULL, incl, o);
+          if (lane >= o) incl += v;
+        }
+        uint32_t cum = below + incl - tot;  // keys before this lane's first bin
+        const bool mine = cum < (uint32_t)k && cum + tot >= (uint32_t)k;
+        if (mine) {
+          int d = 0;
+          while (cum + c[d] < (uint32_t)k) cum += c[d++];
+          s_int[0] = 8 * lane + d;
+          s_int[1] = (int)cum;
+          s_int[2] = cum + c[d] == (uint32_t)k;
+        }
       }
       __syncthreads();
-      pfx = (pfx << 8) | (uint64_t)s_int[0];
+      pfx = (pfx << w) | (uint64_t)s_int[0];
       below = s_int[1];
-      fixed += 8;
-      const bool done = s_int[2] || fixed == 64;
+      lo = sh;
+      const bool done = s_int[2] || lo == 0;
       __syncthreads();
       if (done) break;
     }
-    // winners: keys whose top `fixed` bits are <= pfx (exactly k: keys are unique)
+    // winners: keys whose bits above lo are <= pfx (exactly k: keys are unique)
     if (tid == 0) s_int[3] = 0;
     __syncthreads();
-    const int sh = 64 - fixed;
     for (int i = tid; i < T; i += kBigThreads) {
       const uint64_t x = buf[i];
-      const uint64_t top = sh >= 64 ? 0 : (x >> sh);
+      const uint64_t top = lo >= 64 ? 0 : (x >> lo);
       if (top <= pfx) win[atomicAdd(s_int + 3, 1)] = x;
     }
     __syncthreads();
@@ -309,8 +359,10 @@ static cudaError_t launch_big_select(const int64_t* poff, const int32_t* pcnt, c
                                      int64_t* out_i, const int32_t* nuse, uint64_t* tau, int64_t tmax,
                                      uint8_t* over, cudaStream_t st) {
   const int NK = next_pow2(max(k, 2));
-  const int fixed = NK * 8 + 256 * 4 + (npb + 1) * 4 + 64 + 64;
-  const int cap = (227 * 1024 - fixed) / 8;
+  const int fixed = NK * 8 + kHistWarps * 256 * 4 + (npb + 1) * 4 + 64 + 64;
+  // stage capacity: all of shared memory, or just the bound tmax when that is smaller (several
+  // CTAs per SM: the seeding select's candidates are bounded by the phase-A prefixes)
+  const int cap = (int)min64((227 * 1024 - fixed) / 8, max64(tmax, k));
   if (over && cap >= k) {
     const size_t smem = (size_t)cap * 8 + fixed;
     cudaError_t e = cudaFuncSetAttribute(k_final_big, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);

@@ -631,6 +631,7 @@ static mv_status search_impl(mv_index* ix, const float* queries, int64_t nq, int
     PlanArgs pa;
     pa.probes = P; pa.nq = nq; pa.npb = npb; pa.nlist = nlist; pa.k = k; pa.capk = capk;
     pa.split = split ? 1 : 0; pa.need = std::max<int64_t>(2 * (int64_t)k, k + 32);
+    if (const char* ne = getenv("MV_NEED")) pa.need = std::max<int64_t>(pa.need, atoll(ne));  // sweep override
     // phase A reads the first capA rows of each of a query's nearest lists (a 16-row multiple, at
     // least one tile; measured on configs[1]: 64 rows 14.7M qps, 128 rows 16.0M, 256 rows 15.8M,
     // whole lists 14.7M -- a looser tau_q costs phase-B emissions, more rows cost phase-A reads)
@@ -707,7 +708,9 @@ static mv_status search_impl(mv_index* ix, const float* queries, int64_t nq, int
       prof_mark(ix, st);
       if (split) {
         // ... tau_q = k-th best key of phase A ...
-        CK(launch_tau_select(b.poff + npairs, b.pcnt + npairs, part, nq, npb, ra, k, tau, tmax, over, st));
+        // (phase A emits < need + capA candidates per query: a tighter staging bound than tmax)
+        CK(launch_tau_select(b.poff + npairs, b.pcnt + npairs, part, nq, npb, ra, k, tau,
+                             std::min<int64_t>(tmax, pa.need + pa.capA), over, st));
         prof_mark(ix, st);
         // ... phase B over every probed pair, emitting keys <= tau_q
         tp.phase = 1;

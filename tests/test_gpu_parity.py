@@ -187,7 +187,7 @@ def test_sq8_sift_l2_conditional(k):
     assert frac > 0.999
 
 
-@pytest.mark.parametrize("k", [2048, 16384])
+@pytest.mark.parametrize("k", [300, 1000, 2048, 16384])
 def test_large_k(k):
     """k > 1024: single-pass radix select == plain top-k of the oracle."""
     n = 20_000
