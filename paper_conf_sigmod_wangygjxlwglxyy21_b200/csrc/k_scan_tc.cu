@@ -335,6 +335,19 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
     Pref cur;
     if (item(0) < nwork) cur = prefetch(item(0));
     uint32_t wcount = 0;
+    // the epilogue never waits for its peers at the end of an item: the gatherer publishes an
+    // item's candidate counts when its metadata buffer comes back (every epilogue warp has
+    // arrived on empty_m), each thread for the query slots it is about to overwrite
+    int prev_nqc[2] = {0, 0};
+    auto publish = [&](uint32_t bb) {
+      const Meta om = meta_at(metab + bb * p.meta_bytes, QCP);
+#pragma unroll
+      for (int u = 0; u < 2; ++u) {
+        const int i = tq + 64 * u;
+        if (i < prev_nqc[bb]) p.pcnt[om.pair[i]] = om.cnt[i];
+      }
+      prev_nqc[bb] = 0;
+    };
     for (int i = 0; item(i) < nwork; ++i, ++wcount) {
       Pref nxt;
       if (item(i + 1) < nwork) nxt = prefetch(item(i + 1));
@@ -344,6 +357,8 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
       const uint32_t b = wcount & 1, r = wcount >> 1;
       mbar_wait(&empty_q[b], (r & 1) ^ 1);
       mbar_wait(&empty_m[b], (r & 1) ^ 1);
+      publish(b);
+      prev_nqc[b] = wi.nqc;
       const Meta mt = meta_at(metab + b * p.meta_bytes, QCP);
       if (tq == 0) *mt.wi = wi;
 #pragma unroll
@@ -406,6 +421,13 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
       fence_proxy_async();
       mbar_arrive(&full_q[b]);
       cur = nxt;
+    }
+    // the last (up to) two items: wait until the epilogue is done with them, then publish
+    for (uint32_t e = wcount; e < wcount + 2; ++e) {
+      const uint32_t b = e & 1, r = e >> 1;
+      if (prev_nqc[b] == 0) continue;
+      mbar_wait(&empty_m[b], (r & 1) ^ 1);
+      publish(b);
     }
   } else {
     // ------------------------------------------------------------------ epilogue (8 warps)
@@ -515,7 +537,8 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
             }
           }
           if (__any_sync(MV_FULL, pm != 0) && !(p.dbg & 1)) {
-            // ballot per column; lane j reserves column j's slots with one shared atomic
+            // ballot per column; lane j reserves column j's slots with one shared atomic (measured:
+            // a per-entry atomic path for sparse chunks was slower on configs[1] and [2])
             uint32_t mj[W];
             int mine = 0;
 #pragma unroll
@@ -543,9 +566,8 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
           mbar_arrive(&empty_t[ts]);
         }
       }
-      // every epilogue warp is done with this work item: publish the pairs' counts, free the metadata
-      named_bar(1, 32 * kEpiWarps);
-      for (int i = et; i < wi.nqc; i += 32 * kEpiWarps) p.pcnt[mt.pair[i]] = mt.cnt[i];
+      // this warp is done with the work item (its slot reservations are in mt.cnt): free the
+      // metadata; the gatherer publishes the counts once every epilogue warp has arrived
       __syncwarp();
       if (lane == 0) mbar_arrive(&empty_m[b]);
     }

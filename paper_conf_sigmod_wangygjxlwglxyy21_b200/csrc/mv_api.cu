@@ -631,7 +631,20 @@ static mv_status search_impl(mv_index* ix, const float* queries, int64_t nq, int
     PlanArgs pa;
     pa.probes = P; pa.nq = nq; pa.npb = npb; pa.nlist = nlist; pa.k = k; pa.capk = capk;
     pa.split = split ? 1 : 0; pa.need = std::max<int64_t>(2 * (int64_t)k, k + 32);
-    if (const char* ne = getenv("MV_NEED")) pa.need = std::max<int64_t>(pa.need, atoll(ne));  // sweep override
+    // Sample size of the seeding phase.  tau_q = the k-th best of `need` candidates is about the
+    // (k N / need)-th best of the query's N candidates, so phase B emits ~k N / need keys.  Phase A
+    // costs ~need rows of payload, an emission ~a fixed number of bytes (the key store, the final
+    // select's reads); balancing the two gives need ~ sqrt(k N c / rowbytes).  c is measured
+    // (session-4 sweep): 32 B for k <= 256; the CTA-per-query select for k > 256 costs
+    // ~26x more per candidate (and falls back to global memory past its stage), c = 832 B.
+    {
+      const double ncand = (double)ix->ntotal * npb / std::max(1, nlist);
+      const double rowb = (double)dpad * (ix->type == MV_IVF_FLAT ? 4 : 1);
+      const double c = k > 256 ? 832.0 : 32.0;
+      const int64_t bal = (int64_t)std::sqrt((double)k * ncand * c / rowb);
+      pa.need = std::max<int64_t>(pa.need, std::min<int64_t>(bal, 65536));
+    }
+    if (const char* ne = getenv("MV_NEED")) pa.need = atoll(ne) > 0 ? std::max<int64_t>(2 * (int64_t)k, atoll(ne)) : pa.need;
     // phase A reads the first capA rows of each of a query's nearest lists (a 16-row multiple, at
     // least one tile; measured on configs[1]: 64 rows 14.7M qps, 128 rows 16.0M, 256 rows 15.8M,
     // whole lists 14.7M -- a looser tau_q costs phase-B emissions, more rows cost phase-A reads)
