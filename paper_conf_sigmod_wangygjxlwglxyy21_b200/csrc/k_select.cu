@@ -151,6 +151,71 @@ __global__ void __launch_bounds__(256) k_final_select(const int64_t* __restrict_
   }
 }
 
+
+// Ascending bitonic sort of NK = 512 E keys in shared memory by a 512-thread block.  Warp w holds
+// the contiguous block [32 E w, 32 E (w + 1)) in registers, lane l element 32 j + l in v[j]:
+// strides < 32 are shuffles, strides 32 .. 16 E register pairs, larger strides go through shared
+// memory (10 of the 66 stages for NK = 2048).  Pair (lo, lo + stride) of a size-`size` stage
+// is ascending when (lo & size) == 0: the lower element keeps the minimum.
+template <int E>
+__device__ __forceinline__ void block_sort_regs(uint64_t* win, int NK) {
+  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  const int wbase = wid * 32 * E;
+  uint64_t v[E > 0 ? E : 1];
+  constexpr int SMIN = E > 0 ? 32 * E : 1;  // smallest stride done in shared memory
+  __syncthreads();
+#pragma unroll
+  for (int j = 0; j < E; ++j) v[j] = win[wbase + 32 * j + lane];
+  for (int size = 2; size <= NK; size <<= 1) {
+    int stride = size >> 1;
+    if (stride >= SMIN) {
+#pragma unroll
+      for (int j = 0; j < E; ++j) win[wbase + 32 * j + lane] = v[j];
+      for (; stride >= SMIN; stride >>= 1) {
+        __syncthreads();
+        for (int t = tid; t < (NK >> 1); t += 512) {
+          const int lo = 2 * t - (t & (stride - 1));
+          const int hi = lo + stride;
+          const bool up = (lo & size) == 0;
+          const uint64_t x = win[lo], y = win[hi];
+          if ((x > y) == up) {
+            win[lo] = y;
+            win[hi] = x;
+          }
+        }
+      }
+      __syncthreads();
+#pragma unroll
+      for (int j = 0; j < E; ++j) v[j] = win[wbase + 32 * j + lane];
+    }
+#pragma unroll
+    for (int m = E / 2; m >= 1; m >>= 1) {
+      if (stride == 32 * m) {
+#pragma unroll
+        for (int j = 0; j < E; ++j)
+          if ((j & m) == 0) {
+            const bool up = ((wbase + 32 * j + lane) & size) == 0;
+            const uint64_t x = v[j], y = v[j | m];
+            v[j] = up ? umin64(x, y) : umax64(x, y);
+            v[j | m] = up ? umax64(x, y) : umin64(x, y);
+          }
+        stride >>= 1;
+      }
+    }
+    for (; stride > 0; stride >>= 1) {
+      const bool lower = (lane & stride) == 0;
+#pragma unroll
+      for (int j = 0; j < E; ++j) {
+        const bool up = ((wbase + 32 * j + lane) & size) == 0;
+        const uint64_t o = shfl_xor64(v[j], stride);
+        v[j] = (lower == up) ? umin64(v[j], o) : umax64(v[j], o);
+      }
+    }
+  }
+#pragma unroll
+  for (int j = 0; j < E; ++j) win[wbase + 32 * j + lane] = v[j];
+}
+
 // 256 < k: one CTA (512 threads) per query stages the query's candidates in shared memory (when
 // they fit, else it flags the query for k_final_select's global-memory path), then an MSB radix
 // select over the u64 keys -- 8-bit digits, histogram per pass in shared memory, stopping as soon
@@ -199,12 +264,16 @@ __global__ void __launch_bounds__(kBigThreads) k_final_big(const int64_t* __rest
     return;
   }
   if (tid == 0) over[q] = 0;
+  // staging by fire-and-forget 8-B async copies: every lane keeps its loads in flight (a plain
+  // load/store loop was latency-bound: one ~1 us global round trip per 32 keys per warp)
   for (int j = wid; j < nu; j += kBigThreads / 32) {
     const int c = s_pre[j + 1] - s_pre[j];
     const uint64_t* src = part + po[j];
-    uint64_t* dst = buf + s_pre[j];
-    for (int i = lane; i < c; i += 32) dst[i] = src[i];
+    const uint32_t dst = (uint32_t)__cvta_generic_to_shared(buf + s_pre[j]);
+    for (int i = lane; i < c; i += 32)
+      asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(dst + 8 * i), "l"(src + i) : "memory");
   }
+  asm volatile("cp.async.wait_all;" ::: "memory");
   __syncthreads();
   int nsel;  // winners to sort, in win[]
   if (T <= k) {
@@ -318,21 +387,13 @@ __global__ void __launch_bounds__(kBigThreads) k_final_big(const int64_t* __rest
     }
     return;
   }
-  // bitonic sort of the NK winners (block-wide, shared memory)
-  for (int size = 2; size <= NK; size <<= 1) {
-    for (int stride = size >> 1; stride > 0; stride >>= 1) {
-      __syncthreads();
-      for (int t = tid; t < (NK >> 1); t += kBigThreads) {
-        const int lo = 2 * t - (t & (stride - 1));
-        const int hi = lo + stride;
-        const bool up = ((lo & size) == 0);
-        const uint64_t x = win[lo], y = win[hi];
-        if ((x > y) == up) {
-          win[lo] = y;
-          win[hi] = x;
-        }
-      }
-    }
+  // bitonic sort of the NK winners: register-blocked (strides < 32 E by shuffles and in registers,
+  // only the larger strides through shared memory)
+  switch (NK / kBigThreads) {
+    case 1: block_sort_regs<1>(win, NK); break;
+    case 2: block_sort_regs<2>(win, NK); break;
+    case 4: block_sort_regs<4>(win, NK); break;
+    default: block_sort_regs<0>(win, NK); break;  // NK > 2048: shared memory only (registers stay < 64)
   }
   __syncthreads();
   for (int i = tid; i < k; i += kBigThreads) {
