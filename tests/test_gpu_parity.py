@@ -374,3 +374,24 @@ def test_search_with_probes_equals_search(kind, metric):
     torch.cuda.synchronize()
     assert torch.equal(I0, I1) and torch.equal(D0, D1)
     assert torch.equal(I0, I2) and torch.equal(D0, D2)
+
+
+@pytest.mark.parametrize("kind,metric,k", [("flat", "l2", 10), ("sq8", "ip", 100), ("flat", "l2", 600)])
+@pytest.mark.parametrize("need", ["1", "1000000"])
+def test_seeding_sample_size_extremes(kind, metric, k, need, monkeypatch):
+    """The seeding phase's sample size (DESIGN.md §5 `need`) only changes how tight tau_q is, never
+    the result: the 2k floor (loosest bound, most phase-B emissions) and a sample larger than every
+    query's candidate set (phase A scans all probed lists) both equal the oracle."""
+    monkeypatch.setenv("MV_NEED", need)
+    if kind == "flat":
+        X, Q = _sift(12_000, 60)
+        mo, ko = O.L2, O.FLAT
+    else:
+        X, Q = _deep(12_000, 60)
+        mo, ko = O.IP, O.SQ8
+    ids = G.permuted_ids(12_000, seed=21)
+    C = kmeans(X, 48, iters=4)
+    ix = _build(X, ids, C, metric, kind)
+    bs = G.mod_bitset(12_000, 10) if kind == "sq8" else None
+    frac, _, _ = _run_conditional(ix, X, ids, C, Q, k, 9, mo, ko, bitset=bs, nbits=12_000 if bs is not None else 0)
+    assert frac > (0.999 if kind == "sq8" else 0.9999)
