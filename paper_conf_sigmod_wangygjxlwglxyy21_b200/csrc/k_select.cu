@@ -152,7 +152,12 @@ __global__ void __launch_bounds__(256) k_final_select(const int64_t* __restrict_
 }
 
 
-// Ascending bitonic sort of NK = 512 E keys in shared memory by a 512-thread block.  Warp w holds
+// 256 < k: the CTA-per-query select's block size (32 warps: one CTA per SM when the candidate stage
+// takes all of shared memory, so the warps are the only latency hiding) and private histograms
+constexpr int kBigThreads = 1024;
+constexpr int kHistWarps = 8;  // private radix histograms (warps w, w + 8, ... share one)
+
+// Ascending bitonic sort of NK = kBigThreads E keys in shared memory by a kBigThreads block.  Warp w holds
 // the contiguous block [32 E w, 32 E (w + 1)) in registers, lane l element 32 j + l in v[j]:
 // strides < 32 are shuffles, strides 32 .. 16 E register pairs, larger strides go through shared
 // memory (10 of the 66 stages for NK = 2048).  Pair (lo, lo + stride) of a size-`size` stage
@@ -173,7 +178,7 @@ __device__ __forceinline__ void block_sort_regs(uint64_t* win, int NK) {
       for (int j = 0; j < E; ++j) win[wbase + 32 * j + lane] = v[j];
       for (; stride >= SMIN; stride >>= 1) {
         __syncthreads();
-        for (int t = tid; t < (NK >> 1); t += 512) {
+        for (int t = tid; t < (NK >> 1); t += kBigThreads) {
           const int lo = 2 * t - (t & (stride - 1));
           const int hi = lo + stride;
           const bool up = (lo & size) == 0;
@@ -216,12 +221,10 @@ __device__ __forceinline__ void block_sort_regs(uint64_t* win, int NK) {
   for (int j = 0; j < E; ++j) win[wbase + 32 * j + lane] = v[j];
 }
 
-// 256 < k: one CTA (512 threads) per query stages the query's candidates in shared memory (when
+// 256 < k: one CTA (kBigThreads threads) per query stages the query's candidates in shared memory (when
 // they fit, else it flags the query for k_final_select's global-memory path), then an MSB radix
 // select over the u64 keys -- 8-bit digits, histogram per pass in shared memory, stopping as soon
 // as the keys at or below the current prefix are exactly k -- and a bitonic sort of the k winners.
-constexpr int kBigThreads = 512;
-constexpr int kHistWarps = 8;  // private radix histograms (warps w and w + 8 share one)
 
 __global__ void __launch_bounds__(kBigThreads) k_final_big(const int64_t* __restrict__ poff,
                                                            const int32_t* __restrict__ pcnt,
@@ -393,7 +396,7 @@ __global__ void __launch_bounds__(kBigThreads) k_final_big(const int64_t* __rest
     case 1: block_sort_regs<1>(win, NK); break;
     case 2: block_sort_regs<2>(win, NK); break;
     case 4: block_sort_regs<4>(win, NK); break;
-    default: block_sort_regs<0>(win, NK); break;  // NK > 2048: shared memory only (registers stay < 64)
+    default: block_sort_regs<0>(win, NK); break;  // NK < 1024 or > 4096: shared memory only
   }
   __syncthreads();
   for (int i = tid; i < k; i += kBigThreads) {
