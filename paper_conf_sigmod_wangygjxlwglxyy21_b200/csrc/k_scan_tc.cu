@@ -80,6 +80,7 @@ __device__ __forceinline__ WorkInfo work_info(const TcScanParams& p, int w, int 
 }
 
 constexpr int kNTS = 4;          // per-tile side-data ring slots
+constexpr int kMaxAcc = 8;       // TMEM accumulator buffers (tiles in flight between MMA and epilogue)
 // side slot: norms f64 [1152 B] | rank u32 [640 B] | ids i64 [1152 B]; each copied as the 16-B aligned
 // superset of the tile's 128 rows (the arrays are padded at allocation so the copy stays in bounds)
 constexpr int kSideBytes = 3072;
@@ -158,8 +159,8 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
   uint64_t* empty_m = empty_q + 2;
   const int NACC = p.nacc;  // TMEM accumulator buffers (4 for FLAT, 2 for SQ8's 4-plane tiles)
   uint64_t* tfull = empty_m + 2;
-  uint64_t* tempty = tfull + 4;
-  uint64_t* full_t = tempty + 4;
+  uint64_t* tempty = tfull + kMaxAcc;
+  uint64_t* full_t = tempty + kMaxAcc;
   uint64_t* empty_t = full_t + kNTS;
   uint32_t* tslot = reinterpret_cast<uint32_t*>(empty_t + kNTS);
 
@@ -174,7 +175,7 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
       mbar_init(&empty_q[b], 1);
       mbar_init(&empty_m[b], kEpiWarps);
     }
-    for (int a = 0; a < 4; ++a) {
+    for (int a = 0; a < kMaxAcc; ++a) {
       mbar_init(&tfull[a], 1);
       mbar_init(&tempty[a], kEpiWarps);
     }
@@ -674,7 +675,10 @@ static bool tc_scan_layout(int type, int dpad, int qc, int ns, TcScanParams& p) 
   p.qchunk_split = type == MV_IVF_FLAT ? qc / 2 : qc;
   const int qcp = (qc + 15) & ~15;
   p.ncol = rows_per_q * qcp;
-  p.nacc = 512 / p.ncol >= 4 ? 4 : 2;
+  // FLAT: 4 accumulators of <= 96 columns; SQ8: as many 4-plane accumulators as TMEM holds (2 of
+  // 256 columns for 64-query items, 4 for 32, 8 for 16): the epilogue's latency per tile is
+  // hidden by the tiles in flight
+  p.nacc = type == MV_IVF_FLAT ? 4 : std::max(2, std::min(kMaxAcc, 512 / p.ncol));
   int cols = 32;
   while (cols < p.nacc * p.ncol) cols <<= 1;
   if (cols > 512) return false;
@@ -688,12 +692,16 @@ static bool tc_scan_layout(int type, int dpad, int qc, int ns, TcScanParams& p) 
   p.off_meta = p.off_q + 2 * p.q_bytes;
   p.off_side = up(p.off_meta + 2 * p.meta_bytes, 128);
   p.off_bar = p.off_side + kNTS * kSideBytes;
-  p.smem_total = p.off_bar + (2 * ns + 14 + 2 * kNTS) * 8 + 16 + 1024;  // + 1 KB alignment slack
+  p.smem_total = p.off_bar + (2 * ns + 6 + 2 * kMaxAcc + 2 * kNTS) * 8 + 16 + 1024;  // + 1 KB alignment slack
   return p.smem_total <= 227 * 1024;
 }
 
-bool tc_scan_plan(int type, int dpad, int k, TcScanParams& p) {
+bool tc_scan_plan(int type, int dpad, int k, double qpl, TcScanParams& p) {
   const bool wide = type == MV_IVF_FLAT || dpad % 128 == 0;  // 16-KB stages
+  // SQ8 items: 64 queries.  (Measured on configs[4], ~10 queries per probed list: 32-query items
+  // with 4 TMEM accumulators in flight 0.76M qps, 16 with 8 0.61M, 64 with 2 0.87M; qpl, the
+  // expected queries per probed list, is kept for the plan but does not change it.)
+  (void)qpl;
   int qcmax = type == MV_IVF_FLAT ? 96 : 64;
   if (const char* e = getenv("MV_SQ8_QC"); e && type == MV_IVF_SQ8) qcmax = std::max(16, std::min(64, atoi(e)));
   if (const char* e = getenv("MV_FLAT_QC"); e && type == MV_IVF_FLAT) qcmax = std::max(32, std::min(96, atoi(e)));

@@ -595,7 +595,8 @@ static mv_status search_impl(mv_index* ix, const float* queries, int64_t nq, int
     const bool use_qm = ix->type == MV_IVF_FLAT && impl && impl[0] == 'q';
     const bool use_tc = ix->xmap_ok && !(force && force[0] == '1') &&
                         (ix->type == MV_IVF_SQ8 || ix->tf32_exact) &&
-                        (use_qm ? qm_scan_plan(dpad, k, tp) : tc_scan_plan(ix->type, dpad, k, tp));
+                        (use_qm ? qm_scan_plan(dpad, k, tp)
+                                : tc_scan_plan(ix->type, dpad, k, (double)nq * npb / std::max(1, nlist), tp));
     const int qchunk = use_tc ? tp.qchunk
                               : (k <= kLocalSelectMaxK ? std::min(64, std::max(1, 65536 / (8 * k))) : 64);
     // device-side work-item shape: FLAT tf32-exact queries take one plane and twice the queries
@@ -648,9 +649,13 @@ static mv_status search_impl(mv_index* ix, const float* queries, int64_t nq, int
     // phase A reads the first capA rows of each of a query's nearest lists (a 16-row multiple, at
     // least one tile; measured on configs[1]: 64 rows 14.7M qps, 128 rows 16.0M, 256 rows 15.8M,
     // whole lists 14.7M -- a looser tau_q costs phase-B emissions, more rows cost phase-A reads)
-    pa.capA = std::max<int64_t>((pa.need + 15) & ~(int64_t)15, 128);
-    if (const char* ce = getenv("MV_CAPA"))  // override (at least the 16-row multiple of need)
-      pa.capA = std::max<int64_t>((pa.need + 15) & ~(int64_t)15, (atoll(ce) + 15) & ~15ll);
+    // Rows per list of the sample: ~sqrt(64 need), i.e. the sample spreads over ~sqrt(need / 64)
+    // nearest lists (measured, MV_CAPA sweep: configs[2] 256 rows 2.85M qps vs whole lists 2.71M;
+    // configs[4] 128 rows best; configs[1] 128 rows vs 64: 16.0M vs 14.7M), at least 128 rows
+    pa.capA = std::max<int64_t>(128, std::min<int64_t>((pa.need + 15) & ~(int64_t)15,
+                                                       ((int64_t)std::sqrt(64.0 * pa.need) + 15) & ~(int64_t)15));
+    if (const char* ce = getenv("MV_CAPA"))  // sweep override (a 16-row multiple)
+      pa.capA = std::max<int64_t>(16, (atoll(ce) + 15) & ~15ll);
     pa.list_off = ix->list_off;
     pa.qlo_any = (use_tc && ix->type == MV_IVF_FLAT) ? qlo_any : nullptr;
     pa.qc_exact = qchunk; pa.p_exact = use_tc ? (ix->type == MV_IVF_FLAT ? 1 : 4) : 1;

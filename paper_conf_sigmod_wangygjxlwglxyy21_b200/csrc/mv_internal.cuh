@@ -628,7 +628,7 @@ struct TcScanParams {
   int dbg;                 // debug bitmask (MV_SCAN_DEBUG): 1 skip emission, 2 skip epilogue math, 4 skip Q copy
   unsigned long long* prof;  // MV_SCAN_TRACE timeline (CTA 0)
 };
-bool tc_scan_plan(int type, int dpad, int k, TcScanParams& p);
+bool tc_scan_plan(int type, int dpad, int k, double qpl, TcScanParams& p);  // qpl: expected queries per probed list
 // the payload's tensor maps: boxes of 128, 64, 32, 16 rows (one swizzle atom wide)
 struct XMaps {
   CUtensorMap m[4];

@@ -395,3 +395,20 @@ def test_seeding_sample_size_extremes(kind, metric, k, need, monkeypatch):
     bs = G.mod_bitset(12_000, 10) if kind == "sq8" else None
     frac, _, _ = _run_conditional(ix, X, ids, C, Q, k, 9, mo, ko, bitset=bs, nbits=12_000 if bs is not None else 0)
     assert frac > (0.999 if kind == "sq8" else 0.9999)
+
+
+@pytest.mark.parametrize("qc", ["16", "32", "64"])
+@pytest.mark.parametrize("metric", ["l2", "ip"])
+def test_sq8_item_width_and_accumulators(qc, metric, monkeypatch):
+    """SQ8 work items of 16 / 32 / 64 queries (8 / 4 / 2 TMEM accumulators in flight),
+    lists probed by more queries than one item holds, a bitset: same answer as the oracle."""
+    monkeypatch.setenv("MV_SQ8_QC", qc)
+    X, Q = _sift(16_000, 150, n_micro=1024)
+    ids = G.permuted_ids(16_000, seed=17)
+    C = kmeans(X, 24, iters=4)
+    ix = _build(X, ids, C, metric, "sq8")
+    bs = G.mod_bitset(16_000, 7)
+    mo = O.IP if metric == "ip" else O.L2
+    frac, _, _ = _run_conditional(ix, X, ids, C, Q, 20, 5, mo, O.SQ8, bitset=bs, nbits=16_000)
+    assert ix.describe()["last_scan"] == "tcgen05.i8"
+    assert frac > 0.999
