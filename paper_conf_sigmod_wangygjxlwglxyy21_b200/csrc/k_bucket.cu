@@ -9,11 +9,12 @@
 //   0  zero the counters; the work-item shape {query chunk, planes} (qlo_any decides FLAT's)
 //   1  per query (warp): ra[q] = the fewest nearest lists holding >= need candidates (seeding),
 //      the query's region capacity, and the pair counts per virtual list
-//   2  exclusive scans: pair counts -> bucket offsets (block 0), capacities -> query bases (1)
+//   2  grid-wide exclusive scans: pair counts -> bucket offsets, capacities -> query bases
 //   3  per query: pair region offsets + bucket fill; per virtual list: work-item counts
-//   4  exclusive scan of the work-item counts (block 0)
-//   5  work items (virtual list, first bucket position)
-//   6  longest-first order (block 0, counting sort by cost; seeding phase first)
+//   4  grid-wide exclusive scan of the work-item counts
+//   5  work items (virtual list, first bucket position) + histogram of their cost keys
+//   6  longest-first order (counting sort by cost, seeding phase first: block 0 scans the
+//      histogram, every block scatters)
 #include <cooperative_groups.h>
 #include <cstdlib>
 
@@ -61,10 +62,77 @@ __device__ void block_exclusive_scan(const T* __restrict__ in, int64_t n, T* __r
   __syncthreads();
 }
 
+// Grid-wide exclusive scan out[0..n] (out[n] = total) in two passes separated by a grid barrier:
+// block b owns the contiguous segment [b*seg, (b+1)*seg).  Pass 1 writes the segment sum to
+// bsum[b]; pass 2 adds the sums of the earlier segments and scans the segment 1024 entries at a
+// time (coalesced loads, warp shuffles).  All threads of every block must call both passes.
+__device__ __forceinline__ void plan_segment(int64_t n, int64_t& s, int64_t& e) {
+  const int64_t seg = (n + gridDim.x - 1) / gridDim.x;
+  s = min64(n, (int64_t)blockIdx.x * seg);
+  e = min64(n, s + seg);
+}
+
+// block-wide sum, returned to every thread (red: 32 shared slots)
+__device__ __forceinline__ int64_t plan_block_sum(int64_t v, int64_t* red) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(MV_FULL, v, o);
+  __syncthreads();
+  if (lane == 0) red[warp] = v;
+  __syncthreads();
+  int64_t t = lane < (kPlanThreads >> 5) ? red[lane] : 0;
+  for (int o = 16; o > 0; o >>= 1) t += __shfl_xor_sync(MV_FULL, t, o);
+  return t;
+}
+
+template <typename T>
+__device__ void grid_scan_pass1(const T* __restrict__ in, int64_t n, int64_t* bsum, int64_t* red) {
+  int64_t s, e;
+  plan_segment(n, s, e);
+  int64_t acc = 0;
+  for (int64_t i = s + threadIdx.x; i < e; i += kPlanThreads) acc += in[i];
+  acc = plan_block_sum(acc, red);
+  if (threadIdx.x == 0) bsum[blockIdx.x] = acc;
+}
+
+template <typename T>
+__device__ void grid_scan_pass2(const T* __restrict__ in, int64_t n, T* __restrict__ out, const int64_t* bsum,
+                                int64_t* red) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  int64_t s, e;
+  plan_segment(n, s, e);
+  int64_t off = 0;
+  for (int i = threadIdx.x; i < (int)blockIdx.x; i += kPlanThreads) off += bsum[i];
+  off = plan_block_sum(off, red);
+  for (int64_t c = s; c < e; c += kPlanThreads) {
+    const int64_t i = c + threadIdx.x;
+    const int64_t v = i < e ? (int64_t)in[i] : 0;
+    int64_t incl = v;
+    for (int o = 1; o < 32; o <<= 1) {
+      const int64_t u = __shfl_up_sync(MV_FULL, incl, o);
+      if (lane >= o) incl += u;
+    }
+    __syncthreads();
+    if (lane == 31) red[warp] = incl;
+    __syncthreads();
+    if (warp == 0) {
+      int64_t w = red[lane];
+      for (int o = 1; o < 32; o <<= 1) {
+        const int64_t u = __shfl_up_sync(MV_FULL, w, o);
+        if (lane >= o) w += u;
+      }
+      red[lane] = w;
+    }
+    __syncthreads();
+    if (i < e) out[i] = (T)(off + (warp ? red[warp - 1] : 0) + incl - v);
+    off += red[31];
+  }
+  if (blockIdx.x == gridDim.x - 1 && threadIdx.x == 0) out[n] = (T)off;
+}
+
 __global__ void __launch_bounds__(kPlanThreads) k_plan(const PlanArgs a) {
   cg::grid_group grid = cg::this_grid();
   __shared__ int64_t part64[kPlanThreads];
-  __shared__ int hist[8192];
+  __shared__ int64_t red[32];
   const int tid = threadIdx.x, lane = tid & 31;
   const int64_t gtid = blockIdx.x * (int64_t)blockDim.x + tid;
   const int64_t gthreads = (int64_t)gridDim.x * blockDim.x;
@@ -78,6 +146,7 @@ __global__ void __launch_bounds__(kPlanThreads) k_plan(const PlanArgs a) {
     b.lcount[i] = 0;
     b.bfill[i] = 0;
   }
+  for (int64_t i = gtid; i < kPlanCostBins; i += gthreads) b.whist[i] = 0;
   if (gtid == 0) {
     const bool sp = a.qlo_any != nullptr && *a.qlo_any != 0;
     a.qcfg[0] = sp ? a.qc_split : a.qc_exact;
@@ -134,8 +203,11 @@ __global__ void __launch_bounds__(kPlanThreads) k_plan(const PlanArgs a) {
   grid.sync();
 
   // 2 ---------------------------------------------------------------------------------------
-  if (blockIdx.x == 0) block_exclusive_scan<int32_t>(b.lcount, nv, b.boff, reinterpret_cast<int32_t*>(part64));
-  if (blockIdx.x == gridDim.x - 1) block_exclusive_scan<int64_t>(b.qtot, a.nq, b.qtot + (a.nq + 1), part64);
+  grid_scan_pass1<int32_t>(b.lcount, nv, b.bsum, red);
+  grid_scan_pass1<int64_t>(b.qtot, a.nq, b.bsum + kPlanMaxBlocks, red);
+  grid.sync();
+  grid_scan_pass2<int32_t>(b.lcount, nv, b.boff, b.bsum, red);
+  grid_scan_pass2<int64_t>(b.qtot, a.nq, b.qtot + (a.nq + 1), b.bsum + kPlanMaxBlocks, red);
   grid.sync();
 
   // 3 ---------------------------------------------------------------------------------------
@@ -179,30 +251,29 @@ __global__ void __launch_bounds__(kPlanThreads) k_plan(const PlanArgs a) {
       run += __shfl_sync(MV_FULL, incl, 31);
     }
   }
-  for (int64_t v = gtid; v < nv; v += gthreads) b.wcount[v] = (b.lcount[v] + qchunk - 1) / qchunk;
-  grid.sync();
-
-  // 4 ---------------------------------------------------------------------------------------
-  if (blockIdx.x == 0) block_exclusive_scan<int32_t>(b.wcount, nv, b.woff, reinterpret_cast<int32_t*>(part64));
-  grid.sync();
-
-  // 5 ---------------------------------------------------------------------------------------
-  for (int64_t v = gtid; v < nv; v += gthreads) {
-    const int n = b.wcount[v], o = b.woff[v], bb = b.boff[v];
-    for (int c = 0; c < n; ++c) b.witems_unsorted[o + c] = make_int2((int)v, bb + c * qchunk);
+  {  // work-item counts over this block's segment, and their sum (pass 1 of step 4's scan)
+    int64_t s, e, acc = 0;
+    plan_segment(nv, s, e);
+    for (int64_t v = s + tid; v < e; v += kPlanThreads) {
+      const int c = (b.lcount[v] + qchunk - 1) / qchunk;
+      b.wcount[v] = c;
+      acc += c;
+    }
+    acc = plan_block_sum(acc, red);
+    if (tid == 0) b.bsum[blockIdx.x] = acc;
   }
   grid.sync();
 
-  // 6 --------------------------------------------------------------------------------------- 
-  // counting sort by descending cost key = 64 * tiles + queries (tiles = ceil(|list| / 128));
-  // every phase-A item (virtual list < nlist) precedes every phase-B item
-  if (blockIdx.x != 0) return;
-  constexpr int NB = 8192, HB = 4096;
-  const int nwork = b.woff[nv];
-  for (int i = tid; i < NB; i += kPlanThreads) hist[i] = 0;
-  __syncthreads();
-  auto key = [&](int w) {
-    const int2 it = b.witems_unsorted[w];
+  // 4 ---------------------------------------------------------------------------------------
+  grid_scan_pass2<int32_t>(b.wcount, nv, b.woff, b.bsum, red);
+  grid.sync();
+
+  // 5 ---------------------------------------------------------------------------------------
+  // work items, and the histogram of their cost keys: descending cost = 64 * tiles + queries
+  // (tiles = ceil(|list| / 128)); every phase-A item (virtual list < nlist) precedes every
+  // phase-B item
+  constexpr int HB = kPlanCostBins / 2;
+  auto key = [&](int2 it) {
     const int l = it.x >= nlist ? it.x - nlist : it.x;
     const int nqw = min(qchunk, b.boff[it.x + 1] - it.y);
     int64_t len = a.list_off[l + 1] - a.list_off[l];
@@ -210,29 +281,44 @@ __global__ void __launch_bounds__(kPlanThreads) k_plan(const PlanArgs a) {
     const int tiles = (int)min64((len + 127) / 128, 63);
     return (it.x >= nlist ? HB : 0) + HB - 1 - min(HB - 1, tiles * 64 + min(nqw, 63));
   };
-  for (int w = tid; w < nwork; w += kPlanThreads) atomicAdd(&hist[key(w)], 1);
-  __syncthreads();
-  int loc[8], acc = 0;
-#pragma unroll
-  for (int j = 0; j < 8; ++j) {
-    loc[j] = acc;
-    acc += hist[tid * 8 + j];
+  for (int64_t v = gtid; v < nv; v += gthreads) {
+    const int n = b.wcount[v], o = b.woff[v], bb = b.boff[v];
+    for (int c = 0; c < n; ++c) {
+      const int2 it = make_int2((int)v, bb + c * qchunk);
+      b.witems_unsorted[o + c] = it;
+      atomicAdd(b.whist + key(it), 1);
+    }
   }
-  int32_t* p32 = reinterpret_cast<int32_t*>(part64);
-  p32[tid] = acc;
-  __syncthreads();
-  for (int off = 1; off < kPlanThreads; off <<= 1) {
-    const int v = tid >= off ? p32[tid - off] : 0;
-    __syncthreads();
-    p32[tid] += v;
-    __syncthreads();
-  }
-  const int base = tid ? p32[tid - 1] : 0;
-  __syncthreads();
+  grid.sync();
+
+  // 6 ---------------------------------------------------------------------------------------
+  // counting sort by the cost key: block 0 scans the histogram, then every block scatters
+  if (blockIdx.x == 0) {
+    int loc[8], acc = 0;
 #pragma unroll
-  for (int j = 0; j < 8; ++j) hist[tid * 8 + j] = base + loc[j];
-  __syncthreads();
-  for (int w = tid; w < nwork; w += kPlanThreads) b.witems[atomicAdd(&hist[key(w)], 1)] = b.witems_unsorted[w];
+    for (int j = 0; j < 8; ++j) {
+      loc[j] = acc;
+      acc += b.whist[tid * 8 + j];
+    }
+    int32_t* p32 = reinterpret_cast<int32_t*>(part64);
+    p32[tid] = acc;
+    __syncthreads();
+    for (int off = 1; off < kPlanThreads; off <<= 1) {
+      const int v = tid >= off ? p32[tid - off] : 0;
+      __syncthreads();
+      p32[tid] += v;
+      __syncthreads();
+    }
+    const int base = tid ? p32[tid - 1] : 0;
+#pragma unroll
+    for (int j = 0; j < 8; ++j) b.whist[tid * 8 + j] = base + loc[j];
+  }
+  grid.sync();
+  const int nwork = b.woff[nv];
+  for (int64_t w = gtid; w < nwork; w += gthreads) {
+    const int2 it = b.witems_unsorted[w];
+    b.witems[atomicAdd(b.whist + key(it), 1)] = it;
+  }
 }
 
 // single-CTA exclusive scan for the add path (n up to a few million)
@@ -259,7 +345,7 @@ cudaError_t launch_plan(const PlanArgs& a, cudaStream_t st) {
     cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_plan, kPlanThreads, 0);
     const char* pb = getenv("MV_PLAN_BPS");  // blocks per SM (grid-wide barriers cost more with more blocks)
-    grid = nsm * std::max(1, std::min(per, pb ? atoi(pb) : 2));
+    grid = std::min(kPlanMaxBlocks, nsm * std::max(1, std::min(per, pb ? atoi(pb) : 2)));
   }
   PlanArgs args = a;
   void* kargs[] = {&args};

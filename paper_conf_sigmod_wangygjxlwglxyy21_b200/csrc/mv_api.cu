@@ -627,6 +627,8 @@ static mv_status search_impl(mv_index* ix, const float* queries, int64_t nq, int
     CK(s.alloc(&b.poff, (size_t)nent));
     CK(s.alloc(&b.pcnt, (size_t)nent));
     CK(s.alloc(&b.counter, 1));
+    CK(s.alloc(&b.whist, (size_t)kPlanCostBins));
+    CK(s.alloc(&b.bsum, (size_t)(2 * kPlanMaxBlocks)));
     // pair regions: the whole list (tensor-core scan: emit-all bound), or min(k, |list|) (SIMT)
     const int capk = use_tc ? 0 : k;
     PlanArgs pa;

@@ -547,7 +547,11 @@ struct Bucketing {
   int64_t* poff;     // nq*npb (x2 with seeding: phase-A entries at nq*npb + p)  region offset per pair
   int32_t* pcnt;     // nq*npb (x2 with seeding)  candidates written per pair
   int32_t* counter;  // 1          persistent scan work counter
+  int32_t* whist;    // kPlanCostBins  work-item cost histogram, then its exclusive scan
+  int64_t* bsum;     // 2 x kPlanMaxBlocks  per-block partial sums of the grid-wide scans
 };
+constexpr int kPlanCostBins = 8192;
+constexpr int kPlanMaxBlocks = 1024;
 // a4 in one cooperative launch (k_bucket.cu).  With the seeding split the pairs of query q with
 // probe rank < ra[q] form a first phase (virtual lists 0..nlist-1, work items first) and the
 // others a second (virtual lists nlist..2*nlist-1); arrays are then sized for 2*nlist lists.
