@@ -28,8 +28,8 @@ namespace mv {
 using namespace sm100;
 
 namespace {
-constexpr int kCEpi = 8;
-constexpr int kCThreads = 64 + 32 * kCEpi;  // warp 0 TMA, warp 1 MMA, warps 2..9 epilogue
+constexpr int kCEpiMax = 16;
+constexpr int kCThreads = 64 + 32 * kCEpiMax;  // warp 0 TMA, warp 1 MMA, warps 2..1+nepi epilogue
 }  // namespace
 
 __global__ void __launch_bounds__(kCThreads, 1)
@@ -53,8 +53,9 @@ __global__ void __launch_bounds__(kCThreads, 1)
   uint64_t* empty_a = bars + nstage;
   uint64_t* full_b = empty_a + nstage;
   uint64_t* tfull = full_b + 1;
-  uint64_t* tempty = tfull + 2;
-  uint32_t* tslot = reinterpret_cast<uint32_t*>(tempty + 2);
+  uint64_t* tempty = tfull + 4;
+  uint32_t* tslot = reinterpret_cast<uint32_t*>(tempty + 4);
+  const int nacc = p.nacc;
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
@@ -63,9 +64,9 @@ __global__ void __launch_bounds__(kCThreads, 1)
       mbar_init(&empty_a[s], 1);
     }
     mbar_init(full_b, 1);
-    for (int b = 0; b < 2; ++b) {
+    for (int b = 0; b < nacc; ++b) {
       mbar_init(&tfull[b], 1);
-      mbar_init(&tempty[b], kCEpi);
+      mbar_init(&tempty[b], p.nepi);
     }
     fence_mbar_init();
   }
@@ -108,8 +109,8 @@ __global__ void __launch_bounds__(kCThreads, 1)
       const bool qlo = p.qlo_any == nullptr || *p.qlo_any != 0;  // C_hi . Q_lo vanishes for tf32-exact queries
       uint32_t it = 0;
       for (int t = t0, tl = 0; t < t1; ++t, ++tl) {
-        const uint32_t a = tl & 1;
-        mbar_wait(&tempty[a], ((tl >> 1) & 1) ^ 1);
+        const uint32_t a = tl % nacc;
+        mbar_wait(&tempty[a], ((tl / nacc) & 1) ^ 1);
         tc_fence_after();
         const uint32_t d = tmem + a * NQB;
         for (int c = 0; c < nchunks; ++c, ++it) {
@@ -132,22 +133,22 @@ __global__ void __launch_bounds__(kCThreads, 1)
     }
   } else {
     // ------------------------------------------------------------------ epilogue: scores -> S
-    const int ew = warp - 2;             // 0..7
-    const int quarter = warp & 3;
-    const int half = ew >> 2;
+    const int ew = warp - 2;             // 0..nepi-1
+    const int quarter = warp & 3;        // TMEM lane quarter this warp may read
+    const int sub = ew >> 2, nsub = p.nepi >> 2;
     const int row = quarter * 32 + lane;  // centroid within the tile
     const int nqv = (int)min64(NQB, p.nq - q0);
     float* S = p.S + (int64_t)q0 * p.lds;
     uint32_t* G = p.G + (int64_t)q0 * p.ldg;
     for (int t = t0, tl = 0; t < t1; ++t, ++tl) {
-      const uint32_t a = tl & 1;
+      const uint32_t a = tl % nacc;
       const int cid = t * 128 + row;
       const bool valid = cid < p.nlist;
       const float cn = (valid && p.metric == MV_L2) ? __ldg(p.cnorm + cid) : 0.0f;
-      mbar_wait(&tfull[a], (tl >> 1) & 1);
+      mbar_wait(&tfull[a], (tl / nacc) & 1);
       tc_fence_after();
       const uint32_t tb = tmem + a * NQB + ((uint32_t)(quarter * 32) << 16);
-      for (int qc = half * 16; qc < ((p.dbg & 2) ? 0 : NQB); qc += 32) {
+      for (int qc = sub * 16; qc < ((p.dbg & 2) ? 0 : NQB); qc += 16 * nsub) {
         uint32_t rd[16];
         tmem_ld16(tb + qc, rd);
         tmem_wait_ld();
@@ -161,7 +162,7 @@ __global__ void __launch_bounds__(kCThreads, 1)
           // the minimum score key of the warp's 32 centroids: lets the select skip whole groups
           const uint32_t gm = __reduce_min_sync(MV_FULL, valid ? f2key(sc) : 0xffffffffu);
           if (j < jn) {
-            if (valid) *sp = sc;
+            if (valid && !(p.dbg & 4)) *sp = sc;
             if (lane == 0) *gp = gm;
           }
           sp += p.lds;
@@ -330,8 +331,13 @@ bool coarse_tc_plan(int dpad, int nprobe, int64_t nq, int nlist, int nsm, Coarse
   const int fixed = p.nchunks * 2 * p.nqb * 128;
   p.nstage = std::min(6, (budget - fixed) / stage);
   p.smem_total = fixed + p.nstage * stage + 256 + 1024;
+  p.nepi = 8;
+  p.nacc = 2;
+  if (const char* e = getenv("MV_COARSE_EPI")) p.nepi = std::max(4, std::min(kCEpiMax, atoi(e) / 4 * 4));
+  if (const char* e = getenv("MV_COARSE_NACC")) p.nacc = std::max(1, std::min(4, atoi(e)));
+  while (p.nacc > 1 && p.nacc * p.nqb > 512) --p.nacc;
   int cols = 32;
-  while (cols < 2 * p.nqb) cols <<= 1;
+  while (cols < p.nacc * p.nqb) cols <<= 1;
   p.tmem_cols = cols;
   return p.smem_total <= 227 * 1024;
 }
@@ -341,7 +347,7 @@ cudaError_t launch_coarse_tc(const CUtensorMap* cmap, const CUtensorMap* qmap, c
   const unsigned grid = (unsigned)(((nq + p.nqb - 1) / p.nqb) * p.csplit);
   cudaError_t e = cudaFuncSetAttribute(k_coarse_gemm, cudaFuncAttributeMaxDynamicSharedMemorySize, p.smem_total);
   if (e != cudaSuccess) return e;
-  k_coarse_gemm<<<grid, kCThreads, p.smem_total, st>>>(*cmap, *qmap, p);
+  k_coarse_gemm<<<grid, 64 + 32 * p.nepi, p.smem_total, st>>>(*cmap, *qmap, p);
   if ((e = cudaGetLastError()) != cudaSuccess) return e;
   const unsigned g2 = (unsigned)((nq * 32 + 255) / 256);
   const int R = (p.nprobe + 31) / 32;

@@ -649,7 +649,8 @@ cudaError_t launch_tf32_check(const float* x, int64_t n, int* flag, cudaStream_t
 struct CoarseParams {
   int64_t nq;
   int nlist, nchunks, nstage, nprobe, nqb, csplit, tmem_cols, metric, smem_total;
-  int dbg;                 // MV_COARSE_DEBUG: 2 skip the score stores
+  int nepi, nacc;          // epilogue warps (multiple of 4, <= 16), TMEM accumulators (<= 4)
+  int dbg;                 // MV_COARSE_DEBUG: 2 skip the epilogue, 4 skip the S stores (timing only)
   const float* cnorm;
   float* S;                // nq x lds scores (lds = roundup(nlist, 4))
   int64_t lds;
