@@ -184,7 +184,7 @@ static cudaError_t run_coarse(mv_index* ix, const float* qpad, const float* qhl,
       if (e == cudaSuccess) e = s.alloc(&cp.G, (size_t)nq * cp.ldg);
       if (e != cudaSuccess) return e;
       const char* cdbg = getenv("MV_COARSE_DEBUG");
-      cp.dbg = cdbg ? atoi(cdbg) : 0;
+      cp.dbg = (cdbg && npb > 1) ? atoi(cdbg) : 0;  // never on the add path's assignment (npb = 1)
       ix->last_coarse = "tcgen05.tf32";
       return launch_coarse_tc(&ix->cmap, &qmap, cp, nq, st);
     }
