@@ -140,10 +140,13 @@ __global__ void __launch_bounds__(kCThreads, 1)
     const int nqv = (int)min64(NQB, p.nq - q0);
     float* S = p.S + (int64_t)q0 * p.lds;
     uint32_t* G = p.G + (int64_t)q0 * p.ldg;
+    const bool l2 = p.metric == MV_L2;
+    const uint32_t ldsb = (uint32_t)p.lds * 4u;  // row stride of S in bytes
     for (int t = t0, tl = 0; t < t1; ++t, ++tl) {
       const uint32_t a = tl % nacc;
       const int cid = t * 128 + row;
       const bool valid = cid < p.nlist;
+      const bool store = valid && !(p.dbg & 4);
       const float cn = (valid && p.metric == MV_L2) ? __ldg(p.cnorm + cid) : 0.0f;
       mbar_wait(&tfull[a], (tl / nacc) & 1);
       tc_fence_after();
@@ -152,22 +155,23 @@ __global__ void __launch_bounds__(kCThreads, 1)
         uint32_t rd[16];
         tmem_ld16(tb + qc, rd);
         tmem_wait_ld();
-        float* sp = S + (int64_t)qc * p.lds + cid;
-        uint32_t* gp = G + (int64_t)qc * p.ldg + t * 4 + quarter;
+        // 32-bit strides inside the 16-column chunk (the 64-bit row pointer once per chunk); lane j
+        // keeps group minimum j and the G row stores go out as one instruction after the chunk
+        uint64_t sq;  // opaque to the compiler, so the row address is not rebuilt per column
+        asm("mov.b64 %0, %1;" : "=l"(sq) : "l"(S + (int64_t)qc * p.lds + cid));
         const int jn = min(16, nqv - qc);
+        uint32_t gmine = 0xffffffffu;
 #pragma unroll
         for (int j = 0; j < 16; ++j) {
           const float dot = __uint_as_float(rd[j]);
-          const float sc = p.metric == MV_L2 ? cn - 2.0f * dot : -dot;
+          const float sc = l2 ? cn - 2.0f * dot : -dot;
           // the minimum score key of the warp's 32 centroids: lets the select skip whole groups
           const uint32_t gm = __reduce_min_sync(MV_FULL, valid ? f2key(sc) : 0xffffffffu);
-          if (j < jn) {
-            if (valid && !(p.dbg & 4)) *sp = sc;
-            if (lane == 0) *gp = gm;
-          }
-          sp += p.lds;
-          gp += p.ldg;
+          if (lane == j) gmine = gm;
+          asm volatile("{ .reg .pred p; setp.ne.u32 p, %2, 0; @p st.global.f32 [%0], %1; }"
+                       :: "l"(sq + (uint64_t)((uint32_t)j * ldsb)), "f"(sc), "r"((uint32_t)(j < jn && store)));
         }
+        if (lane < jn) G[(int64_t)(qc + lane) * p.ldg + t * 4 + quarter] = gmine;
       }
       tc_fence_before();
       __syncwarp();
