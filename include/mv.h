@@ -57,6 +57,18 @@ typedef enum {
   MV_IVF_SQ8 = 1   /* fine quantizer keeps one byte per dimension */
 } mv_type;
 
+/* Device-memory allocator supplied by the caller.  alloc(bytes, stream, ctx)
+ * returns device memory on the index's device usable in stream order on `stream` (NULL on
+ * failure -> MV_ENOMEM); free(ptr, stream, ctx) releases it, stream-ordered after the work the
+ * library enqueued on `stream`.  The Python binding routes both to torch's caching allocator.
+ * The index storage is taken from it too (freed by mv_index_destroy).  Per-search scratch is
+ * requested in blocks of >= 16 MB (a few callbacks per search). */
+typedef struct {
+  void* (*alloc)(size_t bytes, void* stream, void* ctx);
+  void (*free)(void* ptr, void* stream, void* ctx);
+  void* ctx;
+} mv_allocator;
+
 typedef enum {
   MV_OK = 0,
   MV_EINVAL = -1, /* bad argument (range, null pointer, reserved id -1 in add, ...) */
@@ -67,11 +79,23 @@ typedef enum {
 } mv_status;
 
 /* Create an empty index on CUDA device `device`.
- *   d      >= 1 (rows are stored zero-padded to a multiple of 32 elements, which changes neither
- *             L2 nor IP); nlist >= 1 buckets (K-means buckets, K=16384 default).
+ *   d      1 <= d <= 512 (rows are stored zero-padded to a multiple of 32 elements, which changes
+ *             neither L2 nor IP; the tensor-core kernels stage a query operand of <= 512 dims in
+ *             shared memory); nlist >= 1 buckets (K-means buckets, K=16384
+ *             default).
+ *   alloc  nullable: every device allocation of the index goes through it (else cudaMalloc for
+ *             the storage and the device's stream-ordered pool for scratch).  Copied.
  * Synchronous.  *out receives the handle (destroy with mv_index_destroy). */
 MV_API mv_status mv_index_create(int32_t d, mv_metric metric, mv_type type, int32_t nlist, int32_t device,
-                          mv_index** out);
+                                 const mv_allocator* alloc, mv_index** out);
+
+/* Tuning options.  None changes a result (tested): they pick launch shapes, the seeding sample and
+ * the scratch budget.  Names: "seeding" (0/1), "need" (seeding sample, candidates), "capa" (rows
+ * per list of the sample), "sq8_qc" / "flat_qc" (queries per scan work item), "coarse_nqb",
+ * "coarse_cs", "coarse_epi", "coarse_nacc" (coarse GEMM shape), "workspace_bytes" (per-search
+ * scratch budget: larger batches run as several query chunks; 0 = half of the free device memory).
+ * value 0 = automatic.  MV_EINVAL for an unknown name or a negative value. */
+MV_API mv_status mv_index_set_option(mv_index* index, const char* name, int64_t value);
 
 /* Supply the coarse codebook C (§3.1): nlist x d fp32, row-major.  The
  * north star consumes supplied centroids; training them (k-means) is outside the library.
@@ -88,7 +112,7 @@ MV_API mv_status mv_index_train_sq8(mv_index* index, const float* sample, int64_
 MV_API mv_status mv_index_set_sq8(mv_index* index, const float* vmin, const float* vdiff);
 
 /* Insert n vectors (n x d fp32, row-major) with caller ids (n int64, any values except the
- * reserved -1; duplicates allowed).  Each vector goes to bucket I(v) = its closest centroid
+ * reserved -1; duplicates allowed); an index holds < 2^31 vectors.  Each vector goes to bucket I(v) = its closest centroid
  * (L2: argmin ||v-c||^2, IP: argmax <v,c>; ties -> smaller bucket id);
  * SQ8 codes are code = floor(255*clamp((x-vmin)/vdiff,0,1)) in fp32 with one rounding per
  * operation (bit-exact with the oracle).  Storage is list-major, each list in insertion order.
@@ -105,9 +129,15 @@ MV_API mv_status mv_index_add(mv_index* index, const float* vectors, const int64
  *   distances nq x k fp32 (out), ids nq x k int64 (out), row-major, best-first: ascending L2 /
  *             descending IP; exact ties ordered by smaller id, then storage position.  Slots
  *             beyond the number of candidates hold id -1 and distance +inf (L2) / -inf (IP).
- * Results are deterministic and independent of the rest of the batch.  Asynchronous on
- * `stream` for device pointers, except when k > 1024 (one stream synchronisation sizes the
- * candidate workspace). */
+ * Results are deterministic and independent of the rest of the batch (the batch runs as query
+ * chunks when its scratch would exceed the "workspace_bytes" budget).  Asynchronous on `stream`
+ * for device pointers.
+ * Precision: IVF_SQ8 distances come from int32-exact digit partials combined in fp64.  IVF_FLAT
+ * is exact on the tensor cores when the stored values and the queries are tf32-representable
+ * (integer-valued data); otherwise the scan runs as a filter whose fp32 badness carries a
+ * rigorous per-query error bound, and every candidate that can still reach the top-k is
+ * re-scored in fp64 from the fp32 vectors: returned distances are the fp64 values
+ * rounded to fp32 and the ids are those of the exact top-k. */
 MV_API mv_status mv_search(mv_index* index, const float* queries, int64_t nq, int32_t k, int32_t nprobe,
                     const uint8_t* bitset, int64_t nbits, float* distances, int64_t* ids, void* stream);
 

@@ -26,8 +26,19 @@ class MvError(RuntimeError):
 _lib = None
 
 _P = C.c_void_p
+
+ALLOC_FN = C.CFUNCTYPE(C.c_void_p, C.c_size_t, C.c_void_p, C.c_void_p)
+FREE_FN = C.CFUNCTYPE(None, C.c_void_p, C.c_void_p, C.c_void_p)
+
+
+class MvAllocator(C.Structure):
+    """mv_allocator of include/mv.h."""
+    _fields_ = [("alloc", ALLOC_FN), ("free", FREE_FN), ("ctx", C.c_void_p)]
+
 _SIGS = {
-    "mv_index_create": (C.c_int, [C.c_int32, C.c_int, C.c_int, C.c_int32, C.c_int32, C.POINTER(C.c_void_p)]),
+    "mv_index_create": (C.c_int, [C.c_int32, C.c_int, C.c_int, C.c_int32, C.c_int32, C.POINTER(MvAllocator),
+                                  C.POINTER(C.c_void_p)]),
+    "mv_index_set_option": (C.c_int, [_P, C.c_char_p, C.c_int64]),
     "mv_index_set_centroids": (C.c_int, [_P, _P]),
     "mv_index_train_sq8": (C.c_int, [_P, _P, C.c_int64]),
     "mv_index_set_sq8": (C.c_int, [_P, _P, _P]),

@@ -172,19 +172,38 @@ cudaError_t launch_id_keys(const int64_t* ids, int64_t n, uint64_t* keys, uint32
   return cudaGetLastError();
 }
 
+// rank[row] = position of (id, row) in sorted order; sorted_ids[rank] = id; row_of_rank[rank] =
+// storage row (nullable: FLAT only, the filter mode's exact re-scoring reads the row back)
 __global__ void k_rank_scatter(const uint64_t* __restrict__ skeys, const uint32_t* __restrict__ svals, int64_t n,
-                               uint32_t* rank, int64_t* sorted_ids) {
+                               uint32_t* rank, int64_t* sorted_ids, uint32_t* row_of_rank) {
   for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < n; t += (int64_t)gridDim.x * blockDim.x) {
     rank[svals[t]] = (uint32_t)t;
     sorted_ids[t] = (int64_t)(skeys[t] ^ 0x8000000000000000ull);
+    if (row_of_rank) row_of_rank[t] = svals[t];
   }
 }
 
 cudaError_t launch_rank_scatter(const uint64_t* skeys, const uint32_t* svals, int64_t n, uint32_t* rank,
-                                int64_t* sorted_ids, cudaStream_t st) {
+                                int64_t* sorted_ids, uint32_t* row_of_rank, cudaStream_t st) {
   if (n == 0) return cudaSuccess;
   int grid = (int)min64(kNumSMs * 8, (n + 255) / 256);
-  k_rank_scatter<<<grid, 256, 0, st>>>(skeys, svals, n, rank, sorted_ids);
+  k_rank_scatter<<<grid, 256, 0, st>>>(skeys, svals, n, rank, sorted_ids, row_of_rank);
+  return cudaGetLastError();
+}
+
+// max of non-negative doubles: their IEEE bit patterns order like unsigned integers
+__global__ void k_max_f64(const double* __restrict__ v, int64_t n, unsigned long long* out) {
+  unsigned long long m = 0;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    m = max(m, (unsigned long long)__double_as_longlong(v[i]));
+  for (int o = 16; o > 0; o >>= 1) m = max(m, __shfl_xor_sync(MV_FULL, m, o));
+  if ((threadIdx.x & 31) == 0) atomicMax(out, m);
+}
+
+cudaError_t launch_max_f64(const double* v, int64_t n, unsigned long long* out, cudaStream_t st) {
+  if (n == 0) return cudaSuccess;
+  int grid = (int)min64(kNumSMs * 4, (n + 255) / 256);
+  k_max_f64<<<grid, 256, 0, st>>>(v, n, out);
   return cudaGetLastError();
 }
 

@@ -16,7 +16,6 @@
 //   6  longest-first order (counting sort by cost, seeding phase first: block 0 scans the
 //      histogram, every block scatters)
 #include <cooperative_groups.h>
-#include <cstdlib>
 
 #include "mv_internal.cuh"
 
@@ -31,11 +30,7 @@ constexpr int kPlanThreads = 1024;
 // entries of virtual list l (phase A: the first min(|l|, capA) rows, region capacity the same,
 // pair id npairs + p).  Without it, pair p is an entry of virtual list l.
 
-// Region capacity of a pair: min(capk, |list|) when the SIMT scan selects locally (capk > 0,
-// k <= 1024), else |list| (every candidate that survives the bitset may be emitted).
-__device__ __forceinline__ int64_t pair_cap(int64_t len, int k, int capk) {
-  return (capk > 0 && k <= kLocalSelectMaxK) ? min64(capk, len) : len;
-}
+// Region capacity of a pair: |list| (every candidate that survives the bitset may be emitted).
 
 // single-block exclusive scan out[0..n] (out[n] = total) with all kPlanThreads threads
 template <typename T>
@@ -168,7 +163,7 @@ __global__ void __launch_bounds__(kPlanThreads) k_plan(const PlanArgs a) {
       if (j < npb) {
         const int l = pq[j];
         len = a.list_off[l + 1] - a.list_off[l];
-        capsum += pair_cap(len, a.k, a.capk);
+        capsum += len;
         if (a.split) len = min64(len, a.capA);  // phase A reads a prefix of each list
       }
       int64_t incl = len;
@@ -221,7 +216,7 @@ __global__ void __launch_bounds__(kPlanThreads) k_plan(const PlanArgs a) {
       int64_t c = 0;
       if (j < npb) {
         const int l = pq[j];
-        c = pair_cap(a.list_off[l + 1] - a.list_off[l], a.k, a.capk);
+        c = a.list_off[l + 1] - a.list_off[l];
         const int v = ra ? l + nlist : l;
         b.bq[b.boff[v] + atomicAdd(b.bfill + v, 1)] = (int32_t)(q * npb + j);
       }
@@ -344,8 +339,8 @@ cudaError_t launch_plan(const PlanArgs& a, cudaStream_t st) {
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_plan, kPlanThreads, 0);
-    const char* pb = getenv("MV_PLAN_BPS");  // blocks per SM (grid-wide barriers cost more with more blocks)
-    grid = std::min(kPlanMaxBlocks, nsm * std::max(1, std::min(per, pb ? atoi(pb) : 2)));
+    // two blocks per SM (grid-wide barriers cost more with more blocks)
+    grid = std::min(kPlanMaxBlocks, nsm * std::max(1, std::min(per, 2)));
   }
   PlanArgs args = a;
   void* kargs[] = {&args};

@@ -19,8 +19,6 @@
 // (Round 1 fused the selection into the GEMM epilogue; with 10 warps per SM that epilogue was
 // latency-bound on the per-tile folds.  Writing S costs 2 x nq x nlist x 4 B of HBM traffic --
 // 0.33 GB for configs[1] -- and buys a selection kernel at full occupancy.)
-#include <cstdlib>
-
 #include "mv_internal.cuh"
 #include "sm100.cuh"
 
@@ -146,12 +144,12 @@ __global__ void __launch_bounds__(kCThreads, 1)
       const uint32_t a = tl % nacc;
       const int cid = t * 128 + row;
       const bool valid = cid < p.nlist;
-      const bool store = valid && !(p.dbg & 4);
+      const bool store = valid;
       const float cn = (valid && p.metric == MV_L2) ? __ldg(p.cnorm + cid) : 0.0f;
       mbar_wait(&tfull[a], (tl / nacc) & 1);
       tc_fence_after();
       const uint32_t tb = tmem + a * NQB + ((uint32_t)(quarter * 32) << 16);
-      for (int qc = sub * 16; qc < ((p.dbg & 2) ? 0 : NQB); qc += 16 * nsub) {
+      for (int qc = sub * 16; qc < NQB; qc += 16 * nsub) {
         uint32_t rd[16];
         tmem_ld16(tb + qc, rd);
         tmem_wait_ld();
@@ -305,8 +303,8 @@ cudaError_t launch_hilo(const float* x, int64_t n, int d, int dpad, float* out, 
 
 // Plan: the query-block size NQB (multiple of 16, <= 128) and centroid split that minimise
 // (waves x per-CTA work) on nsm SMs, with >= 2 centroid stages in shared memory.
-bool coarse_tc_plan(int dpad, int nprobe, int64_t nq, int nlist, int nsm, CoarseParams& p) {
-  if (dpad % 32 != 0 || nprobe > 128) return false;
+bool coarse_tc_plan(int dpad, int nprobe, int64_t nq, int nlist, int nsm, const Options& o, CoarseParams& p) {
+  if (dpad % 32 != 0 || nprobe > 1024) return false;
   p.nchunks = dpad / 32;
   p.nprobe = nprobe;
   const int budget = 227 * 1024 - 1024 - 256;
@@ -330,15 +328,16 @@ bool coarse_tc_plan(int dpad, int nprobe, int64_t nq, int nlist, int nsm, Coarse
     }
   }
   if (best_cost < 0) return false;
-  if (const char* e = getenv("MV_COARSE_NQB")) p.nqb = std::max(16, std::min(128, atoi(e) / 16 * 16));
-  if (const char* e = getenv("MV_COARSE_CS")) p.csplit = std::max(1, std::min(ntiles, atoi(e)));
+  // tuning options (mv_index_set_option): they change the launch shape, never the result
+  if (o.coarse_nqb > 0) p.nqb = std::max(32, std::min(128, o.coarse_nqb / 16 * 16));
+  if (o.coarse_cs > 0) p.csplit = std::max(1, std::min(ntiles, o.coarse_cs));
   const int fixed = p.nchunks * 2 * p.nqb * 128;
   p.nstage = std::min(6, (budget - fixed) / stage);
   p.smem_total = fixed + p.nstage * stage + 256 + 1024;
   p.nepi = 8;
   p.nacc = 2;
-  if (const char* e = getenv("MV_COARSE_EPI")) p.nepi = std::max(4, std::min(kCEpiMax, atoi(e) / 4 * 4));
-  if (const char* e = getenv("MV_COARSE_NACC")) p.nacc = std::max(1, std::min(4, atoi(e)));
+  if (o.coarse_epi > 0) p.nepi = std::max(4, std::min(kCEpiMax, o.coarse_epi / 4 * 4));
+  if (o.coarse_nacc > 0) p.nacc = std::max(1, std::min(4, o.coarse_nacc));
   while (p.nacc > 1 && p.nacc * p.nqb > 512) --p.nacc;
   int cols = 32;
   while (cols < p.nacc * p.nqb) cols <<= 1;
@@ -357,7 +356,10 @@ cudaError_t launch_coarse_tc(const CUtensorMap* cmap, const CUtensorMap* qmap, c
   const int R = (p.nprobe + 31) / 32;
   if (R <= 1) k_probe_select<1><<<g2, 256, 0, st>>>(p.S, p.lds, p.G, p.ldg, nq, p.nlist, p.nprobe, p.probes);
   else if (R == 2) k_probe_select<2><<<g2, 256, 0, st>>>(p.S, p.lds, p.G, p.ldg, nq, p.nlist, p.nprobe, p.probes);
-  else k_probe_select<4><<<g2, 256, 0, st>>>(p.S, p.lds, p.G, p.ldg, nq, p.nlist, p.nprobe, p.probes);
+  else if (R <= 4) k_probe_select<4><<<g2, 256, 0, st>>>(p.S, p.lds, p.G, p.ldg, nq, p.nlist, p.nprobe, p.probes);
+  else if (R <= 8) k_probe_select<8><<<g2, 256, 0, st>>>(p.S, p.lds, p.G, p.ldg, nq, p.nlist, p.nprobe, p.probes);
+  else if (R <= 16) k_probe_select<16><<<g2, 256, 0, st>>>(p.S, p.lds, p.G, p.ldg, nq, p.nlist, p.nprobe, p.probes);
+  else k_probe_select<32><<<g2, 256, 0, st>>>(p.S, p.lds, p.G, p.ldg, nq, p.nlist, p.nprobe, p.probes);
   return cudaGetLastError();
 }
 

@@ -54,11 +54,18 @@ __device__ __forceinline__ float4 lds_f4(const float* p) {
   return v;
 }
 
-// CTA-0 event timeline for MV_SCAN_TRACE (row r holds up to 1024 clock64 stamps)
+// CTA-0 event timeline (row r holds up to 1024 clock64 stamps): a development build option
+// (-DMV_SCAN_TRACE), compiled out of the product library
+#ifdef MV_SCAN_TRACE
 #define MV_TRACE(row, idx)                                                                      \
   do {                                                                                        \
     if (p.prof && blockIdx.x == 0 && (idx) < 1024) p.prof[(row) * 1024 + (idx)] = clock64();  \
   } while (0)
+#else
+#define MV_TRACE(row, idx) \
+  do {                     \
+  } while (0)
+#endif
 
 struct WorkInfo {
   int l, bstart, nqc, len, ntiles;
@@ -143,6 +150,9 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
   const bool use_norms = p.metric == MV_L2;
   const bool use_ids = p.bitset != nullptr;
   const bool phaseB = p.phase != 0;
+  // FLAT filter mode: the tensor-core badness is an approximation with a rigorous error bound
+  // E_q (stored values or queries not tf32-exact); keys are re-scored exactly after the scan
+  const bool approx = TYPE == MV_IVF_FLAT && (p.approx_always || P == 2);
   // epilogue column chunk: 16 (FLAT), 8 (SQ8: few queries per list, so both warps of a lane quarter
   // get columns)
   constexpr int W = TYPE == MV_IVF_FLAT ? 16 : 8;
@@ -196,12 +206,14 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
   tc_fence_after();
   const uint32_t tmem = *tslot;
   const int nwork = *p.nwitems;
+#ifdef MV_SCAN_TRACE
   auto gtimer = []() {
     uint64_t t;
     asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
     return t;
   };
   if (p.prof && threadIdx.x == 0 && blockIdx.x < 148) p.prof[8 * 1024 + blockIdx.x * 3] = gtimer();
+#endif
   // static schedule over the longest-first item order, snake-wise: round i gives CTA b the item
   // i*G + b (even rounds) or i*G + G-1-b (odd rounds), which balances sorted costs far better than
   // plain round-robin (every role walks the same sequence)
@@ -294,10 +306,12 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
         }
         mma_commit(&empty_q[b]);
       }
+#ifdef MV_SCAN_TRACE
       if (p.prof && blockIdx.x < 148) {
         p.prof[8 * 1024 + blockIdx.x * 3 + 1] = gtimer();
         p.prof[8 * 1024 + blockIdx.x * 3 + 2] = titer;
       }
+#endif
     }
   } else if (warp < 4) {
     // ------------------------------------------------------------------ query gatherer (64 thr)
@@ -310,7 +324,7 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
       int pr[2], q[2];
       uint64_t tau[2];
       double qn[2], qa[2];
-      float qs[2];
+      float qs[2], qe[2];
       int64_t base[2];
     };
     auto prefetch = [&](int w) {
@@ -327,6 +341,7 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
           f.tau[u] = phaseB ? p.tau[f.q[u]] : MV_KEY_PAD;
           f.qn[u] = p.qnorm[f.q[u]];
           f.qs[u] = TYPE == MV_IVF_SQ8 ? p.qscale[f.q[u]] : 1.0f;
+          f.qe[u] = (TYPE == MV_IVF_FLAT && approx) ? p.qerr[f.q[u]] : 0.0f;
           f.qa[u] = TYPE == MV_IVF_SQ8 ? p.qa[f.q[u]] : 0.0;
           f.base[u] = p.poff[f.pr[u]];
         }
@@ -372,7 +387,11 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
           mt.pair[i] = cur.pr[u];
           mt.cnt[i] = 0;
           mt.tau[i] = t;
-          mt.thf[i] = t32 >= 0xff800000u ? __int_as_float(0x7f800000) : key2f(t32);
+          // filter mode: tau_q is the k-th best approximate key of phase A, so a candidate of the
+          // exact top-k has an approximate badness <= tau_q + 2 E_q (DESIGN.md §5 "FLAT precision")
+          mt.thf[i] = t32 >= 0xff800000u ? __int_as_float(0x7f800000)
+                      : approx          ? __fadd_ru(key2f(t32), 2.0f * cur.qe[u])
+                                        : key2f(t32);
           mt.qnf[i] = (float)cur.qn[u];
           mt.qn[i] = cur.qn[u];
           mt.qs[i] = cur.qs[u];
@@ -406,7 +425,7 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
       uint8_t* Qb = Qs + b * p.q_bytes;
       constexpr int PIECES = ATOM / 16;
       const int ppr = nchunks * PIECES;  // pieces per row
-      const int nrows = (p.dbg & 4) ? 0 : wi.nqc * P;
+      const int nrows = wi.nqc * P;
       for (int u = gw; u < nrows; u += 2) {
         const int i = P == 1 ? u : (P == 2 ? u >> 1 : u >> 2);
         const int pl = u - i * P;
@@ -464,7 +483,7 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
         if (et == 0) MV_TRACE(6, titer);
         tc_fence_after();
         const uint32_t tbase = tmem + a * p.ncol + ((uint32_t)(quarter * 32) << 16);
-        for (int qc = half * W; qc < ((p.dbg & 2) ? 0 : NQ); qc += NPART * W) {
+        for (int qc = half * W; qc < NQ; qc += NPART * W) {
           uint32_t r[PMAX][W];
 #pragma unroll
           for (int pl = 0; pl < PMAX; ++pl) {
@@ -514,7 +533,7 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
             }
           }
           if (!valid) pm = 0;
-          if (TYPE == MV_IVF_FLAT) pe &= phaseB ? pm : 0u;
+          if (TYPE == MV_IVF_FLAT) pe &= (phaseB && !approx) ? pm : 0u;
           // pass 2 (flagged entries only): SQ8's exact fp64 badness; the exact key test at the bound
           if (__any_sync(MV_FULL, (TYPE == MV_IVF_SQ8 ? pm : pe) != 0)) {
 #pragma unroll
@@ -537,7 +556,7 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
               }
             }
           }
-          if (__any_sync(MV_FULL, pm != 0) && !(p.dbg & 1)) {
+          if (__any_sync(MV_FULL, pm != 0)) {
             // ballot per column; lane j reserves column j's slots with one shared atomic (measured:
             // a per-entry atomic path for sparse chunks was slower on configs[1] and [2])
             uint32_t mj[W];
@@ -588,7 +607,7 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
 // ----------------------------------------------------------------------------------------------
 __global__ void k_qplanes(int type, const float* __restrict__ qpad, int64_t nq, int dpad, const float* __restrict__ vmin,
                           const float* __restrict__ vdiff, uint8_t* __restrict__ out, float* __restrict__ qscale,
-                          double* __restrict__ qa, double* __restrict__ qnorm) {
+                          double* __restrict__ qa, double* __restrict__ qnorm, FlatErr fe, float* __restrict__ qerr) {
   const int lane = threadIdx.x & 31;
   const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
@@ -599,7 +618,19 @@ __global__ void k_qplanes(int type, const float* __restrict__ qpad, int64_t nq, 
     for (int o = 16; o > 0; o >>= 1) nn += __shfl_xor_sync(MV_FULL, nn, o);
     if (lane == 0) qnorm[q] = nn;
     if (type == MV_IVF_FLAT) {
-      // FLAT planes are the plane-major hi/lo split made by launch_hilo (shared with the coarse step)
+      // FLAT planes are the plane-major hi/lo split made by launch_hilo (shared with the coarse step).
+      // Filter-mode bound E_q >= |approximate - exact badness| for every stored x:
+      // the MMA sees x (1 + ex) and q (1 + eq) per element, so |q~.x~ - q.x| <= (ex + eq + ex eq) S
+      // with S = sum |q_j x_j| <= ||q|| X; the fp32 accumulation of dpad exact tf32 products adds
+      // <= dpad 2^-24 S per rounding chain (taken as (dpad + 4) 2^-23: 2x slack for the
+      // accumulator's internal order, + the hi/lo column sum); 5% on top.  L2 doubles the dot's
+      // error and adds the fp32 expansion (||q||^2 + ||x||^2) - 2 dot: <= 2^-22 (||q||^2 + X^2).
+      if (qerr && lane == 0) {
+        const double S = sqrt(nn) * sqrt(fe.xmax2);
+        const double cdot = 1.05 * (fe.ex + fe.eq + fe.ex * fe.eq + (dpad + 4) * 0x1p-23);
+        const double E = fe.metric == MV_L2 ? 2.0 * cdot * S + 0x1p-21 * (nn + fe.xmax2) : cdot * S + 0x1p-23 * S;
+        qerr[q] = __double2float_ru(E);
+      }
     } else {
       // fp64: w_j = q_j b_j, b_j = vdiff_j / 255, a_j = vmin_j + b_j / 2 (mid-bin decode)
       double amax = 0.0, dot = 0.0;
@@ -634,10 +665,12 @@ __global__ void k_qplanes(int type, const float* __restrict__ qpad, int64_t nq, 
 }
 
 cudaError_t launch_qplanes(int type, const float* qpad, int64_t nq, int dpad, const float* vmin, const float* vdiff,
-                           uint8_t* out, float* qscale, double* qa, double* qnorm, cudaStream_t st) {
+                           uint8_t* out, float* qscale, double* qa, double* qnorm, const FlatErr* fe, float* qerr,
+                           cudaStream_t st) {
   if (nq == 0) return cudaSuccess;
   const int grid = (int)min64(kNumSMs * 16, (nq * 32 + 255) / 256);
-  k_qplanes<<<grid, 256, 0, st>>>(type, qpad, nq, dpad, vmin, vdiff, out, qscale, qa, qnorm);
+  const FlatErr f = fe ? *fe : FlatErr{0.0, 0.0, 0.0, 0};
+  k_qplanes<<<grid, 256, 0, st>>>(type, qpad, nq, dpad, vmin, vdiff, out, qscale, qa, qnorm, f, fe ? qerr : nullptr);
   return cudaGetLastError();
 }
 
@@ -674,7 +707,9 @@ static bool tc_scan_layout(int type, int dpad, int qc, int ns, TcScanParams& p) 
   p.qchunk = qc;
   p.qchunk_split = type == MV_IVF_FLAT ? qc / 2 : qc;
   const int qcp = (qc + 15) & ~15;
-  p.ncol = rows_per_q * qcp;
+  // FLAT two-plane items hold qc/2 queries: N = 2 roundup16(qc/2) columns, which exceeds qcp for
+  // qc = 16, 48, 80 -- the operand and the accumulators are sized for the wider of the two shapes
+  p.ncol = type == MV_IVF_FLAT ? std::max(qcp, 2 * ((qc / 2 + 15) & ~15)) : rows_per_q * qcp;
   // FLAT: 4 accumulators of <= 96 columns; SQ8: as many 4-plane accumulators as TMEM holds (2 of
   // 256 columns for 64-query items, 4 for 32, 8 for 16): the epilogue's latency per tile is
   // hidden by the tiles in flight
@@ -683,7 +718,7 @@ static bool tc_scan_layout(int type, int dpad, int qc, int ns, TcScanParams& p) 
   while (cols < p.nacc * p.ncol) cols <<= 1;
   if (cols > 512) return false;
   p.tmem_cols = cols;
-  p.q_bytes = up(rows_per_q * qcp * dpad * esz, 1024);
+  p.q_bytes = up(p.ncol * dpad * esz, 1024);
   p.meta_bytes = up(32 + kMetaPerQuery * qcp, 16);
   const int stage = 128 * atom;
   p.nstage = ns;
@@ -696,15 +731,16 @@ static bool tc_scan_layout(int type, int dpad, int qc, int ns, TcScanParams& p) 
   return p.smem_total <= 227 * 1024;
 }
 
-bool tc_scan_plan(int type, int dpad, int k, double qpl, TcScanParams& p) {
+bool tc_scan_plan(int type, int dpad, int k, double qpl, const Options& o, TcScanParams& p) {
   const bool wide = type == MV_IVF_FLAT || dpad % 128 == 0;  // 16-KB stages
   // SQ8 items: 64 queries.  (Measured on configs[4], ~10 queries per probed list: 32-query items
   // with 4 TMEM accumulators in flight 0.76M qps, 16 with 8 0.61M, 64 with 2 0.87M; qpl, the
   // expected queries per probed list, is kept for the plan but does not change it.)
   (void)qpl;
   int qcmax = type == MV_IVF_FLAT ? 96 : 64;
-  if (const char* e = getenv("MV_SQ8_QC"); e && type == MV_IVF_SQ8) qcmax = std::max(16, std::min(64, atoi(e)));
-  if (const char* e = getenv("MV_FLAT_QC"); e && type == MV_IVF_FLAT) qcmax = std::max(32, std::min(96, atoi(e)));
+  // tuning options (mv_index_set_option "sq8_qc" / "flat_qc"): launch shape only, never the result
+  if (o.sq8_qc > 0 && type == MV_IVF_SQ8) qcmax = std::max(16, std::min(64, o.sq8_qc / 16 * 16));
+  if (o.flat_qc > 0 && type == MV_IVF_FLAT) qcmax = std::max(16, std::min(96, o.flat_qc / 16 * 16));
   const int nscap = wide ? 8 : 24;
   const int nsmin = wide ? 4 : 6;  // >= 64 KB (16-KB stages) / 24 KB (4-KB stages) of list tiles in flight
   p.k = k;

@@ -29,7 +29,9 @@ __global__ void __launch_bounds__(256) k_final_select(const int64_t* __restrict_
                                                       const uint64_t* __restrict__ part, int64_t nq, int npb, int k,
                                                       int metric, const int64_t* __restrict__ sorted_ids, float* out_d,
                                                       int64_t* out_i, int selcap, const int32_t* __restrict__ nuse,
-                                                      uint64_t* tau_out, const uint8_t* __restrict__ only) {
+                                                      uint64_t* tau_out, const uint8_t* __restrict__ only,
+                                                      const int* __restrict__ gate) {
+  if (gate && *gate == 0) return;         // approximate-mode work, not needed by this search
   if (only && !only[blockIdx.x]) return;  // handled by k_final_big
   extern __shared__ __align__(16) uint8_t smem[];
   uint64_t* sel = reinterpret_cast<uint64_t*>(smem);       // selcap
@@ -232,7 +234,8 @@ __global__ void __launch_bounds__(kBigThreads) k_final_big(const int64_t* __rest
                                                            int metric, const int64_t* __restrict__ sorted_ids,
                                                            float* out_d, int64_t* out_i, int cap,
                                                            const int32_t* __restrict__ nuse, uint64_t* tau_out,
-                                                           uint8_t* over) {
+                                                           uint8_t* over, const int* __restrict__ gate) {
+  if (gate && *gate == 0) return;
   extern __shared__ __align__(16) uint8_t smem[];
   const int NK = next_pow2(max(k, 2));
   uint64_t* buf = reinterpret_cast<uint64_t*>(smem);   // cap
@@ -421,7 +424,7 @@ __global__ void __launch_bounds__(kBigThreads) k_final_big(const int64_t* __rest
 static cudaError_t launch_big_select(const int64_t* poff, const int32_t* pcnt, const uint64_t* part, int64_t nq,
                                      int npb, int k, int metric, const int64_t* sorted_ids, float* out_d,
                                      int64_t* out_i, const int32_t* nuse, uint64_t* tau, int64_t tmax,
-                                     uint8_t* over, cudaStream_t st) {
+                                     uint8_t* over, const int* gate, cudaStream_t st) {
   const int NK = next_pow2(max(k, 2));
   const int fixed = NK * 8 + kHistWarps * 256 * 4 + (npb + 1) * 4 + 64 + 64;
   // stage capacity: all of shared memory, or just the bound tmax when that is smaller (several
@@ -432,7 +435,7 @@ static cudaError_t launch_big_select(const int64_t* poff, const int32_t* pcnt, c
     cudaError_t e = cudaFuncSetAttribute(k_final_big, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     k_final_big<<<(unsigned)nq, kBigThreads, smem, st>>>(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d,
-                                                         out_i, cap, nuse, tau, over);
+                                                         out_i, cap, nuse, tau, over, gate);
     if (tmax <= cap) return cudaGetLastError();
   } else {
     over = nullptr;
@@ -442,7 +445,7 @@ static cudaError_t launch_big_select(const int64_t* poff, const int32_t* pcnt, c
   cudaError_t e = cudaFuncSetAttribute(k_final_select, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   k_final_select<<<(unsigned)nq, 256, smem, st>>>(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d, out_i,
-                                                  selcap, nuse, tau, over);
+                                                  selcap, nuse, tau, over, gate);
   return cudaGetLastError();
 }
 
@@ -456,11 +459,11 @@ __global__ void __launch_bounds__(256) k_final_warp(const int64_t* __restrict__ 
                                                     const uint64_t* __restrict__ part, int64_t nq, int npb, int k,
                                                     int metric, const int64_t* __restrict__ sorted_ids, float* out_d,
                                                     int64_t* out_i, const int32_t* __restrict__ nuse,
-                                                    uint64_t* tau_out) {
+                                                    uint64_t* tau_out, const int* __restrict__ gate) {
   __shared__ uint64_t stage_all[8][64];
   const int lane = threadIdx.x & 31;
   const int64_t q = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-  if (q >= nq) return;
+  if (q >= nq || (gate && *gate == 0)) return;
   uint64_t* stage = stage_all[threadIdx.x >> 5];
   const int stride = npb;
   if (nuse) npb = nuse[q];
@@ -577,16 +580,20 @@ __global__ void __launch_bounds__(256) k_final_warp(const int64_t* __restrict__ 
 // k <= 256: the warp kernel with a 32R-entry register list (R = 1, 2, 4, 8)
 static bool launch_warp_select(const int64_t* poff, const int32_t* pcnt, const uint64_t* part, int64_t nq, int npb,
                                int k, int metric, const int64_t* sorted_ids, float* out_d, int64_t* out_i,
-                               const int32_t* nuse, uint64_t* tau, cudaStream_t st) {
+                               const int32_t* nuse, uint64_t* tau, const int* gate, cudaStream_t st) {
   const unsigned grid = (unsigned)((nq * 32 + 255) / 256);
   if (k <= 32)
-    k_final_warp<1><<<grid, 256, 0, st>>>(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d, out_i, nuse, tau);
+    k_final_warp<1><<<grid, 256, 0, st>>>(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d, out_i, nuse, tau,
+                                         gate);
   else if (k <= 64)
-    k_final_warp<2><<<grid, 256, 0, st>>>(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d, out_i, nuse, tau);
+    k_final_warp<2><<<grid, 256, 0, st>>>(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d, out_i, nuse, tau,
+                                         gate);
   else if (k <= 128)
-    k_final_warp<4><<<grid, 256, 0, st>>>(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d, out_i, nuse, tau);
+    k_final_warp<4><<<grid, 256, 0, st>>>(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d, out_i, nuse, tau,
+                                         gate);
   else if (k <= 256)
-    k_final_warp<8><<<grid, 256, 0, st>>>(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d, out_i, nuse, tau);
+    k_final_warp<8><<<grid, 256, 0, st>>>(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d, out_i, nuse, tau,
+                                         gate);
   else
     return false;
   return true;
@@ -596,19 +603,114 @@ cudaError_t launch_final_select(const int64_t* poff, const int32_t* pcnt, const 
                                 int k, int metric, const int64_t* sorted_ids, float* out_d, int64_t* out_i,
                                 int64_t tmax, uint8_t* over, cudaStream_t st) {
   if (nq == 0) return cudaSuccess;
-  if (launch_warp_select(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d, out_i, nullptr, nullptr, st))
+  if (launch_warp_select(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d, out_i, nullptr, nullptr, nullptr,
+                         st))
     return cudaGetLastError();
   return launch_big_select(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d, out_i, nullptr, nullptr, tmax,
-                           over, st);
+                           over, nullptr, st);
 }
 
 cudaError_t launch_tau_select(const int64_t* poff, const int32_t* pcnt, const uint64_t* part, int64_t nq, int npb,
                               const int32_t* nuse, int k, uint64_t* tau, int64_t tmax, uint8_t* over,
-                              cudaStream_t st) {
+                              const int* gate, cudaStream_t st) {
   if (nq == 0) return cudaSuccess;
-  if (launch_warp_select(poff, pcnt, part, nq, npb, k, MV_L2, nullptr, nullptr, nullptr, nuse, tau, st))
+  if (launch_warp_select(poff, pcnt, part, nq, npb, k, MV_L2, nullptr, nullptr, nullptr, nuse, tau, gate, st))
     return cudaGetLastError();
-  return launch_big_select(poff, pcnt, part, nq, npb, k, MV_L2, nullptr, nullptr, nullptr, nuse, tau, tmax, over, st);
+  return launch_big_select(poff, pcnt, part, nq, npb, k, MV_L2, nullptr, nullptr, nullptr, nuse, tau, tmax, over, gate,
+                           st);
+}
+
+// ------------------------------------------------------------------------------------------
+// Exact re-scoring for the FLAT tensor-core scan's filter mode (DESIGN.md §5 "FLAT precision").
+// When the stored vectors or the queries are not tf32-exact, the scan's keys carry the fp32
+// tensor-core badness b~, with |b~ - b| <= E_q (qerr[q], a rigorous bound).  With t~ = the k-th
+// smallest b~ of the query (tau2[q]), every member of the exact top-k has b~ <= t~ + 2 E_q (k
+// candidates have b <= t~ + E_q), and every candidate above that bound has b > t~ + E_q.  So the
+// kernel recomputes b exactly -- fp64 from the fp32 query and the fp32 stored row, the oracle's
+// definition (§2.1) -- for the candidates at or below the bound, rewrites their
+// keys (exact fp32 distance key << 32 | id rank), and turns every other key into padding.  The
+// final select then returns the exact top-k.  One warp per query; the query row lives in
+// registers (dpad <= 512: <= 4 float4 per lane), each re-scored row is read as coalesced float4s.
+// ------------------------------------------------------------------------------------------
+__global__ void __launch_bounds__(256) k_rekey(const int64_t* __restrict__ poff, const int32_t* __restrict__ pcnt,
+                                               uint64_t* __restrict__ part, int64_t nq, int npb,
+                                               const uint64_t* __restrict__ tau2, const float* __restrict__ qerr,
+                                               int metric, const float* __restrict__ qpad, int dpad,
+                                               const float* __restrict__ payload,
+                                               const uint32_t* __restrict__ row_of_rank,
+                                               const int* __restrict__ gate) {
+  const int lane = threadIdx.x & 31;
+  const int64_t q = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  if (q >= nq || (gate && *gate == 0)) return;
+  const uint64_t t = tau2[q];
+  // bound in badness units, rounded up; fewer than k candidates (t = PAD): every candidate
+  const float bound =
+      t == MV_KEY_PAD ? __int_as_float(0x7f800000) : __fadd_ru(key2f((uint32_t)(t >> 32)), 2.0f * qerr[q]);
+  float4 qr[4];
+  const float4* qv = reinterpret_cast<const float4*>(qpad + q * dpad);
+#pragma unroll
+  for (int u = 0; u < 4; ++u) qr[u] = (4 * (lane + 32 * u) < dpad) ? qv[lane + 32 * u] : make_float4(0.f, 0.f, 0.f, 0.f);
+  const bool l2 = metric == MV_L2;
+  for (int g = 0; g < npb; g += 32) {
+    const int j = g + lane;
+    const int cnt = j < npb ? pcnt[q * npb + j] : 0;
+    const int64_t off = j < npb ? poff[q * npb + j] : 0;
+    int incl = cnt;
+    for (int o = 1; o < 32; o <<= 1) {
+      const int v = __shfl_up_sync(MV_FULL, incl, o);
+      if (lane >= o) incl += v;
+    }
+    const int excl = incl - cnt;
+    const int T = __shfl_sync(MV_FULL, incl, 31);
+    for (int e0 = 0; e0 < T; e0 += 32) {
+      const int e = e0 + lane;
+      int lo = 0;
+#pragma unroll
+      for (int step = 16; step > 0; step >>= 1) {
+        const int ex = __shfl_sync(MV_FULL, excl, (lo + step) & 31);
+        if (lo + step < 32 && ex <= e) lo += step;
+      }
+      const int64_t addr = __shfl_sync(MV_FULL, off, lo) + (e - __shfl_sync(MV_FULL, excl, lo));
+      const uint64_t key = e < T ? part[addr] : MV_KEY_PAD;
+      const bool band = key != MV_KEY_PAD && key2f((uint32_t)(key >> 32)) <= bound;
+      uint64_t nk = MV_KEY_PAD;
+      uint32_t m = __ballot_sync(MV_FULL, band);
+      while (m) {
+        const int src = __ffs(m) - 1;
+        m &= m - 1;
+        const uint32_t rk = __shfl_sync(MV_FULL, (uint32_t)key, src);
+        const float4* x = reinterpret_cast<const float4*>(payload + (int64_t)__ldg(row_of_rank + rk) * dpad);
+        double acc = 0.0;
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          if (4 * (lane + 32 * u) < dpad) {
+            const float4 xv = __ldg(x + lane + 32 * u);
+            if (l2) {
+              const double a = (double)qr[u].x - xv.x, b = (double)qr[u].y - xv.y;
+              const double c = (double)qr[u].z - xv.z, d = (double)qr[u].w - xv.w;
+              acc = fma(a, a, acc); acc = fma(b, b, acc); acc = fma(c, c, acc); acc = fma(d, d, acc);
+            } else {
+              acc = fma((double)qr[u].x, (double)xv.x, acc); acc = fma((double)qr[u].y, (double)xv.y, acc);
+              acc = fma((double)qr[u].z, (double)xv.z, acc); acc = fma((double)qr[u].w, (double)xv.w, acc);
+            }
+          }
+        }
+        for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(MV_FULL, acc, o);
+        if (lane == src) nk = ((uint64_t)f2key(l2 ? (float)acc : (float)(-acc)) << 32) | rk;
+      }
+      if (e < T) part[addr] = nk;
+    }
+  }
+}
+
+cudaError_t launch_rekey(const int64_t* poff, const int32_t* pcnt, uint64_t* part, int64_t nq, int npb,
+                         const uint64_t* tau2, const float* qerr, int metric, const float* qpad, int dpad,
+                         const float* payload, const uint32_t* row_of_rank, const int* gate, cudaStream_t st) {
+  if (nq == 0) return cudaSuccess;
+  if (dpad > 512 || dpad % 4) return cudaErrorInvalidValue;
+  k_rekey<<<(unsigned)((nq * 32 + 255) / 256), 256, 0, st>>>(poff, pcnt, part, nq, npb, tau2, qerr, metric, qpad, dpad,
+                                                            payload, row_of_rank, gate);
+  return cudaGetLastError();
 }
 
 // ------------------------------------------------------------------------------------------

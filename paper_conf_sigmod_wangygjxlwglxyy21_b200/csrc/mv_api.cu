@@ -1,14 +1,15 @@
-// mv_api.cu -- the C ABI of include/mv.h: index state, validation, host-pointer staging, and the
-// search pipeline a1 -> a2/a3 -> a4 -> a5/a6 -> a7 enqueued on the caller's stream.
+// mv_api.cu -- the C ABI of include/mv.h: index state, validation, memory (caller allocator or
+// stream-ordered CUDA pools), host-pointer staging, and the search pipeline
+// a1 -> a2/a3 -> a4 -> a5/a6 -> (FLAT filter mode: exact re-scoring) -> a7, enqueued on the
+// caller's stream in query chunks that fit the workspace budget.
 #include <cub/device/device_radix_sort.cuh>
 
 #include <cmath>
 #include <cstdarg>
-#include <cstdlib>
 #include <cstdio>
 #include <cstring>
-#include <string>
 #include <functional>
+#include <string>
 #include <vector>
 
 #include "mv_internal.cuh"
@@ -19,11 +20,12 @@ using namespace mv;
 struct mv_index {
   int d = 0, dpad = 0, metric = 0, type = 0, nlist = 0, device = 0;
   bool has_centroids = false, has_sq8 = false;
+  mv_allocator alloc{};         // caller allocator (alloc.alloc == NULL: CUDA's own)
+  Options opt;
   float* cpad = nullptr;    // nlist x dpad
   float* cnorm = nullptr;   // nlist
   float* chl = nullptr;     // [2][nlist][dpad] tf32 hi / lo planes of the centroids (tcgen05 coarse)
   CUtensorMap cmap;
-  bool cmap_ok = false;
   float* vmin = nullptr;    // dpad (zero padded)
   float* vdiff = nullptr;   // dpad (zero padded)
   float* sq8_t = nullptr;   // 256: (c + 0.5f) / 255.f
@@ -37,15 +39,16 @@ struct mv_index {
   int64_t* ids = nullptr;       // ntotal, storage order
   uint32_t* rank = nullptr;     // ntotal: position of (id, row) in sorted order
   int64_t* sorted_ids = nullptr;  // ntotal: ids in (id, row) order
-  // tensor-core scan state (rebuilt by every add)
-  XMaps xm;                 // payload tensor maps: 128/64/32/16-row boxes
-  bool xmap_ok = false;
-  bool tf32_exact = true;   // FLAT: every stored value exactly representable in tf32
+  uint32_t* row_of_rank = nullptr;  // FLAT: storage row of each rank (exact re-scoring)
+  double xmax2 = 0.0;           // FLAT: max ||x||^2 over the stored rows (filter-mode error bound)
+  XMaps xm;                     // payload tensor maps: 128/64/32/16-row boxes (rebuilt by every add)
+  bool tf32_exact = true;       // FLAT: every stored value exactly representable in tf32
   const char* last_scan = "none";
   const char* last_coarse = "none";
+  int64_t last_chunks = 0;      // query chunks of the last search (workspace budget)
   // profiling
   bool prof = false;
-  std::vector<cudaEvent_t> ev;   // kProfStages + 1 events per profiled search
+  std::vector<cudaEvent_t> ev;   // kProfStages + 1 events per profiled search chunk
   int64_t prof_searches = 0, launches = 0;
 };
 
@@ -63,17 +66,22 @@ mv_status fail(mv_status s, const char* fmt, ...) {
   return s;
 }
 
-#define CK(x)                                                                          \
-  do {                                                                                 \
-    cudaError_t _e = (x);                                                              \
-    if (_e != cudaSuccess) return fail(MV_ECUDA, "%s: %s", #x, cudaGetErrorString(_e)); \
+mv_status from_cuda(cudaError_t e, const char* what) {
+  cudaGetLastError();
+  return fail(e == cudaErrorMemoryAllocation ? MV_ENOMEM : MV_ECUDA, "%s: %s", what, cudaGetErrorString(e));
+}
+
+#define CK(x)                                         \
+  do {                                                \
+    cudaError_t _e = (x);                             \
+    if (_e != cudaSuccess) return from_cuda(_e, #x);  \
   } while (0)
 
 struct DeviceGuard {
   int prev = -1;
   explicit DeviceGuard(int dev) {
     cudaGetDevice(&prev);
-    if (prev != dev) cudaSetDevice(dev);
+    if (dev >= 0 && prev != dev) cudaSetDevice(dev);
   }
   ~DeviceGuard() {
     int cur = -1;
@@ -92,19 +100,57 @@ bool is_host_ptr(const void* p) {
   return at.type == cudaMemoryTypeHost || at.type == cudaMemoryTypeUnregistered;
 }
 
-// Stream-ordered scratch allocations released at scope exit.
+// Long-lived index storage: the caller's allocator, else cudaMalloc.
+void* mem_alloc(const mv_index* ix, size_t bytes, cudaStream_t st) {
+  if (ix->alloc.alloc) return ix->alloc.alloc(bytes, st, ix->alloc.ctx);
+  void* p = nullptr;
+  if (cudaMalloc(&p, bytes) != cudaSuccess) {
+    cudaGetLastError();
+    return nullptr;
+  }
+  return p;
+}
+void mem_free(const mv_index* ix, void* p, cudaStream_t st) {
+  if (!p) return;
+  if (ix->alloc.alloc) ix->alloc.free(p, st, ix->alloc.ctx);
+  else cudaFree(p);
+}
+
+// Per-call scratch, released (stream-ordered) at scope exit.  With a caller allocator it is an
+// arena of >= 16 MB blocks taken from the allocator on the call's stream (a handful of callbacks
+// per search); otherwise stream-ordered cudaMallocAsync from the device pool.
 struct Scratch {
+  const mv_index* ix;
   cudaStream_t st;
   std::vector<void*> ptrs;
-  explicit Scratch(cudaStream_t s) : st(s) {}
+  char* cur = nullptr;
+  size_t left = 0;
+  Scratch(const mv_index* i, cudaStream_t s) : ix(i), st(s) {}
   ~Scratch() {
-    for (void* p : ptrs) cudaFreeAsync(p, st);
+    for (void* p : ptrs) {
+      if (ix && ix->alloc.alloc) ix->alloc.free(p, st, ix->alloc.ctx);
+      else cudaFreeAsync(p, st);
+    }
   }
   template <typename T>
   cudaError_t alloc(T** p, size_t n) {
     *p = nullptr;
-    if (n == 0) n = 1;
-    cudaError_t e = cudaMallocAsync(reinterpret_cast<void**>(p), n * sizeof(T), st);
+    size_t bytes = (std::max<size_t>(n, 1) * sizeof(T) + 255) & ~(size_t)255;
+    if (ix && ix->alloc.alloc) {
+      if (bytes > left) {
+        const size_t c = std::max<size_t>(bytes, (size_t)16 << 20);
+        void* q = ix->alloc.alloc(c, st, ix->alloc.ctx);
+        if (!q) return cudaErrorMemoryAllocation;
+        ptrs.push_back(q);
+        cur = static_cast<char*>(q);
+        left = c;
+      }
+      *p = reinterpret_cast<T*>(cur);
+      cur += bytes;
+      left -= bytes;
+      return cudaSuccess;
+    }
+    cudaError_t e = cudaMallocAsync(reinterpret_cast<void**>(p), bytes, st);
     if (e == cudaSuccess) ptrs.push_back(*p);
     return e;
   }
@@ -146,51 +192,63 @@ void prof_mark(mv_index* ix, cudaStream_t st) {
 }
 
 void free_storage(mv_index* ix) {
-  cudaFree(ix->payload);
-  cudaFree(ix->norms);
-  cudaFree(ix->ids);
-  cudaFree(ix->rank);
-  cudaFree(ix->sorted_ids);
+  mem_free(ix, ix->payload, nullptr);
+  mem_free(ix, ix->norms, nullptr);
+  mem_free(ix, ix->ids, nullptr);
+  mem_free(ix, ix->rank, nullptr);
+  mem_free(ix, ix->sorted_ids, nullptr);
+  mem_free(ix, ix->row_of_rank, nullptr);
   ix->payload = nullptr;
   ix->norms = nullptr;
   ix->ids = nullptr;
   ix->rank = nullptr;
   ix->sorted_ids = nullptr;
+  ix->row_of_rank = nullptr;
 }
-}  // namespace
 
-// a2 + a3: tcgen05 coarse with fused top-nprobe when the shapes fit, else the SIMT kernel
-static cudaError_t run_coarse(mv_index* ix, const float* qpad, const float* qhl, const int* qlo_any, int64_t nq,
-                              int npb, int32_t* P, Scratch& s, cudaStream_t st) {
-  CoarseParams cp;
-  const char* force = getenv("MV_FORCE_SIMT");
+int device_sms() {
   int dev = 0, nsm = kNumSMs;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
-  if (npb < ix->nlist && ix->cmap_ok && !(force && force[0] == '1') &&
-      coarse_tc_plan(ix->dpad, npb, nq, ix->nlist, nsm, cp) && nq <= 0x7fffffffLL - cp.nqb) {
-    CUtensorMap qmap;
-    if (make_tmap_2d(&qmap, qhl, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, (uint64_t)ix->dpad, 2 * (uint64_t)nq,
-                     (uint64_t)ix->dpad * 4, 32, (uint32_t)cp.nqb, CU_TENSOR_MAP_SWIZZLE_128B)) {
-      cp.nq = nq;
-      cp.nlist = ix->nlist;
-      cp.metric = ix->metric;
-      cp.cnorm = ix->cnorm;
-      cp.probes = P;
-      cp.lds = (ix->nlist + 3) & ~3;
-      cp.ldg = ((ix->nlist + 127) / 128) * 4;
-      cp.qlo_any = qlo_any;
-      cudaError_t e = s.alloc(&cp.S, (size_t)nq * cp.lds);
-      if (e == cudaSuccess) e = s.alloc(&cp.G, (size_t)nq * cp.ldg);
-      if (e != cudaSuccess) return e;
-      const char* cdbg = getenv("MV_COARSE_DEBUG");
-      cp.dbg = (cdbg && npb > 1) ? atoi(cdbg) : 0;  // never on the add path's assignment (npb = 1)
-      ix->last_coarse = "tcgen05.tf32";
-      return launch_coarse_tc(&ix->cmap, &qmap, cp, nq, st);
-    }
+  return nsm;
+}
+}  // namespace
+
+// a2 + a3: tcgen05 coarse GEMM + per-query top-nprobe; every bucket (id order) when npb >= nlist
+static cudaError_t run_coarse(mv_index* ix, const float* qhl, const int* qlo_any, int64_t nq, int npb, int32_t* P,
+                              Scratch& s, cudaStream_t st) {
+  if (npb >= ix->nlist) {
+    ix->last_coarse = "all-lists";
+    return launch_all_lists(nq, ix->nlist, P, st);
   }
-  ix->last_coarse = "simt";
-  return launch_coarse(qpad, nq, ix->dpad, ix->cpad, ix->cnorm, ix->nlist, ix->metric, npb, P, st);
+  CoarseParams cp;
+  if (!coarse_tc_plan(ix->dpad, npb, nq, ix->nlist, device_sms(), ix->opt, cp)) return cudaErrorInvalidConfiguration;
+  CUtensorMap qmap;
+  if (!make_tmap_2d(&qmap, qhl, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, (uint64_t)ix->dpad, 2 * (uint64_t)nq,
+                    (uint64_t)ix->dpad * 4, 32, (uint32_t)cp.nqb, CU_TENSOR_MAP_SWIZZLE_128B))
+    return cudaErrorInvalidValue;
+  cp.nq = nq;
+  cp.nlist = ix->nlist;
+  cp.metric = ix->metric;
+  cp.cnorm = ix->cnorm;
+  cp.probes = P;
+  cp.lds = (ix->nlist + 3) & ~3;
+  cp.ldg = ((ix->nlist + 127) / 128) * 4;
+  cp.qlo_any = qlo_any;
+  cudaError_t e = s.alloc(&cp.S, (size_t)nq * cp.lds);
+  if (e == cudaSuccess) e = s.alloc(&cp.G, (size_t)nq * cp.ldg);
+  if (e != cudaSuccess) return e;
+  ix->last_coarse = "tcgen05.tf32";
+  return launch_coarse_tc(&ix->cmap, &qmap, cp, nq, st);
+}
+
+// Scratch bytes per query of one search chunk (an upper bound used to size the chunks)
+static int64_t search_bytes_per_query(const mv_index* ix, int npb, int k) {
+  const int64_t cand = ix->top_len_prefix[std::min<size_t>(npb, ix->top_len_prefix.size() - 1)];
+  const int64_t need = std::max<int64_t>(2 * (int64_t)k, k + 32);
+  const int64_t seed = std::min<int64_t>(65536, std::max<int64_t>(need, 4096)) + 4096;
+  const int64_t coarse = npb < ix->nlist ? 4 * (int64_t)((ix->nlist + 3) & ~3) + (int64_t)ix->nlist / 8 : 0;
+  return 8 * (cand + seed) + coarse + 48 * (int64_t)npb + 32 * (int64_t)ix->dpad + 64;
 }
 
 // ------------------------------------------------------------------------------------------
@@ -198,23 +256,27 @@ extern "C" {
 
 const char* mv_last_error(void) { return g_err.c_str(); }
 
-const char* mv_version(void) { return "libmv 0.1 (sm_100a; IVF_FLAT/IVF_SQ8; L2/IP)"; }
+const char* mv_version(void) { return "libmv 0.2 (sm_100a; IVF_FLAT/IVF_SQ8; L2/IP)"; }
 
 int64_t mv_index_ntotal(const mv_index* ix) { return ix ? ix->ntotal : 0; }
 
-mv_status mv_index_create(int32_t d, mv_metric metric, mv_type type, int32_t nlist, int32_t device, mv_index** out) {
+mv_status mv_index_create(int32_t d, mv_metric metric, mv_type type, int32_t nlist, int32_t device,
+                          const mv_allocator* alloc, mv_index** out) {
   if (!out) return fail(MV_EINVAL, "out is NULL");
   *out = nullptr;
-  if (d < 1 || d > 4096) return fail(MV_EINVAL, "d must be in [1, 4096] (got %d)", d);
+  if (d < 1 || d > kMaxD) return fail(MV_EINVAL, "d must be in [1, %d] (got %d)", kMaxD, d);
   if (metric != MV_L2 && metric != MV_IP) return fail(MV_EINVAL, "unknown metric %d", (int)metric);
   if (type != MV_IVF_FLAT && type != MV_IVF_SQ8) return fail(MV_EINVAL, "unknown index type %d", (int)type);
   if (nlist < 1) return fail(MV_EINVAL, "nlist must be >= 1 (got %d)", nlist);
+  if (alloc && (alloc->alloc == nullptr) != (alloc->free == nullptr))
+    return fail(MV_EINVAL, "allocator: alloc and free must both be set");
   int ndev = 0;
   CK(cudaGetDeviceCount(&ndev));
   if (device < 0 || device >= ndev) return fail(MV_EINVAL, "device %d out of range (%d devices)", device, ndev);
   DeviceGuard g(device);
   set_pool_threshold(device);
   mv_index* ix = new mv_index();
+  if (alloc) ix->alloc = *alloc;
   ix->d = d;
   ix->dpad = (d + 31) / 32 * 32;
   ix->metric = metric;
@@ -223,13 +285,15 @@ mv_status mv_index_create(int32_t d, mv_metric metric, mv_type type, int32_t nli
   ix->device = device;
   ix->h_list_off.assign(nlist + 1, 0);
   ix->top_len_prefix.assign(nlist + 1, 0);
-  cudaError_t e = cudaMalloc(&ix->list_off, sizeof(int64_t) * (nlist + 1));
+  bool ok = (ix->list_off = (int64_t*)mem_alloc(ix, sizeof(int64_t) * (nlist + 1), nullptr)) &&
+            (ix->cpad = (float*)mem_alloc(ix, sizeof(float) * (size_t)nlist * ix->dpad, nullptr)) &&
+            (ix->cnorm = (float*)mem_alloc(ix, sizeof(float) * nlist, nullptr)) &&
+            (ix->chl = (float*)mem_alloc(ix, sizeof(float) * 2 * (size_t)nlist * ix->dpad, nullptr)) &&
+            (ix->vmin = (float*)mem_alloc(ix, sizeof(float) * ix->dpad, nullptr)) &&
+            (ix->vdiff = (float*)mem_alloc(ix, sizeof(float) * ix->dpad, nullptr)) &&
+            (ix->sq8_t = (float*)mem_alloc(ix, sizeof(float) * 256, nullptr));
+  cudaError_t e = ok ? cudaSuccess : cudaErrorMemoryAllocation;
   if (e == cudaSuccess) e = cudaMemset(ix->list_off, 0, sizeof(int64_t) * (nlist + 1));
-  if (e == cudaSuccess) e = cudaMalloc(&ix->cpad, sizeof(float) * (size_t)nlist * ix->dpad);
-  if (e == cudaSuccess) e = cudaMalloc(&ix->cnorm, sizeof(float) * nlist);
-  if (e == cudaSuccess) e = cudaMalloc(&ix->vmin, sizeof(float) * ix->dpad);
-  if (e == cudaSuccess) e = cudaMalloc(&ix->vdiff, sizeof(float) * ix->dpad);
-  if (e == cudaSuccess) e = cudaMalloc(&ix->sq8_t, sizeof(float) * 256);
   if (e == cudaSuccess) {
     float t[256];
     for (int c = 0; c < 256; ++c) t[c] = ((float)c + 0.5f) / 255.0f;  // oracle.sq8_decode's first two ops
@@ -239,9 +303,28 @@ mv_status mv_index_create(int32_t d, mv_metric metric, mv_type type, int32_t nli
   if (e == cudaSuccess) e = cudaMemset(ix->vdiff, 0, sizeof(float) * ix->dpad);
   if (e != cudaSuccess) {
     mv_index_destroy(ix);
-    return fail(e == cudaErrorMemoryAllocation ? MV_ENOMEM : MV_ECUDA, "create: %s", cudaGetErrorString(e));
+    return from_cuda(e, "create");
   }
   *out = ix;
+  return MV_OK;
+}
+
+mv_status mv_index_set_option(mv_index* ix, const char* name, int64_t value) {
+  if (!ix || !name) return fail(MV_EINVAL, "null argument");
+  if (value < 0) return fail(MV_EINVAL, "option %s: value must be >= 0", name);
+  Options& o = ix->opt;
+  const std::string n(name);
+  if (n == "seeding") o.seeding = value != 0;
+  else if (n == "need") o.need = value;
+  else if (n == "capa") o.capa = value;
+  else if (n == "sq8_qc") o.sq8_qc = (int)std::min<int64_t>(value, 64);
+  else if (n == "flat_qc") o.flat_qc = (int)std::min<int64_t>(value, 96);
+  else if (n == "coarse_nqb") o.coarse_nqb = (int)std::min<int64_t>(value, 128);
+  else if (n == "coarse_cs") o.coarse_cs = (int)std::min<int64_t>(value, 64);
+  else if (n == "coarse_epi") o.coarse_epi = (int)std::min<int64_t>(value, 16);
+  else if (n == "coarse_nacc") o.coarse_nacc = (int)std::min<int64_t>(value, 4);
+  else if (n == "workspace_bytes") o.workspace = value;
+  else return fail(MV_EINVAL, "unknown option '%s'", name);
   return MV_OK;
 }
 
@@ -251,13 +334,13 @@ void mv_index_destroy(mv_index* ix) {
   cudaDeviceSynchronize();
   free_storage(ix);
   for (cudaEvent_t e : ix->ev) cudaEventDestroy(e);
-  cudaFree(ix->list_off);
-  cudaFree(ix->cpad);
-  cudaFree(ix->cnorm);
-  cudaFree(ix->chl);
-  cudaFree(ix->vmin);
-  cudaFree(ix->vdiff);
-  cudaFree(ix->sq8_t);
+  mem_free(ix, ix->list_off, nullptr);
+  mem_free(ix, ix->cpad, nullptr);
+  mem_free(ix, ix->cnorm, nullptr);
+  mem_free(ix, ix->chl, nullptr);
+  mem_free(ix, ix->vmin, nullptr);
+  mem_free(ix, ix->vdiff, nullptr);
+  mem_free(ix, ix->sq8_t, nullptr);
   delete ix;
 }
 
@@ -266,16 +349,16 @@ mv_status mv_index_set_centroids(mv_index* ix, const float* centroids) {
   if (ix->ntotal > 0) return fail(MV_ESTATE, "centroids cannot change after vectors were added");
   DeviceGuard g(ix->device);
   cudaStream_t st = 0;
-  Scratch s(st);
+  Scratch s(ix, st);
   bool staged;
   const float* c;
   CK(stage_in(s, centroids, (size_t)ix->nlist * ix->d, &c, &staged));
   CK(launch_centroid_prep(c, ix->nlist, ix->d, ix->dpad, ix->cpad, ix->cnorm, st));
-  if (!ix->chl) CK(cudaMalloc(&ix->chl, sizeof(float) * 2 * (size_t)ix->nlist * ix->dpad));
   CK(launch_hilo(c, ix->nlist, ix->d, ix->dpad, ix->chl, nullptr, st));
   CK(cudaStreamSynchronize(st));
-  ix->cmap_ok = make_tmap_2d(&ix->cmap, ix->chl, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, (uint64_t)ix->dpad,
-                             2 * (uint64_t)ix->nlist, (uint64_t)ix->dpad * 4, 32, 128, CU_TENSOR_MAP_SWIZZLE_128B);
+  if (!make_tmap_2d(&ix->cmap, ix->chl, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, (uint64_t)ix->dpad, 2 * (uint64_t)ix->nlist,
+                    (uint64_t)ix->dpad * 4, 32, 128, CU_TENSOR_MAP_SWIZZLE_128B))
+    return fail(MV_ECUDA, "set_centroids: cannot encode the centroid tensor map");
   ix->has_centroids = true;
   return MV_OK;
 }
@@ -287,7 +370,7 @@ mv_status mv_index_train_sq8(mv_index* ix, const float* sample, int64_t n) {
   if (ix->ntotal > 0) return fail(MV_ESTATE, "SQ8 parameters cannot change after vectors were added");
   DeviceGuard g(ix->device);
   cudaStream_t st = 0;
-  Scratch s(st);
+  Scratch s(ix, st);
   bool staged;
   const float* x;
   CK(stage_in(s, sample, (size_t)n * ix->d, &x, &staged));
@@ -330,10 +413,10 @@ mv_status mv_index_add(mv_index* ix, const float* vectors, const int64_t* ids, i
   if (!ix->has_centroids) return fail(MV_ESTATE, "add before set_centroids");
   if (ix->type == MV_IVF_SQ8 && !ix->has_sq8) return fail(MV_ESTATE, "add on SQ8 index before train_sq8/set_sq8");
   if (n > 0x7fffffffLL) return fail(MV_EINVAL, "one add call takes at most 2^31-1 vectors");
-  if (ix->ntotal + n > 0xffffffffLL) return fail(MV_EINVAL, "an index holds at most 2^32-1 vectors");
+  if (ix->ntotal + n > 0x7fffffffLL) return fail(MV_EINVAL, "an index holds at most 2^31-1 vectors");
   DeviceGuard g(ix->device);
   cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
-  Scratch s(st);
+  Scratch s(ix, st);
   bool sv, si;
   const float* x;
   const int64_t* idv;
@@ -362,25 +445,20 @@ mv_status mv_index_add(mv_index* ix, const float* vectors, const int64_t* ids, i
   CK(s.alloc(&slist, (size_t)n));
   CK(s.alloc(&sizes, nlist));
   CK(s.alloc(&new_off, nlist + 1));
-  // a0: assignment I(v) = closest centroid (the coarse kernel with nprobe = 1)
+  // a0: assignment I(v) = closest centroid -- the tensor-core coarse step with nprobe = 1, in row
+  // blocks whose score matrix stays <= 1 GB
   CK(launch_query_prep(x, n, ix->d, dpad, xpad, xnorm, st));
-  // on the tensor cores in row blocks (each block's score matrix <= 1 GB), else SIMT
   {
     const int64_t lds = (nlist + 3) & ~3;
     const int64_t sub = std::min<int64_t>(n, std::max<int64_t>(4096, (int64_t(1) << 28) / lds));
-    bool done = false;
-    if (nlist > 1 && ix->cmap_ok) {
-      float* qhl;
-      CK(s.alloc(&qhl, (size_t)2 * sub * dpad));
-      for (int64_t r0 = 0; r0 < n; r0 += sub) {
-        const int64_t m = std::min(sub, n - r0);
-        Scratch sb(st);  // the block's score matrix, freed (stream-ordered) before the next block
-        CK(launch_hilo(x + r0 * ix->d, m, ix->d, dpad, qhl, nullptr, st));
-        CK(run_coarse(ix, xpad + r0 * dpad, qhl, nullptr, m, 1, lists + r0, sb, st));
-      }
-      done = true;
+    float* qhl;
+    CK(s.alloc(&qhl, (size_t)2 * sub * dpad));
+    for (int64_t r0 = 0; r0 < n; r0 += sub) {
+      const int64_t m = std::min(sub, n - r0);
+      Scratch sb(ix, st);  // the block's score matrix, freed (stream-ordered) before the next block
+      CK(launch_hilo(x + r0 * ix->d, m, ix->d, dpad, qhl, nullptr, st));
+      CK(run_coarse(ix, qhl, nullptr, m, 1, lists + r0, sb, st));
     }
-    if (!done) CK(launch_coarse(xpad, n, dpad, ix->cpad, ix->cnorm, nlist, ix->metric, 1, lists, st));
   }
   CK(cudaMemsetAsync(cnt, 0, sizeof(int32_t) * nlist, st));
   CK(launch_count_lists(lists, n, cnt, st));
@@ -392,8 +470,8 @@ mv_status mv_index_add(mv_index* ix, const float* vectors, const int64_t* ids, i
   size_t tmp_bytes = 0;
   CK(cub::DeviceRadixSort::SortPairs(nullptr, tmp_bytes, (const uint32_t*)lists, (uint32_t*)slist, idx, sidx, (int)n, 0,
                                      endbit, st));
-  void* tmp;
-  CK(s.alloc(reinterpret_cast<uint8_t**>(&tmp), tmp_bytes));
+  uint8_t* tmp;
+  CK(s.alloc(&tmp, tmp_bytes));
   CK(cub::DeviceRadixSort::SortPairs(tmp, tmp_bytes, (const uint32_t*)lists, (uint32_t*)slist, idx, sidx, (int)n, 0,
                                      endbit, st));
   CK(launch_new_sizes(cnt, nlist, ix->list_off, sizes, st));
@@ -401,30 +479,29 @@ mv_status mv_index_add(mv_index* ix, const float* vectors, const int64_t* ids, i
 
   const int64_t ntot = ix->ntotal + n;
   const size_t esize = ix->type == MV_IVF_FLAT ? 4 : 1;
-  void* payload = nullptr;
-  double* norms = nullptr;
-  int64_t *nids = nullptr, *sorted_ids = nullptr;
-  uint32_t* rank = nullptr;
   // per-row side arrays carry kSidePad zeroed tail elements: the scan bulk-copies 16-B aligned
   // supersets of 128-row tiles
   constexpr int64_t kSidePad = 256;
-  cudaError_t e = cudaMalloc(&payload, (size_t)ntot * dpad * esize);
-  if (e == cudaSuccess) e = cudaMalloc(&norms, sizeof(double) * (ntot + kSidePad));
-  if (e == cudaSuccess) e = cudaMalloc(&nids, sizeof(int64_t) * (ntot + kSidePad));
-  if (e == cudaSuccess) e = cudaMalloc(&rank, sizeof(uint32_t) * (ntot + kSidePad));
-  if (e == cudaSuccess) e = cudaMemsetAsync(norms + ntot, 0, sizeof(double) * kSidePad, st);
-  if (e == cudaSuccess) e = cudaMemsetAsync(nids + ntot, 0, sizeof(int64_t) * kSidePad, st);
-  if (e == cudaSuccess) e = cudaMemsetAsync(rank + ntot, 0, sizeof(uint32_t) * kSidePad, st);
-  if (e == cudaSuccess) e = cudaMalloc(&sorted_ids, sizeof(int64_t) * ntot);
-  if (e != cudaSuccess) {
-    cudaFree(payload); cudaFree(norms); cudaFree(nids); cudaFree(rank); cudaFree(sorted_ids);
-    cudaGetLastError();
+  mv_index nx;  // the new storage (only the pointers are used)
+  nx.alloc = ix->alloc;
+  nx.payload = mem_alloc(ix, (size_t)ntot * dpad * esize, st);
+  nx.norms = (double*)mem_alloc(ix, sizeof(double) * (ntot + kSidePad), st);
+  nx.ids = (int64_t*)mem_alloc(ix, sizeof(int64_t) * (ntot + kSidePad), st);
+  nx.rank = (uint32_t*)mem_alloc(ix, sizeof(uint32_t) * (ntot + kSidePad), st);
+  nx.sorted_ids = (int64_t*)mem_alloc(ix, sizeof(int64_t) * ntot, st);
+  if (ix->type == MV_IVF_FLAT) nx.row_of_rank = (uint32_t*)mem_alloc(ix, sizeof(uint32_t) * ntot, st);
+  if (!nx.payload || !nx.norms || !nx.ids || !nx.rank || !nx.sorted_ids ||
+      (ix->type == MV_IVF_FLAT && !nx.row_of_rank)) {
+    free_storage(&nx);
     return fail(MV_ENOMEM, "add: cannot allocate storage for %lld vectors", (long long)ntot);
   }
-  CK(launch_move_old(ix->type, dpad, nlist, ix->list_off, new_off, ix->payload, ix->norms, ix->ids, ix->ntotal, payload,
-                     norms, nids, st));
-  CK(launch_store_rows(ix->type, ix->metric, xpad, idv, sidx, slist, n, dpad, new_off, ix->list_off, addoff, payload,
-                       norms, nids, ix->vmin, ix->vdiff, ix->sq8_t, st));
+  CK(cudaMemsetAsync(nx.norms + ntot, 0, sizeof(double) * kSidePad, st));
+  CK(cudaMemsetAsync(nx.ids + ntot, 0, sizeof(int64_t) * kSidePad, st));
+  CK(cudaMemsetAsync(nx.rank + ntot, 0, sizeof(uint32_t) * kSidePad, st));
+  CK(launch_move_old(ix->type, dpad, nlist, ix->list_off, new_off, ix->payload, ix->norms, ix->ids, ix->ntotal,
+                     nx.payload, nx.norms, nx.ids, st));
+  CK(launch_store_rows(ix->type, ix->metric, xpad, idv, sidx, slist, n, dpad, new_off, ix->list_off, addoff,
+                       nx.payload, nx.norms, nx.ids, ix->vmin, ix->vdiff, ix->sq8_t, st));
   // id ranks: stable radix sort of (id) over storage rows -> (id, row) order
   uint64_t *keys, *skeys;
   uint32_t *vals, *svals;
@@ -432,38 +509,52 @@ mv_status mv_index_add(mv_index* ix, const float* vectors, const int64_t* ids, i
   CK(s.alloc(&skeys, (size_t)ntot));
   CK(s.alloc(&vals, (size_t)ntot));
   CK(s.alloc(&svals, (size_t)ntot));
-  CK(launch_id_keys(nids, ntot, keys, vals, st));
+  CK(launch_id_keys(nx.ids, ntot, keys, vals, st));
   size_t tmp2 = 0;
   CK(cub::DeviceRadixSort::SortPairs(nullptr, tmp2, keys, skeys, vals, svals, (int64_t)ntot, 0, 64, st));
-  void* t2;
-  CK(s.alloc(reinterpret_cast<uint8_t**>(&t2), tmp2));
+  uint8_t* t2;
+  CK(s.alloc(&t2, tmp2));
   CK(cub::DeviceRadixSort::SortPairs(t2, tmp2, keys, skeys, vals, svals, (int64_t)ntot, 0, 64, st));
-  CK(launch_rank_scatter(skeys, svals, ntot, rank, sorted_ids, st));
+  CK(launch_rank_scatter(skeys, svals, ntot, nx.rank, nx.sorted_ids, nx.row_of_rank, st));
+  unsigned long long* xm;
+  CK(s.alloc(&xm, 1));
+  unsigned long long hxm = 0;
   if (ix->type == MV_IVF_FLAT) {
     CK(cudaMemsetAsync(flag, 0, sizeof(int), st));
     CK(launch_tf32_check(xpad, (int64_t)n * dpad, flag, st));
     CK(cudaMemcpyAsync(&hflag, flag, sizeof(int), cudaMemcpyDeviceToHost, st));
+    CK(cudaMemsetAsync(xm, 0, sizeof(unsigned long long), st));
+    CK(launch_max_f64(nx.norms, ntot, xm, st));
+    CK(cudaMemcpyAsync(&hxm, xm, sizeof(unsigned long long), cudaMemcpyDeviceToHost, st));
   }
   CK(cudaMemcpyAsync(ix->list_off, new_off, sizeof(int64_t) * (nlist + 1), cudaMemcpyDeviceToDevice, st));
   CK(cudaMemcpyAsync(ix->h_list_off.data(), new_off, sizeof(int64_t) * (nlist + 1), cudaMemcpyDeviceToHost, st));
   CK(cudaStreamSynchronize(st));
   free_storage(ix);
-  ix->payload = payload;
-  ix->norms = norms;
-  ix->ids = nids;
-  ix->rank = rank;
-  ix->sorted_ids = sorted_ids;
+  ix->payload = nx.payload;
+  ix->norms = nx.norms;
+  ix->ids = nx.ids;
+  ix->rank = nx.rank;
+  ix->sorted_ids = nx.sorted_ids;
+  ix->row_of_rank = nx.row_of_rank;
+  nx.payload = nx.norms = nullptr;
+  nx.ids = nx.sorted_ids = nullptr;
+  nx.rank = nx.row_of_rank = nullptr;
   ix->ntotal = ntot;
-  if (ix->type == MV_IVF_FLAT && hflag) ix->tf32_exact = false;
-  ix->xmap_ok = ntot <= 0x7fffffffLL;
+  if (ix->type == MV_IVF_FLAT) {
+    if (hflag) ix->tf32_exact = false;
+    double xm2;
+    memcpy(&xm2, &hxm, sizeof xm2);
+    ix->xmax2 = xm2;
+  }
   // one swizzle atom per box row: 128 B (FLAT: 32 fp32; SQ8 when dpad is a multiple of 128), else 32 B
   const bool wide = ix->type == MV_IVF_FLAT || dpad % 128 == 0;
-  for (int i = 0; i < 4 && ix->xmap_ok; ++i)
-    ix->xmap_ok = make_tmap_2d(&ix->xm.m[i], payload,
-                               ix->type == MV_IVF_FLAT ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_UINT8,
-                               (uint64_t)dpad, (uint64_t)ntot, (uint64_t)dpad * esize,
-                               ix->type == MV_IVF_FLAT ? 32 : (wide ? 128 : 32), 128 >> i,
-                               wide ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_32B);
+  for (int i = 0; i < 4; ++i)
+    if (!make_tmap_2d(&ix->xm.m[i], ix->payload,
+                      ix->type == MV_IVF_FLAT ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_UINT8,
+                      (uint64_t)dpad, (uint64_t)ntot, (uint64_t)dpad * esize, ix->type == MV_IVF_FLAT ? 32 : (wide ? 128 : 32),
+                      128 >> i, wide ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_32B))
+      return fail(MV_ECUDA, "add: cannot encode the payload tensor map");
   ix->maxlen = 0;
   std::vector<int64_t> lens(nlist);
   for (int l = 0; l < nlist; ++l) {
@@ -483,10 +574,10 @@ static mv_status validate_search(const mv_index* ix, const float* q, int64_t nq,
   if (k < 1 || k > kMaxK) return fail(MV_EINVAL, "k must be in [1, %d] (got %d)", kMaxK, k);
   if (nprobe < 1) return fail(MV_EINVAL, "nprobe must be >= 1 (got %d)", nprobe);
   const int npb = std::min(nprobe, ix->nlist);
-  if (npb < ix->nlist && npb > 1024) return fail(MV_EINVAL, "nprobe must be <= 1024 or >= nlist (got %d)", nprobe);
+  if (npb < ix->nlist && npb > kMaxNprobe)
+    return fail(MV_EINVAL, "nprobe must be <= %d or >= nlist (got %d)", kMaxNprobe, nprobe);
   if (nq > 0 && (!q || !d || !i)) return fail(MV_EINVAL, "null queries/outputs");
   if (!ix->has_centroids) return fail(MV_ESTATE, "search before set_centroids");
-  if (nq > 0x7fffffffLL / std::max(npb, 1)) return fail(MV_EINVAL, "nq * nprobe must be < 2^31");
   return MV_OK;
 }
 
@@ -497,32 +588,257 @@ mv_status mv_search_probes(mv_index* ix, const float* queries, int64_t nq, int32
   if (nq == 0) return MV_OK;
   DeviceGuard g(ix->device);
   cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
-  Scratch s(st);
   const int npb = std::min(nprobe, ix->nlist);
-  bool sq, sp;
+  bool sq;
+  Scratch s0(ix, st);
   const float* q;
-  CK(stage_in(s, queries, (size_t)nq * ix->d, &q, &sq));
-  sp = is_host_ptr(probes);
-  int32_t* P = probes;
-  if (sp) CK(s.alloc(&P, (size_t)nq * npb));
-  float *qpad, *qnorm;
-  CK(s.alloc(&qpad, (size_t)nq * ix->dpad));
-  CK(s.alloc(&qnorm, (size_t)nq));
-  CK(launch_query_prep(q, nq, ix->d, ix->dpad, qpad, qnorm, st));
-  float* qhl;
-  CK(s.alloc(&qhl, (size_t)2 * nq * ix->dpad));
-  CK(launch_hilo(q, nq, ix->d, ix->dpad, qhl, nullptr, st));
-  CK(run_coarse(ix, qpad, qhl, nullptr, nq, npb, P, s, st));
-  if (sp) {
-    CK(cudaMemcpyAsync(probes, P, sizeof(int32_t) * nq * npb, cudaMemcpyDeviceToHost, st));
-    CK(cudaStreamSynchronize(st));
+  CK(stage_in(s0, queries, (size_t)nq * ix->d, &q, &sq));
+  const bool sp = is_host_ptr(probes);
+  // chunks of queries whose score matrix stays <= 1 GB
+  const int64_t per = 4 * (int64_t)((ix->nlist + 3) & ~3) + 4 * (int64_t)ix->dpad * 2 + 4 * npb + 64;
+  const int64_t chunk = std::max<int64_t>(1, std::min<int64_t>(nq, (int64_t(1) << 30) / per));
+  for (int64_t q0 = 0; q0 < nq; q0 += chunk) {
+    const int64_t m = std::min(chunk, nq - q0);
+    Scratch s(ix, st);
+    int32_t* P = probes + q0 * npb;
+    if (sp) CK(s.alloc(&P, (size_t)m * npb));
+    float* qhl;
+    CK(s.alloc(&qhl, (size_t)2 * m * ix->dpad));
+    CK(launch_hilo(q + q0 * ix->d, m, ix->d, ix->dpad, qhl, nullptr, st));
+    CK(run_coarse(ix, qhl, nullptr, m, npb, P, s, st));
+    if (sp) CK(cudaMemcpyAsync(probes + q0 * npb, P, sizeof(int32_t) * m * npb, cudaMemcpyDeviceToHost, st));
   }
+  if (sp || sq) CK(cudaStreamSynchronize(st));
+  return MV_OK;
+}
+
+// One chunk of queries through the whole pipeline (a1 .. a7).  q: device queries [nq][d];
+// P_in: caller probes [nq][npb] (device) or nullptr; bs: device bitset or nullptr.
+static mv_status search_chunk(mv_index* ix, const float* q, int64_t nq, int32_t k, int npb, const int32_t* P_in,
+                              const uint8_t* bs, int64_t nbits, float* D, int64_t* I, cudaStream_t st) {
+  Scratch s(ix, st);
+  const int nlist = ix->nlist, dpad = ix->dpad;
+  const bool flat = ix->type == MV_IVF_FLAT;
+  // a1 + a2/a3
+  prof_mark(ix, st);
+  float *qpad, *qnorm;
+  int32_t* P;
+  CK(s.alloc(&qpad, (size_t)nq * dpad));
+  CK(s.alloc(&qnorm, (size_t)nq));
+  if (P_in) P = const_cast<int32_t*>(P_in);
+  else CK(s.alloc(&P, (size_t)nq * npb));
+  CK(launch_query_prep(q, nq, ix->d, dpad, qpad, qnorm, st));
+  float* qhl;  // plane-major tf32 hi/lo query planes: coarse B operand and the FLAT scan's query planes
+  CK(s.alloc(&qhl, (size_t)2 * nq * dpad));
+  int* qlo_any;  // does any query need its lo plane (not tf32-exact)?  Decides the FLAT scan shape
+  CK(s.alloc(&qlo_any, 1));
+  CK(cudaMemsetAsync(qlo_any, 0, sizeof(int), st));
+  CK(launch_hilo(q, nq, ix->d, dpad, qhl, qlo_any, st));
+  if (!P_in) CK(run_coarse(ix, qhl, qlo_any, nq, npb, P, s, st));
+  prof_mark(ix, st);
+  // a4 (the work-item shape follows the scan's shared-memory plan)
+  TcScanParams tp;
+  if (!tc_scan_plan(ix->type, dpad, k, (double)nq * npb / std::max(1, nlist), ix->opt, tp))
+    return fail(MV_EINVAL, "search: no tensor-core scan plan fits d = %d", ix->d);
+  const int qchunk = tp.qchunk;
+  const int qchunk_min = tp.qchunk_split;  // FLAT two-plane items
+  int32_t* qcfg;
+  CK(s.alloc(&qcfg, 2));
+  const int64_t npairs = nq * npb;
+  // Seeding (nprobe >= 2): phase A scans the first capA rows of each query's ra[q] nearest lists --
+  // the fewest holding >= need such rows -- and emits all of them; their k-th best key tau_q bounds
+  // the query's final k-th best (k distinct candidates are at or below it), so phase B scans every
+  // probed list and emits only keys <= tau_q.
+  const bool split = npb >= 2 && ix->opt.seeding;
+  int32_t* ra = nullptr;
+  if (split) CK(s.alloc(&ra, (size_t)nq));
+  const int nv = split ? 2 * nlist : nlist;
+  Bucketing b;
+  CK(s.alloc(&b.lcount, nv));
+  CK(s.alloc(&b.boff, nv + 1));
+  CK(s.alloc(&b.bfill, nv));
+  const int64_t nent = split ? 2 * npairs : npairs;  // bucket entries (phase-A entries with seeding)
+  CK(s.alloc(&b.bq, (size_t)nent));
+  CK(s.alloc(&b.wcount, nv));
+  CK(s.alloc(&b.woff, nv + 1));
+  CK(s.alloc(&b.witems, (size_t)(nv + nent / qchunk_min + 1)));
+  CK(s.alloc(&b.witems_unsorted, (size_t)(nv + nent / qchunk_min + 1)));
+  CK(s.alloc(&b.qtot, (size_t)(2 * (nq + 1))));
+  CK(s.alloc(&b.poff, (size_t)nent));
+  CK(s.alloc(&b.pcnt, (size_t)nent));
+  CK(s.alloc(&b.counter, 1));
+  CK(s.alloc(&b.whist, (size_t)kPlanCostBins));
+  CK(s.alloc(&b.bsum, (size_t)(2 * kPlanMaxBlocks)));
+  PlanArgs pa;
+  pa.probes = P; pa.nq = nq; pa.npb = npb; pa.nlist = nlist; pa.k = k;
+  pa.split = split ? 1 : 0; pa.need = std::max<int64_t>(2 * (int64_t)k, k + 32);
+  // Sample size of the seeding phase.  tau_q = the k-th best of `need` candidates is about the
+  // (k N / need)-th best of the query's N candidates, so phase B emits ~k N / need keys.  Phase A
+  // costs ~need rows of payload, an emission ~a fixed number of bytes (the key store, the final
+  // select's reads); balancing the two gives need ~ sqrt(k N c / rowbytes).  c is measured
+  // (session-4 sweep): 32 B for k <= 256; the CTA-per-query select for k > 256 costs
+  // ~26x more per candidate (and falls back to global memory past its stage), c = 832 B.
+  {
+    const double ncand = (double)ix->ntotal * npb / std::max(1, nlist);
+    const double rowb = (double)dpad * (flat ? 4 : 1);
+    const double c = k > 256 ? 832.0 : 32.0;
+    const int64_t bal = (int64_t)std::sqrt((double)k * ncand * c / rowb);
+    pa.need = std::max<int64_t>(pa.need, std::min<int64_t>(bal, 65536));
+  }
+  if (ix->opt.need > 0) pa.need = std::max<int64_t>(2 * (int64_t)k, ix->opt.need);
+  // Rows per list of the sample: ~sqrt(64 need), i.e. the sample spreads over ~sqrt(need / 64)
+  // nearest lists (measured, capA sweep: configs[2] 256 rows 2.85M qps vs whole lists 2.71M;
+  // configs[4] 128 rows best; configs[1] 128 rows vs 64: 16.0M vs 14.7M), at least 128 rows
+  pa.capA = std::max<int64_t>(128, std::min<int64_t>((pa.need + 15) & ~(int64_t)15,
+                                                     ((int64_t)std::sqrt(64.0 * pa.need) + 15) & ~(int64_t)15));
+  if (ix->opt.capa > 0) pa.capA = std::max<int64_t>(16, (ix->opt.capa + 15) & ~15ll);
+  pa.list_off = ix->list_off;
+  // FLAT with tf32-exact stored values: two-plane (hi/lo) items when some query needs its lo plane;
+  // other FLAT data always take one-plane items (the stored side's tf32 error dominates)
+  pa.qlo_any = (flat && ix->tf32_exact) ? qlo_any : nullptr;
+  pa.qc_exact = qchunk; pa.p_exact = flat ? 1 : 4;
+  pa.qc_split = qchunk_min; pa.p_split = flat ? 2 : 4;
+  pa.qcfg = qcfg; pa.ra = ra; pa.b = b;
+  CK(launch_plan(pa, st));
+  prof_mark(ix, st);
+  // candidate regions: the worst case without a device round trip, nq x (the npb longest lists)
+  // (+ the phase-A prefixes: < need + capA rows per query); the chunking bounds it
+  const int64_t tmax = ix->top_len_prefix[std::min<size_t>(npb, ix->top_len_prefix.size() - 1)];
+  int64_t cap = nq * tmax;
+  if (split) cap += nq * std::min<int64_t>(tmax, pa.need + pa.capA);
+  uint8_t* over = nullptr;
+  if (k > 256) CK(s.alloc(&over, (size_t)nq));
+  uint64_t* part;
+  CK(s.alloc(&part, (size_t)max64(cap, 1)));
+  // a5/a6 on the tensor cores
+  uint8_t* qplanes;
+  float *qscale, *qerr = nullptr;
+  double *qa, *qn64;
+  uint64_t* tau;
+  if (!flat) CK(s.alloc(&qplanes, (size_t)nq * 4 * dpad));
+  else qplanes = reinterpret_cast<uint8_t*>(qhl);
+  CK(s.alloc(&qscale, (size_t)nq));
+  CK(s.alloc(&qa, (size_t)nq));
+  CK(s.alloc(&qn64, (size_t)nq));
+  CK(s.alloc(&tau, (size_t)nq));
+  CK(cudaMemsetAsync(tau, 0xff, sizeof(uint64_t) * nq, st));
+  // FLAT filter mode (DESIGN.md §5 "FLAT precision"): the tensor-core badness carries a rigorous
+  // error bound E_q when the stored values (always) or the queries (device flag) are not
+  // tf32-exact; the keys are then re-scored exactly before the final select
+  const bool approx_always = flat && !ix->tf32_exact;
+  const int* gate = approx_always ? nullptr : qlo_any;
+  FlatErr fe{ix->tf32_exact ? 0.0 : 0x1p-10, ix->tf32_exact ? 0x1p-21 : 0x1p-11, ix->xmax2, ix->metric};
+  if (flat) CK(s.alloc(&qerr, (size_t)nq));
+  CK(launch_qplanes(ix->type, qpad, nq, dpad, ix->vmin, ix->vdiff, flat ? nullptr : qplanes, qscale, qa, qn64,
+                    flat ? &fe : nullptr, qerr, st));
+  tp.metric = ix->metric; tp.npb = npb; tp.nq = nq;
+  tp.list_off = ix->list_off; tp.norms = ix->norms; tp.ids = ix->ids; tp.rank = ix->rank;
+  tp.bitset = bs; tp.nbits = bs ? nbits : 0;
+  tp.qplanes = qplanes; tp.qnorm = qn64; tp.qscale = qscale; tp.qa = qa;
+  tp.bq = b.bq; tp.boff = b.boff; tp.witems = b.witems; tp.nlist = nlist; tp.cfg = qcfg;
+  tp.poff = b.poff; tp.pcnt = b.pcnt; tp.part = part; tp.tau = tau;
+  tp.approx_always = approx_always ? 1 : 0; tp.qerr = qerr;
+  tp.prof = nullptr;
+  // phase A (or, without seeding, the whole scan emitting every candidate) ...
+  tp.phase = 0;
+  tp.rowcap = split ? (int)pa.capA : 0x7fffffff;
+  tp.wbeg = nullptr;
+  tp.nwitems = b.woff + nlist;
+  CK(launch_scan_tc(ix->xm, tp, st));
+  prof_mark(ix, st);
+  if (split) {
+    // ... tau_q = k-th best key of phase A (phase A emits < need + capA candidates per query) ...
+    CK(launch_tau_select(b.poff + npairs, b.pcnt + npairs, part, nq, npb, ra, k, tau,
+                         std::min<int64_t>(tmax, pa.need + pa.capA), over, nullptr, st));
+    prof_mark(ix, st);
+    // ... phase B over every probed pair, emitting keys <= tau_q
+    tp.phase = 1;
+    tp.rowcap = 0x7fffffff;
+    tp.wbeg = b.woff + nlist;
+    tp.nwitems = b.woff + 2 * nlist;
+    CK(launch_scan_tc(ix->xm, tp, st));
+  } else {
+    prof_mark(ix, st);
+  }
+  prof_mark(ix, st);
+  if (flat) {
+    // filter mode: t~_q = the k-th best approximate key, then exact re-scoring of the keys within
+    // 2 E_q of it (both skipped on the device when the search is exact: gate = qlo_any == 0)
+    uint64_t* tau2;
+    CK(s.alloc(&tau2, (size_t)nq));
+    CK(cudaMemsetAsync(tau2, 0xff, sizeof(uint64_t) * nq, st));
+    CK(launch_tau_select(b.poff, b.pcnt, part, nq, npb, nullptr, k, tau2, tmax, over, gate, st));
+    CK(launch_rekey(b.poff, b.pcnt, part, nq, npb, tau2, qerr, ix->metric, qpad, dpad,
+                    reinterpret_cast<const float*>(ix->payload), ix->row_of_rank, gate, st));
+    ix->launches += 2;
+  }
+  // a7
+  CK(launch_final_select(b.poff, b.pcnt, part, nq, npb, k, ix->metric, ix->sorted_ids, D, I, tmax, over, st));
+  prof_mark(ix, st);
+  ix->last_scan = flat ? "tcgen05.tf32" : "tcgen05.i8";
+  // prep, hilo, coarse GEMM + probe select, plan, qplanes, scan A (+ tau select, scan B), final select
+  ix->launches += (P_in ? 5 : (npb >= nlist ? 6 : 7)) + (split ? 3 : 1);
   return MV_OK;
 }
 
 static mv_status search_impl(mv_index* ix, const float* queries, int64_t nq, int32_t k, int32_t nprobe,
                              const int32_t* probes_in, const uint8_t* bitset, int64_t nbits, float* distances,
-                             int64_t* out_ids, void* stream);
+                             int64_t* out_ids, void* stream) {
+  mv_status v = validate_search(ix, queries, nq, k, nprobe, distances, out_ids);
+  if (v != MV_OK) return v;
+  if (nbits < 0) return fail(MV_EINVAL, "nbits must be >= 0");
+  if (nq == 0) return MV_OK;
+  if (bitset == nullptr) nbits = 0;
+  DeviceGuard g(ix->device);
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  Scratch s(ix, st);
+  const int npb = std::min(nprobe, ix->nlist);
+  bool sq = false, sb = false, sp = false;
+  const float* q;
+  const uint8_t* bs = nullptr;
+  const int32_t* P = nullptr;
+  CK(stage_in(s, queries, (size_t)nq * ix->d, &q, &sq));
+  if (bitset && nbits > 0) CK(stage_in(s, bitset, (size_t)((nbits + 7) / 8), &bs, &sb));
+  if (probes_in) CK(stage_in(s, probes_in, (size_t)nq * npb, &P, &sp));
+  const bool host_out = is_host_ptr(distances) || is_host_ptr(out_ids);
+  float* D = distances;
+  int64_t* I = out_ids;
+  if (host_out) {
+    CK(s.alloc(&D, (size_t)nq * k));
+    CK(s.alloc(&I, (size_t)nq * k));
+  }
+  if (ix->ntotal == 0) {
+    CK(launch_fill_pad((int64_t)nq * k, ix->metric, D, I, st));
+  } else {
+    // query chunks: each one's scratch (candidate regions, score matrix, ...) within the budget,
+    // and < 2^29 (query, list) pairs (int32 pair ids with the seeding phase's second copy)
+    int64_t budget = ix->opt.workspace;
+    if (budget <= 0) {
+      size_t fr = 0, tot = 0;
+      CK(cudaMemGetInfo(&fr, &tot));
+      budget = (int64_t)(fr / 2);
+    }
+    const int64_t per = search_bytes_per_query(ix, npb, k);
+    int64_t chunk = std::min<int64_t>(nq, std::max<int64_t>(1, budget / std::max<int64_t>(per, 1)));
+    chunk = std::min<int64_t>(chunk, std::max<int64_t>(1, (int64_t(1) << 29) / npb));
+    ix->last_chunks = 0;
+    for (int64_t q0 = 0; q0 < nq; q0 += chunk) {
+      const int64_t m = std::min(chunk, nq - q0);
+      mv_status r = search_chunk(ix, q + q0 * ix->d, m, k, npb, P ? P + q0 * npb : nullptr, bs, nbits,
+                                 D + q0 * k, I + q0 * k, st);
+      if (r != MV_OK) return r;
+      ix->last_chunks++;
+    }
+    if (ix->prof) ix->prof_searches++;
+  }
+  if (host_out) {
+    CK(cudaMemcpyAsync(distances, D, sizeof(float) * nq * k, cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(out_ids, I, sizeof(int64_t) * nq * k, cudaMemcpyDeviceToHost, st));
+  }
+  // host inputs/outputs: the call completes before returning (mv.h)
+  if (host_out || sq || sb || sp) CK(cudaStreamSynchronize(st));
+  return MV_OK;
+}
 
 mv_status mv_search(mv_index* ix, const float* queries, int64_t nq, int32_t k, int32_t nprobe, const uint8_t* bitset,
                     int64_t nbits, float* distances, int64_t* out_ids, void* stream) {
@@ -536,276 +852,22 @@ mv_status mv_search_with_probes(mv_index* ix, const float* queries, int64_t nq, 
   return search_impl(ix, queries, nq, k, nprobe, probes, bitset, nbits, distances, out_ids, stream);
 }
 
-static mv_status search_impl(mv_index* ix, const float* queries, int64_t nq, int32_t k, int32_t nprobe,
-                             const int32_t* probes_in, const uint8_t* bitset, int64_t nbits, float* distances,
-                             int64_t* out_ids, void* stream) {
-  mv_status v = validate_search(ix, queries, nq, k, nprobe, distances, out_ids);
-  if (v != MV_OK) return v;
-  if (nbits < 0) return fail(MV_EINVAL, "nbits must be >= 0");
-  if (nq == 0) return MV_OK;
-  if (bitset == nullptr) nbits = 0;
-  DeviceGuard g(ix->device);
-  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
-  Scratch s(st);
-  const int nlist = ix->nlist, dpad = ix->dpad;
-  const int npb = std::min(nprobe, nlist);
-  bool sq, sb;
-  const float* q;
-  const uint8_t* bs = nullptr;
-  CK(stage_in(s, queries, (size_t)nq * ix->d, &q, &sq));
-  if (bitset && nbits > 0) CK(stage_in(s, bitset, (size_t)((nbits + 7) / 8), &bs, &sb));
-  const bool host_out = is_host_ptr(distances) || is_host_ptr(out_ids);
-  float* D = distances;
-  int64_t* I = out_ids;
-  if (host_out) {
-    CK(s.alloc(&D, (size_t)nq * k));
-    CK(s.alloc(&I, (size_t)nq * k));
-  }
-  if (ix->ntotal == 0) {
-    CK(launch_fill_pad((int64_t)nq * k, ix->metric, D, I, st));
-  } else {
-    // a1 + a2/a3
-    prof_mark(ix, st);
-    float *qpad, *qnorm;
-    int32_t* P;
-    CK(s.alloc(&qpad, (size_t)nq * dpad));
-    CK(s.alloc(&qnorm, (size_t)nq));
-    if (probes_in) {  // caller-supplied probes (staged when on the host): a2/a3 are skipped
-      bool sp;
-      const int32_t* pp;
-      CK(stage_in(s, probes_in, (size_t)nq * npb, &pp, &sp));
-      P = const_cast<int32_t*>(pp);
-    } else {
-      CK(s.alloc(&P, (size_t)nq * npb));
-    }
-    CK(launch_query_prep(q, nq, ix->d, dpad, qpad, qnorm, st));
-    float* qhl;  // plane-major tf32 hi/lo query planes: coarse B operand and the FLAT scan's query planes
-    CK(s.alloc(&qhl, (size_t)2 * nq * dpad));
-    int* qlo_any;  // does any query need its lo plane (not tf32-exact)?  Decides the FLAT scan shape
-    CK(s.alloc(&qlo_any, 1));
-    CK(cudaMemsetAsync(qlo_any, 0, sizeof(int), st));
-    CK(launch_hilo(q, nq, ix->d, dpad, qhl, qlo_any, st));
-    if (!probes_in) CK(run_coarse(ix, qpad, qhl, qlo_any, nq, npb, P, s, st));
-    prof_mark(ix, st);
-    // a4 (work-item size depends on the scan implementation's shared-memory plan)
-    TcScanParams tp;
-    const char* force = getenv("MV_FORCE_SIMT");
-    // MV_SCAN_IMPL=qm selects the queries-as-M FLAT scan (k_scan_qm.cu, experimental)
-    const char* impl = getenv("MV_SCAN_IMPL");
-    const bool use_qm = ix->type == MV_IVF_FLAT && impl && impl[0] == 'q';
-    const bool use_tc = ix->xmap_ok && !(force && force[0] == '1') &&
-                        (ix->type == MV_IVF_SQ8 || ix->tf32_exact) &&
-                        (use_qm ? qm_scan_plan(dpad, k, tp)
-                                : tc_scan_plan(ix->type, dpad, k, (double)nq * npb / std::max(1, nlist), tp));
-    const int qchunk = use_tc ? tp.qchunk
-                              : (k <= kLocalSelectMaxK ? std::min(64, std::max(1, 65536 / (8 * k))) : 64);
-    // device-side work-item shape: FLAT tf32-exact queries take one plane and twice the queries
-    const int qchunk_min = use_tc ? tp.qchunk_split : qchunk;
-    int32_t* qcfg;
-    CK(s.alloc(&qcfg, 2));
-    const int64_t npairs = nq * npb;
-    // Seeding (tensor-core path, nprobe >= 2): phase A scans the first capA rows of each query's
-    // ra[q] nearest lists -- the fewest holding >= max(2k, k+32) such rows -- and emits all of them;
-    // their k-th best key tau_q is an exact upper bound of the query's final k-th best (k distinct
-    // candidates are at or below it), so phase B scans every probed list and emits only keys <= tau_q.
-    const char* seed_env = getenv("MV_SEED");
-    const bool split = use_tc && npb >= 2 && !(seed_env && seed_env[0] == '0');
-    int32_t* ra = nullptr;
-    if (split) CK(s.alloc(&ra, (size_t)nq));
-    const int nv = split ? 2 * nlist : nlist;
-    Bucketing b;
-    CK(s.alloc(&b.lcount, nv));
-    CK(s.alloc(&b.boff, nv + 1));
-    CK(s.alloc(&b.bfill, nv));
-    const int64_t nent = split ? 2 * npairs : npairs;  // bucket entries (phase-A entries with seeding)
-    CK(s.alloc(&b.bq, (size_t)nent));
-    CK(s.alloc(&b.wcount, nv));
-    CK(s.alloc(&b.woff, nv + 1));
-    CK(s.alloc(&b.witems, (size_t)(nv + nent / qchunk_min + 1)));
-    CK(s.alloc(&b.witems_unsorted, (size_t)(nv + nent / qchunk_min + 1)));
-    CK(s.alloc(&b.qtot, (size_t)(2 * (nq + 1))));
-    CK(s.alloc(&b.poff, (size_t)nent));
-    CK(s.alloc(&b.pcnt, (size_t)nent));
-    CK(s.alloc(&b.counter, 1));
-    CK(s.alloc(&b.whist, (size_t)kPlanCostBins));
-    CK(s.alloc(&b.bsum, (size_t)(2 * kPlanMaxBlocks)));
-    // pair regions: the whole list (tensor-core scan: emit-all bound), or min(k, |list|) (SIMT)
-    const int capk = use_tc ? 0 : k;
-    PlanArgs pa;
-    pa.probes = P; pa.nq = nq; pa.npb = npb; pa.nlist = nlist; pa.k = k; pa.capk = capk;
-    pa.split = split ? 1 : 0; pa.need = std::max<int64_t>(2 * (int64_t)k, k + 32);
-    // Sample size of the seeding phase.  tau_q = the k-th best of `need` candidates is about the
-    // (k N / need)-th best of the query's N candidates, so phase B emits ~k N / need keys.  Phase A
-    // costs ~need rows of payload, an emission ~a fixed number of bytes (the key store, the final
-    // select's reads); balancing the two gives need ~ sqrt(k N c / rowbytes).  c is measured
-    // (session-4 sweep): 32 B for k <= 256; the CTA-per-query select for k > 256 costs
-    // ~26x more per candidate (and falls back to global memory past its stage), c = 832 B.
-    {
-      const double ncand = (double)ix->ntotal * npb / std::max(1, nlist);
-      const double rowb = (double)dpad * (ix->type == MV_IVF_FLAT ? 4 : 1);
-      const double c = k > 256 ? 832.0 : 32.0;
-      const int64_t bal = (int64_t)std::sqrt((double)k * ncand * c / rowb);
-      pa.need = std::max<int64_t>(pa.need, std::min<int64_t>(bal, 65536));
-    }
-    if (const char* ne = getenv("MV_NEED")) pa.need = atoll(ne) > 0 ? std::max<int64_t>(2 * (int64_t)k, atoll(ne)) : pa.need;
-    // phase A reads the first capA rows of each of a query's nearest lists (a 16-row multiple, at
-    // least one tile; measured on configs[1]: 64 rows 14.7M qps, 128 rows 16.0M, 256 rows 15.8M,
-    // whole lists 14.7M -- a looser tau_q costs phase-B emissions, more rows cost phase-A reads)
-    // Rows per list of the sample: ~sqrt(64 need), i.e. the sample spreads over ~sqrt(need / 64)
-    // nearest lists (measured, MV_CAPA sweep: configs[2] 256 rows 2.85M qps vs whole lists 2.71M;
-    // configs[4] 128 rows best; configs[1] 128 rows vs 64: 16.0M vs 14.7M), at least 128 rows
-    pa.capA = std::max<int64_t>(128, std::min<int64_t>((pa.need + 15) & ~(int64_t)15,
-                                                       ((int64_t)std::sqrt(64.0 * pa.need) + 15) & ~(int64_t)15));
-    if (const char* ce = getenv("MV_CAPA"))  // sweep override (a 16-row multiple)
-      pa.capA = std::max<int64_t>(16, (atoll(ce) + 15) & ~15ll);
-    pa.list_off = ix->list_off;
-    pa.qlo_any = (use_tc && ix->type == MV_IVF_FLAT) ? qlo_any : nullptr;
-    pa.qc_exact = qchunk; pa.p_exact = use_tc ? (ix->type == MV_IVF_FLAT ? 1 : 4) : 1;
-    pa.qc_split = qchunk_min; pa.p_split = use_tc ? (ix->type == MV_IVF_FLAT ? 2 : 4) : 1;
-    pa.qcfg = qcfg; pa.ra = ra; pa.b = b;
-    CK(launch_plan(pa, st));
-    prof_mark(ix, st);
-    int64_t cap;
-    if (use_tc) {
-      // exact worst case without a device round trip: nq x (the npb longest lists)
-      cap = nq * ix->top_len_prefix[std::min<size_t>(npb, ix->top_len_prefix.size() - 1)];
-      if (split) cap += nq * (pa.need + pa.capA);  // phase-A prefixes: < need + capA rows per query
-    } else if (k <= kLocalSelectMaxK) {
-      cap = nq * npb * min64(capk, max64(ix->maxlen, 1));
-    } else {
-      CK(cudaMemcpyAsync(&cap, b.qtot + (nq + 1) + nq, sizeof(int64_t), cudaMemcpyDeviceToHost, st));
-      CK(cudaStreamSynchronize(st));
-    }
-    // per-query candidate bound (the final select's shared-memory staging decision) + its scratch
-    const int64_t tmax = use_tc ? ix->top_len_prefix[std::min<size_t>(npb, ix->top_len_prefix.size() - 1)]
-                                : (int64_t)npb * (k <= kLocalSelectMaxK ? k : max64(ix->maxlen, 1));
-    uint8_t* over = nullptr;
-    if (k > 256) CK(s.alloc(&over, (size_t)nq));
-    uint64_t* part;
-    cudaError_t ea = s.alloc(&part, (size_t)max64(cap, 1));
-    if (ea != cudaSuccess) {
-      cudaGetLastError();
-      return fail(MV_ENOMEM, "search: cannot allocate %lld candidate slots", (long long)cap);
-    }
-    // a5/a6
-    if (use_tc) {
-      const int P = ix->type == MV_IVF_FLAT ? 2 : 4;
-      const size_t esz = ix->type == MV_IVF_FLAT ? 4 : 1;
-      uint8_t* qplanes;
-      float* qscale;
-      double *qa, *qn64;
-      uint64_t* tau;
-      if (ix->type == MV_IVF_SQ8) CK(s.alloc(&qplanes, (size_t)nq * P * dpad * esz));
-      else qplanes = reinterpret_cast<uint8_t*>(qhl);
-      CK(s.alloc(&qscale, (size_t)nq));
-      CK(s.alloc(&qa, (size_t)nq));
-      CK(s.alloc(&qn64, (size_t)nq));
-      CK(s.alloc(&tau, (size_t)nq));
-      CK(cudaMemsetAsync(tau, 0xff, sizeof(uint64_t) * nq, st));
-      CK(launch_qplanes(ix->type, qpad, nq, dpad, ix->vmin, ix->vdiff, ix->type == MV_IVF_SQ8 ? qplanes : nullptr,
-                        qscale, qa, qn64, st));
-      tp.metric = ix->metric; tp.npb = npb; tp.nq = nq;
-      tp.list_off = ix->list_off; tp.norms = ix->norms; tp.ids = ix->ids; tp.rank = ix->rank;
-      tp.bitset = bs; tp.nbits = bs ? nbits : 0;
-      tp.qplanes = qplanes; tp.qnorm = qn64; tp.qscale = qscale; tp.qa = qa;
-      tp.bq = b.bq; tp.boff = b.boff; tp.witems = b.witems; tp.nlist = nlist; tp.cfg = qcfg;
-      tp.poff = b.poff; tp.pcnt = b.pcnt; tp.part = part; tp.tau = tau;
-      const char* dbg = getenv("MV_SCAN_DEBUG");
-      tp.dbg = dbg ? atoi(dbg) : 0;
-      tp.prof = nullptr;
-      const char* trc = getenv("MV_SCAN_TRACE");
-      if (trc && trc[0] == '1') {
-        CK(s.alloc(&tp.prof, (size_t)9 * 1024));
-        CK(cudaMemsetAsync(tp.prof, 0, 9 * 1024 * 8, st));
-      }
-      // phase A (or, without seeding, the whole scan emitting every candidate) ...
-      auto scan = [&]() { return use_qm ? launch_scan_qm(&ix->xm.m[0], &ix->xm.m[3], tp, st) : launch_scan_tc(ix->xm, tp, st); };
-      tp.phase = 0;
-      tp.rowcap = split ? (int)pa.capA : 0x7fffffff;
-      tp.wbeg = nullptr;
-      tp.nwitems = b.woff + nlist;
-      CK(scan());
-      prof_mark(ix, st);
-      if (split) {
-        // ... tau_q = k-th best key of phase A ...
-        // (phase A emits < need + capA candidates per query: a tighter staging bound than tmax)
-        CK(launch_tau_select(b.poff + npairs, b.pcnt + npairs, part, nq, npb, ra, k, tau,
-                             std::min<int64_t>(tmax, pa.need + pa.capA), over, st));
-        prof_mark(ix, st);
-        // ... phase B over every probed pair, emitting keys <= tau_q
-        tp.phase = 1;
-        tp.rowcap = 0x7fffffff;
-        tp.wbeg = b.woff + nlist;
-        tp.nwitems = b.woff + 2 * nlist;
-        CK(scan());
-      } else {
-        prof_mark(ix, st);
-      }
-      if (tp.prof) {  // debug timeline of CTA 0 (MV_SCAN_TRACE=1): rows = events, cycles since the first TMA issue
-        std::vector<unsigned long long> h(9 * 1024);
-        CK(cudaMemcpyAsync(h.data(), tp.prof, h.size() * 8, cudaMemcpyDeviceToHost, st));
-        CK(cudaStreamSynchronize(st));
-        const char* nm[8] = {"tma_issue[chunk]", "mma_q_ready[wi]", "mma_tile_start[t]", "mma_tile_done[t]",
-                             "epi_math_done[t]", "epi_sel_start[t]", "epi_tfull[t]", "epi_tile_end[t]"};
-        const unsigned long long t0 = h[0];
-        for (int r = 0; r < 8; ++r) {
-          fprintf(stderr, "[trace] %-18s", nm[r]);
-          for (int i = 0; i < 48; ++i)
-            if (h[r * 1024 + i]) fprintf(stderr, " %lld", (long long)(h[r * 1024 + i] - t0));
-          fprintf(stderr, "\n");
-        }
-        unsigned long long gmin = ~0ull;
-        for (int b = 0; b < 148; ++b) gmin = std::min(gmin, h[8 * 1024 + b * 3]);
-        fprintf(stderr, "[events] tiles_with_survivors %llu warmups %llu flushes %llu fallbacks %llu survivors %llu "
-                "folds %llu fold_survivors %llu\n",
-                h[8 * 1024 + 1000], h[8 * 1024 + 1001], h[8 * 1024 + 1002], h[8 * 1024 + 1003], h[8 * 1024 + 1004],
-                h[8 * 1024 + 1005], h[8 * 1024 + 1006]);
-        fprintf(stderr, "[cta] start_us end_us tiles:");
-        for (int b = 0; b < 148; ++b)
-          fprintf(stderr, " %d:%.1f/%.1f/%llu", b, (h[8 * 1024 + b * 3] - gmin) / 1e3, (h[8 * 1024 + b * 3 + 1] - gmin) / 1e3,
-                  h[8 * 1024 + b * 3 + 2]);
-        fprintf(stderr, "\n");
-      }
-      ix->last_scan = ix->type == MV_IVF_FLAT ? (use_qm ? "tcgen05.tf32.qm" : "tcgen05.tf32") : "tcgen05.i8";
-      ix->launches += split ? 4 : 2;  // qplanes, scan A (+ tau select, scan B)
-    } else {
-    ScanArgs a;
-    a.type = ix->type; a.metric = ix->metric; a.d = ix->d; a.dpad = dpad; a.k = k; a.npb = npb;
-    a.qchunk = qchunk; a.nlist = nlist;
-    a.list_off = ix->list_off; a.payload = ix->payload; a.norms = ix->norms; a.ids = ix->ids; a.rank = ix->rank;
-    a.bitset = bs; a.nbits = bs ? nbits : 0;
-    a.qpad = qpad; a.qnorm = qnorm; a.vmin = ix->vmin; a.vdiff = ix->vdiff; a.sq8_t = ix->sq8_t;
-    a.bq = b.bq; a.boff = b.boff; a.witems = b.witems; a.nwitems = b.woff + nlist; a.counter = b.counter;
-    a.poff = b.poff; a.pcnt = b.pcnt; a.part = part;
-    CK(launch_scan(a, st));
-    prof_mark(ix, st);
-    prof_mark(ix, st);
-    ix->last_scan = "simt";
-    }
-    prof_mark(ix, st);
-    // a7
-    CK(launch_final_select(b.poff, b.pcnt, part, nq, npb, k, ix->metric, ix->sorted_ids, D, I, tmax, over, st));
-    prof_mark(ix, st);
-    if (ix->prof) ix->prof_searches++;
-    ix->launches += 6;  // prep, hilo, coarse GEMM + probe select (or SIMT coarse), plan, final select
-    if (!use_tc) ix->launches += 1;
-  }
-  if (host_out) {
-    CK(cudaMemcpyAsync(distances, D, sizeof(float) * nq * k, cudaMemcpyDeviceToHost, st));
-    CK(cudaMemcpyAsync(out_ids, I, sizeof(int64_t) * nq * k, cudaMemcpyDeviceToHost, st));
-  }
-  if (host_out || sq) CK(cudaStreamSynchronize(st));
-  return MV_OK;
-}
-
 mv_status mv_merge_topk(mv_metric metric, const float* dists, const int64_t* ids, int32_t nsrc, int64_t nq, int32_t k,
                         float* out_d, int64_t* out_i, void* stream) {
   if (metric != MV_L2 && metric != MV_IP) return fail(MV_EINVAL, "unknown metric");
   if (nsrc < 1 || k < 1 || k > kMaxK || nq < 0) return fail(MV_EINVAL, "bad nsrc/k/nq");
   if (nq == 0) return MV_OK;
   if (!dists || !ids || !out_d || !out_i) return fail(MV_EINVAL, "null argument");
+  // the device of the (first) device buffer, else the current one: scratch goes there
+  int dev = -1;
+  for (const void* p : {(const void*)out_d, (const void*)dists}) {
+    cudaPointerAttributes at;
+    if (dev < 0 && cudaPointerGetAttributes(&at, p) == cudaSuccess && at.type == cudaMemoryTypeDevice) dev = at.device;
+    cudaGetLastError();
+  }
+  DeviceGuard g(dev);
   cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
-  Scratch s(st);
+  Scratch s(nullptr, st);
   const size_t per = (size_t)nq * k;
   bool sd, si;
   const float* D;
@@ -846,12 +908,17 @@ mv_status mv_merge_topk(mv_metric metric, const float* dists, const int64_t* ids
 
 mv_status mv_index_describe(const mv_index* ix, char* buf, size_t len) {
   if (!ix || !buf || len == 0) return fail(MV_EINVAL, "null argument");
+  const char* refine = ix->type != MV_IVF_FLAT ? "n/a (SQ8: exact int32 digit partials)"
+                       : ix->tf32_exact        ? "when a query is not tf32-exact"
+                                               : "always (stored values not tf32-exact)";
   snprintf(buf, len,
            "{\"d\": %d, \"dpad\": %d, \"nlist\": %d, \"ntotal\": %lld, \"maxlen\": %lld, \"type\": \"%s\", "
-           "\"metric\": \"%s\", \"tensor_map\": %s, \"tf32_exact\": %s, \"last_scan\": \"%s\", \"last_coarse\": \"%s\"}",
+           "\"metric\": \"%s\", \"tf32_exact\": %s, \"flat_refine\": \"%s\", \"xmax2\": %.17g, "
+           "\"allocator\": \"%s\", \"last_scan\": \"%s\", \"last_coarse\": \"%s\", \"last_chunks\": %lld}",
            ix->d, ix->dpad, ix->nlist, (long long)ix->ntotal, (long long)ix->maxlen,
            ix->type == MV_IVF_FLAT ? "IVF_FLAT" : "IVF_SQ8", ix->metric == MV_L2 ? "L2" : "IP",
-           ix->xmap_ok ? "true" : "false", ix->tf32_exact ? "true" : "false", ix->last_scan, ix->last_coarse);
+           ix->tf32_exact ? "true" : "false", refine, ix->xmax2, ix->alloc.alloc ? "caller" : "cuda-pool",
+           ix->last_scan, ix->last_coarse, (long long)ix->last_chunks);
   return MV_OK;
 }
 

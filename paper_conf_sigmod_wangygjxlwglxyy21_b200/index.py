@@ -2,11 +2,15 @@
 
 Tensors are passed as raw pointers (device tensors stay on the device; CPU tensors / numpy arrays
 are staged by the library itself).  Every step of the search runs in libmv's CUDA kernels; torch
-only provides device memory and the current stream.
+only provides device memory (the library's mv_allocator is routed to torch's caching allocator),
+the current stream and process groups.
 """
 from __future__ import annotations
 
+import atexit
+import contextlib
 import ctypes as C
+import weakref
 
 import numpy as np
 import torch
@@ -24,7 +28,7 @@ def _ptr(x):
     raise TypeError(f"unsupported buffer type {type(x)}")
 
 
-def _as_f32(x, d=None):
+def _as_f32(x):
     if isinstance(x, torch.Tensor):
         x = x.contiguous()
         if x.dtype != torch.float32:
@@ -39,12 +43,43 @@ def _as_i64(x):
     return np.ascontiguousarray(x, dtype=np.int64)
 
 
-def _stream(device: int, stream=None):
+def _torch_stream(device: int, stream=None) -> torch.cuda.Stream:
     if stream is None:
-        return C.c_void_p(torch.cuda.current_stream(device).cuda_stream)
+        return torch.cuda.current_stream(device)
     if isinstance(stream, torch.cuda.Stream):
-        return C.c_void_p(stream.cuda_stream)
-    return C.c_void_p(int(stream))
+        return stream
+    return torch.cuda.ExternalStream(int(stream), device=device)
+
+
+# ---- mv_allocator -> torch's caching allocator ------------------------------------------------
+# Blocks are taken on the library's stream, so torch reuses them only in that stream's order
+# (the library frees its scratch stream-ordered at the end of each call).
+@L.ALLOC_FN
+def _torch_alloc(nbytes, stream, ctx):
+    try:
+        return torch.cuda.caching_allocator_alloc(int(nbytes), device=int(ctx or 0), stream=int(stream or 0))
+    except Exception:  # reported to the caller as MV_ENOMEM
+        return None
+
+
+@L.FREE_FN
+def _torch_free(ptr, stream, ctx):
+    try:
+        torch.cuda.caching_allocator_delete(int(ptr))
+    except Exception:
+        pass
+
+
+_LIVE = weakref.WeakSet()
+
+
+@atexit.register
+def _close_all():  # destroy indexes while torch's allocator is still alive
+    for ix in list(_LIVE):
+        try:
+            ix.close()
+        except Exception:
+            pass
 
 
 METRICS = {"l2": L.MV_L2, "ip": L.MV_IP, L.MV_L2: L.MV_L2, L.MV_IP: L.MV_IP}
@@ -53,17 +88,28 @@ TYPES = {"flat": L.MV_IVF_FLAT, "ivf_flat": L.MV_IVF_FLAT, "sq8": L.MV_IVF_SQ8, 
 
 
 class Index:
-    """mv_index_create(d, metric, type, nlist) and friends (§3.2.1)."""
+    """mv_index_create(d, metric, type, nlist) and friends (§3.2.1).
 
-    def __init__(self, d: int, metric="l2", kind="flat", nlist: int = 1, device: int | None = None):
+    allocator: "torch" (default: every device allocation of the library goes through torch's
+    caching allocator) or None (the library's own cudaMalloc / stream-ordered pool)."""
+
+    def __init__(self, d: int, metric="l2", kind="flat", nlist: int = 1, device: int | None = None,
+                 allocator: str | None = "torch"):
         self._lib = L.load()
         self.d, self.nlist = int(d), int(nlist)
         self.metric = METRICS[metric.lower() if isinstance(metric, str) else metric]
         self.kind = TYPES[kind.lower() if isinstance(kind, str) else kind]
         self.device = torch.cuda.current_device() if device is None else int(device)
+        self._alloc = None
+        if allocator == "torch":
+            self._alloc = L.MvAllocator(_torch_alloc, _torch_free, C.c_void_p(self.device))
+        elif allocator is not None:
+            raise ValueError(f"unknown allocator {allocator!r}")
         h = C.c_void_p()
-        L.check(self._lib.mv_index_create(self.d, self.metric, self.kind, self.nlist, self.device, C.byref(h)))
+        L.check(self._lib.mv_index_create(self.d, self.metric, self.kind, self.nlist, self.device,
+                                          C.byref(self._alloc) if self._alloc is not None else None, C.byref(h)))
         self._h = h
+        _LIVE.add(self)
 
     # -- lifecycle -----------------------------------------------------------------------------
     def close(self):
@@ -80,6 +126,10 @@ class Index:
     @property
     def ntotal(self) -> int:
         return int(self._lib.mv_index_ntotal(self._h))
+
+    def set_option(self, name: str, value: int):
+        """mv_index_set_option: launch-shape / sample / workspace tuning (never changes results)."""
+        L.check(self._lib.mv_index_set_option(self._h, name.encode(), int(value)))
 
     # -- build -------------------------------------------------------------------------------
     def set_centroids(self, c):
@@ -100,13 +150,21 @@ class Index:
         L.check(self._lib.mv_index_get_sq8(self._h, _ptr(vmin), _ptr(vdiff)))
         return vmin, vdiff
 
+    def _on(self, stream):
+        """(torch stream, context manager making it current): temporaries made by the binding are
+        then allocated in the same stream order as the library's work."""
+        s = _torch_stream(self.device, stream)
+        return s, (torch.cuda.stream(s) if stream is not None else contextlib.nullcontext())
+
     def add(self, x, ids, stream=None):
-        x = _as_f32(x)
-        ids = _as_i64(ids)
-        n = int(x.shape[0])
-        if int(ids.shape[0]) != n:
-            raise ValueError("ids and vectors differ in length")
-        L.check(self._lib.mv_index_add(self._h, _ptr(x), _ptr(ids), n, _stream(self.device, stream)))
+        s, ctx = self._on(stream)
+        with ctx:
+            x = _as_f32(x)
+            ids = _as_i64(ids)
+            n = int(x.shape[0])
+            if int(ids.shape[0]) != n:
+                raise ValueError("ids and vectors differ in length")
+            L.check(self._lib.mv_index_add(self._h, _ptr(x), _ptr(ids), n, C.c_void_p(s.cuda_stream)))
 
     # -- search ------------------------------------------------------------------------------
     def search(self, q, k: int, nprobe: int, bitset=None, nbits: int | None = None, out=None, stream=None,
@@ -114,35 +172,40 @@ class Index:
         """Returns (D[nq,k] float32, I[nq,k] int64) on the index device (or into `out`).
         probes: optional int32 [nq, min(nprobe, nlist)] best-first buckets per query (as
         search_probes returns them); the coarse step is then skipped (mv_search_with_probes)."""
-        q = _as_f32(q)
-        nq = int(q.shape[0])
-        if out is None:
-            dev = torch.device("cuda", self.device)
-            D = torch.empty((nq, k), dtype=torch.float32, device=dev)
-            I = torch.empty((nq, k), dtype=torch.int64, device=dev)
-        else:
-            D, I = out
-        nb = 0
-        if bitset is not None:
-            nb = int(nbits) if nbits is not None else int(bitset.shape[0]) * 8
-        if probes is not None:
-            npb = min(int(nprobe), self.nlist)
-            if probes.dtype != torch.int32 or tuple(probes.shape) != (nq, npb) or not probes.is_contiguous():
-                raise ValueError(f"probes must be a contiguous int32 tensor of shape ({nq}, {npb})")
-            L.check(self._lib.mv_search_with_probes(self._h, _ptr(q), nq, int(k), int(nprobe), _ptr(probes),
-                                                    _ptr(bitset), nb, _ptr(D), _ptr(I), _stream(self.device, stream)))
+        s, ctx = self._on(stream)
+        with ctx:
+            q = _as_f32(q)
+            nq = int(q.shape[0])
+            if out is None:
+                dev = torch.device("cuda", self.device)
+                D = torch.empty((nq, k), dtype=torch.float32, device=dev)
+                I = torch.empty((nq, k), dtype=torch.int64, device=dev)
+            else:
+                D, I = out
+            nb = 0
+            if bitset is not None:
+                nb = int(nbits) if nbits is not None else int(bitset.shape[0]) * 8
+            sp = C.c_void_p(s.cuda_stream)
+            if probes is not None:
+                npb = min(int(nprobe), self.nlist)
+                if probes.dtype != torch.int32 or tuple(probes.shape) != (nq, npb) or not probes.is_contiguous():
+                    raise ValueError(f"probes must be a contiguous int32 tensor of shape ({nq}, {npb})")
+                L.check(self._lib.mv_search_with_probes(self._h, _ptr(q), nq, int(k), int(nprobe), _ptr(probes),
+                                                        _ptr(bitset), nb, _ptr(D), _ptr(I), sp))
+                return D, I
+            L.check(self._lib.mv_search(self._h, _ptr(q), nq, int(k), int(nprobe), _ptr(bitset), nb, _ptr(D), _ptr(I),
+                                        sp))
             return D, I
-        L.check(self._lib.mv_search(self._h, _ptr(q), nq, int(k), int(nprobe), _ptr(bitset), nb, _ptr(D), _ptr(I),
-                                    _stream(self.device, stream)))
-        return D, I
 
     def search_probes(self, q, nprobe: int, stream=None):
-        q = _as_f32(q)
-        nq = int(q.shape[0])
-        npb = min(int(nprobe), self.nlist)
-        P = torch.empty((nq, npb), dtype=torch.int32, device=torch.device("cuda", self.device))
-        L.check(self._lib.mv_search_probes(self._h, _ptr(q), nq, int(nprobe), _ptr(P), _stream(self.device, stream)))
-        return P
+        s, ctx = self._on(stream)
+        with ctx:
+            q = _as_f32(q)
+            nq = int(q.shape[0])
+            npb = min(int(nprobe), self.nlist)
+            P = torch.empty((nq, npb), dtype=torch.int32, device=torch.device("cuda", self.device))
+            L.check(self._lib.mv_search_probes(self._h, _ptr(q), nq, int(nprobe), _ptr(P), C.c_void_p(s.cuda_stream)))
+            return P
 
     # -- measurement ---------------------------------------------------------------------------
     STAGES = ("coarse", "bucket", "scan_a", "seed", "scan", "select")
@@ -160,8 +223,8 @@ class Index:
 
     def describe(self) -> dict:
         import json
-        buf = C.create_string_buffer(1024)
-        L.check(self._lib.mv_index_describe(self._h, buf, 1024))
+        buf = C.create_string_buffer(2048)
+        L.check(self._lib.mv_index_describe(self._h, buf, 2048))
         return json.loads(buf.value.decode())
 
     # -- parity hooks --------------------------------------------------------------------------
@@ -177,12 +240,14 @@ def merge_topk(dists, ids, metric="l2", stream=None):
     """mv_merge_topk: dists/ids [nsrc, nq, k] device tensors -> merged [nq, k]."""
     lib = L.load()
     m = METRICS[metric.lower() if isinstance(metric, str) else metric]
-    dists = dists.contiguous().float()
-    ids = ids.contiguous().to(torch.int64)
-    nsrc, nq, k = dists.shape
-    D = torch.empty((nq, k), dtype=torch.float32, device=dists.device)
-    I = torch.empty((nq, k), dtype=torch.int64, device=dists.device)
-    dev = dists.device.index if dists.is_cuda else 0
-    L.check(lib.mv_merge_topk(m, _ptr(dists), _ptr(ids), int(nsrc), int(nq), int(k), _ptr(D), _ptr(I),
-                              _stream(dev, stream) if dists.is_cuda else None))
+    dev = dists.device.index if dists.is_cuda else torch.cuda.current_device()
+    s = _torch_stream(dev, stream)
+    with (torch.cuda.stream(s) if stream is not None else contextlib.nullcontext()):
+        dists = dists.contiguous().float()
+        ids = ids.contiguous().to(torch.int64)
+        nsrc, nq, k = dists.shape
+        D = torch.empty((nq, k), dtype=torch.float32, device=dists.device)
+        I = torch.empty((nq, k), dtype=torch.int64, device=dists.device)
+        L.check(lib.mv_merge_topk(m, _ptr(dists), _ptr(ids), int(nsrc), int(nq), int(k), _ptr(D), _ptr(I),
+                                  C.c_void_p(s.cuda_stream) if dists.is_cuda else None))
     return D, I

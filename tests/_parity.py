@@ -105,3 +105,35 @@ def check_probes(Pg, Q, C, nprobe, metric, rtol=1e-5):
         for c in a ^ b:
             assert abs(s[c] - kth) <= rtol * max(abs(kth), 1e-30), f"query {i}: probe {c} not tied with the boundary"
     return nd
+
+
+def sampled_oracle_topk(Qs, Ps, off, sids, rows_of, metric, kind, k, sq8=None, bitset=None, nbits=0):
+    """Oracle step O5 for a sample of queries at sizes where building the whole oracle index is
+    impractical (configs[2..4] full size): for each query, its candidates are the members of the
+    (GPU-accepted, separately checked) probed lists, minus the excluded ids; distances to the
+    stored (FLAT) or decoded (SQ8, the oracle codec) vectors in fp64; the exact top-k by the total
+    order.  These are exactly the steps of oracle.IvfIndex.search, restricted to the probed lists.
+    rows_of(ids) -> the raw fp32 vectors of those ids (regenerated or indexed by the caller).
+    Returns (D, I, candidate maps)."""
+    m = len(Qs)
+    outD = np.empty((m, k))
+    outI = np.empty((m, k), dtype=np.int64)
+    cmaps = []
+    for i in range(m):
+        rows = np.concatenate([np.arange(off[l], off[l + 1]) for l in Ps[i]] + [np.zeros(0, np.int64)])
+        cid = sids[rows]
+        keep = ~O.bit_is_set(bitset, nbits, cid)
+        rows, cid = rows[keep], cid[keep]
+        V = np.asarray(rows_of(cid), dtype=np.float32)
+        if kind == O.SQ8:
+            V = O.sq8_decode(O.sq8_encode(V, *sq8), *sq8)
+        D = O.distances(Qs[i], V, metric)
+        outD[i], outI[i], _ = O.select_topk(D, cid, rows, k, metric)
+        cmaps.append(dict(zip(cid.tolist(), D.tolist())))
+    return outD, outI, cmaps
+
+
+def gpu_lists_of(ids_sample, off, pos_of):
+    """The GPU's list of each sampled id: its storage position -> the list whose range holds it."""
+    pos = pos_of(ids_sample)
+    return np.searchsorted(off, pos, side="right") - 1

@@ -20,7 +20,7 @@ def test_header_declares_the_boundary():
     syms = L.header_symbols()
     for s in ["mv_index_create", "mv_index_set_centroids", "mv_index_train_sq8", "mv_index_set_sq8", "mv_index_add",
               "mv_search", "mv_merge_topk", "mv_index_destroy", "mv_last_error", "mv_search_probes",
-              "mv_index_ntotal", "mv_index_storage"]:
+              "mv_index_ntotal", "mv_index_storage", "mv_index_set_option", "mv_search_with_probes"]:
         assert s in syms
 
 
@@ -48,10 +48,15 @@ def test_version_and_error_strings(lib):
 def test_argument_errors_before_any_device_work(lib):
     # argument validation returns synchronously without touching a device
     h = ctypes.c_void_p()
-    assert lib.mv_index_create(0, 0, 0, 4, 0, ctypes.byref(h)) == -1
+    assert lib.mv_index_create(0, 0, 0, 4, 0, None, ctypes.byref(h)) == -1
     assert b"d must be" in lib.mv_last_error()
-    assert lib.mv_index_create(8, 7, 0, 4, 0, ctypes.byref(h)) == -1
-    assert lib.mv_index_create(8, 0, 0, 0, 0, ctypes.byref(h)) == -1
+    assert lib.mv_index_create(513, 0, 0, 4, 0, None, ctypes.byref(h)) == -1   # d <= 512 (mv.h)
+    assert lib.mv_index_create(8, 7, 0, 4, 0, None, ctypes.byref(h)) == -1
+    assert lib.mv_index_create(8, 0, 0, 0, 0, None, ctypes.byref(h)) == -1
+    half = L.MvAllocator(L.ALLOC_FN(lambda n, s, c: None), L.FREE_FN(), None)  # alloc without free
+    assert lib.mv_index_create(8, 0, 0, 4, 0, ctypes.byref(half), ctypes.byref(h)) == -1
+    assert b"allocator" in lib.mv_last_error()
+    assert lib.mv_index_set_option(None, b"need", 1) == -1
     assert lib.mv_merge_topk(0, None, None, 0, 1, 1, None, None, None) == -1
     assert lib.mv_search(None, None, 1, 10, 1, None, 0, None, None, None) == -1
     assert lib.mv_index_ntotal(None) == 0

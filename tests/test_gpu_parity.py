@@ -84,38 +84,28 @@ def test_flat_l2_sift_conditional(n, nlist, nprobe, nq, k):
     assert frac == 1.0  # integer data: no ties can be broken differently except exact ties by id
 
 
-@pytest.mark.parametrize("frac_q", [False, True])
-def test_flat_qm_scan_conditional(frac_q, monkeypatch):
-    """The experimental queries-as-M FLAT scan (MV_SCAN_IMPL=qm) meets the same parity
-    bar: one-plane (tf32-exact) and two-plane (fractional) queries, lists longer than one tile."""
-    monkeypatch.setenv("MV_SCAN_IMPL", "qm")
-    X, Q = _sift(20_000, 150)
-    if frac_q:
-        Q = Q * 0.7311 + 0.377
-    ids = G.permuted_ids(20_000, seed=9)
-    C = kmeans(X, 64, iters=5)
-    ix = _build(X, ids, C, "l2", "flat")
-    atol = 2e-6 * float((Q * Q).sum(1).max() + (X * X).sum(1).max()) if frac_q else 0.0
-    frac, _, _ = _run_conditional(ix, X, ids, C, Q, 10, 7, O.L2, O.FLAT, atol=atol)
-    assert ix.describe()["last_scan"] == "tcgen05.tf32.qm"
-    assert frac > 0.999
-
-
 @pytest.mark.parametrize("metric", ["l2", "ip"])
-def test_flat_tc_fractional_queries(metric):
-    """Integer (tf32-exact) base data with fractional queries: the tensor-core scan must take the
-    two-plane (hi/lo) query split instead of the one-plane shape used for tf32-exact queries."""
-    X, Q = _sift(15_000, 130)
+@pytest.mark.parametrize("d,flat_qc", [(128, 0), (128, 80), (128, 48), (192, 0), (320, 0), (64, 16)])
+def test_flat_tc_fractional_queries(metric, d, flat_qc):
+    """Integer (tf32-exact) base data with fractional queries: the tensor-core scan takes the
+    two-plane (hi/lo) items and the filter mode (DESIGN.md §5 "FLAT precision"); distances are the
+    exact fp64 values (rtol 1e-5, atol 0).  flat_qc / d pick the 80-, 48- and 16-query item shapes
+    whose two-plane width 2 roundup16(qc/2) exceeds roundup16(qc) (the operand and the TMEM
+    accumulators must be sized for it)."""
+    X, Q = _sift(15_000, 130, d=d, n_micro=2048)
     Q = Q * 0.7311 + 0.377  # not tf32-representable
     ids = G.permuted_ids(15_000, seed=5)
     C = kmeans(X, 128, iters=5)
-    ix = _build(X, ids, C, metric, "flat")
+    Index, _ = _mv()
+    ix = Index(d, metric, "flat", 128)
+    if flat_qc:
+        ix.set_option("flat_qc", flat_qc)
+    ix.set_centroids(C.cuda())
+    ix.add(X.cuda(), ids.cuda())
     mo = O.L2 if metric == "l2" else O.IP
-    # the fp32 expansion ||q||^2 + ||x||^2 - 2 q.x (and the fp32 MMA accumulation of q.x) carries an
-    # absolute error proportional to the norms, not to the distance (DESIGN.md §6)
-    atol = 2e-6 * float((Q * Q).sum(1).max() + (X * X).sum(1).max())
-    frac, _, _ = _run_conditional(ix, X, ids, C, Q, 10, 9, mo, O.FLAT, atol=atol)
-    assert ix.describe()["last_scan"].startswith("tcgen05.tf32")
+    frac, _, _ = _run_conditional(ix, X, ids, C, Q, 10, 9, mo, O.FLAT)
+    desc = ix.describe()
+    assert desc["last_scan"] == "tcgen05.tf32" and desc["tf32_exact"]
     assert frac > 0.999
 
 
@@ -141,12 +131,34 @@ def test_coarse_probe_sets(nprobe, metric):
     assert (np.diff(sc, axis=1) >= -1e-5 * np.abs(sc[:, 1:])).all()
 
 
-def test_flat_ip_deep_conditional():
+@pytest.mark.parametrize("metric,k", [("ip", 20), ("l2", 20), ("ip", 300), ("l2", 1)])
+def test_flat_deep_conditional(metric, k):
+    """Arbitrary fp32 data (unit-norm Deep-shaped, not tf32-representable) on the tensor cores:
+    tf32 filter with a rigorous bound + exact fp64 re-scoring; the exact top-k, distances within
+    1e-5 relative with atol 0 (IVF_FLAT keeps the original vectors)."""
     X, Q = _deep(20_000, 150)
     ids = torch.arange(20_000, dtype=torch.int64) * 2 + 1
     C = kmeans(X, 128, iters=6, spherical=True)
-    ix = _build(X, ids, C, "ip", "flat")
-    frac, _, _ = _run_conditional(ix, X, ids, C, Q, 20, 8, O.IP, O.FLAT, atol=1e-6)
+    ix = _build(X, ids, C, metric, "flat")
+    mo = O.IP if metric == "ip" else O.L2
+    frac, _, _ = _run_conditional(ix, X, ids, C, Q, k, 8, mo, O.FLAT)
+    desc = ix.describe()
+    assert desc["last_scan"] == "tcgen05.tf32" and not desc["tf32_exact"]
+    assert frac > 0.999
+
+
+@pytest.mark.parametrize("kind,metric,d", [("flat", "l2", 512), ("flat", "ip", 500), ("sq8", "l2", 320),
+                                           ("sq8", "ip", 512)])
+def test_large_d_gaussian(kind, metric, d):
+    """d up to the 512 limit of mv.h, fp32 Gaussian data (filter mode for FLAT)."""
+    X = G.gaussian(6000, d, seed=31)
+    Q = G.gaussian(70, d, seed=32)
+    ids = G.permuted_ids(6000, seed=33)
+    C = kmeans(X, 24, iters=4)
+    ix = _build(X, ids, C, metric, kind)
+    mo = O.IP if metric == "ip" else O.L2
+    frac, _, _ = _run_conditional(ix, X, ids, C, Q, 25, 5, mo, O.FLAT if kind == "flat" else O.SQ8,
+                                  atol=0.0 if kind == "flat" else 2e-6 * d)
     assert frac > 0.999
 
 
@@ -195,7 +207,7 @@ def test_large_k(k):
     ids = G.permuted_ids(n, seed=5)
     C = kmeans(X, 40, iters=5)
     ix = _build(X, ids, C, "l2", "flat")
-    nprobe = 40 if k == 16384 else 12
+    nprobe = 40 if k == 16384 else 12  # 40 = nlist: every bucket
     frac, D, I = _run_conditional(ix, X, ids, C, Q, k, nprobe, O.L2, O.FLAT)
     assert frac == 1.0
 
@@ -233,7 +245,7 @@ def test_edge_cases():
     # k > candidates -> padding; nprobe > nlist clamps; all-ones bitset -> padding
     D, I = ix.search(Q.cuda(), 600, 100)
     De, Ie = O.exact_knn(X.numpy(), ids.numpy(), Q.numpy(), 600, O.L2)
-    check_topk(D.cpu().numpy(), I.cpu().numpy(), De, Ie, atol=1e-4,
+    check_topk(D.cpu().numpy(), I.cpu().numpy(), De, Ie,
                cmaps=[{i: dd for i, dd in zip(range(500), O.distances(Q.numpy()[j], X.numpy(), O.L2))} for j in range(9)])
     ones = torch.full((63,), 255, dtype=torch.uint8)
     D, I = ix.search(Q.cuda(), 5, 7, bitset=ones.cuda(), nbits=500)
@@ -332,30 +344,83 @@ def test_c2_full_size_sampled():
     check_topk(D.cpu().numpy()[sel], I.cpu().numpy()[sel], Do, Io, exact=True)
 
 
+OPTION_SETS = [{"seeding": 0}, {"need": 1, "capa": 16}, {"flat_qc": 32, "sq8_qc": 16},
+               {"coarse_nqb": 64, "coarse_cs": 3, "coarse_epi": 16, "coarse_nacc": 1},
+               {"workspace_bytes": 1 << 20}]
+
+
 @pytest.mark.parametrize("kind,metric,k", [("flat", "l2", 10), ("flat", "l2", 300), ("flat", "ip", 10),
                                            ("sq8", "l2", 10), ("sq8", "ip", 64)])
-def test_tensor_core_path_matches_simt_path(kind, metric, k, monkeypatch):
-    """The tcgen05 scan (default) and the SIMT bring-up scan (MV_FORCE_SIMT=1) agree: bit-for-bit
-    ids on integer data; SQ8 distances within the digit-plane tolerance."""
+def test_options_never_change_results(kind, metric, k):
+    """mv_index_set_option picks launch shapes, the seeding sample and the workspace budget (the
+    tiny budget forces many query chunks): results are bit-identical to the defaults."""
     X, Q = _sift(12_000, 300, n_micro=512)
     ids = G.permuted_ids(12_000, seed=11)
     C = kmeans(X, 64, iters=4)
+    Qd = Q.cuda()
     ix = _build(X, ids, C, metric, kind)
-    D1, I1 = ix.search(Q.cuda(), k, 6)
-    assert ix.describe()["last_scan"].startswith("tcgen05")
-    assert ix.describe()["last_coarse"].startswith("tcgen05")
-    monkeypatch.setenv("MV_FORCE_SIMT", "1")
-    D2, I2 = ix.search(Q.cuda(), k, 6)
-    torch.cuda.synchronize()
-    if kind == "flat":
-        assert torch.equal(I1, I2) and torch.equal(D1, D2)
-    else:
-        # both paths are within 1e-5 of the fp64 oracle (test_sq8_sift_l2_conditional), so they
-        # agree within 2e-5; ids may differ only where distances tie
-        assert torch.allclose(D1, D2, rtol=2e-5, atol=1e-3)
-        diff = I1 != I2
-        assert torch.allclose(D1[diff], D2[diff], rtol=2e-5, atol=1e-3)
-        assert (~diff).float().mean().item() > 0.99
+    D0, I0 = ix.search(Qd, k, 6)
+    assert ix.describe()["last_chunks"] == 1
+    for opts in OPTION_SETS:
+        jx = _build(X, ids, C, metric, kind)
+        for name, v in opts.items():
+            jx.set_option(name, v)
+        D1, I1 = jx.search(Qd, k, 6)
+        torch.cuda.synchronize()
+        assert torch.equal(I0, I1) and torch.equal(D0, D1), opts
+        if "workspace_bytes" in opts:
+            assert jx.describe()["last_chunks"] > 1
+    from paper_conf_sigmod_wangygjxlwglxyy21_b200 import MvError
+    with pytest.raises(MvError):
+        ix.set_option("no_such_option", 1)
+
+
+def test_cuda_pool_allocator_equals_torch_allocator():
+    """mv_allocator routed to torch's caching allocator (default) vs the library's own pools."""
+    Index, _ = _mv()
+    X, Q = _sift(8000, 64)
+    ids = G.permuted_ids(8000, seed=2)
+    C = kmeans(X, 32, iters=4)
+    out = []
+    for alloc in ("torch", None):
+        ix = Index(128, "l2", "flat", 32, allocator=alloc)
+        ix.set_centroids(C.cuda())
+        ix.add(X.cuda(), ids.cuda())
+        out.append(ix.search(Q.cuda(), 15, 4))
+        assert ix.describe()["allocator"] == ("caller" if alloc else "cuda-pool")
+    assert torch.equal(out[0][0], out[1][0]) and torch.equal(out[0][1], out[1][1])
+
+
+@pytest.mark.parametrize("nprobe", [200, 700, 1024])
+def test_coarse_large_nprobe(nprobe):
+    """nprobe up to 1024 on the tensor-core coarse step (k_probe_select R = 8, 32)."""
+    X, Q = _sift(30_000, 64)
+    Q = Q * 0.93 + 0.21
+    C = kmeans(X, 2048, iters=2)
+    Index, _ = _mv()
+    ix = Index(128, "l2", "flat", 2048)
+    ix.set_centroids(C.cuda())
+    P = ix.search_probes(Q.cuda(), nprobe).cpu().numpy()
+    assert ix.describe()["last_coarse"] == "tcgen05.tf32"
+    check_probes(P, Q.numpy(), C.numpy(), nprobe, O.L2)
+
+
+def test_large_k_select_overflow_mix():
+    """k = 2048 with nprobe = 1 over lists of 30k and 8k rows: queries of the long list exceed
+    k_final_big's shared-memory stage (~26k keys) and take the global-memory radix select, the
+    others stay on k_final_big (the `over` routing of k_select.cu)."""
+    r = np.random.default_rng(5)
+    cA, cB, cC = (np.full(16, v, np.float32) for v in (40.0, 140.0, 240.0))
+    X = np.concatenate([cA + r.integers(-12, 13, (30_000, 16)), cB + r.integers(-12, 13, (8000, 16)),
+                        cC + r.integers(-12, 13, (8000, 16))]).astype(np.float32)
+    Qn = np.concatenate([cA + r.integers(-6, 7, (6, 16)), cB + r.integers(-6, 7, (6, 16))]).astype(np.float32)
+    ids = G.permuted_ids(len(X), seed=8)
+    C = torch.tensor(np.stack([cA, cB, cC]))
+    ix = _build(torch.tensor(X), ids, C, "l2", "flat")
+    off, _, _ = ix.storage()
+    assert sorted(np.diff(off).tolist()) == [8000, 8000, 30_000]
+    frac, _, _ = _run_conditional(ix, torch.tensor(X), ids, C, torch.tensor(Qn), 2048, 1, O.L2, O.FLAT, exact=True)
+    assert frac == 1.0
 
 
 @pytest.mark.parametrize("kind,metric", [("flat", "l2"), ("sq8", "ip")])
@@ -378,11 +443,10 @@ def test_search_with_probes_equals_search(kind, metric):
 
 @pytest.mark.parametrize("kind,metric,k", [("flat", "l2", 10), ("sq8", "ip", 100), ("flat", "l2", 600)])
 @pytest.mark.parametrize("need", ["1", "1000000"])
-def test_seeding_sample_size_extremes(kind, metric, k, need, monkeypatch):
+def test_seeding_sample_size_extremes(kind, metric, k, need):
     """The seeding phase's sample size (DESIGN.md §5 `need`) only changes how tight tau_q is, never
     the result: the 2k floor (loosest bound, most phase-B emissions) and a sample larger than every
     query's candidate set (phase A scans all probed lists) both equal the oracle."""
-    monkeypatch.setenv("MV_NEED", need)
     if kind == "flat":
         X, Q = _sift(12_000, 60)
         mo, ko = O.L2, O.FLAT
@@ -392,6 +456,7 @@ def test_seeding_sample_size_extremes(kind, metric, k, need, monkeypatch):
     ids = G.permuted_ids(12_000, seed=21)
     C = kmeans(X, 48, iters=4)
     ix = _build(X, ids, C, metric, kind)
+    ix.set_option("need", int(need))
     bs = G.mod_bitset(12_000, 10) if kind == "sq8" else None
     frac, _, _ = _run_conditional(ix, X, ids, C, Q, k, 9, mo, ko, bitset=bs, nbits=12_000 if bs is not None else 0)
     assert frac > (0.999 if kind == "sq8" else 0.9999)
@@ -399,14 +464,18 @@ def test_seeding_sample_size_extremes(kind, metric, k, need, monkeypatch):
 
 @pytest.mark.parametrize("qc", ["16", "32", "64"])
 @pytest.mark.parametrize("metric", ["l2", "ip"])
-def test_sq8_item_width_and_accumulators(qc, metric, monkeypatch):
+def test_sq8_item_width_and_accumulators(qc, metric):
     """SQ8 work items of 16 / 32 / 64 queries (8 / 4 / 2 TMEM accumulators in flight),
     lists probed by more queries than one item holds, a bitset: same answer as the oracle."""
-    monkeypatch.setenv("MV_SQ8_QC", qc)
     X, Q = _sift(16_000, 150, n_micro=1024)
     ids = G.permuted_ids(16_000, seed=17)
     C = kmeans(X, 24, iters=4)
-    ix = _build(X, ids, C, metric, "sq8")
+    Index, _ = _mv()
+    ix = Index(128, metric, "sq8", 24)
+    ix.set_option("sq8_qc", int(qc))
+    ix.set_centroids(C.cuda())
+    ix.train_sq8(X.cuda())
+    ix.add(X.cuda(), ids.cuda())
     bs = G.mod_bitset(16_000, 7)
     mo = O.IP if metric == "ip" else O.L2
     frac, _, _ = _run_conditional(ix, X, ids, C, Q, 20, 5, mo, O.SQ8, bitset=bs, nbits=16_000)
