@@ -96,6 +96,13 @@ def shard_ground_truth(Qg, xb_iter, k=10):
     return gd, gi
 
 
+def c5_spec(d=128):
+    """configs[4]'s generator: the SIFT-shaped mixture with the points-per-micro-centre density of
+    the c2 calibration (~15) kept at 1B rows -- 2^26 micro centres instead of 2^16."""
+    import mvgen as G
+    return G.SiftSpec(d=d, n_micro=1 << 26)
+
+
 def build_sharded(cfg, device, shard, nshard, Index, chunk=1 << 24, ngt=1000):
     """c5: 1B-row SIFT-shaped IVF_SQ8 index, this GPU's shard (rows r with r % nshard == shard),
     generated on the device chunk by chunk (mvgen's counter hash regenerates any row anywhere) and
@@ -104,7 +111,7 @@ def build_sharded(cfg, device, shard, nshard, Index, chunk=1 << 24, ngt=1000):
     exact top-10 over this shard's raw rows for the first `ngt` queries (dist, ids)."""
     import mvgen as G
     from mvgen.kmeans import kmeans
-    spec = G.SiftSpec(d=cfg["d"])
+    spec = c5_spec(cfg["d"])
     ntr = min(cfg["n"], 64 * cfg["nlist"])
     Xtr = G.sift_base(ntr, d=cfg["d"], device=device, spec=spec)
     C = kmeans(Xtr, cfg["nlist"], iters=10)
@@ -452,17 +459,26 @@ def main():
     D, I, ms, stage_ms, launches, clocks = measure(nprobe)
     rec = recall_all(I)
     fixed = None
-    # the metric is qps AT recall@10 >= 0.95: double nprobe until it holds
-    if not args.no_recall_sweep:
+    # the metric is qps AT recall@10 >= 0.95: double nprobe until it holds; stop
+    # early when recall has plateaued (then the configured nprobe is reported)
+    if not args.no_recall_sweep and rec < RECALL_TARGET:
         sweep = [{"nprobe": nprobe, "value": nq / (ms / 1e3), "recall@10": rec}]
-        while rec < RECALL_TARGET and nprobe * 2 <= min(1024, cfg["nlist"]):
-            nprobe *= 2
+        np_ = nprobe
+        while sweep[-1]["recall@10"] < RECALL_TARGET and np_ * 2 <= min(1024, cfg["nlist"]):
+            np_ *= 2
+            D2, I2, ms2, _, _, _ = measure(np_)
+            sweep.append({"nprobe": np_, "value": nq / (ms2 / 1e3), "recall@10": recall_all(I2)})
+            if sweep[-1]["recall@10"] < sweep[-2]["recall@10"] + 0.002:
+                break  # plateau: more probes do not buy recall (e.g. SQ8 quantization-limited)
+        ok = [e for e in sweep if e["recall@10"] >= RECALL_TARGET]
+        if ok and ok[0]["nprobe"] != nprobe:
+            nprobe = ok[0]["nprobe"]
             D, I, ms, stage_ms, launches, clocks = measure(nprobe)
             rec = recall_all(I)
-            sweep.append({"nprobe": nprobe, "value": nq / (ms / 1e3), "recall@10": rec})
-        if len(sweep) > 1:
-            fixed = {"note": f"recall@10 < {RECALL_TARGET} at the config's nprobe: nprobe doubled until it "
-                             "holds; `value` is at the smallest such nprobe", "sweep": sweep}
+        fixed = {"sweep": sweep, "chosen_nprobe": nprobe,
+                 "note": (f"recall@10 < {RECALL_TARGET} at the config's nprobe: nprobe doubled; `value` is at the "
+                          "smallest nprobe that reaches it") if ok else
+                         (f"recall@10 plateaus below {RECALL_TARGET}: `value` is at the config's nprobe")}
     qps = nq / (ms / 1e3)
 
     # ---- e2e through the public API with host (pinned) buffers ----

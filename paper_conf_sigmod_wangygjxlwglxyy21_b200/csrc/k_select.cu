@@ -157,7 +157,6 @@ __global__ void __launch_bounds__(256) k_final_select(const int64_t* __restrict_
 // 256 < k: the CTA-per-query select's block size (32 warps: one CTA per SM when the candidate stage
 // takes all of shared memory, so the warps are the only latency hiding) and private histograms
 constexpr int kBigThreads = 1024;
-constexpr int kHistWarps = 8;  // private radix histograms (warps w, w + 8, ... share one)
 
 // Ascending bitonic sort of NK = kBigThreads E keys in shared memory by a kBigThreads block.  Warp w holds
 // the contiguous block [32 E w, 32 E (w + 1)) in registers, lane l element 32 j + l in v[j]:
@@ -223,10 +222,55 @@ __device__ __forceinline__ void block_sort_regs(uint64_t* win, int NK) {
   for (int j = 0; j < E; ++j) win[wbase + 32 * j + lane] = v[j];
 }
 
-// 256 < k: one CTA (kBigThreads threads) per query stages the query's candidates in shared memory (when
-// they fit, else it flags the query for k_final_select's global-memory path), then an MSB radix
-// select over the u64 keys -- 8-bit digits, histogram per pass in shared memory, stopping as soon
-// as the keys at or below the current prefix are exactly k -- and a bitonic sort of the k winners.
+// 256 < k: one CTA (kBigThreads threads) per query stages the query's candidates in shared memory
+// (when they fit, else it flags the query for k_final_select's global-memory path), then a radix
+// select over the u64 keys below their common prefix: 12-bit digits, one shared histogram with
+// warp-aggregated atomics (__match_any: near-neighbour keys crowd a few bins), a block scan for
+// the digit.  As soon as the digit's boundary bin holds <= kBoundBig keys, one gather pass moves
+// the keys below it to the winners (ballot-aggregated appends) and the boundary keys to a small
+// buffer that is sorted to complete the k; otherwise the next digit refines the boundary bin
+// (u64 keys are unique, so this ends).  Then a bitonic sort of the k winners.
+constexpr int kDigitBits = 12;
+constexpr int kBins = 1 << kDigitBits;
+constexpr int kBoundBig = kBins / 2;  // boundary keys gathered into the histogram's space (u64)
+
+// exclusive scan of kBins bins held by the kBigThreads threads (4 per thread): the thread whose
+// range holds the k-th key (counting from `below`) writes {bin, keys before the bin, keys in it}
+__device__ __forceinline__ void big_find_digit(const uint32_t* hist, int below, int k, int* red, int* s_int) {
+  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  constexpr int PER = kBins / kBigThreads;
+  uint32_t c[PER], tot = 0;
+#pragma unroll
+  for (int j = 0; j < PER; ++j) {
+    c[j] = hist[tid * PER + j];
+    tot += c[j];
+  }
+  uint32_t incl = tot;
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t v = __shfl_up_sync(MV_FULL, incl, o);
+    if (lane >= o) incl += v;
+  }
+  if (lane == 31) red[wid] = (int)incl;
+  __syncthreads();
+  if (wid == 0) {
+    int w = lane < kBigThreads / 32 ? red[lane] : 0;
+    for (int o = 1; o < 32; o <<= 1) {
+      const int v = __shfl_up_sync(MV_FULL, w, o);
+      if (lane >= o) w += v;
+    }
+    red[32 + lane] = w;  // inclusive scan of the warp totals
+  }
+  __syncthreads();
+  uint32_t cum = (uint32_t)below + (wid ? (uint32_t)red[32 + wid - 1] : 0u) + incl - tot;
+  if (cum < (uint32_t)k && cum + tot >= (uint32_t)k) {
+    int d = 0;
+    while (cum + c[d] < (uint32_t)k) cum += c[d++];
+    s_int[0] = tid * PER + d;
+    s_int[1] = (int)cum;
+    s_int[2] = (int)c[d];
+  }
+  __syncthreads();
+}
 
 __global__ void __launch_bounds__(kBigThreads) k_final_big(const int64_t* __restrict__ poff,
                                                            const int32_t* __restrict__ pcnt,
@@ -240,11 +284,14 @@ __global__ void __launch_bounds__(kBigThreads) k_final_big(const int64_t* __rest
   const int NK = next_pow2(max(k, 2));
   uint64_t* buf = reinterpret_cast<uint64_t*>(smem);   // cap
   uint64_t* win = buf + cap;                           // NK
-  uint32_t* whist = reinterpret_cast<uint32_t*>(win + NK);  // kHistWarps x 256 (>= 66 u64 for the min/max)
-  int32_t* s_pre = reinterpret_cast<int32_t*>(whist + kHistWarps * 256);  // npb + 1
-  int32_t* s_int = s_pre + npb + 1;                    // misc
+  uint32_t* hist = reinterpret_cast<uint32_t*>(win + NK);  // kBins u32; later the boundary keys (kBoundBig u64)
+  uint64_t* bnd = reinterpret_cast<uint64_t*>(hist);
+  int32_t* s_pre = reinterpret_cast<int32_t*>(hist + kBins);  // npb + 1
+  int32_t* s_int = s_pre + npb + 1;                    // misc (8)
+  int32_t* red = s_int + 8;                            // 64
   const int64_t q = blockIdx.x;
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  const uint32_t ltmask = (1u << lane) - 1;
   const int64_t* po = poff + q * npb;
   const int32_t* pc = pcnt + q * npb;
   const int nu = nuse ? nuse[q] : npb;
@@ -269,7 +316,7 @@ __global__ void __launch_bounds__(kBigThreads) k_final_big(const int64_t* __rest
     if (tid == 0) over[q] = 1;
     return;
   }
-  if (tid == 0) over[q] = 0;
+  if (tid == 0 && over) over[q] = 0;
   // staging by fire-and-forget 8-B async copies: every lane keeps its loads in flight (a plain
   // load/store loop was latency-bound: one ~1 us global round trip per 32 keys per warp)
   for (int j = wid; j < nu; j += kBigThreads / 32) {
@@ -282,15 +329,10 @@ __global__ void __launch_bounds__(kBigThreads) k_final_big(const int64_t* __rest
   asm volatile("cp.async.wait_all;" ::: "memory");
   __syncthreads();
   int nsel;  // winners to sort, in win[]
-  if (T <= k) {
+  if (T < k || (T == k && tau_out == nullptr)) {
     for (int i = tid; i < NK; i += kBigThreads) win[i] = i < T ? buf[i] : MV_KEY_PAD;
     nsel = T;
-  } else {
-    // radix select over the bits below the keys' common prefix: the first digit starts at the
-    // highest bit where the smallest and largest key differ (near-neighbour distance keys share
-    // their top ~10 bits, which a fixed MSB digit would pile into one contended bin).  8-bit
-    // digits, per-warp private histograms, a warp prefix scan for the digit; it stops as soon as
-    // the keys at or below the current prefix are exactly k (keys are unique).
+  } else {  // (the seeding select with exactly k candidates also needs the k-th key)
     uint64_t mn = MV_KEY_PAD, mx = 0;
     for (int i = tid; i < T; i += kBigThreads) {
       const uint64_t x = buf[i];
@@ -301,96 +343,88 @@ __global__ void __launch_bounds__(kBigThreads) k_final_big(const int64_t* __rest
       mn = umin64(mn, shfl_xor64(mn, o));
       mx = umax64(mx, shfl_xor64(mx, o));
     }
-    uint64_t* red = reinterpret_cast<uint64_t*>(whist);
+    uint64_t* r64 = reinterpret_cast<uint64_t*>(hist);
     if (lane == 0) {
-      red[wid] = mn;
-      red[32 + wid] = mx;
+      r64[wid] = mn;
+      r64[32 + wid] = mx;
     }
     __syncthreads();
     if (tid == 0) {
       for (int w = 1; w < kBigThreads / 32; ++w) {
-        mn = umin64(mn, red[w]);
-        mx = umax64(mx, red[32 + w]);
+        mn = umin64(mn, r64[w]);
+        mx = umax64(mx, r64[32 + w]);
       }
-      red[64] = mn;
-      red[65] = mx;
+      r64[64] = mn;
+      r64[65] = mx;
     }
     __syncthreads();
-    mn = red[64];
-    mx = red[65];
+    mn = r64[64];
+    mx = r64[65];
     __syncthreads();
     int lo = 64 - __clzll((long long)(mn ^ mx));  // bits [lo, 64) are common to every key
     uint64_t pfx = lo >= 64 ? 0 : (mn >> lo);
-    int below = 0;  // keys whose bits above lo are < pfx
-    for (;;) {
-      const int w = min(8, lo), sh = lo - w;
+    int below = 0, nb = 0;
+    for (;;) {  // digits until the boundary bin is small enough to gather
+      const int w = min(kDigitBits, lo), sh = lo - w;
       const uint32_t dmask = (1u << w) - 1;
-      for (int i = tid; i < kHistWarps * 256; i += kBigThreads) whist[i] = 0;
+      for (int i = tid; i < kBins; i += kBigThreads) hist[i] = 0;
       __syncthreads();
-      uint32_t* hw = whist + (wid % kHistWarps) * 256;
-      for (int i = tid; i < T; i += kBigThreads) {
-        const uint64_t x = buf[i];
-        if (lo >= 64 || (x >> lo) == pfx) atomicAdd(hw + ((uint32_t)(x >> sh) & dmask), 1u);
+      for (int b0 = 0; b0 < T; b0 += kBigThreads) {
+        const int i = b0 + tid;
+        uint32_t bin = 0xffffffffu;
+        if (i < T) {
+          const uint64_t x = buf[i];
+          if (lo >= 64 || (x >> lo) == pfx) bin = (uint32_t)(x >> sh) & dmask;
+        }
+        const uint32_t peers = __match_any_sync(MV_FULL, bin);
+        if (bin != 0xffffffffu && (__ffs(peers) - 1) == lane) atomicAdd(hist + bin, (uint32_t)__popc(peers));
       }
       __syncthreads();
-      if (wid == 0) {  // bins 8 * lane .. 8 * lane + 7, summed over the private histograms
-        uint32_t c[8];
-        uint32_t tot = 0;
-#pragma unroll
-        for (int j = 0; j < 8; ++j) {
-          uint32_t v = 0;
-          for (int h = 0; h < kHistWarps; ++h) v += whist[h * 256 + 8 * lane + j];
-          c[j] = v;
-          tot += v;
-        }
-        uint32_t incl = tot;
-        for (int o = 1; o < 32; o <<= 1) {
-          const uint32_t v = __shfl_up_sync(MV_FULL, incl, o);
-          if (lane >= o) incl += v;
-        }
-        uint32_t cum = below + incl - tot;  // keys before this lane's first bin
-        const bool mine = cum < (uint32_t)k && cum + tot >= (uint32_t)k;
-        if (mine) {
-          int d = 0;
-          while (cum + c[d] < (uint32_t)k) cum += c[d++];
-          s_int[0] = 8 * lane + d;
-          s_int[1] = (int)cum;
-          s_int[2] = cum + c[d] == (uint32_t)k;
-        }
-      }
-      __syncthreads();
+      big_find_digit(hist, below, k, red, s_int);
       pfx = (pfx << w) | (uint64_t)s_int[0];
       below = s_int[1];
+      nb = s_int[2];
       lo = sh;
-      const bool done = s_int[2] || lo == 0;
       __syncthreads();
-      if (done) break;
+      if (nb <= kBoundBig || lo == 0) break;
     }
-    // winners: keys whose bits above lo are <= pfx (exactly k: keys are unique)
-    if (tid == 0) s_int[3] = 0;
+    // gather: keys below the boundary bin -> win (exactly `below` of them), the bin's keys -> bnd
+    if (tid == 0) {
+      s_int[3] = 0;
+      s_int[4] = 0;
+    }
     __syncthreads();
-    for (int i = tid; i < T; i += kBigThreads) {
-      const uint64_t x = buf[i];
+    for (int b0 = 0; b0 < T; b0 += kBigThreads) {
+      const int i = b0 + tid;
+      const uint64_t x = i < T ? buf[i] : MV_KEY_PAD;
       const uint64_t top = lo >= 64 ? 0 : (x >> lo);
-      if (top <= pfx) win[atomicAdd(s_int + 3, 1)] = x;
+      const bool isw = i < T && top < pfx, isb = i < T && top == pfx;
+      const uint32_t mw = __ballot_sync(MV_FULL, isw), mb = __ballot_sync(MV_FULL, isb);
+      int ow = 0, ob = 0;
+      if (lane == 0) {
+        if (mw) ow = atomicAdd(s_int + 3, __popc(mw));
+        if (mb) ob = atomicAdd(s_int + 4, __popc(mb));
+      }
+      ow = __shfl_sync(MV_FULL, ow, 0);
+      ob = __shfl_sync(MV_FULL, ob, 0);
+      if (isw) win[ow + __popc(mw & ltmask)] = x;
+      if (isb && ob + __popc(mb & ltmask) < kBoundBig) bnd[ob + __popc(mb & ltmask)] = x;
     }
     __syncthreads();
+    const int nbb = min(nb, kBoundBig);
+    const int NB = next_pow2(max(nbb, 2));
+    for (int i = nbb + tid; i < NB; i += kBigThreads) bnd[i] = MV_KEY_PAD;
+    block_bitonic_sort(bnd, NB);
+    for (int i = tid; i < k - below; i += kBigThreads) win[below + i] = bnd[i];
     nsel = k;
     for (int i = k + tid; i < NK; i += kBigThreads) win[i] = MV_KEY_PAD;
+    if (tau_out) {  // seeding: the k-th best key
+      if (tid == 0) tau_out[q] = bnd[k - below - 1];
+      return;
+    }
   }
   __syncthreads();
-  if (tau_out) {  // seeding: only the k-th best key is needed (the largest winner)
-    if (nsel < k) return;
-    uint64_t m = 0;
-    for (int i = tid; i < k; i += kBigThreads) m = umax64(m, win[i]);
-    for (int o = 16; o > 0; o >>= 1) m = umax64(m, shfl_xor64(m, o));
-    if (lane == 0) buf[wid] = m;
-    __syncthreads();
-    if (tid == 0) {
-      uint64_t mm = 0;
-      for (int w = 0; w < kBigThreads / 32; ++w) mm = umax64(mm, buf[w]);
-      tau_out[q] = mm;
-    }
+  if (tau_out) {  // fewer than k candidates: tau stays untouched
     return;
   }
   // bitonic sort of the NK winners: register-blocked (strides < 32 E by shuffles and in registers,
@@ -426,7 +460,7 @@ static cudaError_t launch_big_select(const int64_t* poff, const int32_t* pcnt, c
                                      int64_t* out_i, const int32_t* nuse, uint64_t* tau, int64_t tmax,
                                      uint8_t* over, const int* gate, cudaStream_t st) {
   const int NK = next_pow2(max(k, 2));
-  const int fixed = NK * 8 + kHistWarps * 256 * 4 + (npb + 1) * 4 + 64 + 64;
+  const int fixed = NK * 8 + kBins * 4 + (npb + 1) * 4 + 72 * 4 + 64;
   // stage capacity: all of shared memory, or just the bound tmax when that is smaller (several
   // CTAs per SM: the seeding select's candidates are bounded by the phase-A prefixes)
   const int cap = (int)min64((227 * 1024 - fixed) / 8, max64(tmax, k));

@@ -46,6 +46,9 @@ struct mv_index {
   const char* last_scan = "none";
   const char* last_coarse = "none";
   int64_t last_chunks = 0;      // query chunks of the last search (workspace budget)
+  int64_t auto_budget = 0;      // half of the free device memory, sampled at create and after each add
+                                // (cudaMemGetInfo is a driver call that can stall behind NVML
+                                // queries, so it is kept off the search path)
   // profiling
   bool prof = false;
   std::vector<cudaEvent_t> ev;   // kProfStages + 1 events per profiled search chunk
@@ -305,6 +308,8 @@ mv_status mv_index_create(int32_t d, mv_metric metric, mv_type type, int32_t nli
     mv_index_destroy(ix);
     return from_cuda(e, "create");
   }
+  size_t fr = 0, tot = 0;
+  if (cudaMemGetInfo(&fr, &tot) == cudaSuccess) ix->auto_budget = (int64_t)(fr / 2);
   *out = ix;
   return MV_OK;
 }
@@ -564,6 +569,8 @@ mv_status mv_index_add(mv_index* ix, const float* vectors, const int64_t* ids, i
   std::sort(lens.begin(), lens.end(), std::greater<int64_t>());
   ix->top_len_prefix.assign(nlist + 1, 0);
   for (int l = 0; l < nlist; ++l) ix->top_len_prefix[l + 1] = ix->top_len_prefix[l] + lens[l];
+  size_t fr = 0, tot = 0;
+  if (cudaMemGetInfo(&fr, &tot) == cudaSuccess) ix->auto_budget = (int64_t)(fr / 2);
   return MV_OK;
 }
 
@@ -812,12 +819,7 @@ static mv_status search_impl(mv_index* ix, const float* queries, int64_t nq, int
   } else {
     // query chunks: each one's scratch (candidate regions, score matrix, ...) within the budget,
     // and < 2^29 (query, list) pairs (int32 pair ids with the seeding phase's second copy)
-    int64_t budget = ix->opt.workspace;
-    if (budget <= 0) {
-      size_t fr = 0, tot = 0;
-      CK(cudaMemGetInfo(&fr, &tot));
-      budget = (int64_t)(fr / 2);
-    }
+    int64_t budget = ix->opt.workspace > 0 ? ix->opt.workspace : std::max<int64_t>(ix->auto_budget, 1 << 30);
     const int64_t per = search_bytes_per_query(ix, npb, k);
     int64_t chunk = std::min<int64_t>(nq, std::max<int64_t>(1, budget / std::max<int64_t>(per, 1)));
     chunk = std::min<int64_t>(chunk, std::max<int64_t>(1, (int64_t(1) << 29) / npb));

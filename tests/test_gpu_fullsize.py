@@ -108,7 +108,7 @@ def test_c5_shard_sift1b_sq8_sampled_protocol():
     k, nprobe = cfg["k"], cfg["nprobe"]
     D, I = ix.search(Q, k, nprobe)
     torch.cuda.synchronize()
-    spec = G.SiftSpec(d=128)
+    spec = bench.c5_spec(128)
     Cn = C.cpu().numpy()
     off, sids, _ = ix.storage()
     assert len(sids) == nloc and np.all(sids % nshard == shard)
