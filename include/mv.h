@@ -92,7 +92,8 @@ MV_API mv_status mv_index_create(int32_t d, mv_metric metric, mv_type type, int3
 /* Tuning options.  None changes a result (tested): they pick launch shapes, the seeding sample and
  * the scratch budget.  Names: "seeding" (0/1), "need" (seeding sample, candidates), "capa" (rows
  * per list of the sample), "sq8_qc" / "flat_qc" (queries per scan work item), "coarse_nqb",
- * "coarse_cs", "coarse_epi", "coarse_nacc" (coarse GEMM shape), "workspace_bytes" (per-search
+ * "coarse_cs", "coarse_epi", "coarse_nacc" (coarse GEMM shape), "large_k_select" (k > 256: 0 = the
+ * staged radix select, 1 = the sample-threshold select), "workspace_bytes" (per-search
  * scratch budget: larger batches run as several query chunks; 0 = half of the device memory that was
  * free after the last create/add).
  * value 0 = automatic.  MV_EINVAL for an unknown name or a negative value. */

@@ -7,18 +7,26 @@
 //
 // k_coarse_gemm: CTA = one block of NQB queries (B operand: tf32 hi/lo planes, loaded once by TMA)
 // x a range of centroid tiles (A operand: 128 centroids, tf32 hi and lo planes, TMA ring).  Per
-// K-step two MMAs:  D[:, 0:2NQB] (=) C_hi . [Q_hi ; Q_lo]^T   and   D[:, 0:NQB] += C_lo . Q_hi^T,
-// so q.c = D[:, j] + D[:, NQB + j] up to the dropped lo x lo term (~2^-22 relative).  The epilogue
-// (8 warps, two per TMEM lane quarter) writes the score s(q, c) = ||c||^2 - 2 q.c (L2) or -q.c
-// (IP) to S[q][c] (coalesced: a warp's lanes are 32 consecutive centroids).
-// k_probe_select: one warp per query over its row of S -- pass 1 keeps every lane's R smallest
-// keys (key = score key << 32 | centroid id, so ties go to the smaller id), whose nprobe-th
-// smallest bounds the answer; pass 2 streams the keys at or below the bound through a 32-entry
-// staging buffer into a sorted register list (sort-32 + bitonic merge).
+// K-step, into one accumulator: C_hi Q_hi^T + C_lo Q_hi^T (+ C_hi Q_lo^T when some query needs its
+// lo plane), so q.c to ~2^-22 relative.  The epilogue (two warps per TMEM lane quarter; a warp's
+// lanes are 32 consecutive centroids) scores s(q, c) = ||c||^2 - 2 q.c (L2) or -q.c (IP) and
+//   pass 0: writes the minimum score key of each (query, 32-centroid group) to G (redux.sync);
+//   pass 1: stores key = (score key << 32 | centroid) when (score key, group) <= gbound[q], else
+//           padding, to the group's slots of the query's list.
+// k_group_bound (warp per query): gbound[q] = the nprobe-th smallest (G, group id) pair, by an
+// MSB bisection over the u32 keys and a ballot walk over the tied groups.  Exactly nprobe groups
+// are at or below it and each holds a centroid scoring at most its key, so the nprobe best
+// centroids all pass, and only centroids of those nprobe groups can (a passing centroid's group
+// minimum is at or below it): each selected group owns 32 fixed slots of the query's list
+// (gslot), so pass 1 stores without atomics.  Ties among equal scores go to the smaller centroid
+// id, as in the oracle.
+// k_probe_final (warp per query): pass 1 keeps every lane's R smallest appended keys, whose
+// nprobe-th smallest bounds the answer; pass 2 streams the keys at or below it through a 32-entry
+// staging buffer into a sorted register list.
 //
-// (Round 1 fused the selection into the GEMM epilogue; with 10 warps per SM that epilogue was
-// latency-bound on the per-tile folds.  Writing S costs 2 x nq x nlist x 4 B of HBM traffic --
-// 0.33 GB for configs[1] -- and buys a selection kernel at full occupancy.)
+// (Round 1 fused the selection into the GEMM epilogue and was latency-bound on the per-tile folds;
+// round 1's final form wrote the score matrix S -- 2.6 GB per search on configs[4] -- and
+// selected from it.  Two passes of the GEMM cost flops, which are cheap here, instead of bytes.)
 #include "mv_internal.cuh"
 #include "sm100.cuh"
 
@@ -53,6 +61,7 @@ __global__ void __launch_bounds__(kCThreads, 1)
   uint64_t* tfull = full_b + 1;
   uint64_t* tempty = tfull + 4;
   uint32_t* tslot = reinterpret_cast<uint32_t*>(tempty + 4);
+  uint64_t* sbound = reinterpret_cast<uint64_t*>(tslot + 2);  // pass 1: the block's per-query bounds
   const int nacc = p.nacc;
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -68,6 +77,9 @@ __global__ void __launch_bounds__(kCThreads, 1)
     }
     fence_mbar_init();
   }
+  if (p.mode == 1)
+    for (int i = threadIdx.x; i < NQB; i += blockDim.x)
+      sbound[i] = q0 + i < p.nq ? p.gbound[q0 + i] : 0ull;
   if (warp == 1) {
     tmem_alloc(tslot, p.tmem_cols);
     tmem_relinquish();
@@ -130,22 +142,21 @@ __global__ void __launch_bounds__(kCThreads, 1)
       }
     }
   } else {
-    // ------------------------------------------------------------------ epilogue: scores -> S
+    // ------------------------------------------------------------------ epilogue
     const int ew = warp - 2;             // 0..nepi-1
     const int quarter = warp & 3;        // TMEM lane quarter this warp may read
     const int sub = ew >> 2, nsub = p.nepi >> 2;
     const int row = quarter * 32 + lane;  // centroid within the tile
     const int nqv = (int)min64(NQB, p.nq - q0);
-    float* S = p.S + (int64_t)q0 * p.lds;
     uint32_t* G = p.G + (int64_t)q0 * p.ldg;
     const bool l2 = p.metric == MV_L2;
-    const uint32_t ldsb = (uint32_t)p.lds * 4u;  // row stride of S in bytes
+    const int ngr = (p.nlist + 31) / 32;
     for (int t = t0, tl = 0; t < t1; ++t, ++tl) {
       const uint32_t a = tl % nacc;
       const int cid = t * 128 + row;
+      const uint32_t grp = (uint32_t)(t * 4 + quarter);
       const bool valid = cid < p.nlist;
-      const bool store = valid;
-      const float cn = (valid && p.metric == MV_L2) ? __ldg(p.cnorm + cid) : 0.0f;
+      const float cn = (valid && l2) ? __ldg(p.cnorm + cid) : 0.0f;
       mbar_wait(&tfull[a], (tl / nacc) & 1);
       tc_fence_after();
       const uint32_t tb = tmem + a * NQB + ((uint32_t)(quarter * 32) << 16);
@@ -153,23 +164,45 @@ __global__ void __launch_bounds__(kCThreads, 1)
         uint32_t rd[16];
         tmem_ld16(tb + qc, rd);
         tmem_wait_ld();
-        // 32-bit strides inside the 16-column chunk (the 64-bit row pointer once per chunk); lane j
-        // keeps group minimum j and the G row stores go out as one instruction after the chunk
-        uint64_t sq;  // opaque to the compiler, so the row address is not rebuilt per column
-        asm("mov.b64 %0, %1;" : "=l"(sq) : "l"(S + (int64_t)qc * p.lds + cid));
         const int jn = min(16, nqv - qc);
-        uint32_t gmine = 0xffffffffu;
+        if (p.mode == 0) {
+          // lane j keeps group minimum j; the G row stores go out as one instruction per chunk
+          uint32_t gmine = 0xffffffffu;
 #pragma unroll
-        for (int j = 0; j < 16; ++j) {
-          const float dot = __uint_as_float(rd[j]);
-          const float sc = l2 ? cn - 2.0f * dot : -dot;
-          // the minimum score key of the warp's 32 centroids: lets the select skip whole groups
-          const uint32_t gm = __reduce_min_sync(MV_FULL, valid ? f2key(sc) : 0xffffffffu);
-          if (lane == j) gmine = gm;
-          asm volatile("{ .reg .pred p; setp.ne.u32 p, %2, 0; @p st.global.f32 [%0], %1; }"
-                       :: "l"(sq + (uint64_t)((uint32_t)j * ldsb)), "f"(sc), "r"((uint32_t)(j < jn && store)));
+          for (int j = 0; j < 16; ++j) {
+            const float dot = __uint_as_float(rd[j]);
+            const float sc = l2 ? cn - 2.0f * dot : -dot;
+            const uint32_t gm = __reduce_min_sync(MV_FULL, valid ? f2key(sc) : 0xffffffffu);
+            if (lane == j) gmine = gm;
+          }
+          if (lane < jn) G[(int64_t)(qc + lane) * p.ldg + grp] = gmine;
+        } else {
+          // keys and the pass test for the 16 columns; a column with a passing centroid belongs to
+          // one of the query's nprobe groups: lane j fetches column j's slot (one load per chunk)
+          uint32_t key[16], m[16], any = 0;
+#pragma unroll
+          for (int j = 0; j < 16; ++j) {
+            const float dot = __uint_as_float(rd[j]);
+            key[j] = f2key(l2 ? cn - 2.0f * dot : -dot);
+            const uint64_t b = sbound[qc + j];
+            const uint32_t bk = (uint32_t)(b >> 32);
+            const bool pass = valid && j < jn && (key[j] < bk || (key[j] == bk && grp <= (uint32_t)b));
+            m[j] = __ballot_sync(MV_FULL, pass);
+            any |= (m[j] != 0u) << j;
+          }
+          if (any) {
+            int sl = -1;
+            if (lane < 16 && ((any >> lane) & 1)) sl = (int)__ldg(p.gslot + (q0 + qc + lane) * (int64_t)ngr + grp);
+#pragma unroll
+            for (int j = 0; j < 16; ++j) {
+              if (!((any >> j) & 1)) continue;  // warp-uniform
+              const int slj = __shfl_sync(MV_FULL, sl, j);
+              const bool pass = (m[j] >> lane) & 1;
+              p.cand[(q0 + qc + j) * (int64_t)p.ccap + slj * 32 + lane] =
+                  pass ? (((uint64_t)key[j] << 32) | (uint32_t)cid) : MV_KEY_PAD;
+            }
+          }
         }
-        if (lane < jn) G[(int64_t)(qc + lane) * p.ldg + t * 4 + quarter] = gmine;
       }
       tc_fence_before();
       __syncwarp();
@@ -183,26 +216,101 @@ __global__ void __launch_bounds__(kCThreads, 1)
   }
 }
 
-// per-query top-nprobe of a score row (R = ceil(nprobe / 32) <= 4); see the file comment
+// gbound[q] = the nprobe-th smallest (group minimum key, group id) of the query's G row, and
+// gslot[q][g] = the rank (in group order) of group g among the nprobe groups at or below it, -1
+// for the others: pass 1 writes a selected group's 32 keys to slots [32 rank, 32 rank + 32) of
+// the query's candidate list -- no atomics.  One warp per query; a row of <= 32 kReg groups
+// lives in registers (group i * 32 + lane in v[i]), longer rows are re-read from L1/L2.
+constexpr int kReg = 64;
+
+template <int NRT>  // values per lane held in registers (0: re-read from L1/L2)
+__global__ void __launch_bounds__(256) k_group_bound(const uint32_t* __restrict__ G, int64_t ldg, int ng, int64_t nq,
+                                                     int nprobe, uint64_t* __restrict__ gbound,
+                                                     int16_t* __restrict__ gslot) {
+  const int lane = threadIdx.x & 31;
+  const int64_t q = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  if (q >= nq) return;
+  const uint32_t* g = G + q * ldg;
+  const uint32_t ltmask = (1u << lane) - 1;
+  constexpr bool REG = NRT > 0;
+  constexpr int NR = REG ? NRT : 1;
+  uint32_t v[NR];
+#pragma unroll
+  for (int i = 0; i < NR; ++i) v[i] = (REG && i * 32 + lane < ng) ? g[i * 32 + lane] : 0xffffffffu;
+  auto val = [&](int i) -> uint32_t {  // group i * 32 + lane (REG: i is a compile-time index)
+    if (REG) {
+      uint32_t x = 0xffffffffu;
+#pragma unroll
+      for (int j = 0; j < NR; ++j)
+        if (j == i) x = v[j];
+      return x;
+    }
+    return i * 32 + lane < ng ? __ldg(g + i * 32 + lane) : 0xffffffffu;
+  };
+  const int nrow = (ng + 31) / 32;
+  auto count_below = [&](uint32_t trial) {  // groups with key < trial
+    int c = 0;
+    if (REG) {
+#pragma unroll
+      for (int i = 0; i < NR; ++i) c += v[i] < trial;
+    } else {
+      for (int i = 0; i < nrow; ++i) c += val(i) < trial;
+    }
+    return (int)__reduce_add_sync(MV_FULL, (uint32_t)c);
+  };
+  // the nprobe-th smallest key b: the largest b with count(< b) < nprobe
+  uint32_t b = 0;
+  for (int bit = 31; bit >= 0; --bit) {
+    const uint32_t trial = b | (1u << bit);
+    if (count_below(trial) < nprobe) b = trial;
+  }
+  // among the groups with key == b (group order), the (nprobe - count(< b))-th; then the ranks
+  int r = nprobe - count_below(b);
+  uint32_t gsel = 0xffffffffu;
+  int base = 0;
+#pragma unroll
+  for (int i = 0; i < (REG ? NR : 1); ++i) {
+    for (int ii = REG ? i : 0; ii < (REG ? i + 1 : nrow); ++ii) {
+      const uint32_t x = val(ii);
+      const int gid = ii * 32 + lane;
+      const uint32_t tie = __ballot_sync(MV_FULL, gid < ng && x == b);
+      if (gsel == 0xffffffffu && tie) {
+        const int c = __popc(tie);
+        if (c >= r) {
+          uint32_t mm = tie;
+          for (int t = 1; t < r; ++t) mm &= mm - 1;
+          gsel = (uint32_t)(ii * 32 + __ffs(mm) - 1);
+        } else {
+          r -= c;
+        }
+      }
+      // selected: key < b, or key == b up to the chosen tied group (gsel is final once set, and
+      // every tied group before it in group order has been seen)
+      const bool sel = gid < ng && (x < b || (x == b && (gsel == 0xffffffffu || (uint32_t)gid <= gsel)));
+      const uint32_t m = __ballot_sync(MV_FULL, sel);
+      if (gid < ng) gslot[q * ng + gid] = sel ? (int16_t)(base + __popc(m & ltmask)) : (int16_t)-1;
+      base += __popc(m);
+    }
+  }
+  if (lane == 0) gbound[q] = ((uint64_t)b << 32) | gsel;
+}
+
+// per-query top-nprobe of the appended candidates (R = ceil(nprobe / 32)); see the file comment
 template <int R>
-__global__ void __launch_bounds__(256) k_probe_select(const float* __restrict__ S, int64_t lds,
-                                                      const uint32_t* __restrict__ G, int64_t ldg, int64_t nq,
-                                                      int nlist, int nprobe, int32_t* __restrict__ probes) {
+__global__ void __launch_bounds__(256) k_probe_final(const uint64_t* __restrict__ cand, int ccap, int64_t nq, int nprobe,
+                                                     int32_t* __restrict__ probes) {
   __shared__ uint64_t stage_all[8][64];
   const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
   const int64_t q = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   if (q >= nq) return;
   uint64_t* stage = stage_all[wib];
-  const float* s = S + q * lds;
-  const uint32_t* g = G + q * ldg;
-  const int ng = (int)ldg;
-  // pass 1: each lane's R smallest group minima; the nprobe-th smallest of those 32R bounds the
-  // answer (nprobe distinct centroids have score keys at or below it)
+  const uint64_t* c = cand + q * ccap;
+  const int n = ccap;  // 32 nprobe slots: the selected groups' keys, PAD where a centroid fails
   uint64_t t[R];
 #pragma unroll
   for (int r = 0; r < R; ++r) t[r] = MV_KEY_PAD;
-  for (int i = lane; i < ng; i += 32) {
-    const uint64_t key = ((uint64_t)g[i] << 32) | (uint32_t)i;
+  for (int i = lane; i < n; i += 32) {
+    const uint64_t key = c[i];
     if (key < t[R - 1]) {
       t[R - 1] = key;
 #pragma unroll
@@ -219,21 +327,19 @@ __global__ void __launch_bounds__(256) k_probe_select(const float* __restrict__ 
 #pragma unroll
   for (int r = 1; r < R; ++r)
     if (r == ((nprobe - 1) >> 5)) bsel = t[r];
-  const uint32_t bound = (uint32_t)(shfl64(bsel, (nprobe - 1) & 31) >> 32);
-  // pass 2: the groups whose minimum is within the bound; their keys at or below it -> staging ->
-  // sorted list L (32R, L[r] holds element r*32 + lane)
+  const uint64_t bound = shfl64(bsel, (nprobe - 1) & 31);
   uint64_t L[R];
 #pragma unroll
   for (int r = 0; r < R; ++r) L[r] = MV_KEY_PAD;
   int ns = 0;
   auto flush32 = [&]() {
-    uint64_t c[R];
+    uint64_t cc[R];
     uint64_t c1[1] = {lane < ns ? stage[lane] : MV_KEY_PAD};
     warp_bitonic_sort<1>(c1);
-    c[0] = c1[0];
+    cc[0] = c1[0];
 #pragma unroll
-    for (int r = 1; r < R; ++r) c[r] = MV_KEY_PAD;
-    warp_merge_smallest<R>(L, c);
+    for (int r = 1; r < R; ++r) cc[r] = MV_KEY_PAD;
+    warp_merge_smallest<R>(L, cc);
     const int rest = ns > 32 ? ns - 32 : 0;
     const uint64_t mv = lane < rest ? stage[32 + lane] : 0;
     __syncwarp();
@@ -241,25 +347,15 @@ __global__ void __launch_bounds__(256) k_probe_select(const float* __restrict__ 
     __syncwarp();
     ns = rest;
   };
-  for (int i0 = 0; i0 < ng; i0 += 32) {
-    const int gi = i0 + lane;
-    uint32_t m = __ballot_sync(MV_FULL, gi < ng && g[gi] <= bound);
-    while (m) {
-      const int grp = i0 + __ffs(m) - 1;
-      m &= m - 1;
-      const int c = grp * 32 + lane;
-      uint64_t key = MV_KEY_PAD;
-      if (c < nlist) {
-        const uint32_t k32 = f2key(s[c]);
-        if (k32 <= bound) key = ((uint64_t)k32 << 32) | (uint32_t)c;
-      }
-      const bool ps = key != MV_KEY_PAD;
-      const uint32_t bm = __ballot_sync(MV_FULL, ps);
-      if (ps) stage[ns + __popc(bm & ((1u << lane) - 1))] = key;
-      ns += __popc(bm);
-      __syncwarp();
-      if (ns >= 32) flush32();
-    }
+  for (int i0 = 0; i0 < n; i0 += 32) {
+    const int i = i0 + lane;
+    const uint64_t key = i < n ? c[i] : MV_KEY_PAD;
+    const bool ps = key != MV_KEY_PAD && key <= bound;
+    const uint32_t bm = __ballot_sync(MV_FULL, ps);
+    if (ps) stage[ns + __popc(bm & ((1u << lane) - 1))] = key;
+    ns += __popc(bm);
+    __syncwarp();
+    if (ns >= 32) flush32();
   }
   if (ns > 0) flush32();
 #pragma unroll
@@ -333,7 +429,7 @@ bool coarse_tc_plan(int dpad, int nprobe, int64_t nq, int nlist, int nsm, const 
   if (o.coarse_cs > 0) p.csplit = std::max(1, std::min(ntiles, o.coarse_cs));
   const int fixed = p.nchunks * 2 * p.nqb * 128;
   p.nstage = std::min(6, (budget - fixed) / stage);
-  p.smem_total = fixed + p.nstage * stage + 256 + 1024;
+  p.smem_total = fixed + p.nstage * stage + 256 + 128 * 8 + 1024;
   p.nepi = 8;
   p.nacc = 2;
   if (o.coarse_epi > 0) p.nepi = std::max(4, std::min(kCEpiMax, o.coarse_epi / 4 * 4));
@@ -345,21 +441,36 @@ bool coarse_tc_plan(int dpad, int nprobe, int64_t nq, int nlist, int nsm, const 
   return p.smem_total <= 227 * 1024;
 }
 
-cudaError_t launch_coarse_tc(const CUtensorMap* cmap, const CUtensorMap* qmap, const CoarseParams& p, int64_t nq,
+cudaError_t launch_coarse_tc(const CUtensorMap* cmap, const CUtensorMap* qmap, const CoarseParams& p0, int64_t nq,
                              cudaStream_t st) {
-  const unsigned grid = (unsigned)(((nq + p.nqb - 1) / p.nqb) * p.csplit);
-  cudaError_t e = cudaFuncSetAttribute(k_coarse_gemm, cudaFuncAttributeMaxDynamicSharedMemorySize, p.smem_total);
+  const unsigned grid = (unsigned)(((nq + p0.nqb - 1) / p0.nqb) * p0.csplit);
+  cudaError_t e = cudaFuncSetAttribute(k_coarse_gemm, cudaFuncAttributeMaxDynamicSharedMemorySize, p0.smem_total);
   if (e != cudaSuccess) return e;
+  CoarseParams p = p0;
+  p.mode = 0;  // pass 0: group minima
   k_coarse_gemm<<<grid, 64 + 32 * p.nepi, p.smem_total, st>>>(*cmap, *qmap, p);
   if ((e = cudaGetLastError()) != cudaSuccess) return e;
-  const unsigned g2 = (unsigned)((nq * 32 + 255) / 256);
+  const unsigned gw = (unsigned)((nq * 32 + 255) / 256);
+  const int ng = (p.nlist + 31) / 32;
+  if (ng <= 64) k_group_bound<2><<<gw, 256, 0, st>>>(p.G, p.ldg, ng, nq, p.nprobe, p.gbound, p.gslot);
+  else if (ng <= 128) k_group_bound<4><<<gw, 256, 0, st>>>(p.G, p.ldg, ng, nq, p.nprobe, p.gbound, p.gslot);
+  else if (ng <= 256) k_group_bound<8><<<gw, 256, 0, st>>>(p.G, p.ldg, ng, nq, p.nprobe, p.gbound, p.gslot);
+  else if (ng <= 512) k_group_bound<16><<<gw, 256, 0, st>>>(p.G, p.ldg, ng, nq, p.nprobe, p.gbound, p.gslot);
+  else if (ng <= 1024) k_group_bound<32><<<gw, 256, 0, st>>>(p.G, p.ldg, ng, nq, p.nprobe, p.gbound, p.gslot);
+  else if (ng <= 2048) k_group_bound<64><<<gw, 256, 0, st>>>(p.G, p.ldg, ng, nq, p.nprobe, p.gbound, p.gslot);
+  else k_group_bound<0><<<gw, 256, 0, st>>>(p.G, p.ldg, ng, nq, p.nprobe, p.gbound, p.gslot);
+  // fewer groups than probes: every group is selected and the slots past them stay padding
+  if (ng < p.nprobe && (e = cudaMemsetAsync(p.cand, 0xff, sizeof(uint64_t) * nq * p.ccap, st)) != cudaSuccess) return e;
+  p.mode = 1;  // pass 1: the same scores, the selected groups' keys stored to their slots
+  k_coarse_gemm<<<grid, 64 + 32 * p.nepi, p.smem_total, st>>>(*cmap, *qmap, p);
+  if ((e = cudaGetLastError()) != cudaSuccess) return e;
   const int R = (p.nprobe + 31) / 32;
-  if (R <= 1) k_probe_select<1><<<g2, 256, 0, st>>>(p.S, p.lds, p.G, p.ldg, nq, p.nlist, p.nprobe, p.probes);
-  else if (R == 2) k_probe_select<2><<<g2, 256, 0, st>>>(p.S, p.lds, p.G, p.ldg, nq, p.nlist, p.nprobe, p.probes);
-  else if (R <= 4) k_probe_select<4><<<g2, 256, 0, st>>>(p.S, p.lds, p.G, p.ldg, nq, p.nlist, p.nprobe, p.probes);
-  else if (R <= 8) k_probe_select<8><<<g2, 256, 0, st>>>(p.S, p.lds, p.G, p.ldg, nq, p.nlist, p.nprobe, p.probes);
-  else if (R <= 16) k_probe_select<16><<<g2, 256, 0, st>>>(p.S, p.lds, p.G, p.ldg, nq, p.nlist, p.nprobe, p.probes);
-  else k_probe_select<32><<<g2, 256, 0, st>>>(p.S, p.lds, p.G, p.ldg, nq, p.nlist, p.nprobe, p.probes);
+  if (R <= 1) k_probe_final<1><<<gw, 256, 0, st>>>(p.cand, p.ccap, nq, p.nprobe, p.probes);
+  else if (R == 2) k_probe_final<2><<<gw, 256, 0, st>>>(p.cand, p.ccap, nq, p.nprobe, p.probes);
+  else if (R <= 4) k_probe_final<4><<<gw, 256, 0, st>>>(p.cand, p.ccap, nq, p.nprobe, p.probes);
+  else if (R <= 8) k_probe_final<8><<<gw, 256, 0, st>>>(p.cand, p.ccap, nq, p.nprobe, p.probes);
+  else if (R <= 16) k_probe_final<16><<<gw, 256, 0, st>>>(p.cand, p.ccap, nq, p.nprobe, p.probes);
+  else k_probe_final<32><<<gw, 256, 0, st>>>(p.cand, p.ccap, nq, p.nprobe, p.probes);
   return cudaGetLastError();
 }
 

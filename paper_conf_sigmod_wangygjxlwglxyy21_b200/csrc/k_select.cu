@@ -157,6 +157,7 @@ __global__ void __launch_bounds__(256) k_final_select(const int64_t* __restrict_
 // 256 < k: the CTA-per-query select's block size (32 warps: one CTA per SM when the candidate stage
 // takes all of shared memory, so the warps are the only latency hiding) and private histograms
 constexpr int kBigThreads = 1024;
+constexpr int kHistWarps = 8;  // private radix histograms (warps w, w + 8, ... share one)
 
 // Ascending bitonic sort of NK = kBigThreads E keys in shared memory by a kBigThreads block.  Warp w holds
 // the contiguous block [32 E w, 32 E (w + 1)) in registers, lane l element 32 j + l in v[j]:
@@ -222,55 +223,10 @@ __device__ __forceinline__ void block_sort_regs(uint64_t* win, int NK) {
   for (int j = 0; j < E; ++j) win[wbase + 32 * j + lane] = v[j];
 }
 
-// 256 < k: one CTA (kBigThreads threads) per query stages the query's candidates in shared memory
-// (when they fit, else it flags the query for k_final_select's global-memory path), then a radix
-// select over the u64 keys below their common prefix: 12-bit digits, one shared histogram with
-// warp-aggregated atomics (__match_any: near-neighbour keys crowd a few bins), a block scan for
-// the digit.  As soon as the digit's boundary bin holds <= kBoundBig keys, one gather pass moves
-// the keys below it to the winners (ballot-aggregated appends) and the boundary keys to a small
-// buffer that is sorted to complete the k; otherwise the next digit refines the boundary bin
-// (u64 keys are unique, so this ends).  Then a bitonic sort of the k winners.
-constexpr int kDigitBits = 12;
-constexpr int kBins = 1 << kDigitBits;
-constexpr int kBoundBig = kBins / 2;  // boundary keys gathered into the histogram's space (u64)
-
-// exclusive scan of kBins bins held by the kBigThreads threads (4 per thread): the thread whose
-// range holds the k-th key (counting from `below`) writes {bin, keys before the bin, keys in it}
-__device__ __forceinline__ void big_find_digit(const uint32_t* hist, int below, int k, int* red, int* s_int) {
-  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
-  constexpr int PER = kBins / kBigThreads;
-  uint32_t c[PER], tot = 0;
-#pragma unroll
-  for (int j = 0; j < PER; ++j) {
-    c[j] = hist[tid * PER + j];
-    tot += c[j];
-  }
-  uint32_t incl = tot;
-  for (int o = 1; o < 32; o <<= 1) {
-    const uint32_t v = __shfl_up_sync(MV_FULL, incl, o);
-    if (lane >= o) incl += v;
-  }
-  if (lane == 31) red[wid] = (int)incl;
-  __syncthreads();
-  if (wid == 0) {
-    int w = lane < kBigThreads / 32 ? red[lane] : 0;
-    for (int o = 1; o < 32; o <<= 1) {
-      const int v = __shfl_up_sync(MV_FULL, w, o);
-      if (lane >= o) w += v;
-    }
-    red[32 + lane] = w;  // inclusive scan of the warp totals
-  }
-  __syncthreads();
-  uint32_t cum = (uint32_t)below + (wid ? (uint32_t)red[32 + wid - 1] : 0u) + incl - tot;
-  if (cum < (uint32_t)k && cum + tot >= (uint32_t)k) {
-    int d = 0;
-    while (cum + c[d] < (uint32_t)k) cum += c[d++];
-    s_int[0] = tid * PER + d;
-    s_int[1] = (int)cum;
-    s_int[2] = (int)c[d];
-  }
-  __syncthreads();
-}
+// 256 < k: one CTA (kBigThreads threads) per query stages the query's candidates in shared memory (when
+// they fit, else it flags the query for k_final_select's global-memory path), then an MSB radix
+// select over the u64 keys -- 8-bit digits, histogram per pass in shared memory, stopping as soon
+// as the keys at or below the current prefix are exactly k -- and a bitonic sort of the k winners.
 
 __global__ void __launch_bounds__(kBigThreads) k_final_big(const int64_t* __restrict__ poff,
                                                            const int32_t* __restrict__ pcnt,
@@ -278,20 +234,22 @@ __global__ void __launch_bounds__(kBigThreads) k_final_big(const int64_t* __rest
                                                            int metric, const int64_t* __restrict__ sorted_ids,
                                                            float* out_d, int64_t* out_i, int cap,
                                                            const int32_t* __restrict__ nuse, uint64_t* tau_out,
-                                                           uint8_t* over, const int* __restrict__ gate) {
+                                                           uint8_t* over, const int* __restrict__ gate,
+                                                           const uint8_t* __restrict__ only) {
   if (gate && *gate == 0) return;
+  if (only && !only[blockIdx.x]) {  // done by k_final_sample
+    if (threadIdx.x == 0) over[blockIdx.x] = 0;
+    return;
+  }
   extern __shared__ __align__(16) uint8_t smem[];
   const int NK = next_pow2(max(k, 2));
   uint64_t* buf = reinterpret_cast<uint64_t*>(smem);   // cap
   uint64_t* win = buf + cap;                           // NK
-  uint32_t* hist = reinterpret_cast<uint32_t*>(win + NK);  // kBins u32; later the boundary keys (kBoundBig u64)
-  uint64_t* bnd = reinterpret_cast<uint64_t*>(hist);
-  int32_t* s_pre = reinterpret_cast<int32_t*>(hist + kBins);  // npb + 1
-  int32_t* s_int = s_pre + npb + 1;                    // misc (8)
-  int32_t* red = s_int + 8;                            // 64
+  uint32_t* whist = reinterpret_cast<uint32_t*>(win + NK);  // kHistWarps x 256 (>= 66 u64 for the min/max)
+  int32_t* s_pre = reinterpret_cast<int32_t*>(whist + kHistWarps * 256);  // npb + 1
+  int32_t* s_int = s_pre + npb + 1;                    // misc
   const int64_t q = blockIdx.x;
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
-  const uint32_t ltmask = (1u << lane) - 1;
   const int64_t* po = poff + q * npb;
   const int32_t* pc = pcnt + q * npb;
   const int nu = nuse ? nuse[q] : npb;
@@ -316,7 +274,7 @@ __global__ void __launch_bounds__(kBigThreads) k_final_big(const int64_t* __rest
     if (tid == 0) over[q] = 1;
     return;
   }
-  if (tid == 0 && over) over[q] = 0;
+  if (tid == 0) over[q] = 0;
   // staging by fire-and-forget 8-B async copies: every lane keeps its loads in flight (a plain
   // load/store loop was latency-bound: one ~1 us global round trip per 32 keys per warp)
   for (int j = wid; j < nu; j += kBigThreads / 32) {
@@ -329,10 +287,15 @@ __global__ void __launch_bounds__(kBigThreads) k_final_big(const int64_t* __rest
   asm volatile("cp.async.wait_all;" ::: "memory");
   __syncthreads();
   int nsel;  // winners to sort, in win[]
-  if (T < k || (T == k && tau_out == nullptr)) {
+  if (T <= k) {
     for (int i = tid; i < NK; i += kBigThreads) win[i] = i < T ? buf[i] : MV_KEY_PAD;
     nsel = T;
-  } else {  // (the seeding select with exactly k candidates also needs the k-th key)
+  } else {
+    // radix select over the bits below the keys' common prefix: the first digit starts at the
+    // highest bit where the smallest and largest key differ (near-neighbour distance keys share
+    // their top ~10 bits, which a fixed MSB digit would pile into one contended bin).  8-bit
+    // digits, per-warp private histograms, a warp prefix scan for the digit; it stops as soon as
+    // the keys at or below the current prefix are exactly k (keys are unique).
     uint64_t mn = MV_KEY_PAD, mx = 0;
     for (int i = tid; i < T; i += kBigThreads) {
       const uint64_t x = buf[i];
@@ -343,88 +306,96 @@ __global__ void __launch_bounds__(kBigThreads) k_final_big(const int64_t* __rest
       mn = umin64(mn, shfl_xor64(mn, o));
       mx = umax64(mx, shfl_xor64(mx, o));
     }
-    uint64_t* r64 = reinterpret_cast<uint64_t*>(hist);
+    uint64_t* red = reinterpret_cast<uint64_t*>(whist);
     if (lane == 0) {
-      r64[wid] = mn;
-      r64[32 + wid] = mx;
+      red[wid] = mn;
+      red[32 + wid] = mx;
     }
     __syncthreads();
     if (tid == 0) {
       for (int w = 1; w < kBigThreads / 32; ++w) {
-        mn = umin64(mn, r64[w]);
-        mx = umax64(mx, r64[32 + w]);
+        mn = umin64(mn, red[w]);
+        mx = umax64(mx, red[32 + w]);
       }
-      r64[64] = mn;
-      r64[65] = mx;
+      red[64] = mn;
+      red[65] = mx;
     }
     __syncthreads();
-    mn = r64[64];
-    mx = r64[65];
+    mn = red[64];
+    mx = red[65];
     __syncthreads();
     int lo = 64 - __clzll((long long)(mn ^ mx));  // bits [lo, 64) are common to every key
     uint64_t pfx = lo >= 64 ? 0 : (mn >> lo);
-    int below = 0, nb = 0;
-    for (;;) {  // digits until the boundary bin is small enough to gather
-      const int w = min(kDigitBits, lo), sh = lo - w;
+    int below = 0;  // keys whose bits above lo are < pfx
+    for (;;) {
+      const int w = min(8, lo), sh = lo - w;
       const uint32_t dmask = (1u << w) - 1;
-      for (int i = tid; i < kBins; i += kBigThreads) hist[i] = 0;
+      for (int i = tid; i < kHistWarps * 256; i += kBigThreads) whist[i] = 0;
       __syncthreads();
-      for (int b0 = 0; b0 < T; b0 += kBigThreads) {
-        const int i = b0 + tid;
-        uint32_t bin = 0xffffffffu;
-        if (i < T) {
-          const uint64_t x = buf[i];
-          if (lo >= 64 || (x >> lo) == pfx) bin = (uint32_t)(x >> sh) & dmask;
-        }
-        const uint32_t peers = __match_any_sync(MV_FULL, bin);
-        if (bin != 0xffffffffu && (__ffs(peers) - 1) == lane) atomicAdd(hist + bin, (uint32_t)__popc(peers));
+      uint32_t* hw = whist + (wid % kHistWarps) * 256;
+      for (int i = tid; i < T; i += kBigThreads) {
+        const uint64_t x = buf[i];
+        if (lo >= 64 || (x >> lo) == pfx) atomicAdd(hw + ((uint32_t)(x >> sh) & dmask), 1u);
       }
       __syncthreads();
-      big_find_digit(hist, below, k, red, s_int);
+      if (wid == 0) {  // bins 8 * lane .. 8 * lane + 7, summed over the private histograms
+        uint32_t c[8];
+        uint32_t tot = 0;
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+          uint32_t v = 0;
+          for (int h = 0; h < kHistWarps; ++h) v += whist[h * 256 + 8 * lane + j];
+          c[j] = v;
+          tot += v;
+        }
+        uint32_t incl = tot;
+        for (int o = 1; o < 32; o <<= 1) {
+          const uint32_t v = __shfl_up_sync(MV_FULL, incl, o);
+          if (lane >= o) incl += v;
+        }
+        uint32_t cum = below + incl - tot;  // keys before this lane's first bin
+        const bool mine = cum < (uint32_t)k && cum + tot >= (uint32_t)k;
+        if (mine) {
+          int d = 0;
+          while (cum + c[d] < (uint32_t)k) cum += c[d++];
+          s_int[0] = 8 * lane + d;
+          s_int[1] = (int)cum;
+          s_int[2] = cum + c[d] == (uint32_t)k;
+        }
+      }
+      __syncthreads();
       pfx = (pfx << w) | (uint64_t)s_int[0];
       below = s_int[1];
-      nb = s_int[2];
       lo = sh;
+      const bool done = s_int[2] || lo == 0;
       __syncthreads();
-      if (nb <= kBoundBig || lo == 0) break;
+      if (done) break;
     }
-    // gather: keys below the boundary bin -> win (exactly `below` of them), the bin's keys -> bnd
-    if (tid == 0) {
-      s_int[3] = 0;
-      s_int[4] = 0;
-    }
+    // winners: keys whose bits above lo are <= pfx (exactly k: keys are unique)
+    if (tid == 0) s_int[3] = 0;
     __syncthreads();
-    for (int b0 = 0; b0 < T; b0 += kBigThreads) {
-      const int i = b0 + tid;
-      const uint64_t x = i < T ? buf[i] : MV_KEY_PAD;
+    for (int i = tid; i < T; i += kBigThreads) {
+      const uint64_t x = buf[i];
       const uint64_t top = lo >= 64 ? 0 : (x >> lo);
-      const bool isw = i < T && top < pfx, isb = i < T && top == pfx;
-      const uint32_t mw = __ballot_sync(MV_FULL, isw), mb = __ballot_sync(MV_FULL, isb);
-      int ow = 0, ob = 0;
-      if (lane == 0) {
-        if (mw) ow = atomicAdd(s_int + 3, __popc(mw));
-        if (mb) ob = atomicAdd(s_int + 4, __popc(mb));
-      }
-      ow = __shfl_sync(MV_FULL, ow, 0);
-      ob = __shfl_sync(MV_FULL, ob, 0);
-      if (isw) win[ow + __popc(mw & ltmask)] = x;
-      if (isb && ob + __popc(mb & ltmask) < kBoundBig) bnd[ob + __popc(mb & ltmask)] = x;
+      if (top <= pfx) win[atomicAdd(s_int + 3, 1)] = x;
     }
     __syncthreads();
-    const int nbb = min(nb, kBoundBig);
-    const int NB = next_pow2(max(nbb, 2));
-    for (int i = nbb + tid; i < NB; i += kBigThreads) bnd[i] = MV_KEY_PAD;
-    block_bitonic_sort(bnd, NB);
-    for (int i = tid; i < k - below; i += kBigThreads) win[below + i] = bnd[i];
     nsel = k;
     for (int i = k + tid; i < NK; i += kBigThreads) win[i] = MV_KEY_PAD;
-    if (tau_out) {  // seeding: the k-th best key
-      if (tid == 0) tau_out[q] = bnd[k - below - 1];
-      return;
-    }
   }
   __syncthreads();
-  if (tau_out) {  // fewer than k candidates: tau stays untouched
+  if (tau_out) {  // seeding: only the k-th best key is needed (the largest winner)
+    if (nsel < k) return;
+    uint64_t m = 0;
+    for (int i = tid; i < k; i += kBigThreads) m = umax64(m, win[i]);
+    for (int o = 16; o > 0; o >>= 1) m = umax64(m, shfl_xor64(m, o));
+    if (lane == 0) buf[wid] = m;
+    __syncthreads();
+    if (tid == 0) {
+      uint64_t mm = 0;
+      for (int w = 0; w < kBigThreads / 32; ++w) mm = umax64(mm, buf[w]);
+      tau_out[q] = mm;
+    }
     return;
   }
   // bitonic sort of the NK winners: register-blocked (strides < 32 E by shuffles and in registers,
@@ -452,31 +423,264 @@ __global__ void __launch_bounds__(kBigThreads) k_final_big(const int64_t* __rest
   }
 }
 
-// k > 256: k_final_big for every query whose candidates fit its shared-memory stage (cap keys),
-// k_final_select (global-memory radix) for the others -- launched only when some query could
-// exceed cap (tmax = an upper bound of the candidates per query)
+
+// 256 < k <= 4096 (the common large-k case, configs[3]'s k = 2048): a sample-threshold select
+// that reads each candidate key once and sorts only the k winners.  One CTA per query, no staging
+// of the candidates (two CTAs share an SM):
+//   1. kSamp keys at a uniform stride; the sample's js-th smallest distance key (js ~ 1.25 k kSamp
+//      / T + 12, found by bisection with block counts) is a threshold t expected a little above the
+//      k-th key;
+//   2. one pass gathers the keys <= t (ballot-aggregated appends) into a window of wcap keys; when
+//      k <= count <= wcap the window holds the top-k (else t moves, up to two more passes, and
+//      failing that the query is flagged for the staged radix select k_final_big, exact for any
+//      input);
+//   3. the k-th key of the window by bisection (distance key, then the tied id ranks), the k
+//      winners compacted, and a bitonic sort of those k alone (the seeding select stops at the
+//      k-th key: no sort at all).
+constexpr int kSamp = kBigThreads;
+constexpr int kGU = 8;  // gather: keys per lane per step
+
+// number of values in v[0..E) (per thread, masked by cnt) below `trial`, summed over the block
+template <int E>
+__device__ __forceinline__ int block_count_below(const uint32_t (&v)[E], int nv, uint32_t trial, int* cell) {
+  int c = 0;
+#pragma unroll
+  for (int j = 0; j < E; ++j) c += (j < nv && v[j] < trial) ? 1 : 0;
+  c = (int)__reduce_add_sync(MV_FULL, (uint32_t)c);
+  __syncthreads();
+  if (threadIdx.x == 0) *cell = 0;
+  __syncthreads();
+  if ((threadIdx.x & 31) == 0 && c) atomicAdd(cell, c);
+  __syncthreads();
+  return *cell;
+}
+
+// the r-th smallest (1-based) of the u32 values held per thread (E each, nv valid): MSB bisection
+template <int E>
+__device__ __forceinline__ uint32_t block_select_u32(const uint32_t (&v)[E], int nv, int r, int* cell) {
+  uint32_t b = 0;
+  for (int bit = 31; bit >= 0; --bit) {
+    const uint32_t trial = b | (1u << bit);
+    if (block_count_below<E>(v, nv, trial, cell) < r) b = trial;
+  }
+  return b;
+}
+
+__global__ void __launch_bounds__(kBigThreads) k_final_sample(const int64_t* __restrict__ poff,
+                                                              const int32_t* __restrict__ pcnt,
+                                                              const uint64_t* __restrict__ part, int64_t nq, int npb,
+                                                              int k, int metric, const int64_t* __restrict__ sorted_ids,
+                                                              float* out_d, int64_t* out_i, int wcap,
+                                                              const int32_t* __restrict__ nuse, uint64_t* tau_out,
+                                                              uint8_t* redo, const int* __restrict__ gate) {
+  if (gate && *gate == 0) return;
+  extern __shared__ __align__(16) uint8_t smem[];
+  const int NK = next_pow2(max(k, 2));
+  uint64_t* win = reinterpret_cast<uint64_t*>(smem);  // wcap (<= 4 kBigThreads)
+  uint64_t* top = win + wcap;                          // NK: the winners
+  int32_t* s_pre = reinterpret_cast<int32_t*>(top + NK);  // npb + 1
+  int32_t* s_int = s_pre + npb + 1;                    // misc (4)
+  const int64_t q = blockIdx.x;
+  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  const uint32_t ltmask = (1u << lane) - 1;
+  const int64_t* po = poff + q * npb;
+  const int32_t* pc = pcnt + q * npb;
+  const int nu = nuse ? nuse[q] : npb;
+  if (wid == 0) {
+    int run = 0;
+    for (int j0 = 0; j0 < nu; j0 += 32) {
+      const int j = j0 + lane;
+      const int c = j < nu ? pc[j] : 0;
+      int incl = c;
+      for (int o = 1; o < 32; o <<= 1) {
+        const int v = __shfl_up_sync(MV_FULL, incl, o);
+        if (lane >= o) incl += v;
+      }
+      if (j < nu) s_pre[j] = run + incl - c;
+      run += __shfl_sync(MV_FULL, incl, 31);
+    }
+    if (lane == 0) s_pre[nu] = run;
+  }
+  __syncthreads();
+  const int T = s_pre[nu];
+  if (tid == 0) redo[q] = 0;
+  // gather every key <= t into win (first wcap of them); returns the number of keys <= t
+  auto gather = [&](uint64_t t) {
+    if (tid == 0) s_int[0] = 0;
+    __syncthreads();
+    for (int j = wid; j < nu; j += kBigThreads / 32) {
+      const int c = s_pre[j + 1] - s_pre[j];
+      const uint64_t* src = part + po[j];
+      for (int i0 = 0; i0 < c; i0 += 32 * kGU) {  // kGU loads per lane in flight
+        uint64_t x[kGU];
+#pragma unroll
+        for (int u = 0; u < kGU; ++u) {
+          const int i = i0 + 32 * u + lane;
+          x[u] = i < c ? __ldg(src + i) : MV_KEY_PAD;
+        }
+#pragma unroll
+        for (int u = 0; u < kGU; ++u) {
+          const bool p = i0 + 32 * u + lane < c && x[u] <= t;
+          const uint32_t m = __ballot_sync(MV_FULL, p);
+          if (m) {
+            int base = 0;
+            if (lane == 0) base = atomicAdd(s_int, __popc(m));
+            base = __shfl_sync(MV_FULL, base, 0);
+            const int pos = base + __popc(m & ltmask);
+            if (p && pos < wcap) win[pos] = x[u];
+          }
+        }
+      }
+    }
+    __syncthreads();
+    return s_int[0];
+  };
+  int cnt;
+  if (T <= wcap) {
+    cnt = gather(MV_KEY_PAD);
+  } else {
+    uint32_t sv[1];
+    {  // the uniform-stride sample: thread i takes candidate floor(i T / kSamp) (its distance key)
+      const int pos = (int)((int64_t)tid * T / kSamp);
+      int lo = 0, hi = nu - 1;
+      while (lo < hi) {
+        const int mid = (lo + hi + 1) >> 1;
+        if (s_pre[mid] <= pos) lo = mid; else hi = mid - 1;
+      }
+      sv[0] = (uint32_t)(part[po[lo] + (pos - s_pre[lo])] >> 32);
+    }
+    int js = min(kSamp - 1, (int)((double)kSamp * k * 1.25 / T) + 12);
+    int lo_ok = -1, hi_bad = kSamp;  // sample ranks known too low (< k keys) / too high (> wcap)
+    cnt = -1;
+    for (int attempt = 0; attempt < 3; ++attempt) {
+      const uint32_t td = block_select_u32<1>(sv, 1, js + 1, s_int + 1);
+      const int c = gather(((uint64_t)td << 32) | 0xffffffffull);
+      if (c >= k && c <= wcap) {
+        cnt = c;
+        break;
+      }
+      if (c < k) lo_ok = js; else hi_bad = js;
+      const int nj = c < k ? min(kSamp - 1, js + max(8, (js + 1) / 4)) : (lo_ok + js) / 2;
+      if (nj == js || nj <= lo_ok || nj >= hi_bad) break;
+      js = nj;
+    }
+    if (cnt < 0) {  // the staged radix select takes this query
+      if (tid == 0) redo[q] = 1;
+      return;
+    }
+  }
+  const int n = min(cnt, wcap);
+  int nsel = n;
+  if (n > k) {
+    // the k-th key of the window: its distance key by bisection, then the tied ranks
+    constexpr int E = 4;  // wcap <= 4 kBigThreads
+    uint32_t dv[E];
+#pragma unroll
+    for (int j = 0; j < E; ++j) dv[j] = j * kBigThreads + tid < n ? (uint32_t)(win[j * kBigThreads + tid] >> 32) : 0u;
+    const int nv = (n - tid + kBigThreads - 1) / kBigThreads;
+    const uint32_t dk = block_select_u32<E>(dv, nv, k, s_int + 1);
+    const int below = block_count_below<E>(dv, nv, dk, s_int + 1);  // keys with a smaller distance key
+    uint32_t rv[E];
+#pragma unroll
+    for (int j = 0; j < E; ++j)
+      rv[j] = (j < nv && dv[j] == dk) ? (uint32_t)win[j * kBigThreads + tid] : 0xffffffffu;
+    const uint32_t rk = block_select_u32<E>(rv, nv, k - below, s_int + 1);
+    const uint64_t kth = ((uint64_t)dk << 32) | rk;
+    if (tau_out) {
+      if (tid == 0) tau_out[q] = kth;
+      return;
+    }
+    // compact the k winners (keys are unique: exactly k are <= kth)
+    if (tid == 0) s_int[0] = 0;
+    __syncthreads();
+    for (int j = 0; j < E; ++j) {
+      const int i = j * kBigThreads + tid;
+      const uint64_t x = i < n ? win[i] : MV_KEY_PAD;
+      const bool p = i < n && x <= kth;
+      const uint32_t m = __ballot_sync(MV_FULL, p);
+      int base = 0;
+      if (lane == 0 && m) base = atomicAdd(s_int, __popc(m));
+      base = __shfl_sync(MV_FULL, base, 0);
+      if (p) top[base + __popc(m & ltmask)] = x;
+    }
+    nsel = k;
+  } else {
+    if (tau_out) {  // fewer than k candidates: tau untouched; exactly k: the largest
+      if (n == k) {
+        uint64_t m = 0;
+        for (int i = tid; i < n; i += kBigThreads) m = umax64(m, win[i]);
+        for (int o = 16; o > 0; o >>= 1) m = umax64(m, shfl_xor64(m, o));
+        if (lane == 0) top[wid] = m;
+        __syncthreads();
+        if (tid == 0) {
+          for (int w = 1; w < kBigThreads / 32; ++w) m = umax64(m, top[w]);
+          tau_out[q] = m;
+        }
+      }
+      return;
+    }
+    for (int i = tid; i < n; i += kBigThreads) top[i] = win[i];
+  }
+  __syncthreads();
+  for (int i = nsel + tid; i < NK; i += kBigThreads) top[i] = MV_KEY_PAD;
+  switch (NK / kBigThreads) {
+    case 1: block_sort_regs<1>(top, NK); break;
+    case 2: block_sort_regs<2>(top, NK); break;
+    case 4: block_sort_regs<4>(top, NK); break;
+    default: block_sort_regs<0>(top, NK); break;
+  }
+  __syncthreads();
+  for (int i = tid; i < k; i += kBigThreads) {
+    float dv;
+    int64_t iv;
+    const uint64_t key = i < nsel ? top[i] : MV_KEY_PAD;
+    if (key != MV_KEY_PAD) {
+      dv = key_dist((uint32_t)(key >> 32), metric);
+      iv = sorted_ids[(uint32_t)(key & 0xffffffffu)];
+    } else {
+      dv = metric == MV_L2 ? __int_as_float(0x7f800000) : __int_as_float(0xff800000);
+      iv = -1;
+    }
+    out_d[q * k + i] = dv;
+    out_i[q * k + i] = iv;
+  }
+}
+
 static cudaError_t launch_big_select(const int64_t* poff, const int32_t* pcnt, const uint64_t* part, int64_t nq,
                                      int npb, int k, int metric, const int64_t* sorted_ids, float* out_d,
                                      int64_t* out_i, const int32_t* nuse, uint64_t* tau, int64_t tmax,
-                                     uint8_t* over, const int* gate, cudaStream_t st) {
+                                     uint8_t* over, const int* gate, int big_mode, cudaStream_t st) {
+  cudaError_t e;
+  // over: 2 nq bytes -- [0, nq) queries past k_final_big's stage, [nq, 2 nq) k_final_sample's redo flags
+  uint8_t* redo = over ? over + nq : nullptr;
+  if (redo && k <= 3072 && big_mode == 1) {
+    const int wcap = 4 * kBigThreads;  // >= k + the threshold's slack for k <= 2048; less for larger k
+    const size_t smem = (size_t)(wcap + next_pow2(max(k, 2))) * 8 + (size_t)(npb + 1) * 4 + 64;
+    if ((e = cudaFuncSetAttribute(k_final_sample, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)) != cudaSuccess)
+      return e;
+    k_final_sample<<<(unsigned)nq, kBigThreads, smem, st>>>(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d,
+                                                            out_i, wcap, nuse, tau, redo, gate);
+  } else {
+    redo = nullptr;
+  }
   const int NK = next_pow2(max(k, 2));
-  const int fixed = NK * 8 + kBins * 4 + (npb + 1) * 4 + 72 * 4 + 64;
+  const int fixed = NK * 8 + kHistWarps * 256 * 4 + (npb + 1) * 4 + 64 + 64;
   // stage capacity: all of shared memory, or just the bound tmax when that is smaller (several
   // CTAs per SM: the seeding select's candidates are bounded by the phase-A prefixes)
   const int cap = (int)min64((227 * 1024 - fixed) / 8, max64(tmax, k));
   if (over && cap >= k) {
     const size_t smem = (size_t)cap * 8 + fixed;
-    cudaError_t e = cudaFuncSetAttribute(k_final_big, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    e = cudaFuncSetAttribute(k_final_big, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     k_final_big<<<(unsigned)nq, kBigThreads, smem, st>>>(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d,
-                                                         out_i, cap, nuse, tau, over, gate);
+                                                         out_i, cap, nuse, tau, over, gate, redo);
     if (tmax <= cap) return cudaGetLastError();
   } else {
     over = nullptr;
   }
   const int selcap = max(4096, next_pow2(k));
   size_t smem = (size_t)(selcap + kBoundCap) * 8 + (size_t)(npb + 1) * 4 + 256 * 4 + 8 * 4 + 64;
-  cudaError_t e = cudaFuncSetAttribute(k_final_select, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  e = cudaFuncSetAttribute(k_final_select, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   k_final_select<<<(unsigned)nq, 256, smem, st>>>(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d, out_i,
                                                   selcap, nuse, tau, over, gate);
@@ -635,23 +839,23 @@ static bool launch_warp_select(const int64_t* poff, const int32_t* pcnt, const u
 
 cudaError_t launch_final_select(const int64_t* poff, const int32_t* pcnt, const uint64_t* part, int64_t nq, int npb,
                                 int k, int metric, const int64_t* sorted_ids, float* out_d, int64_t* out_i,
-                                int64_t tmax, uint8_t* over, cudaStream_t st) {
+                                int64_t tmax, uint8_t* over, int big_mode, cudaStream_t st) {
   if (nq == 0) return cudaSuccess;
   if (launch_warp_select(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d, out_i, nullptr, nullptr, nullptr,
                          st))
     return cudaGetLastError();
   return launch_big_select(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d, out_i, nullptr, nullptr, tmax,
-                           over, nullptr, st);
+                           over, nullptr, big_mode, st);
 }
 
 cudaError_t launch_tau_select(const int64_t* poff, const int32_t* pcnt, const uint64_t* part, int64_t nq, int npb,
                               const int32_t* nuse, int k, uint64_t* tau, int64_t tmax, uint8_t* over,
-                              const int* gate, cudaStream_t st) {
+                              const int* gate, int big_mode, cudaStream_t st) {
   if (nq == 0) return cudaSuccess;
   if (launch_warp_select(poff, pcnt, part, nq, npb, k, MV_L2, nullptr, nullptr, nullptr, nuse, tau, gate, st))
     return cudaGetLastError();
   return launch_big_select(poff, pcnt, part, nq, npb, k, MV_L2, nullptr, nullptr, nullptr, nuse, tau, tmax, over, gate,
-                           st);
+                           big_mode, st);
 }
 
 // ------------------------------------------------------------------------------------------

@@ -235,11 +235,13 @@ static cudaError_t run_coarse(mv_index* ix, const float* qhl, const int* qlo_any
   cp.metric = ix->metric;
   cp.cnorm = ix->cnorm;
   cp.probes = P;
-  cp.lds = (ix->nlist + 3) & ~3;
   cp.ldg = ((ix->nlist + 127) / 128) * 4;
+  cp.ccap = 32 * npb;
   cp.qlo_any = qlo_any;
-  cudaError_t e = s.alloc(&cp.S, (size_t)nq * cp.lds);
-  if (e == cudaSuccess) e = s.alloc(&cp.G, (size_t)nq * cp.ldg);
+  cudaError_t e = s.alloc(&cp.G, (size_t)nq * cp.ldg);
+  if (e == cudaSuccess) e = s.alloc(&cp.gbound, (size_t)nq);
+  if (e == cudaSuccess) e = s.alloc(&cp.cand, (size_t)nq * cp.ccap);
+  if (e == cudaSuccess) e = s.alloc(&cp.gslot, (size_t)nq * ((ix->nlist + 31) / 32));
   if (e != cudaSuccess) return e;
   ix->last_coarse = "tcgen05.tf32";
   return launch_coarse_tc(&ix->cmap, &qmap, cp, nq, st);
@@ -250,7 +252,7 @@ static int64_t search_bytes_per_query(const mv_index* ix, int npb, int k) {
   const int64_t cand = ix->top_len_prefix[std::min<size_t>(npb, ix->top_len_prefix.size() - 1)];
   const int64_t need = std::max<int64_t>(2 * (int64_t)k, k + 32);
   const int64_t seed = std::min<int64_t>(65536, std::max<int64_t>(need, 4096)) + 4096;
-  const int64_t coarse = npb < ix->nlist ? 4 * (int64_t)((ix->nlist + 3) & ~3) + (int64_t)ix->nlist / 8 : 0;
+  const int64_t coarse = npb < ix->nlist ? (int64_t)ix->nlist / 8 + 256 * (int64_t)npb + 16 : 0;
   return 8 * (cand + seed) + coarse + 48 * (int64_t)npb + 32 * (int64_t)ix->dpad + 64;
 }
 
@@ -329,6 +331,7 @@ mv_status mv_index_set_option(mv_index* ix, const char* name, int64_t value) {
   else if (n == "coarse_epi") o.coarse_epi = (int)std::min<int64_t>(value, 16);
   else if (n == "coarse_nacc") o.coarse_nacc = (int)std::min<int64_t>(value, 4);
   else if (n == "workspace_bytes") o.workspace = value;
+  else if (n == "large_k_select") o.large_k_select = value != 0;
   else return fail(MV_EINVAL, "unknown option '%s'", name);
   return MV_OK;
 }
@@ -451,11 +454,11 @@ mv_status mv_index_add(mv_index* ix, const float* vectors, const int64_t* ids, i
   CK(s.alloc(&sizes, nlist));
   CK(s.alloc(&new_off, nlist + 1));
   // a0: assignment I(v) = closest centroid -- the tensor-core coarse step with nprobe = 1, in row
-  // blocks whose score matrix stays <= 1 GB
+  // blocks whose group-minimum matrix stays <= 512 MB
   CK(launch_query_prep(x, n, ix->d, dpad, xpad, xnorm, st));
   {
-    const int64_t lds = (nlist + 3) & ~3;
-    const int64_t sub = std::min<int64_t>(n, std::max<int64_t>(4096, (int64_t(1) << 28) / lds));
+    const int64_t ldg = ((nlist + 127) / 128) * 4;
+    const int64_t sub = std::min<int64_t>(n, std::max<int64_t>(4096, (int64_t(1) << 27) / ldg));
     float* qhl;
     CK(s.alloc(&qhl, (size_t)2 * sub * dpad));
     for (int64_t r0 = 0; r0 < n; r0 += sub) {
@@ -601,8 +604,8 @@ mv_status mv_search_probes(mv_index* ix, const float* queries, int64_t nq, int32
   const float* q;
   CK(stage_in(s0, queries, (size_t)nq * ix->d, &q, &sq));
   const bool sp = is_host_ptr(probes);
-  // chunks of queries whose score matrix stays <= 1 GB
-  const int64_t per = 4 * (int64_t)((ix->nlist + 3) & ~3) + 4 * (int64_t)ix->dpad * 2 + 4 * npb + 64;
+  // chunks of queries whose coarse scratch stays <= 1 GB
+  const int64_t per = (int64_t)ix->nlist / 8 + 256 * (int64_t)npb + 8 * (int64_t)ix->dpad + 64;
   const int64_t chunk = std::max<int64_t>(1, std::min<int64_t>(nq, (int64_t(1) << 30) / per));
   for (int64_t q0 = 0; q0 < nq; q0 += chunk) {
     const int64_t m = std::min(chunk, nq - q0);
@@ -714,7 +717,7 @@ static mv_status search_chunk(mv_index* ix, const float* q, int64_t nq, int32_t 
   int64_t cap = nq * tmax;
   if (split) cap += nq * std::min<int64_t>(tmax, pa.need + pa.capA);
   uint8_t* over = nullptr;
-  if (k > 256) CK(s.alloc(&over, (size_t)nq));
+  if (k > 256) CK(s.alloc(&over, (size_t)2 * nq));
   uint64_t* part;
   CK(s.alloc(&part, (size_t)max64(cap, 1)));
   // a5/a6 on the tensor cores
@@ -756,7 +759,8 @@ static mv_status search_chunk(mv_index* ix, const float* q, int64_t nq, int32_t 
   if (split) {
     // ... tau_q = k-th best key of phase A (phase A emits < need + capA candidates per query) ...
     CK(launch_tau_select(b.poff + npairs, b.pcnt + npairs, part, nq, npb, ra, k, tau,
-                         std::min<int64_t>(tmax, pa.need + pa.capA), over, nullptr, st));
+                         std::min<int64_t>(tmax, pa.need + pa.capA), over, nullptr,
+                         ix->opt.large_k_select, st));
     prof_mark(ix, st);
     // ... phase B over every probed pair, emitting keys <= tau_q
     tp.phase = 1;
@@ -774,13 +778,15 @@ static mv_status search_chunk(mv_index* ix, const float* q, int64_t nq, int32_t 
     uint64_t* tau2;
     CK(s.alloc(&tau2, (size_t)nq));
     CK(cudaMemsetAsync(tau2, 0xff, sizeof(uint64_t) * nq, st));
-    CK(launch_tau_select(b.poff, b.pcnt, part, nq, npb, nullptr, k, tau2, tmax, over, gate, st));
+    CK(launch_tau_select(b.poff, b.pcnt, part, nq, npb, nullptr, k, tau2, tmax, over, gate, ix->opt.large_k_select,
+                         st));
     CK(launch_rekey(b.poff, b.pcnt, part, nq, npb, tau2, qerr, ix->metric, qpad, dpad,
                     reinterpret_cast<const float*>(ix->payload), ix->row_of_rank, gate, st));
     ix->launches += 2;
   }
   // a7
-  CK(launch_final_select(b.poff, b.pcnt, part, nq, npb, k, ix->metric, ix->sorted_ids, D, I, tmax, over, st));
+  CK(launch_final_select(b.poff, b.pcnt, part, nq, npb, k, ix->metric, ix->sorted_ids, D, I, tmax, over,
+                         ix->opt.large_k_select, st));
   prof_mark(ix, st);
   ix->last_scan = flat ? "tcgen05.tf32" : "tcgen05.i8";
   // prep, hilo, coarse GEMM + probe select, plan, qplanes, scan A (+ tau select, scan B), final select

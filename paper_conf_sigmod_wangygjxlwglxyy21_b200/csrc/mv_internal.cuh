@@ -177,6 +177,7 @@ struct Options {
   int flat_qc = 0;          // FLAT queries per scan work item (16..96)
   int coarse_nqb = 0, coarse_cs = 0, coarse_epi = 0, coarse_nacc = 0;  // coarse GEMM launch shape
   int64_t workspace = 0;    // per-search scratch budget in bytes (0: half of the free device memory)
+  int large_k_select = 0;   // k > 256: 0 staged radix select, 1 sample-threshold select (radix fallback)
 };
 }  // namespace mv
 
@@ -305,15 +306,23 @@ cudaError_t launch_qplanes(int type, const float* qpad, int64_t nq, int dpad, co
 cudaError_t launch_tf32_check(const float* x, int64_t n, int* flag, cudaStream_t st);
 
 // k_coarse_tc.cu (tcgen05 coarse GEMM -> score matrix S, then a warp-per-query top-nprobe)
+// The coarse step never materialises the nq x nlist score matrix: the same GEMM runs twice
+// (bitwise-identical scores).  Pass 0 writes only the minimum score key of every 32-centroid group
+// (G); k_group_bound picks, per query, the nprobe-th smallest (group minimum, group id) pair; pass
+// 1 appends the (score key, centroid) keys at or below it -- at most 32 nprobe per query -- and a
+// warp per query sorts out the nprobe best (k_probe_final).
 struct CoarseParams {
   int64_t nq;
   int nlist, nchunks, nstage, nprobe, nqb, csplit, tmem_cols, metric, smem_total;
   int nepi, nacc;          // epilogue warps (multiple of 4, <= 16), TMEM accumulators (<= 4)
+  int mode;                // 0: group minima -> G; 1: append keys <= gbound -> cand
   const float* cnorm;
-  float* S;                // nq x lds scores (lds = roundup(nlist, 4))
-  int64_t lds;
-  uint32_t* G;             // nq x ldg: minimum score key of each 32-centroid group (ldg = ceil(nlist/32))
+  uint32_t* G;             // nq x ldg: minimum score key of each 32-centroid group (ldg = 4 ceil(nlist/128))
   int64_t ldg;
+  uint64_t* gbound;        // nq: (bound score key << 32) | bound group id
+  int16_t* gslot;          // nq x ceil(nlist/32): rank of the group among the query's nprobe selected, or -1
+  uint64_t* cand;          // nq x ccap: (score key << 32) | centroid id, PAD for failing centroids
+  int ccap;                // 32 nprobe
   const int* qlo_any;      // device: some query needs its lo plane (nullable = yes)
   int32_t* probes;
 };
@@ -327,12 +336,14 @@ cudaError_t launch_hilo(const float* x, int64_t n, int d, int dpad, float* out, 
 // final select over the pairs of each query; with tau != nullptr instead: tau[q] = the k-th best
 // key over the first nuse[q] pairs of query q (left untouched when they hold fewer than k).
 // tmax bounds the candidates of one query; over (nq bytes, nullable) is scratch for k > 256.
+// big_mode (k > 256): 0 = the staged radix select (default), 1 = the sample-threshold select with
+// the staged radix select as its fallback.  over: 2 nq bytes of scratch for k > 256.
 cudaError_t launch_final_select(const int64_t* poff, const int32_t* pcnt, const uint64_t* part, int64_t nq, int npb,
                                 int k, int metric, const int64_t* sorted_ids, float* out_d, int64_t* out_i,
-                                int64_t tmax, uint8_t* over, cudaStream_t st);
+                                int64_t tmax, uint8_t* over, int big_mode, cudaStream_t st);
 cudaError_t launch_tau_select(const int64_t* poff, const int32_t* pcnt, const uint64_t* part, int64_t nq, int npb,
                               const int32_t* nuse, int k, uint64_t* tau, int64_t tmax, uint8_t* over,
-                              const int* gate, cudaStream_t st);
+                              const int* gate, int big_mode, cudaStream_t st);
 // FLAT filter mode: exact fp64 re-scoring of the keys at or below tau2[q] + 2 qerr[q] (the others
 // become padding); gate (nullable): skipped when *gate == 0
 cudaError_t launch_rekey(const int64_t* poff, const int32_t* pcnt, uint64_t* part, int64_t nq, int npb,

@@ -199,7 +199,7 @@ def test_sq8_sift_l2_conditional(k):
     assert frac > 0.999
 
 
-@pytest.mark.parametrize("k", [300, 1000, 2048, 16384])
+@pytest.mark.parametrize("k", [300, 1000, 2048, 3000, 4096, 16384])
 def test_large_k(k):
     """k > 1024: single-pass radix select == plain top-k of the oracle."""
     n = 20_000
@@ -346,7 +346,7 @@ def test_c2_full_size_sampled():
 
 OPTION_SETS = [{"seeding": 0}, {"need": 1, "capa": 16}, {"flat_qc": 32, "sq8_qc": 16},
                {"coarse_nqb": 64, "coarse_cs": 3, "coarse_epi": 16, "coarse_nacc": 1},
-               {"workspace_bytes": 1 << 20}]
+               {"workspace_bytes": 1 << 20}, {"large_k_select": 1}]
 
 
 @pytest.mark.parametrize("kind,metric,k", [("flat", "l2", 10), ("flat", "l2", 300), ("flat", "ip", 10),
@@ -389,6 +389,22 @@ def test_cuda_pool_allocator_equals_torch_allocator():
         out.append(ix.search(Q.cuda(), 15, 4))
         assert ix.describe()["allocator"] == ("caller" if alloc else "cuda-pool")
     assert torch.equal(out[0][0], out[1][0]) and torch.equal(out[0][1], out[1][1])
+
+
+@pytest.mark.parametrize("nprobe", [1, 5, 33, 100])
+def test_coarse_exact_ties_follow_centroid_ids(nprobe):
+    """Duplicated centroids and integer data: exact score ties everywhere.  The two-pass coarse step
+    (group bound, then the keys at or below it) must return exactly the oracle's order -- best
+    score first, ties by the smaller centroid id (reading R2)."""
+    X, Q = _sift(20_000, 96, n_micro=512)
+    base = kmeans(X, 160, iters=3).round()
+    C = torch.cat([base, base[:96], base[::3]])          # 309 centroids, many exact duplicates
+    Index, _ = _mv()
+    ix = Index(128, "l2", "flat", C.shape[0])
+    ix.set_centroids(C.cuda())
+    P = ix.search_probes(Q.cuda(), nprobe).cpu().numpy()
+    Po = O.probe(Q.numpy(), C.numpy(), nprobe, O.L2)
+    assert np.array_equal(P, Po)
 
 
 @pytest.mark.parametrize("nprobe", [200, 700, 1024])
