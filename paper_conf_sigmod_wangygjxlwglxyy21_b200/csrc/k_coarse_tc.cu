@@ -51,6 +51,12 @@ __global__ void __launch_bounds__(kCThreads, 1)
   const int qb = blockIdx.x / p.csplit, cs = blockIdx.x % p.csplit;
   const int t0 = (int)((int64_t)ntiles_all * cs / p.csplit), t1 = (int)((int64_t)ntiles_all * (cs + 1) / p.csplit);
   const int q0 = qb * NQB;
+  // tf32-exact queries (device flag): no lo plane, so the B buffer holds the hi rows of 2 NQB
+  // queries and every MMA is N = 2 NQB wide -- half the centroid stream per query; the odd query
+  // blocks' CTAs have nothing to do
+  const bool wide = p.qlo_any != nullptr && *p.qlo_any == 0;
+  if (wide && (qb & 1)) return;
+  const int NQW = wide ? 2 * NQB : NQB;  // queries of this CTA
 
   uint8_t* Bs = sm;                                       // nchunks x BROWS x 128 B
   uint8_t* As = Bs + nchunks * BROWS * ATOM;              // nstage x (hi chunk, lo chunk)
@@ -61,7 +67,6 @@ __global__ void __launch_bounds__(kCThreads, 1)
   uint64_t* tfull = full_b + 1;
   uint64_t* tempty = tfull + 4;
   uint32_t* tslot = reinterpret_cast<uint32_t*>(tempty + 4);
-  uint64_t* sbound = reinterpret_cast<uint64_t*>(tslot + 2);  // pass 1: the block's per-query bounds
   const int nacc = p.nacc;
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -77,9 +82,6 @@ __global__ void __launch_bounds__(kCThreads, 1)
     }
     fence_mbar_init();
   }
-  if (p.mode == 1)
-    for (int i = threadIdx.x; i < NQB; i += blockDim.x)
-      sbound[i] = q0 + i < p.nq ? p.gbound[q0 + i] : 0ull;
   if (warp == 1) {
     tmem_alloc(tslot, p.tmem_cols);
     tmem_relinquish();
@@ -96,10 +98,11 @@ __global__ void __launch_bounds__(kCThreads, 1)
   if (warp == 0) {
     if (lane == 0) {
       // query block: hi rows [q0, q0+NQB) and lo rows [nq + q0, ...) of the plane-major matrix
+      // (wide: the hi rows of [q0, q0 + 2 NQB))
       mbar_expect_tx(full_b, nchunks * BROWS * ATOM);
       for (int c = 0; c < nchunks; ++c) {
         tma_load_2d(Bs + c * BROWS * ATOM, &qmap, full_b, c * 32, q0);
-        tma_load_2d(Bs + c * BROWS * ATOM + NQB * ATOM, &qmap, full_b, c * 32, (int)p.nq + q0);
+        tma_load_2d(Bs + c * BROWS * ATOM + NQB * ATOM, &qmap, full_b, c * 32, wide ? q0 + NQB : (int)p.nq + q0);
       }
       uint32_t it = 0;
       for (int t = t0; t < t1; ++t)
@@ -115,14 +118,14 @@ __global__ void __launch_bounds__(kCThreads, 1)
     if (lane == 0) {
       mbar_wait(full_b, 0);
       tc_fence_after();
-      const uint32_t id_q = idesc_tf32(NQB);
-      const bool qlo = p.qlo_any == nullptr || *p.qlo_any != 0;  // C_hi . Q_lo vanishes for tf32-exact queries
+      const uint32_t id_q = idesc_tf32(NQW);
+      const bool qlo = !wide;  // C_hi . Q_lo vanishes for tf32-exact queries
       uint32_t it = 0;
       for (int t = t0, tl = 0; t < t1; ++t, ++tl) {
         const uint32_t a = tl % nacc;
         mbar_wait(&tempty[a], ((tl / nacc) & 1) ^ 1);
         tc_fence_after();
-        const uint32_t d = tmem + a * NQB;
+        const uint32_t d = tmem + a * NQW;
         for (int c = 0; c < nchunks; ++c, ++it) {
           const uint32_t s = it % nstage;
           mbar_wait(&full_a[s], (it / nstage) & 1);
@@ -147,7 +150,7 @@ __global__ void __launch_bounds__(kCThreads, 1)
     const int quarter = warp & 3;        // TMEM lane quarter this warp may read
     const int sub = ew >> 2, nsub = p.nepi >> 2;
     const int row = quarter * 32 + lane;  // centroid within the tile
-    const int nqv = (int)min64(NQB, p.nq - q0);
+    const int nqv = (int)min64(NQW, p.nq - q0);
     uint32_t* G = p.G + (int64_t)q0 * p.ldg;
     const bool l2 = p.metric == MV_L2;
     const int ngr = (p.nlist + 31) / 32;
@@ -159,8 +162,8 @@ __global__ void __launch_bounds__(kCThreads, 1)
       const float cn = (valid && l2) ? __ldg(p.cnorm + cid) : 0.0f;
       mbar_wait(&tfull[a], (tl / nacc) & 1);
       tc_fence_after();
-      const uint32_t tb = tmem + a * NQB + ((uint32_t)(quarter * 32) << 16);
-      for (int qc = sub * 16; qc < NQB; qc += 16 * nsub) {
+      const uint32_t tb = tmem + a * NQW + ((uint32_t)(quarter * 32) << 16);
+      for (int qc = sub * 16; qc < NQW; qc += 16 * nsub) {
         uint32_t rd[16];
         tmem_ld16(tb + qc, rd);
         tmem_wait_ld();
@@ -184,7 +187,7 @@ __global__ void __launch_bounds__(kCThreads, 1)
           for (int j = 0; j < 16; ++j) {
             const float dot = __uint_as_float(rd[j]);
             key[j] = f2key(l2 ? cn - 2.0f * dot : -dot);
-            const uint64_t b = sbound[qc + j];
+            const uint64_t b = j < jn ? __ldg(p.gbound + q0 + qc + j) : 0ull;  // (L1-resident)
             const uint32_t bk = (uint32_t)(b >> 32);
             const bool pass = valid && j < jn && (key[j] < bk || (key[j] == bk && grp <= (uint32_t)b));
             m[j] = __ballot_sync(MV_FULL, pass);
@@ -403,7 +406,7 @@ bool coarse_tc_plan(int dpad, int nprobe, int64_t nq, int nlist, int nsm, const 
   if (dpad % 32 != 0 || nprobe > 1024) return false;
   p.nchunks = dpad / 32;
   p.nprobe = nprobe;
-  const int budget = 227 * 1024 - 1024 - 256;
+  const int budget = 227 * 1024 - 1024 - 256;  // alignment slack, barriers
   const int stage = 2 * 128 * 128;
   const int ntiles = (nlist + 127) / 128;
   int64_t best_cost = -1;
@@ -429,14 +432,14 @@ bool coarse_tc_plan(int dpad, int nprobe, int64_t nq, int nlist, int nsm, const 
   if (o.coarse_cs > 0) p.csplit = std::max(1, std::min(ntiles, o.coarse_cs));
   const int fixed = p.nchunks * 2 * p.nqb * 128;
   p.nstage = std::min(6, (budget - fixed) / stage);
-  p.smem_total = fixed + p.nstage * stage + 256 + 128 * 8 + 1024;
+  p.smem_total = fixed + p.nstage * stage + 256 + 1024;
   p.nepi = 8;
   p.nacc = 2;
   if (o.coarse_epi > 0) p.nepi = std::max(4, std::min(kCEpiMax, o.coarse_epi / 4 * 4));
   if (o.coarse_nacc > 0) p.nacc = std::max(1, std::min(4, o.coarse_nacc));
-  while (p.nacc > 1 && p.nacc * p.nqb > 512) --p.nacc;
+  while (p.nacc > 1 && p.nacc * 2 * p.nqb > 512) --p.nacc;  // (wide mode: 2 nqb columns per accumulator)
   int cols = 32;
-  while (cols < p.nacc * p.nqb) cols <<= 1;
+  while (cols < p.nacc * 2 * p.nqb) cols <<= 1;
   p.tmem_cols = cols;
   return p.smem_total <= 227 * 1024;
 }

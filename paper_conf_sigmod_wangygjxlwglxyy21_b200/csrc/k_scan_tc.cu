@@ -150,9 +150,10 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
   const bool use_norms = p.metric == MV_L2;
   const bool use_ids = p.bitset != nullptr;
   const bool phaseB = p.phase != 0;
-  // FLAT filter mode: the tensor-core badness is an approximation with a rigorous error bound
-  // E_q (stored values or queries not tf32-exact); keys are re-scored exactly after the scan
-  const bool approx = TYPE == MV_IVF_FLAT && (p.approx_always || P == 2);
+  // filter mode: the tensor-core badness is an approximation with a rigorous error bound E_q
+  // (SQ8 always; FLAT when the stored values or the queries are not tf32-exact); the keys are
+  // re-scored exactly after the scan (k_select.cu k_rekey)
+  const bool approx = TYPE == MV_IVF_SQ8 || p.approx_always || P == 2;
   // epilogue column chunk: 16 (FLAT), 8 (SQ8: few queries per list, so both warps of a lane quarter
   // get columns)
   constexpr int W = TYPE == MV_IVF_FLAT ? 16 : 8;
@@ -341,7 +342,7 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
           f.tau[u] = phaseB ? p.tau[f.q[u]] : MV_KEY_PAD;
           f.qn[u] = p.qnorm[f.q[u]];
           f.qs[u] = TYPE == MV_IVF_SQ8 ? p.qscale[f.q[u]] : 1.0f;
-          f.qe[u] = (TYPE == MV_IVF_FLAT && approx) ? p.qerr[f.q[u]] : 0.0f;
+          f.qe[u] = approx ? p.qerr[f.q[u]] : 0.0f;
           f.qa[u] = TYPE == MV_IVF_SQ8 ? p.qa[f.q[u]] : 0.0;
           f.base[u] = p.poff[f.pr[u]];
         }
@@ -397,17 +398,6 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
           mt.qs[i] = cur.qs[u];
           mt.qa[i] = cur.qa[u];
           mt.qaf[i] = (float)cur.qa[u];
-          if (TYPE == MV_IVF_SQ8) {
-            // |fp32 filter - exact| <= 2^-21 (||q||^2 + ||x||^2 + 2 (s Amax + |q.a|)) with Amax the
-            // largest |digit-weighted partial| (127 * 255 * dpad * (1 + 2^-7 + ...)); + 2^-23 |thf|
-            // for the final rounding to fp32.  ||x||^2's share is taken per row (xnlo).
-            const float thf = mt.thf[i];
-            const double amax = 127.0 * 255.0 * p.dpad * 1.0079;
-            const double mcol = 4.76837158203125e-7 * (cur.qn[u] + 2.0 * ((double)cur.qs[u] * amax + fabs(cur.qa[u])));
-            mt.thc[i] = (float)((double)thf + mcol + fabs((double)thf) * 1.1920928955078125e-7);
-          } else {
-            mt.thc[i] = mt.thf[i];
-          }
           mt.base[i] = cur.base[u];
         } else if (i < NQ) {  // padding column: no comparison passes
           mt.thf[i] = __int_as_float(0x7fffffff);
@@ -416,7 +406,6 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
           mt.qs[i] = 0.f;
           mt.qa[i] = 0.0;
           mt.qaf[i] = 0.f;
-          mt.thc[i] = __int_as_float(0x7fffffff);
         }
       }
       named_bar(2, 64);
@@ -478,7 +467,6 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
           valid = !bit_excluded(p.bitset, p.nbits, reinterpret_cast<const int64_t*>(sd + kSideIds)[(row0 & 1) + row]);
         const double xn = use_norms ? reinterpret_cast<const double*>(sd)[(row0 & 1) + row] : 0.0;
         const float xnf = (float)xn;
-        const float xnlo = xnf - xnf * 4.76837158203125e-7f;  // SQ8 filter: the row's share of the margin
         mbar_wait(&tfull[a], (titer / NACC) & 1);
         if (et == 0) MV_TRACE(6, titer);
         tc_fence_after();
@@ -493,14 +481,14 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
               for (int j = 0; j < W; ++j) r[pl][j] = 0u;
           }
           tmem_wait_ld();
-          // pass 1 (every row x column): the threshold filter, branch-free.  FLAT computes the exact
-          // fp32 distance; SQ8 an fp32 bound-checked approximation (the exact fp64 value in pass 2)
+          // the threshold filter, branch-free.  FLAT computes the fp32 distance (exact for
+          // tf32-exact data and queries); SQ8 an fp32 approximation within E_q of the exact value
           float bad[W];
           uint32_t pm = 0, pe = 0;  // pe (FLAT): entries exactly at the bound, which need the key test
 #pragma unroll
           for (int v = 0; v < W / 4; ++v) {
             const float4 qn4 = lds_f4(mt.qnf + qc + 4 * v);
-            const float4 th4 = lds_f4((TYPE == MV_IVF_SQ8 ? mt.thc : mt.thf) + qc + 4 * v);
+            const float4 th4 = lds_f4(mt.thf + qc + 4 * v);
             float4 qs4 = qn4, qa4 = qn4;
             if (TYPE == MV_IVF_SQ8) {
               qs4 = lds_f4(mt.qs + qc + 4 * v);
@@ -517,7 +505,7 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
                 bad[j] = use_norms ? (qnv[u] + xnf) - 2.0f * dot : -dot;
               } else {
                 // digit partials converted exactly (magic number: |D| < 2^22 for rows of <= 128
-                // codes), combined in fp32; the error bound is folded into thc (per column) and xnlo
+                // codes), combined in fp32; the error is bounded by E_q (k_qplanes)
                 float fd[4];
 #pragma unroll
                 for (int pl = 0; pl < 4; ++pl)
@@ -526,7 +514,7 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
                 const float accf =
                     fmaf(fd[3], 4.76837158203125e-7f, fmaf(fd[2], 6.103515625e-5f, fmaf(fd[1], 0.0078125f, fd[0])));
                 const float dotf = fmaf(qsv[u], accf, qav[u]);
-                bad[j] = use_norms ? (qnv[u] + xnlo) - 2.0f * dotf : -dotf;
+                bad[j] = use_norms ? (qnv[u] + xnf) - 2.0f * dotf : -dotf;
               }
               pm |= (bad[j] <= thv[u] ? 1u : 0u) << j;
               if (TYPE == MV_IVF_FLAT) pe |= (bad[j] == thv[u] ? 1u : 0u) << j;
@@ -534,27 +522,11 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
           }
           if (!valid) pm = 0;
           if (TYPE == MV_IVF_FLAT) pe &= (phaseB && !approx) ? pm : 0u;
-          // pass 2 (flagged entries only): SQ8's exact fp64 badness; the exact key test at the bound
-          if (__any_sync(MV_FULL, (TYPE == MV_IVF_SQ8 ? pm : pe) != 0)) {
+          // FLAT exact mode, entries exactly at the bound: the (distance key, id rank) <= tau_q test
+          if (TYPE == MV_IVF_FLAT && __any_sync(MV_FULL, pe != 0)) {
 #pragma unroll
-            for (int j = 0; j < W; ++j) {
-              if (((TYPE == MV_IVF_SQ8 ? pm : pe) >> j) & 1) {
-                const int i = qc + j;
-                const float thj = mt.thf[i];
-                if (TYPE == MV_IVF_SQ8) {
-                  // int32-exact digit partials; the L2 expansion is combined in fp64 (the norms are
-                  // ~400x the near-neighbour distances on SIFT-scale data)
-                  const double acc = (double)(int)r[0][j] + (double)(int)r[1 % PMAX][j] * (1.0 / 128.0) +
-                                     (double)(int)r[2 % PMAX][j] * (1.0 / 16384.0) +
-                                     (double)(int)r[3 % PMAX][j] * (1.0 / 2097152.0);
-                  const double dot = fma((double)mt.qs[i], acc, mt.qa[i]);
-                  bad[j] = use_norms ? (float)((mt.qn[i] + xn) - 2.0 * dot) : (float)(-dot);
-                }
-                bool ok = bad[j] <= thj;
-                if (ok && phaseB && bad[j] == thj) ok = (((uint64_t)f2key(bad[j]) << 32) | rk) <= mt.tau[i];
-                if (!ok) pm &= ~(1u << j);
-              }
-            }
+            for (int j = 0; j < W; ++j)
+              if (((pe >> j) & 1) && (((uint64_t)f2key(bad[j]) << 32) | rk) > mt.tau[qc + j]) pm &= ~(1u << j);
           }
           if (__any_sync(MV_FULL, pm != 0)) {
             // ballot per column; lane j reserves column j's slots with one shared atomic (measured:
@@ -633,16 +605,18 @@ __global__ void k_qplanes(int type, const float* __restrict__ qpad, int64_t nq, 
       }
     } else {
       // fp64: w_j = q_j b_j, b_j = vdiff_j / 255, a_j = vmin_j + b_j / 2 (mid-bin decode)
-      double amax = 0.0, dot = 0.0;
+      double amax = 0.0, dot = 0.0, qdec = 0.0;
       for (int j = lane; j < dpad; j += 32) {
         const double bj = (double)vdiff[j] / 255.0;
         const double aj = fma(0.5, bj, (double)vmin[j]);
         dot = fma((double)x[j], aj, dot);
         amax = fmax(amax, fabs((double)x[j] * bj));
+        qdec = fma(fabs((double)x[j]), 2.0 * (double)vdiff[j] + fabs((double)vmin[j]), qdec);
       }
       for (int o = 16; o > 0; o >>= 1) {
         amax = fmax(amax, __shfl_xor_sync(MV_FULL, amax, o));
         dot += __shfl_xor_sync(MV_FULL, dot, o);
+        qdec += __shfl_xor_sync(MV_FULL, qdec, o);
       }
       // the scale is rounded up to fp32 first, so the digits and the epilogue use the same exact s
       const double s = amax > 0.0 ? (double)__double2float_ru(amax / 127.0) : 1.0;
@@ -659,6 +633,20 @@ __global__ void k_qplanes(int type, const float* __restrict__ qpad, int64_t nq, 
       if (lane == 0) {
         qscale[q] = (float)s;
         qa[q] = dot;
+        // Filter-mode bound E_q >= |fp32 filter badness - the oracle's badness|:
+        //   the fp32 conversions, three FMAs and the expansion: 2^-21 (||q||^2 + X^2 + 2 (s Amax + |q.a|)),
+        //   Amax = the largest |digit-weighted partial| (127 * 255 * dpad * (1 + 2^-7 + ...));
+        //   the digits' residual (<= 2^-22 s per weight, times the codes): s 2^-22 255 dpad;
+        //   the oracle's fp32 decode vmin + ((c + 0.5)/255) vdiff vs the exact affine map:
+        //   2^-22 sum |q_j| (2 vdiff_j + |vmin_j|);  L2 doubles the dot's share;  + 2^-22 (||q||^2 + X^2)
+        //   for the roundings of the result.
+        if (qerr) {
+          const double amx = 127.0 * 255.0 * dpad * 1.0079;
+          const double mc = 0x1p-21 * (nn + fe.xmax2 + 2.0 * (s * amx + fabs(dot)));
+          const double dd = 0x1p-22 * (s * 255.0 * dpad + qdec);
+          const double E = mc + (fe.metric == MV_L2 ? 2.0 : 1.0) * dd + 0x1p-22 * (nn + fe.xmax2);
+          qerr[q] = __double2float_ru(1.05 * E);
+        }
       }
     }
   }

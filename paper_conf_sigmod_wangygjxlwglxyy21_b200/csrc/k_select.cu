@@ -372,19 +372,41 @@ __global__ void __launch_bounds__(kBigThreads) k_final_big(const int64_t* __rest
       if (done) break;
     }
     // winners: keys whose bits above lo are <= pfx (exactly k: keys are unique)
+    if (tau_out) {  // seeding: only the k-th best key is needed -- the largest winner, no gather
+      uint64_t m = 0;
+      for (int i = tid; i < T; i += kBigThreads) {
+        const uint64_t x = buf[i];
+        if ((lo >= 64 ? 0 : (x >> lo)) <= pfx) m = umax64(m, x);
+      }
+      for (int o = 16; o > 0; o >>= 1) m = umax64(m, shfl_xor64(m, o));
+      __syncthreads();
+      if (lane == 0) win[wid] = m;
+      __syncthreads();
+      if (tid == 0) {
+        uint64_t mm = 0;
+        for (int w = 0; w < kBigThreads / 32; ++w) mm = umax64(mm, win[w]);
+        tau_out[q] = mm;
+      }
+      return;
+    }
     if (tid == 0) s_int[3] = 0;
     __syncthreads();
-    for (int i = tid; i < T; i += kBigThreads) {
-      const uint64_t x = buf[i];
-      const uint64_t top = lo >= 64 ? 0 : (x >> lo);
-      if (top <= pfx) win[atomicAdd(s_int + 3, 1)] = x;
+    for (int b0 = 0; b0 < T; b0 += kBigThreads) {  // ballot-aggregated appends (one atomic per warp)
+      const int i = b0 + tid;
+      const uint64_t x = i < T ? buf[i] : MV_KEY_PAD;
+      const bool p = i < T && (lo >= 64 ? 0 : (x >> lo)) <= pfx;
+      const uint32_t m = __ballot_sync(MV_FULL, p);
+      int base = 0;
+      if (lane == 0 && m) base = atomicAdd(s_int + 3, __popc(m));
+      base = __shfl_sync(MV_FULL, base, 0);
+      if (p) win[base + __popc(m & ((1u << lane) - 1))] = x;
     }
     __syncthreads();
     nsel = k;
     for (int i = k + tid; i < NK; i += kBigThreads) win[i] = MV_KEY_PAD;
   }
   __syncthreads();
-  if (tau_out) {  // seeding: only the k-th best key is needed (the largest winner)
+  if (tau_out) {  // seeding with exactly k candidates: the largest
     if (nsel < k) return;
     uint64_t m = 0;
     for (int i = tid; i < k; i += kBigThreads) m = umax64(m, win[i]);
@@ -687,11 +709,177 @@ static cudaError_t launch_big_select(const int64_t* poff, const int32_t* pcnt, c
   return cudaGetLastError();
 }
 
+// ------------------------------------------------------------------------------------------
+// Filter mode's exact re-scoring: the oracle's badness of one stored row for a
+// query held in registers by the warp -- fp64 from the fp32 query and the stored row (FLAT: the
+// fp32 vector; SQ8: the codes decoded in fp32 in the oracle's order, vmin + ((c + 0.5)/255) vdiff;
+// PAPER.md:290-294 §2.1), rounded to fp32.  Warp-cooperative: dims 4 (lane + 32 u) .. +3 per lane
+// (dpad <= 512); every lane returns the result.
+// ------------------------------------------------------------------------------------------
+struct QueryRegs {
+  float4 q[4], vm[4], vd[4];
+};
+
+template <int TYPE>
+__device__ __forceinline__ void load_query_regs(QueryRegs& r, const float* qrow, int dpad, const float* vmin,
+                                                const float* vdiff) {
+  const int lane = threadIdx.x & 31;
+#pragma unroll
+  for (int u = 0; u < 4; ++u) {
+    const bool in = 4 * (lane + 32 * u) < dpad;
+    const float4 z = make_float4(0.f, 0.f, 0.f, 0.f);
+    r.q[u] = in ? reinterpret_cast<const float4*>(qrow)[lane + 32 * u] : z;
+    if (TYPE == MV_IVF_SQ8) {
+      r.vm[u] = in ? reinterpret_cast<const float4*>(vmin)[lane + 32 * u] : z;
+      r.vd[u] = in ? reinterpret_cast<const float4*>(vdiff)[lane + 32 * u] : z;
+    }
+  }
+}
+
+template <int TYPE>
+__device__ __forceinline__ float exact_badness(const QueryRegs& r, int64_t row, int dpad, bool l2, const void* payload,
+                                               const float* __restrict__ sq8_t) {
+  const int lane = threadIdx.x & 31;
+  double acc = 0.0;
+#pragma unroll
+  for (int u = 0; u < 4; ++u) {
+    if (4 * (lane + 32 * u) < dpad) {
+      float4 xv;
+      if (TYPE == MV_IVF_FLAT) {
+        xv = __ldg(reinterpret_cast<const float4*>(reinterpret_cast<const float*>(payload) + row * dpad) + lane + 32 * u);
+      } else {  // the oracle's decode, fp32, one rounding per operation: (t_c * vdiff) + vmin
+        const uint32_t cw =
+            __ldg(reinterpret_cast<const uint32_t*>(reinterpret_cast<const uint8_t*>(payload) + row * dpad) + lane + 32 * u);
+        xv.x = __fadd_rn(__fmul_rn(__ldg(sq8_t + (cw & 0xff)), r.vd[u].x), r.vm[u].x);
+        xv.y = __fadd_rn(__fmul_rn(__ldg(sq8_t + ((cw >> 8) & 0xff)), r.vd[u].y), r.vm[u].y);
+        xv.z = __fadd_rn(__fmul_rn(__ldg(sq8_t + ((cw >> 16) & 0xff)), r.vd[u].z), r.vm[u].z);
+        xv.w = __fadd_rn(__fmul_rn(__ldg(sq8_t + (cw >> 24)), r.vd[u].w), r.vm[u].w);
+      }
+      if (l2) {
+        const double a = (double)r.q[u].x - xv.x, b = (double)r.q[u].y - xv.y;
+        const double c = (double)r.q[u].z - xv.z, d = (double)r.q[u].w - xv.w;
+        acc = fma(a, a, acc); acc = fma(b, b, acc); acc = fma(c, c, acc); acc = fma(d, d, acc);
+      } else {
+        acc = fma((double)r.q[u].x, (double)xv.x, acc); acc = fma((double)r.q[u].y, (double)xv.y, acc);
+        acc = fma((double)r.q[u].z, (double)xv.z, acc); acc = fma((double)r.q[u].w, (double)xv.w, acc);
+      }
+    }
+  }
+  for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(MV_FULL, acc, o);
+  return l2 ? (float)acc : (float)(-acc);
+}
+
+// up to 4 rows at once (n <= 4, warp-uniform): their loads are in flight together
+template <int TYPE>
+__device__ __forceinline__ void exact_badness4(const QueryRegs& r, const int64_t (&row)[4], int n, int dpad, bool l2,
+                                               const void* payload, const float* __restrict__ sq8_t, float (&out)[4]) {
+  const int lane = threadIdx.x & 31;
+  double acc[4] = {0.0, 0.0, 0.0, 0.0};
+#pragma unroll
+  for (int u = 0; u < 4; ++u) {
+    if (4 * (lane + 32 * u) < dpad) {
+      float4 xv[4];
+#pragma unroll
+      for (int m = 0; m < 4; ++m) {
+        if (m < n) {
+          if (TYPE == MV_IVF_FLAT) {
+            xv[m] = __ldg(reinterpret_cast<const float4*>(reinterpret_cast<const float*>(payload) + row[m] * dpad) +
+                          lane + 32 * u);
+          } else {
+            const uint32_t cw = __ldg(
+                reinterpret_cast<const uint32_t*>(reinterpret_cast<const uint8_t*>(payload) + row[m] * dpad) + lane + 32 * u);
+            xv[m].x = __fadd_rn(__fmul_rn(__ldg(sq8_t + (cw & 0xff)), r.vd[u].x), r.vm[u].x);
+            xv[m].y = __fadd_rn(__fmul_rn(__ldg(sq8_t + ((cw >> 8) & 0xff)), r.vd[u].y), r.vm[u].y);
+            xv[m].z = __fadd_rn(__fmul_rn(__ldg(sq8_t + ((cw >> 16) & 0xff)), r.vd[u].z), r.vm[u].z);
+            xv[m].w = __fadd_rn(__fmul_rn(__ldg(sq8_t + (cw >> 24)), r.vd[u].w), r.vm[u].w);
+          }
+        }
+      }
+#pragma unroll
+      for (int m = 0; m < 4; ++m) {
+        if (m < n) {
+          if (l2) {
+            const double a = (double)r.q[u].x - xv[m].x, b = (double)r.q[u].y - xv[m].y;
+            const double c = (double)r.q[u].z - xv[m].z, d = (double)r.q[u].w - xv[m].w;
+            acc[m] = fma(a, a, acc[m]); acc[m] = fma(b, b, acc[m]); acc[m] = fma(c, c, acc[m]); acc[m] = fma(d, d, acc[m]);
+          } else {
+            acc[m] = fma((double)r.q[u].x, (double)xv[m].x, acc[m]); acc[m] = fma((double)r.q[u].y, (double)xv[m].y, acc[m]);
+            acc[m] = fma((double)r.q[u].z, (double)xv[m].z, acc[m]); acc[m] = fma((double)r.q[u].w, (double)xv[m].w, acc[m]);
+          }
+        }
+      }
+    }
+  }
+#pragma unroll
+  for (int m = 0; m < 4; ++m) {
+    for (int o = 16; o > 0; o >>= 1) acc[m] += __shfl_xor_sync(MV_FULL, acc[m], o);
+    out[m] = l2 ? (float)acc[m] : (float)(-acc[m]);
+  }
+}
+
+// One lane re-scores one stored row (the band members of a 32-key chunk in parallel, one per
+// lane); the query row (and SQ8's vmin / vdiff) sit in the warp's shared memory, read as
+// broadcasts.  Same arithmetic as exact_badness.
+template <int TYPE>
+__device__ __forceinline__ float lane_exact_badness(int64_t row, const float* sq, const float* svm, const float* svd,
+                                                    int dpad, bool l2, const void* payload,
+                                                    const float* __restrict__ sq8_t) {
+  double acc = 0.0;
+  if (TYPE == MV_IVF_FLAT) {
+    const float4* x = reinterpret_cast<const float4*>(reinterpret_cast<const float*>(payload) + row * dpad);
+    for (int j4 = 0; j4 < dpad / 4; ++j4) {
+      const float4 xv = __ldg(x + j4);
+      const float4 qv = reinterpret_cast<const float4*>(sq)[j4];
+      if (l2) {
+        const double a = (double)qv.x - xv.x, b = (double)qv.y - xv.y, c = (double)qv.z - xv.z, d = (double)qv.w - xv.w;
+        acc = fma(a, a, acc); acc = fma(b, b, acc); acc = fma(c, c, acc); acc = fma(d, d, acc);
+      } else {
+        acc = fma((double)qv.x, (double)xv.x, acc); acc = fma((double)qv.y, (double)xv.y, acc);
+        acc = fma((double)qv.z, (double)xv.z, acc); acc = fma((double)qv.w, (double)xv.w, acc);
+      }
+    }
+  } else {
+    const uint32_t* x = reinterpret_cast<const uint32_t*>(reinterpret_cast<const uint8_t*>(payload) + row * dpad);
+    for (int j4 = 0; j4 < dpad / 4; ++j4) {
+      const uint32_t cw = __ldg(x + j4);
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const int j = 4 * j4 + u;
+        const float xv = __fadd_rn(__fmul_rn(sq8_t[(cw >> (8 * u)) & 0xff], svd[j]), svm[j]);
+        if (l2) {
+          const double a = (double)sq[j] - xv;
+          acc = fma(a, a, acc);
+        } else {
+          acc = fma((double)sq[j], (double)xv, acc);
+        }
+      }
+    }
+  }
+  return l2 ? (float)acc : (float)(-acc);
+}
+
 // k <= 32 R: one warp per query, two passes over the query's candidates (its pairs' regions,
 // walked in 32-key chunks through a flattened index over groups of 32 pairs located by a shuffle
 // binary search).  Pass 1 keeps every lane's R smallest keys; the k-th smallest of those 32R keys
 // bounds the answer (k distinct keys are at or below it).  Pass 2 streams the keys at or below the
 // bound through a 32-entry staging buffer into a sorted register list (sort-32 + bitonic merge).
+//
+// RT >= 0 (MV_IVF_FLAT / MV_IVF_SQ8): the filter mode's fused refine.  The keys are
+// approximate (|b~ - b| <= E_q) unless rf.rgate says the search is exact; pass 1's bound t~ is then
+// >= the k-th approximate key, every member of the exact top-k has b~ <= t~ + 2 E_q, and pass 2
+// re-scores exactly (exact_badness) only those band keys before staging them -- the sorted list
+// keeps the k smallest exact keys.  One kernel instead of a separate k-th select, re-scoring pass
+// and final select.
+struct RefineArgs {
+  const float* qerr;
+  const float* qpad;
+  int dpad;
+  const void* payload;
+  const uint32_t* row_of_rank;
+  const float *vmin, *vdiff, *sq8_t;
+  const int* rgate;  // nullable: filter mode always; else only when *rgate != 0
+};
+
 template <int R>
 __global__ void __launch_bounds__(256) k_final_warp(const int64_t* __restrict__ poff, const int32_t* __restrict__ pcnt,
                                                     const uint64_t* __restrict__ part, int64_t nq, int npb, int k,
@@ -815,6 +1003,121 @@ __global__ void __launch_bounds__(256) k_final_warp(const int64_t* __restrict__ 
   }
 }
 
+// k <= 256, filter mode, second kernel (the first is k_final_warp in tau mode: t~ = the exact
+// k-th smallest approximate key): one pass over the query's keys; the band b~ <= t~ + 2 E_q is
+// re-scored exactly (exact_badness4: four rows in flight), staged and merged into a sorted list
+// of the k smallest exact keys, which is the answer.  Kept apart from the select
+// so that each kernel has its own register budget (the selects run at full occupancy).
+template <int R, int TYPE>
+__global__ void __launch_bounds__(256) k_refine_band(const int64_t* __restrict__ poff, const int32_t* __restrict__ pcnt,
+                                                     const uint64_t* __restrict__ part, int64_t nq, int npb, int k,
+                                                     int metric, const int64_t* __restrict__ sorted_ids, float* out_d,
+                                                     int64_t* out_i, const uint64_t* __restrict__ tau2,
+                                                     const RefineArgs rf) {
+  __shared__ uint64_t stage_all[8][64];
+  // shared: SQ8's decode table (256), then per warp q (+ SQ8: vmin, vdiff), dpad floats each
+  extern __shared__ __align__(16) float qsm[];
+  const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+  const int64_t q = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int dpad = rf.dpad;
+  float* stab = qsm;
+  if (TYPE == MV_IVF_SQ8) {
+    for (int i = threadIdx.x; i < 256; i += blockDim.x) stab[i] = rf.sq8_t[i];
+    __syncthreads();
+  }
+  if (q >= nq || (rf.rgate && *rf.rgate == 0)) return;
+  uint64_t* stage = stage_all[wib];
+  float* sq = qsm + (TYPE == MV_IVF_SQ8 ? 256 + wib * 3 * dpad : wib * dpad);
+  float* svm = sq + dpad;
+  float* svd = svm + dpad;
+  for (int j = lane; j < dpad; j += 32) {
+    sq[j] = rf.qpad[q * dpad + j];
+    if (TYPE == MV_IVF_SQ8) {
+      svm[j] = rf.vmin[j];
+      svd[j] = rf.vdiff[j];
+    }
+  }
+  __syncwarp();
+  const uint64_t kth = tau2[q];
+  const float band =
+      kth == MV_KEY_PAD ? __int_as_float(0x7f800000) : __fadd_ru(key2f((uint32_t)(kth >> 32)), 2.0f * rf.qerr[q]);
+  uint64_t best[R];
+#pragma unroll
+  for (int r = 0; r < R; ++r) best[r] = MV_KEY_PAD;
+  int ns = 0;
+  // a flush re-scores the (up to) 32 staged band keys, one per lane -- every lane busy -- before the
+  // sort + merge (re-scoring in the chunk loop would run a whole warp for one or two band keys)
+  auto flush32 = [&]() {
+    uint64_t c[R];
+    uint64_t c1[1] = {MV_KEY_PAD};
+    if (lane < ns) {
+      const uint64_t key = stage[lane];
+      const int64_t row = (int64_t)__ldg(rf.row_of_rank + (uint32_t)key);
+      const float b = lane_exact_badness<TYPE>(row, sq, svm, svd, dpad, metric == MV_L2, rf.payload, stab);
+      c1[0] = ((uint64_t)f2key(b) << 32) | (uint32_t)key;
+    }
+    warp_bitonic_sort<1>(c1);
+    c[0] = c1[0];
+#pragma unroll
+    for (int r = 1; r < R; ++r) c[r] = MV_KEY_PAD;
+    warp_merge_smallest<R>(best, c);
+    const int rest = ns > 32 ? ns - 32 : 0;
+    const uint64_t mv = lane < rest ? stage[32 + lane] : 0;
+    __syncwarp();
+    if (lane < rest) stage[lane] = mv;
+    __syncwarp();
+    ns = rest;
+  };
+  for (int g = 0; g < npb; g += 32) {
+    const int j = g + lane;
+    const int cnt = j < npb ? pcnt[q * npb + j] : 0;
+    const int64_t off = j < npb ? poff[q * npb + j] : 0;
+    int incl = cnt;
+    for (int o = 1; o < 32; o <<= 1) {
+      const int v = __shfl_up_sync(MV_FULL, incl, o);
+      if (lane >= o) incl += v;
+    }
+    const int excl = incl - cnt;
+    const int T = __shfl_sync(MV_FULL, incl, 31);
+    for (int e0 = 0; e0 < T; e0 += 32) {
+      const int e = e0 + lane;
+      int lo = 0;
+#pragma unroll
+      for (int step = 16; step > 0; step >>= 1) {
+        const int ex = __shfl_sync(MV_FULL, excl, (lo + step) & 31);
+        if (lo + step < 32 && ex <= e) lo += step;
+      }
+      const int64_t addr = __shfl_sync(MV_FULL, off, lo) + (e - __shfl_sync(MV_FULL, excl, lo));
+      const uint64_t key = e < T ? part[addr] : MV_KEY_PAD;
+      const bool ps = key != MV_KEY_PAD && key2f((uint32_t)(key >> 32)) <= band;
+      const uint32_t m = __ballot_sync(MV_FULL, ps);
+      if (ps) stage[ns + __popc(m & ((1u << lane) - 1))] = key;  // re-scored at the flush
+      ns += __popc(m);
+      __syncwarp();
+      if (ns >= 32) flush32();
+    }
+  }
+  if (ns > 0) flush32();
+#pragma unroll
+  for (int r = 0; r < R; ++r) {
+    const int i = r * 32 + lane;
+    if (i < k) {
+      const uint64_t key = best[r];
+      float dv;
+      int64_t iv;
+      if (key != MV_KEY_PAD) {
+        dv = key_dist((uint32_t)(key >> 32), metric);
+        iv = sorted_ids[(uint32_t)(key & 0xffffffffu)];
+      } else {
+        dv = metric == MV_L2 ? __int_as_float(0x7f800000) : __int_as_float(0xff800000);
+        iv = -1;
+      }
+      out_d[q * k + i] = dv;
+      out_i[q * k + i] = iv;
+    }
+  }
+}
+
 // k <= 256: the warp kernel with a 32R-entry register list (R = 1, 2, 4, 8)
 static bool launch_warp_select(const int64_t* poff, const int32_t* pcnt, const uint64_t* part, int64_t nq, int npb,
                                int k, int metric, const int64_t* sorted_ids, float* out_d, int64_t* out_i,
@@ -835,6 +1138,49 @@ static bool launch_warp_select(const int64_t* poff, const int32_t* pcnt, const u
   else
     return false;
   return true;
+}
+
+// k <= 256 with the filter mode's refine: k_final_warp in tau mode (t~ = the k-th approximate key)
+// then k_refine_band; an exact search (rgate set and *rgate == 0) takes the plain final select
+__global__ void k_not(const int* __restrict__ g, int* __restrict__ out) { *out = g ? (*g == 0) : 0; }
+
+cudaError_t launch_final_refine(int type, const int64_t* poff, const int32_t* pcnt, const uint64_t* part, int64_t nq,
+                                int npb, int k, int metric, const int64_t* sorted_ids, float* out_d, int64_t* out_i,
+                                const float* qerr, const float* qpad, int dpad, const void* payload,
+                                const uint32_t* row_of_rank, const float* vmin, const float* vdiff, const float* sq8_t,
+                                const int* rgate, uint64_t* tau2, int* notgate, cudaStream_t st) {
+  if (nq == 0) return cudaSuccess;
+  if (k > 256 || dpad > 512 || dpad % 4) return cudaErrorInvalidValue;
+  const RefineArgs rf{qerr, qpad, dpad, payload, row_of_rank, vmin, vdiff, sq8_t, rgate};
+  const unsigned grid = (unsigned)((nq * 32 + 255) / 256);
+  cudaError_t e;
+  // shared: (SQ8: the 256-entry decode table +) per warp q (, vmin, vdiff)
+  const size_t qsm = ((type == MV_IVF_SQ8 ? 256 : 0) + (size_t)8 * (type == MV_IVF_SQ8 ? 3 : 1) * dpad) * sizeof(float);
+  if (rgate) {  // exact searches: the plain select, gated by !*rgate
+    k_not<<<1, 1, 0, st>>>(rgate, notgate);
+    if (!launch_warp_select(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d, out_i, nullptr, nullptr, notgate,
+                            st))
+      return cudaErrorInvalidValue;
+  }
+  if ((e = cudaMemsetAsync(tau2, 0xff, sizeof(uint64_t) * nq, st)) != cudaSuccess) return e;
+  launch_warp_select(poff, pcnt, part, nq, npb, k, MV_L2, nullptr, nullptr, nullptr, nullptr, tau2, rgate, st);
+#define MV_REFINE_LAUNCH(R)                                                                                           \
+  if (type == MV_IVF_FLAT) {                                                                                          \
+    k_refine_band<R, MV_IVF_FLAT><<<grid, 256, qsm, st>>>(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d,    \
+                                                          out_i, tau2, rf);                                           \
+  } else {                                                                                                            \
+    if ((e = cudaFuncSetAttribute(k_refine_band<R, MV_IVF_SQ8>, cudaFuncAttributeMaxDynamicSharedMemorySize,         \
+                                  (int)qsm)) != cudaSuccess)                                                          \
+      return e;                                                                                                       \
+    k_refine_band<R, MV_IVF_SQ8><<<grid, 256, qsm, st>>>(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d,     \
+                                                         out_i, tau2, rf);                                            \
+  }
+  if (k <= 32) { MV_REFINE_LAUNCH(1) }
+  else if (k <= 64) { MV_REFINE_LAUNCH(2) }
+  else if (k <= 128) { MV_REFINE_LAUNCH(4) }
+  else { MV_REFINE_LAUNCH(8) }
+#undef MV_REFINE_LAUNCH
+  return cudaGetLastError();
 }
 
 cudaError_t launch_final_select(const int64_t* poff, const int32_t* pcnt, const uint64_t* part, int64_t nq, int npb,
@@ -859,24 +1205,28 @@ cudaError_t launch_tau_select(const int64_t* poff, const int32_t* pcnt, const ui
 }
 
 // ------------------------------------------------------------------------------------------
-// Exact re-scoring for the FLAT tensor-core scan's filter mode (DESIGN.md §5 "FLAT precision").
-// When the stored vectors or the queries are not tf32-exact, the scan's keys carry the fp32
-// tensor-core badness b~, with |b~ - b| <= E_q (qerr[q], a rigorous bound).  With t~ = the k-th
-// smallest b~ of the query (tau2[q]), every member of the exact top-k has b~ <= t~ + 2 E_q (k
-// candidates have b <= t~ + E_q), and every candidate above that bound has b > t~ + E_q.  So the
-// kernel recomputes b exactly -- fp64 from the fp32 query and the fp32 stored row, the oracle's
-// definition (§2.1) -- for the candidates at or below the bound, rewrites their
-// keys (exact fp32 distance key << 32 | id rank), and turns every other key into padding.  The
-// final select then returns the exact top-k.  One warp per query; the query row lives in
-// registers (dpad <= 512: <= 4 float4 per lane), each re-scored row is read as coalesced float4s.
+// Exact re-scoring for the tensor-core scan's filter mode (DESIGN.md §5 "Filter mode").  The
+// scan's keys carry the fp32 tensor-core badness b~ with |b~ - b| <= E_q (qerr[q], a rigorous
+// bound), b the oracle's badness: FLAT when the stored vectors or the queries are not
+// tf32-exact, SQ8 always.  With t~ = the k-th smallest b~ of the query (tau2[q]), every member of
+// the exact top-k has b~ <= t~ + 2 E_q (k candidates have b <= t~ + E_q), and every candidate
+// above that bound has b > t~ + E_q.  So the kernel recomputes b exactly for the candidates at or
+// below the bound -- fp64 from the fp32 query and the stored row (FLAT: the fp32 vector; SQ8: the
+// codes decoded in fp32 in the oracle's order, vmin + ((c + 0.5) / 255) vdiff), the definition of
+// PAPER.md:290-294 (§2.1) -- rewrites their keys (exact fp32 distance key << 32 | id rank), and
+// turns every other key into padding.  The final select then returns the exact top-k.  One warp
+// per query; the query row lives in registers (dpad <= 512: <= 4 float4 per lane), each
+// re-scored row is read as coalesced float4s (FLAT) or 4-code words (SQ8).
 // ------------------------------------------------------------------------------------------
+template <int TYPE>
 __global__ void __launch_bounds__(256) k_rekey(const int64_t* __restrict__ poff, const int32_t* __restrict__ pcnt,
                                                uint64_t* __restrict__ part, int64_t nq, int npb,
                                                const uint64_t* __restrict__ tau2, const float* __restrict__ qerr,
                                                int metric, const float* __restrict__ qpad, int dpad,
-                                               const float* __restrict__ payload,
+                                               const void* __restrict__ payload,
                                                const uint32_t* __restrict__ row_of_rank,
-                                               const int* __restrict__ gate) {
+                                               const float* __restrict__ vmin, const float* __restrict__ vdiff,
+                                               const float* __restrict__ sq8_t, const int* __restrict__ gate) {
   const int lane = threadIdx.x & 31;
   const int64_t q = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   if (q >= nq || (gate && *gate == 0)) return;
@@ -884,10 +1234,8 @@ __global__ void __launch_bounds__(256) k_rekey(const int64_t* __restrict__ poff,
   // bound in badness units, rounded up; fewer than k candidates (t = PAD): every candidate
   const float bound =
       t == MV_KEY_PAD ? __int_as_float(0x7f800000) : __fadd_ru(key2f((uint32_t)(t >> 32)), 2.0f * qerr[q]);
-  float4 qr[4];
-  const float4* qv = reinterpret_cast<const float4*>(qpad + q * dpad);
-#pragma unroll
-  for (int u = 0; u < 4; ++u) qr[u] = (4 * (lane + 32 * u) < dpad) ? qv[lane + 32 * u] : make_float4(0.f, 0.f, 0.f, 0.f);
+  QueryRegs qr;
+  load_query_regs<TYPE>(qr, qpad + q * dpad, dpad, vmin, vdiff);
   const bool l2 = metric == MV_L2;
   for (int g = 0; g < npb; g += 32) {
     const int j = g + lane;
@@ -911,43 +1259,35 @@ __global__ void __launch_bounds__(256) k_rekey(const int64_t* __restrict__ poff,
       const int64_t addr = __shfl_sync(MV_FULL, off, lo) + (e - __shfl_sync(MV_FULL, excl, lo));
       const uint64_t key = e < T ? part[addr] : MV_KEY_PAD;
       const bool band = key != MV_KEY_PAD && key2f((uint32_t)(key >> 32)) <= bound;
-      uint64_t nk = MV_KEY_PAD;
+      uint64_t nk = key;
       uint32_t m = __ballot_sync(MV_FULL, band);
       while (m) {
         const int src = __ffs(m) - 1;
         m &= m - 1;
         const uint32_t rk = __shfl_sync(MV_FULL, (uint32_t)key, src);
-        const float4* x = reinterpret_cast<const float4*>(payload + (int64_t)__ldg(row_of_rank + rk) * dpad);
-        double acc = 0.0;
-#pragma unroll
-        for (int u = 0; u < 4; ++u) {
-          if (4 * (lane + 32 * u) < dpad) {
-            const float4 xv = __ldg(x + lane + 32 * u);
-            if (l2) {
-              const double a = (double)qr[u].x - xv.x, b = (double)qr[u].y - xv.y;
-              const double c = (double)qr[u].z - xv.z, d = (double)qr[u].w - xv.w;
-              acc = fma(a, a, acc); acc = fma(b, b, acc); acc = fma(c, c, acc); acc = fma(d, d, acc);
-            } else {
-              acc = fma((double)qr[u].x, (double)xv.x, acc); acc = fma((double)qr[u].y, (double)xv.y, acc);
-              acc = fma((double)qr[u].z, (double)xv.z, acc); acc = fma((double)qr[u].w, (double)xv.w, acc);
-            }
-          }
-        }
-        for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(MV_FULL, acc, o);
-        if (lane == src) nk = ((uint64_t)f2key(l2 ? (float)acc : (float)(-acc)) << 32) | rk;
+        const float b = exact_badness<TYPE>(qr, (int64_t)__ldg(row_of_rank + rk), dpad, l2, payload, sq8_t);
+        if (lane == src) nk = ((uint64_t)f2key(b) << 32) | rk;
       }
-      if (e < T) part[addr] = nk;
+      // only the band is rewritten: its k smallest exact keys (<= t~ + E) are below every key left
+      // approximate (> t~ + 2 E), so the final select returns the exact top-k
+      if (band) part[addr] = nk;
     }
   }
 }
 
-cudaError_t launch_rekey(const int64_t* poff, const int32_t* pcnt, uint64_t* part, int64_t nq, int npb,
+cudaError_t launch_rekey(int type, const int64_t* poff, const int32_t* pcnt, uint64_t* part, int64_t nq, int npb,
                          const uint64_t* tau2, const float* qerr, int metric, const float* qpad, int dpad,
-                         const float* payload, const uint32_t* row_of_rank, const int* gate, cudaStream_t st) {
+                         const void* payload, const uint32_t* row_of_rank, const float* vmin, const float* vdiff,
+                         const float* sq8_t, const int* gate, cudaStream_t st) {
   if (nq == 0) return cudaSuccess;
   if (dpad > 512 || dpad % 4) return cudaErrorInvalidValue;
-  k_rekey<<<(unsigned)((nq * 32 + 255) / 256), 256, 0, st>>>(poff, pcnt, part, nq, npb, tau2, qerr, metric, qpad, dpad,
-                                                            payload, row_of_rank, gate);
+  const unsigned grid = (unsigned)((nq * 32 + 255) / 256);
+  if (type == MV_IVF_FLAT)
+    k_rekey<MV_IVF_FLAT><<<grid, 256, 0, st>>>(poff, pcnt, part, nq, npb, tau2, qerr, metric, qpad, dpad, payload,
+                                               row_of_rank, vmin, vdiff, sq8_t, gate);
+  else
+    k_rekey<MV_IVF_SQ8><<<grid, 256, 0, st>>>(poff, pcnt, part, nq, npb, tau2, qerr, metric, qpad, dpad, payload,
+                                              row_of_rank, vmin, vdiff, sq8_t, gate);
   return cudaGetLastError();
 }
 

@@ -39,8 +39,8 @@ struct mv_index {
   int64_t* ids = nullptr;       // ntotal, storage order
   uint32_t* rank = nullptr;     // ntotal: position of (id, row) in sorted order
   int64_t* sorted_ids = nullptr;  // ntotal: ids in (id, row) order
-  uint32_t* row_of_rank = nullptr;  // FLAT: storage row of each rank (exact re-scoring)
-  double xmax2 = 0.0;           // FLAT: max ||x||^2 over the stored rows (filter-mode error bound)
+  uint32_t* row_of_rank = nullptr;  // storage row of each rank (the filter mode's exact re-scoring)
+  double xmax2 = 0.0;           // max ||x||^2 (SQ8: ||x_hat||^2) over the stored rows (filter-mode bound)
   XMaps xm;                     // payload tensor maps: 128/64/32/16-row boxes (rebuilt by every add)
   bool tf32_exact = true;       // FLAT: every stored value exactly representable in tf32
   const char* last_scan = "none";
@@ -460,12 +460,15 @@ mv_status mv_index_add(mv_index* ix, const float* vectors, const int64_t* ids, i
     const int64_t ldg = ((nlist + 127) / 128) * 4;
     const int64_t sub = std::min<int64_t>(n, std::max<int64_t>(4096, (int64_t(1) << 27) / ldg));
     float* qhl;
+    int* lo_any;  // the rows' lo planes vanish (integer data): the GEMM's wide mode
     CK(s.alloc(&qhl, (size_t)2 * sub * dpad));
+    CK(s.alloc(&lo_any, 1));
     for (int64_t r0 = 0; r0 < n; r0 += sub) {
       const int64_t m = std::min(sub, n - r0);
-      Scratch sb(ix, st);  // the block's score matrix, freed (stream-ordered) before the next block
-      CK(launch_hilo(x + r0 * ix->d, m, ix->d, dpad, qhl, nullptr, st));
-      CK(run_coarse(ix, qhl, nullptr, m, 1, lists + r0, sb, st));
+      Scratch sb(ix, st);  // the block's coarse scratch, freed (stream-ordered) before the next block
+      CK(cudaMemsetAsync(lo_any, 0, sizeof(int), st));
+      CK(launch_hilo(x + r0 * ix->d, m, ix->d, dpad, qhl, lo_any, st));
+      CK(run_coarse(ix, qhl, lo_any, m, 1, lists + r0, sb, st));
     }
   }
   CK(cudaMemsetAsync(cnt, 0, sizeof(int32_t) * nlist, st));
@@ -497,9 +500,8 @@ mv_status mv_index_add(mv_index* ix, const float* vectors, const int64_t* ids, i
   nx.ids = (int64_t*)mem_alloc(ix, sizeof(int64_t) * (ntot + kSidePad), st);
   nx.rank = (uint32_t*)mem_alloc(ix, sizeof(uint32_t) * (ntot + kSidePad), st);
   nx.sorted_ids = (int64_t*)mem_alloc(ix, sizeof(int64_t) * ntot, st);
-  if (ix->type == MV_IVF_FLAT) nx.row_of_rank = (uint32_t*)mem_alloc(ix, sizeof(uint32_t) * ntot, st);
-  if (!nx.payload || !nx.norms || !nx.ids || !nx.rank || !nx.sorted_ids ||
-      (ix->type == MV_IVF_FLAT && !nx.row_of_rank)) {
+  nx.row_of_rank = (uint32_t*)mem_alloc(ix, sizeof(uint32_t) * ntot, st);
+  if (!nx.payload || !nx.norms || !nx.ids || !nx.rank || !nx.sorted_ids || !nx.row_of_rank) {
     free_storage(&nx);
     return fail(MV_ENOMEM, "add: cannot allocate storage for %lld vectors", (long long)ntot);
   }
@@ -531,10 +533,10 @@ mv_status mv_index_add(mv_index* ix, const float* vectors, const int64_t* ids, i
     CK(cudaMemsetAsync(flag, 0, sizeof(int), st));
     CK(launch_tf32_check(xpad, (int64_t)n * dpad, flag, st));
     CK(cudaMemcpyAsync(&hflag, flag, sizeof(int), cudaMemcpyDeviceToHost, st));
-    CK(cudaMemsetAsync(xm, 0, sizeof(unsigned long long), st));
-    CK(launch_max_f64(nx.norms, ntot, xm, st));
-    CK(cudaMemcpyAsync(&hxm, xm, sizeof(unsigned long long), cudaMemcpyDeviceToHost, st));
   }
+  CK(cudaMemsetAsync(xm, 0, sizeof(unsigned long long), st));
+  CK(launch_max_f64(nx.norms, ntot, xm, st));
+  CK(cudaMemcpyAsync(&hxm, xm, sizeof(unsigned long long), cudaMemcpyDeviceToHost, st));
   CK(cudaMemcpyAsync(ix->list_off, new_off, sizeof(int64_t) * (nlist + 1), cudaMemcpyDeviceToDevice, st));
   CK(cudaMemcpyAsync(ix->h_list_off.data(), new_off, sizeof(int64_t) * (nlist + 1), cudaMemcpyDeviceToHost, st));
   CK(cudaStreamSynchronize(st));
@@ -549,12 +551,10 @@ mv_status mv_index_add(mv_index* ix, const float* vectors, const int64_t* ids, i
   nx.ids = nx.sorted_ids = nullptr;
   nx.rank = nx.row_of_rank = nullptr;
   ix->ntotal = ntot;
-  if (ix->type == MV_IVF_FLAT) {
-    if (hflag) ix->tf32_exact = false;
-    double xm2;
-    memcpy(&xm2, &hxm, sizeof xm2);
-    ix->xmax2 = xm2;
-  }
+  if (ix->type == MV_IVF_FLAT && hflag) ix->tf32_exact = false;
+  double xm2;
+  memcpy(&xm2, &hxm, sizeof xm2);
+  ix->xmax2 = xm2;
   // one swizzle atom per box row: 128 B (FLAT: 32 fp32; SQ8 when dpad is a multiple of 128), else 32 B
   const bool wide = ix->type == MV_IVF_FLAT || dpad % 128 == 0;
   for (int i = 0; i < 4; ++i)
@@ -613,9 +613,12 @@ mv_status mv_search_probes(mv_index* ix, const float* queries, int64_t nq, int32
     int32_t* P = probes + q0 * npb;
     if (sp) CK(s.alloc(&P, (size_t)m * npb));
     float* qhl;
+    int* lo_any;
     CK(s.alloc(&qhl, (size_t)2 * m * ix->dpad));
-    CK(launch_hilo(q + q0 * ix->d, m, ix->d, ix->dpad, qhl, nullptr, st));
-    CK(run_coarse(ix, qhl, nullptr, m, npb, P, s, st));
+    CK(s.alloc(&lo_any, 1));
+    CK(cudaMemsetAsync(lo_any, 0, sizeof(int), st));
+    CK(launch_hilo(q + q0 * ix->d, m, ix->d, ix->dpad, qhl, lo_any, st));
+    CK(run_coarse(ix, qhl, lo_any, m, npb, P, s, st));
     if (sp) CK(cudaMemcpyAsync(probes + q0 * npb, P, sizeof(int32_t) * m * npb, cudaMemcpyDeviceToHost, st));
   }
   if (sp || sq) CK(cudaStreamSynchronize(st));
@@ -732,15 +735,15 @@ static mv_status search_chunk(mv_index* ix, const float* q, int64_t nq, int32_t 
   CK(s.alloc(&qn64, (size_t)nq));
   CK(s.alloc(&tau, (size_t)nq));
   CK(cudaMemsetAsync(tau, 0xff, sizeof(uint64_t) * nq, st));
-  // FLAT filter mode (DESIGN.md §5 "FLAT precision"): the tensor-core badness carries a rigorous
-  // error bound E_q when the stored values (always) or the queries (device flag) are not
-  // tf32-exact; the keys are then re-scored exactly before the final select
-  const bool approx_always = flat && !ix->tf32_exact;
+  // filter mode: the tensor-core badness carries a rigorous error bound E_q -- SQ8
+  // always, FLAT when the stored values (always) or the queries (device flag) are not tf32-exact;
+  // the keys are then re-scored exactly before the final select
+  const bool approx_always = !flat || !ix->tf32_exact;
   const int* gate = approx_always ? nullptr : qlo_any;
   FlatErr fe{ix->tf32_exact ? 0.0 : 0x1p-10, ix->tf32_exact ? 0x1p-21 : 0x1p-11, ix->xmax2, ix->metric};
-  if (flat) CK(s.alloc(&qerr, (size_t)nq));
-  CK(launch_qplanes(ix->type, qpad, nq, dpad, ix->vmin, ix->vdiff, flat ? nullptr : qplanes, qscale, qa, qn64,
-                    flat ? &fe : nullptr, qerr, st));
+  CK(s.alloc(&qerr, (size_t)nq));
+  CK(launch_qplanes(ix->type, qpad, nq, dpad, ix->vmin, ix->vdiff, flat ? nullptr : qplanes, qscale, qa, qn64, &fe,
+                    qerr, st));
   tp.metric = ix->metric; tp.npb = npb; tp.nq = nq;
   tp.list_off = ix->list_off; tp.norms = ix->norms; tp.ids = ix->ids; tp.rank = ix->rank;
   tp.bitset = bs; tp.nbits = bs ? nbits : 0;
@@ -772,25 +775,34 @@ static mv_status search_chunk(mv_index* ix, const float* q, int64_t nq, int32_t 
     prof_mark(ix, st);
   }
   prof_mark(ix, st);
-  if (flat) {
-    // filter mode: t~_q = the k-th best approximate key, then exact re-scoring of the keys within
-    // 2 E_q of it (both skipped on the device when the search is exact: gate = qlo_any == 0)
+  if (k <= 256) {
+    // a7 with the filter mode's exact re-scoring fused in (a plain exact select when the search is
+    // exact: FLAT with tf32-exact data and queries, gate = qlo_any == 0 on the device)
+    uint64_t* tau2;
+    int* notgate;
+    CK(s.alloc(&tau2, (size_t)nq));
+    CK(s.alloc(&notgate, 1));
+    CK(launch_final_refine(ix->type, b.poff, b.pcnt, part, nq, npb, k, ix->metric, ix->sorted_ids, D, I, qerr, qpad,
+                           dpad, ix->payload, ix->row_of_rank, ix->vmin, ix->vdiff, ix->sq8_t, gate, tau2, notgate, st));
+  } else {
+    // filter mode: t~_q = the k-th best approximate key, exact re-scoring in place of the keys within
+    // 2 E_q of it (both skipped on the device when the search is exact), then a7
     uint64_t* tau2;
     CK(s.alloc(&tau2, (size_t)nq));
     CK(cudaMemsetAsync(tau2, 0xff, sizeof(uint64_t) * nq, st));
     CK(launch_tau_select(b.poff, b.pcnt, part, nq, npb, nullptr, k, tau2, tmax, over, gate, ix->opt.large_k_select,
                          st));
-    CK(launch_rekey(b.poff, b.pcnt, part, nq, npb, tau2, qerr, ix->metric, qpad, dpad,
-                    reinterpret_cast<const float*>(ix->payload), ix->row_of_rank, gate, st));
+    CK(launch_rekey(ix->type, b.poff, b.pcnt, part, nq, npb, tau2, qerr, ix->metric, qpad, dpad, ix->payload,
+                    ix->row_of_rank, ix->vmin, ix->vdiff, ix->sq8_t, gate, st));
     ix->launches += 2;
+    CK(launch_final_select(b.poff, b.pcnt, part, nq, npb, k, ix->metric, ix->sorted_ids, D, I, tmax, over,
+                           ix->opt.large_k_select, st));
   }
-  // a7
-  CK(launch_final_select(b.poff, b.pcnt, part, nq, npb, k, ix->metric, ix->sorted_ids, D, I, tmax, over,
-                         ix->opt.large_k_select, st));
   prof_mark(ix, st);
   ix->last_scan = flat ? "tcgen05.tf32" : "tcgen05.i8";
-  // prep, hilo, coarse GEMM + probe select, plan, qplanes, scan A (+ tau select, scan B), final select
-  ix->launches += (P_in ? 5 : (npb >= nlist ? 6 : 7)) + (split ? 3 : 1);
+  // prep, hilo, coarse (GEMM pass 0, group bound, GEMM pass 1, top-nprobe | all lists), plan, qplanes,
+  // scan A (+ seed select, scan B), final select
+  ix->launches += 5 + (P_in ? 0 : (npb >= nlist ? 1 : 4)) + (split ? 2 : 0) + 1;
   return MV_OK;
 }
 
@@ -916,7 +928,7 @@ mv_status mv_merge_topk(mv_metric metric, const float* dists, const int64_t* ids
 
 mv_status mv_index_describe(const mv_index* ix, char* buf, size_t len) {
   if (!ix || !buf || len == 0) return fail(MV_EINVAL, "null argument");
-  const char* refine = ix->type != MV_IVF_FLAT ? "n/a (SQ8: exact int32 digit partials)"
+  const char* refine = ix->type != MV_IVF_FLAT ? "always (SQ8 digit-plane filter)"
                        : ix->tf32_exact        ? "when a query is not tf32-exact"
                                                : "always (stored values not tf32-exact)";
   snprintf(buf, len,

@@ -284,8 +284,8 @@ struct TcScanParams {
   int32_t* pcnt;           // per pair: keys emitted
   uint64_t* part;
   const uint64_t* tau;     // nq: per-query bound for phase B (exact k-th key of phase A)
-  int approx_always;       // FLAT: stored values not tf32-exact -> filter mode for every search
-  const float* qerr;       // FLAT filter mode: E_q, the bound on |approximate - exact badness|
+  int approx_always;       // FLAT: stored values not tf32-exact -> filter mode for every search (SQ8: always)
+  const float* qerr;       // filter mode: E_q, the bound on |approximate - exact badness|
   unsigned long long* prof;  // -DMV_SCAN_TRACE builds only: CTA-0 timeline
 };
 bool tc_scan_plan(int type, int dpad, int k, double qpl, const Options& o, TcScanParams& p);  // qpl: queries per probed list
@@ -294,8 +294,9 @@ struct XMaps {
   CUtensorMap m[4];
 };
 cudaError_t launch_scan_tc(const XMaps& xm, const TcScanParams& p, cudaStream_t st);
-// FLAT filter-mode error model: ex / eq = relative representation error of the
-// stored value / of the query as the MMA sees them, xmax2 = max ||x||^2 over the index
+// filter-mode error model: FLAT ex / eq = relative representation error of the
+// stored value / of the query as the MMA sees them; xmax2 = max ||x||^2 (SQ8: ||x_hat||^2) over the
+// index
 struct FlatErr {
   double ex, eq, xmax2;
   int metric;
@@ -344,11 +345,19 @@ cudaError_t launch_final_select(const int64_t* poff, const int32_t* pcnt, const 
 cudaError_t launch_tau_select(const int64_t* poff, const int32_t* pcnt, const uint64_t* part, int64_t nq, int npb,
                               const int32_t* nuse, int k, uint64_t* tau, int64_t tmax, uint8_t* over,
                               const int* gate, int big_mode, cudaStream_t st);
-// FLAT filter mode: exact fp64 re-scoring of the keys at or below tau2[q] + 2 qerr[q] (the others
-// become padding); gate (nullable): skipped when *gate == 0
-cudaError_t launch_rekey(const int64_t* poff, const int32_t* pcnt, uint64_t* part, int64_t nq, int npb,
+// k <= 256: the final select with the filter mode's fused exact re-scoring (k_final_warp<R, type>);
+// rgate (nullable = always): refine only when *rgate != 0, else the plain exact select
+cudaError_t launch_final_refine(int type, const int64_t* poff, const int32_t* pcnt, const uint64_t* part, int64_t nq,
+                                int npb, int k, int metric, const int64_t* sorted_ids, float* out_d, int64_t* out_i,
+                                const float* qerr, const float* qpad, int dpad, const void* payload,
+                                const uint32_t* row_of_rank, const float* vmin, const float* vdiff, const float* sq8_t,
+                                const int* rgate, uint64_t* tau2, int* notgate, cudaStream_t st);
+// k > 256, filter mode: exact fp64 re-scoring in place of the keys at or below tau2[q] + 2 qerr[q];
+// gate (nullable): skipped when *gate == 0
+cudaError_t launch_rekey(int type, const int64_t* poff, const int32_t* pcnt, uint64_t* part, int64_t nq, int npb,
                          const uint64_t* tau2, const float* qerr, int metric, const float* qpad, int dpad,
-                         const float* payload, const uint32_t* row_of_rank, const int* gate, cudaStream_t st);
+                         const void* payload, const uint32_t* row_of_rank, const float* vmin, const float* vdiff,
+                         const float* sq8_t, const int* gate, cudaStream_t st);
 cudaError_t launch_fill_pad(int64_t n, int metric, float* d, int64_t* i, cudaStream_t st);
 cudaError_t launch_merge2(int metric, const float* ad, const int64_t* ai, const float* bd, const int64_t* bi,
                           int64_t nq, int k, float* od, int64_t* oi, cudaStream_t st);
