@@ -219,6 +219,187 @@ __global__ void __launch_bounds__(kCThreads, 1)
   }
 }
 
+// dpad <= 128: the same two passes with the QUERIES on the MMA's M side.  CTA = 128 queries (A
+// operand: hi [+ lo] planes resident in shared memory) x a range of 128-centroid tiles (B operand:
+// centroid hi and lo planes streamed by TMA, 32 dims per stage).  D[128 q x 128 c] += Q_hi C_hi^T
+// + Q_hi C_lo^T (+ Q_lo C_hi^T): the same products as k_coarse_gemm, one accumulator.  The
+// epilogue owns one query per thread and one 32-centroid group per warp (16 epilogue warps, four
+// per TMEM lane quarter): a group minimum is a register fminf chain over the thread's 32 columns --
+// no cross-lane reduction -- and pass 1 touches a group's keys only when that minimum passes the
+// thread's own bound (held in a register).  The centroid norms of each tile come in by bulk copy.
+constexpr int kQmEpi = 16;
+constexpr int kQmThreads = 64 + 32 * kQmEpi;
+constexpr int kQmAcc = 2;  // TMEM accumulators of 128 columns (3 centroid stages fit next to the queries at dpad 128)
+
+__global__ void __launch_bounds__(kQmThreads, 1)
+    k_coarse_qm(const __grid_constant__ CUtensorMap cmap, const __grid_constant__ CUtensorMap qmap,
+                const CoarseParams p) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~(uintptr_t)1023);
+  constexpr int ATOM = 128;
+  constexpr int PBYTES = 128 * ATOM;  // one 32-dim chunk of 128 rows of one plane
+  const int nchunks = p.nchunks, nstage = p.nstage;
+  const int ntiles_all = (p.nlist + 127) >> 7;
+  const int qb = blockIdx.x / p.csplit, cs = blockIdx.x % p.csplit;
+  const int t0 = (int)((int64_t)ntiles_all * cs / p.csplit), t1 = (int)((int64_t)ntiles_all * (cs + 1) / p.csplit);
+  const int q0 = qb * 128;
+  const bool qlo = p.qlo_any == nullptr || *p.qlo_any != 0;
+
+  uint8_t* Aq = sm;                                     // [2 planes][nchunks][128 rows][128 B]
+  uint8_t* Bs = Aq + 2 * nchunks * PBYTES;              // nstage x (hi chunk, lo chunk)
+  float* cns = reinterpret_cast<float*>(Bs + nstage * 2 * PBYTES);  // kQmAcc x 128 centroid norms
+  uint64_t* bars = reinterpret_cast<uint64_t*>(cns + kQmAcc * 128);
+  uint64_t* full_a = bars;
+  uint64_t* full_b = full_a + 1;
+  uint64_t* empty_b = full_b + nstage;
+  uint64_t* tfull = empty_b + nstage;
+  uint64_t* tempty = tfull + kQmAcc;
+  uint64_t* full_c = tempty + kQmAcc;
+  uint32_t* tslot = reinterpret_cast<uint32_t*>(full_c + kQmAcc);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x == 0) {
+    mbar_init(full_a, 1);
+    for (int s = 0; s < nstage; ++s) {
+      mbar_init(&full_b[s], 1);
+      mbar_init(&empty_b[s], 1);
+    }
+    for (int a = 0; a < kQmAcc; ++a) {
+      mbar_init(&tfull[a], 1);
+      mbar_init(&tempty[a], kQmEpi);
+      mbar_init(&full_c[a], 1);
+    }
+    fence_mbar_init();
+  }
+  if (warp == 1) {
+    tmem_alloc(tslot, 128 * kQmAcc);
+    tmem_relinquish();
+  }
+  if (warp == 0 && lane == 0) {
+    tma_prefetch(&cmap);
+    tma_prefetch(&qmap);
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tslot;
+
+  if (warp == 0) {
+    if (lane == 0) {
+      // the query block: hi rows [q0, q0+128) (and lo rows [nq + q0, ...)) of the plane-major matrix
+      mbar_expect_tx(full_a, (qlo ? 2 : 1) * nchunks * PBYTES);
+      for (int pl = 0; pl < (qlo ? 2 : 1); ++pl)
+        for (int c = 0; c < nchunks; ++c)
+          tma_load_2d(Aq + (pl * nchunks + c) * PBYTES, &qmap, full_a, c * 32, pl * (int)p.nq + q0);
+      uint32_t it = 0;
+      for (int t = t0, tl = 0; t < t1; ++t, ++tl) {
+        const uint32_t a = tl % kQmAcc;
+        // the tile's centroid norms, once the epilogue is done with the slot's previous tile
+        mbar_wait(&tempty[a], ((tl / kQmAcc) & 1) ^ 1);
+        mbar_expect_tx(&full_c[a], 512);
+        bulk_g2s(cns + a * 128, p.cnorm + (int64_t)t * 128, 512, &full_c[a]);
+        for (int c = 0; c < nchunks; ++c, ++it) {
+          const uint32_t s = it % nstage, r = it / nstage;
+          mbar_wait(&empty_b[s], (r & 1) ^ 1);
+          mbar_expect_tx(&full_b[s], 2 * PBYTES);
+          tma_load_2d(Bs + s * 2 * PBYTES, &cmap, &full_b[s], c * 32, t * 128);
+          tma_load_2d(Bs + s * 2 * PBYTES + PBYTES, &cmap, &full_b[s], c * 32, p.nlist + t * 128);
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0) {
+      mbar_wait(full_a, 0);
+      tc_fence_after();
+      const uint32_t id = idesc_tf32(128);
+      uint32_t it = 0;
+      for (int t = t0, tl = 0; t < t1; ++t, ++tl) {
+        const uint32_t a = tl % kQmAcc;
+        mbar_wait(&tempty[a], ((tl / kQmAcc) & 1) ^ 1);
+        tc_fence_after();
+        const uint32_t d = tmem + a * 128;
+        for (int c = 0; c < nchunks; ++c, ++it) {
+          const uint32_t s = it % nstage;
+          mbar_wait(&full_b[s], (it / nstage) & 1);
+          tc_fence_after();
+          const uint32_t qh = smem_u32(Aq + c * PBYTES), ql = smem_u32(Aq + (nchunks + c) * PBYTES);
+          const uint32_t ch = smem_u32(Bs + s * 2 * PBYTES), cl = ch + PBYTES;
+#pragma unroll
+          for (int ks = 0; ks < 4; ++ks) {
+            mma_tf32(d, kmajor_desc(qh + ks * 32, ATOM), kmajor_desc(ch + ks * 32, ATOM), id, (c | ks) != 0);
+            mma_tf32(d, kmajor_desc(qh + ks * 32, ATOM), kmajor_desc(cl + ks * 32, ATOM), id, 1);
+            if (qlo) mma_tf32(d, kmajor_desc(ql + ks * 32, ATOM), kmajor_desc(ch + ks * 32, ATOM), id, 1);
+          }
+          mma_commit(&empty_b[s]);
+        }
+        mma_commit(&tfull[a]);
+      }
+    }
+  } else {
+    // ------------------------------------------------------------------ epilogue
+    const int ew = warp - 2;           // 0..15
+    const int quarter = warp & 3;      // TMEM lane quarter: queries quarter*32 .. +31
+    const int gsub = ew >> 2;          // this warp's group within the tile (columns 32 gsub .. +31)
+    const int64_t q = q0 + quarter * 32 + lane;
+    const bool vq = q < p.nq;
+    const bool l2 = p.metric == MV_L2;
+    const int ngr = (p.nlist + 31) / 32;
+    const uint64_t bq = (p.mode == 1 && vq) ? __ldg(p.gbound + q) : 0ull;
+    const uint32_t bk = (uint32_t)(bq >> 32), bg = (uint32_t)bq;
+    for (int t = t0, tl = 0; t < t1; ++t, ++tl) {
+      const uint32_t a = tl % kQmAcc;
+      const uint32_t grp = (uint32_t)(t * 4 + gsub);
+      const int c0 = t * 128 + gsub * 32;  // first centroid of the group
+      mbar_wait(&full_c[a], (tl / kQmAcc) & 1);
+      mbar_wait(&tfull[a], (tl / kQmAcc) & 1);
+      tc_fence_after();
+      uint32_t rd[32];
+      tmem_ld32(tmem + a * 128 + gsub * 32 + ((uint32_t)(quarter * 32) << 16), rd);
+      tmem_wait_ld();
+      const float4* cn4 = reinterpret_cast<const float4*>(cns + a * 128 + gsub * 32);
+      float sc[32];
+      float mn = __int_as_float(0x7f800000);
+#pragma unroll
+      for (int v = 0; v < 8; ++v) {
+        const float4 cv = cn4[v];
+        const float cvv[4] = {cv.x, cv.y, cv.z, cv.w};
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const int j = 4 * v + u;
+          const float dot = __uint_as_float(rd[j]);
+          sc[j] = c0 + j < p.nlist ? (l2 ? cvv[u] - 2.0f * dot : -dot) : __int_as_float(0x7f800000);
+          mn = fminf(mn, sc[j]);
+        }
+      }
+      const uint32_t kmin = f2key(mn);
+      if (p.mode == 0) {
+        if (vq && grp < (uint32_t)ngr) p.G[q * p.ldg + grp] = kmin;
+      } else if (vq && grp < (uint32_t)ngr && (kmin < bk || (kmin == bk && grp <= bg))) {
+        // one of the query's nprobe groups: its 32 keys (padding above the bound) to the group's slots
+        const int sl = (int)__ldg(p.gslot + q * (int64_t)ngr + grp);
+        uint64_t* dst = p.cand + q * (int64_t)p.ccap + sl * 32;
+#pragma unroll
+        for (int j = 0; j < 32; j += 2) {
+          const uint32_t k0 = f2key(sc[j]), k1 = f2key(sc[j + 1]);
+          const bool p0 = c0 + j < p.nlist && (k0 < bk || (k0 == bk && grp <= bg));
+          const bool p1 = c0 + j + 1 < p.nlist && (k1 < bk || (k1 == bk && grp <= bg));
+          reinterpret_cast<ulonglong2*>(dst)[j / 2] =
+              make_ulonglong2(p0 ? (((uint64_t)k0 << 32) | (uint32_t)(c0 + j)) : MV_KEY_PAD,
+                              p1 ? (((uint64_t)k1 << 32) | (uint32_t)(c0 + j + 1)) : MV_KEY_PAD);
+        }
+      }
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&tempty[a]);
+    }
+  }
+  __syncthreads();
+  if (warp == 1) {
+    tc_fence_after();
+    tmem_dealloc(tmem, 128 * kQmAcc);
+  }
+}
+
 // gbound[q] = the nprobe-th smallest (group minimum key, group id) of the query's G row, and
 // gslot[q][g] = the rank (in group order) of group g among the nprobe groups at or below it, -1
 // for the others: pass 1 writes a selected group's 32 keys to slots [32 rank, 32 rank + 32) of
@@ -404,6 +585,25 @@ cudaError_t launch_hilo(const float* x, int64_t n, int d, int dpad, float* out, 
 // (waves x per-CTA work) on nsm SMs, with >= 2 centroid stages in shared memory.
 bool coarse_tc_plan(int dpad, int nprobe, int64_t nq, int nlist, int nsm, const Options& o, CoarseParams& p) {
   if (dpad % 32 != 0 || nprobe > 1024) return false;
+  if (dpad <= 128 && o.coarse_nqb == 0) {
+    // queries on the M side (k_coarse_qm): 128 queries per CTA; centroid splits fill the SMs
+    p.qm = 1;
+    p.nchunks = dpad / 32;
+    p.nprobe = nprobe;
+    p.nqb = 128;
+    const int ntiles = (nlist + 127) / 128;
+    const int64_t blocks = (nq + 127) / 128;
+    p.csplit = (int)std::max<int64_t>(1, std::min<int64_t>(ntiles, (2 * nsm + blocks - 1) / blocks));
+    if (o.coarse_cs > 0) p.csplit = std::max(1, std::min(ntiles, o.coarse_cs));
+    const int fixed = 2 * p.nchunks * 128 * 128 + kQmAcc * 128 * 4 + 256 + 1024;
+    p.nstage = std::min(8, (227 * 1024 - fixed) / (2 * 128 * 128));
+    p.smem_total = fixed + p.nstage * 2 * 128 * 128;
+    p.nepi = 16;
+    p.nacc = kQmAcc;
+    p.tmem_cols = 128 * kQmAcc;
+    return p.nstage >= 2 && p.smem_total <= 227 * 1024;
+  }
+  p.qm = 0;
   p.nchunks = dpad / 32;
   p.nprobe = nprobe;
   const int budget = 227 * 1024 - 1024 - 256;  // alignment slack, barriers
@@ -447,11 +647,13 @@ bool coarse_tc_plan(int dpad, int nprobe, int64_t nq, int nlist, int nsm, const 
 cudaError_t launch_coarse_tc(const CUtensorMap* cmap, const CUtensorMap* qmap, const CoarseParams& p0, int64_t nq,
                              cudaStream_t st) {
   const unsigned grid = (unsigned)(((nq + p0.nqb - 1) / p0.nqb) * p0.csplit);
-  cudaError_t e = cudaFuncSetAttribute(k_coarse_gemm, cudaFuncAttributeMaxDynamicSharedMemorySize, p0.smem_total);
+  auto kern = p0.qm ? k_coarse_qm : k_coarse_gemm;
+  const int nthr = p0.qm ? kQmThreads : 64 + 32 * p0.nepi;
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, p0.smem_total);
   if (e != cudaSuccess) return e;
   CoarseParams p = p0;
   p.mode = 0;  // pass 0: group minima
-  k_coarse_gemm<<<grid, 64 + 32 * p.nepi, p.smem_total, st>>>(*cmap, *qmap, p);
+  kern<<<grid, nthr, p.smem_total, st>>>(*cmap, *qmap, p);
   if ((e = cudaGetLastError()) != cudaSuccess) return e;
   const unsigned gw = (unsigned)((nq * 32 + 255) / 256);
   const int ng = (p.nlist + 31) / 32;
@@ -465,7 +667,7 @@ cudaError_t launch_coarse_tc(const CUtensorMap* cmap, const CUtensorMap* qmap, c
   // fewer groups than probes: every group is selected and the slots past them stay padding
   if (ng < p.nprobe && (e = cudaMemsetAsync(p.cand, 0xff, sizeof(uint64_t) * nq * p.ccap, st)) != cudaSuccess) return e;
   p.mode = 1;  // pass 1: the same scores, the selected groups' keys stored to their slots
-  k_coarse_gemm<<<grid, 64 + 32 * p.nepi, p.smem_total, st>>>(*cmap, *qmap, p);
+  kern<<<grid, nthr, p.smem_total, st>>>(*cmap, *qmap, p);
   if ((e = cudaGetLastError()) != cudaSuccess) return e;
   const int R = (p.nprobe + 31) / 32;
   if (R <= 1) k_probe_final<1><<<gw, 256, 0, st>>>(p.cand, p.ccap, nq, p.nprobe, p.probes);

@@ -728,7 +728,7 @@ bool tc_scan_plan(int type, int dpad, int k, double qpl, const Options& o, TcSca
   int qcmax = type == MV_IVF_FLAT ? 96 : 64;
   // tuning options (mv_index_set_option "sq8_qc" / "flat_qc"): launch shape only, never the result
   if (o.sq8_qc > 0 && type == MV_IVF_SQ8) qcmax = std::max(16, std::min(64, o.sq8_qc / 16 * 16));
-  if (o.flat_qc > 0 && type == MV_IVF_FLAT) qcmax = std::max(16, std::min(96, o.flat_qc / 16 * 16));
+  if (o.flat_qc > 0 && type == MV_IVF_FLAT) qcmax = std::max(16, std::min(128, o.flat_qc / 16 * 16));
   const int nscap = wide ? 8 : 24;
   const int nsmin = wide ? 4 : 6;  // >= 64 KB (16-KB stages) / 24 KB (4-KB stages) of list tiles in flight
   p.k = k;

@@ -292,13 +292,14 @@ mv_status mv_index_create(int32_t d, mv_metric metric, mv_type type, int32_t nli
   ix->top_len_prefix.assign(nlist + 1, 0);
   bool ok = (ix->list_off = (int64_t*)mem_alloc(ix, sizeof(int64_t) * (nlist + 1), nullptr)) &&
             (ix->cpad = (float*)mem_alloc(ix, sizeof(float) * (size_t)nlist * ix->dpad, nullptr)) &&
-            (ix->cnorm = (float*)mem_alloc(ix, sizeof(float) * nlist, nullptr)) &&
+            (ix->cnorm = (float*)mem_alloc(ix, sizeof(float) * ((size_t)(nlist + 127) / 128 * 128), nullptr)) &&
             (ix->chl = (float*)mem_alloc(ix, sizeof(float) * 2 * (size_t)nlist * ix->dpad, nullptr)) &&
             (ix->vmin = (float*)mem_alloc(ix, sizeof(float) * ix->dpad, nullptr)) &&
             (ix->vdiff = (float*)mem_alloc(ix, sizeof(float) * ix->dpad, nullptr)) &&
             (ix->sq8_t = (float*)mem_alloc(ix, sizeof(float) * 256, nullptr));
   cudaError_t e = ok ? cudaSuccess : cudaErrorMemoryAllocation;
   if (e == cudaSuccess) e = cudaMemset(ix->list_off, 0, sizeof(int64_t) * (nlist + 1));
+  if (e == cudaSuccess) e = cudaMemset(ix->cnorm, 0, sizeof(float) * ((size_t)(nlist + 127) / 128 * 128));
   if (e == cudaSuccess) {
     float t[256];
     for (int c = 0; c < 256; ++c) t[c] = ((float)c + 0.5f) / 255.0f;  // oracle.sq8_decode's first two ops
@@ -325,7 +326,7 @@ mv_status mv_index_set_option(mv_index* ix, const char* name, int64_t value) {
   else if (n == "need") o.need = value;
   else if (n == "capa") o.capa = value;
   else if (n == "sq8_qc") o.sq8_qc = (int)std::min<int64_t>(value, 64);
-  else if (n == "flat_qc") o.flat_qc = (int)std::min<int64_t>(value, 96);
+  else if (n == "flat_qc") o.flat_qc = (int)std::min<int64_t>(value, 128);
   else if (n == "coarse_nqb") o.coarse_nqb = (int)std::min<int64_t>(value, 128);
   else if (n == "coarse_cs") o.coarse_cs = (int)std::min<int64_t>(value, 64);
   else if (n == "coarse_epi") o.coarse_epi = (int)std::min<int64_t>(value, 16);

@@ -174,7 +174,7 @@ struct Options {
   int64_t need = 0;         // seeding sample size (candidates); clamped to >= max(2k, k + 32)
   int64_t capa = 0;         // rows per list of the seeding sample (16-row multiple)
   int sq8_qc = 0;           // SQ8 queries per scan work item (16..64)
-  int flat_qc = 0;          // FLAT queries per scan work item (16..96)
+  int flat_qc = 0;          // FLAT queries per scan work item (16..128)
   int coarse_nqb = 0, coarse_cs = 0, coarse_epi = 0, coarse_nacc = 0;  // coarse GEMM launch shape
   int64_t workspace = 0;    // per-search scratch budget in bytes (0: half of the free device memory)
   int large_k_select = 0;   // k > 256: 0 staged radix select, 1 sample-threshold select (radix fallback)
@@ -316,7 +316,8 @@ struct CoarseParams {
   int64_t nq;
   int nlist, nchunks, nstage, nprobe, nqb, csplit, tmem_cols, metric, smem_total;
   int nepi, nacc;          // epilogue warps (multiple of 4, <= 16), TMEM accumulators (<= 4)
-  int mode;                // 0: group minima -> G; 1: append keys <= gbound -> cand
+  int mode;                // 0: group minima -> G; 1: the selected groups' keys -> cand
+  int qm;                  // 1: k_coarse_qm (queries on the MMA's M side, dpad <= 128)
   const float* cnorm;
   uint32_t* G;             // nq x ldg: minimum score key of each 32-centroid group (ldg = 4 ceil(nlist/128))
   int64_t ldg;
