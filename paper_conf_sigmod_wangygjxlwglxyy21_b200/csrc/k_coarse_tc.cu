@@ -201,8 +201,9 @@ __global__ void __launch_bounds__(kCThreads, 1)
               if (!((any >> j) & 1)) continue;  // warp-uniform
               const int slj = __shfl_sync(MV_FULL, sl, j);
               const bool pass = (m[j] >> lane) & 1;
-              p.cand[(q0 + qc + j) * (int64_t)p.ccap + slj * 32 + lane] =
-                  pass ? (((uint64_t)key[j] << 32) | (uint32_t)cid) : MV_KEY_PAD;
+              const int64_t qq = q0 + qc + j;  // passing keys compacted, their count in ccnt
+              if (pass) p.cand[qq * p.ccap + slj * 32 + __popc(m[j] & ((1u << lane) - 1))] = ((uint64_t)key[j] << 32) | (uint32_t)cid;
+              if (lane == 0) p.ccnt[qq * p.nprobe + slj] = (uint8_t)__popc(m[j]);
             }
           }
         }
@@ -229,7 +230,8 @@ __global__ void __launch_bounds__(kCThreads, 1)
 // thread's own bound (held in a register).  The centroid norms of each tile come in by bulk copy.
 constexpr int kQmEpi = 16;
 constexpr int kQmThreads = 64 + 32 * kQmEpi;
-constexpr int kQmAcc = 2;  // TMEM accumulators of 128 columns (3 centroid stages fit next to the queries at dpad 128)
+constexpr int kQmAcc = 2;      // TMEM accumulators of 128 columns
+constexpr int kQmMaxStage = 8;  // centroid ring stages (3 next to hi+lo query planes at dpad 128, 5 next to hi only)
 
 __global__ void __launch_bounds__(kQmThreads, 1)
     k_coarse_qm(const __grid_constant__ CUtensorMap cmap, const __grid_constant__ CUtensorMap qmap,
@@ -238,21 +240,25 @@ __global__ void __launch_bounds__(kQmThreads, 1)
   uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~(uintptr_t)1023);
   constexpr int ATOM = 128;
   constexpr int PBYTES = 128 * ATOM;  // one 32-dim chunk of 128 rows of one plane
-  const int nchunks = p.nchunks, nstage = p.nstage;
+  const int nchunks = p.nchunks;
   const int ntiles_all = (p.nlist + 127) >> 7;
   const int qb = blockIdx.x / p.csplit, cs = blockIdx.x % p.csplit;
   const int t0 = (int)((int64_t)ntiles_all * cs / p.csplit), t1 = (int)((int64_t)ntiles_all * (cs + 1) / p.csplit);
   const int q0 = qb * 128;
   const bool qlo = p.qlo_any == nullptr || *p.qlo_any != 0;
 
-  uint8_t* Aq = sm;                                     // [2 planes][nchunks][128 rows][128 B]
-  uint8_t* Bs = Aq + 2 * nchunks * PBYTES;              // nstage x (hi chunk, lo chunk)
-  float* cns = reinterpret_cast<float*>(Bs + nstage * 2 * PBYTES);  // kQmAcc x 128 centroid norms
-  uint64_t* bars = reinterpret_cast<uint64_t*>(cns + kQmAcc * 128);
+  // layout: centroid norms, barriers, then the query planes and the centroid ring; without a lo
+  // plane (tf32-exact queries, device flag) the ring takes its room: more stages in flight
+  float* cns = reinterpret_cast<float*>(sm);  // kQmAcc x 128 centroid norms (1 KB)
+  uint64_t* bars = reinterpret_cast<uint64_t*>(sm + 1024);  // (<= 1 KB)
+  uint8_t* Aq = sm + 2048;                      // [qlo ? 2 : 1 planes][nchunks][128 rows][128 B]
+  uint8_t* Bs = Aq + (qlo ? 2 : 1) * nchunks * PBYTES;  // nstage x (hi chunk, lo chunk)
+  // (p.smem_total includes 1 KB of alignment slack for the 1 KB-aligned base)
+  const int nstage = min(kQmMaxStage, (p.smem_total - 1024 - 2048 - (qlo ? 2 : 1) * nchunks * PBYTES) / (2 * PBYTES));
   uint64_t* full_a = bars;
   uint64_t* full_b = full_a + 1;
-  uint64_t* empty_b = full_b + nstage;
-  uint64_t* tfull = empty_b + nstage;
+  uint64_t* empty_b = full_b + kQmMaxStage;
+  uint64_t* tfull = empty_b + kQmMaxStage;
   uint64_t* tempty = tfull + kQmAcc;
   uint64_t* full_c = tempty + kQmAcc;
   uint32_t* tslot = reinterpret_cast<uint32_t*>(full_c + kQmAcc);
@@ -376,17 +382,16 @@ __global__ void __launch_bounds__(kQmThreads, 1)
         if (vq && grp < (uint32_t)ngr) p.G[q * p.ldg + grp] = kmin;
       } else if (vq && grp < (uint32_t)ngr && (kmin < bk || (kmin == bk && grp <= bg))) {
         // one of the query's nprobe groups: its 32 keys (padding above the bound) to the group's slots
+        // (compacted: the passing keys first, their count in ccnt)
         const int sl = (int)__ldg(p.gslot + q * (int64_t)ngr + grp);
         uint64_t* dst = p.cand + q * (int64_t)p.ccap + sl * 32;
+        int n = 0;
 #pragma unroll
-        for (int j = 0; j < 32; j += 2) {
-          const uint32_t k0 = f2key(sc[j]), k1 = f2key(sc[j + 1]);
-          const bool p0 = c0 + j < p.nlist && (k0 < bk || (k0 == bk && grp <= bg));
-          const bool p1 = c0 + j + 1 < p.nlist && (k1 < bk || (k1 == bk && grp <= bg));
-          reinterpret_cast<ulonglong2*>(dst)[j / 2] =
-              make_ulonglong2(p0 ? (((uint64_t)k0 << 32) | (uint32_t)(c0 + j)) : MV_KEY_PAD,
-                              p1 ? (((uint64_t)k1 << 32) | (uint32_t)(c0 + j + 1)) : MV_KEY_PAD);
+        for (int j = 0; j < 32; ++j) {
+          const uint32_t kj = f2key(sc[j]);
+          if (c0 + j < p.nlist && (kj < bk || (kj == bk && grp <= bg))) dst[n++] = ((uint64_t)kj << 32) | (uint32_t)(c0 + j);
         }
+        p.ccnt[q * (int64_t)p.nprobe + sl] = (uint8_t)n;
       }
       tc_fence_before();
       __syncwarp();
@@ -481,20 +486,28 @@ __global__ void __launch_bounds__(256) k_group_bound(const uint32_t* __restrict_
 
 // per-query top-nprobe of the appended candidates (R = ceil(nprobe / 32)); see the file comment
 template <int R>
-__global__ void __launch_bounds__(256) k_probe_final(const uint64_t* __restrict__ cand, int ccap, int64_t nq, int nprobe,
-                                                     int32_t* __restrict__ probes) {
+__global__ void __launch_bounds__(256) k_probe_final(const uint64_t* __restrict__ cand, const uint8_t* __restrict__ ccnt,
+                                                     int ccap, int64_t nq, int nprobe, int32_t* __restrict__ probes) {
   __shared__ uint64_t stage_all[8][64];
   const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
   const int64_t q = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   if (q >= nq) return;
   uint64_t* stage = stage_all[wib];
   const uint64_t* c = cand + q * ccap;
-  const int n = ccap;  // 32 nprobe slots: the selected groups' keys, PAD where a centroid fails
+  const uint8_t* cn = ccnt + q * nprobe;
+  // every key of the query: lane l walks slots l, l + 32, ... (each slot's keys are compacted)
+  auto for_each_key = [&](auto&& f) {
+    for (int s0 = 0; s0 < nprobe; s0 += 32) {
+      const int sl = s0 + lane;
+      const int n = sl < nprobe ? cn[sl] : 0;
+      const int nmax = __reduce_max_sync(MV_FULL, (uint32_t)n);
+      for (int i = 0; i < nmax; ++i) f(i < n ? c[sl * 32 + i] : MV_KEY_PAD);
+    }
+  };
   uint64_t t[R];
 #pragma unroll
   for (int r = 0; r < R; ++r) t[r] = MV_KEY_PAD;
-  for (int i = lane; i < n; i += 32) {
-    const uint64_t key = c[i];
+  for_each_key([&](uint64_t key) {
     if (key < t[R - 1]) {
       t[R - 1] = key;
 #pragma unroll
@@ -505,7 +518,7 @@ __global__ void __launch_bounds__(256) k_probe_final(const uint64_t* __restrict_
           t[r - 1] = x;
         }
     }
-  }
+  });
   warp_bitonic_sort<R>(t);
   uint64_t bsel = t[0];
 #pragma unroll
@@ -531,16 +544,14 @@ __global__ void __launch_bounds__(256) k_probe_final(const uint64_t* __restrict_
     __syncwarp();
     ns = rest;
   };
-  for (int i0 = 0; i0 < n; i0 += 32) {
-    const int i = i0 + lane;
-    const uint64_t key = i < n ? c[i] : MV_KEY_PAD;
+  for_each_key([&](uint64_t key) {
     const bool ps = key != MV_KEY_PAD && key <= bound;
     const uint32_t bm = __ballot_sync(MV_FULL, ps);
     if (ps) stage[ns + __popc(bm & ((1u << lane) - 1))] = key;
     ns += __popc(bm);
     __syncwarp();
     if (ns >= 32) flush32();
-  }
+  });
   if (ns > 0) flush32();
 #pragma unroll
   for (int r = 0; r < R; ++r) {
@@ -595,9 +606,10 @@ bool coarse_tc_plan(int dpad, int nprobe, int64_t nq, int nlist, int nsm, const 
     const int64_t blocks = (nq + 127) / 128;
     p.csplit = (int)std::max<int64_t>(1, std::min<int64_t>(ntiles, (2 * nsm + blocks - 1) / blocks));
     if (o.coarse_cs > 0) p.csplit = std::max(1, std::min(ntiles, o.coarse_cs));
-    const int fixed = 2 * p.nchunks * 128 * 128 + kQmAcc * 128 * 4 + 256 + 1024;
-    p.nstage = std::min(8, (227 * 1024 - fixed) / (2 * 128 * 128));
-    p.smem_total = fixed + p.nstage * 2 * 128 * 128;
+    // shared memory: 1 KB of norms + barriers, 1 KB alignment slack, the query planes and the ring
+    // (the kernel derives the ring depth from p.smem_total and its query-plane count)
+    p.smem_total = 227 * 1024;
+    p.nstage = (p.smem_total - 3072 - 2 * p.nchunks * 128 * 128) / (2 * 128 * 128);  // (hi + lo queries)
     p.nepi = 16;
     p.nacc = kQmAcc;
     p.tmem_cols = 128 * kQmAcc;
@@ -665,17 +677,17 @@ cudaError_t launch_coarse_tc(const CUtensorMap* cmap, const CUtensorMap* qmap, c
   else if (ng <= 2048) k_group_bound<64><<<gw, 256, 0, st>>>(p.G, p.ldg, ng, nq, p.nprobe, p.gbound, p.gslot);
   else k_group_bound<0><<<gw, 256, 0, st>>>(p.G, p.ldg, ng, nq, p.nprobe, p.gbound, p.gslot);
   // fewer groups than probes: every group is selected and the slots past them stay padding
-  if (ng < p.nprobe && (e = cudaMemsetAsync(p.cand, 0xff, sizeof(uint64_t) * nq * p.ccap, st)) != cudaSuccess) return e;
+  if (ng < p.nprobe && (e = cudaMemsetAsync(p.ccnt, 0, (size_t)nq * p.nprobe, st)) != cudaSuccess) return e;
   p.mode = 1;  // pass 1: the same scores, the selected groups' keys stored to their slots
   kern<<<grid, nthr, p.smem_total, st>>>(*cmap, *qmap, p);
   if ((e = cudaGetLastError()) != cudaSuccess) return e;
   const int R = (p.nprobe + 31) / 32;
-  if (R <= 1) k_probe_final<1><<<gw, 256, 0, st>>>(p.cand, p.ccap, nq, p.nprobe, p.probes);
-  else if (R == 2) k_probe_final<2><<<gw, 256, 0, st>>>(p.cand, p.ccap, nq, p.nprobe, p.probes);
-  else if (R <= 4) k_probe_final<4><<<gw, 256, 0, st>>>(p.cand, p.ccap, nq, p.nprobe, p.probes);
-  else if (R <= 8) k_probe_final<8><<<gw, 256, 0, st>>>(p.cand, p.ccap, nq, p.nprobe, p.probes);
-  else if (R <= 16) k_probe_final<16><<<gw, 256, 0, st>>>(p.cand, p.ccap, nq, p.nprobe, p.probes);
-  else k_probe_final<32><<<gw, 256, 0, st>>>(p.cand, p.ccap, nq, p.nprobe, p.probes);
+  if (R <= 1) k_probe_final<1><<<gw, 256, 0, st>>>(p.cand, p.ccnt, p.ccap, nq, p.nprobe, p.probes);
+  else if (R == 2) k_probe_final<2><<<gw, 256, 0, st>>>(p.cand, p.ccnt, p.ccap, nq, p.nprobe, p.probes);
+  else if (R <= 4) k_probe_final<4><<<gw, 256, 0, st>>>(p.cand, p.ccnt, p.ccap, nq, p.nprobe, p.probes);
+  else if (R <= 8) k_probe_final<8><<<gw, 256, 0, st>>>(p.cand, p.ccnt, p.ccap, nq, p.nprobe, p.probes);
+  else if (R <= 16) k_probe_final<16><<<gw, 256, 0, st>>>(p.cand, p.ccnt, p.ccap, nq, p.nprobe, p.probes);
+  else k_probe_final<32><<<gw, 256, 0, st>>>(p.cand, p.ccnt, p.ccap, nq, p.nprobe, p.probes);
   return cudaGetLastError();
 }
 

@@ -242,6 +242,7 @@ static cudaError_t run_coarse(mv_index* ix, const float* qhl, const int* qlo_any
   if (e == cudaSuccess) e = s.alloc(&cp.gbound, (size_t)nq);
   if (e == cudaSuccess) e = s.alloc(&cp.cand, (size_t)nq * cp.ccap);
   if (e == cudaSuccess) e = s.alloc(&cp.gslot, (size_t)nq * ((ix->nlist + 31) / 32));
+  if (e == cudaSuccess) e = s.alloc(&cp.ccnt, (size_t)nq * npb);
   if (e != cudaSuccess) return e;
   ix->last_coarse = "tcgen05.tf32";
   return launch_coarse_tc(&ix->cmap, &qmap, cp, nq, st);

@@ -323,7 +323,8 @@ struct CoarseParams {
   int64_t ldg;
   uint64_t* gbound;        // nq: (bound score key << 32) | bound group id
   int16_t* gslot;          // nq x ceil(nlist/32): rank of the group among the query's nprobe selected, or -1
-  uint64_t* cand;          // nq x ccap: (score key << 32) | centroid id, PAD for failing centroids
+  uint64_t* cand;          // nq x ccap: per selected group 32 slots, its passing (score key << 32 | centroid) first
+  uint8_t* ccnt;           // nq x nprobe: passing keys per slot group
   int ccap;                // 32 nprobe
   const int* qlo_any;      // device: some query needs its lo plane (nullable = yes)
   int32_t* probes;
