@@ -604,7 +604,16 @@ bool coarse_tc_plan(int dpad, int nprobe, int64_t nq, int nlist, int nsm, const 
     p.nqb = 128;
     const int ntiles = (nlist + 127) / 128;
     const int64_t blocks = (nq + 127) / 128;
-    p.csplit = (int)std::max<int64_t>(1, std::min<int64_t>(ntiles, (2 * nsm + blocks - 1) / blocks));
+    // centroid splits: minimise waves x (tiles per CTA + the query block's load, ~2 tiles of time)
+    int64_t best = -1;
+    for (int cs = 1; cs <= std::min(ntiles, 64); ++cs) {
+      const int64_t waves = (blocks * cs + nsm - 1) / nsm;
+      const int64_t cost = waves * ((ntiles + cs - 1) / cs + 2);
+      if (best < 0 || cost < best) {
+        best = cost;
+        p.csplit = cs;
+      }
+    }
     if (o.coarse_cs > 0) p.csplit = std::max(1, std::min(ntiles, o.coarse_cs));
     // shared memory: 1 KB of norms + barriers, 1 KB alignment slack, the query planes and the ring
     // (the kernel derives the ring depth from p.smem_total and its query-plane count)
