@@ -96,14 +96,17 @@ def shard_ground_truth(Qg, xb_iter, k=10):
     return gd, gi
 
 
-def c5_spec(d=128):
-    """configs[4]'s generator: the SIFT-shaped mixture with the points-per-micro-centre density of
-    the c2 calibration (~15) kept at 1B rows -- 2^26 micro centres instead of 2^16."""
+C5_MICRO_LOG2 = 22
+
+
+def c5_spec(d=128, micro_log2=None):
+    """configs[4]'s generator: the SIFT-shaped mixture with 2^C5_MICRO_LOG2 micro centres at 1B rows
+    instead of c1-c4's 2^16 (reading R15)."""
     import mvgen as G
-    return G.SiftSpec(d=d, n_micro=1 << 26)
+    return G.SiftSpec(d=d, n_micro=1 << (micro_log2 or C5_MICRO_LOG2))
 
 
-def build_sharded(cfg, device, shard, nshard, Index, chunk=1 << 24, ngt=1000):
+def build_sharded(cfg, device, shard, nshard, Index, chunk=1 << 24, ngt=1000, spec=None):
     """c5: 1B-row SIFT-shaped IVF_SQ8 index, this GPU's shard (rows r with r % nshard == shard),
     generated on the device chunk by chunk (mvgen's counter hash regenerates any row anywhere) and
     added through mv_index_add.  Centroids: seeded k-means on the first 64*nlist rows; SQ8 params:
@@ -111,7 +114,7 @@ def build_sharded(cfg, device, shard, nshard, Index, chunk=1 << 24, ngt=1000):
     exact top-10 over this shard's raw rows for the first `ngt` queries (dist, ids)."""
     import mvgen as G
     from mvgen.kmeans import kmeans
-    spec = c5_spec(cfg["d"])
+    spec = spec or c5_spec(cfg["d"])
     ntr = min(cfg["n"], 64 * cfg["nlist"])
     Xtr = G.sift_base(ntr, d=cfg["d"], device=device, spec=spec)
     C = kmeans(Xtr, cfg["nlist"], iters=10)
