@@ -129,13 +129,14 @@ def build_sharded(cfg, device, shard, nshard, Index, chunk=1 << 24, ngt=1000, sp
     nloc = (cfg["n"] - shard + nshard - 1) // nshard
     Xc = torch.empty((min(chunk, nloc), cfg["d"]), dtype=torch.float32, device=device)
     gts = []
+    BUILD.update(vectors=0, seconds=0.0, calls=0)
     for s0 in range(0, nloc, chunk):
         m = min(chunk, nloc - s0)
         rows = torch.arange(s0, s0 + m, dtype=torch.int64, device=device) * nshard + shard
         for a in range(0, m, 1 << 18):
             b = min(m, a + (1 << 18))
             Xc[a:b] = spec.rows_at(rows[a:b], G.SEED_BASE)
-        ix.add(Xc[:m], rows)
+        timed_add(ix, Xc[:m], rows)
         if ngt:
             gts.append(shard_ground_truth(Q[:ngt], ((Xc[a:a + (1 << 20)][: m - a], rows[a:a + (1 << 20)])
                                                       for a in range(0, m, 1 << 20))))
@@ -145,6 +146,21 @@ def build_sharded(cfg, device, shard, nshard, Index, chunk=1 << 24, ngt=1000, sp
     del Xc
     torch.cuda.empty_cache()
     return ix, Q, C, (gts[0] if gts else None), nloc
+
+
+BUILD = {}
+
+
+def timed_add(ix, x, ids):
+    """mv_index_add with its device time recorded (build throughput; the add is
+    synchronous, so wall time around it is the build's time)."""
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    ix.add(x, ids)
+    torch.cuda.synchronize()
+    BUILD["seconds"] = BUILD.get("seconds", 0.0) + time.perf_counter() - t0
+    BUILD["vectors"] = BUILD.get("vectors", 0) + int(ids.shape[0])
+    BUILD["calls"] = BUILD.get("calls", 0) + 1
 
 
 def _merge_gt(parts, k=10):
@@ -400,7 +416,11 @@ def main():
         (sh.set_centroids if dist else ix.set_centroids)(C)
         if cfg["kind"] == "sq8":
             (sh.set_sq8 if dist else ix.set_sq8)(*sq8_params(cfg, X))
-        (sh.add if dist else ix.add)(X, ids)   # every rank keeps the rows it owns (id % world == rank)
+        BUILD.update(vectors=0, seconds=0.0, calls=0)
+        if dist:
+            sh.add(X, ids)   # every rank keeps the rows it owns (id % world == rank)
+        else:
+            timed_add(ix, X, ids)
     sh = ShardedIndex(ix) if dist else None
     torch.cuda.synchronize()
     log(f"[bench] rank {rank}: data + index build {time.perf_counter() - t0:.1f}s (ntotal {ix.ntotal})")
@@ -594,6 +614,11 @@ def main():
             "e2e": {"value": nq / (ms_e2e / 1e3), "unit": "queries/s", "h2d_bytes_per_step": nq * cfg["d"] * 4 +
                     ((nbits + 7) // 8 if bs is not None else 0), "d2h_bytes_per_step": nq * k * 12},
             "gpu_launches": launches,
+            "build": ({"vectors_per_s": BUILD["vectors"] / BUILD["seconds"], "vectors": BUILD["vectors"],
+                       "seconds": BUILD["seconds"], "add_calls": BUILD["calls"],
+                       "note": "mv_index_add (tensor-core assignment, SQ8 encode, list-major scatter, id ranks); "
+                               "each call re-lays out the whole index (O(n) copy)"}
+                      if BUILD.get("seconds") else None),
             "clocks": clocks,
             "cpu_baseline": cpu,
         }

@@ -93,7 +93,9 @@ MV_API mv_status mv_index_create(int32_t d, mv_metric metric, mv_type type, int3
  * the scratch budget.  Names: "seeding" (0/1), "need" (seeding sample, candidates), "capa" (rows
  * per list of the sample), "sq8_qc" / "flat_qc" (queries per scan work item), "coarse_nqb",
  * "coarse_cs", "coarse_epi", "coarse_nacc" (coarse GEMM shape), "large_k_select" (k > 256: 0 = the
- * staged radix select, 1 = the sample-threshold select), "workspace_bytes" (per-search
+ * staged radix select, 1 = the sample-threshold select), "big_ctas" / "big_cap" (the staged
+ * select's first launch: CTAs per SM, 1..4, and candidates staged per query; queries past it are
+ * redone with all of shared memory), "workspace_bytes" (per-search
  * scratch budget: larger batches run as several query chunks; 0 = half of the device memory that was
  * free after the last create/add).
  * value 0 = automatic.  MV_EINVAL for an unknown name or a negative value. */
@@ -187,6 +189,10 @@ MV_API mv_status mv_index_get_sq8(const mv_index* index, float* vmin, float* vdi
  * milliseconds since the last reset (ms[6]); *searches = profiled mv_search calls; *launches =
  * kernels libmv launched in them.  `reset` != 0 clears the accumulators after reading. */
 MV_API mv_status mv_profile_enable(mv_index* index, int on);
+/* Emission counters of the profiled searches (measurement, §8(d)): out[0] = queries, out[1] =
+ * candidates the seeding phase emitted, out[2] = candidates the main scan emitted (what the
+ * selects read).  Synchronises the device.  `reset` != 0 clears them. */
+MV_API mv_status mv_profile_counters(mv_index* index, int64_t* out, int reset);
 MV_API mv_status mv_profile_read(mv_index* index, double* ms, int64_t* searches, int64_t* launches, int reset);
 
 /* Human-readable index state (JSON object): d, nlist, ntotal, max list length, whether the

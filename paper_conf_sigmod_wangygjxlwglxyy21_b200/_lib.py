@@ -54,6 +54,7 @@ _SIGS = {
     "mv_profile_enable": (C.c_int, [_P, C.c_int]),
     "mv_index_describe": (C.c_int, [_P, C.c_char_p, C.c_size_t]),
     "mv_profile_read": (C.c_int, [_P, _P, _P, _P, C.c_int]),
+    "mv_profile_counters": (C.c_int, [_P, _P, C.c_int]),
     "mv_last_error": (C.c_char_p, []),
     "mv_version": (C.c_char_p, []),
 }

@@ -191,6 +191,28 @@ cudaError_t launch_rank_scatter(const uint64_t* skeys, const uint32_t* svals, in
   return cudaGetLastError();
 }
 
+// profiling counters: *out += sum of v[q * npb + j] over j < (ra ? ra[q] : npb) / += n
+__global__ void k_sum_i32(const int32_t* __restrict__ v, int64_t n, int npb, const int32_t* __restrict__ ra,
+                          unsigned long long* out) {
+  unsigned long long acc = 0;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    if (!ra || (int)(i % npb) < ra[i / npb]) acc += (unsigned)v[i];
+  for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(MV_FULL, acc, o);
+  if ((threadIdx.x & 31) == 0 && acc) atomicAdd(out, acc);
+}
+__global__ void k_count_add(int64_t n, unsigned long long* out) { *out += (unsigned long long)n; }
+
+cudaError_t launch_sum_i32(const int32_t* v, int64_t n, int npb, const int32_t* ra, unsigned long long* out,
+                           cudaStream_t st) {
+  if (n == 0) return cudaSuccess;
+  k_sum_i32<<<(int)min64(kNumSMs * 4, (n + 255) / 256), 256, 0, st>>>(v, n, npb, ra, out);
+  return cudaGetLastError();
+}
+cudaError_t launch_count_add(int64_t n, unsigned long long* out, cudaStream_t st) {
+  k_count_add<<<1, 1, 0, st>>>(n, out);
+  return cudaGetLastError();
+}
+
 // max of non-negative doubles: their IEEE bit patterns order like unsigned integers
 __global__ void k_max_f64(const double* __restrict__ v, int64_t n, unsigned long long* out) {
   unsigned long long m = 0;

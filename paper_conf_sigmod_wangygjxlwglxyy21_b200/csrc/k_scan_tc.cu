@@ -45,13 +45,22 @@ __device__ __forceinline__ void tmem_ld_w(uint32_t taddr, uint32_t (&r)[W]) {
   if constexpr (W == 16) sm100::tmem_ld16(taddr, r);
   else sm100::tmem_ld8(taddr, r);
 }
-// 16-B shared-memory load through an explicit shared address (the metadata pointers are generic)
-__device__ __forceinline__ float4 lds_f4(const float* p) {
+// shared-memory accesses through explicit 32-bit shared addresses (the metadata pointers are
+// generic: every generic access to them costs an address-window conversion)
+__device__ __forceinline__ float4 lds_f4(uint32_t a) {
   float4 v;
-  asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];"
-               : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w)
-               : "r"(sm100::smem_u32(p)));
+  asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "r"(a));
   return v;
+}
+__device__ __forceinline__ int64_t lds_s64(uint32_t a) {
+  int64_t v;
+  asm volatile("ld.shared.s64 %0, [%1];" : "=l"(v) : "r"(a));
+  return v;
+}
+__device__ __forceinline__ int atoms_add(uint32_t a, int v) {
+  int old;
+  asm volatile("atom.shared.add.u32 %0, [%1], %2;" : "=r"(old) : "r"(a), "r"(v) : "memory");
+  return old;
 }
 
 // CTA-0 event timeline (row r holds up to 1024 clock64 stamps): a development build option
@@ -141,11 +150,11 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
   extern __shared__ uint8_t smem_raw[];
   uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~(uintptr_t)1023);
   constexpr int ESZ = TYPE == MV_IVF_FLAT ? 4 : 1;
-  constexpr int PMAX = TYPE == MV_IVF_FLAT ? 2 : 4;
+  constexpr int PMAX = 2;  // FLAT: hi/lo query planes; SQ8: kSq8Planes digit planes
   const int nstage = p.nstage, nchunks = p.nchunks;
   const int QCP = (p.qchunk + 15) & ~15;       // metadata capacity (the largest chunk)
   const int QC = p.cfg[0];                      // queries per work item in this search
-  const int P = TYPE == MV_IVF_FLAT ? p.cfg[1] : 4;  // query planes: FLAT 1 (tf32-exact queries) or 2
+  const int P = TYPE == MV_IVF_FLAT ? p.cfg[1] : kSq8Planes;  // query planes: FLAT 1 (tf32-exact queries) or 2
   const int rowbytes = p.dpad * ESZ;
   const bool use_norms = p.metric == MV_L2;
   const bool use_ids = p.bitset != nullptr;
@@ -454,6 +463,8 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
       const Meta mt = meta_at(metab + b * p.meta_bytes, QCP);
       const WorkInfo wi = *mt.wi;
       const int NQ = (wi.nqc + 15) & ~15;
+      const uint32_t s_qnf = smem_u32(mt.qnf), s_thf = smem_u32(mt.thf), s_qs = smem_u32(mt.qs),
+                     s_qaf = smem_u32(mt.qaf), s_cnt = smem_u32(mt.cnt), s_base = smem_u32(mt.base);
       for (int t = 0; t < wi.ntiles; ++t, ++titer) {
         const uint32_t a = titer % NACC;
         const uint32_t ts = titer % kNTS;
@@ -484,15 +495,15 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
           // the threshold filter, branch-free.  FLAT computes the fp32 distance (exact for
           // tf32-exact data and queries); SQ8 an fp32 approximation within E_q of the exact value
           float bad[W];
-          uint32_t pm = 0, pe = 0;  // pe (FLAT): entries exactly at the bound, which need the key test
+          uint32_t pm = 0;
 #pragma unroll
           for (int v = 0; v < W / 4; ++v) {
-            const float4 qn4 = lds_f4(mt.qnf + qc + 4 * v);
-            const float4 th4 = lds_f4(mt.thf + qc + 4 * v);
+            const float4 qn4 = lds_f4(s_qnf + 4 * (qc + 4 * v));
+            const float4 th4 = lds_f4(s_thf + 4 * (qc + 4 * v));
             float4 qs4 = qn4, qa4 = qn4;
             if (TYPE == MV_IVF_SQ8) {
-              qs4 = lds_f4(mt.qs + qc + 4 * v);
-              qa4 = lds_f4(mt.qaf + qc + 4 * v);
+              qs4 = lds_f4(s_qs + 4 * (qc + 4 * v));
+              qa4 = lds_f4(s_qaf + 4 * (qc + 4 * v));
             }
             const float qnv[4] = {qn4.x, qn4.y, qn4.z, qn4.w}, thv[4] = {th4.x, th4.y, th4.z, th4.w};
             const float qsv[4] = {qs4.x, qs4.y, qs4.z, qs4.w}, qav[4] = {qa4.x, qa4.y, qa4.z, qa4.w};
@@ -506,31 +517,25 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
               } else {
                 // digit partials converted exactly (magic number: |D| < 2^22 for rows of <= 128
                 // codes), combined in fp32; the error is bounded by E_q (k_qplanes)
-                float fd[4];
+                float fd[kSq8Planes];
 #pragma unroll
-                for (int pl = 0; pl < 4; ++pl)
-                  fd[pl] = SMALLD ? __int_as_float(0x4B400000 + (int)r[pl % PMAX][j]) - 12582912.0f
-                                  : __int2float_rn((int)r[pl % PMAX][j]);
-                const float accf =
-                    fmaf(fd[3], 4.76837158203125e-7f, fmaf(fd[2], 6.103515625e-5f, fmaf(fd[1], 0.0078125f, fd[0])));
+                for (int pl = 0; pl < kSq8Planes; ++pl)
+                  fd[pl] = SMALLD ? __int_as_float(0x4B400000 + (int)r[pl][j]) - 12582912.0f
+                                  : __int2float_rn((int)r[pl][j]);
+                const float accf = fmaf(fd[1], 0.0078125f, fd[0]);  // D0 + D1 / 2^7
                 const float dotf = fmaf(qsv[u], accf, qav[u]);
                 bad[j] = use_norms ? (qnv[u] + xnf) - 2.0f * dotf : -dotf;
               }
               pm |= (bad[j] <= thv[u] ? 1u : 0u) << j;
-              if (TYPE == MV_IVF_FLAT) pe |= (bad[j] == thv[u] ? 1u : 0u) << j;
             }
           }
           if (!valid) pm = 0;
-          if (TYPE == MV_IVF_FLAT) pe &= (phaseB && !approx) ? pm : 0u;
-          // FLAT exact mode, entries exactly at the bound: the (distance key, id rank) <= tau_q test
-          if (TYPE == MV_IVF_FLAT && __any_sync(MV_FULL, pe != 0)) {
-#pragma unroll
-            for (int j = 0; j < W; ++j)
-              if (((pe >> j) & 1) && (((uint64_t)f2key(bad[j]) << 32) | rk) > mt.tau[qc + j]) pm &= ~(1u << j);
-          }
+          // (FLAT exact mode: an entry exactly at the bound's distance passes whatever its id rank
+          // -- a few extra keys at tau_q's distance, never a missing one; the final select ranks them)
           if (__any_sync(MV_FULL, pm != 0)) {
-            // ballot per column; lane j reserves column j's slots with one shared atomic (measured:
-            // a per-entry atomic path for sparse chunks was slower on configs[1] and [2])
+            // ballot per column; lane j reserves column j's slots with one shared atomic and
+            // broadcasts the column's output address (measured: a per-entry atomic path for sparse
+            // chunks was slower on configs[1] and [2])
             uint32_t mj[W];
             int mine = 0;
 #pragma unroll
@@ -538,14 +543,13 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
               mj[j] = __ballot_sync(MV_FULL, (pm >> j) & 1);
               if (lane == j) mine = __popc(mj[j]);
             }
-            int pos = 0;
-            if (mine) pos = atomicAdd(mt.cnt + qc + lane, mine);
+            int64_t cb = 0;
+            if (mine) cb = lds_s64(s_base + 8 * (qc + lane)) + atoms_add(s_cnt + 4 * (qc + lane), mine);
 #pragma unroll
             for (int j = 0; j < W; ++j) {
               if (mj[j]) {
-                const int pj = __shfl_sync(MV_FULL, pos, j);
-                if ((pm >> j) & 1)
-                  p.part[mt.base[qc + j] + pj + __popc(mj[j] & ltmask)] = ((uint64_t)f2key(bad[j]) << 32) | rk;
+                const int64_t dj = __shfl_sync(MV_FULL, cb, j);
+                if ((pm >> j) & 1) p.part[dj + __popc(mj[j] & ltmask)] = ((uint64_t)f2key(bad[j]) << 32) | rk;
               }
             }
           }
@@ -620,11 +624,11 @@ __global__ void k_qplanes(int type, const float* __restrict__ qpad, int64_t nq, 
       }
       // the scale is rounded up to fp32 first, so the digits and the epilogue use the same exact s
       const double s = amax > 0.0 ? (double)__double2float_ru(amax / 127.0) : 1.0;
-      int8_t* o = reinterpret_cast<int8_t*>(out) + q * 4 * dpad;
+      int8_t* o = reinterpret_cast<int8_t*>(out) + q * kSq8Planes * dpad;
       for (int j = lane; j < dpad; j += 32) {
         double u = (double)x[j] * ((double)vdiff[j] / 255.0) / s;  // in [-127, 127]
 #pragma unroll
-        for (int dgt = 0; dgt < 4; ++dgt) {  // base-2^7 signed digits: u ~ d0 + d1/2^7 + d2/2^14 + d3/2^21
+        for (int dgt = 0; dgt < kSq8Planes; ++dgt) {  // base-2^7 signed digits: u ~ d0 + d1/2^7
           const double dd = fmin(fmax(rint(u), -127.0), 127.0);
           o[dgt * dpad + j] = (int8_t)dd;
           u = (u - dd) * 128.0;
@@ -643,7 +647,8 @@ __global__ void k_qplanes(int type, const float* __restrict__ qpad, int64_t nq, 
         if (qerr) {
           const double amx = 127.0 * 255.0 * dpad * 1.0079;
           const double mc = 0x1p-21 * (nn + fe.xmax2 + 2.0 * (s * amx + fabs(dot)));
-          const double dd = 0x1p-22 * (s * 255.0 * dpad + qdec);
+          // (kSq8Planes digits: the last one is rounded, |residual| <= 2^-(7 kSq8Planes - 6) s per weight)
+          const double dd = ldexp(1.0, -(7 * kSq8Planes - 6)) * s * 255.0 * dpad + 0x1p-22 * qdec;
           const double E = mc + (fe.metric == MV_L2 ? 2.0 : 1.0) * dd + 0x1p-22 * (nn + fe.xmax2);
           qerr[q] = __double2float_ru(1.05 * E);
         }
@@ -687,7 +692,7 @@ static bool tc_scan_layout(int type, int dpad, int qc, int ns, TcScanParams& p) 
   p.atom = atom;
   // FLAT: qc queries of one plane (tf32-exact queries) or qc/2 queries of two (hi/lo) in the same
   // operand rows; SQ8: four digit planes
-  const int rows_per_q = type == MV_IVF_FLAT ? 1 : 4;
+  const int rows_per_q = type == MV_IVF_FLAT ? 1 : kSq8Planes;
   auto up = [](int x, int a) { return (x + a - 1) / a * a; };
   p.type = type;
   p.dpad = dpad;

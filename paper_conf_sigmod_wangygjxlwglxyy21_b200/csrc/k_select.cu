@@ -164,7 +164,7 @@ constexpr int kHistWarps = 8;  // private radix histograms (warps w, w + 8, ... 
 // strides < 32 are shuffles, strides 32 .. 16 E register pairs, larger strides go through shared
 // memory (10 of the 66 stages for NK = 2048).  Pair (lo, lo + stride) of a size-`size` stage
 // is ascending when (lo & size) == 0: the lower element keeps the minimum.
-template <int E>
+template <int E, int NT = kBigThreads>
 __device__ __forceinline__ void block_sort_regs(uint64_t* win, int NK) {
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   const int wbase = wid * 32 * E;
@@ -180,7 +180,7 @@ __device__ __forceinline__ void block_sort_regs(uint64_t* win, int NK) {
       for (int j = 0; j < E; ++j) win[wbase + 32 * j + lane] = v[j];
       for (; stride >= SMIN; stride >>= 1) {
         __syncthreads();
-        for (int t = tid; t < (NK >> 1); t += kBigThreads) {
+        for (int t = tid; t < (NK >> 1); t += NT) {
           const int lo = 2 * t - (t & (stride - 1));
           const int hi = lo + stride;
           const bool up = (lo & size) == 0;
@@ -228,16 +228,19 @@ __device__ __forceinline__ void block_sort_regs(uint64_t* win, int NK) {
 // select over the u64 keys -- 8-bit digits, histogram per pass in shared memory, stopping as soon
 // as the keys at or below the current prefix are exactly k -- and a bitonic sort of the k winners.
 
-__global__ void __launch_bounds__(kBigThreads) k_final_big(const int64_t* __restrict__ poff,
+template <int NT>
+__global__ void __launch_bounds__(NT, 2048 / NT) k_final_big(const int64_t* __restrict__ poff,
                                                            const int32_t* __restrict__ pcnt,
                                                            const uint64_t* __restrict__ part, int64_t nq, int npb, int k,
                                                            int metric, const int64_t* __restrict__ sorted_ids,
                                                            float* out_d, int64_t* out_i, int cap,
                                                            const int32_t* __restrict__ nuse, uint64_t* tau_out,
                                                            uint8_t* over, const int* __restrict__ gate,
-                                                           const uint8_t* __restrict__ only) {
+                                                           const uint8_t* only) {
   if (gate && *gate == 0) return;
-  if (only && !only[blockIdx.x]) {  // done by k_final_sample
+  // only: the queries to do (k_final_sample's redo flags, or the flags of a smaller-stage launch --
+  // then the same array as over: this CTA reads its flag before rewriting it)
+  if (only && !only[blockIdx.x]) {
     if (threadIdx.x == 0) over[blockIdx.x] = 0;
     return;
   }
@@ -277,7 +280,7 @@ __global__ void __launch_bounds__(kBigThreads) k_final_big(const int64_t* __rest
   if (tid == 0) over[q] = 0;
   // staging by fire-and-forget 8-B async copies: every lane keeps its loads in flight (a plain
   // load/store loop was latency-bound: one ~1 us global round trip per 32 keys per warp)
-  for (int j = wid; j < nu; j += kBigThreads / 32) {
+  for (int j = wid; j < nu; j += NT / 32) {
     const int c = s_pre[j + 1] - s_pre[j];
     const uint64_t* src = part + po[j];
     const uint32_t dst = (uint32_t)__cvta_generic_to_shared(buf + s_pre[j]);
@@ -288,7 +291,7 @@ __global__ void __launch_bounds__(kBigThreads) k_final_big(const int64_t* __rest
   __syncthreads();
   int nsel;  // winners to sort, in win[]
   if (T <= k) {
-    for (int i = tid; i < NK; i += kBigThreads) win[i] = i < T ? buf[i] : MV_KEY_PAD;
+    for (int i = tid; i < NK; i += NT) win[i] = i < T ? buf[i] : MV_KEY_PAD;
     nsel = T;
   } else {
     // radix select over the bits below the keys' common prefix: the first digit starts at the
@@ -297,7 +300,7 @@ __global__ void __launch_bounds__(kBigThreads) k_final_big(const int64_t* __rest
     // digits, per-warp private histograms, a warp prefix scan for the digit; it stops as soon as
     // the keys at or below the current prefix are exactly k (keys are unique).
     uint64_t mn = MV_KEY_PAD, mx = 0;
-    for (int i = tid; i < T; i += kBigThreads) {
+    for (int i = tid; i < T; i += NT) {
       const uint64_t x = buf[i];
       mn = umin64(mn, x);
       mx = umax64(mx, x);
@@ -313,7 +316,7 @@ __global__ void __launch_bounds__(kBigThreads) k_final_big(const int64_t* __rest
     }
     __syncthreads();
     if (tid == 0) {
-      for (int w = 1; w < kBigThreads / 32; ++w) {
+      for (int w = 1; w < NT / 32; ++w) {
         mn = umin64(mn, red[w]);
         mx = umax64(mx, red[32 + w]);
       }
@@ -330,10 +333,10 @@ __global__ void __launch_bounds__(kBigThreads) k_final_big(const int64_t* __rest
     for (;;) {
       const int w = min(8, lo), sh = lo - w;
       const uint32_t dmask = (1u << w) - 1;
-      for (int i = tid; i < kHistWarps * 256; i += kBigThreads) whist[i] = 0;
+      for (int i = tid; i < kHistWarps * 256; i += NT) whist[i] = 0;
       __syncthreads();
       uint32_t* hw = whist + (wid % kHistWarps) * 256;
-      for (int i = tid; i < T; i += kBigThreads) {
+      for (int i = tid; i < T; i += NT) {
         const uint64_t x = buf[i];
         if (lo >= 64 || (x >> lo) == pfx) atomicAdd(hw + ((uint32_t)(x >> sh) & dmask), 1u);
       }
@@ -374,7 +377,7 @@ __global__ void __launch_bounds__(kBigThreads) k_final_big(const int64_t* __rest
     // winners: keys whose bits above lo are <= pfx (exactly k: keys are unique)
     if (tau_out) {  // seeding: only the k-th best key is needed -- the largest winner, no gather
       uint64_t m = 0;
-      for (int i = tid; i < T; i += kBigThreads) {
+      for (int i = tid; i < T; i += NT) {
         const uint64_t x = buf[i];
         if ((lo >= 64 ? 0 : (x >> lo)) <= pfx) m = umax64(m, x);
       }
@@ -384,14 +387,14 @@ __global__ void __launch_bounds__(kBigThreads) k_final_big(const int64_t* __rest
       __syncthreads();
       if (tid == 0) {
         uint64_t mm = 0;
-        for (int w = 0; w < kBigThreads / 32; ++w) mm = umax64(mm, win[w]);
+        for (int w = 0; w < NT / 32; ++w) mm = umax64(mm, win[w]);
         tau_out[q] = mm;
       }
       return;
     }
     if (tid == 0) s_int[3] = 0;
     __syncthreads();
-    for (int b0 = 0; b0 < T; b0 += kBigThreads) {  // ballot-aggregated appends (one atomic per warp)
+    for (int b0 = 0; b0 < T; b0 += NT) {  // ballot-aggregated appends (one atomic per warp)
       const int i = b0 + tid;
       const uint64_t x = i < T ? buf[i] : MV_KEY_PAD;
       const bool p = i < T && (lo >= 64 ? 0 : (x >> lo)) <= pfx;
@@ -403,33 +406,39 @@ __global__ void __launch_bounds__(kBigThreads) k_final_big(const int64_t* __rest
     }
     __syncthreads();
     nsel = k;
-    for (int i = k + tid; i < NK; i += kBigThreads) win[i] = MV_KEY_PAD;
+    for (int i = k + tid; i < NK; i += NT) win[i] = MV_KEY_PAD;
   }
   __syncthreads();
   if (tau_out) {  // seeding with exactly k candidates: the largest
     if (nsel < k) return;
     uint64_t m = 0;
-    for (int i = tid; i < k; i += kBigThreads) m = umax64(m, win[i]);
+    for (int i = tid; i < k; i += NT) m = umax64(m, win[i]);
     for (int o = 16; o > 0; o >>= 1) m = umax64(m, shfl_xor64(m, o));
     if (lane == 0) buf[wid] = m;
     __syncthreads();
     if (tid == 0) {
       uint64_t mm = 0;
-      for (int w = 0; w < kBigThreads / 32; ++w) mm = umax64(mm, buf[w]);
+      for (int w = 0; w < NT / 32; ++w) mm = umax64(mm, buf[w]);
       tau_out[q] = mm;
     }
     return;
   }
   // bitonic sort of the NK winners: register-blocked (strides < 32 E by shuffles and in registers,
   // only the larger strides through shared memory)
-  switch (NK / kBigThreads) {
-    case 1: block_sort_regs<1>(win, NK); break;
-    case 2: block_sort_regs<2>(win, NK); break;
-    case 4: block_sort_regs<4>(win, NK); break;
-    default: block_sort_regs<0>(win, NK); break;  // NK < 1024 or > 4096: shared memory only
+  switch (NK / NT) {
+    case 1: block_sort_regs<1, NT>(win, NK); break;
+    case 2: block_sort_regs<2, NT>(win, NK); break;
+    case 4: block_sort_regs<4, NT>(win, NK); break;
+    case 8:
+      if constexpr (NT <= 512) {
+        block_sort_regs<8, NT>(win, NK);
+        break;
+      }
+      [[fallthrough]];
+    default: block_sort_regs<0, NT>(win, NK); break;  // NK < 1024 or > 4096: shared memory only
   }
   __syncthreads();
-  for (int i = tid; i < k; i += kBigThreads) {
+  for (int i = tid; i < k; i += NT) {
     float dv;
     int64_t iv;
     const uint64_t key = win[i];
@@ -671,11 +680,11 @@ __global__ void __launch_bounds__(kBigThreads) k_final_sample(const int64_t* __r
 static cudaError_t launch_big_select(const int64_t* poff, const int32_t* pcnt, const uint64_t* part, int64_t nq,
                                      int npb, int k, int metric, const int64_t* sorted_ids, float* out_d,
                                      int64_t* out_i, const int32_t* nuse, uint64_t* tau, int64_t tmax,
-                                     uint8_t* over, const int* gate, int big_mode, cudaStream_t st) {
+                                     uint8_t* over, const int* gate, BigSel bsel, cudaStream_t st) {
   cudaError_t e;
   // over: 2 nq bytes -- [0, nq) queries past k_final_big's stage, [nq, 2 nq) k_final_sample's redo flags
   uint8_t* redo = over ? over + nq : nullptr;
-  if (redo && k <= 3072 && big_mode == 1) {
+  if (redo && k <= 3072 && bsel.mode == 1) {
     const int wcap = 4 * kBigThreads;  // >= k + the threshold's slack for k <= 2048; less for larger k
     const size_t smem = (size_t)(wcap + next_pow2(max(k, 2))) * 8 + (size_t)(npb + 1) * 4 + 64;
     if ((e = cudaFuncSetAttribute(k_final_sample, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)) != cudaSuccess)
@@ -687,16 +696,42 @@ static cudaError_t launch_big_select(const int64_t* poff, const int32_t* pcnt, c
   }
   const int NK = next_pow2(max(k, 2));
   const int fixed = NK * 8 + kHistWarps * 256 * 4 + (npb + 1) * 4 + 64 + 64;
-  // stage capacity: all of shared memory, or just the bound tmax when that is smaller (several
-  // CTAs per SM: the seeding select's candidates are bounded by the phase-A prefixes)
-  const int cap = (int)min64((227 * 1024 - fixed) / 8, max64(tmax, k));
+  const int64_t want = max64(tmax, k);  // stage capacity that holds every query
+  const int capmax = (227 * 1024 - fixed) / 8;
+  // first launch: `ctas` CTAs per SM (228 KB of shared memory per SM, 1 KB reserved per CTA), each
+  // staging at most cap1 candidates; the queries past it are flagged and redone by a one-CTA-per-SM
+  // launch with all of shared memory (then by k_final_select's global-memory path)
+  const int ctas = bsel.ctas > 0 ? min(bsel.ctas, 4) : 2;
+  int cap1 = (int)min64((228 * 1024 / ctas - 2048 - fixed) / 8, want);
+  if (bsel.cap > 0) cap1 = (int)min64(cap1, max64(bsel.cap, k));
+  const uint8_t* only = redo;
+  if (over && (ctas > 1 || bsel.cap > 0) && cap1 >= k && cap1 < capmax && bsel.tlo <= cap1) {
+    const size_t smem = (size_t)cap1 * 8 + fixed;
+    if (ctas <= 2) {
+      if ((e = cudaFuncSetAttribute(k_final_big<1024>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)) !=
+          cudaSuccess)
+        return e;
+      k_final_big<1024><<<(unsigned)nq, 1024, smem, st>>>(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d,
+                                                          out_i, cap1, nuse, tau, over, gate, only);
+    } else {
+      if ((e = cudaFuncSetAttribute(k_final_big<512>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)) !=
+          cudaSuccess)
+        return e;
+      k_final_big<512><<<(unsigned)nq, 512, smem, st>>>(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d,
+                                                        out_i, cap1, nuse, tau, over, gate, only);
+    }
+    if (want <= cap1) return cudaGetLastError();
+    only = over;  // the next launch redoes the flagged queries alone
+  }
+  // all of shared memory, or just the bound tmax when that is smaller
+  const int cap = (int)min64(capmax, want);
   if (over && cap >= k) {
     const size_t smem = (size_t)cap * 8 + fixed;
-    e = cudaFuncSetAttribute(k_final_big, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    e = cudaFuncSetAttribute(k_final_big<1024>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
-    k_final_big<<<(unsigned)nq, kBigThreads, smem, st>>>(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d,
-                                                         out_i, cap, nuse, tau, over, gate, redo);
-    if (tmax <= cap) return cudaGetLastError();
+    k_final_big<1024><<<(unsigned)nq, 1024, smem, st>>>(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d,
+                                                        out_i, cap, nuse, tau, over, gate, only);
+    if (want <= cap) return cudaGetLastError();
   } else {
     over = nullptr;
   }
@@ -1185,23 +1220,23 @@ cudaError_t launch_final_refine(int type, const int64_t* poff, const int32_t* pc
 
 cudaError_t launch_final_select(const int64_t* poff, const int32_t* pcnt, const uint64_t* part, int64_t nq, int npb,
                                 int k, int metric, const int64_t* sorted_ids, float* out_d, int64_t* out_i,
-                                int64_t tmax, uint8_t* over, int big_mode, cudaStream_t st) {
+                                int64_t tmax, uint8_t* over, BigSel bsel, cudaStream_t st) {
   if (nq == 0) return cudaSuccess;
   if (launch_warp_select(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d, out_i, nullptr, nullptr, nullptr,
                          st))
     return cudaGetLastError();
   return launch_big_select(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d, out_i, nullptr, nullptr, tmax,
-                           over, nullptr, big_mode, st);
+                           over, nullptr, bsel, st);
 }
 
 cudaError_t launch_tau_select(const int64_t* poff, const int32_t* pcnt, const uint64_t* part, int64_t nq, int npb,
                               const int32_t* nuse, int k, uint64_t* tau, int64_t tmax, uint8_t* over,
-                              const int* gate, int big_mode, cudaStream_t st) {
+                              const int* gate, BigSel bsel, cudaStream_t st) {
   if (nq == 0) return cudaSuccess;
   if (launch_warp_select(poff, pcnt, part, nq, npb, k, MV_L2, nullptr, nullptr, nullptr, nuse, tau, gate, st))
     return cudaGetLastError();
   return launch_big_select(poff, pcnt, part, nq, npb, k, MV_L2, nullptr, nullptr, nullptr, nuse, tau, tmax, over, gate,
-                           big_mode, st);
+                           bsel, st);
 }
 
 // ------------------------------------------------------------------------------------------

@@ -53,6 +53,7 @@ struct mv_index {
   bool prof = false;
   std::vector<cudaEvent_t> ev;   // kProfStages + 1 events per profiled search chunk
   int64_t prof_searches = 0, launches = 0;
+  unsigned long long* d_count = nullptr;  // profiled: [queries, phase-A emissions, phase-B emissions]
 };
 
 // ------------------------------------------------------------------------------------------
@@ -334,6 +335,8 @@ mv_status mv_index_set_option(mv_index* ix, const char* name, int64_t value) {
   else if (n == "coarse_nacc") o.coarse_nacc = (int)std::min<int64_t>(value, 4);
   else if (n == "workspace_bytes") o.workspace = value;
   else if (n == "large_k_select") o.large_k_select = value != 0;
+  else if (n == "big_cap") o.big_cap = std::max<int64_t>(value, 0);
+  else if (n == "big_ctas") o.big_ctas = (int)std::min<int64_t>(std::max<int64_t>(value, 0), 4);
   else return fail(MV_EINVAL, "unknown option '%s'", name);
   return MV_OK;
 }
@@ -351,6 +354,7 @@ void mv_index_destroy(mv_index* ix) {
   mem_free(ix, ix->vmin, nullptr);
   mem_free(ix, ix->vdiff, nullptr);
   mem_free(ix, ix->sq8_t, nullptr);
+  cudaFree(ix->d_count);
   delete ix;
 }
 
@@ -711,8 +715,8 @@ static mv_status search_chunk(mv_index* ix, const float* q, int64_t nq, int32_t 
   // FLAT with tf32-exact stored values: two-plane (hi/lo) items when some query needs its lo plane;
   // other FLAT data always take one-plane items (the stored side's tf32 error dominates)
   pa.qlo_any = (flat && ix->tf32_exact) ? qlo_any : nullptr;
-  pa.qc_exact = qchunk; pa.p_exact = flat ? 1 : 4;
-  pa.qc_split = qchunk_min; pa.p_split = flat ? 2 : 4;
+  pa.qc_exact = qchunk; pa.p_exact = flat ? 1 : kSq8Planes;
+  pa.qc_split = qchunk_min; pa.p_split = flat ? 2 : kSq8Planes;
   pa.qcfg = qcfg; pa.ra = ra; pa.b = b;
   CK(launch_plan(pa, st));
   prof_mark(ix, st);
@@ -730,7 +734,7 @@ static mv_status search_chunk(mv_index* ix, const float* q, int64_t nq, int32_t 
   float *qscale, *qerr = nullptr;
   double *qa, *qn64;
   uint64_t* tau;
-  if (!flat) CK(s.alloc(&qplanes, (size_t)nq * 4 * dpad));
+  if (!flat) CK(s.alloc(&qplanes, (size_t)nq * kSq8Planes * dpad));
   else qplanes = reinterpret_cast<uint8_t*>(qhl);
   CK(s.alloc(&qscale, (size_t)nq));
   CK(s.alloc(&qa, (size_t)nq));
@@ -765,7 +769,7 @@ static mv_status search_chunk(mv_index* ix, const float* q, int64_t nq, int32_t 
     // ... tau_q = k-th best key of phase A (phase A emits < need + capA candidates per query) ...
     CK(launch_tau_select(b.poff + npairs, b.pcnt + npairs, part, nq, npb, ra, k, tau,
                          std::min<int64_t>(tmax, pa.need + pa.capA), over, nullptr,
-                         ix->opt.large_k_select, st));
+                         BigSel{ix->opt.large_k_select, ix->opt.big_ctas, ix->opt.big_cap, std::min<int64_t>(tmax, pa.need)}, st));
     prof_mark(ix, st);
     // ... phase B over every probed pair, emitting keys <= tau_q
     tp.phase = 1;
@@ -777,6 +781,15 @@ static mv_status search_chunk(mv_index* ix, const float* q, int64_t nq, int32_t 
     prof_mark(ix, st);
   }
   prof_mark(ix, st);
+  if (ix->prof) {  // emission counters (mv_profile_counters): what the selects have to read
+    if (!ix->d_count) {
+      CK(cudaMalloc(&ix->d_count, 4 * sizeof(unsigned long long)));
+      CK(cudaMemset(ix->d_count, 0, 4 * sizeof(unsigned long long)));
+    }
+    CK(launch_count_add(nq, ix->d_count, st));
+    if (split) CK(launch_sum_i32(b.pcnt + npairs, npairs, npb, ra, ix->d_count + 1, st));
+    CK(launch_sum_i32(b.pcnt, npairs, npb, nullptr, ix->d_count + 2, st));
+  }
   if (k <= 256) {
     // a7 with the filter mode's exact re-scoring fused in (a plain exact select when the search is
     // exact: FLAT with tf32-exact data and queries, gate = qlo_any == 0 on the device)
@@ -792,13 +805,13 @@ static mv_status search_chunk(mv_index* ix, const float* q, int64_t nq, int32_t 
     uint64_t* tau2;
     CK(s.alloc(&tau2, (size_t)nq));
     CK(cudaMemsetAsync(tau2, 0xff, sizeof(uint64_t) * nq, st));
-    CK(launch_tau_select(b.poff, b.pcnt, part, nq, npb, nullptr, k, tau2, tmax, over, gate, ix->opt.large_k_select,
-                         st));
+    CK(launch_tau_select(b.poff, b.pcnt, part, nq, npb, nullptr, k, tau2, tmax, over, gate,
+                         BigSel{ix->opt.large_k_select, ix->opt.big_ctas, ix->opt.big_cap, 0}, st));
     CK(launch_rekey(ix->type, b.poff, b.pcnt, part, nq, npb, tau2, qerr, ix->metric, qpad, dpad, ix->payload,
                     ix->row_of_rank, ix->vmin, ix->vdiff, ix->sq8_t, gate, st));
     ix->launches += 2;
     CK(launch_final_select(b.poff, b.pcnt, part, nq, npb, k, ix->metric, ix->sorted_ids, D, I, tmax, over,
-                           ix->opt.large_k_select, st));
+                           BigSel{ix->opt.large_k_select, ix->opt.big_ctas, ix->opt.big_cap, 0}, st));
   }
   prof_mark(ix, st);
   ix->last_scan = flat ? "tcgen05.tf32" : "tcgen05.i8";
@@ -973,6 +986,19 @@ mv_status mv_profile_read(mv_index* ix, double* ms, int64_t* searches, int64_t* 
     ix->prof_searches = 0;
     ix->launches = 0;
   }
+  return MV_OK;
+}
+
+mv_status mv_profile_counters(mv_index* ix, int64_t* out, int reset) {
+  if (!ix || !out) return fail(MV_EINVAL, "null argument");
+  DeviceGuard g(ix->device);
+  unsigned long long h[4] = {0, 0, 0, 0};
+  if (ix->d_count) {
+    CK(cudaDeviceSynchronize());
+    CK(cudaMemcpy(h, ix->d_count, sizeof h, cudaMemcpyDeviceToHost));
+    if (reset) CK(cudaMemset(ix->d_count, 0, sizeof h));
+  }
+  for (int i = 0; i < 3; ++i) out[i] = (int64_t)h[i];
   return MV_OK;
 }
 

@@ -18,6 +18,10 @@ constexpr int kMaxK = 16384;          // PAPER.md:801-802 (§3.3 fn. 5): k <= 16
 constexpr int kMaxD = 512;            // the tensor-core kernels stage query operands of <= 512 dims
 constexpr int kMaxNprobe = 1024;      // ranked probes per query (k_probe_select's register list)
 constexpr int kNumSMs = 148;
+// SQ8 query-side digit planes (kind::i8, base 2^7): the scan is a filter whose error bound E_q
+// includes the last digit's residual; the band is re-scored exactly, so two planes
+// suffice (round 1 used four for an exact in-scan fp64 value)
+constexpr int kSq8Planes = 2;
 constexpr int kProfStages = 6;   // coarse, bucket, scan A, seed select, scan B, final select (mv.h)
 
 __host__ __device__ __forceinline__ int64_t min64(int64_t a, int64_t b) { return a < b ? a : b; }
@@ -178,6 +182,17 @@ struct Options {
   int coarse_nqb = 0, coarse_cs = 0, coarse_epi = 0, coarse_nacc = 0;  // coarse GEMM launch shape
   int64_t workspace = 0;    // per-search scratch budget in bytes (0: half of the free device memory)
   int large_k_select = 0;   // k > 256: 0 staged radix select, 1 sample-threshold select (radix fallback)
+  int big_ctas = 0;         // k > 256 staged select: CTAs per SM of its first launch (1..4; 0 = 2)
+  int64_t big_cap = 0;      // ... and its stage capacity in keys (0: the most that fits big_ctas per SM)
+};
+
+// k > 256 select launch choices: Options::large_k_select / big_ctas, and a lower bound on the
+// candidates per query when the caller knows one (the seeding sample: >= need)
+struct BigSel {
+  int mode = 0;
+  int ctas = 0;
+  int64_t cap = 0;
+  int64_t tlo = 0;
 };
 }  // namespace mv
 
@@ -202,6 +217,10 @@ cudaError_t launch_move_old(int type, int dpad, int nlist, const int64_t* old_of
 cudaError_t launch_id_keys(const int64_t* ids, int64_t n, uint64_t* keys, uint32_t* vals, cudaStream_t st);
 cudaError_t launch_rank_scatter(const uint64_t* skeys, const uint32_t* svals, int64_t n, uint32_t* rank,
                                 int64_t* sorted_ids, uint32_t* row_of_rank, cudaStream_t st);
+// profiling counters: *out += sum of v[0..n) / += n
+cudaError_t launch_sum_i32(const int32_t* v, int64_t n, int npb, const int32_t* ra, unsigned long long* out,
+                           cudaStream_t st);
+cudaError_t launch_count_add(int64_t n, unsigned long long* out, cudaStream_t st);
 // *out = max(*out, max_i v[i]) for non-negative doubles (atomicMax on the bit patterns)
 cudaError_t launch_max_f64(const double* v, int64_t n, unsigned long long* out, cudaStream_t st);
 cudaError_t launch_check_ids(const int64_t* ids, int64_t n, int* flag, cudaStream_t st);
@@ -343,10 +362,10 @@ cudaError_t launch_hilo(const float* x, int64_t n, int d, int dpad, float* out, 
 // the staged radix select as its fallback.  over: 2 nq bytes of scratch for k > 256.
 cudaError_t launch_final_select(const int64_t* poff, const int32_t* pcnt, const uint64_t* part, int64_t nq, int npb,
                                 int k, int metric, const int64_t* sorted_ids, float* out_d, int64_t* out_i,
-                                int64_t tmax, uint8_t* over, int big_mode, cudaStream_t st);
+                                int64_t tmax, uint8_t* over, BigSel bsel, cudaStream_t st);
 cudaError_t launch_tau_select(const int64_t* poff, const int32_t* pcnt, const uint64_t* part, int64_t nq, int npb,
                               const int32_t* nuse, int k, uint64_t* tau, int64_t tmax, uint8_t* over,
-                              const int* gate, int big_mode, cudaStream_t st);
+                              const int* gate, BigSel bsel, cudaStream_t st);
 // k <= 256: the final select with the filter mode's fused exact re-scoring (k_final_warp<R, type>);
 // rgate (nullable = always): refine only when *rgate != 0, else the plain exact select
 cudaError_t launch_final_refine(int type, const int64_t* poff, const int32_t* pcnt, const uint64_t* part, int64_t nq,

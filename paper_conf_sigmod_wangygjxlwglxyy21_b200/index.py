@@ -221,6 +221,12 @@ class Index:
         L.check(self._lib.mv_profile_read(self._h, ms, C.byref(ns), C.byref(nl), int(reset)))
         return dict(zip(self.STAGES, list(ms))), int(ns.value), int(nl.value)
 
+    def profile_counters(self, reset: bool = True) -> dict:
+        """Emission counters of the profiled searches: queries, seeding-phase and main-scan emissions."""
+        out = (C.c_int64 * 3)()
+        L.check(self._lib.mv_profile_counters(self._h, out, int(reset)))
+        return {"queries": int(out[0]), "phase_a_emitted": int(out[1]), "phase_b_emitted": int(out[2])}
+
     def describe(self) -> dict:
         import json
         buf = C.create_string_buffer(2048)

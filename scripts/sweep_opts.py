@@ -41,7 +41,7 @@ def main():
     nprobe = a.nprobe or cfg["nprobe"]
     nbits = n if bs is not None else 0
     names = ["seeding", "need", "capa", "sq8_qc", "flat_qc", "coarse_nqb", "coarse_cs", "coarse_epi", "coarse_nacc",
-             "large_k_select"]
+             "large_k_select", "big_ctas", "big_cap"]
     for st in a.sets:
         for nm in names:
             ix.set_option(nm, 1 if nm == "seeding" else 0)
@@ -61,9 +61,12 @@ def main():
         torch.cuda.synchronize()
         ix.profile(False)
         stg, ns, _ = ix.profile_read(reset=True)
+        cnt = ix.profile_counters(reset=True)
+        qn = max(cnt["queries"], 1)
         ms = e0.elapsed_time(e1) / a.steps
         print(f"{a.config} [{st or 'default'}] {ms:.3f} ms/search {cfg['nq'] / ms * 1e3 / 1e6:.3f} Mqps | "
-              + " ".join(f"{k} {v / max(ns, 1):.3f}" for k, v in stg.items()), flush=True)
+              + " ".join(f"{k} {v / max(ns, 1):.3f}" for k, v in stg.items())
+              + f" | emitted/query A {cnt['phase_a_emitted'] / qn:.0f} B {cnt['phase_b_emitted'] / qn:.0f}", flush=True)
 
 
 if __name__ == "__main__":
