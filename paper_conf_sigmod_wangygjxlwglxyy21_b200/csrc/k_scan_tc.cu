@@ -59,8 +59,17 @@ __device__ __forceinline__ int64_t lds_s64(uint32_t a) {
 }
 __device__ __forceinline__ int atoms_add(uint32_t a, int v) {
   int old;
-  asm volatile("atom.shared.add.u32 %0, [%1], %2;" : "=r"(old) : "r"(a), "r"(v) : "memory");
+  asm volatile("atom.shared.add.u32 %0, [%1], %2;" : "=r"(old) : "r"(a), "r"(v));
   return old;
+}
+// predicated 8-B global store (no divergent branch around the emission)
+__device__ __forceinline__ void st_u64_if(uint32_t pred, uint64_t* a, uint64_t v) {
+  asm volatile("{\n .reg .pred q;\n setp.ne.u32 q, %0, 0;\n @q st.global.u64 [%1], %2;\n}" ::"r"(pred), "l"(a), "l"(v));
+}
+// f2key (mv_internal.cuh) in two integer ops
+__device__ __forceinline__ uint32_t f2key_fast(float f) {
+  const uint32_t b = __float_as_uint(__fadd_rn(f, 0.0f));
+  return b ^ ((uint32_t)((int32_t)b >> 31) | 0x80000000u);
 }
 
 // CTA-0 event timeline (row r holds up to 1024 clock64 stamps): a development build option
@@ -484,14 +493,13 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
         const uint32_t tbase = tmem + a * p.ncol + ((uint32_t)(quarter * 32) << 16);
         for (int qc = half * W; qc < NQ; qc += NPART * W) {
           uint32_t r[PMAX][W];
-#pragma unroll
-          for (int pl = 0; pl < PMAX; ++pl) {
-            if (pl < P) tmem_ld_w<W>(tbase + pl * NQ + qc, r[pl]);
-            else
-#pragma unroll
-              for (int j = 0; j < W; ++j) r[pl][j] = 0u;
-          }
+          tmem_ld_w<W>(tbase + qc, r[0]);
+          if (TYPE == MV_IVF_SQ8 || P == 2) tmem_ld_w<W>(tbase + NQ + qc, r[1]);
           tmem_wait_ld();
+          if (TYPE == MV_IVF_FLAT && P == 2) {  // hi + lo query planes
+#pragma unroll
+            for (int j = 0; j < W; ++j) r[0][j] = __float_as_uint(__uint_as_float(r[0][j]) + __uint_as_float(r[1][j]));
+          }
           // the threshold filter, branch-free.  FLAT computes the fp32 distance (exact for
           // tf32-exact data and queries); SQ8 an fp32 approximation within E_q of the exact value
           float bad[W];
@@ -511,9 +519,10 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
             for (int u = 0; u < 4; ++u) {
               const int j = 4 * v + u;
               if (TYPE == MV_IVF_FLAT) {
-                // badness = L2 distance or -IP; exact for tf32-representable data
-                const float dot = __uint_as_float(r[0][j]) + __uint_as_float(r[1 % PMAX][j]);
-                bad[j] = use_norms ? (qnv[u] + xnf) - 2.0f * dot : -dot;
+                // badness = L2 distance or -IP; exact for tf32-representable data (2 dot is exact,
+                // so the fma rounds exactly like (|q|^2 + |x|^2) - 2 dot)
+                const float dot = __uint_as_float(r[0][j]);
+                bad[j] = use_norms ? fmaf(-2.0f, dot, qnv[u] + xnf) : -dot;
               } else {
                 // digit partials converted exactly (magic number: |D| < 2^22 for rows of <= 128
                 // codes), combined in fp32; the error is bounded by E_q (k_qplanes)
@@ -524,7 +533,7 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
                                   : __int2float_rn((int)r[pl][j]);
                 const float accf = fmaf(fd[1], 0.0078125f, fd[0]);  // D0 + D1 / 2^7
                 const float dotf = fmaf(qsv[u], accf, qav[u]);
-                bad[j] = use_norms ? (qnv[u] + xnf) - 2.0f * dotf : -dotf;
+                bad[j] = use_norms ? fmaf(-2.0f, dotf, qnv[u] + xnf) : -dotf;
               }
               pm |= (bad[j] <= thv[u] ? 1u : 0u) << j;
             }
@@ -543,13 +552,15 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
               mj[j] = __ballot_sync(MV_FULL, (pm >> j) & 1);
               if (lane == j) mine = __popc(mj[j]);
             }
-            int64_t cb = 0;
-            if (mine) cb = lds_s64(s_base + 8 * (qc + lane)) + atoms_add(s_cnt + 4 * (qc + lane), mine);
+            uint64_t cp = 0;  // lane j: the address of column j's first reserved slot
+            if (mine)
+              cp = reinterpret_cast<uint64_t>(p.part + lds_s64(s_base + 8 * (qc + lane)) +
+                                              atoms_add(s_cnt + 4 * (qc + lane), mine));
 #pragma unroll
             for (int j = 0; j < W; ++j) {
-              if (mj[j]) {
-                const int64_t dj = __shfl_sync(MV_FULL, cb, j);
-                if ((pm >> j) & 1) p.part[dj + __popc(mj[j] & ltmask)] = ((uint64_t)f2key(bad[j]) << 32) | rk;
+              if (mj[j]) {  // warp-uniform
+                uint64_t* dst = reinterpret_cast<uint64_t*>(__shfl_sync(MV_FULL, cp, j)) + __popc(mj[j] & ltmask);
+                st_u64_if((pm >> j) & 1, dst, ((uint64_t)f2key_fast(bad[j]) << 32) | rk);
               }
             }
           }
