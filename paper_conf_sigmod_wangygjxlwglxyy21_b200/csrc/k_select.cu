@@ -248,9 +248,10 @@ __global__ void __launch_bounds__(NT, 2048 / NT) k_final_big(const int64_t* __re
   const int NK = next_pow2(max(k, 2));
   uint64_t* buf = reinterpret_cast<uint64_t*>(smem);   // cap
   uint64_t* win = buf + cap;                           // NK
-  uint32_t* whist = reinterpret_cast<uint32_t*>(win + NK);  // kHistWarps x 256 (>= 66 u64 for the min/max)
-  int32_t* s_pre = reinterpret_cast<int32_t*>(whist + kHistWarps * 256);  // npb + 1
-  int32_t* s_int = s_pre + npb + 1;                    // misc
+  uint32_t* whist = reinterpret_cast<uint32_t*>(win + NK);  // kHistWarps x 256
+  uint64_t* s_mm = reinterpret_cast<uint64_t*>(whist + kHistWarps * 256);  // min, max
+  int32_t* s_pre = reinterpret_cast<int32_t*>(s_mm + 2);  // npb + 1
+  int32_t* s_int = s_pre + npb + 1;                    // misc: [0..3) digit, [8..16) warp totals
   const int64_t q = blockIdx.x;
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   const int64_t* po = poff + q * npb;
@@ -270,6 +271,11 @@ __global__ void __launch_bounds__(NT, 2048 / NT) k_final_big(const int64_t* __re
       run += __shfl_sync(MV_FULL, incl, 31);
     }
     if (lane == 0) s_pre[nu] = run;
+  }
+  for (int i = tid; i < kHistWarps * 256; i += NT) whist[i] = 0;
+  if (tid == 0) {
+    s_mm[0] = MV_KEY_PAD;
+    s_mm[1] = 0;
   }
   __syncthreads();
   const int T = s_pre[nu];
@@ -297,8 +303,10 @@ __global__ void __launch_bounds__(NT, 2048 / NT) k_final_big(const int64_t* __re
     // radix select over the bits below the keys' common prefix: the first digit starts at the
     // highest bit where the smallest and largest key differ (near-neighbour distance keys share
     // their top ~10 bits, which a fixed MSB digit would pile into one contended bin).  8-bit
-    // digits, per-warp private histograms, a warp prefix scan for the digit; it stops as soon as
-    // the keys at or below the current prefix are exactly k (keys are unique).
+    // digits, private histograms (warps w, w + 8, ... share one), a block-wide scan of the 256
+    // bins; it stops as soon as the keys at or below the current prefix are exactly k (keys are
+    // unique) -- or, for the seeding bound, at most k + k/64: any bound with >= k candidates at
+    // or below it is valid, a looser one only lets phase B emit a few more keys
     uint64_t mn = MV_KEY_PAD, mx = 0;
     for (int i = tid; i < T; i += NT) {
       const uint64_t x = buf[i];
@@ -309,61 +317,50 @@ __global__ void __launch_bounds__(NT, 2048 / NT) k_final_big(const int64_t* __re
       mn = umin64(mn, shfl_xor64(mn, o));
       mx = umax64(mx, shfl_xor64(mx, o));
     }
-    uint64_t* red = reinterpret_cast<uint64_t*>(whist);
     if (lane == 0) {
-      red[wid] = mn;
-      red[32 + wid] = mx;
+      atomicMin(reinterpret_cast<unsigned long long*>(s_mm), (unsigned long long)mn);
+      atomicMax(reinterpret_cast<unsigned long long*>(s_mm + 1), (unsigned long long)mx);
     }
     __syncthreads();
-    if (tid == 0) {
-      for (int w = 1; w < NT / 32; ++w) {
-        mn = umin64(mn, red[w]);
-        mx = umax64(mx, red[32 + w]);
-      }
-      red[64] = mn;
-      red[65] = mx;
-    }
-    __syncthreads();
-    mn = red[64];
-    mx = red[65];
-    __syncthreads();
+    mn = s_mm[0];
+    mx = s_mm[1];
     int lo = 64 - __clzll((long long)(mn ^ mx));  // bits [lo, 64) are common to every key
     uint64_t pfx = lo >= 64 ? 0 : (mn >> lo);
     int below = 0;  // keys whose bits above lo are < pfx
+    const uint32_t slack = tau_out ? (uint32_t)(k >> 6) : 0u;
     for (;;) {
       const int w = min(8, lo), sh = lo - w;
       const uint32_t dmask = (1u << w) - 1;
-      for (int i = tid; i < kHistWarps * 256; i += NT) whist[i] = 0;
-      __syncthreads();
       uint32_t* hw = whist + (wid % kHistWarps) * 256;
       for (int i = tid; i < T; i += NT) {
         const uint64_t x = buf[i];
         if (lo >= 64 || (x >> lo) == pfx) atomicAdd(hw + ((uint32_t)(x >> sh) & dmask), 1u);
       }
       __syncthreads();
-      if (wid == 0) {  // bins 8 * lane .. 8 * lane + 7, summed over the private histograms
-        uint32_t c[8];
-        uint32_t tot = 0;
+      // bin tid (< 256): its count over the private histograms (cleared for the next pass), a
+      // warp scan, the warp totals, and the bin holding the k-th key
+      uint32_t v = 0, incl = 0;
+      if (tid < 256) {
 #pragma unroll
-        for (int j = 0; j < 8; ++j) {
-          uint32_t v = 0;
-          for (int h = 0; h < kHistWarps; ++h) v += whist[h * 256 + 8 * lane + j];
-          c[j] = v;
-          tot += v;
+        for (int h = 0; h < kHistWarps; ++h) {
+          v += whist[h * 256 + tid];
+          whist[h * 256 + tid] = 0;
         }
-        uint32_t incl = tot;
+        incl = v;
         for (int o = 1; o < 32; o <<= 1) {
-          const uint32_t v = __shfl_up_sync(MV_FULL, incl, o);
-          if (lane >= o) incl += v;
+          const uint32_t u = __shfl_up_sync(MV_FULL, incl, o);
+          if (lane >= o) incl += u;
         }
-        uint32_t cum = below + incl - tot;  // keys before this lane's first bin
-        const bool mine = cum < (uint32_t)k && cum + tot >= (uint32_t)k;
-        if (mine) {
-          int d = 0;
-          while (cum + c[d] < (uint32_t)k) cum += c[d++];
-          s_int[0] = 8 * lane + d;
+        if (lane == 31) s_int[8 + wid] = (int)incl;
+      }
+      __syncthreads();
+      if (tid < 256) {
+        uint32_t cum = (uint32_t)below + incl - v;  // keys before bin tid
+        for (int w2 = 0; w2 < wid; ++w2) cum += (uint32_t)s_int[8 + w2];
+        if (cum < (uint32_t)k && cum + v >= (uint32_t)k) {
+          s_int[0] = tid;
           s_int[1] = (int)cum;
-          s_int[2] = cum + c[d] == (uint32_t)k;
+          s_int[2] = cum + v - (uint32_t)k <= slack;
         }
       }
       __syncthreads();
@@ -374,22 +371,10 @@ __global__ void __launch_bounds__(NT, 2048 / NT) k_final_big(const int64_t* __re
       __syncthreads();
       if (done) break;
     }
-    // winners: keys whose bits above lo are <= pfx (exactly k: keys are unique)
-    if (tau_out) {  // seeding: only the k-th best key is needed -- the largest winner, no gather
-      uint64_t m = 0;
-      for (int i = tid; i < T; i += NT) {
-        const uint64_t x = buf[i];
-        if ((lo >= 64 ? 0 : (x >> lo)) <= pfx) m = umax64(m, x);
-      }
-      for (int o = 16; o > 0; o >>= 1) m = umax64(m, shfl_xor64(m, o));
-      __syncthreads();
-      if (lane == 0) win[wid] = m;
-      __syncthreads();
-      if (tid == 0) {
-        uint64_t mm = 0;
-        for (int w = 0; w < NT / 32; ++w) mm = umax64(mm, win[w]);
-        tau_out[q] = mm;
-      }
+    // winners: keys whose bits above lo are <= pfx (exactly k, or k..k+slack for the seeding bound)
+    if (tau_out) {  // seeding: the bound is the winners' upper edge -- no key of the sample lies
+                    // between it and the largest winner; no gather, no sort
+      if (tid == 0) tau_out[q] = (pfx << lo) | (lo ? (~0ull >> (64 - lo)) : 0ull);
       return;
     }
     if (tid == 0) s_int[3] = 0;
@@ -402,7 +387,11 @@ __global__ void __launch_bounds__(NT, 2048 / NT) k_final_big(const int64_t* __re
       int base = 0;
       if (lane == 0 && m) base = atomicAdd(s_int + 3, __popc(m));
       base = __shfl_sync(MV_FULL, base, 0);
-      if (p) win[base + __popc(m & ((1u << lane) - 1))] = x;
+      if (p) {
+        win[base + __popc(m & ((1u << lane) - 1))] = x;
+        // the output's id gather reads sorted_ids[rank] after the sort: start it now
+        if (sorted_ids) asm volatile("prefetch.global.L2 [%0];" ::"l"(sorted_ids + (uint32_t)(x & 0xffffffffu)));
+      }
     }
     __syncthreads();
     nsel = k;
@@ -695,7 +684,7 @@ static cudaError_t launch_big_select(const int64_t* poff, const int32_t* pcnt, c
     redo = nullptr;
   }
   const int NK = next_pow2(max(k, 2));
-  const int fixed = NK * 8 + kHistWarps * 256 * 4 + (npb + 1) * 4 + 64 + 64;
+  const int fixed = NK * 8 + kHistWarps * 256 * 4 + 16 + (npb + 1) * 4 + 64 + 64;
   const int64_t want = max64(tmax, k);  // stage capacity that holds every query
   const int capmax = (227 * 1024 - fixed) / 8;
   // first launch: `ctas` CTAs per SM (228 KB of shared memory per SM, 1 KB reserved per CTA), each
