@@ -223,6 +223,80 @@ __device__ __forceinline__ void block_sort_regs(uint64_t* win, int NK) {
   for (int j = 0; j < E; ++j) win[wbase + 32 * j + lane] = v[j];
 }
 
+// Bucket sort of n unique keys win[0..n), all in [mn, hi], by one NT-thread block: 2048 buckets
+// of equal key width, a counting pass, a scan, a scatter into tmp, and each key's rank within its
+// bucket (keys are unique: rank = the bucket's keys below it).  cnt: 2048 zeroed u32; misc: 33
+// ints.  ~6 barriers and a few dozen instructions per key against a bitonic network's ~60
+// compare-exchange stages; false (win untouched) when a bucket holds more than kBucketMax keys
+// (piles of keys within a narrow key range), for the caller's bitonic sort.
+constexpr int kBucketBins = 2048, kBucketMax = 64;
+static_assert(kBucketBins == kHistWarps * 256, "the bucket sort reuses the radix histograms");
+template <int NT>
+__device__ bool block_bucket_sort(uint64_t* win, int n, uint64_t mn, uint64_t hi, uint32_t* cnt, uint64_t* tmp,
+                                  int* misc) {
+  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  const uint64_t range = hi - mn;
+  const int sh = max(0, 64 - __clzll((long long)range) - 11);  // (x - mn) >> sh < 2048
+  if (tid == 0) misc[32] = 0;
+  __syncthreads();
+  int mx = 0;
+  for (int i = tid; i < n; i += NT) mx = max(mx, (int)atomicAdd(cnt + ((win[i] - mn) >> sh), 1u) + 1);
+  mx = __reduce_max_sync(MV_FULL, mx);
+  if (lane == 0) atomicMax(misc + 32, mx);
+  __syncthreads();
+  if (misc[32] > kBucketMax) {
+    for (int i = tid; i < kBucketBins; i += NT) cnt[i] = 0;
+    __syncthreads();
+    return false;
+  }
+  constexpr int PER = kBucketBins / NT;
+  uint32_t v[PER], sum = 0;
+#pragma unroll
+  for (int j = 0; j < PER; ++j) {
+    v[j] = cnt[tid * PER + j];
+    sum += v[j];
+  }
+  uint32_t incl = sum;
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t u = __shfl_up_sync(MV_FULL, incl, o);
+    if (lane >= o) incl += u;
+  }
+  if (lane == 31) misc[wid] = (int)incl;
+  __syncthreads();
+  if (wid == 0) {
+    uint32_t t = lane < NT / 32 ? (uint32_t)misc[lane] : 0u;
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t u = __shfl_up_sync(MV_FULL, t, o);
+      if (lane >= o) t += u;
+    }
+    __syncwarp();
+    misc[lane] = (int)t;
+  }
+  __syncthreads();
+  uint32_t run = (wid ? (uint32_t)misc[wid - 1] : 0u) + incl - sum;
+#pragma unroll
+  for (int j = 0; j < PER; ++j) {
+    cnt[tid * PER + j] = run;  // bucket start; the scatter's atomics turn it into the bucket end
+    run += v[j];
+  }
+  __syncthreads();
+  for (int i = tid; i < n; i += NT) {
+    const uint64_t x = win[i];
+    tmp[atomicAdd(cnt + ((x - mn) >> sh), 1u)] = x;
+  }
+  __syncthreads();
+  for (int i = tid; i < n; i += NT) {
+    const uint64_t x = tmp[i];
+    const int b = (int)((x - mn) >> sh);
+    const int s0 = b ? (int)cnt[b - 1] : 0, e0 = (int)cnt[b];
+    int r = 0;
+    for (int j = s0; j < e0; ++j) r += tmp[j] < x ? 1 : 0;
+    win[s0 + r] = x;
+  }
+  __syncthreads();
+  return true;
+}
+
 // 256 < k: one CTA (kBigThreads threads) per query stages the query's candidates in shared memory (when
 // they fit, else it flags the query for k_final_select's global-memory path), then an MSB radix
 // select over the u64 keys -- 8-bit digits, histogram per pass in shared memory, stopping as soon
@@ -251,7 +325,7 @@ __global__ void __launch_bounds__(NT, 2048 / NT) k_final_big(const int64_t* __re
   uint32_t* whist = reinterpret_cast<uint32_t*>(win + NK);  // kHistWarps x 256
   uint64_t* s_mm = reinterpret_cast<uint64_t*>(whist + kHistWarps * 256);  // min, max
   int32_t* s_pre = reinterpret_cast<int32_t*>(s_mm + 2);  // npb + 1
-  int32_t* s_int = s_pre + npb + 1;                    // misc: [0..3) digit, [8..16) warp totals
+  int32_t* s_int = s_pre + npb + 1;                    // misc: [0..3) digit, [8..16) warp totals, [16..49) sort
   const int64_t q = blockIdx.x;
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   const int64_t* po = poff + q * npb;
@@ -295,7 +369,8 @@ __global__ void __launch_bounds__(NT, 2048 / NT) k_final_big(const int64_t* __re
   }
   asm volatile("cp.async.wait_all;" ::: "memory");
   __syncthreads();
-  int nsel;  // winners to sort, in win[]
+  int nsel;              // winners to sort, in win[]
+  bool sorted = false;   // ... already sorted (the bucket sort)
   if (T <= k) {
     for (int i = tid; i < NK; i += NT) win[i] = i < T ? buf[i] : MV_KEY_PAD;
     nsel = T;
@@ -396,6 +471,9 @@ __global__ void __launch_bounds__(NT, 2048 / NT) k_final_big(const int64_t* __re
     __syncthreads();
     nsel = k;
     for (int i = k + tid; i < NK; i += NT) win[i] = MV_KEY_PAD;
+    // the k winners lie in [mn, the prefix's upper edge]
+    sorted = block_bucket_sort<NT>(win, k, mn, (pfx << lo) | (lo ? (~0ull >> (64 - lo)) : 0ull), whist, buf,
+                                   s_int + 16);
   }
   __syncthreads();
   if (tau_out) {  // seeding with exactly k candidates: the largest
@@ -412,9 +490,9 @@ __global__ void __launch_bounds__(NT, 2048 / NT) k_final_big(const int64_t* __re
     }
     return;
   }
-  // bitonic sort of the NK winners: register-blocked (strides < 32 E by shuffles and in registers,
-  // only the larger strides through shared memory)
-  switch (NK / NT) {
+  // else a bitonic sort of the NK winners: register-blocked (strides < 32 E by shuffles and in
+  // registers, only the larger strides through shared memory)
+  if (!sorted) switch (NK / NT) {
     case 1: block_sort_regs<1, NT>(win, NK); break;
     case 2: block_sort_regs<2, NT>(win, NK); break;
     case 4: block_sort_regs<4, NT>(win, NK); break;
@@ -684,7 +762,7 @@ static cudaError_t launch_big_select(const int64_t* poff, const int32_t* pcnt, c
     redo = nullptr;
   }
   const int NK = next_pow2(max(k, 2));
-  const int fixed = NK * 8 + kHistWarps * 256 * 4 + 16 + (npb + 1) * 4 + 64 + 64;
+  const int fixed = NK * 8 + kHistWarps * 256 * 4 + 16 + (npb + 1) * 4 + 64 * 4 + 64;
   const int64_t want = max64(tmax, k);  // stage capacity that holds every query
   const int capmax = (227 * 1024 - fixed) / 8;
   // first launch: `ctas` CTAs per SM (228 KB of shared memory per SM, 1 KB reserved per CTA), each

@@ -212,6 +212,29 @@ def test_large_k(k):
     assert frac == 1.0
 
 
+def test_large_k_bucket_piles():
+    """k = 1000 where 3000 candidates share one distance and ten lie much closer: the winners pile
+    into one bucket of k_final_big's bucket sort, which then falls back to the bitonic sort; both
+    orders are the oracle's (distance, id) order (§3.3)."""
+    d, n = 16, 4000
+    r = np.random.default_rng(11)
+    X = np.full((n, d), 100.0, np.float32)
+    X[:3000] = 5.0                                         # 3000 rows at one distance from q = 0
+    X[3000:3010] = r.integers(0, 3, (10, d)).astype(np.float32)  # ten much closer
+    Q = np.zeros((3, d), np.float32)
+    Q[1, 0] = 1.0
+    Q[2] = 60.0                                            # the far rows are its nearest
+    ids = G.permuted_ids(n, seed=3)
+    Xt, Qt = torch.from_numpy(X), torch.from_numpy(Q)
+    C = torch.from_numpy(X[:1].copy())
+    ix = _build(Xt, ids, C, "l2", "flat")
+    for k in (1000, 300):
+        D, I = ix.search(Qt.cuda(), k, 1)
+        De, Ie = O.exact_knn(X, ids.numpy(), Q, k, O.L2)
+        assert np.array_equal(I.cpu().numpy(), Ie), k
+        np.testing.assert_array_equal(D.cpu().numpy(), De.astype(np.float32))
+
+
 def test_large_k_rounds_crosscheck():
     """The paper's rounds-of-1024 procedure on the oracle candidates gives the GPU answer."""
     n = 6000
