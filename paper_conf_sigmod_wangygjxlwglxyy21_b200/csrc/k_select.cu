@@ -229,26 +229,14 @@ __device__ __forceinline__ void block_sort_regs(uint64_t* win, int NK) {
 // ints.  ~6 barriers and a few dozen instructions per key against a bitonic network's ~60
 // compare-exchange stages; false (win untouched) when a bucket holds more than kBucketMax keys
 // (piles of keys within a narrow key range), for the caller's bitonic sort.
-constexpr int kBucketBins = 2048, kBucketMax = 64;
+constexpr int kBucketBins = 2048, kBucketMax = 256;
 static_assert(kBucketBins == kHistWarps * 256, "the bucket sort reuses the radix histograms");
+// Exclusive scan, in place, of the kBucketBins counts cnt[] by an NT-thread block (misc: >= 32
+// ints of scratch; misc[40..43) gets the bucket holding rank r -- its index, start and count --
+// when 0 <= r < the total).  Ends with a barrier.
 template <int NT>
-__device__ bool block_bucket_sort(uint64_t* win, int n, uint64_t mn, uint64_t hi, uint32_t* cnt, uint64_t* tmp,
-                                  int* misc) {
+__device__ void block_scan_bins(uint32_t* cnt, int* misc, int r) {
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
-  const uint64_t range = hi - mn;
-  const int sh = max(0, 64 - __clzll((long long)range) - 11);  // (x - mn) >> sh < 2048
-  if (tid == 0) misc[32] = 0;
-  __syncthreads();
-  int mx = 0;
-  for (int i = tid; i < n; i += NT) mx = max(mx, (int)atomicAdd(cnt + ((win[i] - mn) >> sh), 1u) + 1);
-  mx = __reduce_max_sync(MV_FULL, mx);
-  if (lane == 0) atomicMax(misc + 32, mx);
-  __syncthreads();
-  if (misc[32] > kBucketMax) {
-    for (int i = tid; i < kBucketBins; i += NT) cnt[i] = 0;
-    __syncthreads();
-    return false;
-  }
   constexpr int PER = kBucketBins / NT;
   uint32_t v[PER], sum = 0;
 #pragma unroll
@@ -276,10 +264,36 @@ __device__ bool block_bucket_sort(uint64_t* win, int n, uint64_t mn, uint64_t hi
   uint32_t run = (wid ? (uint32_t)misc[wid - 1] : 0u) + incl - sum;
 #pragma unroll
   for (int j = 0; j < PER; ++j) {
-    cnt[tid * PER + j] = run;  // bucket start; the scatter's atomics turn it into the bucket end
+    if (r >= 0 && run <= (uint32_t)r && (uint32_t)r < run + v[j]) {
+      misc[40] = tid * PER + j;
+      misc[41] = (int)run;
+      misc[42] = (int)v[j];
+    }
+    cnt[tid * PER + j] = run;
     run += v[j];
   }
   __syncthreads();
+}
+
+template <int NT>
+__device__ bool block_bucket_sort(uint64_t* win, int n, uint64_t mn, uint64_t hi, uint32_t* cnt, uint64_t* tmp,
+                                  int* misc) {
+  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  const uint64_t range = hi - mn;
+  const int sh = max(0, 64 - __clzll((long long)range) - 11);  // (x - mn) >> sh < 2048
+  if (tid == 0) misc[32] = 0;
+  __syncthreads();
+  int mx = 0;
+  for (int i = tid; i < n; i += NT) mx = max(mx, (int)atomicAdd(cnt + ((win[i] - mn) >> sh), 1u) + 1);
+  mx = __reduce_max_sync(MV_FULL, mx);
+  if (lane == 0) atomicMax(misc + 32, mx);
+  __syncthreads();
+  if (misc[32] > kBucketMax) {
+    for (int i = tid; i < kBucketBins; i += NT) cnt[i] = 0;
+    __syncthreads();
+    return false;
+  }
+  block_scan_bins<NT>(cnt, misc, -1);
   for (int i = tid; i < n; i += NT) {
     const uint64_t x = win[i];
     tmp[atomicAdd(cnt + ((x - mn) >> sh), 1u)] = x;
@@ -321,11 +335,11 @@ __global__ void __launch_bounds__(NT, 2048 / NT) k_final_big(const int64_t* __re
   extern __shared__ __align__(16) uint8_t smem[];
   const int NK = next_pow2(max(k, 2));
   uint64_t* buf = reinterpret_cast<uint64_t*>(smem);   // cap
-  uint64_t* win = buf + cap;                           // NK
-  uint32_t* whist = reinterpret_cast<uint32_t*>(win + NK);  // kHistWarps x 256
+  uint64_t* win = buf + cap;                           // NK + kBucketMax
+  uint32_t* whist = reinterpret_cast<uint32_t*>(win + NK + kBucketMax);  // kHistWarps x 256
   uint64_t* s_mm = reinterpret_cast<uint64_t*>(whist + kHistWarps * 256);  // min, max
   int32_t* s_pre = reinterpret_cast<int32_t*>(s_mm + 2);  // npb + 1
-  int32_t* s_int = s_pre + npb + 1;                    // misc: [0..3) digit, [8..16) warp totals, [16..49) sort
+  int32_t* s_int = s_pre + npb + 1;  // misc (128): [0..3) digit, [8..16) warp totals, [16..59) sort, [64..107) fast path
   const int64_t q = blockIdx.x;
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   const int64_t* po = poff + q * npb;
@@ -371,6 +385,7 @@ __global__ void __launch_bounds__(NT, 2048 / NT) k_final_big(const int64_t* __re
   __syncthreads();
   int nsel;              // winners to sort, in win[]
   bool sorted = false;   // ... already sorted (the bucket sort)
+  uint64_t* res = win;   // the sorted winners
   if (T <= k) {
     for (int i = tid; i < NK; i += NT) win[i] = i < T ? buf[i] : MV_KEY_PAD;
     nsel = T;
@@ -396,9 +411,77 @@ __global__ void __launch_bounds__(NT, 2048 / NT) k_final_big(const int64_t* __re
       atomicMin(reinterpret_cast<unsigned long long*>(s_mm), (unsigned long long)mn);
       atomicMax(reinterpret_cast<unsigned long long*>(s_mm + 1), (unsigned long long)mx);
     }
+    if (tid == 0) s_int[120] = 0;
     __syncthreads();
     mn = s_mm[0];
     mx = s_mm[1];
+    // Fast path: one counting pass over kBucketBins equal-width buckets of [mn, mx] and a scan
+    // locate the bucket b* holding the k-th key.  Seeding: the bound is b*'s upper edge (or, when
+    // b* holds more than 64 keys, the upper edge of the sub-bucket of a second counting pass over
+    // b*'s keys).  Final select: the keys of buckets <= b* are scattered bucket-wise and each is
+    // placed by its rank within its bucket -- the first k places are the sorted top-k; taken when
+    // no bucket <= b* holds more than kBucketMax keys, else the radix select below.
+    const int shv = max(0, 64 - __clzll((long long)(mx - mn)) - 11);
+    for (int i = tid; i < T; i += NT) atomicAdd(whist + ((buf[i] - mn) >> shv), 1u);
+    __syncthreads();
+    {
+      int* misc = s_int + 64;
+      block_scan_bins<NT>(whist, misc, k - 1);
+      const int bs = misc[40], st = misc[41], nb = misc[42];
+      if (tau_out) {
+        const uint64_t b0 = mn + ((uint64_t)bs << shv);  // b*'s first key value
+        uint64_t edge = b0 + (shv ? (~0ull >> (64 - shv)) : 0ull);
+        if (nb > 64 && shv > 0) {
+          const int sh2 = max(0, shv - 11);
+          for (int i = tid; i < kBucketBins; i += NT) whist[i] = 0;
+          __syncthreads();
+          for (int i = tid; i < T; i += NT) {
+            const uint64_t x = buf[i];
+            if ((int)((x - mn) >> shv) == bs) atomicAdd(whist + ((x - b0) >> sh2), 1u);
+          }
+          __syncthreads();
+          block_scan_bins<NT>(whist, misc, k - 1 - st);
+          edge = b0 + ((uint64_t)misc[40] << sh2) + (sh2 ? (~0ull >> (64 - sh2)) : 0ull);
+        }
+        if (tid == 0) tau_out[q] = edge < mn || edge > mx ? mx : edge;
+        return;
+      }
+      // the largest bucket <= b*
+      int mxc = 0;
+      constexpr int PER = kBucketBins / NT;
+#pragma unroll
+      for (int j = 0; j < PER; ++j) {
+        const int b = tid * PER + j;
+        if (b < bs) mxc = max(mxc, (int)(whist[b + 1] - whist[b]));
+      }
+      if (tid == 0) mxc = max(mxc, nb);
+      mxc = __reduce_max_sync(MV_FULL, mxc);
+      if (lane == 0) atomicMax(s_int + 120, mxc);
+      __syncthreads();
+      if (s_int[120] <= kBucketMax) {
+        for (int i = tid; i < T; i += NT) {  // bucket-wise scatter into win (st + nb <= k - 1 + kBucketMax)
+          const uint64_t x = buf[i];
+          const int b = (int)((x - mn) >> shv);
+          if (b <= bs) win[atomicAdd(whist + b, 1u)] = x;
+        }
+        __syncthreads();
+        for (int i = tid; i < st + nb; i += NT) {
+          const uint64_t x = win[i];
+          const int b = (int)((x - mn) >> shv);
+          const int s0 = b ? (int)whist[b - 1] : 0, e0 = (int)whist[b];
+          int r = 0;
+          for (int j = s0; j < e0; ++j) r += win[j] < x ? 1 : 0;
+          if (s0 + r < k) buf[s0 + r] = x;
+        }
+        __syncthreads();
+        res = buf;
+        nsel = k;
+        sorted = true;
+        goto output;
+      }
+    }
+    for (int i = tid; i < kBucketBins; i += NT) whist[i] = 0;
+    __syncthreads();
     int lo = 64 - __clzll((long long)(mn ^ mx));  // bits [lo, 64) are common to every key
     uint64_t pfx = lo >= 64 ? 0 : (mn >> lo);
     int below = 0;  // keys whose bits above lo are < pfx
@@ -505,10 +588,11 @@ __global__ void __launch_bounds__(NT, 2048 / NT) k_final_big(const int64_t* __re
     default: block_sort_regs<0, NT>(win, NK); break;  // NK < 1024 or > 4096: shared memory only
   }
   __syncthreads();
+output:
   for (int i = tid; i < k; i += NT) {
     float dv;
     int64_t iv;
-    const uint64_t key = win[i];
+    const uint64_t key = res[i];
     if (i < nsel && key != MV_KEY_PAD) {
       dv = key_dist((uint32_t)(key >> 32), metric);
       iv = sorted_ids[(uint32_t)(key & 0xffffffffu)];
@@ -762,7 +846,7 @@ static cudaError_t launch_big_select(const int64_t* poff, const int32_t* pcnt, c
     redo = nullptr;
   }
   const int NK = next_pow2(max(k, 2));
-  const int fixed = NK * 8 + kHistWarps * 256 * 4 + 16 + (npb + 1) * 4 + 64 * 4 + 64;
+  const int fixed = (NK + kBucketMax) * 8 + kHistWarps * 256 * 4 + 16 + (npb + 1) * 4 + 128 * 4 + 64;
   const int64_t want = max64(tmax, k);  // stage capacity that holds every query
   const int capmax = (227 * 1024 - fixed) / 8;
   // first launch: `ctas` CTAs per SM (228 KB of shared memory per SM, 1 KB reserved per CTA), each
