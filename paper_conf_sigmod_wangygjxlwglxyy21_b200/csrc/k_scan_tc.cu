@@ -103,12 +103,40 @@ __device__ __forceinline__ WorkInfo work_info_of(const TcScanParams& p, int2 it,
 __device__ __forceinline__ WorkInfo work_info(const TcScanParams& p, int w, int qchunk) {
   return work_info_of(p, p.witems[w], qchunk);
 }
+// A work item's dependent loads are software-pipelined across items (producer and gatherer): the
+// (list, bucket) entry of item i+3, then the bucket end and list range of item i+2 (ItemRaw), are
+// loaded while item i runs, and nothing derived from a load is computed in the iteration that
+// issues it -- so no global round trip sits between two items (short items: c3, c5).
+struct ItemRaw {
+  int2 it;
+  int bend;
+  int64_t lo0, lo1;
+};
+__device__ __forceinline__ ItemRaw item_raw(const TcScanParams& p, int2 it) {
+  ItemRaw r;
+  r.it = it;
+  const int l = it.x >= p.nlist ? it.x - p.nlist : it.x;
+  r.bend = p.boff[it.x + 1];
+  r.lo0 = p.list_off[l];
+  r.lo1 = p.list_off[l + 1];
+  return r;
+}
+__device__ __forceinline__ WorkInfo work_info_raw(const TcScanParams& p, const ItemRaw& r, int qchunk) {
+  WorkInfo wi;
+  wi.l = r.it.x >= p.nlist ? r.it.x - p.nlist : r.it.x;
+  wi.bstart = r.it.y;
+  wi.nqc = min(qchunk, r.bend - wi.bstart);
+  wi.lstart = r.lo0;
+  wi.len = (int)min64(r.lo1 - r.lo0, p.rowcap);
+  wi.ntiles = (wi.len + 127) >> 7;
+  return wi;
+}
 
-constexpr int kNTS = 4;          // per-tile side-data ring slots
+constexpr int kMaxNTS = 16;      // per-tile side-data ring slots (p.nts <= kMaxNTS)
 constexpr int kMaxAcc = 8;       // TMEM accumulator buffers (tiles in flight between MMA and epilogue)
 // side slot: norms f64 [1152 B] | rank u32 [640 B] | ids i64 [1152 B]; each copied as the 16-B aligned
 // superset of the tile's 128 rows (the arrays are padded at allocation so the copy stays in bounds)
-constexpr int kSideBytes = 3072;
+// (p.side_bytes: 3072 with a bitset, else 1792 -- the ids are not copied)
 constexpr int kSideRank = 1152, kSideIds = 1792;
 // epilogue warps: three per TMEM lane quarter (<= 128 registers per thread: 512 threads fit the
 // register file).  Measured: 8 -> 12 took configs[1]'s phase B from 289 to 256 us and configs[4]'s
@@ -190,8 +218,9 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
   uint64_t* tfull = empty_m + 2;
   uint64_t* tempty = tfull + kMaxAcc;
   uint64_t* full_t = tempty + kMaxAcc;
-  uint64_t* empty_t = full_t + kNTS;
-  uint32_t* tslot = reinterpret_cast<uint32_t*>(empty_t + kNTS);
+  uint64_t* empty_t = full_t + kMaxNTS;
+  uint32_t* tslot = reinterpret_cast<uint32_t*>(empty_t + kMaxNTS);
+  const int NTS = p.nts, SIDEB = p.side_bytes;
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
@@ -206,11 +235,11 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
     }
     for (int a = 0; a < kMaxAcc; ++a) {
       mbar_init(&tfull[a], 1);
-      mbar_init(&tempty[a], kEpiWarps);
+      mbar_init(&tempty[a], 4);  // the tile's epilogue warp of each lane quarter
     }
-    for (int s = 0; s < kNTS; ++s) {
+    for (int s = 0; s < NTS; ++s) {
       mbar_init(&full_t[s], 1);
-      mbar_init(&empty_t[s], kEpiWarps);
+      mbar_init(&empty_t[s], 4);
     }
     fence_mbar_init();
   }
@@ -245,20 +274,22 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
       uint32_t it = 0, tcount = 0;
       const uint32_t side_tx = 528 + (use_norms ? 1040 : 0) + (use_ids ? 1040 : 0);
       const uint64_t pol = l2_evict_first_policy();
-      // two-deep prefetch: the next item's list range and the one after's (list, bucket) pair are
-      // in flight while this item's tiles are issued, so no dependent load sits between items
-      int2 itn = item(1) < nwork ? p.witems[item(1)] : make_int2(0, 0);
+      // three-deep load pipeline (ItemRaw): item i+1's work info is ready when item i starts
+      int2 it3 = item(2) < nwork ? p.witems[item(2)] : make_int2(0, 0);
+      ItemRaw r2{};
+      if (item(1) < nwork) r2 = item_raw(p, p.witems[item(1)]);
       WorkInfo wn = item(0) < nwork ? work_info(p, item(0), QC) : WorkInfo{};
       for (int i = 0; item(i) < nwork; ++i) {
         const WorkInfo wi = wn;
-        if (item(i + 1) < nwork) wn = work_info_of(p, itn, QC);
-        if (item(i + 2) < nwork) itn = p.witems[item(i + 2)];
+        if (item(i + 1) < nwork) wn = work_info_raw(p, r2, QC);
+        if (item(i + 2) < nwork) r2 = item_raw(p, it3);
+        if (item(i + 3) < nwork) it3 = p.witems[item(i + 3)];
         for (int t = 0; t < wi.ntiles; ++t, ++tcount) {
           const int row0 = (int)(wi.lstart + t * 128);
-          const uint32_t ts = tcount % kNTS, tr = tcount / kNTS;
+          const uint32_t ts = tcount % NTS, tr = tcount / NTS;
           mbar_wait(&empty_t[ts], (tr & 1) ^ 1);
           mbar_expect_tx(&full_t[ts], side_tx);
-          uint8_t* sd = side + ts * kSideBytes;
+          uint8_t* sd = side + ts * SIDEB;
           bulk_g2s(sd + kSideRank, p.rank + (row0 & ~3), 528, &full_t[ts]);
           if (use_norms) bulk_g2s(sd, p.norms + (row0 & ~1), 1040, &full_t[ts]);
           if (use_ids) bulk_g2s(sd + kSideIds, p.ids + (row0 & ~1), 1040, &full_t[ts]);
@@ -308,6 +339,7 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
           for (int c = 0; c < nchunks; ++c, ++it) {
             const uint32_t s = it % nstage;
             mbar_wait(&full_x[s], (it / nstage) & 1);
+            MV_TRACE(7, it);
             tc_fence_after();
             const uint32_t xb = smem_u32(Xs + s * 128 * ATOM);
             const uint32_t qb = qbase + c * N * ATOM;
@@ -346,14 +378,32 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
       float qs[2], qe[2];
       int64_t base[2];
     };
-    auto prefetch = [&](int w) {
+    // raw loads of the (list, bucket) level: the item's ranges and its queries' pair ids (bq
+    // entries past the item are read but unused; nbq bounds the read)
+    struct QRaw {
+      ItemRaw r;
+      int pr[2];
+    };
+    auto q_raw = [&](int2 it) {
+      QRaw x;
+      x.r = item_raw(p, it);
+#pragma unroll
+      for (int u = 0; u < 2; ++u) {
+        const int i = tq + 64 * u;
+        const int64_t pos = (int64_t)it.y + i;
+        x.pr[u] = (i < QC && pos < p.nbq) ? p.bq[pos] : 0;
+      }
+      return x;
+    };
+    // the per-query level (issued one item ahead; used when the item is processed)
+    auto prefetch = [&](const QRaw& x) {
       Pref f;
-      f.wi = work_info(p, w, QC);
+      f.wi = work_info_raw(p, x.r, QC);
 #pragma unroll
       for (int u = 0; u < 2; ++u) {
         const int i = tq + 64 * u;
         if (i < f.wi.nqc) {
-          f.pr[u] = p.bq[f.wi.bstart + i];
+          f.pr[u] = x.pr[u];
           // phase-A entries carry pair id npairs + p (their own output regions)
           const int64_t npairs = p.nq * p.npb;
           f.q[u] = (int)((f.pr[u] >= npairs ? f.pr[u] - npairs : f.pr[u]) / p.npb);
@@ -368,7 +418,10 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
       return f;
     };
     Pref cur;
-    if (item(0) < nwork) cur = prefetch(item(0));
+    if (item(0) < nwork) cur = prefetch(q_raw(p.witems[item(0)]));
+    QRaw n2{};
+    if (item(1) < nwork) n2 = q_raw(p.witems[item(1)]);
+    int2 n1 = item(2) < nwork ? p.witems[item(2)] : make_int2(0, 0);
     uint32_t wcount = 0;
     // the epilogue never waits for its peers at the end of an item: the gatherer publishes an
     // item's candidate counts when its metadata buffer comes back (every epilogue warp has
@@ -385,7 +438,9 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
     };
     for (int i = 0; item(i) < nwork; ++i, ++wcount) {
       Pref nxt;
-      if (item(i + 1) < nwork) nxt = prefetch(item(i + 1));
+      if (item(i + 1) < nwork) nxt = prefetch(n2);
+      if (item(i + 2) < nwork) n2 = q_raw(n1);
+      if (item(i + 3) < nwork) n1 = p.witems[item(i + 3)];
       const WorkInfo wi = cur.wi;
       const int NQ = (wi.nqc + 15) & ~15;
       const int N = P * NQ;
@@ -447,6 +502,7 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
       cp_async_wait_all();
       fence_proxy_async();
       mbar_arrive(&full_q[b]);
+      if (tq == 0) MV_TRACE(5, wcount);
       cur = nxt;
     }
     // the last (up to) two items: wait until the epilogue is done with them, then publish
@@ -460,8 +516,12 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
     // ------------------------------------------------------------------ epilogue (8 warps)
     const int ew = warp - 4;            // 0..7
     const int quarter = warp & 3;       // TMEM lane quarter this warp may access
-    const int half = ew >> 2;           // which column chunks of the accumulator it reads
+    // the NPART warps of a lane quarter take the tiles in turn (tile titer: warp part titer % NPART),
+    // each a whole tile's columns: one warp's per-tile latency chain (side data, TMEM loads, the
+    // filter, the emission) overlaps its peers' tiles (measured: splitting every tile's columns
+    // over the three warps left configs[4]'s 16-query tiles epilogue-bound at ~2300 cycles each)
     constexpr int NPART = kEpiWarps / 4;  // epilogue warps per lane quarter
+    const int part = ew >> 2;
     const int row = quarter * 32 + lane;
     const int et = threadIdx.x - 128;   // 0..255
     const uint32_t ltmask = (1u << lane) - 1;
@@ -475,12 +535,13 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
       const uint32_t s_qnf = smem_u32(mt.qnf), s_thf = smem_u32(mt.thf), s_qs = smem_u32(mt.qs),
                      s_qaf = smem_u32(mt.qaf), s_cnt = smem_u32(mt.cnt), s_base = smem_u32(mt.base);
       for (int t = 0; t < wi.ntiles; ++t, ++titer) {
+        if ((int)(titer % NPART) != part) continue;
         const uint32_t a = titer % NACC;
-        const uint32_t ts = titer % kNTS;
+        const uint32_t ts = titer % NTS;
         const int vrow = t * 128 + row;
         const int row0 = (int)(wi.lstart + t * 128);
-        mbar_wait(&full_t[ts], (titer / kNTS) & 1);
-        const uint8_t* sd = side + ts * kSideBytes;
+        mbar_wait(&full_t[ts], (titer / NTS) & 1);
+        const uint8_t* sd = side + ts * SIDEB;
         const uint32_t rk = reinterpret_cast<const uint32_t*>(sd + kSideRank)[(row0 & 3) + row];
         bool valid = vrow < wi.len;
         if (valid && use_ids)
@@ -491,7 +552,7 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
         if (et == 0) MV_TRACE(6, titer);
         tc_fence_after();
         const uint32_t tbase = tmem + a * p.ncol + ((uint32_t)(quarter * 32) << 16);
-        for (int qc = half * W; qc < NQ; qc += NPART * W) {
+        for (int qc = 0; qc < NQ; qc += W) {
           uint32_t r[PMAX][W];
           tmem_ld_w<W>(tbase + qc, r[0]);
           if (TYPE == MV_IVF_SQ8 || P == 2) tmem_ld_w<W>(tbase + NQ + qc, r[1]);
@@ -696,7 +757,7 @@ cudaError_t launch_tf32_check(const float* x, int64_t n, int* flag, cudaStream_t
 // ----------------------------------------------------------------------------------------------
 // Shared-memory plan: X ring + double-buffered query planes + double-buffered per-query metadata
 // + the side-data ring; the deepest X ring (<= the type's cap) that fits in 227 KB.
-static bool tc_scan_layout(int type, int dpad, int qc, int ns, TcScanParams& p) {
+static bool tc_scan_layout(int type, int dpad, int qc, int ns, bool ids, TcScanParams& p) {
   const int esz = type == MV_IVF_FLAT ? 4 : 1;
   // swizzle-atom row: 128 B (FLAT: 32 fp32; SQ8 rows of a multiple of 128 codes), else 32 B (SQ8)
   const int atom = (type == MV_IVF_FLAT || dpad % 128 == 0) ? 128 : 32;
@@ -730,12 +791,17 @@ static bool tc_scan_layout(int type, int dpad, int qc, int ns, TcScanParams& p) 
   p.off_q = ns * stage;
   p.off_meta = p.off_q + 2 * p.q_bytes;
   p.off_side = up(p.off_meta + 2 * p.meta_bytes, 128);
-  p.off_bar = p.off_side + kNTS * kSideBytes;
-  p.smem_total = p.off_bar + (2 * ns + 6 + 2 * kMaxAcc + 2 * kNTS) * 8 + 16 + 1024;  // + 1 KB alignment slack
+  // side-data slots: every tile in the X ring, in the accumulators and in the epilogue holds one
+  // (with too few the producer stalls on them and the ring never fills: 4 slots capped configs[4]'s
+  // one-stage SQ8 tiles at 4 tiles in flight)
+  p.side_bytes = ids ? 3072 : 1792;
+  p.nts = std::max(4, std::min(kMaxNTS, ns / p.nchunks + p.nacc + 1));
+  p.off_bar = p.off_side + p.nts * p.side_bytes;
+  p.smem_total = p.off_bar + (2 * ns + 6 + 2 * kMaxAcc + 2 * kMaxNTS) * 8 + 16 + 1024;  // + 1 KB alignment slack
   return p.smem_total <= 227 * 1024;
 }
 
-bool tc_scan_plan(int type, int dpad, int k, double qpl, const Options& o, TcScanParams& p) {
+bool tc_scan_plan(int type, int dpad, int k, double qpl, bool ids, const Options& o, TcScanParams& p) {
   const bool wide = type == MV_IVF_FLAT || dpad % 128 == 0;  // 16-KB stages
   // SQ8 items: 64 queries.  (Measured on configs[4], ~10 queries per probed list: 32-query items
   // with 4 TMEM accumulators in flight 0.76M qps, 16 with 8 0.61M, 64 with 2 0.87M; qpl, the
@@ -745,12 +811,12 @@ bool tc_scan_plan(int type, int dpad, int k, double qpl, const Options& o, TcSca
   // tuning options (mv_index_set_option "sq8_qc" / "flat_qc"): launch shape only, never the result
   if (o.sq8_qc > 0 && type == MV_IVF_SQ8) qcmax = std::max(16, std::min(64, o.sq8_qc / 16 * 16));
   if (o.flat_qc > 0 && type == MV_IVF_FLAT) qcmax = std::max(16, std::min(128, o.flat_qc / 16 * 16));
-  const int nscap = wide ? 8 : 24;
+  const int nscap = wide ? 12 : 36;
   const int nsmin = wide ? 4 : 6;  // >= 64 KB (16-KB stages) / 24 KB (4-KB stages) of list tiles in flight
   p.k = k;
   for (int qc = qcmax; qc >= 16; qc -= 16)
     for (int ns = nscap; ns >= nsmin; --ns)
-      if (tc_scan_layout(type, dpad, qc, ns, p)) return true;
+      if (tc_scan_layout(type, dpad, qc, ns, ids, p)) return true;
   return false;
 }
 

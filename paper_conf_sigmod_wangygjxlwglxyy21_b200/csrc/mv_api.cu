@@ -334,6 +334,7 @@ mv_status mv_index_set_option(mv_index* ix, const char* name, int64_t value) {
   else if (n == "coarse_epi") o.coarse_epi = (int)std::min<int64_t>(value, 16);
   else if (n == "coarse_nacc") o.coarse_nacc = (int)std::min<int64_t>(value, 4);
   else if (n == "workspace_bytes") o.workspace = value;
+  else if (n == "scan_trace") o.scan_trace = value;  // development builds only (-DMV_SCAN_TRACE)
   else if (n == "large_k_select") o.large_k_select = value != 0;
   else if (n == "big_cap") o.big_cap = std::max<int64_t>(value, 0);
   else if (n == "big_ctas") o.big_ctas = (int)std::min<int64_t>(std::max<int64_t>(value, 0), 4);
@@ -657,7 +658,7 @@ static mv_status search_chunk(mv_index* ix, const float* q, int64_t nq, int32_t 
   prof_mark(ix, st);
   // a4 (the work-item shape follows the scan's shared-memory plan)
   TcScanParams tp;
-  if (!tc_scan_plan(ix->type, dpad, k, (double)nq * npb / std::max(1, nlist), ix->opt, tp))
+  if (!tc_scan_plan(ix->type, dpad, k, (double)nq * npb / std::max(1, nlist), bs != nullptr, ix->opt, tp))
     return fail(MV_EINVAL, "search: no tensor-core scan plan fits d = %d", ix->d);
   const int qchunk = tp.qchunk;
   const int qchunk_min = tp.qchunk_split;  // FLAT two-plane items
@@ -754,7 +755,7 @@ static mv_status search_chunk(mv_index* ix, const float* q, int64_t nq, int32_t 
   tp.list_off = ix->list_off; tp.norms = ix->norms; tp.ids = ix->ids; tp.rank = ix->rank;
   tp.bitset = bs; tp.nbits = bs ? nbits : 0;
   tp.qplanes = qplanes; tp.qnorm = qn64; tp.qscale = qscale; tp.qa = qa;
-  tp.bq = b.bq; tp.boff = b.boff; tp.witems = b.witems; tp.nlist = nlist; tp.cfg = qcfg;
+  tp.bq = b.bq; tp.nbq = nent; tp.boff = b.boff; tp.witems = b.witems; tp.nlist = nlist; tp.cfg = qcfg;
   tp.poff = b.poff; tp.pcnt = b.pcnt; tp.part = part; tp.tau = tau;
   tp.approx_always = approx_always ? 1 : 0; tp.qerr = qerr;
   tp.prof = nullptr;
@@ -773,6 +774,7 @@ static mv_status search_chunk(mv_index* ix, const float* q, int64_t nq, int32_t 
     prof_mark(ix, st);
     // ... phase B over every probed pair, emitting keys <= tau_q
     tp.phase = 1;
+    tp.prof = reinterpret_cast<unsigned long long*>(ix->opt.scan_trace);
     tp.rowcap = 0x7fffffff;
     tp.wbeg = b.woff + nlist;
     tp.nwitems = b.woff + 2 * nlist;

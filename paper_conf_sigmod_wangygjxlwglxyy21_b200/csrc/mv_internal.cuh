@@ -181,6 +181,7 @@ struct Options {
   int flat_qc = 0;          // FLAT queries per scan work item (16..128)
   int coarse_nqb = 0, coarse_cs = 0, coarse_epi = 0, coarse_nacc = 0;  // coarse GEMM launch shape
   int64_t workspace = 0;    // per-search scratch budget in bytes (0: half of the free device memory)
+  int64_t scan_trace = 0;   // -DMV_SCAN_TRACE builds: device address of the phase-B timeline buffer
   int large_k_select = 0;   // k > 256: 0 staged radix select, 1 sample-threshold select (radix fallback)
   int big_ctas = 0;         // k > 256 staged select: CTAs per SM of its first launch (1..4; 0 = 2)
   int64_t big_cap = 0;      // ... and its stage capacity in keys (0: the most that fits big_ctas per SM)
@@ -284,6 +285,7 @@ struct TcScanParams {
   int rowcap;              // rows scanned per list in this launch (phase A: capA; else INT_MAX)
   int64_t nq;              // FLAT query planes are plane-major [2][nq][dpad]
   int off_x, off_q, q_bytes, off_meta, meta_bytes, off_side, off_bar, smem_total;
+  int nts, side_bytes;     // side-data ring: slots and bytes per slot
   const int64_t* list_off;
   const double* norms;     // ||x||^2 (FLAT) or ||x_hat||^2 (SQ8), fp64
   const int64_t* ids;
@@ -295,6 +297,7 @@ struct TcScanParams {
   const float* qscale;
   const double* qa;        // SQ8: q.a fp64
   const int32_t* bq;
+  int64_t nbq;             // entries of bq
   const int32_t* boff;
   const int2* witems;
   const int32_t* wbeg;     // device: first work item of this launch (nullable = 0)
@@ -307,7 +310,7 @@ struct TcScanParams {
   const float* qerr;       // filter mode: E_q, the bound on |approximate - exact badness|
   unsigned long long* prof;  // -DMV_SCAN_TRACE builds only: CTA-0 timeline
 };
-bool tc_scan_plan(int type, int dpad, int k, double qpl, const Options& o, TcScanParams& p);  // qpl: queries per probed list
+bool tc_scan_plan(int type, int dpad, int k, double qpl, bool ids, const Options& o, TcScanParams& p);  // qpl: queries per probed list
 // the payload's tensor maps: boxes of 128, 64, 32, 16 rows (one swizzle atom wide)
 struct XMaps {
   CUtensorMap m[4];
