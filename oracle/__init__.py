@@ -14,8 +14,13 @@ Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s ``cpu_baseline``
 Parity status of each function (DESIGN.md §2 lists the pins):
   exact_knn, assign, sq8_train/encode/decode, probe, IvfIndex.search, topk_rounds,
   merge_topk, recall -- all pinned by tests/test_oracle_*.py.
+  multi.py: range_bitset, partition_plan, partition_search (strategy E),
+  multivector_scores / multivector_topk (§4.2) -- pinned by tests/test_oracle_multi.py.
 """
 from .ivf import (  # noqa: F401
     FLAT, IP, L2, SQ8, IvfIndex, assign, bit_is_set, distances, exact_knn, merge_topk, pad_value, probe,
     recall_at_k, select_topk, sq8_decode, sq8_encode, sq8_train, topk_rounds,
+)
+from .multi import (  # noqa: F401,E402
+    multivector_scores, multivector_topk, partition_plan, partition_search, range_bitset,
 )
