@@ -146,7 +146,8 @@ __global__ void __launch_bounds__(kPlanThreads) k_plan(const PlanArgs a) {
     const bool sp = a.qlo_any != nullptr && *a.qlo_any != 0;
     a.qcfg[0] = sp ? a.qc_split : a.qc_exact;
     a.qcfg[1] = sp ? a.p_split : a.p_exact;
-    *b.counter = 0;
+    b.counter[0] = 0;
+    b.counter[1] = 0;
   }
   grid.sync();
   const int qchunk = a.qcfg[0];
@@ -265,29 +266,29 @@ __global__ void __launch_bounds__(kPlanThreads) k_plan(const PlanArgs a) {
 
   // 5 ---------------------------------------------------------------------------------------
   // work items, and the histogram of their cost keys: descending cost = 64 * tiles + queries
-  // (tiles = ceil(|list| / 128)); every phase-A item (virtual list < nlist) precedes every
-  // phase-B item
+  // (tiles = ceil(|list| / 128), queries of the list's first item); every phase-A item (virtual
+  // list < nlist) precedes every phase-B item.  A list's items (several when more than qchunk
+  // queries probe it) get one key and consecutive places in the order, so the static schedule
+  // runs them at the same time on neighbouring CTAs and the siblings' tile reads hit L2 (round 2
+  // sorted items one by one: c4's phase B read 1.83x its algorithmic bytes from DRAM)
   constexpr int HB = kPlanCostBins / 2;
-  auto key = [&](int2 it) {
-    const int l = it.x >= nlist ? it.x - nlist : it.x;
-    const int nqw = min(qchunk, b.boff[it.x + 1] - it.y);
+  auto key = [&](int v) {
+    const int l = v >= nlist ? v - nlist : v;
+    const int nqw = min(qchunk, b.boff[v + 1] - b.boff[v]);
     int64_t len = a.list_off[l + 1] - a.list_off[l];
-    if (a.split && it.x < nlist) len = min64(len, a.capA);
+    if (a.split && v < nlist) len = min64(len, a.capA);
     const int tiles = (int)min64((len + 127) / 128, 63);
-    return (it.x >= nlist ? HB : 0) + HB - 1 - min(HB - 1, tiles * 64 + min(nqw, 63));
+    return (v >= nlist ? HB : 0) + HB - 1 - min(HB - 1, tiles * 64 + min(nqw, 63));
   };
   for (int64_t v = gtid; v < nv; v += gthreads) {
-    const int n = b.wcount[v], o = b.woff[v], bb = b.boff[v];
-    for (int c = 0; c < n; ++c) {
-      const int2 it = make_int2((int)v, bb + c * qchunk);
-      b.witems_unsorted[o + c] = it;
-      atomicAdd(b.whist + key(it), 1);
-    }
+    const int n = b.wcount[v];
+    if (n) atomicAdd(b.whist + key((int)v), n);
   }
   grid.sync();
 
   // 6 ---------------------------------------------------------------------------------------
-  // counting sort by the cost key: block 0 scans the histogram, then every block scatters
+  // counting sort by the cost key: block 0 scans the histogram, then every list reserves its
+  // items' places in one piece (kItemMulti marks the items of a list with siblings)
   if (blockIdx.x == 0) {
     int loc[8], acc = 0;
 #pragma unroll
@@ -309,10 +310,12 @@ __global__ void __launch_bounds__(kPlanThreads) k_plan(const PlanArgs a) {
     for (int j = 0; j < 8; ++j) b.whist[tid * 8 + j] = base + loc[j];
   }
   grid.sync();
-  const int nwork = b.woff[nv];
-  for (int64_t w = gtid; w < nwork; w += gthreads) {
-    const int2 it = b.witems_unsorted[w];
-    b.witems[atomicAdd(b.whist + key(it), 1)] = it;
+  for (int64_t v = gtid; v < nv; v += gthreads) {
+    const int n = b.wcount[v], bb = b.boff[v];
+    if (!n) continue;
+    const int o = atomicAdd(b.whist + key((int)v), n);
+    const int x = (int)v | (n > 1 ? kItemMulti : 0);
+    for (int c = 0; c < n; ++c) b.witems[o + c] = make_int2(x, bb + c * qchunk);
   }
 }
 

@@ -87,11 +87,15 @@ __device__ __forceinline__ uint32_t f2key_fast(float f) {
 
 struct WorkInfo {
   int l, bstart, nqc, len, ntiles;
+  int multi;  // the list has sibling items (kItemMulti): its tiles are kept in L2 for them
   int64_t lstart;
 };
+static_assert(sizeof(WorkInfo) == 32, "the metadata header holds one WorkInfo");
 
 __device__ __forceinline__ WorkInfo work_info_of(const TcScanParams& p, int2 it, int qchunk) {
   WorkInfo wi;
+  wi.multi = it.x & kItemMulti;
+  it.x &= ~kItemMulti;
   wi.l = it.x >= p.nlist ? it.x - p.nlist : it.x;
   wi.bstart = it.y;
   wi.nqc = min(qchunk, p.boff[it.x + 1] - wi.bstart);
@@ -115,6 +119,7 @@ struct ItemRaw {
 __device__ __forceinline__ ItemRaw item_raw(const TcScanParams& p, int2 it) {
   ItemRaw r;
   r.it = it;
+  it.x &= ~kItemMulti;
   const int l = it.x >= p.nlist ? it.x - p.nlist : it.x;
   r.bend = p.boff[it.x + 1];
   r.lo0 = p.list_off[l];
@@ -123,7 +128,9 @@ __device__ __forceinline__ ItemRaw item_raw(const TcScanParams& p, int2 it) {
 }
 __device__ __forceinline__ WorkInfo work_info_raw(const TcScanParams& p, const ItemRaw& r, int qchunk) {
   WorkInfo wi;
-  wi.l = r.it.x >= p.nlist ? r.it.x - p.nlist : r.it.x;
+  wi.multi = r.it.x & kItemMulti;
+  const int v = r.it.x & ~kItemMulti;
+  wi.l = v >= p.nlist ? v - p.nlist : v;
   wi.bstart = r.it.y;
   wi.nqc = min(qchunk, r.bend - wi.bstart);
   wi.lstart = r.lo0;
@@ -134,6 +141,8 @@ __device__ __forceinline__ WorkInfo work_info_raw(const TcScanParams& p, const I
 
 constexpr int kMaxNTS = 16;      // per-tile side-data ring slots (p.nts <= kMaxNTS)
 constexpr int kMaxAcc = 8;       // TMEM accumulator buffers (tiles in flight between MMA and epilogue)
+constexpr int kRing = 16;        // item-position ring (gatherer -> producer)
+constexpr int kLook = 12;        // the gatherer takes positions this many items ahead (<= kRing + 1)
 // side slot: norms f64 [1152 B] | rank u32 [640 B] | ids i64 [1152 B]; each copied as the 16-B aligned
 // superset of the tile's 128 rows (the arrays are padded at allocation so the copy stays in bounds)
 // (p.side_bytes: 3072 with a bitset, else 1792 -- the ids are not copied)
@@ -203,6 +212,11 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
   // epilogue column chunk: 16 (FLAT), 8 (SQ8: few queries per list, so both warps of a lane quarter
   // get columns)
   constexpr int W = TYPE == MV_IVF_FLAT ? 16 : 8;
+  // query columns per plane: a multiple of the epilogue chunk.  The MMA's N = P x NQ must be a
+  // multiple of 16: SQ8's two digit planes allow 8-column granularity (c3 averages ~20 queries per
+  // probed list, c5 ~10: 24 / 16 columns per plane instead of 32 / 16)
+  constexpr int QG = W;
+  static_assert(TYPE == MV_IVF_FLAT || (kSq8Planes * QG) % 16 == 0, "SQ8 MMA width must be a multiple of 16");
 
   uint8_t* Xs = sm + p.off_x;
   uint8_t* Qs = sm + p.off_q;
@@ -219,7 +233,10 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
   uint64_t* tempty = tfull + kMaxAcc;
   uint64_t* full_t = tempty + kMaxAcc;
   uint64_t* empty_t = full_t + kMaxNTS;
-  uint32_t* tslot = reinterpret_cast<uint32_t*>(empty_t + kMaxNTS);
+  uint64_t* sfull = empty_t + kMaxNTS;   // item-position ring: filled by the gatherer ...
+  uint64_t* sempty = sfull + kRing;      // ... drained by the producer
+  int32_t* ring = reinterpret_cast<int32_t*>(sempty + kRing);
+  uint32_t* tslot = reinterpret_cast<uint32_t*>(ring + kRing);
   const int NTS = p.nts, SIDEB = p.side_bytes;
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -240,6 +257,10 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
     for (int s = 0; s < NTS; ++s) {
       mbar_init(&full_t[s], 1);
       mbar_init(&empty_t[s], 4);
+    }
+    for (int s = 0; s < kRing; ++s) {
+      mbar_init(&sfull[s], 1);
+      mbar_init(&sempty[s], 1);
     }
     fence_mbar_init();
   }
@@ -262,28 +283,46 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
   };
   if (p.prof && threadIdx.x == 0 && blockIdx.x < 148) p.prof[8 * 1024 + blockIdx.x * 3] = gtimer();
 #endif
-  // static schedule over the longest-first item order, snake-wise: round i gives CTA b the item
-  // i*G + b (even rounds) or i*G + G-1-b (odd rounds), which balances sorted costs far better than
-  // plain round-robin (every role walks the same sequence)
-  const int wb = p.wbeg ? *p.wbeg : 0, G = gridDim.x, bx = blockIdx.x;
-  auto item = [&](int i) { return wb + i * G + ((i & 1) ? G - 1 - bx : bx); };
+  // dynamic schedule over the longest-first item order: the gatherer takes the next position from
+  // the launch's global counter kLook items ahead of its own iteration and hands the positions to
+  // the producer through a shared-memory ring (the MMA and epilogue warps get each item from the
+  // gatherer's metadata).  Items are taken in order by whichever CTA is free: a list's sibling items
+  // (consecutive positions) run at the same time on several CTAs, so its tiles come from DRAM once
+  // and from L2 for the siblings (round 2's static snake schedule read c4's lists 1.83x)
+  const int wb = p.wbeg ? *p.wbeg : 0;
 
   if (warp == 0) {
     // ------------------------------------------------------------------ TMA producer
     if (lane == 0) {
       uint32_t it = 0, tcount = 0;
       const uint32_t side_tx = 528 + (use_norms ? 1040 : 0) + (use_ids ? 1040 : 0);
-      const uint64_t pol = l2_evict_first_policy();
+      // list tiles stream through L2 evict-first, except a list with sibling items: its neighbours
+      // in the schedule read the same tiles at about the same time
+      const uint64_t pol_first = l2_evict_first_policy(), pol_normal = l2_evict_normal_policy();
+      // the item positions, in the gatherer's order
+      auto take = [&](uint32_t j) {
+        const uint32_t sl = j % kRing;
+        mbar_wait(&sfull[sl], (j / kRing) & 1);
+        const int v = ring[sl];
+        mbar_arrive(&sempty[sl]);
+        return v;
+      };
       // three-deep load pipeline (ItemRaw): item i+1's work info is ready when item i starts
-      int2 it3 = item(2) < nwork ? p.witems[item(2)] : make_int2(0, 0);
+      int q0 = take(0), q1 = take(1), q2 = take(2);
+      int2 it3 = q2 < nwork ? p.witems[q2] : make_int2(0, 0);
       ItemRaw r2{};
-      if (item(1) < nwork) r2 = item_raw(p, p.witems[item(1)]);
-      WorkInfo wn = item(0) < nwork ? work_info(p, item(0), QC) : WorkInfo{};
-      for (int i = 0; item(i) < nwork; ++i) {
+      if (q1 < nwork) r2 = item_raw(p, p.witems[q1]);
+      WorkInfo wn = q0 < nwork ? work_info(p, q0, QC) : WorkInfo{};
+      for (uint32_t i = 0; q0 < nwork; ++i) {
         const WorkInfo wi = wn;
-        if (item(i + 1) < nwork) wn = work_info_raw(p, r2, QC);
-        if (item(i + 2) < nwork) r2 = item_raw(p, it3);
-        if (item(i + 3) < nwork) it3 = p.witems[item(i + 3)];
+        const int q3 = q2 < nwork ? take(i + 3) : nwork;  // (positions only grow)
+        if (q1 < nwork) wn = work_info_raw(p, r2, QC);
+        if (q2 < nwork) r2 = item_raw(p, it3);
+        if (q3 < nwork) it3 = p.witems[q3];
+        q0 = q1;
+        q1 = q2;
+        q2 = q3;
+        const uint64_t pol = wi.multi ? pol_normal : pol_first;
         for (int t = 0; t < wi.ntiles; ++t, ++tcount) {
           const int row0 = (int)(wi.lstart + t * 128);
           const uint32_t ts = tcount % NTS, tr = tcount / NTS;
@@ -319,14 +358,15 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
   } else if (warp == 1) {
     // ------------------------------------------------------------------ MMA issuer
     if (lane == 0) {
-      uint32_t it = 0, titer = 0, wcount = 0;
-      for (int i = 0; item(i) < nwork; ++i, ++wcount) {
+      uint32_t it = 0, titer = 0;
+      for (uint32_t wcount = 0;; ++wcount) {
         const uint32_t b = wcount & 1;
         mbar_wait(&full_q[b], (wcount >> 1) & 1);
         MV_TRACE(1, wcount);
         tc_fence_after();
         const WorkInfo wi = *meta_at(metab + b * p.meta_bytes, QCP).wi;
-        const int NQ = (wi.nqc + 15) & ~15;
+        if (wi.ntiles < 0) break;  // the gatherer's end marker
+        const int NQ = (wi.nqc + QG - 1) & ~(QG - 1);
         const int N = P * NQ;
         const uint32_t idesc = TYPE == MV_IVF_FLAT ? idesc_tf32(N) : idesc_u8s8(N);
         const uint32_t qbase = smem_u32(Qs + b * p.q_bytes);
@@ -417,11 +457,24 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
       }
       return f;
     };
+    // item positions: thread tq == 0 takes them from the launch's counter kLook items ahead and
+    // publishes them in the ring (for the producer, and for every gatherer thread after the
+    // iteration's named barrier: position j is read at iteration j - 3 >= its publication + 1)
+    int pend = 0;
+    if (tq == 0) {
+      for (int j = 0; j < kLook - 1; ++j) {
+        ring[j] = wb + atomicAdd(p.counter, 1);
+        mbar_arrive(&sfull[j]);
+      }
+      pend = wb + atomicAdd(p.counter, 1);  // position kLook - 1: published at iteration 0
+    }
+    named_bar(2, 64);
+    auto pos = [&](uint32_t j) { return ring[j % kRing]; };
     Pref cur;
-    if (item(0) < nwork) cur = prefetch(q_raw(p.witems[item(0)]));
+    if (pos(0) < nwork) cur = prefetch(q_raw(p.witems[pos(0)]));
     QRaw n2{};
-    if (item(1) < nwork) n2 = q_raw(p.witems[item(1)]);
-    int2 n1 = item(2) < nwork ? p.witems[item(2)] : make_int2(0, 0);
+    if (pos(1) < nwork) n2 = q_raw(p.witems[pos(1)]);
+    int2 n1 = pos(2) < nwork ? p.witems[pos(2)] : make_int2(0, 0);
     uint32_t wcount = 0;
     // the epilogue never waits for its peers at the end of an item: the gatherer publishes an
     // item's candidate counts when its metadata buffer comes back (every epilogue warp has
@@ -436,20 +489,36 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
       }
       prev_nqc[bb] = 0;
     };
-    for (int i = 0; item(i) < nwork; ++i, ++wcount) {
+    for (uint32_t i = 0;; ++i, ++wcount) {
+      const bool done = pos(i) >= nwork;  // positions only grow: every later one is past the end too
       Pref nxt;
-      if (item(i + 1) < nwork) nxt = prefetch(n2);
-      if (item(i + 2) < nwork) n2 = q_raw(n1);
-      if (item(i + 3) < nwork) n1 = p.witems[item(i + 3)];
+      if (!done) {
+        if (pos(i + 1) < nwork) nxt = prefetch(n2);
+        if (pos(i + 2) < nwork) n2 = q_raw(n1);
+        if (pos(i + 3) < nwork) n1 = p.witems[pos(i + 3)];
+        if (tq == 0) {  // publish position i + kLook - 1, take position i + kLook
+          const uint32_t j = i + kLook - 1, sl = j % kRing;
+          mbar_wait(&sempty[sl], ((j / kRing) & 1) ^ 1);
+          ring[sl] = pend;
+          mbar_arrive(&sfull[sl]);
+          pend = wb + atomicAdd(p.counter, 1);
+        }
+      }
       const WorkInfo wi = cur.wi;
-      const int NQ = (wi.nqc + 15) & ~15;
+      const int NQ = (wi.nqc + QG - 1) & ~(QG - 1);
       const int N = P * NQ;
       const uint32_t b = wcount & 1, r = wcount >> 1;
       mbar_wait(&empty_q[b], (r & 1) ^ 1);
       mbar_wait(&empty_m[b], (r & 1) ^ 1);
       publish(b);
-      prev_nqc[b] = wi.nqc;
       const Meta mt = meta_at(metab + b * p.meta_bytes, QCP);
+      if (done) {  // end marker for the MMA and epilogue warps
+        if (tq == 0) mt.wi->ntiles = -1;
+        named_bar(2, 64);
+        mbar_arrive(&full_q[b]);
+        break;
+      }
+      prev_nqc[b] = wi.nqc;
       if (tq == 0) *mt.wi = wi;
 #pragma unroll
       for (int u = 0; u < 2; ++u) {
@@ -505,12 +574,14 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
       if (tq == 0) MV_TRACE(5, wcount);
       cur = nxt;
     }
-    // the last (up to) two items: wait until the epilogue is done with them, then publish
-    for (uint32_t e = wcount; e < wcount + 2; ++e) {
-      const uint32_t b = e & 1, r = e >> 1;
-      if (prev_nqc[b] == 0) continue;
-      mbar_wait(&empty_m[b], (r & 1) ^ 1);
-      publish(b);
+    // the last item (the end marker's step published the one before): wait until the epilogue is
+    // done with it, then publish
+    {
+      const uint32_t e = wcount + 1, b = e & 1, r = e >> 1;
+      if (prev_nqc[b] != 0) {
+        mbar_wait(&empty_m[b], (r & 1) ^ 1);
+        publish(b);
+      }
     }
   } else {
     // ------------------------------------------------------------------ epilogue (8 warps)
@@ -525,13 +596,14 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
     const int row = quarter * 32 + lane;
     const int et = threadIdx.x - 128;   // 0..255
     const uint32_t ltmask = (1u << lane) - 1;
-    uint32_t titer = 0, wcount = 0;
-    for (int i = 0; item(i) < nwork; ++i, ++wcount) {
+    uint32_t titer = 0;
+    for (uint32_t wcount = 0;; ++wcount) {
       const uint32_t b = wcount & 1;
       mbar_wait(&full_q[b], (wcount >> 1) & 1);
       const Meta mt = meta_at(metab + b * p.meta_bytes, QCP);
       const WorkInfo wi = *mt.wi;
-      const int NQ = (wi.nqc + 15) & ~15;
+      if (wi.ntiles < 0) break;  // the gatherer's end marker
+      const int NQ = (wi.nqc + QG - 1) & ~(QG - 1);
       const uint32_t s_qnf = smem_u32(mt.qnf), s_thf = smem_u32(mt.thf), s_qs = smem_u32(mt.qs),
                      s_qaf = smem_u32(mt.qaf), s_cnt = smem_u32(mt.cnt), s_base = smem_u32(mt.base);
       for (int t = 0; t < wi.ntiles; ++t, ++titer) {
@@ -797,7 +869,8 @@ static bool tc_scan_layout(int type, int dpad, int qc, int ns, bool ids, TcScanP
   p.side_bytes = ids ? 3072 : 1792;
   p.nts = std::max(4, std::min(kMaxNTS, ns / p.nchunks + p.nacc + 1));
   p.off_bar = p.off_side + p.nts * p.side_bytes;
-  p.smem_total = p.off_bar + (2 * ns + 6 + 2 * kMaxAcc + 2 * kMaxNTS) * 8 + 16 + 1024;  // + 1 KB alignment slack
+  p.smem_total = p.off_bar + (2 * ns + 6 + 2 * kMaxAcc + 2 * kMaxNTS + 2 * kRing) * 8 + 4 * kRing + 16 +
+                 1024;  // + 1 KB alignment slack
   return p.smem_total <= 227 * 1024;
 }
 

@@ -682,11 +682,10 @@ static mv_status search_chunk(mv_index* ix, const float* q, int64_t nq, int32_t 
   CK(s.alloc(&b.wcount, nv));
   CK(s.alloc(&b.woff, nv + 1));
   CK(s.alloc(&b.witems, (size_t)(nv + nent / qchunk_min + 1)));
-  CK(s.alloc(&b.witems_unsorted, (size_t)(nv + nent / qchunk_min + 1)));
   CK(s.alloc(&b.qtot, (size_t)(2 * (nq + 1))));
   CK(s.alloc(&b.poff, (size_t)nent));
   CK(s.alloc(&b.pcnt, (size_t)nent));
-  CK(s.alloc(&b.counter, 1));
+  CK(s.alloc(&b.counter, 2));
   CK(s.alloc(&b.whist, (size_t)kPlanCostBins));
   CK(s.alloc(&b.bsum, (size_t)(2 * kPlanMaxBlocks)));
   PlanArgs pa;
@@ -764,6 +763,7 @@ static mv_status search_chunk(mv_index* ix, const float* q, int64_t nq, int32_t 
   tp.rowcap = split ? (int)pa.capA : 0x7fffffff;
   tp.wbeg = nullptr;
   tp.nwitems = b.woff + nlist;
+  tp.counter = b.counter;
   CK(launch_scan_tc(ix->xm, tp, st));
   prof_mark(ix, st);
   if (split) {
@@ -778,6 +778,7 @@ static mv_status search_chunk(mv_index* ix, const float* q, int64_t nq, int32_t 
     tp.rowcap = 0x7fffffff;
     tp.wbeg = b.woff + nlist;
     tp.nwitems = b.woff + 2 * nlist;
+    tp.counter = b.counter + 1;
     CK(launch_scan_tc(ix->xm, tp, st));
   } else {
     prof_mark(ix, st);
@@ -887,6 +888,49 @@ mv_status mv_search_with_probes(mv_index* ix, const float* queries, int64_t nq, 
                                 int64_t* out_ids, void* stream) {
   if (probes == nullptr && nq > 0) return fail(MV_EINVAL, "probes is NULL");
   return search_impl(ix, queries, nq, k, nprobe, probes, bitset, nbits, distances, out_ids, stream);
+}
+
+mv_status mv_attr_bitset(const int64_t* ids, const int64_t* attr, int64_t n, int64_t lo, int64_t hi,
+                         uint8_t* bitset, int64_t nbits, void* stream) {
+  if (n < 0 || nbits < 0) return fail(MV_EINVAL, "n and nbits must be >= 0");
+  if ((n > 0 && (!ids || !attr)) || (nbits > 0 && !bitset)) return fail(MV_EINVAL, "null argument");
+  if (nbits == 0) return MV_OK;
+  if (reinterpret_cast<uintptr_t>(bitset) % 4) return fail(MV_EINVAL, "bitset must be 4-byte aligned");
+  if (is_host_ptr(ids) || is_host_ptr(attr) || is_host_ptr(bitset)) return fail(MV_EINVAL, "device pointers only");
+  cudaPointerAttributes at;
+  if (cudaPointerGetAttributes(&at, bitset) != cudaSuccess) return from_cuda(cudaGetLastError(), "bitset");
+  DeviceGuard g(at.device);
+  CK(launch_attr_bitset(ids, attr, n, lo, hi, bitset, nbits, reinterpret_cast<cudaStream_t>(stream)));
+  return MV_OK;
+}
+
+mv_status mv_fuse_rows(const float* const* parts, const int32_t* dims, const float* weights, int32_t m, int64_t n,
+                       float* out, void* stream) {
+  if (m < 1 || m > kMaxFuse) return fail(MV_EINVAL, "m must be in [1, %d]", kMaxFuse);
+  if (n < 0) return fail(MV_EINVAL, "n must be >= 0");
+  if (!parts || !dims || (n > 0 && !out)) return fail(MV_EINVAL, "null argument");
+  FuseArgs a{};
+  a.m = m;
+  int64_t tot = 0;
+  for (int i = 0; i < m; ++i) {
+    if (dims[i] < 1 || (n > 0 && !parts[i])) return fail(MV_EINVAL, "part %d: bad dims or null pointer", i);
+    a.part[i] = parts[i];
+    a.dim[i] = dims[i];
+    a.off[i] = (int)tot;
+    a.w[i] = weights ? weights[i] : 1.0f;
+    tot += dims[i];
+  }
+  if (tot > (1 << 20)) return fail(MV_EINVAL, "fused dimension too large");
+  a.dtot = (int)tot;
+  if (n == 0) return MV_OK;
+  if (is_host_ptr(out)) return fail(MV_EINVAL, "device pointers only");
+  for (int i = 0; i < m; ++i)
+    if (is_host_ptr(parts[i])) return fail(MV_EINVAL, "device pointers only");
+  cudaPointerAttributes at;
+  if (cudaPointerGetAttributes(&at, out) != cudaSuccess) return from_cuda(cudaGetLastError(), "out");
+  DeviceGuard g(at.device);
+  CK(launch_fuse_rows(a, n, out, reinterpret_cast<cudaStream_t>(stream)));
+  return MV_OK;
 }
 
 mv_status mv_merge_topk(mv_metric metric, const float* dists, const int64_t* ids, int32_t nsrc, int64_t nq, int32_t k,

@@ -242,16 +242,17 @@ struct Bucketing {
   int32_t* bq;       // nq*npb (x2 with seeding)  pair ids grouped by list
   int32_t* wcount;   // nlist      work items per list
   int32_t* woff;     // nlist+1
-  int2* witems;      // <= nlist + nq*npb   (list, first bucket position), longest first
-  int2* witems_unsorted;
+  int2* witems;      // <= nlist + nq*npb   (list | kItemMulti, first bucket position), longest first
   int64_t* qtot;     // nq+1       per-query candidate capacity, then exclusive scan
   int64_t* poff;     // nq*npb (x2 with seeding: phase-A entries at nq*npb + p)  region offset per pair
   int32_t* pcnt;     // nq*npb (x2 with seeding)  candidates written per pair
-  int32_t* counter;  // 1          persistent scan work counter
+  int32_t* counter;  // 2          scan work-item counters (phase A, phase B)
   int32_t* whist;    // kPlanCostBins  work-item cost histogram, then its exclusive scan
   int64_t* bsum;     // 2 x kPlanMaxBlocks  per-block partial sums of the grid-wide scans
 };
 constexpr int kPlanCostBins = 8192;
+// work-item flag (bit 30 of the virtual list): the list has several items (sibling reads share L2)
+constexpr int kItemMulti = 1 << 30;
 constexpr int kPlanMaxBlocks = 1024;
 // a4 in one cooperative launch (k_bucket.cu).  With the seeding split the pairs of query q with
 // probe rank < ra[q] form a first phase (virtual lists 0..nlist-1, work items first) and the
@@ -274,6 +275,18 @@ cudaError_t launch_plan(const PlanArgs& a, cudaStream_t st);
 // single-CTA exclusive scans (the add path): out[0..n], out[n] = total
 cudaError_t launch_scan_i32(const int32_t* in, int n, int32_t* out, cudaStream_t st);   // out[n+1]
 cudaError_t launch_scan_i64(const int64_t* in, int64_t n, int64_t* out, cudaStream_t st);  // out[n+1]
+
+// k_filter.cu: strategy E's range bitmap and vector fusion
+cudaError_t launch_attr_bitset(const int64_t* ids, const int64_t* attr, int64_t n, int64_t lo, int64_t hi,
+                               uint8_t* bitset, int64_t nbits, cudaStream_t st);
+constexpr int kMaxFuse = 16;  // vectors per entity (mv_fuse_rows)
+struct FuseArgs {
+  const float* part[kMaxFuse];
+  int dim[kMaxFuse], off[kMaxFuse];
+  float w[kMaxFuse];
+  int m, dtot;
+};
+cudaError_t launch_fuse_rows(const FuseArgs& a, int64_t n, float* out, cudaStream_t st);
 
 // k_scan_tc.cu (tcgen05 path): a filter-and-emit scan run in two phases
 struct TcScanParams {
@@ -302,6 +315,7 @@ struct TcScanParams {
   const int2* witems;
   const int32_t* wbeg;     // device: first work item of this launch (nullable = 0)
   const int32_t* nwitems;  // device: one past the last work item of this launch
+  int32_t* counter;        // device: work items taken so far in this launch (zeroed by k_plan)
   const int64_t* poff;     // per pair: output region (capacity = the list length)
   int32_t* pcnt;           // per pair: keys emitted
   uint64_t* part;

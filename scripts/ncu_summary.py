@@ -18,7 +18,10 @@ scale = {"ns": 1e-3, "nsecond": 1e-3, "us": 1.0, "usecond": 1.0, "ms": 1e3, "mse
          "byte": 1e-6, "Kbyte": 1e-3, "Mbyte": 1.0, "Gbyte": 1e3, "%": 1.0}
 for r in rows[1:]:
     d = launch.setdefault(int(r[idi]), {"name": r[ki].split("(")[0].replace("void ", "").replace("mv::", "")})
-    d[r[mi]] = float(r[vi].replace(",", "")) * scale.get(r[ui], 1.0)
+    try:
+        d[r[mi]] = float(r[vi].replace(",", "")) * scale.get(r[ui], 1.0)
+    except ValueError:  # "n/a" (a metric this chip does not expose)
+        pass
 tot = sum(d.get("gpu__time_duration.sum", 0.0) for d in launch.values())
 print(f"{len(launch)} launches, {tot:.1f} us of device time (cold-cache, serialised)")
 print(f"{'#':>3} {'kernel':<34} {'us':>9} {'share':>6} {'DRAM rd MB':>11} {'DRAM wr MB':>11} {'tensor %':>9}")
