@@ -169,6 +169,25 @@ MV_API mv_status mv_search_with_probes(mv_index* index, const float* queries, in
 MV_API mv_status mv_merge_topk(mv_metric metric, const float* dists, const int64_t* ids, int32_t nsrc, int64_t nq,
                         int32_t k, float* out_d, int64_t* out_i, void* stream);
 
+/* Strategy E's per-partition bitmap (§4.1 with strategy B's
+ * bitmap): writes the whole bitset -- ceil(nbits/32) 32-bit words, LSB-first,
+ * bit = 1 means excluded (the polarity mv_search takes) -- with bit ids[i] set for every i < n
+ * whose attr[i] is outside [lo, hi].  ids / attr: n int64 each (the partition's entity ids and
+ * attribute values, device); bitset: device, 4-byte aligned, caller-owned; ids outside
+ * [0, nbits) are ignored (size nbits above the largest id).  Asynchronous on `stream`.
+ * MV_EINVAL for n < 0, nbits < 0, lo > hi is allowed (everything excluded), null pointers with n > 0. */
+MV_API mv_status mv_attr_bitset(const int64_t* ids, const int64_t* attr, int64_t n, int64_t lo, int64_t hi,
+                                uint8_t* bitset, int64_t nbits, void* stream);
+
+/* Vector fusion (§4.2): out[r] = [w_0 parts[0][r] | ... |
+ * w_{m-1} parts[m-1][r]] for r < n -- the concatenated entity vectors (weights 1) or the
+ * aggregated query (weights = the weighted-sum aggregation's w_i), so that one MV_IP search
+ * returns the top-k by sum_i w_i (q.v_i . e.v_i).  parts: host array of m device pointers, part i
+ * row-major [n][dims[i]] fp32; dims, weights: host arrays of m (weights NULL = all 1);
+ * out: device [n][sum dims] fp32.  1 <= m <= 16.  Asynchronous on `stream`. */
+MV_API mv_status mv_fuse_rows(const float* const* parts, const int32_t* dims, const float* weights, int32_t m,
+                              int64_t n, float* out, void* stream);
+
 /* Number of stored vectors. */
 MV_API int64_t mv_index_ntotal(const mv_index* index);
 
