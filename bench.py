@@ -118,6 +118,7 @@ def build_sharded(cfg, device, shard, nshard, Index, chunk=1 << 24, ngt=1000, sp
     ntr = min(cfg["n"], 64 * cfg["nlist"])
     Xtr = G.sift_base(ntr, d=cfg["d"], device=device, spec=spec)
     C = kmeans(Xtr, cfg["nlist"], iters=10)
+    time_kmeans(Xtr, cfg)
     vmin = Xtr.min(0).values.contiguous()
     vdiff = (Xtr.max(0).values - vmin).contiguous()
     del Xtr
@@ -181,8 +182,31 @@ def make_data(cfg, device):
         X = G.deep_base(n, d=d, device=device)
         Q = G.deep_queries(cfg["nq"], d=d, device=device)
     C = kmeans(X, cfg["nlist"], iters=10, spherical=cfg["data"] == "deep")
+    if device.type == "cuda":
+        time_kmeans(X, cfg)
     bs = G.mod_bitset(n, cfg["bitset"], device=device) if cfg["bitset"] else None
     return X, Q, C, bs
+
+
+def time_kmeans(X, cfg, iters=10):
+    """the same k-means training (n_train = 64 nlist seeded rows, 10 Lloyd
+    iterations) on the device through mv_kmeans, timed (the index keeps mvgen's data-prep centroids,
+    so the search numbers stay comparable across rounds)."""
+    import mvgen as G
+    from paper_conf_sigmod_wangygjxlwglxyy21_b200 import kmeans as mv_kmeans
+    n = X.shape[0]
+    ntr = min(n, 64 * cfg["nlist"])
+    order = torch.argsort(G.hash64(G.SEED_KMEANS, 1, torch.arange(n, dtype=torch.int64, device=X.device)))
+    xt = X[order[:ntr]].float().contiguous()
+    mv_kmeans(xt, cfg["nlist"], niter=1, metric=cfg["metric"], spherical=cfg["data"] == "deep")  # warm-up
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    mv_kmeans(xt, cfg["nlist"], niter=iters, metric=cfg["metric"], spherical=cfg["data"] == "deep")
+    torch.cuda.synchronize()
+    dt = time.perf_counter() - t0
+    BUILD["kmeans"] = {"rows": ntr, "nlist": cfg["nlist"], "iters": iters, "seconds": dt,
+                       "row_iters_per_s": ntr * iters / dt,
+                       "note": "mv_kmeans: tensor-core assignment (the add path's coarse step) + fp64 centroid means"}
 
 
 def sq8_params(cfg, X):
@@ -617,7 +641,8 @@ def main():
             "build": ({"vectors_per_s": BUILD["vectors"] / BUILD["seconds"], "vectors": BUILD["vectors"],
                        "seconds": BUILD["seconds"], "add_calls": BUILD["calls"],
                        "note": "mv_index_add (tensor-core assignment, SQ8 encode, list-major scatter, id ranks); "
-                               "each call re-lays out the whole index (O(n) copy)"}
+                               "each call re-lays out the whole index (O(n) copy)",
+                       "kmeans": BUILD.get("kmeans")}
                       if BUILD.get("seconds") else None),
             "clocks": clocks,
             "cpu_baseline": cpu,

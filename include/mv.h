@@ -93,7 +93,9 @@ MV_API mv_status mv_index_create(int32_t d, mv_metric metric, mv_type type, int3
  * the scratch budget.  Names: "seeding" (0/1), "need" (seeding sample, candidates), "capa" (rows
  * per list of the sample), "sq8_qc" / "flat_qc" (queries per scan work item), "coarse_nqb",
  * "coarse_cs", "coarse_epi", "coarse_nacc" (coarse GEMM shape), "large_k_select" (k > 256: 0 = the
- * staged radix select, 1 = the sample-threshold select), "big_ctas" / "big_cap" (the staged
+ * streaming select when the search seeds (k <= 4096; the staged radix select for the rest and as
+ * its fallback), 1 = the sample-threshold select, 2 = the staged radix select only, 3 = the
+ * streaming select for the seeding bound too), "big_ctas" / "big_cap" (the staged
  * select's first launch: CTAs per SM, 1..4, and candidates staged per query; queries past it are
  * redone with all of shared memory), "workspace_bytes" (per-search
  * scratch budget: larger batches run as several query chunks; 0 = half of the device memory that was
@@ -168,6 +170,17 @@ MV_API mv_status mv_search_with_probes(mv_index* index, const float* queries, in
  * pointers (or host; staged).  Asynchronous on `stream` for device pointers. */
 MV_API mv_status mv_merge_topk(mv_metric metric, const float* dists, const int64_t* ids, int32_t nsrc, int64_t nq,
                         int32_t k, float* out_d, int64_t* out_i, void* stream);
+
+/* Lloyd k-means training of the coarse codebook on the device (PAPER.md:503-514
+ * §3.1: the buckets are K-means clusters).  x: device [n][d] fp32 training rows; centroids: device
+ * [nlist][d] fp32 -- in: the initial centroids (e.g. nlist seeded training rows), out: after niter
+ * iterations.  Each iteration assigns every row to its closest centroid under `metric` with the
+ * index's tensor-core coarse step (the assignment mv_index_add makes: exact to the oracle up to
+ * ties) and sets each centroid to the mean of its rows (fp64 sums, one rounding to fp32; spherical
+ * != 0 normalises it); a centroid without rows keeps its position.  Synchronous; the scratch comes
+ * from cudaMallocAsync.  MV_EINVAL: null pointers, nlist < 1, n < nlist, niter < 0, host pointers. */
+MV_API mv_status mv_kmeans(const float* x, int64_t n, int32_t d, mv_metric metric, int32_t nlist, int32_t niter,
+                           int32_t spherical, float* centroids, int32_t device, void* stream);
 
 /* Strategy E's per-partition bitmap (§4.1 with strategy B's
  * bitmap): writes the whole bitset -- ceil(nbits/32) 32-bit words, LSB-first,

@@ -48,6 +48,7 @@ _SIGS = {
     "mv_search_probes": (C.c_int, [_P, _P, C.c_int64, C.c_int32, _P, _P]),
     "mv_search_with_probes": (C.c_int, [_P, _P, C.c_int64, C.c_int32, C.c_int32, _P, _P, C.c_int64, _P, _P, _P]),
     "mv_merge_topk": (C.c_int, [C.c_int, _P, _P, C.c_int32, C.c_int64, C.c_int32, _P, _P, _P]),
+    "mv_kmeans": (C.c_int, [_P, C.c_int64, C.c_int32, C.c_int, C.c_int32, C.c_int32, C.c_int32, _P, C.c_int32, _P]),
     "mv_attr_bitset": (C.c_int, [_P, _P, C.c_int64, C.c_int64, C.c_int64, _P, C.c_int64, _P]),
     "mv_fuse_rows": (C.c_int, [C.POINTER(C.c_void_p), C.POINTER(C.c_int32), C.POINTER(C.c_float), C.c_int32,
                                C.c_int64, _P, _P]),

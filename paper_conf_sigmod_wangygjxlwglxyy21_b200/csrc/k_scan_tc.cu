@@ -327,11 +327,16 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
           const int row0 = (int)(wi.lstart + t * 128);
           const uint32_t ts = tcount % NTS, tr = tcount / NTS;
           mbar_wait(&empty_t[ts], (tr & 1) ^ 1);
+#ifdef MV_EXP_NOSIDE  // timing experiment only (wrong results): no side data
+          mbar_arrive(&full_t[ts]);
+          (void)side_tx;
+#else
           mbar_expect_tx(&full_t[ts], side_tx);
           uint8_t* sd = side + ts * SIDEB;
           bulk_g2s(sd + kSideRank, p.rank + (row0 & ~3), 528, &full_t[ts]);
           if (use_norms) bulk_g2s(sd, p.norms + (row0 & ~1), 1040, &full_t[ts]);
           if (use_ids) bulk_g2s(sd + kSideIds, p.ids + (row0 & ~1), 1040, &full_t[ts]);
+#endif
           for (int c = 0; c < nchunks; ++c, ++it) {
             const uint32_t s = it % nstage, r = it / nstage;
             mbar_wait(&empty_x[s], (r & 1) ^ 1);
@@ -384,6 +389,12 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
             const uint32_t xb = smem_u32(Xs + s * 128 * ATOM);
             const uint32_t qb = qbase + c * N * ATOM;
 #pragma unroll
+#ifdef MV_EXP_NOMMA  // timing experiment only (wrong results): stages released without MMAs
+            (void)xb; (void)qb; (void)dcol; (void)idesc;
+            mbar_arrive(&empty_x[s]);
+          }
+          mbar_arrive(&tfull[a]);
+#else
             for (int ks = 0; ks < ATOM / 32; ++ks) {
               const uint64_t ad = kmajor_desc(xb + ks * 32, ATOM);
               const uint64_t bd = kmajor_desc(qb + ks * 32, ATOM);
@@ -393,6 +404,7 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
             mma_commit(&empty_x[s]);
           }
           mma_commit(&tfull[a]);
+#endif
           MV_TRACE(3, titer);
         }
         mma_commit(&empty_q[b]);
@@ -565,7 +577,11 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
         const uint8_t* src = p.qplanes + prow * rowbytes;
         for (int e = lane; e < ppr; e += 32) {
           const int c = e / PIECES, pc = e % PIECES;  // PIECES is a power of two
+#ifndef MV_EXP_NOGATHER  // timing experiment only (wrong results): no query-plane copies
           cp_async16(Qb + c * N * ATOM + swz_off(pl * NQ + i, pc, ATOM), src + e * 16);
+#else
+          (void)src; (void)c; (void)pc;
+#endif
         }
       }
       cp_async_wait_all();
@@ -614,17 +630,28 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
         const int row0 = (int)(wi.lstart + t * 128);
         mbar_wait(&full_t[ts], (titer / NTS) & 1);
         const uint8_t* sd = side + ts * SIDEB;
+#ifdef MV_EXP_NOSIDE
+        const uint32_t rk = 0;
+        const bool valid = vrow < wi.len;
+        const double xn = 0.0;
+        (void)sd;
+#else
         const uint32_t rk = reinterpret_cast<const uint32_t*>(sd + kSideRank)[(row0 & 3) + row];
         bool valid = vrow < wi.len;
         if (valid && use_ids)
           valid = !bit_excluded(p.bitset, p.nbits, reinterpret_cast<const int64_t*>(sd + kSideIds)[(row0 & 1) + row]);
         const double xn = use_norms ? reinterpret_cast<const double*>(sd)[(row0 & 1) + row] : 0.0;
+#endif
         const float xnf = (float)xn;
         mbar_wait(&tfull[a], (titer / NACC) & 1);
         if (et == 0) MV_TRACE(6, titer);
         tc_fence_after();
         const uint32_t tbase = tmem + a * p.ncol + ((uint32_t)(quarter * 32) << 16);
+#ifdef MV_EXP_NOEPI  // timing experiment only (wrong results): no epilogue work
+        for (int qc = 0; qc < 0; qc += W) {
+#else
         for (int qc = 0; qc < NQ; qc += W) {
+#endif
           uint32_t r[PMAX][W];
           tmem_ld_w<W>(tbase + qc, r[0]);
           if (TYPE == MV_IVF_SQ8 || P == 2) tmem_ld_w<W>(tbase + NQ + qc, r[1]);

@@ -324,7 +324,7 @@ __global__ void __launch_bounds__(NT, 2048 / NT) k_final_big(const int64_t* __re
                                                            float* out_d, int64_t* out_i, int cap,
                                                            const int32_t* __restrict__ nuse, uint64_t* tau_out,
                                                            uint8_t* over, const int* __restrict__ gate,
-                                                           const uint8_t* only) {
+                                                           const uint8_t* only, uint64_t* kmin) {
   if (gate && *gate == 0) return;
   // only: the queries to do (k_final_sample's redo flags, or the flags of a smaller-stage launch --
   // then the same array as over: this CTA reads its flag before rewriting it)
@@ -415,6 +415,7 @@ __global__ void __launch_bounds__(NT, 2048 / NT) k_final_big(const int64_t* __re
     __syncthreads();
     mn = s_mm[0];
     mx = s_mm[1];
+    if (tau_out && kmin && tid == 0) kmin[q] = mn;  // the streaming final select's lower bin edge
     // Fast path: one counting pass over kBucketBins equal-width buckets of [mn, mx] and a scan
     // locate the bucket b* holding the k-th key.  Seeding: the bound is b*'s upper edge (or, when
     // b* holds more than 64 keys, the upper edge of the sub-bucket of a second counting pass over
@@ -828,14 +829,279 @@ __global__ void __launch_bounds__(kBigThreads) k_final_sample(const int64_t* __r
   }
 }
 
+// 256 < k <= 4096 without staging the candidates: one CTA per query streams the query's keys from
+// global memory (every pair's region read by one warp, coalesced) -- a few tens of KB of shared
+// memory per CTA, so several CTAs per SM keep their loads in flight (k_final_big stages every
+// candidate in shared memory first: one CTA per SM at configs[3]'s sizes, load and compute phases
+// in series).  Keys are binned by their distance key into kBucketBins equal-width bins over
+// [lo32, hi32] (keys outside go to the end bins):
+//   TAU (the seeding select): lo/hi = the keys' min/max distance keys (pass 0); a counting pass and
+//     a scan locate the bin b* of the k-th key; the bound is b*'s upper edge (with a second counting
+//     pass over b*'s sub-bins when it holds > 64 keys) with every id rank: >= k candidates lie at or
+//     below it.  kmin[q] = the smallest key (the final select's lower bin edge).
+//   final: lo = kmin[q], hi = khi[q] (the seeding bound: phase B emits nothing above it); a
+//     counting pass locates b*; a second pass gathers the keys of bins <= b* (the top-k and b*'s
+//     rest, <= cap keys) into shared memory, a bucket sort (bitonic fallback) orders them, the first
+//     k are the answer.  A query whose gathered keys exceed cap is flagged in redo[] for the staged
+//     select.
+template <int NT, bool TAU>
+__global__ void __launch_bounds__(NT) k_select_stream(const int64_t* __restrict__ poff, const int32_t* __restrict__ pcnt,
+                                                      const uint64_t* __restrict__ part, int64_t nq, int npb, int k,
+                                                      int metric, const int64_t* __restrict__ sorted_ids, float* out_d,
+                                                      int64_t* out_i, int cap, const int32_t* __restrict__ nuse,
+                                                      uint64_t* tau_out, uint64_t* kmin, const uint64_t* __restrict__ khi,
+                                                      uint8_t* redo, const int* __restrict__ gate) {
+  if (gate && *gate == 0) return;
+  extern __shared__ __align__(16) uint8_t smem[];
+  uint32_t* hist = reinterpret_cast<uint32_t*>(smem);                 // kBucketBins
+  int* misc = reinterpret_cast<int*>(hist + kBucketBins);             // 64
+  uint64_t* s_mm = reinterpret_cast<uint64_t*>(misc + 64);            // 2
+  int64_t* s_po = reinterpret_cast<int64_t*>(s_mm + 2);               // npb: the non-empty pairs' regions
+  int32_t* s_pre = reinterpret_cast<int32_t*>(s_po + npb);            // npb + 33: their key prefix, then padding
+  uint64_t* win = reinterpret_cast<uint64_t*>(s_pre + ((npb + 34) & ~1));  // cap (final)
+  uint64_t* tmp = win + (TAU ? 0 : cap);                              // cap (final)
+  constexpr int NW = NT / 32, U = 4;
+  const int64_t q = blockIdx.x;
+  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  const int64_t* po = poff + q * npb;
+  const int32_t* pc = pcnt + q * npb;
+  const int nu = nuse ? nuse[q] : npb;
+  for (int i = tid; i < kBucketBins; i += NT) hist[i] = 0;
+  if (wid == 0) {  // the non-empty pairs, compacted, and the prefix of their key counts
+    int run = 0, ne = 0;
+    for (int j0 = 0; j0 < nu; j0 += 32) {
+      const int j = j0 + lane;
+      const int c = j < nu ? pc[j] : 0;
+      int incl = c;
+      for (int o = 1; o < 32; o <<= 1) {
+        const int v = __shfl_up_sync(MV_FULL, incl, o);
+        if (lane >= o) incl += v;
+      }
+      const uint32_t nz = __ballot_sync(MV_FULL, c > 0);
+      if (c > 0) {
+        const int ci = ne + __popc(nz & ((1u << lane) - 1));
+        s_pre[ci] = run + incl - c;
+        s_po[ci] = po[j];
+      }
+      run += __shfl_sync(MV_FULL, incl, 31);
+      ne += __popc(nz);
+    }
+    s_pre[ne + lane] = lane ? 0x7fffffff : run;  // s_pre[ne] = the total, then padding
+    if (lane == 0) {
+      misc[50] = ne;
+      s_mm[0] = MV_KEY_PAD;
+      s_mm[1] = 0;
+      misc[48] = 0;
+      misc[49] = 0;
+    }
+    s_pre[ne + 32] = 0x7fffffff;
+  }
+  __syncthreads();
+  const int nne = misc[50];
+  const int T = s_pre[nne];
+  // every key of the query: warp w takes a contiguous slice of the flattened (pair, key) index, U
+  // windows of 32 keys per round (independent loads in flight); a window's pair starts are found
+  // by one shared load per lane and an OR-reduce (the pair starts strictly increase: empty pairs
+  // were dropped).  f(x, valid) is called by all 32 lanes together.
+  const int per = ((T + NW - 1) / NW + 31) & ~31;
+  auto each = [&](auto&& f) {
+    const int b0 = min(T, wid * per), b1 = min(T, b0 + per);
+    int c0 = 0;  // pair starts below the window
+    {
+      int lo = 0, hi = nne;  // the first m with s_pre[m] >= b0
+      while (lo < hi) {
+        const int mid = (lo + hi) >> 1;
+        if (s_pre[mid] < b0) lo = mid + 1; else hi = mid;
+      }
+      c0 = lo;
+    }
+    const uint32_t upto = lane == 31 ? 0xffffffffu : (2u << lane) - 1;
+    for (int i0 = b0; i0 < b1; i0 += 32 * U) {
+      uint64_t x[U];
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        const int w0 = i0 + 32 * u;
+        const uint32_t off = (uint32_t)(s_pre[min(c0 + lane, nne + 32)] - w0);
+        const uint32_t M = __reduce_or_sync(MV_FULL, off < 32u ? 1u << off : 0u);
+        const int j = c0 - 1 + __popc(M & upto);
+        c0 += __popc(M);
+        const int i = w0 + lane;
+        x[u] = i < b1 ? __ldg(part + s_po[j] + (i - s_pre[j])) : MV_KEY_PAD;
+      }
+#pragma unroll
+      for (int u = 0; u < U; ++u) f(x[u], x[u] != MV_KEY_PAD);
+    }
+  };
+  uint32_t lo32, hi32;
+  if (TAU) {
+    uint64_t mn = MV_KEY_PAD, mx = 0;
+    each([&](uint64_t x, bool v) {
+      if (v) {
+        mn = umin64(mn, x);
+        mx = umax64(mx, x);
+      }
+    });
+    for (int o = 16; o > 0; o >>= 1) {
+      mn = umin64(mn, shfl_xor64(mn, o));
+      mx = umax64(mx, shfl_xor64(mx, o));
+    }
+    if (lane == 0) {
+      atomicMin(reinterpret_cast<unsigned long long*>(s_mm), (unsigned long long)mn);
+      atomicMax(reinterpret_cast<unsigned long long*>(s_mm + 1), (unsigned long long)mx);
+    }
+    __syncthreads();
+    lo32 = (uint32_t)(s_mm[0] >> 32);
+    hi32 = (uint32_t)(s_mm[1] >> 32);
+    if (s_mm[0] == MV_KEY_PAD) lo32 = hi32 = 0;
+  } else {
+    lo32 = (uint32_t)(kmin[q] >> 32);
+    hi32 = max(lo32, (uint32_t)(khi[q] >> 32));
+  }
+  const uint32_t span = hi32 - lo32;
+  const int sh = span ? max(0, 32 - __clz((int)span) - 11) : 0;  // (d - lo32) >> sh < 2048
+  auto bin = [&](uint64_t x) {
+    const uint32_t d = (uint32_t)(x >> 32);
+    return d <= lo32 ? 0 : (int)min((uint32_t)(kBucketBins - 1), (d - lo32) >> sh);
+  };
+  {
+    int cnt = 0;
+    each([&](uint64_t x, bool v) {
+      if (v) {
+        atomicAdd(hist + bin(x), 1u);
+        ++cnt;
+      }
+    });
+    for (int o = 16; o > 0; o >>= 1) cnt += __shfl_xor_sync(MV_FULL, cnt, o);
+    if (lane == 0) atomicAdd(misc + 49, cnt);
+  }
+  __syncthreads();
+  const int ntot = misc[49];
+  if (TAU) {
+    if (ntot < k) {  // fewer than k candidates: no bound (tau stays at padding), the whole key range
+      if (tid == 0 && kmin) kmin[q] = 0;
+      return;
+    }
+    if (tid == 0 && kmin) kmin[q] = s_mm[0];
+    block_scan_bins<NT>(hist, misc, k - 1);
+    const int bs = misc[40], st = misc[41], nb = misc[42];
+    // b*'s upper edge: the bins below b* hold < k keys, so the k-th key's distance is <= the edge
+    uint64_t dedge = (uint64_t)lo32 + (((uint64_t)bs + 1) << sh) - 1;
+    if (nb > 64 && sh > 0) {  // refine within b*: 2048 sub-bins of width 2^(sh - 11)
+      const int sh2 = max(0, sh - 11);
+      const uint32_t b0 = lo32 + ((uint32_t)bs << sh);
+      for (int i = tid; i < kBucketBins; i += NT) hist[i] = 0;
+      __syncthreads();
+      each([&](uint64_t x, bool v) {
+        if (v && bin(x) == bs) atomicAdd(hist + (int)((((uint32_t)(x >> 32)) - b0) >> sh2), 1u);
+      });
+      __syncthreads();
+      block_scan_bins<NT>(hist, misc, k - 1 - st);
+      dedge = (uint64_t)b0 + (((uint64_t)misc[40] + 1) << sh2) - 1;
+    }
+    if (tid == 0) tau_out[q] = umin64((dedge << 32) | 0xffffffffull, s_mm[1]);
+    return;
+  } else {
+    // winners: the keys of bins <= b* (every key when there are at most k)
+    int lim = kBucketBins, n = ntot;
+    if (ntot > k) {
+      block_scan_bins<NT>(hist, misc, k - 1);
+      lim = misc[40];
+      n = misc[41] + misc[42];
+    }
+    if (n > cap) {
+      if (tid == 0) redo[q] = 1;
+      return;
+    }
+    if (tid == 0) redo[q] = 0;
+    each([&](uint64_t x, bool v) {
+      const bool p = v && bin(x) <= lim;
+      const uint32_t bal = __ballot_sync(MV_FULL, p);
+      int base = 0;
+      if (lane == 0 && bal) base = atomicAdd(misc + 48, __popc(bal));
+      base = __shfl_sync(MV_FULL, base, 0);
+      if (p) win[base + __popc(bal & ((1u << lane) - 1))] = x;
+    });
+    __syncthreads();
+    const int ng = misc[48];
+    uint64_t mn = MV_KEY_PAD, mx = 0;
+    for (int i = tid; i < ng; i += NT) {
+      mn = umin64(mn, win[i]);
+      mx = umax64(mx, win[i]);
+    }
+    for (int o = 16; o > 0; o >>= 1) {
+      mn = umin64(mn, shfl_xor64(mn, o));
+      mx = umax64(mx, shfl_xor64(mx, o));
+    }
+    for (int i = tid; i < kBucketBins; i += NT) hist[i] = 0;
+    if (tid == 0) {
+      s_mm[0] = MV_KEY_PAD;
+      s_mm[1] = 0;
+    }
+    __syncthreads();
+    if (lane == 0) {
+      atomicMin(reinterpret_cast<unsigned long long*>(s_mm), (unsigned long long)mn);
+      atomicMax(reinterpret_cast<unsigned long long*>(s_mm + 1), (unsigned long long)mx);
+    }
+    __syncthreads();
+    if (ng > 1 && !block_bucket_sort<NT>(win, ng, s_mm[0], s_mm[1], hist, tmp, misc)) {
+      const int NK = next_pow2(max(ng, 2));
+      for (int i = ng + tid; i < NK; i += NT) win[i] = MV_KEY_PAD;
+      switch (NK / NT) {
+        case 1: block_sort_regs<1, NT>(win, NK); break;
+        case 2: block_sort_regs<2, NT>(win, NK); break;
+        case 4: block_sort_regs<4, NT>(win, NK); break;
+        case 8: block_sort_regs<8, NT>(win, NK); break;
+        default: block_sort_regs<0, NT>(win, NK); break;
+      }
+    }
+    __syncthreads();
+    for (int i = tid; i < k; i += NT) {
+      float dv;
+      int64_t iv;
+      if (i < ng) {
+        const uint64_t key = win[i];
+        dv = key_dist((uint32_t)(key >> 32), metric);
+        iv = sorted_ids[(uint32_t)(key & 0xffffffffu)];
+      } else {
+        dv = metric == MV_L2 ? __int_as_float(0x7f800000) : __int_as_float(0xff800000);
+        iv = -1;
+      }
+      out_d[q * k + i] = dv;
+      out_i[q * k + i] = iv;
+    }
+  }
+}
+
 static cudaError_t launch_big_select(const int64_t* poff, const int32_t* pcnt, const uint64_t* part, int64_t nq,
                                      int npb, int k, int metric, const int64_t* sorted_ids, float* out_d,
                                      int64_t* out_i, const int32_t* nuse, uint64_t* tau, int64_t tmax,
                                      uint8_t* over, const int* gate, BigSel bsel, cudaStream_t st) {
   cudaError_t e;
-  // over: 2 nq bytes -- [0, nq) queries past k_final_big's stage, [nq, 2 nq) k_final_sample's redo flags
+  // over: 2 nq bytes -- [0, nq) queries past k_final_big's stage, [nq, 2 nq) the redo flags of the
+  // first-choice select (streaming or sample-threshold)
   uint8_t* redo = over ? over + nq : nullptr;
-  if (redo && k <= 3072 && bsel.mode == 1) {
+  // streaming select: the final select by default (mode 0), the seeding select only as mode 3 (the
+  // staged select measured faster there: configs[3] 0.63 vs 0.72 ms)
+  if (k <= 4096 && (tau ? bsel.mode == 3 && bsel.kmin != nullptr : bsel.mode == 0 && bsel.kmin && bsel.khi && redo)) {
+    constexpr int NT = 512;
+    const size_t base = kBucketBins * 4 + 64 * 4 + 16 + (size_t)npb * 8 + (size_t)((npb + 34) & ~1) * 4;
+    if (tau) {
+      e = cudaFuncSetAttribute(k_select_stream<NT, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)base);
+      if (e != cudaSuccess) return e;
+      k_select_stream<NT, true><<<(unsigned)nq, NT, base, st>>>(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d,
+                                                               out_i, 0, nuse, tau, bsel.kmin, nullptr, nullptr, gate);
+      return cudaGetLastError();
+    }
+    // the top-k plus the k-th key's bin (tens of keys); win + tmp also hold the bitonic fallback's
+    // next_pow2(gathered) keys.  k = 2048: 52 KB per CTA, four CTAs per SM
+    const int cap = k + max(256, k / 4);
+    const size_t smem = base + (size_t)cap * 16;
+    e = cudaFuncSetAttribute(k_select_stream<NT, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    k_select_stream<NT, false><<<(unsigned)nq, NT, smem, st>>>(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d,
+                                                              out_i, cap, nuse, nullptr, bsel.kmin, bsel.khi, redo, gate);
+    if ((e = cudaGetLastError()) != cudaSuccess) return e;
+  } else if (redo && k <= 3072 && bsel.mode == 1) {
     const int wcap = 4 * kBigThreads;  // >= k + the threshold's slack for k <= 2048; less for larger k
     const size_t smem = (size_t)(wcap + next_pow2(max(k, 2))) * 8 + (size_t)(npb + 1) * 4 + 64;
     if ((e = cudaFuncSetAttribute(k_final_sample, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)) != cudaSuccess)
@@ -863,13 +1129,13 @@ static cudaError_t launch_big_select(const int64_t* poff, const int32_t* pcnt, c
           cudaSuccess)
         return e;
       k_final_big<1024><<<(unsigned)nq, 1024, smem, st>>>(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d,
-                                                          out_i, cap1, nuse, tau, over, gate, only);
+                                                          out_i, cap1, nuse, tau, over, gate, only, bsel.kmin);
     } else {
       if ((e = cudaFuncSetAttribute(k_final_big<512>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)) !=
           cudaSuccess)
         return e;
       k_final_big<512><<<(unsigned)nq, 512, smem, st>>>(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d,
-                                                        out_i, cap1, nuse, tau, over, gate, only);
+                                                        out_i, cap1, nuse, tau, over, gate, only, bsel.kmin);
     }
     if (want <= cap1) return cudaGetLastError();
     only = over;  // the next launch redoes the flagged queries alone
@@ -881,7 +1147,7 @@ static cudaError_t launch_big_select(const int64_t* poff, const int32_t* pcnt, c
     e = cudaFuncSetAttribute(k_final_big<1024>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     k_final_big<1024><<<(unsigned)nq, 1024, smem, st>>>(poff, pcnt, part, nq, npb, k, metric, sorted_ids, out_d,
-                                                        out_i, cap, nuse, tau, over, gate, only);
+                                                        out_i, cap, nuse, tau, over, gate, only, bsel.kmin);
     if (want <= cap) return cudaGetLastError();
   } else {
     over = nullptr;

@@ -335,7 +335,7 @@ mv_status mv_index_set_option(mv_index* ix, const char* name, int64_t value) {
   else if (n == "coarse_nacc") o.coarse_nacc = (int)std::min<int64_t>(value, 4);
   else if (n == "workspace_bytes") o.workspace = value;
   else if (n == "scan_trace") o.scan_trace = value;  // development builds only (-DMV_SCAN_TRACE)
-  else if (n == "large_k_select") o.large_k_select = value != 0;
+  else if (n == "large_k_select") o.large_k_select = (int)std::min<int64_t>(std::max<int64_t>(value, 0), 3);
   else if (n == "big_cap") o.big_cap = std::max<int64_t>(value, 0);
   else if (n == "big_ctas") o.big_ctas = (int)std::min<int64_t>(std::max<int64_t>(value, 0), 4);
   else return fail(MV_EINVAL, "unknown option '%s'", name);
@@ -726,7 +726,12 @@ static mv_status search_chunk(mv_index* ix, const float* q, int64_t nq, int32_t 
   int64_t cap = nq * tmax;
   if (split) cap += nq * std::min<int64_t>(tmax, pa.need + pa.capA);
   uint8_t* over = nullptr;
+  uint64_t* kmin = nullptr;  // k > 256 with seeding: each query's smallest phase-A key (streaming select)
   if (k > 256) CK(s.alloc(&over, (size_t)2 * nq));
+  if (k > 256 && split) {
+    CK(s.alloc(&kmin, (size_t)nq));
+    CK(cudaMemsetAsync(kmin, 0, sizeof(uint64_t) * nq, st));  // (a query the seeding select skips: bins from 0)
+  }
   uint64_t* part;
   CK(s.alloc(&part, (size_t)max64(cap, 1)));
   // a5/a6 on the tensor cores
@@ -770,7 +775,9 @@ static mv_status search_chunk(mv_index* ix, const float* q, int64_t nq, int32_t 
     // ... tau_q = k-th best key of phase A (phase A emits < need + capA candidates per query) ...
     CK(launch_tau_select(b.poff + npairs, b.pcnt + npairs, part, nq, npb, ra, k, tau,
                          std::min<int64_t>(tmax, pa.need + pa.capA), over, nullptr,
-                         BigSel{ix->opt.large_k_select, ix->opt.big_ctas, ix->opt.big_cap, std::min<int64_t>(tmax, pa.need)}, st));
+                         BigSel{ix->opt.large_k_select, ix->opt.big_ctas, ix->opt.big_cap, std::min<int64_t>(tmax, pa.need),
+                                kmin, nullptr},
+                         st));
     prof_mark(ix, st);
     // ... phase B over every probed pair, emitting keys <= tau_q
     tp.phase = 1;
@@ -814,7 +821,7 @@ static mv_status search_chunk(mv_index* ix, const float* q, int64_t nq, int32_t 
                     ix->row_of_rank, ix->vmin, ix->vdiff, ix->sq8_t, gate, st));
     ix->launches += 2;
     CK(launch_final_select(b.poff, b.pcnt, part, nq, npb, k, ix->metric, ix->sorted_ids, D, I, tmax, over,
-                           BigSel{ix->opt.large_k_select, ix->opt.big_ctas, ix->opt.big_cap, 0}, st));
+                           BigSel{ix->opt.large_k_select, ix->opt.big_ctas, ix->opt.big_cap, 0, kmin, tau}, st));
   }
   prof_mark(ix, st);
   ix->last_scan = flat ? "tcgen05.tf32" : "tcgen05.i8";
@@ -888,6 +895,58 @@ mv_status mv_search_with_probes(mv_index* ix, const float* queries, int64_t nq, 
                                 int64_t* out_ids, void* stream) {
   if (probes == nullptr && nq > 0) return fail(MV_EINVAL, "probes is NULL");
   return search_impl(ix, queries, nq, k, nprobe, probes, bitset, nbits, distances, out_ids, stream);
+}
+
+mv_status mv_kmeans(const float* x, int64_t n, int32_t d, mv_metric metric, int32_t nlist, int32_t niter,
+                    int32_t spherical, float* centroids, int32_t device, void* stream) {
+  if (!x || !centroids) return fail(MV_EINVAL, "null argument");
+  if (n < nlist || nlist < 1) return fail(MV_EINVAL, "k-means needs 1 <= nlist <= n (n = %lld, nlist = %d)",
+                                          (long long)n, nlist);
+  if (niter < 0) return fail(MV_EINVAL, "niter must be >= 0");
+  if (n > 0x7fffffffLL) return fail(MV_EINVAL, "at most 2^31-1 training rows");
+  if (is_host_ptr(x) || is_host_ptr(centroids)) return fail(MV_EINVAL, "device pointers only");
+  mv_index* ix = nullptr;
+  mv_status v = mv_index_create(d, metric, MV_IVF_FLAT, nlist, device, nullptr, &ix);
+  if (v != MV_OK) return v;
+  struct Closer {
+    mv_index* p;
+    ~Closer() { mv_index_destroy(p); }
+  } closer{ix};
+  DeviceGuard g(device);
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  const int dpad = ix->dpad;
+  Scratch s(ix, st);
+  int32_t* lists;
+  double* sums;
+  unsigned long long* cnt;
+  CK(s.alloc(&lists, (size_t)n));
+  CK(s.alloc(&sums, (size_t)nlist * d));
+  CK(s.alloc(&cnt, (size_t)nlist));
+  const int64_t ldg = ((nlist + 127) / 128) * 4;
+  const int64_t sub = std::min<int64_t>(n, std::max<int64_t>(4096, (int64_t(1) << 27) / ldg));
+  float* qhl;
+  int* lo_any;
+  CK(s.alloc(&qhl, (size_t)2 * sub * dpad));
+  CK(s.alloc(&lo_any, 1));
+  for (int it = 0; it < niter; ++it) {
+    CK(cudaStreamSynchronize(st));  // set_centroids works on the legacy stream
+    v = mv_index_set_centroids(ix, centroids);
+    if (v != MV_OK) return v;
+    // assignment: the tensor-core coarse step with nprobe = 1 (as mv_index_add)
+    for (int64_t r0 = 0; r0 < n; r0 += sub) {
+      const int64_t m = std::min(sub, n - r0);
+      Scratch sb(ix, st);
+      CK(cudaMemsetAsync(lo_any, 0, sizeof(int), st));
+      CK(launch_hilo(x + r0 * d, m, d, dpad, qhl, lo_any, st));
+      CK(run_coarse(ix, qhl, lo_any, m, 1, lists + r0, sb, st));
+    }
+    CK(cudaMemsetAsync(sums, 0, sizeof(double) * (size_t)nlist * d, st));
+    CK(cudaMemsetAsync(cnt, 0, sizeof(unsigned long long) * nlist, st));
+    CK(launch_kmeans_accum(x, n, d, lists, sums, cnt, st));
+    CK(launch_kmeans_update(sums, cnt, nlist, d, spherical, centroids, st));
+  }
+  CK(cudaStreamSynchronize(st));
+  return MV_OK;
 }
 
 mv_status mv_attr_bitset(const int64_t* ids, const int64_t* attr, int64_t n, int64_t lo, int64_t hi,

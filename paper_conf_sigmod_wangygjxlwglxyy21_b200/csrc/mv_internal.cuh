@@ -182,7 +182,7 @@ struct Options {
   int coarse_nqb = 0, coarse_cs = 0, coarse_epi = 0, coarse_nacc = 0;  // coarse GEMM launch shape
   int64_t workspace = 0;    // per-search scratch budget in bytes (0: half of the free device memory)
   int64_t scan_trace = 0;   // -DMV_SCAN_TRACE builds: device address of the phase-B timeline buffer
-  int large_k_select = 0;   // k > 256: 0 staged radix select, 1 sample-threshold select (radix fallback)
+  int large_k_select = 0;   // k > 256: 0 streaming select (staged radix fallback), 1 sample-threshold select, 2 staged radix only
   int big_ctas = 0;         // k > 256 staged select: CTAs per SM of its first launch (1..4; 0 = 2)
   int64_t big_cap = 0;      // ... and its stage capacity in keys (0: the most that fits big_ctas per SM)
 };
@@ -194,6 +194,10 @@ struct BigSel {
   int ctas = 0;
   int64_t cap = 0;
   int64_t tlo = 0;
+  // streaming select (k_select_stream, mode 0): the seeding select writes each query's smallest
+  // key to kmin; the final select bins the keys over [kmin, khi] (khi = the seeding bound tau)
+  uint64_t* kmin = nullptr;
+  const uint64_t* khi = nullptr;
 };
 }  // namespace mv
 
@@ -276,6 +280,11 @@ cudaError_t launch_plan(const PlanArgs& a, cudaStream_t st);
 cudaError_t launch_scan_i32(const int32_t* in, int n, int32_t* out, cudaStream_t st);   // out[n+1]
 cudaError_t launch_scan_i64(const int64_t* in, int64_t n, int64_t* out, cudaStream_t st);  // out[n+1]
 
+// k_kmeans.cu: Lloyd k-means accumulation and update
+cudaError_t launch_kmeans_accum(const float* x, int64_t n, int d, const int32_t* lists, double* sums,
+                                unsigned long long* cnt, cudaStream_t st);
+cudaError_t launch_kmeans_update(const double* sums, const unsigned long long* cnt, int nlist, int d, int spherical,
+                                 float* c, cudaStream_t st);
 // k_filter.cu: strategy E's range bitmap and vector fusion
 cudaError_t launch_attr_bitset(const int64_t* ids, const int64_t* attr, int64_t n, int64_t lo, int64_t hi,
                                uint8_t* bitset, int64_t nbits, cudaStream_t st);

@@ -257,3 +257,18 @@ def merge_topk(dists, ids, metric="l2", stream=None):
         L.check(lib.mv_merge_topk(m, _ptr(dists), _ptr(ids), int(nsrc), int(nq), int(k), _ptr(D), _ptr(I),
                                   C.c_void_p(s.cuda_stream) if dists.is_cuda else None))
     return D, I
+
+
+def kmeans(x, nlist: int, niter: int = 10, metric="l2", spherical: bool = False, init=None, stream=None):
+    """mv_kmeans: niter Lloyd iterations of the coarse codebook on the device.
+    x: device [n, d] fp32 training rows; init: [nlist, d] initial centroids (default: the first
+    nlist rows -- pass a seeded sample).  Returns the [nlist, d] fp32 centroids."""
+    lib = L.load()
+    x = x.contiguous().float()
+    n, d = x.shape
+    c = (x[:nlist] if init is None else init).contiguous().float().clone()
+    m = METRICS[metric.lower() if isinstance(metric, str) else metric]
+    s = _torch_stream(x.device.index, stream)
+    L.check(lib.mv_kmeans(_ptr(x), int(n), int(d), m, int(nlist), int(niter), int(bool(spherical)), _ptr(c),
+                          int(x.device.index), C.c_void_p(s.cuda_stream)))
+    return c

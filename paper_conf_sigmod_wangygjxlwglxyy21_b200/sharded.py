@@ -98,14 +98,16 @@ class ShardedIndex:
     # -- search: local top-k, one all-gather, on-device merge -----------------------------------
     def search(self, q: torch.Tensor, k: int, nprobe: int, bitset=None, nbits: int | None = None):
         nlist = int(getattr(self.local, "nlist", 1))
-        split = self.world > 1 and (self.coarse == "split" or
-                                    (self.coarse == "auto" and q.shape[0] * nlist >= (1 << 28)))
+        # an explicit mode runs its collectives at any world size (world 1 included: the NCCL path
+        # on a single GPU, tests/test_gpu_sharded.py); "auto" skips them when there is no peer
+        split = dist.is_initialized() and (self.coarse == "split" or (
+            self.coarse == "auto" and self.world > 1 and q.shape[0] * nlist >= (1 << 28)))
         if split:
             P = self._split_probes(q, nprobe, nlist)
             D, I = self.local.search(q, k, nprobe, bitset=bitset, nbits=nbits, probes=P)
         else:
             D, I = self.local.search(q, k, nprobe, bitset=bitset, nbits=nbits)
-        if self.world == 1:
+        if self.world == 1 and (self.exchange == "auto" or not dist.is_initialized()):
             return D, I
         mode = self.exchange if self.exchange != "auto" else ("alltoall" if k >= 256 else "allgather")
         if mode == "alltoall":

@@ -1,5 +1,9 @@
-O=gpurun_out/q_e; mkdir -p $O
-timeout 600 python -m pytest tests/test_gpu_filtering.py -x -q -p no:cacheprovider > $O/pytest_f4.log 2>&1; echo f4=$?; tail -3 $O/pytest_f4.log
-timeout 900 python scripts/sweep_opts.py --config c4 --sets "" "flat_qc=80" "flat_qc=64" "flat_qc=48" > $O/sweep_c4.txt 2>&1; echo s4=$?
-timeout 900 python scripts/sweep_opts.py --config c2 --sets "" "flat_qc=80" "flat_qc=64" "flat_qc=48" > $O/sweep_c2.txt 2>&1; echo s2=$?
-timeout 900 ncu --profile-from-start off --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none --csv python scripts/prof_search.py --config c4 > $O/launches_c4.csv 2>/dev/null; python scripts/ncu_summary.py $O/launches_c4.csv > $O/launches_c4_summary.txt
+O=gpurun_out/q_k; mkdir -p $O
+L=paper_conf_sigmod_wangygjxlwglxyy21_b200/libmv.so
+timeout 900 python -m pytest tests -m "gpu and not slow" -x -q -p no:cacheprovider > $O/pytest.log 2>&1; echo pytest=$?; tail -3 $O/pytest.log
+timeout 900 python scripts/sweep_opts.py --config c4 --sets "" "large_k_select=2" "large_k_select=3" > $O/sweep_c4.txt 2>&1; echo s4=$?
+for v in nommaepi nogather nothing; do
+  cp exp/lib_$v.so $L
+  for c in c5 c3 c4; do timeout 600 python scripts/sweep_opts.py --config $c --steps 5 --sets "" 2>&1 | grep -v "^\[bench" | sed "s/^/$v /" >> $O/exp.txt; done
+done
+cp exp/lib_prod.so $L

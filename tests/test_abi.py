@@ -70,3 +70,12 @@ def test_no_cpu_fallback_in_the_binding():
         if fn.endswith(".py"):
             src = open(os.path.join(pkg, fn)).read()
             assert "import oracle" not in src and "from oracle" not in src, fn
+
+
+def test_f1_f4_entry_points_validate_arguments(lib):
+    import ctypes as C
+    assert lib.mv_kmeans(None, 10, 4, 0, 2, 1, 0, None, 0, None) == -1
+    assert lib.mv_attr_bitset(None, None, -1, 0, 1, None, 8, None) == -1
+    dims = (C.c_int32 * 1)(4)
+    assert lib.mv_fuse_rows(None, dims, None, 0, 1, None, None) == -1      # m = 0
+    assert lib.mv_fuse_rows(None, dims, None, 17, 1, None, None) == -1     # m > 16

@@ -369,7 +369,7 @@ def test_c2_full_size_sampled():
 
 OPTION_SETS = [{"seeding": 0}, {"need": 1, "capa": 16}, {"flat_qc": 32, "sq8_qc": 16},
                {"coarse_nqb": 64, "coarse_cs": 3, "coarse_epi": 16, "coarse_nacc": 1},
-               {"workspace_bytes": 1 << 20}, {"large_k_select": 1},
+               {"workspace_bytes": 1 << 20}, {"large_k_select": 1}, {"large_k_select": 2}, {"large_k_select": 3},
                {"seeding": 0, "big_cap": 1100}, {"big_ctas": 4, "big_cap": 700}, {"big_ctas": 1}]
 
 

@@ -36,3 +36,39 @@ def test_g_shards_equal_one_index(kind, metric, nshard):
     torch.cuda.synchronize()
     assert torch.equal(I, I1)
     assert torch.equal(D, D1)
+
+
+@pytest.mark.parametrize("exchange,coarse,k", [("allgather", "replicated", 20), ("alltoall", "split", 300),
+                                               ("alltoall", "replicated", 2048)])
+def test_nccl_exchange_paths_on_one_gpu(exchange, coarse, k):
+    """The NCCL code of ShardedIndex (all_gather_into_tensor, all_to_all_single, the query-split
+    coarse step's probe all-gather) on hardware: a one-rank NCCL group (the box has one GPU) must
+    return exactly the local index's result."""
+    import os
+    import socket
+    import torch.distributed as dist
+    from paper_conf_sigmod_wangygjxlwglxyy21_b200 import Index
+    from paper_conf_sigmod_wangygjxlwglxyy21_b200.sharded import ShardedIndex
+    spec = G.SiftSpec(d=128, n_micro=1024)
+    X = G.sift_base(20_000, spec=spec).cuda()
+    Q = G.sift_queries(150, spec=spec).cuda()
+    ids = G.permuted_ids(20_000, seed=3).cuda()
+    C = kmeans(X.cpu(), 48, iters=4).cuda()
+    ix = Index(128, "l2", "flat", 48)
+    ix.set_centroids(C)
+    ix.add(X, ids)
+    D1, I1 = ix.search(Q, k, 6)
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", 0))
+    try:
+        sh = ShardedIndex(ix, exchange=exchange, coarse=coarse)
+        D, I = sh.search(Q, k, 6)
+        torch.cuda.synchronize()
+        assert dist.get_backend() == "nccl"
+        assert torch.equal(I, I1) and torch.equal(D, D1)
+    finally:
+        dist.destroy_process_group()

@@ -120,13 +120,13 @@ def _free_port():
     return p
 
 
-def _worker(rank, world, port, metric, out, exchange="auto", nq=25, k=37):
+def _worker(rank, world, port, metric, out, exchange="auto", nq=25, k=37, n=900):
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     dist.init_process_group("gloo", rank=rank, world_size=world)
     try:
         r = np.random.default_rng(7)
-        X = r.integers(0, 6, (900, 4)).astype(np.float32)   # small integers: many exact ties
-        ids = r.permutation(5000)[:900].astype(np.int64)
+        X = r.integers(0, 6, (n, 4)).astype(np.float32)   # small integers: many exact ties
+        ids = r.permutation(6 * n)[:n].astype(np.int64)
         Q = r.integers(0, 6, (nq, 4)).astype(np.float32)
         sh = ShardedIndex(OracleShard(metric), merge=oracle_merge, exchange=exchange)
         sh.set_centroids(torch.zeros(1, 4))
@@ -172,6 +172,25 @@ def test_gloo_alltoall_exchange_equals_single_index(world, nq, k, metric):
         p.join(timeout=60)
         assert p.exitcode == 0
     De, Ie = O.exact_knn(X, ids, Q, k, metric)
+    assert np.array_equal(I, Ie)
+    assert np.array_equal(D, De.astype(np.float32))
+
+
+def test_gloo_eight_ranks_k16384_alltoall():
+    """k = 16384 at G = 8 through the all-to-all exchange
+    equals one index (nq = 9, not a multiple of 8; every shard holds fewer than k rows)."""
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    world, nq, k, n = 8, 9, 16384, 20000
+    procs = [ctx.Process(target=_worker, args=(r, world, port, O.L2, q, "alltoall", nq, k, n)) for r in range(world)]
+    for p in procs:
+        p.start()
+    D, I, X, ids, Q = q.get(timeout=400)
+    for p in procs:
+        p.join(timeout=120)
+        assert p.exitcode == 0
+    De, Ie = O.exact_knn(X, ids, Q, k, O.L2)
     assert np.array_equal(I, Ie)
     assert np.array_equal(D, De.astype(np.float32))
 
