@@ -17,6 +17,7 @@ Parity status of each function (DESIGN.md §2 lists the pins):
   multi.py: range_bitset, partition_plan, partition_search (strategy E),
   multivector_scores / multivector_topk (§4.2) -- pinned by tests/test_oracle_multi.py.
   kmeans.py: lloyd_step, kmeans, sse -- pinned by tests/test_oracle_kmeans.py.
+  pq.py: pq_encode, pq_decode, IvfPqIndex -- pinned by tests/test_oracle_pq.py.
 """
 from .ivf import (  # noqa: F401
     FLAT, IP, L2, SQ8, IvfIndex, assign, bit_is_set, distances, exact_knn, merge_topk, pad_value, probe,
@@ -26,3 +27,4 @@ from .multi import (  # noqa: F401,E402
     multivector_scores, multivector_topk, partition_plan, partition_search, range_bitset,
 )
 from . import kmeans as km  # noqa: F401,E402
+from .pq import IvfPqIndex, pq_decode, pq_encode  # noqa: F401,E402
