@@ -43,6 +43,9 @@ CONFIGS = {
                nlist=16384, nprobe=32, nq=10_000, k=100, kind="sq8", metric="ip", bitset=10),
     "c4": dict(workload="sift10m_ivfflat_l2_nlist16384_nprobe128_k2048", data="sift", n=10_000_000, d=128,
                nlist=16384, nprobe=128, nq=10_000, k=2048, kind="flat", metric="l2", bitset=0),
+    # configs[2]'s workload on IVF_PQ (M = 16 one-byte sub-codes: 16 B per vector)
+    "c3pq": dict(workload="deep10m_ivfpq16_ip_nlist16384_nprobe32_k100_bitset10", data="deep", n=10_000_000, d=96,
+                 nlist=16384, nprobe=32, nq=10_000, k=100, kind="pq", pq_m=16, metric="ip", bitset=10),
     # 1B rows, vector-sharded (row r -> shard r mod S).  Under N ranks, S = N: the full index,
     # strong scaling.  At N = 1 the GPU holds shard 0 of --c5-shards (default 8): the per-GPU
     # workload of the 8-GPU job.
@@ -440,6 +443,10 @@ def main():
         (sh.set_centroids if dist else ix.set_centroids)(C)
         if cfg["kind"] == "sq8":
             (sh.set_sq8 if dist else ix.set_sq8)(*sq8_params(cfg, X))
+        if cfg["kind"] == "pq":  # per-sub-space k-means on 64 nlist seeded rows (mv_kmeans; untimed)
+            g = torch.Generator(device="cpu").manual_seed(5)
+            samp = torch.randperm(n, generator=g)[: min(n, 64 * cfg["nlist"])].to(dev)
+            ix.train_pq(cfg["pq_m"], X[samp].contiguous(), niter=10)
         BUILD.update(vectors=0, seconds=0.0, calls=0)
         if dist:
             sh.add(X, ids)   # every rank keeps the rows it owns (id % world == rank)
@@ -566,7 +573,7 @@ def main():
     lens = np.diff(off)
     probed = np.unique(P.cpu().numpy())
     dpad = (cfg["d"] + 31) // 32 * 32
-    bpv = (4 * dpad if cfg["kind"] == "flat" else dpad) + (8 if bs is not None else 0)
+    bpv = ({"flat": 4 * dpad, "sq8": dpad, "pq": cfg.get("pq_m", 0)}[cfg["kind"]]) + (8 if bs is not None else 0)
     units = int(lens[probed].sum())  # distinct probed vectors per launch (this GPU's shard)
     scan_bytes = units * bpv
     scan_ms = stage_ms["scan_a"] + stage_ms["scan"]  # both launches of the scan kernel (phases A and B)

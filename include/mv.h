@@ -54,7 +54,8 @@ typedef enum {
 
 typedef enum {
   MV_IVF_FLAT = 0, /* fine quantizer keeps the fp32 vector */
-  MV_IVF_SQ8 = 1   /* fine quantizer keeps one byte per dimension */
+  MV_IVF_SQ8 = 1,  /* fine quantizer keeps one byte per dimension */
+  MV_IVF_PQ = 2    /* product quantization: M one-byte sub-codes */
 } mv_type;
 
 /* Device-memory allocator supplied by the caller.  alloc(bytes, stream, ctx)
@@ -171,6 +172,19 @@ MV_API mv_status mv_search_with_probes(mv_index* index, const float* queries, in
 MV_API mv_status mv_merge_topk(mv_metric metric, const float* dists, const int64_t* ids, int32_t nsrc, int64_t nq,
                         int32_t k, float* out_d, int64_t* out_i, void* stream);
 
+/* IVF_PQ fine quantizer ("splits each vector into multiple
+ * sub-vectors and applies k-means for each sub-space"; reading R19): M sub-spaces of d / M
+ * consecutive dimensions (d % M == 0, M % 4 == 0, M <= 64), 256 sub-centroids each.
+ * set_pq: codebooks [M][256][d/M] fp32 (host or device), copied.  train_pq: per sub-space
+ * mv_kmeans (L2, niter iterations, initial sub-centroids = the first 256 rows) over the
+ * sample's sub-vectors (device [n][d] fp32, n >= 256).  Both synchronous; only before the first
+ * add, on an MV_IVF_PQ index (else MV_ESTATE).  A search on an IVF_PQ index returns the
+ * asymmetric distance from each query to the decoded vector (fp32 sums of fp32 table entries). */
+MV_API mv_status mv_index_set_pq(mv_index* index, int32_t M, const float* codebooks);
+MV_API mv_status mv_index_train_pq(mv_index* index, int32_t M, const float* sample, int64_t n, int32_t niter);
+/* Parity hook: the PQ codebooks ([M][256][d/M] fp32, host or device) and M.  Synchronous. */
+MV_API mv_status mv_index_get_pq(const mv_index* index, int32_t* M, float* codebooks);
+
 /* Lloyd k-means training of the coarse codebook on the device (PAPER.md:503-514
  * §3.1: the buckets are K-means clusters).  x: device [n][d] fp32 training rows; centroids: device
  * [nlist][d] fp32 -- in: the initial centroids (e.g. nlist seeded training rows), out: after niter
@@ -205,8 +219,8 @@ MV_API mv_status mv_fuse_rows(const float* const* parts, const int32_t* dims, co
 MV_API int64_t mv_index_ntotal(const mv_index* index);
 
 /* Parity hook: copy the list-major storage description.  list_off: nlist+1 int64 (may be
- * NULL); ids: ntotal int64 in storage order (may be NULL); codes: ntotal x d uint8 (SQ8 only,
- * unpadded, may be NULL).  Host or device pointers.  Synchronous. */
+ * NULL); ids: ntotal int64 in storage order (may be NULL); codes: ntotal x d uint8 (SQ8,
+ * unpadded) or ntotal x M uint8 (IVF_PQ), may be NULL.  Host or device pointers.  Synchronous. */
 MV_API mv_status mv_index_storage(const mv_index* index, int64_t* list_off, int64_t* ids, uint8_t* codes);
 
 /* Parity hook: SQ8 parameters (d floats each). Synchronous. */

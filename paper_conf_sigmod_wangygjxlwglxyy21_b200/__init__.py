@@ -8,7 +8,7 @@ path of Milvus (Wang et al., SIGMOD'21), behind the C ABI of include/mv.h.
 
 There is no CPU fallback: importing the binding loads libmv.so and fails loudly without it.
 """
-from ._lib import MV_IP, MV_IVF_FLAT, MV_IVF_SQ8, MV_L2, MvError, load  # noqa: F401
+from ._lib import MV_IP, MV_IVF_FLAT, MV_IVF_PQ, MV_IVF_SQ8, MV_L2, MvError, load  # noqa: F401
 from .index import Index, kmeans, merge_topk  # noqa: F401
 
 __all__ = ["Index", "kmeans", "merge_topk", "MvError", "MV_L2", "MV_IP", "MV_IVF_FLAT", "MV_IVF_SQ8"]

@@ -13,7 +13,7 @@ LIB_PATH = os.path.join(_PKG, "libmv.so")
 HEADER = os.path.join(os.path.dirname(_PKG), "include", "mv.h")
 
 MV_L2, MV_IP = 0, 1
-MV_IVF_FLAT, MV_IVF_SQ8 = 0, 1
+MV_IVF_FLAT, MV_IVF_SQ8, MV_IVF_PQ = 0, 1, 2
 STATUS = {0: "MV_OK", -1: "MV_EINVAL", -2: "MV_ESTATE", -3: "MV_ENOMEM", -4: "MV_ECUDA", -5: "MV_ENCCL"}
 
 
@@ -48,6 +48,9 @@ _SIGS = {
     "mv_search_probes": (C.c_int, [_P, _P, C.c_int64, C.c_int32, _P, _P]),
     "mv_search_with_probes": (C.c_int, [_P, _P, C.c_int64, C.c_int32, C.c_int32, _P, _P, C.c_int64, _P, _P, _P]),
     "mv_merge_topk": (C.c_int, [C.c_int, _P, _P, C.c_int32, C.c_int64, C.c_int32, _P, _P, _P]),
+    "mv_index_set_pq": (C.c_int, [_P, C.c_int32, _P]),
+    "mv_index_get_pq": (C.c_int, [_P, _P, _P]),
+    "mv_index_train_pq": (C.c_int, [_P, C.c_int32, _P, C.c_int64, C.c_int32]),
     "mv_kmeans": (C.c_int, [_P, C.c_int64, C.c_int32, C.c_int, C.c_int32, C.c_int32, C.c_int32, _P, C.c_int32, _P]),
     "mv_attr_bitset": (C.c_int, [_P, _P, C.c_int64, C.c_int64, C.c_int64, _P, C.c_int64, _P]),
     "mv_fuse_rows": (C.c_int, [C.POINTER(C.c_void_p), C.POINTER(C.c_int32), C.POINTER(C.c_float), C.c_int32,

@@ -19,7 +19,9 @@ using namespace mv;
 
 struct mv_index {
   int d = 0, dpad = 0, metric = 0, type = 0, nlist = 0, device = 0;
-  bool has_centroids = false, has_sq8 = false;
+  bool has_centroids = false, has_sq8 = false, has_pq = false;
+  int pq_m = 0, pq_dsub = 0;    // IVF_PQ: sub-spaces and their dimension
+  float* pq_cb = nullptr;       // IVF_PQ: [M][256][dsub] sub-centroids
   mv_allocator alloc{};         // caller allocator (alloc.alloc == NULL: CUDA's own)
   Options opt;
   float* cpad = nullptr;    // nlist x dpad
@@ -273,7 +275,8 @@ mv_status mv_index_create(int32_t d, mv_metric metric, mv_type type, int32_t nli
   *out = nullptr;
   if (d < 1 || d > kMaxD) return fail(MV_EINVAL, "d must be in [1, %d] (got %d)", kMaxD, d);
   if (metric != MV_L2 && metric != MV_IP) return fail(MV_EINVAL, "unknown metric %d", (int)metric);
-  if (type != MV_IVF_FLAT && type != MV_IVF_SQ8) return fail(MV_EINVAL, "unknown index type %d", (int)type);
+  if (type != MV_IVF_FLAT && type != MV_IVF_SQ8 && type != MV_IVF_PQ)
+    return fail(MV_EINVAL, "unknown index type %d", (int)type);
   if (nlist < 1) return fail(MV_EINVAL, "nlist must be >= 1 (got %d)", nlist);
   if (alloc && (alloc->alloc == nullptr) != (alloc->free == nullptr))
     return fail(MV_EINVAL, "allocator: alloc and free must both be set");
@@ -355,6 +358,7 @@ void mv_index_destroy(mv_index* ix) {
   mem_free(ix, ix->vmin, nullptr);
   mem_free(ix, ix->vdiff, nullptr);
   mem_free(ix, ix->sq8_t, nullptr);
+  mem_free(ix, ix->pq_cb, nullptr);
   cudaFree(ix->d_count);
   delete ix;
 }
@@ -395,6 +399,64 @@ mv_status mv_index_train_sq8(mv_index* ix, const float* sample, int64_t n) {
   return MV_OK;
 }
 
+static mv_status pq_check(const mv_index* ix, int32_t M) {
+  if (!ix) return fail(MV_EINVAL, "null index");
+  if (ix->type != MV_IVF_PQ) return fail(MV_ESTATE, "PQ parameters on a non-IVF_PQ index");
+  if (ix->ntotal > 0) return fail(MV_ESTATE, "PQ parameters cannot change after vectors were added");
+  if (M < 4 || M > 64 || M % 4 || ix->d % M) return fail(MV_EINVAL, "M must divide d, be a multiple of 4 and <= 64");
+  return MV_OK;
+}
+
+mv_status mv_index_set_pq(mv_index* ix, int32_t M, const float* codebooks) {
+  mv_status v = pq_check(ix, M);
+  if (v != MV_OK) return v;
+  if (!codebooks) return fail(MV_EINVAL, "null codebooks");
+  DeviceGuard g(ix->device);
+  const size_t bytes = sizeof(float) * 256 * (size_t)ix->d;
+  if (!ix->pq_cb && !(ix->pq_cb = (float*)mem_alloc(ix, bytes, nullptr)))
+    return fail(MV_ENOMEM, "set_pq: cannot allocate the codebooks");
+  CK(cudaMemcpy(ix->pq_cb, codebooks, bytes, cudaMemcpyDefault));
+  ix->pq_m = M;
+  ix->pq_dsub = ix->d / M;
+  ix->has_pq = true;
+  return MV_OK;
+}
+
+mv_status mv_index_get_pq(const mv_index* ix, int32_t* M, float* codebooks) {
+  if (!ix) return fail(MV_EINVAL, "null index");
+  if (ix->type != MV_IVF_PQ || !ix->has_pq) return fail(MV_ESTATE, "no PQ parameters");
+  DeviceGuard g(ix->device);
+  if (M) *M = ix->pq_m;
+  if (codebooks) CK(cudaMemcpy(codebooks, ix->pq_cb, sizeof(float) * 256 * (size_t)ix->d, cudaMemcpyDefault));
+  return MV_OK;
+}
+
+mv_status mv_index_train_pq(mv_index* ix, int32_t M, const float* sample, int64_t n, int32_t niter) {
+  mv_status v = pq_check(ix, M);
+  if (v != MV_OK) return v;
+  if (!sample || n < 256) return fail(MV_EINVAL, "train_pq needs >= 256 sample rows");
+  if (is_host_ptr(sample)) return fail(MV_EINVAL, "train_pq: device sample only");
+  DeviceGuard g(ix->device);
+  const int dsub = ix->d / M;
+  float *sub = nullptr, *cb = nullptr;
+  CK(cudaMalloc(&sub, sizeof(float) * (size_t)n * dsub));
+  struct F {
+    float** a;
+    float** b;
+    ~F() { cudaFree(*a); cudaFree(*b); }
+  } f{&sub, &cb};
+  CK(cudaMalloc(&cb, sizeof(float) * 256 * (size_t)ix->d));
+  for (int m = 0; m < M; ++m) {  // k-means of each sub-space, 256 sub-centroids
+    CK(cudaMemcpy2D(sub, sizeof(float) * dsub, sample + m * dsub, sizeof(float) * ix->d, sizeof(float) * dsub, n,
+                    cudaMemcpyDeviceToDevice));
+    float* cbm = cb + (size_t)m * 256 * dsub;
+    CK(cudaMemcpy(cbm, sub, sizeof(float) * 256 * dsub, cudaMemcpyDeviceToDevice));
+    v = mv_kmeans(sub, n, dsub, MV_L2, 256, niter, 0, cbm, ix->device, nullptr);
+    if (v != MV_OK) return v;
+  }
+  return mv_index_set_pq(ix, M, cb);
+}
+
 mv_status mv_index_set_sq8(mv_index* ix, const float* vmin, const float* vdiff) {
   if (!ix || !vmin || !vdiff) return fail(MV_EINVAL, "null argument");
   if (ix->type != MV_IVF_SQ8) return fail(MV_ESTATE, "set_sq8 on a non-SQ8 index");
@@ -427,6 +489,7 @@ mv_status mv_index_add(mv_index* ix, const float* vectors, const int64_t* ids, i
   if (!vectors || !ids) return fail(MV_EINVAL, "null vectors/ids");
   if (!ix->has_centroids) return fail(MV_ESTATE, "add before set_centroids");
   if (ix->type == MV_IVF_SQ8 && !ix->has_sq8) return fail(MV_ESTATE, "add on SQ8 index before train_sq8/set_sq8");
+  if (ix->type == MV_IVF_PQ && !ix->has_pq) return fail(MV_ESTATE, "add on IVF_PQ index before train_pq/set_pq");
   if (n > 0x7fffffffLL) return fail(MV_EINVAL, "one add call takes at most 2^31-1 vectors");
   if (ix->ntotal + n > 0x7fffffffLL) return fail(MV_EINVAL, "an index holds at most 2^31-1 vectors");
   DeviceGuard g(ix->device);
@@ -496,13 +559,15 @@ mv_status mv_index_add(mv_index* ix, const float* vectors, const int64_t* ids, i
   CK(launch_scan_i64(sizes, nlist, new_off, st));
 
   const int64_t ntot = ix->ntotal + n;
+  const bool pq = ix->type == MV_IVF_PQ;
   const size_t esize = ix->type == MV_IVF_FLAT ? 4 : 1;
+  const int prow = pq ? ix->pq_m : dpad;  // payload elements per row (PQ: M sub-codes)
   // per-row side arrays carry kSidePad zeroed tail elements: the scan bulk-copies 16-B aligned
   // supersets of 128-row tiles
   constexpr int64_t kSidePad = 256;
   mv_index nx;  // the new storage (only the pointers are used)
   nx.alloc = ix->alloc;
-  nx.payload = mem_alloc(ix, (size_t)ntot * dpad * esize, st);
+  nx.payload = mem_alloc(ix, (size_t)ntot * prow * esize + 16, st);
   nx.norms = (double*)mem_alloc(ix, sizeof(double) * (ntot + kSidePad), st);
   nx.ids = (int64_t*)mem_alloc(ix, sizeof(int64_t) * (ntot + kSidePad), st);
   nx.rank = (uint32_t*)mem_alloc(ix, sizeof(uint32_t) * (ntot + kSidePad), st);
@@ -515,10 +580,14 @@ mv_status mv_index_add(mv_index* ix, const float* vectors, const int64_t* ids, i
   CK(cudaMemsetAsync(nx.norms + ntot, 0, sizeof(double) * kSidePad, st));
   CK(cudaMemsetAsync(nx.ids + ntot, 0, sizeof(int64_t) * kSidePad, st));
   CK(cudaMemsetAsync(nx.rank + ntot, 0, sizeof(uint32_t) * kSidePad, st));
-  CK(launch_move_old(ix->type, dpad, nlist, ix->list_off, new_off, ix->payload, ix->norms, ix->ids, ix->ntotal,
-                     nx.payload, nx.norms, nx.ids, st));
-  CK(launch_store_rows(ix->type, ix->metric, xpad, idv, sidx, slist, n, dpad, new_off, ix->list_off, addoff,
-                       nx.payload, nx.norms, nx.ids, ix->vmin, ix->vdiff, ix->sq8_t, st));
+  CK(launch_move_old(pq ? MV_IVF_SQ8 : ix->type, prow, nlist, ix->list_off, new_off, ix->payload, ix->norms, ix->ids,
+                     ix->ntotal, nx.payload, nx.norms, nx.ids, st));
+  if (pq)
+    CK(launch_pq_encode(xpad, idv, sidx, slist, n, dpad, ix->pq_m, ix->pq_dsub, ix->pq_cb, new_off, ix->list_off, addoff,
+                        reinterpret_cast<uint8_t*>(nx.payload), nx.norms, nx.ids, st));
+  else
+    CK(launch_store_rows(ix->type, ix->metric, xpad, idv, sidx, slist, n, dpad, new_off, ix->list_off, addoff,
+                         nx.payload, nx.norms, nx.ids, ix->vmin, ix->vdiff, ix->sq8_t, st));
   // id ranks: stable radix sort of (id) over storage rows -> (id, row) order
   uint64_t *keys, *skeys;
   uint32_t *vals, *svals;
@@ -564,7 +633,7 @@ mv_status mv_index_add(mv_index* ix, const float* vectors, const int64_t* ids, i
   ix->xmax2 = xm2;
   // one swizzle atom per box row: 128 B (FLAT: 32 fp32; SQ8 when dpad is a multiple of 128), else 32 B
   const bool wide = ix->type == MV_IVF_FLAT || dpad % 128 == 0;
-  for (int i = 0; i < 4; ++i)
+  for (int i = 0; i < 4 && !pq; ++i)
     if (!make_tmap_2d(&ix->xm.m[i], ix->payload,
                       ix->type == MV_IVF_FLAT ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_UINT8,
                       (uint64_t)dpad, (uint64_t)ntot, (uint64_t)dpad * esize, ix->type == MV_IVF_FLAT ? 32 : (wide ? 128 : 32),
@@ -639,6 +708,7 @@ static mv_status search_chunk(mv_index* ix, const float* q, int64_t nq, int32_t 
   Scratch s(ix, st);
   const int nlist = ix->nlist, dpad = ix->dpad;
   const bool flat = ix->type == MV_IVF_FLAT;
+  const bool pq = ix->type == MV_IVF_PQ;  // the query-major ADC scan (k_pq.cu) instead of k_scan_tc
   // a1 + a2/a3
   prof_mark(ix, st);
   float *qpad, *qnorm;
@@ -658,7 +728,9 @@ static mv_status search_chunk(mv_index* ix, const float* q, int64_t nq, int32_t 
   prof_mark(ix, st);
   // a4 (the work-item shape follows the scan's shared-memory plan)
   TcScanParams tp;
-  if (!tc_scan_plan(ix->type, dpad, k, (double)nq * npb / std::max(1, nlist), bs != nullptr, ix->opt, tp))
+  // (IVF_PQ: the planner's pair regions and seeding lists are used, its work items are not)
+  if (!tc_scan_plan(pq ? (int)MV_IVF_SQ8 : ix->type, dpad, k, (double)nq * npb / std::max(1, nlist), bs != nullptr,
+                    ix->opt, tp))
     return fail(MV_EINVAL, "search: no tensor-core scan plan fits d = %d", ix->d);
   const int qchunk = tp.qchunk;
   const int qchunk_min = tp.qchunk_split;  // FLAT two-plane items
@@ -699,7 +771,7 @@ static mv_status search_chunk(mv_index* ix, const float* q, int64_t nq, int32_t 
   // ~26x more per candidate (and falls back to global memory past its stage), c = 832 B.
   {
     const double ncand = (double)ix->ntotal * npb / std::max(1, nlist);
-    const double rowb = (double)dpad * (flat ? 4 : 1);
+    const double rowb = pq ? (double)ix->pq_m : (double)dpad * (flat ? 4 : 1);
     const double c = k > 256 ? 832.0 : 32.0;
     const int64_t bal = (int64_t)std::sqrt((double)k * ncand * c / rowb);
     pa.need = std::max<int64_t>(pa.need, std::min<int64_t>(bal, 65536));
@@ -739,7 +811,7 @@ static mv_status search_chunk(mv_index* ix, const float* q, int64_t nq, int32_t 
   float *qscale, *qerr = nullptr;
   double *qa, *qn64;
   uint64_t* tau;
-  if (!flat) CK(s.alloc(&qplanes, (size_t)nq * kSq8Planes * dpad));
+  if (!flat && !pq) CK(s.alloc(&qplanes, (size_t)nq * kSq8Planes * dpad));
   else qplanes = reinterpret_cast<uint8_t*>(qhl);
   CK(s.alloc(&qscale, (size_t)nq));
   CK(s.alloc(&qa, (size_t)nq));
@@ -753,8 +825,16 @@ static mv_status search_chunk(mv_index* ix, const float* q, int64_t nq, int32_t 
   const int* gate = approx_always ? nullptr : qlo_any;
   FlatErr fe{ix->tf32_exact ? 0.0 : 0x1p-10, ix->tf32_exact ? 0x1p-21 : 0x1p-11, ix->xmax2, ix->metric};
   CK(s.alloc(&qerr, (size_t)nq));
-  CK(launch_qplanes(ix->type, qpad, nq, dpad, ix->vmin, ix->vdiff, flat ? nullptr : qplanes, qscale, qa, qn64, &fe,
-                    qerr, st));
+  if (!pq)
+    CK(launch_qplanes(ix->type, qpad, nq, dpad, ix->vmin, ix->vdiff, flat ? nullptr : qplanes, qscale, qa, qn64, &fe,
+                      qerr, st));
+  PqScanParams pp{};
+  if (pq) {
+    pp.metric = ix->metric; pp.dpad = dpad; pp.M = ix->pq_m; pp.dsub = ix->pq_dsub; pp.npb = npb; pp.nq = nq;
+    pp.qpad = qpad; pp.codebooks = ix->pq_cb; pp.probes = P; pp.ra = ra; pp.tau = tau; pp.list_off = ix->list_off;
+    pp.codes = reinterpret_cast<const uint8_t*>(ix->payload); pp.rank = ix->rank; pp.ids = ix->ids;
+    pp.bitset = bs; pp.nbits = bs ? nbits : 0; pp.poff = b.poff; pp.pcnt = b.pcnt; pp.part = part;
+  }
   tp.metric = ix->metric; tp.npb = npb; tp.nq = nq;
   tp.list_off = ix->list_off; tp.norms = ix->norms; tp.ids = ix->ids; tp.rank = ix->rank;
   tp.bitset = bs; tp.nbits = bs ? nbits : 0;
@@ -769,7 +849,13 @@ static mv_status search_chunk(mv_index* ix, const float* q, int64_t nq, int32_t 
   tp.wbeg = nullptr;
   tp.nwitems = b.woff + nlist;
   tp.counter = b.counter;
-  CK(launch_scan_tc(ix->xm, tp, st));
+  if (pq) {
+    pp.phase = split ? 0 : 1;  // without seeding: one pass over every pair, everything emitted (tau = pad)
+    pp.rowcap = split ? (int)pa.capA : 0x7fffffff;
+    CK(launch_pq_scan(pp, st));
+  } else {
+    CK(launch_scan_tc(ix->xm, tp, st));
+  }
   prof_mark(ix, st);
   if (split) {
     // ... tau_q = k-th best key of phase A (phase A emits < need + capA candidates per query) ...
@@ -786,7 +872,13 @@ static mv_status search_chunk(mv_index* ix, const float* q, int64_t nq, int32_t 
     tp.wbeg = b.woff + nlist;
     tp.nwitems = b.woff + 2 * nlist;
     tp.counter = b.counter + 1;
-    CK(launch_scan_tc(ix->xm, tp, st));
+    if (pq) {
+      pp.phase = 1;
+      pp.rowcap = 0x7fffffff;
+      CK(launch_pq_scan(pp, st));
+    } else {
+      CK(launch_scan_tc(ix->xm, tp, st));
+    }
   } else {
     prof_mark(ix, st);
   }
@@ -800,7 +892,11 @@ static mv_status search_chunk(mv_index* ix, const float* q, int64_t nq, int32_t 
     if (split) CK(launch_sum_i32(b.pcnt + npairs, npairs, npb, ra, ix->d_count + 1, st));
     CK(launch_sum_i32(b.pcnt, npairs, npb, nullptr, ix->d_count + 2, st));
   }
-  if (k <= 256) {
+  if (pq) {
+    // IVF_PQ: the keys are the asymmetric distances themselves -- the plain exact select
+    CK(launch_final_select(b.poff, b.pcnt, part, nq, npb, k, ix->metric, ix->sorted_ids, D, I, tmax, over,
+                           BigSel{ix->opt.large_k_select, ix->opt.big_ctas, ix->opt.big_cap, 0, kmin, tau}, st));
+  } else if (k <= 256) {
     // a7 with the filter mode's exact re-scoring fused in (a plain exact select when the search is
     // exact: FLAT with tf32-exact data and queries, gate = qlo_any == 0 on the device)
     uint64_t* tau2;
@@ -824,7 +920,7 @@ static mv_status search_chunk(mv_index* ix, const float* q, int64_t nq, int32_t 
                            BigSel{ix->opt.large_k_select, ix->opt.big_ctas, ix->opt.big_cap, 0, kmin, tau}, st));
   }
   prof_mark(ix, st);
-  ix->last_scan = flat ? "tcgen05.tf32" : "tcgen05.i8";
+  ix->last_scan = pq ? "simt.pq_adc" : (flat ? "tcgen05.tf32" : "tcgen05.i8");
   // prep, hilo, coarse (GEMM pass 0, group bound, GEMM pass 1, top-nprobe | all lists), plan, qplanes,
   // scan A (+ seed select, scan B), final select
   ix->launches += 5 + (P_in ? 0 : (npb >= nlist ? 1 : 4)) + (split ? 2 : 0) + 1;
@@ -1056,7 +1152,8 @@ mv_status mv_index_describe(const mv_index* ix, char* buf, size_t len) {
            "\"metric\": \"%s\", \"tf32_exact\": %s, \"flat_refine\": \"%s\", \"xmax2\": %.17g, "
            "\"allocator\": \"%s\", \"last_scan\": \"%s\", \"last_coarse\": \"%s\", \"last_chunks\": %lld}",
            ix->d, ix->dpad, ix->nlist, (long long)ix->ntotal, (long long)ix->maxlen,
-           ix->type == MV_IVF_FLAT ? "IVF_FLAT" : "IVF_SQ8", ix->metric == MV_L2 ? "L2" : "IP",
+           ix->type == MV_IVF_FLAT ? "IVF_FLAT" : (ix->type == MV_IVF_SQ8 ? "IVF_SQ8" : "IVF_PQ"),
+           ix->metric == MV_L2 ? "L2" : "IP",
            ix->tf32_exact ? "true" : "false", refine, ix->xmax2, ix->alloc.alloc ? "caller" : "cuda-pool",
            ix->last_scan, ix->last_coarse, (long long)ix->last_chunks);
   return MV_OK;
@@ -1113,7 +1210,11 @@ mv_status mv_index_storage(const mv_index* ix, int64_t* list_off, int64_t* ids, 
   if (list_off) CK(cudaMemcpy(list_off, ix->list_off, sizeof(int64_t) * (ix->nlist + 1), cudaMemcpyDefault));
   if (ids && ix->ntotal) CK(cudaMemcpy(ids, ix->ids, sizeof(int64_t) * ix->ntotal, cudaMemcpyDefault));
   if (codes && ix->ntotal) {
-    if (ix->type != MV_IVF_SQ8) return fail(MV_ESTATE, "codes requested from a non-SQ8 index");
+    if (ix->type == MV_IVF_PQ) {
+      CK(cudaMemcpy(codes, ix->payload, (size_t)ix->ntotal * ix->pq_m, cudaMemcpyDefault));
+      return MV_OK;
+    }
+    if (ix->type != MV_IVF_SQ8) return fail(MV_ESTATE, "codes requested from a FLAT index");
     CK(cudaMemcpy2D(codes, ix->d, ix->payload, ix->dpad, ix->d, ix->ntotal, cudaMemcpyDefault));
   }
   return MV_OK;

@@ -285,6 +285,30 @@ cudaError_t launch_kmeans_accum(const float* x, int64_t n, int d, const int32_t*
                                 unsigned long long* cnt, cudaStream_t st);
 cudaError_t launch_kmeans_update(const double* sums, const unsigned long long* cnt, int nlist, int d, int spherical,
                                  float* c, cudaStream_t st);
+// k_pq.cu: IVF_PQ encode (add path) and the query-major ADC scan
+struct PqScanParams {
+  int metric, dpad, M, dsub, npb, phase, rowcap;
+  int64_t nq;
+  const float* qpad;        // nq x dpad
+  const float* codebooks;   // [M][256][dsub]
+  const int32_t* probes;    // nq x npb
+  const int32_t* ra;        // phase A: the query's seeding lists
+  const uint64_t* tau;      // phase B: emit keys <= tau_q
+  const int64_t* list_off;
+  const uint8_t* codes;     // ntotal x M, list-major
+  const uint32_t* rank;
+  const int64_t* ids;
+  const uint8_t* bitset;
+  int64_t nbits;
+  const int64_t* poff;
+  int32_t* pcnt;
+  uint64_t* part;
+};
+cudaError_t launch_pq_encode(const float* xpad, const int64_t* ids, const int32_t* sorted_idx,
+                             const int32_t* sorted_list, int64_t n, int dpad, int M, int dsub, const float* cb,
+                             const int64_t* new_off, const int64_t* old_off, const int32_t* add_off, uint8_t* payload,
+                             double* norms, int64_t* out_ids, cudaStream_t st);
+cudaError_t launch_pq_scan(const PqScanParams& p, cudaStream_t st);
 // k_filter.cu: strategy E's range bitmap and vector fusion
 cudaError_t launch_attr_bitset(const int64_t* ids, const int64_t* attr, int64_t n, int64_t lo, int64_t hi,
                                uint8_t* bitset, int64_t nbits, cudaStream_t st);

@@ -84,7 +84,8 @@ def _close_all():  # destroy indexes while torch's allocator is still alive
 
 METRICS = {"l2": L.MV_L2, "ip": L.MV_IP, L.MV_L2: L.MV_L2, L.MV_IP: L.MV_IP}
 TYPES = {"flat": L.MV_IVF_FLAT, "ivf_flat": L.MV_IVF_FLAT, "sq8": L.MV_IVF_SQ8, "ivf_sq8": L.MV_IVF_SQ8,
-         L.MV_IVF_FLAT: L.MV_IVF_FLAT, L.MV_IVF_SQ8: L.MV_IVF_SQ8}
+         "pq": L.MV_IVF_PQ, "ivf_pq": L.MV_IVF_PQ,
+         L.MV_IVF_FLAT: L.MV_IVF_FLAT, L.MV_IVF_SQ8: L.MV_IVF_SQ8, L.MV_IVF_PQ: L.MV_IVF_PQ}
 
 
 class Index:
@@ -143,6 +144,25 @@ class Index:
     def set_sq8(self, vmin, vdiff):
         a, b = _as_f32(vmin), _as_f32(vdiff)
         L.check(self._lib.mv_index_set_sq8(self._h, _ptr(a), _ptr(b)))
+
+    def set_pq(self, M: int, codebooks):
+        """IVF_PQ sub-centroids [M, 256, d / M]."""
+        cb = _as_f32(codebooks)
+        L.check(self._lib.mv_index_set_pq(self._h, int(M), _ptr(cb)))
+        self.pq_m = int(M)
+
+    def train_pq(self, M: int, sample, niter: int = 10):
+        """Per-sub-space k-means (mv_kmeans) over a device sample [n, d], n >= 256."""
+        s = _as_f32(sample)
+        L.check(self._lib.mv_index_train_pq(self._h, int(M), _ptr(s), int(s.shape[0]), int(niter)))
+        self.pq_m = int(M)
+
+    def get_pq(self):
+        m = C.c_int32()
+        L.check(self._lib.mv_index_get_pq(self._h, C.byref(m), None))
+        cb = np.empty((m.value, 256, self.d // m.value), np.float32)
+        L.check(self._lib.mv_index_get_pq(self._h, None, _ptr(cb)))
+        return cb
 
     def get_sq8(self):
         vmin = np.empty(self.d, np.float32)
@@ -237,7 +257,8 @@ class Index:
     def storage(self, codes: bool = False):
         off = np.empty(self.nlist + 1, np.int64)
         ids = np.empty(self.ntotal, np.int64)
-        cd = np.empty((self.ntotal, self.d), np.uint8) if codes else None
+        cw = getattr(self, "pq_m", 0) if self.kind == L.MV_IVF_PQ else self.d
+        cd = np.empty((self.ntotal, cw), np.uint8) if codes else None
         L.check(self._lib.mv_index_storage(self._h, _ptr(off), _ptr(ids), _ptr(cd)))
         return off, ids, cd
 
