@@ -98,7 +98,10 @@ MV_API mv_status mv_index_create(int32_t d, mv_metric metric, mv_type type, int3
  * its fallback), 1 = the sample-threshold select, 2 = the staged radix select only, 3 = the
  * streaming select for the seeding bound too), "big_ctas" / "big_cap" (the staged
  * select's first launch: CTAs per SM, 1..4, and candidates staged per query; queries past it are
- * redone with all of shared memory), "workspace_bytes" (per-search
+ * redone with all of shared memory), "async_host" (1: a search whose host buffers are all page-locked
+ * enqueues its copies on `stream` and returns without synchronising -- the caller synchronises
+ * `stream` before reading the results; pageable host buffers still complete synchronously),
+ * "workspace_bytes" (per-search
  * scratch budget: larger batches run as several query chunks; 0 = half of the device memory that was
  * free after the last create/add).
  * value 0 = automatic.  MV_EINVAL for an unknown name or a negative value. */

@@ -13,6 +13,7 @@
 namespace mv {
 
 constexpr int kBoundCap = 4096;   // boundary-bucket capacity (u64) for the radix path
+constexpr int kUnroll = 4;        // warp selects: 32-key chunks loaded per round
 
 __device__ __forceinline__ bool seg_locate(const int32_t* s_pre, int npb, int idx, int& j) {
   // binary search: largest j with s_pre[j] <= idx
@@ -1358,17 +1359,26 @@ __global__ void __launch_bounds__(256) k_final_warp(const int64_t* __restrict__ 
       }
       const int excl = incl - cnt;
       const int T = __shfl_sync(MV_FULL, incl, 31);
-      for (int e0 = 0; e0 < T; e0 += 32) {
-        const int e = e0 + lane;
-        int lo = 0;  // pair holding element e: the largest s with excl[s] <= e
+      // kUnroll chunks' loads in flight per lane (one dependent global load per chunk was the
+      // warp's latency chain: configs[2]'s ~1500 keys per query = ~47 round trips per pass)
+      for (int e00 = 0; e00 < T; e00 += 32 * kUnroll) {
+        uint64_t kk[kUnroll];
 #pragma unroll
-        for (int step = 16; step > 0; step >>= 1) {
-          const int ex = __shfl_sync(MV_FULL, excl, (lo + step) & 31);
-          if (lo + step < 32 && ex <= e) lo += step;
+        for (int u = 0; u < kUnroll; ++u) {
+          const int e = e00 + 32 * u + lane;
+          int lo = 0;  // pair holding element e: the largest s with excl[s] <= e
+#pragma unroll
+          for (int step = 16; step > 0; step >>= 1) {
+            const int ex = __shfl_sync(MV_FULL, excl, (lo + step) & 31);
+            if (lo + step < 32 && ex <= e) lo += step;
+          }
+          const int64_t o = __shfl_sync(MV_FULL, off, lo);
+          const int ex = __shfl_sync(MV_FULL, excl, lo);
+          kk[u] = e < T ? part[o + (e - ex)] : MV_KEY_PAD;
         }
-        const int64_t o = __shfl_sync(MV_FULL, off, lo);
-        const int ex = __shfl_sync(MV_FULL, excl, lo);
-        f(e < T ? part[o + (e - ex)] : MV_KEY_PAD);
+#pragma unroll
+        for (int u = 0; u < kUnroll; ++u)
+          if (e00 + 32 * u < T) f(kk[u]);  // warp-uniform
       }
     }
   };
@@ -1531,22 +1541,31 @@ __global__ void __launch_bounds__(256) k_refine_band(const int64_t* __restrict__
     }
     const int excl = incl - cnt;
     const int T = __shfl_sync(MV_FULL, incl, 31);
-    for (int e0 = 0; e0 < T; e0 += 32) {
-      const int e = e0 + lane;
-      int lo = 0;
+    for (int e00 = 0; e00 < T; e00 += 32 * kUnroll) {
+      uint64_t kk[kUnroll];
 #pragma unroll
-      for (int step = 16; step > 0; step >>= 1) {
-        const int ex = __shfl_sync(MV_FULL, excl, (lo + step) & 31);
-        if (lo + step < 32 && ex <= e) lo += step;
+      for (int u = 0; u < kUnroll; ++u) {  // kUnroll chunks' loads in flight (as k_final_warp)
+        const int e = e00 + 32 * u + lane;
+        int lo = 0;
+#pragma unroll
+        for (int step = 16; step > 0; step >>= 1) {
+          const int ex = __shfl_sync(MV_FULL, excl, (lo + step) & 31);
+          if (lo + step < 32 && ex <= e) lo += step;
+        }
+        const int64_t addr = __shfl_sync(MV_FULL, off, lo) + (e - __shfl_sync(MV_FULL, excl, lo));
+        kk[u] = e < T ? part[addr] : MV_KEY_PAD;
       }
-      const int64_t addr = __shfl_sync(MV_FULL, off, lo) + (e - __shfl_sync(MV_FULL, excl, lo));
-      const uint64_t key = e < T ? part[addr] : MV_KEY_PAD;
-      const bool ps = key != MV_KEY_PAD && key2f((uint32_t)(key >> 32)) <= band;
-      const uint32_t m = __ballot_sync(MV_FULL, ps);
-      if (ps) stage[ns + __popc(m & ((1u << lane) - 1))] = key;  // re-scored at the flush
-      ns += __popc(m);
-      __syncwarp();
-      if (ns >= 32) flush32();
+#pragma unroll
+      for (int u = 0; u < kUnroll; ++u) {
+        if (e00 + 32 * u >= T) break;  // warp-uniform
+        const uint64_t key = kk[u];
+        const bool ps = key != MV_KEY_PAD && key2f((uint32_t)(key >> 32)) <= band;
+        const uint32_t m = __ballot_sync(MV_FULL, ps);
+        if (ps) stage[ns + __popc(m & ((1u << lane) - 1))] = key;  // re-scored at the flush
+        ns += __popc(m);
+        __syncwarp();
+        if (ns >= 32) flush32();
+      }
     }
   }
   if (ns > 0) flush32();

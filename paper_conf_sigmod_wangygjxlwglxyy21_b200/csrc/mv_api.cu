@@ -96,6 +96,17 @@ struct DeviceGuard {
   }
 };
 
+// page-locked host memory (cudaHostAlloc / cudaHostRegister): stream-ordered copies need no sync
+bool is_pinned_ptr(const void* p) {
+  if (p == nullptr) return true;
+  cudaPointerAttributes at;
+  if (cudaPointerGetAttributes(&at, p) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return at.type == cudaMemoryTypeHost || at.type == cudaMemoryTypeDevice || at.type == cudaMemoryTypeManaged;
+}
+
 bool is_host_ptr(const void* p) {
   if (p == nullptr) return false;
   cudaPointerAttributes at;
@@ -338,6 +349,7 @@ mv_status mv_index_set_option(mv_index* ix, const char* name, int64_t value) {
   else if (n == "coarse_nacc") o.coarse_nacc = (int)std::min<int64_t>(value, 4);
   else if (n == "workspace_bytes") o.workspace = value;
   else if (n == "scan_trace") o.scan_trace = value;  // development builds only (-DMV_SCAN_TRACE)
+  else if (n == "async_host") o.async_host = value != 0;
   else if (n == "large_k_select") o.large_k_select = (int)std::min<int64_t>(std::max<int64_t>(value, 0), 3);
   else if (n == "big_cap") o.big_cap = std::max<int64_t>(value, 0);
   else if (n == "big_ctas") o.big_ctas = (int)std::min<int64_t>(std::max<int64_t>(value, 0), 4);
@@ -976,8 +988,14 @@ static mv_status search_impl(mv_index* ix, const float* queries, int64_t nq, int
     CK(cudaMemcpyAsync(distances, D, sizeof(float) * nq * k, cudaMemcpyDeviceToHost, st));
     CK(cudaMemcpyAsync(out_ids, I, sizeof(int64_t) * nq * k, cudaMemcpyDeviceToHost, st));
   }
-  // host inputs/outputs: the call completes before returning (mv.h)
-  if (host_out || sq || sb || sp) CK(cudaStreamSynchronize(st));
+  // host inputs/outputs: the call completes before returning (mv.h) -- unless the caller asked for
+  // stream-ordered host I/O (option "async_host") and every host buffer is page-locked: then the
+  // copies are ordered on `stream` like the kernels (a serving loop overlaps one batch's copies
+  // with another batch's search on a second stream)
+  const bool async_io = ix->opt.async_host && is_pinned_ptr(queries) && is_pinned_ptr(distances) &&
+                        is_pinned_ptr(out_ids) && (!bitset || is_pinned_ptr(bitset)) &&
+                        (!probes_in || is_pinned_ptr(probes_in));
+  if ((host_out || sq || sb || sp) && !async_io) CK(cudaStreamSynchronize(st));
   return MV_OK;
 }
 

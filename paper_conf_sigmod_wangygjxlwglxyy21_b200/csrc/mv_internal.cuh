@@ -182,6 +182,7 @@ struct Options {
   int coarse_nqb = 0, coarse_cs = 0, coarse_epi = 0, coarse_nacc = 0;  // coarse GEMM launch shape
   int64_t workspace = 0;    // per-search scratch budget in bytes (0: half of the free device memory)
   int64_t scan_trace = 0;   // -DMV_SCAN_TRACE builds: device address of the phase-B timeline buffer
+  int async_host = 0;       // 1: searches with pinned host buffers return without synchronising
   int large_k_select = 0;   // k > 256: 0 streaming select (staged radix fallback), 1 sample-threshold select, 2 staged radix only
   int big_ctas = 0;         // k > 256 staged select: CTAs per SM of its first launch (1..4; 0 = 2)
   int64_t big_cap = 0;      // ... and its stage capacity in keys (0: the most that fits big_ctas per SM)

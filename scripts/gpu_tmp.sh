@@ -1,4 +1,3 @@
-O=gpurun_out/q_m; mkdir -p $O
-timeout 600 python -m pytest tests/test_gpu_pq.py -x -q -p no:cacheprovider > $O/pytest_pq.log 2>&1; echo pq=$?; tail -15 $O/pytest_pq.log
-timeout 900 python -m pytest tests -m "gpu and not slow" -q -p no:cacheprovider > $O/pytest.log 2>&1; echo pytest=$?; tail -3 $O/pytest.log
-timeout 600 python bench.py --config c4 --no-cpu-baseline > $O/bench_c4.json 2> $O/bench_c4.err; echo c4=$?
+O=gpurun_out/q_o; mkdir -p $O
+timeout 900 python -m pytest tests -m "gpu and not slow" -x -q -p no:cacheprovider > $O/pytest.log 2>&1; echo pytest=$?; tail -3 $O/pytest.log
+for c in c3 c2 c5 c4; do timeout 600 python bench.py --config $c --no-cpu-baseline > $O/bench_$c.json 2> $O/bench_$c.err; echo $c=$?; done
