@@ -205,6 +205,8 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
   const bool use_norms = p.metric == MV_L2;
   const bool use_ids = p.bitset != nullptr;
   const bool phaseB = p.phase != 0;
+  // phase A of a k > 256 search emits 4-byte distance keys (its tau select needs no id ranks)
+  const bool key32 = !phaseB && p.key32;
   // filter mode: the tensor-core badness is an approximation with a rigorous error bound E_q
   // (SQ8 always; FLAT when the stored values or the queries are not tf32-exact); the keys are
   // re-scored exactly after the scan (k_select.cu k_rekey)
@@ -713,6 +715,18 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
               if (lane == j) mine = __popc(mj[j]);
             }
             uint64_t cp = 0;  // lane j: the address of column j's first reserved slot
+            if (key32) {  // seeding sample of a large-k search: the distance key alone (4 B)
+              if (mine)
+                cp = reinterpret_cast<uint64_t>(reinterpret_cast<uint32_t*>(p.part) + lds_s64(s_base + 8 * (qc + lane)) +
+                                                atoms_add(s_cnt + 4 * (qc + lane), mine));
+#pragma unroll
+              for (int j = 0; j < W; ++j)
+                if (mj[j]) {  // warp-uniform
+                  uint32_t* dst = reinterpret_cast<uint32_t*>(__shfl_sync(MV_FULL, cp, j)) + __popc(mj[j] & ltmask);
+                  if ((pm >> j) & 1) *dst = f2key_fast(bad[j]);
+                }
+              continue;
+            }
             if (mine)
               cp = reinterpret_cast<uint64_t>(p.part + lds_s64(s_base + 8 * (qc + lane)) +
                                               atoms_add(s_cnt + 4 * (qc + lane), mine));

@@ -1073,6 +1073,120 @@ __global__ void __launch_bounds__(NT) k_select_stream(const int64_t* __restrict_
   }
 }
 
+// Seeding bound of a k > 256 search from 4-byte distance keys (phase A with key32): one CTA per
+// query stages its sample (the ra nearest lists' keys) in shared memory, bins it into kBucketBins
+// equal-width bins over [min, max] (a second counting pass over the k-th key's bin when it holds
+// more than 64 keys) and returns that bin's upper edge with every id rank: >= k candidates lie at
+// or below it.  kmin[q] = the smallest key (the streaming final select's lower bin edge).  A query
+// with fewer than k sample keys, or more than `cap`, keeps tau = padding (phase B then emits every
+// candidate of it; the final select's staged fallbacks take any count).
+template <int NT>
+__global__ void __launch_bounds__(NT) k_tau32(const int64_t* __restrict__ poff, const int32_t* __restrict__ pcnt,
+                                             const uint32_t* __restrict__ part32, int64_t nq, int npb,
+                                             const int32_t* __restrict__ nuse, int k, uint64_t* tau_out,
+                                             uint64_t* kmin, int cap) {
+  extern __shared__ __align__(16) uint8_t smem[];
+  uint32_t* hist = reinterpret_cast<uint32_t*>(smem);   // kBucketBins
+  int* misc = reinterpret_cast<int*>(hist + kBucketBins);  // 64
+  int32_t* s_pre = misc + 64;                             // npb + 1
+  uint32_t* keys = reinterpret_cast<uint32_t*>(s_pre + ((npb + 4) & ~3));  // cap
+  const int64_t q = blockIdx.x;
+  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  const int64_t* po = poff + q * npb;
+  const int32_t* pc = pcnt + q * npb;
+  const int nu = nuse ? nuse[q] : npb;
+  for (int i = tid; i < kBucketBins; i += NT) hist[i] = 0;
+  if (wid == 0) {
+    int run = 0;
+    for (int j0 = 0; j0 < nu; j0 += 32) {
+      const int j = j0 + lane;
+      const int c = j < nu ? pc[j] : 0;
+      int incl = c;
+      for (int o = 1; o < 32; o <<= 1) {
+        const int v = __shfl_up_sync(MV_FULL, incl, o);
+        if (lane >= o) incl += v;
+      }
+      if (j < nu) s_pre[j] = run + incl - c;
+      run += __shfl_sync(MV_FULL, incl, 31);
+    }
+    if (lane == 0) {
+      s_pre[nu] = run;
+      misc[48] = (int)0xffffffff;  // min (as u32 via atomicMin on unsigned)
+      misc[49] = 0;                // max
+    }
+  }
+  __syncthreads();
+  const int T = s_pre[nu];
+  if (T < k || T > cap) {
+    if (tid == 0 && kmin) kmin[q] = 0;
+    return;
+  }
+  for (int j = wid; j < nu; j += NT / 32) {
+    const int c = s_pre[j + 1] - s_pre[j];
+    const uint32_t* src = part32 + po[j];
+    const uint32_t dst = (uint32_t)__cvta_generic_to_shared(keys + s_pre[j]);
+    for (int i = lane; i < c; i += 32)
+      asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(dst + 4 * i), "l"(src + i) : "memory");
+  }
+  asm volatile("cp.async.wait_all;" ::: "memory");
+  __syncthreads();
+  uint32_t mn = 0xffffffffu, mx = 0;
+  for (int i = tid; i < T; i += NT) {
+    mn = min(mn, keys[i]);
+    mx = max(mx, keys[i]);
+  }
+  mn = __reduce_min_sync(MV_FULL, mn);
+  mx = __reduce_max_sync(MV_FULL, mx);
+  if (lane == 0) {
+    atomicMin(reinterpret_cast<unsigned*>(misc + 48), mn);
+    atomicMax(reinterpret_cast<unsigned*>(misc + 49), mx);
+  }
+  __syncthreads();
+  mn = (uint32_t)misc[48];
+  mx = (uint32_t)misc[49];
+  const uint32_t span = mx - mn;
+  const int sh = span ? max(0, 32 - __clz((int)span) - 11) : 0;  // (x - mn) >> sh < 2048
+  for (int i = tid; i < T; i += NT) atomicAdd(hist + ((keys[i] - mn) >> sh), 1u);
+  __syncthreads();
+  block_scan_bins<NT>(hist, misc, k - 1);
+  const int bs = misc[40], st = misc[41], nb = misc[42];
+  uint64_t edge = (uint64_t)mn + (((uint64_t)bs + 1) << sh) - 1;
+  if (nb > 64 && sh > 0) {
+    const int sh2 = max(0, sh - 11);
+    const uint32_t b0 = mn + ((uint32_t)bs << sh);
+    for (int i = tid; i < kBucketBins; i += NT) hist[i] = 0;
+    __syncthreads();
+    for (int i = tid; i < T; i += NT) {
+      const uint32_t x = keys[i];
+      if ((int)((x - mn) >> sh) == bs) atomicAdd(hist + ((x - b0) >> sh2), 1u);
+    }
+    __syncthreads();
+    block_scan_bins<NT>(hist, misc, k - 1 - st);
+    edge = (uint64_t)b0 + (((uint64_t)misc[40] + 1) << sh2) - 1;
+  }
+  if (tid == 0) {
+    edge = min(edge, (uint64_t)mx);
+    tau_out[q] = (edge << 32) | 0xffffffffull;
+    if (kmin) kmin[q] = (uint64_t)mn << 32;
+  }
+}
+
+cudaError_t launch_tau32(const int64_t* poff, const int32_t* pcnt, const uint64_t* part, int64_t nq, int npb,
+                         const int32_t* nuse, int k, uint64_t* tau, uint64_t* kmin, int64_t tmax, cudaStream_t st) {
+  if (nq == 0) return cudaSuccess;
+  constexpr int NT = 1024;
+  const size_t fixed = kBucketBins * 4 + 64 * 4 + (size_t)((npb + 4) & ~3) * 4;
+  // two CTAs per SM when the sample fits (configs[3]: need + capA ~ 17k keys), else all of it
+  int cap = (int)min64(tmax, (int64_t)((112 * 1024 - fixed) / 4));
+  if (cap < tmax) cap = (int)min64(tmax, (int64_t)((226 * 1024 - fixed) / 4));
+  const size_t smem = fixed + (size_t)cap * 4;
+  cudaError_t e = cudaFuncSetAttribute(k_tau32<NT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  k_tau32<NT><<<(unsigned)nq, NT, smem, st>>>(poff, pcnt, reinterpret_cast<const uint32_t*>(part), nq, npb, nuse, k,
+                                              tau, kmin, cap);
+  return cudaGetLastError();
+}
+
 static cudaError_t launch_big_select(const int64_t* poff, const int32_t* pcnt, const uint64_t* part, int64_t nq,
                                      int npb, int k, int metric, const int64_t* sorted_ids, float* out_d,
                                      int64_t* out_i, const int32_t* nuse, uint64_t* tau, int64_t tmax,

@@ -854,6 +854,10 @@ static mv_status search_chunk(mv_index* ix, const float* q, int64_t nq, int32_t 
   tp.bq = b.bq; tp.nbq = nent; tp.boff = b.boff; tp.witems = b.witems; tp.nlist = nlist; tp.cfg = qcfg;
   tp.poff = b.poff; tp.pcnt = b.pcnt; tp.part = part; tp.tau = tau;
   tp.approx_always = approx_always ? 1 : 0; tp.qerr = qerr;
+  // k > 256 with seeding: phase A emits 4-byte distance keys and k_tau32 takes the bound from them
+  // (half the sample's bytes written and read; large_k_select = 2 keeps the 8-byte keys)
+  const bool key32 = k > 256 && split && !pq && ix->opt.large_k_select == 0;
+  tp.key32 = key32 ? 1 : 0;
   tp.prof = nullptr;
   // phase A (or, without seeding, the whole scan emitting every candidate) ...
   tp.phase = 0;
@@ -871,6 +875,10 @@ static mv_status search_chunk(mv_index* ix, const float* q, int64_t nq, int32_t 
   prof_mark(ix, st);
   if (split) {
     // ... tau_q = k-th best key of phase A (phase A emits < need + capA candidates per query) ...
+    if (key32)
+      CK(launch_tau32(b.poff + npairs, b.pcnt + npairs, part, nq, npb, ra, k, tau, kmin,
+                      std::min<int64_t>(tmax, pa.need + pa.capA), st));
+    else
     CK(launch_tau_select(b.poff + npairs, b.pcnt + npairs, part, nq, npb, ra, k, tau,
                          std::min<int64_t>(tmax, pa.need + pa.capA), over, nullptr,
                          BigSel{ix->opt.large_k_select, ix->opt.big_ctas, ix->opt.big_cap, std::min<int64_t>(tmax, pa.need),

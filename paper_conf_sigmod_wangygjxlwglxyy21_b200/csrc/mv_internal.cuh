@@ -329,6 +329,7 @@ struct TcScanParams {
   const int32_t* cfg;      // device {query chunk, planes} of this search (launch_scan_cfg)
   int nlist;               // virtual list v >= nlist is list v - nlist (phase-B pairs)
   int phase;               // 0: seeding phase A (emit every candidate); 1: phase B (emit keys <= tau_q)
+  int key32;               // phase A: emit 4-byte distance keys into a u32 view of the regions (k > 256)
   int rowcap;              // rows scanned per list in this launch (phase A: capA; else INT_MAX)
   int64_t nq;              // FLAT query planes are plane-major [2][nq][dpad]
   int off_x, off_q, q_bytes, off_meta, meta_bytes, off_side, off_bar, smem_total;
@@ -414,6 +415,9 @@ cudaError_t launch_hilo(const float* x, int64_t n, int d, int dpad, float* out, 
 cudaError_t launch_final_select(const int64_t* poff, const int32_t* pcnt, const uint64_t* part, int64_t nq, int npb,
                                 int k, int metric, const int64_t* sorted_ids, float* out_d, int64_t* out_i,
                                 int64_t tmax, uint8_t* over, BigSel bsel, cudaStream_t st);
+// k > 256 seeding bound from phase A's 4-byte distance keys (scan key32); tmax bounds a query's sample
+cudaError_t launch_tau32(const int64_t* poff, const int32_t* pcnt, const uint64_t* part, int64_t nq, int npb,
+                         const int32_t* nuse, int k, uint64_t* tau, uint64_t* kmin, int64_t tmax, cudaStream_t st);
 cudaError_t launch_tau_select(const int64_t* poff, const int32_t* pcnt, const uint64_t* part, int64_t nq, int npb,
                               const int32_t* nuse, int k, uint64_t* tau, int64_t tmax, uint8_t* over,
                               const int* gate, BigSel bsel, cudaStream_t st);
