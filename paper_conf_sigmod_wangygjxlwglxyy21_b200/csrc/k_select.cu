@@ -846,7 +846,7 @@ __global__ void __launch_bounds__(kBigThreads) k_final_sample(const int64_t* __r
 //     k are the answer.  A query whose gathered keys exceed cap is flagged in redo[] for the staged
 //     select.
 template <int NT, bool TAU>
-__global__ void __launch_bounds__(NT) k_select_stream(const int64_t* __restrict__ poff, const int32_t* __restrict__ pcnt,
+__global__ void __launch_bounds__(NT, TAU ? 1 : 3) k_select_stream(const int64_t* __restrict__ poff, const int32_t* __restrict__ pcnt,
                                                       const uint64_t* __restrict__ part, int64_t nq, int npb, int k,
                                                       int metric, const int64_t* __restrict__ sorted_ids, float* out_d,
                                                       int64_t* out_i, int cap, const int32_t* __restrict__ nuse,
