@@ -730,7 +730,9 @@ def run_reference(args, cfg, cname):
     bsn = bs.cpu().numpy() if bs is not None else None
     del X
     ot = OracleTimer(cfg, Xn, np.arange(cfg["n"], dtype=np.int64), lists, Cn, sq8, bsn)
-    per_step = args.oracle_sample or {"c1": 100, "c2": 400, "c3": 100, "c4": 48}.get(cname, 100)
+    # (each oracle call re-lays out the whole index per worker: ~10 queries per worker per step
+    # amortise it the way cpu_baseline's single call does)
+    per_step = args.oracle_sample or {"c1": 100, "c2": 400, "c3": 160, "c4": 160}.get(cname, 100)
     vals = []
     try:
         for i in range(args.warmup + args.steps):

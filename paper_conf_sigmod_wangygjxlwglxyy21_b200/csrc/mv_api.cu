@@ -276,7 +276,7 @@ extern "C" {
 
 const char* mv_last_error(void) { return g_err.c_str(); }
 
-const char* mv_version(void) { return "libmv 0.2 (sm_100a; IVF_FLAT/IVF_SQ8; L2/IP)"; }
+const char* mv_version(void) { return "libmv 0.2 (sm_100a; IVF_FLAT/IVF_SQ8/IVF_PQ; L2/IP)"; }
 
 int64_t mv_index_ntotal(const mv_index* ix) { return ix ? ix->ntotal : 0; }
 
