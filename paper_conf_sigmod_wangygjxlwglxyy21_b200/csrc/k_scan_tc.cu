@@ -295,29 +295,40 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
 
   if (warp == 0) {
     // ------------------------------------------------------------------ TMA producer
-    if (lane == 0) {
-      uint32_t it = 0, tcount = 0;
+    // the whole warp runs the loop (warp-uniform values), one elected lane issues each copy; ring
+    // positions advance without divisions (as the MMA warp)
+    {
+      uint32_t s = 0, sph = 0;    // X ring stage / phase
+      uint32_t ts = 0, tph = 0;   // side-data slot / phase
+#ifdef MV_SCAN_TRACE
+      uint32_t it = 0;
+#endif
       const uint32_t side_tx = 528 + (use_norms ? 1040 : 0) + (use_ids ? 1040 : 0);
       // list tiles stream through L2 evict-first, except a list with sibling items: its neighbours
       // in the schedule read the same tiles at about the same time
       const uint64_t pol_first = l2_evict_first_policy(), pol_normal = l2_evict_normal_policy();
       // the item positions, in the gatherer's order
-      auto take = [&](uint32_t j) {
-        const uint32_t sl = j % kRing;
-        mbar_wait(&sfull[sl], (j / kRing) & 1);
-        const int v = ring[sl];
-        mbar_arrive(&sempty[sl]);
+      uint32_t rs = 0, rph = 0;
+      auto take = [&]() {
+        mbar_wait(&sfull[rs], rph);
+        const int v = ring[rs];
+        __syncwarp();
+        mbar_arrive_elect(&sempty[rs]);
+        if (++rs == (uint32_t)kRing) {
+          rs = 0;
+          rph ^= 1;
+        }
         return v;
       };
       // three-deep load pipeline (ItemRaw): item i+1's work info is ready when item i starts
-      int q0 = take(0), q1 = take(1), q2 = take(2);
+      int q0 = take(), q1 = take(), q2 = take();
       int2 it3 = q2 < nwork ? p.witems[q2] : make_int2(0, 0);
       ItemRaw r2{};
       if (q1 < nwork) r2 = item_raw(p, p.witems[q1]);
       WorkInfo wn = q0 < nwork ? work_info(p, q0, QC) : WorkInfo{};
-      for (uint32_t i = 0; q0 < nwork; ++i) {
+      while (q0 < nwork) {
         const WorkInfo wi = wn;
-        const int q3 = q2 < nwork ? take(i + 3) : nwork;  // (positions only grow)
+        const int q3 = q2 < nwork ? take() : nwork;  // (positions only grow)
         if (q1 < nwork) wn = work_info_raw(p, r2, QC);
         if (q2 < nwork) r2 = item_raw(p, it3);
         if (q3 < nwork) it3 = p.witems[q3];
@@ -325,38 +336,47 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
         q1 = q2;
         q2 = q3;
         const uint64_t pol = wi.multi ? pol_normal : pol_first;
-        for (int t = 0; t < wi.ntiles; ++t, ++tcount) {
+        for (int t = 0; t < wi.ntiles; ++t) {
           const int row0 = (int)(wi.lstart + t * 128);
-          const uint32_t ts = tcount % NTS, tr = tcount / NTS;
-          mbar_wait(&empty_t[ts], (tr & 1) ^ 1);
+          mbar_wait(&empty_t[ts], tph ^ 1);
 #ifdef MV_EXP_NOSIDE  // timing experiment only (wrong results): no side data
-          mbar_arrive(&full_t[ts]);
+          mbar_arrive_elect(&full_t[ts]);
           (void)side_tx;
 #else
-          mbar_expect_tx(&full_t[ts], side_tx);
+          mbar_expect_tx_elect(&full_t[ts], side_tx);
           uint8_t* sd = side + ts * SIDEB;
-          bulk_g2s(sd + kSideRank, p.rank + (row0 & ~3), 528, &full_t[ts]);
-          if (use_norms) bulk_g2s(sd, p.norms + (row0 & ~1), 1040, &full_t[ts]);
-          if (use_ids) bulk_g2s(sd + kSideIds, p.ids + (row0 & ~1), 1040, &full_t[ts]);
+          bulk_g2s_elect(sd + kSideRank, p.rank + (row0 & ~3), 528, &full_t[ts]);
+          if (use_norms) bulk_g2s_elect(sd, p.norms + (row0 & ~1), 1040, &full_t[ts]);
+          if (use_ids) bulk_g2s_elect(sd + kSideIds, p.ids + (row0 & ~1), 1040, &full_t[ts]);
 #endif
-          for (int c = 0; c < nchunks; ++c, ++it) {
-            const uint32_t s = it % nstage, r = it / nstage;
-            mbar_wait(&empty_x[s], (r & 1) ^ 1);
-            MV_TRACE(0, it);
-            // a list's tail tile loads roundup16(rows) rows as 64/32/16-row boxes (< 16 rows past the
-            // list end); its stale smem rows beyond are masked lanes of the MMA's M = 128
-            const int rows = min(128, wi.len - t * 128);
+          if (++ts == (uint32_t)NTS) {
+            ts = 0;
+            tph ^= 1;
+          }
+          // a list's tail tile loads roundup16(rows) rows as 64/32/16-row boxes (< 16 rows past the
+          // list end); its stale smem rows beyond are masked lanes of the MMA's M = 128
+          const int rows = min(128, wi.len - t * 128);
+          const int r16 = (rows + 15) & ~15;
+          for (int c = 0; c < nchunks; ++c) {
+            mbar_wait(&empty_x[s], sph ^ 1);
+#ifdef MV_SCAN_TRACE
+            if (lane == 0) MV_TRACE(0, it);
+            ++it;
+#endif
             uint8_t* dst = Xs + s * 128 * ATOM;
             if (rows > 112) {
-              mbar_expect_tx(&full_x[s], 128 * ATOM);
-              tma_load_2d_hint(dst, &xm.m[0], &full_x[s], c * ATOM / ESZ, row0, pol);
+              mbar_expect_tx_elect(&full_x[s], 128 * ATOM);
+              tma_load_2d_hint_elect(dst, &xm.m[0], &full_x[s], c * ATOM / ESZ, row0, pol);
             } else {
-              const int r16 = (rows + 15) & ~15;
-              mbar_expect_tx(&full_x[s], r16 * ATOM);
+              mbar_expect_tx_elect(&full_x[s], r16 * ATOM);
               int o = 0;
-              if (r16 & 64) { tma_load_2d_hint(dst, &xm.m[1], &full_x[s], c * ATOM / ESZ, row0, pol); o += 64; }
-              if (r16 & 32) { tma_load_2d_hint(dst + o * ATOM, &xm.m[2], &full_x[s], c * ATOM / ESZ, row0 + o, pol); o += 32; }
-              if (r16 & 16) tma_load_2d_hint(dst + o * ATOM, &xm.m[3], &full_x[s], c * ATOM / ESZ, row0 + o, pol);
+              if (r16 & 64) { tma_load_2d_hint_elect(dst, &xm.m[1], &full_x[s], c * ATOM / ESZ, row0, pol); o += 64; }
+              if (r16 & 32) { tma_load_2d_hint_elect(dst + o * ATOM, &xm.m[2], &full_x[s], c * ATOM / ESZ, row0 + o, pol); o += 32; }
+              if (r16 & 16) tma_load_2d_hint_elect(dst + o * ATOM, &xm.m[3], &full_x[s], c * ATOM / ESZ, row0 + o, pol);
+            }
+            if (++s == (uint32_t)nstage) {
+              s = 0;
+              sph ^= 1;
             }
           }
         }
@@ -364,12 +384,19 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
     }
   } else if (warp == 1) {
     // ------------------------------------------------------------------ MMA issuer
-    if (lane == 0) {
-      uint32_t it = 0, titer = 0;
+    // the whole warp runs the loop (warp-uniform values in uniform registers), one elected lane
+    // issues each tcgen05 instruction; ring / accumulator positions advance without divisions
+    {
+      uint32_t s = 0, sph = 0;     // X ring stage and its phase
+      uint32_t acc = 0, aph = 0;   // TMEM accumulator and its phase
+#ifdef MV_SCAN_TRACE
+      uint32_t it = 0;
+#endif
+      uint32_t titer = 0;
       for (uint32_t wcount = 0;; ++wcount) {
         const uint32_t b = wcount & 1;
         mbar_wait(&full_q[b], (wcount >> 1) & 1);
-        MV_TRACE(1, wcount);
+        if (lane == 0) MV_TRACE(1, wcount);
         tc_fence_after();
         const WorkInfo wi = *meta_at(metab + b * p.meta_bytes, QCP).wi;
         if (wi.ntiles < 0) break;  // the gatherer's end marker
@@ -378,41 +405,52 @@ __global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
         const uint32_t idesc = TYPE == MV_IVF_FLAT ? idesc_tf32(N) : idesc_u8s8(N);
         const uint32_t qbase = smem_u32(Qs + b * p.q_bytes);
         for (int t = 0; t < wi.ntiles; ++t, ++titer) {
-          const uint32_t a = titer % NACC;
-          mbar_wait(&tempty[a], ((titer / NACC) & 1) ^ 1);
-          MV_TRACE(2, titer);
+          mbar_wait(&tempty[acc], aph ^ 1);
+          if (lane == 0) MV_TRACE(2, titer);
           tc_fence_after();
-          const uint32_t dcol = tmem + a * p.ncol;
-          for (int c = 0; c < nchunks; ++c, ++it) {
-            const uint32_t s = it % nstage;
-            mbar_wait(&full_x[s], (it / nstage) & 1);
-            MV_TRACE(7, it);
+          const uint32_t dcol = tmem + acc * p.ncol;
+          for (int c = 0; c < nchunks; ++c) {
+            mbar_wait(&full_x[s], sph);
+#ifdef MV_SCAN_TRACE
+            if (lane == 0) MV_TRACE(7, it);
+            ++it;
+#endif
             tc_fence_after();
             const uint32_t xb = smem_u32(Xs + s * 128 * ATOM);
             const uint32_t qb = qbase + c * N * ATOM;
-#pragma unroll
 #ifdef MV_EXP_NOMMA  // timing experiment only (wrong results): stages released without MMAs
             (void)xb; (void)qb; (void)dcol; (void)idesc;
-            mbar_arrive(&empty_x[s]);
-          }
-          mbar_arrive(&tfull[a]);
+            if (lane == 0) mbar_arrive(&empty_x[s]);
 #else
+#pragma unroll
             for (int ks = 0; ks < ATOM / 32; ++ks) {
               const uint64_t ad = kmajor_desc(xb + ks * 32, ATOM);
               const uint64_t bd = kmajor_desc(qb + ks * 32, ATOM);
-              if (TYPE == MV_IVF_FLAT) mma_tf32(dcol, ad, bd, idesc, (c | ks) != 0);
-              else mma_i8(dcol, ad, bd, idesc, (c | ks) != 0);
+              if (TYPE == MV_IVF_FLAT) mma_tf32_elect(dcol, ad, bd, idesc, (c | ks) != 0);
+              else mma_i8_elect(dcol, ad, bd, idesc, (c | ks) != 0);
             }
-            mma_commit(&empty_x[s]);
-          }
-          mma_commit(&tfull[a]);
+            mma_commit_elect(&empty_x[s]);
 #endif
-          MV_TRACE(3, titer);
+            if (++s == (uint32_t)nstage) {
+              s = 0;
+              sph ^= 1;
+            }
+          }
+#ifdef MV_EXP_NOMMA
+          if (lane == 0) mbar_arrive(&tfull[acc]);
+#else
+          mma_commit_elect(&tfull[acc]);
+#endif
+          if (lane == 0) MV_TRACE(3, titer);
+          if (++acc == (uint32_t)NACC) {
+            acc = 0;
+            aph ^= 1;
+          }
         }
-        mma_commit(&empty_q[b]);
+        mma_commit_elect(&empty_q[b]);
       }
 #ifdef MV_SCAN_TRACE
-      if (p.prof && blockIdx.x < 148) {
+      if (lane == 0 && p.prof && blockIdx.x < 148) {
         p.prof[8 * 1024 + blockIdx.x * 3 + 1] = gtimer();
         p.prof[8 * 1024 + blockIdx.x * 3 + 2] = titer;
       }

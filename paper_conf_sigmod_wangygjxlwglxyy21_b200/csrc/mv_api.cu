@@ -789,11 +789,13 @@ static mv_status search_chunk(mv_index* ix, const float* q, int64_t nq, int32_t 
     pa.need = std::max<int64_t>(pa.need, std::min<int64_t>(bal, 65536));
   }
   if (ix->opt.need > 0) pa.need = std::max<int64_t>(2 * (int64_t)k, ix->opt.need);
-  // Rows per list of the sample: ~sqrt(64 need), i.e. the sample spreads over ~sqrt(need / 64)
-  // nearest lists (measured, capA sweep: configs[2] 256 rows 2.85M qps vs whole lists 2.71M;
-  // configs[4] 128 rows best; configs[1] 128 rows vs 64: 16.0M vs 14.7M), at least 128 rows
+  // Rows per list of the sample: ~sqrt(f need), i.e. the sample spreads over ~sqrt(need / f)
+  // nearest lists, at least 128 rows.  f = 64 (configs[3]: capA 1024 best of 128..1024;
+  // configs[2], k = 100: 240 rows, 464 measured 5% slower); f = 256 for k <= 32 (round-2 sweep:
+  // configs[4] capA 384 vs 192: 7.68 vs 7.90 ms; configs[1] unchanged: its sample is 128 rows)
+  const double capf = k <= 32 ? 256.0 : 64.0;
   pa.capA = std::max<int64_t>(128, std::min<int64_t>((pa.need + 15) & ~(int64_t)15,
-                                                     ((int64_t)std::sqrt(64.0 * pa.need) + 15) & ~(int64_t)15));
+                                                     ((int64_t)std::sqrt(capf * pa.need) + 15) & ~(int64_t)15));
   if (ix->opt.capa > 0) pa.capA = std::max<int64_t>(16, (ix->opt.capa + 15) & ~15ll);
   pa.list_off = ix->list_off;
   // FLAT with tf32-exact stored values: two-plane (hi/lo) items when some query needs its lo plane;
