@@ -297,48 +297,62 @@ __global__ void __launch_bounds__(kQmThreads, 1)
       for (int pl = 0; pl < (qlo ? 2 : 1); ++pl)
         for (int c = 0; c < nchunks; ++c)
           tma_load_2d(Aq + (pl * nchunks + c) * PBYTES, &qmap, full_a, c * 32, pl * (int)p.nq + q0);
-      uint32_t it = 0;
-      for (int t = t0, tl = 0; t < t1; ++t, ++tl) {
-        const uint32_t a = tl % kQmAcc;
+      uint32_t s = 0, sph = 0, a = 0, aph = 0;
+      for (int t = t0; t < t1; ++t) {
         // the tile's centroid norms, once the epilogue is done with the slot's previous tile
-        mbar_wait(&tempty[a], ((tl / kQmAcc) & 1) ^ 1);
+        mbar_wait(&tempty[a], aph ^ 1);
         mbar_expect_tx(&full_c[a], 512);
         bulk_g2s(cns + a * 128, p.cnorm + (int64_t)t * 128, 512, &full_c[a]);
-        for (int c = 0; c < nchunks; ++c, ++it) {
-          const uint32_t s = it % nstage, r = it / nstage;
-          mbar_wait(&empty_b[s], (r & 1) ^ 1);
+        if (++a == (uint32_t)kQmAcc) {
+          a = 0;
+          aph ^= 1;
+        }
+        for (int c = 0; c < nchunks; ++c) {
+          mbar_wait(&empty_b[s], sph ^ 1);
           mbar_expect_tx(&full_b[s], 2 * PBYTES);
           tma_load_2d(Bs + s * 2 * PBYTES, &cmap, &full_b[s], c * 32, t * 128);
           tma_load_2d(Bs + s * 2 * PBYTES + PBYTES, &cmap, &full_b[s], c * 32, p.nlist + t * 128);
+          if (++s == (uint32_t)nstage) {
+            s = 0;
+            sph ^= 1;
+          }
         }
       }
     }
   } else if (warp == 1) {
-    if (lane == 0) {
+    // the whole warp runs the loop, one elected lane issues (k_scan_tc.cu: no per-MMA R2UR elect
+    // loops, no divisions for the ring positions)
+    {
       mbar_wait(full_a, 0);
       tc_fence_after();
       const uint32_t id = idesc_tf32(128);
-      uint32_t it = 0;
-      for (int t = t0, tl = 0; t < t1; ++t, ++tl) {
-        const uint32_t a = tl % kQmAcc;
-        mbar_wait(&tempty[a], ((tl / kQmAcc) & 1) ^ 1);
+      uint32_t s = 0, sph = 0, a = 0, aph = 0;
+      for (int t = t0; t < t1; ++t) {
+        mbar_wait(&tempty[a], aph ^ 1);
         tc_fence_after();
         const uint32_t d = tmem + a * 128;
-        for (int c = 0; c < nchunks; ++c, ++it) {
-          const uint32_t s = it % nstage;
-          mbar_wait(&full_b[s], (it / nstage) & 1);
+        for (int c = 0; c < nchunks; ++c) {
+          mbar_wait(&full_b[s], sph);
           tc_fence_after();
           const uint32_t qh = smem_u32(Aq + c * PBYTES), ql = smem_u32(Aq + (nchunks + c) * PBYTES);
           const uint32_t ch = smem_u32(Bs + s * 2 * PBYTES), cl = ch + PBYTES;
 #pragma unroll
           for (int ks = 0; ks < 4; ++ks) {
-            mma_tf32(d, kmajor_desc(qh + ks * 32, ATOM), kmajor_desc(ch + ks * 32, ATOM), id, (c | ks) != 0);
-            mma_tf32(d, kmajor_desc(qh + ks * 32, ATOM), kmajor_desc(cl + ks * 32, ATOM), id, 1);
-            if (qlo) mma_tf32(d, kmajor_desc(ql + ks * 32, ATOM), kmajor_desc(ch + ks * 32, ATOM), id, 1);
+            mma_tf32_elect(d, kmajor_desc(qh + ks * 32, ATOM), kmajor_desc(ch + ks * 32, ATOM), id, (c | ks) != 0);
+            mma_tf32_elect(d, kmajor_desc(qh + ks * 32, ATOM), kmajor_desc(cl + ks * 32, ATOM), id, 1);
+            if (qlo) mma_tf32_elect(d, kmajor_desc(ql + ks * 32, ATOM), kmajor_desc(ch + ks * 32, ATOM), id, 1);
           }
-          mma_commit(&empty_b[s]);
+          mma_commit_elect(&empty_b[s]);
+          if (++s == (uint32_t)nstage) {
+            s = 0;
+            sph ^= 1;
+          }
         }
-        mma_commit(&tfull[a]);
+        mma_commit_elect(&tfull[a]);
+        if (++a == (uint32_t)kQmAcc) {
+          a = 0;
+          aph ^= 1;
+        }
       }
     }
   } else {
