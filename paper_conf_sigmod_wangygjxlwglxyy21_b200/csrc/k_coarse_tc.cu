@@ -291,29 +291,27 @@ __global__ void __launch_bounds__(kQmThreads, 1)
   const uint32_t tmem = *tslot;
 
   if (warp == 0) {
-    // the whole warp runs the producer loop, one elected lane issues (as the MMA warp)
-    {
-      const uint64_t pol = l2_evict_normal_policy();
+    if (lane == 0) {
       // the query block: hi rows [q0, q0+128) (and lo rows [nq + q0, ...)) of the plane-major matrix
-      mbar_expect_tx_elect(full_a, (qlo ? 2 : 1) * nchunks * PBYTES);
+      mbar_expect_tx(full_a, (qlo ? 2 : 1) * nchunks * PBYTES);
       for (int pl = 0; pl < (qlo ? 2 : 1); ++pl)
         for (int c = 0; c < nchunks; ++c)
-          tma_load_2d_hint_elect(Aq + (pl * nchunks + c) * PBYTES, &qmap, full_a, c * 32, pl * (int)p.nq + q0, pol);
+          tma_load_2d(Aq + (pl * nchunks + c) * PBYTES, &qmap, full_a, c * 32, pl * (int)p.nq + q0);
       uint32_t s = 0, sph = 0, a = 0, aph = 0;
       for (int t = t0; t < t1; ++t) {
         // the tile's centroid norms, once the epilogue is done with the slot's previous tile
         mbar_wait(&tempty[a], aph ^ 1);
-        mbar_expect_tx_elect(&full_c[a], 512);
-        bulk_g2s_elect(cns + a * 128, p.cnorm + (int64_t)t * 128, 512, &full_c[a]);
+        mbar_expect_tx(&full_c[a], 512);
+        bulk_g2s(cns + a * 128, p.cnorm + (int64_t)t * 128, 512, &full_c[a]);
         if (++a == (uint32_t)kQmAcc) {
           a = 0;
           aph ^= 1;
         }
         for (int c = 0; c < nchunks; ++c) {
           mbar_wait(&empty_b[s], sph ^ 1);
-          mbar_expect_tx_elect(&full_b[s], 2 * PBYTES);
-          tma_load_2d_hint_elect(Bs + s * 2 * PBYTES, &cmap, &full_b[s], c * 32, t * 128, pol);
-          tma_load_2d_hint_elect(Bs + s * 2 * PBYTES + PBYTES, &cmap, &full_b[s], c * 32, p.nlist + t * 128, pol);
+          mbar_expect_tx(&full_b[s], 2 * PBYTES);
+          tma_load_2d(Bs + s * 2 * PBYTES, &cmap, &full_b[s], c * 32, t * 128);
+          tma_load_2d(Bs + s * 2 * PBYTES + PBYTES, &cmap, &full_b[s], c * 32, p.nlist + t * 128);
           if (++s == (uint32_t)nstage) {
             s = 0;
             sph ^= 1;
