@@ -461,12 +461,35 @@ __global__ void __launch_bounds__(256) k_group_bound(const uint32_t* __restrict_
     }
     return (int)__reduce_add_sync(MV_FULL, (uint32_t)c);
   };
-  // the nprobe-th smallest key b: the largest b with count(< b) < nprobe
-  uint32_t b = 0;
-  for (int bit = 31; bit >= 0; --bit) {
+  // the nprobe-th smallest key b: the largest b with count(< b) < nprobe.  The bisection starts
+  // below the bits every group key shares (the row's min and max agree above them: b lies in
+  // [min, max], so its higher bits are those of min)
+  uint32_t mn = 0xffffffffu, mx = 0;
+  if (REG) {
+#pragma unroll
+    for (int i = 0; i < NR; ++i)
+      if (i * 32 + lane < ng) {
+        mn = min(mn, v[i]);
+        mx = max(mx, v[i]);
+      }
+  } else {
+    for (int i = 0; i < nrow; ++i)
+      if (i * 32 + lane < ng) {
+        const uint32_t x = val(i);
+        mn = min(mn, x);
+        mx = max(mx, x);
+      }
+  }
+  mn = __reduce_min_sync(MV_FULL, mn);
+  mx = __reduce_max_sync(MV_FULL, mx);
+  // (fewer groups than nprobe: every group is selected, b = the full 32-bit search's 0xffffffff)
+  const int top = ng < nprobe ? 31 : (mn == mx ? -1 : 31 - __clz((int)(mn ^ mx)));  // highest differing bit
+  uint32_t b = top >= 31 ? 0u : (mn >> (top + 1)) << (top + 1);
+  for (int bit = top; bit >= 0; --bit) {
     const uint32_t trial = b | (1u << bit);
     if (count_below(trial) < nprobe) b = trial;
   }
+  if (top < 0) b = mn;  // every group key equal (and ng >= nprobe)
   // among the groups with key == b (group order), the (nprobe - count(< b))-th; then the ranks
   int r = nprobe - count_below(b);
   uint32_t gsel = 0xffffffffu;

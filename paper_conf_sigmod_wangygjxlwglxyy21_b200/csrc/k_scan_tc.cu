@@ -848,14 +848,27 @@ __global__ void k_qplanes(int type, const float* __restrict__ qpad, int64_t nq, 
       // the scale is rounded up to fp32 first, so the digits and the epilogue use the same exact s
       const double s = amax > 0.0 ? (double)__double2float_ru(amax / 127.0) : 1.0;
       int8_t* o = reinterpret_cast<int8_t*>(out) + q * kSq8Planes * dpad;
+      // the digits' residual r_j = w_j / s - (d0 + d1 / 2^7 + ...), summed by sign: the filter's
+      // error from the digits is s sum_j r_j c_j with codes c_j in [0, 255], at most
+      // 255 s max(sum r+, sum r-) -- the actual residuals of this query, not the worst case
+      double rp = 0.0, rn = 0.0;
       for (int j = lane; j < dpad; j += 32) {
         double u = (double)x[j] * ((double)vdiff[j] / 255.0) / s;  // in [-127, 127]
+        double scale = 1.0;
 #pragma unroll
         for (int dgt = 0; dgt < kSq8Planes; ++dgt) {  // base-2^7 signed digits: u ~ d0 + d1/2^7
           const double dd = fmin(fmax(rint(u), -127.0), 127.0);
           o[dgt * dpad + j] = (int8_t)dd;
           u = (u - dd) * 128.0;
+          scale *= 1.0 / 128.0;
         }
+        const double r = u * scale;  // (the last digit's remainder, in units of s)
+        rp += fmax(r, 0.0);
+        rn += fmax(-r, 0.0);
+      }
+      for (int o2 = 16; o2 > 0; o2 >>= 1) {
+        rp += __shfl_xor_sync(MV_FULL, rp, o2);
+        rn += __shfl_xor_sync(MV_FULL, rn, o2);
       }
       if (lane == 0) {
         qscale[q] = (float)s;
@@ -863,15 +876,15 @@ __global__ void k_qplanes(int type, const float* __restrict__ qpad, int64_t nq, 
         // Filter-mode bound E_q >= |fp32 filter badness - the oracle's badness|:
         //   the fp32 conversions, three FMAs and the expansion: 2^-21 (||q||^2 + X^2 + 2 (s Amax + |q.a|)),
         //   Amax = the largest |digit-weighted partial| (127 * 255 * dpad * (1 + 2^-7 + ...));
-        //   the digits' residual (<= 2^-22 s per weight, times the codes): s 2^-22 255 dpad;
+        //   the digits' residual: 255 s max(sum r+, sum r-) over this query's remainders r_j;
         //   the oracle's fp32 decode vmin + ((c + 0.5)/255) vdiff vs the exact affine map:
         //   2^-22 sum |q_j| (2 vdiff_j + |vmin_j|);  L2 doubles the dot's share;  + 2^-22 (||q||^2 + X^2)
         //   for the roundings of the result.
         if (qerr) {
           const double amx = 127.0 * 255.0 * dpad * 1.0079;
           const double mc = 0x1p-21 * (nn + fe.xmax2 + 2.0 * (s * amx + fabs(dot)));
-          // (kSq8Planes digits: the last one is rounded, |residual| <= 2^-(7 kSq8Planes - 6) s per weight)
-          const double dd = ldexp(1.0, -(7 * kSq8Planes - 6)) * s * 255.0 * dpad + 0x1p-22 * qdec;
+          // (x 1.001 + a 2^-40 floor for the fp64 rounding of the residual sums)
+          const double dd = (255.0 * s * fmax(rp, rn) * 1.001 + 0x1p-40 * s * dpad) + 0x1p-22 * qdec;
           const double E = mc + (fe.metric == MV_L2 ? 2.0 : 1.0) * dd + 0x1p-22 * (nn + fe.xmax2);
           qerr[q] = __double2float_ru(1.05 * E);
         }
