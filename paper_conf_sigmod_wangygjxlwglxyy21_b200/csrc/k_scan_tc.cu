@@ -150,8 +150,10 @@ constexpr int kSideRank = 1152, kSideIds = 1792;
 // epilogue warps: three per TMEM lane quarter (<= 128 registers per thread: 512 threads fit the
 // register file).  Measured: 8 -> 12 took configs[1]'s phase B from 289 to 256 us and configs[4]'s
 // per-GPU scan from 9.4 to 8.9 ms; 16 was slower for FLAT (6 chunks of 16 columns over 4 warps)
-template <int TYPE>
-constexpr int epi_warps() { return 12; }
+// SQ8 with 128-code rows: four per quarter (640 threads, <= 102 registers; configs[4]'s phase B
+// 3.98 -> 3.70 ms; configs[2]'s 96-code rows measured slower with four)
+template <int TYPE, int ATOM>
+constexpr int epi_warps() { return TYPE == MV_IVF_SQ8 && ATOM == 128 ? 16 : 12; }
 
 // per-query metadata of one work item (QCP = roundup16(qchunk) entries per array)
 struct Meta {
@@ -190,9 +192,9 @@ __device__ __forceinline__ Meta meta_at(uint8_t* m, int QCP) {
 constexpr int kMetaPerQuery = 64;  // bytes (+ a 32-B work-item header)
 
 template <int TYPE, int ATOM, bool SMALLD>
-__global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE>(), 1)
+__global__ void __launch_bounds__(128 + 32 * epi_warps<TYPE, ATOM>(), 1)
     k_scan_tc(const __grid_constant__ XMaps xm, const TcScanParams p) {
-  constexpr int kEpiWarps = epi_warps<TYPE>();
+  constexpr int kEpiWarps = epi_warps<TYPE, ATOM>();
   extern __shared__ uint8_t smem_raw[];
   uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~(uintptr_t)1023);
   constexpr int ESZ = TYPE == MV_IVF_FLAT ? 4 : 1;
@@ -996,7 +998,10 @@ cudaError_t launch_scan_tc(const XMaps& xm, const TcScanParams& p, cudaStream_t 
   int dev = 0, nsm = kNumSMs;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
-  kern<<<nsm, 128 + 32 * (p.type == MV_IVF_FLAT ? epi_warps<MV_IVF_FLAT>() : epi_warps<MV_IVF_SQ8>()), p.smem_total,
+  const int nepi = p.type == MV_IVF_FLAT ? epi_warps<MV_IVF_FLAT, 128>()
+                   : p.atom == 128       ? epi_warps<MV_IVF_SQ8, 128>()
+                                         : epi_warps<MV_IVF_SQ8, 32>();
+  kern<<<nsm, 128 + 32 * nepi, p.smem_total,
          st>>>(xm, p);
   return cudaGetLastError();
 }
