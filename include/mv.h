@@ -94,9 +94,9 @@ MV_API mv_status mv_index_create(int32_t d, mv_metric metric, mv_type type, int3
  * the scratch budget.  Names: "seeding" (0/1), "need" (seeding sample, candidates), "capa" (rows
  * per list of the sample), "sq8_qc" / "flat_qc" (queries per scan work item), "coarse_nqb",
  * "coarse_cs", "coarse_epi", "coarse_nacc" (coarse GEMM shape), "large_k_select" (k > 256: 0 = the
- * streaming select when the search seeds (k <= 4096; the staged radix select for the rest and as
- * its fallback), 1 = the sample-threshold select, 2 = the staged radix select only, 3 = the
- * streaming select for the seeding bound too), "big_ctas" / "big_cap" (the staged
+ * seeding sample as 4-byte keys + the staged radix select, 1 = the sample-threshold select, 2 =
+ * 8-byte seeding keys + the staged radix select, 3 = the streaming select for the seeding bound,
+ * 4 = 4-byte seeding keys + the streaming final select (k <= 4096, staged fallback)), "big_ctas" / "big_cap" (the staged
  * select's first launch: CTAs per SM, 1..4, and candidates staged per query; queries past it are
  * redone with all of shared memory), "async_host" (1: a search whose host buffers are all page-locked
  * enqueues its copies on `stream` and returns without synchronising -- the caller synchronises

@@ -265,4 +265,19 @@ cudaError_t launch_iota_i32(int32_t* out, int64_t n, cudaStream_t st) {
   return cudaGetLastError();
 }
 
+// any sorted_ids[t] != t?  (ids exactly 0..n-1: the selects map a rank to its id without a gather)
+__global__ void k_check_identity(const int64_t* __restrict__ sorted_ids, int64_t n, int* flag) {
+  bool bad = false;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    bad |= sorted_ids[i] != i;
+  if (__syncthreads_or(bad) && threadIdx.x == 0) atomicOr(flag, 1);
+}
+
+cudaError_t launch_check_identity(const int64_t* sorted_ids, int64_t n, int* flag, cudaStream_t st) {
+  if (n == 0) return cudaSuccess;
+  const int grid = (int)min64(kNumSMs * 8, (n + 255) / 256);
+  k_check_identity<<<grid, 256, 0, st>>>(sorted_ids, n, flag);
+  return cudaGetLastError();
+}
+
 }  // namespace mv

@@ -15,6 +15,13 @@ namespace mv {
 constexpr int kBoundCap = 4096;   // boundary-bucket capacity (u64) for the radix path
 constexpr int kUnroll = 4;        // warp selects: 32-key chunks loaded per round
 
+// the id of a key's rank: sorted_ids[rank], or the rank itself when the index's ids are exactly
+// 0..ntotal-1 (the caller passes sorted_ids = nullptr: no random 8-byte gather per result)
+__device__ __forceinline__ int64_t rank_to_id(const int64_t* __restrict__ sorted_ids, uint64_t key) {
+  const uint32_t r = (uint32_t)(key & 0xffffffffu);
+  return sorted_ids ? __ldg(sorted_ids + r) : (int64_t)r;
+}
+
 __device__ __forceinline__ bool seg_locate(const int32_t* s_pre, int npb, int idx, int& j) {
   // binary search: largest j with s_pre[j] <= idx
   int lo = 0, hi = npb - 1;
@@ -144,7 +151,7 @@ __global__ void __launch_bounds__(256) k_final_select(const int64_t* __restrict_
     if (i < nout && sel[i] != MV_KEY_PAD) {
       const uint64_t key = sel[i];
       dv = key_dist((uint32_t)(key >> 32), metric);
-      iv = sorted_ids[(uint32_t)(key & 0xffffffffu)];
+      iv = rank_to_id(sorted_ids, key);
     } else {
       dv = metric == MV_L2 ? __int_as_float(0x7f800000) : __int_as_float(0xff800000);
       iv = -1;
@@ -597,7 +604,7 @@ output:
     const uint64_t key = res[i];
     if (i < nsel && key != MV_KEY_PAD) {
       dv = key_dist((uint32_t)(key >> 32), metric);
-      iv = sorted_ids[(uint32_t)(key & 0xffffffffu)];
+      iv = rank_to_id(sorted_ids, key);
     } else {
       dv = metric == MV_L2 ? __int_as_float(0x7f800000) : __int_as_float(0xff800000);
       iv = -1;
@@ -820,7 +827,7 @@ __global__ void __launch_bounds__(kBigThreads) k_final_sample(const int64_t* __r
     const uint64_t key = i < nsel ? top[i] : MV_KEY_PAD;
     if (key != MV_KEY_PAD) {
       dv = key_dist((uint32_t)(key >> 32), metric);
-      iv = sorted_ids[(uint32_t)(key & 0xffffffffu)];
+      iv = rank_to_id(sorted_ids, key);
     } else {
       dv = metric == MV_L2 ? __int_as_float(0x7f800000) : __int_as_float(0xff800000);
       iv = -1;
@@ -1062,7 +1069,7 @@ __global__ void __launch_bounds__(NT, TAU ? 1 : 3) k_select_stream(const int64_t
       if (i < ng) {
         const uint64_t key = win[i];
         dv = key_dist((uint32_t)(key >> 32), metric);
-        iv = sorted_ids[(uint32_t)(key & 0xffffffffu)];
+        iv = rank_to_id(sorted_ids, key);
       } else {
         dv = metric == MV_L2 ? __int_as_float(0x7f800000) : __int_as_float(0xff800000);
         iv = -1;
@@ -1195,9 +1202,11 @@ static cudaError_t launch_big_select(const int64_t* poff, const int32_t* pcnt, c
   // over: 2 nq bytes -- [0, nq) queries past k_final_big's stage, [nq, 2 nq) the redo flags of the
   // first-choice select (streaming or sample-threshold)
   uint8_t* redo = over ? over + nq : nullptr;
-  // streaming select: the final select by default (mode 0), the seeding select only as mode 3 (the
-  // staged select measured faster there: configs[3] 0.63 vs 0.72 ms)
-  if (k <= 4096 && (tau ? bsel.mode == 3 && bsel.kmin != nullptr : bsel.mode == 0 && bsel.kmin && bsel.khi && redo)) {
+  // streaming select: options only -- mode 3 for the seeding bound, mode 4 for the final select.
+  // The staged select measured faster for both once the id gather went away (configs[3], ids
+  // 0..n-1: final 0.75 ms staged vs 0.88-1.38 ms streaming, the latter with a large run-to-run
+  // spread; seeding 0.63 vs 0.72 ms)
+  if (k <= 4096 && (tau ? bsel.mode == 3 && bsel.kmin != nullptr : bsel.mode == 4 && bsel.kmin && bsel.khi && redo)) {
     constexpr int NT = 512;
     const size_t base = kBucketBins * 4 + 64 * 4 + 16 + (size_t)npb * 8 + (size_t)((npb + 34) & ~1) * 4;
     if (tau) {
@@ -1568,7 +1577,7 @@ __global__ void __launch_bounds__(256) k_final_warp(const int64_t* __restrict__ 
       int64_t iv;
       if (key != MV_KEY_PAD) {
         dv = key_dist((uint32_t)(key >> 32), metric);
-        iv = sorted_ids[(uint32_t)(key & 0xffffffffu)];
+        iv = rank_to_id(sorted_ids, key);
       } else {
         dv = metric == MV_L2 ? __int_as_float(0x7f800000) : __int_as_float(0xff800000);
         iv = -1;
@@ -1692,7 +1701,7 @@ __global__ void __launch_bounds__(256) k_refine_band(const int64_t* __restrict__
       int64_t iv;
       if (key != MV_KEY_PAD) {
         dv = key_dist((uint32_t)(key >> 32), metric);
-        iv = sorted_ids[(uint32_t)(key & 0xffffffffu)];
+        iv = rank_to_id(sorted_ids, key);
       } else {
         dv = metric == MV_L2 ? __int_as_float(0x7f800000) : __int_as_float(0xff800000);
         iv = -1;

@@ -41,6 +41,7 @@ struct mv_index {
   int64_t* ids = nullptr;       // ntotal, storage order
   uint32_t* rank = nullptr;     // ntotal: position of (id, row) in sorted order
   int64_t* sorted_ids = nullptr;  // ntotal: ids in (id, row) order
+  bool ids_identity = false;      // sorted_ids[r] == r (ids exactly 0..ntotal-1): no id gather
   uint32_t* row_of_rank = nullptr;  // storage row of each rank (the filter mode's exact re-scoring)
   double xmax2 = 0.0;           // max ||x||^2 (SQ8: ||x_hat||^2) over the stored rows (filter-mode bound)
   XMaps xm;                     // payload tensor maps: 128/64/32/16-row boxes (rebuilt by every add)
@@ -350,7 +351,7 @@ mv_status mv_index_set_option(mv_index* ix, const char* name, int64_t value) {
   else if (n == "workspace_bytes") o.workspace = value;
   else if (n == "scan_trace") o.scan_trace = value;  // development builds only (-DMV_SCAN_TRACE)
   else if (n == "async_host") o.async_host = value != 0;
-  else if (n == "large_k_select") o.large_k_select = (int)std::min<int64_t>(std::max<int64_t>(value, 0), 3);
+  else if (n == "large_k_select") o.large_k_select = (int)std::min<int64_t>(std::max<int64_t>(value, 0), 4);
   else if (n == "big_cap") o.big_cap = std::max<int64_t>(value, 0);
   else if (n == "big_ctas") o.big_ctas = (int)std::min<int64_t>(std::max<int64_t>(value, 0), 4);
   else return fail(MV_EINVAL, "unknown option '%s'", name);
@@ -614,6 +615,12 @@ mv_status mv_index_add(mv_index* ix, const float* vectors, const int64_t* ids, i
   CK(s.alloc(&t2, tmp2));
   CK(cub::DeviceRadixSort::SortPairs(t2, tmp2, keys, skeys, vals, svals, (int64_t)ntot, 0, 64, st));
   CK(launch_rank_scatter(skeys, svals, ntot, nx.rank, nx.sorted_ids, nx.row_of_rank, st));
+  int* idflag;
+  CK(s.alloc(&idflag, 1));
+  CK(cudaMemsetAsync(idflag, 0, sizeof(int), st));
+  CK(launch_check_identity(nx.sorted_ids, ntot, idflag, st));
+  int hid = 1;
+  CK(cudaMemcpyAsync(&hid, idflag, sizeof(int), cudaMemcpyDeviceToHost, st));
   unsigned long long* xm;
   CK(s.alloc(&xm, 1));
   unsigned long long hxm = 0;
@@ -639,6 +646,7 @@ mv_status mv_index_add(mv_index* ix, const float* vectors, const int64_t* ids, i
   nx.ids = nx.sorted_ids = nullptr;
   nx.rank = nx.row_of_rank = nullptr;
   ix->ntotal = ntot;
+  ix->ids_identity = hid == 0;
   if (ix->type == MV_IVF_FLAT && hflag) ix->tf32_exact = false;
   double xm2;
   memcpy(&xm2, &hxm, sizeof xm2);
@@ -721,6 +729,7 @@ static mv_status search_chunk(mv_index* ix, const float* q, int64_t nq, int32_t 
   const int nlist = ix->nlist, dpad = ix->dpad;
   const bool flat = ix->type == MV_IVF_FLAT;
   const bool pq = ix->type == MV_IVF_PQ;  // the query-major ADC scan (k_pq.cu) instead of k_scan_tc
+  const int64_t* idmap = ix->ids_identity ? nullptr : ix->sorted_ids;  // rank -> id (nullptr: identity)
   // a1 + a2/a3
   prof_mark(ix, st);
   float *qpad, *qnorm;
@@ -858,7 +867,7 @@ static mv_status search_chunk(mv_index* ix, const float* q, int64_t nq, int32_t 
   tp.approx_always = approx_always ? 1 : 0; tp.qerr = qerr;
   // k > 256 with seeding: phase A emits 4-byte distance keys and k_tau32 takes the bound from them
   // (half the sample's bytes written and read; large_k_select = 2 keeps the 8-byte keys)
-  const bool key32 = k > 256 && split && !pq && ix->opt.large_k_select == 0;
+  const bool key32 = k > 256 && split && !pq && (ix->opt.large_k_select == 0 || ix->opt.large_k_select == 4);
   tp.key32 = key32 ? 1 : 0;
   tp.prof = nullptr;
   // phase A (or, without seeding, the whole scan emitting every candidate) ...
@@ -916,7 +925,7 @@ static mv_status search_chunk(mv_index* ix, const float* q, int64_t nq, int32_t 
   }
   if (pq) {
     // IVF_PQ: the keys are the asymmetric distances themselves -- the plain exact select
-    CK(launch_final_select(b.poff, b.pcnt, part, nq, npb, k, ix->metric, ix->sorted_ids, D, I, tmax, over,
+    CK(launch_final_select(b.poff, b.pcnt, part, nq, npb, k, ix->metric, idmap, D, I, tmax, over,
                            BigSel{ix->opt.large_k_select, ix->opt.big_ctas, ix->opt.big_cap, 0, kmin, tau}, st));
   } else if (k <= 256) {
     // a7 with the filter mode's exact re-scoring fused in (a plain exact select when the search is
@@ -925,7 +934,7 @@ static mv_status search_chunk(mv_index* ix, const float* q, int64_t nq, int32_t 
     int* notgate;
     CK(s.alloc(&tau2, (size_t)nq));
     CK(s.alloc(&notgate, 1));
-    CK(launch_final_refine(ix->type, b.poff, b.pcnt, part, nq, npb, k, ix->metric, ix->sorted_ids, D, I, qerr, qpad,
+    CK(launch_final_refine(ix->type, b.poff, b.pcnt, part, nq, npb, k, ix->metric, idmap, D, I, qerr, qpad,
                            dpad, ix->payload, ix->row_of_rank, ix->vmin, ix->vdiff, ix->sq8_t, gate, tau2, notgate, st));
   } else {
     // filter mode: t~_q = the k-th best approximate key, exact re-scoring in place of the keys within
@@ -938,7 +947,7 @@ static mv_status search_chunk(mv_index* ix, const float* q, int64_t nq, int32_t 
     CK(launch_rekey(ix->type, b.poff, b.pcnt, part, nq, npb, tau2, qerr, ix->metric, qpad, dpad, ix->payload,
                     ix->row_of_rank, ix->vmin, ix->vdiff, ix->sq8_t, gate, st));
     ix->launches += 2;
-    CK(launch_final_select(b.poff, b.pcnt, part, nq, npb, k, ix->metric, ix->sorted_ids, D, I, tmax, over,
+    CK(launch_final_select(b.poff, b.pcnt, part, nq, npb, k, ix->metric, idmap, D, I, tmax, over,
                            BigSel{ix->opt.large_k_select, ix->opt.big_ctas, ix->opt.big_cap, 0, kmin, tau}, st));
   }
   prof_mark(ix, st);

@@ -310,6 +310,7 @@ cudaError_t launch_pq_encode(const float* xpad, const int64_t* ids, const int32_
                              const int64_t* new_off, const int64_t* old_off, const int32_t* add_off, uint8_t* payload,
                              double* norms, int64_t* out_ids, cudaStream_t st);
 cudaError_t launch_pq_scan(const PqScanParams& p, cudaStream_t st);
+cudaError_t launch_check_identity(const int64_t* sorted_ids, int64_t n, int* flag, cudaStream_t st);
 // k_filter.cu: strategy E's range bitmap and vector fusion
 cudaError_t launch_attr_bitset(const int64_t* ids, const int64_t* attr, int64_t n, int64_t lo, int64_t hi,
                                uint8_t* bitset, int64_t nbits, cudaStream_t st);

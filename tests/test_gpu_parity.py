@@ -369,7 +369,7 @@ def test_c2_full_size_sampled():
 
 OPTION_SETS = [{"seeding": 0}, {"need": 1, "capa": 16}, {"flat_qc": 32, "sq8_qc": 16},
                {"coarse_nqb": 64, "coarse_cs": 3, "coarse_epi": 16, "coarse_nacc": 1},
-               {"workspace_bytes": 1 << 20}, {"large_k_select": 1}, {"large_k_select": 2}, {"large_k_select": 3},
+               {"workspace_bytes": 1 << 20}, {"large_k_select": 1}, {"large_k_select": 2}, {"large_k_select": 3}, {"large_k_select": 4},
                {"seeding": 0, "big_cap": 1100}, {"big_ctas": 4, "big_cap": 700}, {"big_ctas": 1}]
 
 
@@ -521,3 +521,16 @@ def test_sq8_item_width_and_accumulators(qc, metric):
     frac, _, _ = _run_conditional(ix, X, ids, C, Q, 20, 5, mo, O.SQ8, bitset=bs, nbits=16_000)
     assert ix.describe()["last_scan"] == "tcgen05.i8"
     assert frac > 0.999
+
+
+@pytest.mark.parametrize("k", [10, 300])
+def test_identity_ids_fast_path(k):
+    """Ids exactly 0..n-1 (the selects map a rank to its id without the sorted_ids gather) and a
+    shifted copy (the gather) both equal the oracle."""
+    n = 15_000
+    X, Q = _sift(n, 40)
+    C = kmeans(X, 48, iters=4)
+    for ids in (torch.arange(n), torch.arange(n) + 7):
+        ix = _build(X, ids, C, "l2", "flat")
+        frac, _, _ = _run_conditional(ix, X, ids, C, Q, k, 6, O.L2, O.FLAT, exact=True)
+        assert frac == 1.0
