@@ -788,12 +788,13 @@ static mv_status search_chunk(mv_index* ix, const float* q, int64_t nq, int32_t 
   // (k N / need)-th best of the query's N candidates, so phase B emits ~k N / need keys.  Phase A
   // costs ~need rows of payload, an emission ~a fixed number of bytes (the key store, the final
   // select's reads); balancing the two gives need ~ sqrt(k N c / rowbytes).  c is measured
-  // (session-4 sweep): 32 B for k <= 256; the CTA-per-query select for k > 256 costs
-  // ~26x more per candidate (and falls back to global memory past its stage), c = 832 B.
+  // (DESIGN.md §5): 96 B for k <= 256 (round-2 sweep on the current kernels: configs[2] need 1200
+  // vs 806 2.13 vs 2.20 ms, configs[4] 1000 vs 552 5.86 vs 5.94 ms; round 1 measured 32 B); the
+  // CTA-per-query select for k > 256 costs ~26x more per candidate, c = 832 B.
   {
     const double ncand = (double)ix->ntotal * npb / std::max(1, nlist);
     const double rowb = pq ? (double)ix->pq_m : (double)dpad * (flat ? 4 : 1);
-    const double c = k > 256 ? 832.0 : 32.0;
+    const double c = k > 256 ? 832.0 : 96.0;
     const int64_t bal = (int64_t)std::sqrt((double)k * ncand * c / rowb);
     pa.need = std::max<int64_t>(pa.need, std::min<int64_t>(bal, 65536));
   }

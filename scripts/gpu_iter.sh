@@ -1,3 +1,4 @@
-O=gpurun_out/q_af; mkdir -p $O
-timeout 900 python -m pytest tests -m "gpu and not slow" -x -q -p no:cacheprovider > $O/pytest.log 2>&1; echo pytest=$?; tail -2 $O/pytest.log
-for i in 1 2; do timeout 900 python scripts/sweep_opts.py --config c4 --sets "" "large_k_select=4" > $O/sweep_c4_$i.txt 2>&1; grep -v "^\[bench" $O/sweep_c4_$i.txt; done
+O=gpurun_out/q_ag; mkdir -p $O
+timeout 900 python scripts/sweep_opts.py --config c5 --sets "" "need=1000" "need=1000,capa=512" "capa=512" > $O/sweep_c5.txt 2>&1; grep -v "^\[bench" $O/sweep_c5.txt
+timeout 900 python scripts/sweep_opts.py --config c3 --sets "" "need=600" "need=1200" "capa=128" > $O/sweep_c3.txt 2>&1; grep -v "^\[bench" $O/sweep_c3.txt
+timeout 900 python scripts/sweep_opts.py --config c2 --sets "" "need=100" "capa=256" > $O/sweep_c2.txt 2>&1; grep -v "^\[bench" $O/sweep_c2.txt
