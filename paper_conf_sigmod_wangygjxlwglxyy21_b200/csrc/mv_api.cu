@@ -794,7 +794,7 @@ static mv_status search_chunk(mv_index* ix, const float* q, int64_t nq, int32_t 
   {
     const double ncand = (double)ix->ntotal * npb / std::max(1, nlist);
     const double rowb = pq ? (double)ix->pq_m : (double)dpad * (flat ? 4 : 1);
-    const double c = k > 256 ? 832.0 : 96.0;
+    const double c = k > 256 ? 832.0 : (pq ? 32.0 : 96.0);  // (IVF_PQ's query-major scan: 32 B, c3pq 4.10 vs 4.25 ms)
     const int64_t bal = (int64_t)std::sqrt((double)k * ncand * c / rowb);
     pa.need = std::max<int64_t>(pa.need, std::min<int64_t>(bal, 65536));
   }
