@@ -143,12 +143,25 @@ __global__ void __launch_bounds__(kPqThreads) k_pq_scan(const PqScanParams p) {
       uint64_t key = 0;
       if (i < len) {
         const int64_t row = l0 + i;
-        const uint32_t* cw = reinterpret_cast<const uint32_t*>(p.codes + row * M);
         float acc = 0.0f;
-        for (int w = 0; w < words; ++w) {
-          const uint32_t v = __ldg(cw + w);
+        if ((M & 15) == 0) {  // 16 sub-codes per 16-byte load
+          const uint4* cq = reinterpret_cast<const uint4*>(p.codes + row * M);
+          for (int w4 = 0; w4 < (M >> 4); ++w4) {
+            const uint4 v4 = __ldg(cq + w4);
+            const uint32_t vv[4] = {v4.x, v4.y, v4.z, v4.w};
 #pragma unroll
-          for (int u = 0; u < 4; ++u) acc = __fadd_rn(acc, T[(w * 4 + u) * 256 + ((v >> (8 * u)) & 0xff)]);
+            for (int w = 0; w < 4; ++w)
+#pragma unroll
+              for (int u = 0; u < 4; ++u)
+                acc = __fadd_rn(acc, T[((w4 * 4 + w) * 4 + u) * 256 + ((vv[w] >> (8 * u)) & 0xff)]);
+          }
+        } else {
+          const uint32_t* cw = reinterpret_cast<const uint32_t*>(p.codes + row * M);
+          for (int w = 0; w < words; ++w) {
+            const uint32_t v = __ldg(cw + w);
+#pragma unroll
+            for (int u = 0; u < 4; ++u) acc = __fadd_rn(acc, T[(w * 4 + u) * 256 + ((v >> (8 * u)) & 0xff)]);
+          }
         }
         bool valid = true;
         if (p.bitset) valid = !bit_excluded(p.bitset, p.nbits, p.ids[row]);

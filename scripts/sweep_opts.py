@@ -36,6 +36,9 @@ def main():
         ix.set_centroids(C)
         if cfg["kind"] == "sq8":
             ix.set_sq8(*bench.sq8_params(cfg, X))
+        if cfg["kind"] == "pq":
+            samp = torch.randperm(n, generator=torch.Generator().manual_seed(5))[: min(n, 64 * cfg["nlist"])]
+            ix.train_pq(cfg["pq_m"], X[samp.to(dev)].contiguous(), niter=10)
         ix.add(X, torch.arange(n, dtype=torch.int64, device=dev))
         del X
     nprobe = a.nprobe or cfg["nprobe"]
