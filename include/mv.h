@@ -4,8 +4,10 @@
  * Problem (§3.2.1): given a batch of m queries and n data vectors, find for
  * each query its top-k most similar vectors; results are (int64 id, float distance) pairs
  * (Eq. (1) sizes heap entries as sizeof(int64)+sizeof(float)).
- * Indexes: IVF_FLAT and IVF_SQ8 (§2.2, 510-520 §3.1), metrics squared L2 and
- * inner product (§2.1).  Query processing is the two-step IVF procedure of
+ * Indexes: IVF_FLAT and IVF_SQ8 (§2.2, 510-520 §3.1) and IVF_PQ (PAPER.md:519-521,
+ * SURVEY §8(f) f3), metrics squared L2 and inner product (§2.1).  Also on the
+ * device: k-means training of the coarse codebook (mv_kmeans, f1), strategy E's range bitmap
+ * (mv_attr_bitset) and multi-vector fusion (mv_fuse_rows, f4).  Query processing is the two-step IVF procedure of
  * PAPER.md:523-532 (§3.1): find the nprobe closest buckets, then scan them.  k <= 16384
  * (§3.3).  A bitmap of entity ids is checked whenever a vector is
  * encountered, before the top-k (strategy B, §4.1).
