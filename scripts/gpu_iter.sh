@@ -1,3 +1,4 @@
-O=gpurun_out/q_al; mkdir -p $O
-timeout 900 python -m pytest tests/test_gpu_parity.py -x -q -p no:cacheprovider -k "large_k or options" > $O/pytest.log 2>&1; echo pytest=$?; tail -2 $O/pytest.log
-timeout 900 python scripts/sweep_opts.py --config c4 --sets "" > $O/sweep_c4.txt 2>&1; grep -v "^\[bench" $O/sweep_c4.txt
+O=gpurun_out/q_final; mkdir -p $O
+timeout 600 python -c "import __graft_entry__ as g; g.smoke()" > $O/smoke.log 2>&1; echo smoke=$?; tail -1 $O/smoke.log
+timeout 2400 python -m pytest tests -m gpu -q -p no:cacheprovider > $O/pytest_gpu.log 2>&1; echo pytest=$?; tail -1 $O/pytest_gpu.log
+timeout 900 python bench.py > $O/bench_default.json 2> $O/bench_default.err; echo bench=$?
