@@ -1,4 +1,4 @@
-O=gpurun_out/q_final; mkdir -p $O
-timeout 600 python -c "import __graft_entry__ as g; g.smoke()" > $O/smoke.log 2>&1; echo smoke=$?; tail -1 $O/smoke.log
-timeout 2400 python -m pytest tests -m gpu -q -p no:cacheprovider > $O/pytest_gpu.log 2>&1; echo pytest=$?; tail -1 $O/pytest_gpu.log
-timeout 900 python bench.py > $O/bench_default.json 2> $O/bench_default.err; echo bench=$?
+O=gpurun_out/q_am; mkdir -p $O
+timeout 900 python scripts/sweep_opts.py --config c4 --sets "" "flat_qc=112" "flat_qc=128" "flat_qc=80" > $O/sweep_c4.txt 2>&1; grep -v "^\[bench" $O/sweep_c4.txt
+timeout 900 python scripts/sweep_opts.py --config c5 --sets "" "sq8_qc=48" "sq8_qc=32" > $O/sweep_c5.txt 2>&1; grep -v "^\[bench" $O/sweep_c5.txt
+timeout 900 python scripts/sweep_opts.py --config c2 --sets "" "flat_qc=112" "flat_qc=64" > $O/sweep_c2.txt 2>&1; grep -v "^\[bench" $O/sweep_c2.txt
